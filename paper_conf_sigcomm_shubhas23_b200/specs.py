@@ -1,0 +1,147 @@
+"""Model architectures on the hot path, as plain op lists (no arithmetic here).
+
+Each spec is ``{"name", "in_h", "in_w", "in_c", "ops": [...]}`` with ops
+``conv(kh,kw,stride,pad,cout,act,residual)``, ``maxpool(k,stride,pad)``, ``block(cout,stride)``
+(cout>0 -> 1x1 projection shortcut), ``exit(num_classes, loss_weight)``, ``det_head(...)``.
+The same description is marshalled into the C-ABI's ``adainf_op`` (``binding.py``) and, by the tests
+only, into the oracle's own ``or_op``.
+
+Readings: exits at ResNet stage boundaries (Q3, "every 3 layers"),
+GAP->FC exit heads (Q4), BN folded (Q10), TinyYOLOv3-like single-scale detector (Q18),
+synthetic audio DAG (Q24).
+"""
+from __future__ import annotations
+
+RELU, LEAKY, NONE = 1, 2, 0
+
+# TinyYOLOv3 13x13-scale anchors (w, h) in pixels (reading Q18)
+YOLO_ANCHORS = [81.0, 82.0, 135.0, 169.0, 344.0, 319.0]
+
+
+def conv(k, cout, stride=1, pad=None, act=RELU, residual=False):
+    return {"kind": "conv", "kh": k, "kw": k, "stride": stride, "pad": (k // 2) if pad is None else pad,
+            "cout": cout, "act": act, "residual": int(residual)}
+
+
+def maxpool(k, stride, pad=0):
+    return {"kind": "maxpool", "kh": k, "kw": k, "stride": stride, "pad": pad}
+
+
+def block(cout=0, stride=1):
+    return {"kind": "block", "cout": cout, "stride": stride}
+
+
+def exit_(num_classes, loss_weight=1.0):
+    return {"kind": "exit", "num_classes": num_classes, "loss_weight": loss_weight}
+
+
+def tiny_cnn_ee(num_classes=10):
+    """BASELINE config 1: 3-conv early-exit CNN, 2 exits, 32x32x3 (95,188 params)."""
+    ops = [conv(3, 32), maxpool(2, 2), conv(3, 64), maxpool(2, 2), exit_(num_classes), conv(3, 128),
+           exit_(num_classes)]
+    return {"name": "tiny_cnn_ee", "in_h": 32, "in_w": 32, "in_c": 3, "ops": ops}
+
+
+def _basic_block(cout, stride, cin):
+    proj = stride != 1 or cin != cout
+    return [block(cout if proj else 0, stride), conv(3, cout, stride=stride), conv(3, cout, residual=True)]
+
+
+def resnet18_ee(num_classes=10, in_hw=224, in_c=3):
+    """BASELINE config 2: ResNet-18 with exits after layer1..layer3 + final (11,181,352 params at 10 cls)."""
+    ops = [conv(7, 64, stride=2, pad=3), maxpool(3, 2, 1)]
+    cin = 64
+    for cout, stride in ((64, 1), (128, 2), (256, 2), (512, 2)):
+        ops += _basic_block(cout, stride, cin)
+        ops += _basic_block(cout, 1, cout)
+        ops.append(exit_(num_classes))
+        cin = cout
+    return {"name": "resnet18_ee", "in_h": in_hw, "in_w": in_hw, "in_c": in_c, "ops": ops}
+
+
+def tiny_yolo_det(in_hw=416, det_classes=2, anchors=3, width=512):
+    """BASELINE config 3 detector: TinyYOLOv3-like single-scale, 'compressed' (layer 7 1024->512)."""
+    ops = []
+    for c in (16, 32, 64, 128, 256):
+        ops += [conv(3, c, act=LEAKY), maxpool(2, 2)]
+    ops += [conv(3, 512, act=LEAKY), maxpool(3, 1, 1), conv(3, width, act=LEAKY), conv(1, 256, act=LEAKY),
+            conv(3, 512, act=LEAKY), conv(1, anchors * (5 + det_classes), act=NONE),
+            {"kind": "det_head", "anchors": anchors, "det_classes": det_classes, "grid_stride": 32,
+             "anchor_wh": YOLO_ANCHORS[:2 * anchors]}]
+    return {"name": "tiny_yolo_det", "in_h": in_hw, "in_w": in_hw, "in_c": 3, "ops": ops}
+
+
+def num_params(spec) -> int:
+    """Parameter count from the documented flat layout (include/adainf.h)."""
+    H, W, Cc = spec["in_h"], spec["in_w"], spec["in_c"]
+    n = 0
+    for o in spec["ops"]:
+        k = o["kind"]
+        if k == "conv":
+            n += o["cout"] * o["kh"] * o["kw"] * Cc + o["cout"]
+            H = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
+            W = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
+            Cc = o["cout"]
+        elif k == "maxpool":
+            H = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
+            W = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
+        elif k == "block" and o["cout"] > 0:
+            n += o["cout"] * Cc + o["cout"]
+        elif k == "exit":
+            n += Cc * o["num_classes"] + o["num_classes"]
+    return n
+
+
+def param_segments(spec):
+    """[(kind, op_index, offset, shape)] of the flat fp32 parameter vector, in layout order."""
+    H, W, Cc = spec["in_h"], spec["in_w"], spec["in_c"]
+    segs, off = [], 0
+    for i, o in enumerate(spec["ops"]):
+        k = o["kind"]
+        if k == "conv":
+            shp = (o["cout"], o["kh"], o["kw"], Cc)
+            segs.append(("conv_w", i, off, shp))
+            off += o["cout"] * o["kh"] * o["kw"] * Cc
+            segs.append(("conv_b", i, off, (o["cout"],)))
+            off += o["cout"]
+            H = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
+            W = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
+            Cc = o["cout"]
+        elif k == "maxpool":
+            H = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
+            W = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
+        elif k == "block" and o["cout"] > 0:
+            segs.append(("proj_w", i, off, (o["cout"], 1, 1, Cc)))
+            off += o["cout"] * Cc
+            segs.append(("proj_b", i, off, (o["cout"],)))
+            off += o["cout"]
+        elif k == "exit":
+            segs.append(("exit_w", i, off, (Cc, o["num_classes"])))
+            off += Cc * o["num_classes"]
+            segs.append(("exit_b", i, off, (o["num_classes"],)))
+            off += o["num_classes"]
+    return segs
+
+
+def macs_per_sample(spec):
+    """Per-op forward MACs of one sample (conv + projection + exit FC), list aligned with ops."""
+    H, W, Cc = spec["in_h"], spec["in_w"], spec["in_c"]
+    out = []
+    for o in spec["ops"]:
+        k = o["kind"]
+        m = 0
+        if k == "conv":
+            Ho = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
+            Wo = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
+            m = Ho * Wo * o["cout"] * o["kh"] * o["kw"] * Cc
+            H, W, Cc = Ho, Wo, o["cout"]
+        elif k == "maxpool":
+            H = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
+            W = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
+        elif k == "block" and o["cout"] > 0:
+            Ho, Wo = (H - 1) // o["stride"] + 1, (W - 1) // o["stride"] + 1
+            m = Ho * Wo * o["cout"] * Cc
+        elif k == "exit":
+            m = Cc * o["num_classes"]
+        out.append(m)
+    return out

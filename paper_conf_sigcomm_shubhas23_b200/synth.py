@@ -1,0 +1,213 @@
+"""Seeded synthetic inputs shaped like the paper's workloads (no method arithmetic here).
+
+Serves both the CUDA path (bench, GPU tests) and the oracle (tests) from one place, as the only code
+they share.  Recipe (DESIGN.md §Input recipe):
+
+* images   x = clip(c_p * (proto_y + 0.3 * eps) + b_p, -2, 2) -> bf16, proto_y a low-frequency class
+  pattern, eps spatially smoothed Gaussian noise; per 50 s period brightness b_p ~
+  U(-0.3, 0.3), contrast c_p ~ U(0.7, 1.3), occlusion rectangle with prob 0.1 (lighting / occlusion
+  drift); label priors pi_p ~ Dirichlet(5) mild / Dirichlet(0.3) heavy (label drift).
+* spectrograms: 128 mel x 128 frames log-energy, class harmonic stripes + 1/f noise (reading Q24).
+* weights: He-normal conv weights, small biases, exit heads x4 to spread confidences.
+* embeddings for selection: old features ~ N(mu_old, I), new features drifted; PCA basis from the old
+  features (fitted off the hot path).
+
+bf16 values are produced by numpy RNE rounding of fp32 bit patterns so that both sides receive
+identical bits.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+from . import specs as S
+
+
+def to_bf16_bits(x: np.ndarray) -> np.ndarray:
+    """fp32 -> bf16 bit patterns (uint16), round-to-nearest-even."""
+    u = np.ascontiguousarray(x, np.float32).view(np.uint32).astype(np.uint64)
+    u = (u + 0x7FFF + ((u >> 16) & 1)) >> 16
+    return u.astype(np.uint16)
+
+
+def bf16_bits_to_f32(b: np.ndarray) -> np.ndarray:
+    return (np.ascontiguousarray(b, np.uint16).astype(np.uint32) << 16).view(np.float32)
+
+
+def round_bf16(x: np.ndarray) -> np.ndarray:
+    return bf16_bits_to_f32(to_bf16_bits(x))
+
+
+def _smooth(a: np.ndarray, r: int, axes=(1, 2)) -> np.ndarray:
+    """Box blur of radius r along two axes via cumulative sums (edge-clamped)."""
+    for ax in axes:
+        n = a.shape[ax]
+        pad = [(0, 0)] * a.ndim
+        pad[ax] = (r + 1, r)
+        c = np.cumsum(np.pad(a, pad, mode="edge"), axis=ax, dtype=np.float32)
+        hi = np.take(c, np.arange(2 * r + 1, 2 * r + 1 + n), axis=ax)
+        lo = np.take(c, np.arange(0, n), axis=ax)
+        a = (hi - lo) / np.float32(2 * r + 1)
+    return a
+
+
+def class_prototypes(num_classes: int, H: int, W: int, C: int, seed: int = 1234) -> np.ndarray:
+    """Low-frequency class patterns: a few random 2-D sinusoids per class and channel."""
+    rng = np.random.default_rng(seed)
+    yy, xx = np.meshgrid(np.linspace(0, 1, H, dtype=np.float32), np.linspace(0, 1, W, dtype=np.float32),
+                         indexing="ij")
+    P = np.zeros((num_classes, H, W, C), np.float32)
+    for k in range(num_classes):
+        for c in range(C):
+            for _ in range(3):
+                fy, fx = rng.uniform(0.5, 3.0, 2)
+                ph = rng.uniform(0, 2 * np.pi)
+                P[k, :, :, c] += np.float32(rng.uniform(0.3, 0.8)) * np.sin(
+                    2 * np.pi * (fy * yy + fx * xx) + ph).astype(np.float32)
+    return P
+
+
+def label_priors(num_classes: int, periods: int, heavy: bool, seed: int) -> np.ndarray:
+    rng = np.random.default_rng(seed)
+    alpha = 0.3 if heavy else 5.0
+    return rng.dirichlet(np.full(num_classes, alpha), size=periods).astype(np.float64)
+
+
+def js_divergence(p: np.ndarray, q: np.ndarray) -> float:
+    """Jensen-Shannon divergence (base 2) of two label distributions (generator check vs P:86, Fig 6)."""
+    m = 0.5 * (p + q)
+
+    def kl(a, b):
+        nz = a > 0
+        return float(np.sum(a[nz] * np.log2(a[nz] / b[nz])))
+
+    return 0.5 * kl(p, m) + 0.5 * kl(q, m)
+
+
+def drifted_images(B: int, H: int, W: int, C: int = 3, num_classes: int = 10, period: int = 0,
+                   heavy: bool = False, seed: int = 0, protos: np.ndarray | None = None):
+    """One request batch of period `period`: returns (bf16 bits [B,H,W,C] uint16, labels int32)."""
+    rng = np.random.default_rng([seed, period])
+    if protos is None:
+        protos = class_prototypes(num_classes, H, W, C, seed=1234 + num_classes)
+    pri = label_priors(num_classes, period + 1, heavy, seed=seed)[period]
+    labels = rng.choice(num_classes, size=B, p=pri).astype(np.int32)
+    contrast = np.float32(rng.uniform(0.7, 1.3 if not heavy else 1.6))
+    bright = np.float32(rng.uniform(-0.3, 0.3) * (2.0 if heavy else 1.0))
+    out = np.empty((B, H, W, C), np.uint16)
+    chunk = max(1, (1 << 24) // (H * W * C))
+    for s in range(0, B, chunk):
+        e = min(B, s + chunk)
+        eps = rng.standard_normal((e - s, H, W, C), dtype=np.float32)
+        eps = _smooth(eps, max(1, H // 64)) * np.float32(2.0)
+        x = contrast * (protos[labels[s:e]] + np.float32(0.3) * eps) + bright
+        occ = rng.random(e - s) < 0.1
+        for i in np.nonzero(occ)[0]:
+            h0, w0 = rng.integers(0, H // 2), rng.integers(0, W // 2)
+            x[i, h0:h0 + H // 3, w0:w0 + W // 3, :] = np.float32(rng.uniform(-1, 1))
+        out[s:e] = to_bf16_bits(np.clip(x, -2.0, 2.0))
+    return out, labels
+
+
+def spectrograms(B: int, num_classes: int = 8, F: int = 128, T: int = 128, period: int = 0, seed: int = 0):
+    """Synthetic log-mel spectrograms [B,F,T,1] (bf16 bits) with class harmonic stripes + 1/f noise."""
+    rng = np.random.default_rng([seed, 7, period])
+    labels = rng.integers(0, num_classes, size=B).astype(np.int32)
+    f = np.arange(F, dtype=np.float32)[:, None]
+    t = np.arange(T, dtype=np.float32)[None, :]
+    snr = np.float32(rng.uniform(0.5, 1.5))
+    out = np.empty((B, F, T, 1), np.uint16)
+    for i in range(B):
+        f0 = 6 + 5 * labels[i]
+        stripes = sum(np.exp(-0.5 * ((f - h * f0) / 1.5) ** 2) for h in range(1, 5)).astype(np.float32)
+        mod = (0.5 + 0.5 * np.sin(2 * np.pi * t / (16 + 4 * labels[i]))).astype(np.float32)
+        noise = _smooth(rng.standard_normal((1, F, T, 1), dtype=np.float32), 2)[0, :, :, 0] / (1 + f / 16)
+        x = snr * stripes * mod + 0.5 * noise - 0.5
+        out[i, :, :, 0] = to_bf16_bits(np.clip(x, -2, 2))
+    return out, labels
+
+
+def init_params(spec: dict, seed: int = 0, exit_scale: float = 4.0) -> np.ndarray:
+    """He-normal conv weights, small biases, exit heads scaled x`exit_scale` (fp32 flat vector)."""
+    rng = np.random.default_rng(seed)
+    n = S.num_params(spec)
+    p = np.zeros(n, np.float32)
+    for kind, _i, off, shp in S.param_segments(spec):
+        cnt = int(np.prod(shp))
+        if kind in ("conv_w", "proj_w"):
+            fan_in = shp[1] * shp[2] * shp[3]
+            p[off:off + cnt] = rng.standard_normal(cnt, dtype=np.float32) * np.float32(np.sqrt(2.0 / fan_in))
+        elif kind in ("conv_b", "proj_b"):
+            p[off:off + cnt] = rng.standard_normal(cnt, dtype=np.float32) * np.float32(0.01)
+        elif kind == "exit_w":
+            p[off:off + cnt] = rng.standard_normal(cnt, dtype=np.float32) * np.float32(
+                exit_scale / np.sqrt(shp[0]))
+        elif kind == "exit_b":
+            p[off:off + cnt] = rng.standard_normal(cnt, dtype=np.float32) * np.float32(0.1)
+    return p
+
+
+def det_head_params(spec: dict, params: np.ndarray, obj_bias: float, seed: int = 0) -> np.ndarray:
+    """Bias the detector's final 1x1 conv so the objectness logits sit near `obj_bias` (controls the
+    detection rate before tau_det calibration)."""
+    p = params.copy()
+    segs = S.param_segments(spec)
+    head = [s for s in segs if s[0] == "conv_b"][-1]
+    _, _, off, shp = head
+    A = next(o for o in spec["ops"] if o["kind"] == "det_head")
+    per = 5 + A["det_classes"]
+    for a in range(A["anchors"]):
+        p[off + a * per + 4] = obj_bias
+    wseg = [s for s in segs if s[0] == "conv_w"][-1]
+    _, _, woff, wshp = wseg
+    cnt = int(np.prod(wshp))
+    p[woff:woff + cnt] *= np.float32(0.25)
+    return p
+
+
+def embeddings(N: int, D: int, P: int, drift: float = 1.0, seed: int = 0, M: int = 1):
+    """Selection inputs: new-sample features X [N,D] (bf16 bits), PCA basis W [D,P] (bf16 bits,
+    fitted on synthetic old features off the hot path), reference rows [M,D] fp32 (M=1: the old mean)."""
+    rng = np.random.default_rng([seed, 11])
+    mu_old = rng.standard_normal(D).astype(np.float32) + 2.0
+    old = mu_old + rng.standard_normal((4 * D, D)).astype(np.float32) * 0.5
+    # PCA basis of the old features (uncentred projection, reading Q13)
+    _, _, vt = np.linalg.svd(old - old.mean(0), full_matrices=False)
+    Wp = vt[:P].T.astype(np.float32)
+    shift = (rng.standard_normal(D).astype(np.float32) * drift).astype(np.float32)
+    frac = rng.random(N).astype(np.float32)[:, None]
+    X = mu_old + frac * shift + rng.standard_normal((N, D)).astype(np.float32) * 0.5
+    if M == 1:
+        ref = old.mean(0, keepdims=True).astype(np.float32)
+    else:
+        ref = old[rng.choice(old.shape[0], M, replace=False)].astype(np.float32)
+    return to_bf16_bits(X), to_bf16_bits(Wp), ref
+
+
+def calibrate_thresholds(conf: np.ndarray, fractions, band: float = 2e-3) -> np.ndarray:
+    """Thresholds tau_k placing the exit fractions near `fractions` (fraction of ALL samples exiting at
+    each early exit), each at the midpoint of the widest confidence gap near the target quantile so the
+    1e-3 decision bands stay sparse (SURVEY §8(d) "Thresholds").  conf: [B, E] (full depth)."""
+    B, E = conf.shape
+    alive = np.ones(B, bool)
+    taus = []
+    for k in range(E - 1):
+        want = int(round(fractions[k] * B))
+        c = np.sort(conf[alive, k])[::-1]
+        nalive = c.shape[0]
+        if want <= 0 or nalive == 0:
+            taus.append(2.0)
+            continue
+        if want >= nalive:
+            taus.append(0.0)
+            alive[:] = False
+            continue
+        lo, hi = max(0, want - max(2, nalive // 20)), min(nalive - 1, want + max(2, nalive // 20))
+        best, bi = -1.0, want
+        for j in range(max(lo, 1), hi + 1):
+            g = c[j - 1] - c[j]
+            if g > best:
+                best, bi = g, j
+        tau = float(0.5 * (c[bi - 1] + c[bi]))
+        taus.append(tau)
+        alive &= ~(conf[:, k] >= tau)
+    return np.asarray(taus, np.float32)
