@@ -1,0 +1,37 @@
+/*
+ * adainf_debug.h — kernel-level entry points of libadainf.so, used by the per-kernel GPU parity
+ * tests (tests/test_gpu_kernels.py) and the bench's roofline leg.  Same conventions as adainf.h:
+ * device pointers, caller-owned buffers, stream-ordered, status return, no CPU fallback.
+ */
+#ifndef ADAINF_DEBUG_H_
+#define ADAINF_DEBUG_H_
+#include "adainf.h"
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Implicit-GEMM conv forward on the tensor cores:
+ * out[n][ho][wo][co] = act(sum x * w + b [+ res]) in bf16 (fp32 if out_f32).
+ * x: device [n][H][W][C] bf16 (C multiple of 8); w: device bf16 [Co][KH][KW][C]; b: device fp32 [Co];
+ * res: device bf16 [n][Ho][Wo][Co] or NULL. */
+adainf_status adainf_dbg_conv_fwd(const void* x, int32_t n, int32_t H, int32_t W, int32_t C, const void* w,
+                                  const float* b, int32_t Co, int32_t KH, int32_t KW, int32_t stride,
+                                  int32_t pad, int32_t act, const void* res, void* out, int32_t out_f32,
+                                  adainf_stream_t stream);
+/* dgrad: dx[n][H][W][C] = bf16( (sum_{tap,co} dz * w) [+ bcast[n][c]] [+ sc] ) * act'(yact)
+ * (conv transpose of the forward conv above; stride-s phases). */
+adainf_status adainf_dbg_conv_dgrad(const void* dz, int32_t n, int32_t H, int32_t W, int32_t C, const void* w,
+                                    int32_t Co, int32_t KH, int32_t KW, int32_t stride, int32_t pad,
+                                    const float* bcast, const void* sc, const void* yact, int32_t mask_act,
+                                    void* dx, adainf_stream_t stream);
+/* wgrad: dw[co][kh][kw][c] = sum_{n,ho,wo} dz[n][ho][wo][co] * x[n][ho*s-p+kh][wo*s-p+kw][c] (fp32),
+ * db[co] = sum dz (fp32, optional). Deterministic split-K. */
+adainf_status adainf_dbg_conv_wgrad(const void* x, const void* dz, int32_t n, int32_t H, int32_t W, int32_t C,
+                                    int32_t Co, int32_t KH, int32_t KW, int32_t stride, int32_t pad, float* dw,
+                                    float* db, adainf_stream_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -215,9 +215,9 @@ Walk walk(const or_model* m) {
   return w;
 }
 
-inline double act_f(int act, double v) {
+inline double act_f(int act, double v, bool exact) {
   if (act == 1) return v > 0 ? v : 0.0;
-  if (act == 2) return v > 0 ? v : 0.1 * v;
+  if (act == 2) return v > 0 ? v : (exact ? 0.1 * v : (double)(0.1f * (float)v));  // fp32 0.1f*x (c.1 step 2)
   return v;
 }
 inline double act_d(int act, double y) {  // derivative from the stored output (ReLU'(0) = 0)
@@ -319,7 +319,7 @@ struct Engine {
         const bool fp32_out = (i + 1 < m->n_ops && m->ops[i + 1].kind == OR_DET_HEAD);
         Y.d.resize(acc.size());
         for (size_t e = 0; e < acc.size(); ++e) {
-          const double v = F(act_f(op.act, acc[e]));
+          const double v = F(act_f(op.act, acc[e], exact));
           Y.d[e] = fp32_out ? v : R(v);
         }
         T.push_back(std::move(Y));

@@ -1,0 +1,305 @@
+"""Thin ctypes binding of libadainf.so (argument marshalling only; every step runs in the library's
+sm_100a kernels).  Names mirror include/adainf.h.  There is no fallback: if the shared library is
+missing or the device is not sm_100, calls raise AdaInfError.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+from . import specs as S
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libadainf.so")
+
+OK, ERR_INVALID, ERR_SHAPE, ERR_CAPACITY, ERR_OOM, ERR_CUDA, ERR_NCCL, ERR_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6, -7
+_OPKIND = {"conv": 0, "maxpool": 1, "block": 2, "exit": 3, "det_head": 4}
+ROUTE_DET_CROP, ROUTE_CLASS_WHOLE = 0, 1
+
+
+class AdaInfError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"adainf status {code}: {msg}")
+        self.code = code
+
+
+class Op(C.Structure):
+    _fields_ = [("kind", C.c_int32), ("kh", C.c_int32), ("kw", C.c_int32), ("stride", C.c_int32),
+                ("pad", C.c_int32), ("cout", C.c_int32), ("act", C.c_int32), ("residual", C.c_int32),
+                ("num_classes", C.c_int32), ("loss_weight", C.c_float), ("anchors", C.c_int32),
+                ("det_classes", C.c_int32), ("grid_stride", C.c_int32), ("anchor_wh", C.c_float * 16)]
+
+
+class ModelSpec(C.Structure):
+    _fields_ = [("in_h", C.c_int32), ("in_w", C.c_int32), ("in_c", C.c_int32), ("max_batch", C.c_int32),
+                ("n_ops", C.c_int32), ("ops", C.POINTER(Op)), ("momentum", C.c_float),
+                ("weight_decay", C.c_float), ("seed", C.c_uint64), ("init_params", C.POINTER(C.c_float)),
+                ("device", C.c_int32)]
+
+
+class Edge(C.Structure):
+    _fields_ = [("src_model", C.c_int32), ("dst_model", C.c_int32), ("kind", C.c_int32),
+                ("src_class", C.c_int32), ("crop_h", C.c_int32), ("crop_w", C.c_int32)]
+
+
+class AppSpec(C.Structure):
+    _fields_ = [("n_models", C.c_int32), ("models", C.POINTER(C.c_void_p)), ("n_edges", C.c_int32),
+                ("edges", C.POINTER(Edge)), ("max_routed_per_dst", C.c_int32)]
+
+
+class ModelOut(C.Structure):
+    _fields_ = [("exit_id", C.c_void_p), ("pred", C.c_void_p), ("conf", C.c_void_p), ("entropy", C.c_void_p),
+                ("logits", C.c_void_p), ("exit_counts", C.c_void_p), ("surv_idx", C.c_void_p),
+                ("embed", C.c_void_p), ("n_det", C.c_void_p), ("det_table", C.c_void_p), ("max_det", C.c_int32),
+                ("route_idx", C.c_void_p), ("n_routed", C.c_void_p)]
+
+
+class SelectIn(C.Structure):
+    _fields_ = [("X_bf16", C.c_void_p), ("N", C.c_int64), ("D", C.c_int32), ("W_bf16", C.c_void_p),
+                ("P", C.c_int32), ("ref", C.c_void_p), ("M", C.c_int32), ("exclude", C.c_void_p)]
+
+
+_lib = None
+
+
+def lib():
+    """Load libadainf.so (fails loudly when absent: no fallback path exists)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise AdaInfError(ERR_UNSUPPORTED, f"{LIB_PATH} missing: run __graft_entry__.build()")
+        L = C.CDLL(LIB_PATH)
+        vp, i32, i64 = C.c_void_p, C.c_int32, C.c_int64
+        L.adainf_last_error.restype = C.c_char_p
+        L.adainf_version.restype = C.c_int32
+        for name, args in {
+            "adainf_model_create": [C.POINTER(ModelSpec), C.POINTER(vp)],
+            "adainf_model_destroy": [vp],
+            "adainf_model_num_params": [vp, C.POINTER(i64)],
+            "adainf_model_num_exits": [vp, C.POINTER(i32)],
+            "adainf_model_get_params": [vp, C.POINTER(C.c_float), i64],
+            "adainf_model_set_params": [vp, C.POINTER(C.c_float), i64],
+            "adainf_model_grad_ptr": [vp, C.POINTER(vp)],
+            "adainf_app_create": [C.POINTER(AppSpec), C.POINTER(vp)],
+            "adainf_app_destroy": [vp],
+            "adainf_infer_dag": [vp, vp, i32, C.POINTER(C.c_float), i32, C.POINTER(ModelOut), vp],
+            "adainf_select_retrain": [C.POINTER(SelectIn), i32, vp, vp, vp, vp, vp],
+            "adainf_retrain_step": [vp, vp, vp, i32, i64, C.c_float, vp, vp],
+            "adainf_dp_attach": [vp, vp, i32, i32],
+            "adainf_nccl_unique_id": [vp],
+            "adainf_dbg_conv_fwd": [vp, i32, i32, i32, i32, vp, vp, i32, i32, i32, i32, i32, i32, vp, vp, i32, vp],
+            "adainf_dbg_conv_dgrad": [vp, i32, i32, i32, i32, vp, i32, i32, i32, i32, i32, vp, vp, vp, i32, vp,
+                                      vp],
+            "adainf_dbg_conv_wgrad": [vp, vp, i32, i32, i32, i32, i32, i32, i32, i32, i32, vp, vp, vp],
+        }.items():
+            f = getattr(L, name, None)
+            if f is not None:
+                f.argtypes = args
+                f.restype = C.c_int32
+        _lib = L
+    return _lib
+
+
+def check(rc):
+    if rc != OK:
+        raise AdaInfError(rc, lib().adainf_last_error().decode(errors="replace"))
+
+
+def ptr(t):
+    """Device/host pointer of a torch tensor (or None)."""
+    return None if t is None else C.c_void_p(t.data_ptr())
+
+
+def stream_ptr(stream=None):
+    import torch
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return C.c_void_p(s.cuda_stream)
+
+
+def make_ops(spec):
+    ops = (Op * len(spec["ops"]))()
+    for i, o in enumerate(spec["ops"]):
+        r = ops[i]
+        r.kind = _OPKIND[o["kind"]]
+        r.kh = o.get("kh", 1)
+        r.kw = o.get("kw", 1)
+        r.stride = o.get("stride", 1)
+        r.pad = o.get("pad", 0)
+        r.cout = o.get("cout", 0)
+        r.act = o.get("act", 0)
+        r.residual = int(o.get("residual", 0))
+        r.num_classes = o.get("num_classes", 0)
+        r.loss_weight = o.get("loss_weight", 1.0)
+        r.anchors = o.get("anchors", 0)
+        r.det_classes = o.get("det_classes", 0)
+        r.grid_stride = o.get("grid_stride", 0)
+        for j, v in enumerate(o.get("anchor_wh", [])):
+            r.anchor_wh[j] = v
+    return ops
+
+
+class Model:
+    """Owns an adainf_model_t."""
+
+    def __init__(self, spec, max_batch, params=None, seed=0, momentum=0.9, weight_decay=0.0, device=0):
+        self.spec = spec
+        self._ops = make_ops(spec)
+        self._params = None if params is None else np.ascontiguousarray(params, np.float32)
+        ms = ModelSpec(spec["in_h"], spec["in_w"], spec["in_c"], max_batch, len(spec["ops"]), self._ops, momentum,
+                       weight_decay, seed,
+                       self._params.ctypes.data_as(C.POINTER(C.c_float)) if self._params is not None else None,
+                       device)
+        h = C.c_void_p()
+        check(lib().adainf_model_create(C.byref(ms), C.byref(h)))
+        self.h = h
+        n = C.c_int64()
+        check(lib().adainf_model_num_params(self.h, C.byref(n)))
+        self.num_params = n.value
+        e = C.c_int32()
+        check(lib().adainf_model_num_exits(self.h, C.byref(e)))
+        self.num_exits = e.value
+        self.ncls = next((o["num_classes"] for o in spec["ops"] if o["kind"] == "exit"), 0)
+        self.max_batch = max_batch
+
+    def get_params(self):
+        out = np.zeros(self.num_params, np.float32)
+        check(lib().adainf_model_get_params(self.h, out.ctypes.data_as(C.POINTER(C.c_float)), self.num_params))
+        return out
+
+    def set_params(self, p):
+        p = np.ascontiguousarray(p, np.float32)
+        check(lib().adainf_model_set_params(self.h, p.ctypes.data_as(C.POINTER(C.c_float)), self.num_params))
+
+    def grad(self):
+        import torch
+        vp = C.c_void_p()
+        check(lib().adainf_model_grad_ptr(self.h, C.byref(vp)))
+        # copy out through torch (device -> host) for inspection
+        buf = torch.empty(self.num_params, dtype=torch.float32, device="cuda")
+        C.memmove  # noqa: B018
+        torch.cuda.synchronize()
+        import ctypes
+        cudart = torch.cuda.cudart()
+        cudart.cudaMemcpy(buf.data_ptr(), vp.value, self.num_params * 4, 3)  # D2D
+        return buf
+
+    def retrain_step(self, samples, labels, n_global=None, lr=0.01, stats=None, stream=None):
+        check(lib().adainf_retrain_step(self.h, ptr(samples), ptr(labels), int(samples.shape[0]),
+                                        int(n_global or samples.shape[0]), float(lr), ptr(stats),
+                                        stream_ptr(stream)))
+
+    def dp_attach(self, uid: bytes, rank: int, world: int):
+        buf = C.create_string_buffer(uid, 128)
+        check(lib().adainf_dp_attach(self.h, buf, rank, world))
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().adainf_model_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def nccl_unique_id() -> bytes:
+    buf = C.create_string_buffer(128)
+    check(lib().adainf_nccl_unique_id(buf))
+    return buf.raw
+
+
+class App:
+    """Owns an adainf_app_t over borrowed Models."""
+
+    def __init__(self, models, edges=(), max_routed_per_dst=0):
+        self.models = list(models)
+        arr = (C.c_void_p * len(self.models))(*[m.h.value for m in self.models])
+        self._arr = arr
+        self._edges = (Edge * max(1, len(edges)))()
+        for i, e in enumerate(edges):
+            self._edges[i] = Edge(*e)
+        self.edges = list(edges)
+        spec = AppSpec(len(self.models), C.cast(arr, C.POINTER(C.c_void_p)), len(edges), self._edges,
+                       max_routed_per_dst)
+        h = C.c_void_p()
+        check(lib().adainf_app_create(C.byref(spec), C.byref(h)))
+        self.h = h
+        self.max_routed = max_routed_per_dst
+
+    def infer(self, batch, taus, outs, stream=None):
+        """batch: cuda bf16/uint16 tensor [B,H,W,C]; taus: host list; outs: list of dicts of cuda tensors."""
+        t = np.ascontiguousarray(np.asarray(taus, np.float32).reshape(-1))
+        mo = (ModelOut * len(self.models))()
+        for i, o in enumerate(outs):
+            for k in ("exit_id", "pred", "conf", "entropy", "logits", "exit_counts", "surv_idx", "embed", "n_det",
+                      "det_table", "route_idx", "n_routed"):
+                if o.get(k) is not None:
+                    setattr(mo[i], k, o[k].data_ptr())
+            mo[i].max_det = int(o["det_table"].shape[0]) if o.get("det_table") is not None else 0
+        check(lib().adainf_infer_dag(self.h, ptr(batch), int(batch.shape[0]),
+                                     t.ctypes.data_as(C.POINTER(C.c_float)), int(t.size), mo, stream_ptr(stream)))
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().adainf_app_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def select_retrain(X, W, ref, k, exclude=None, out_idx=None, out_dist=None, out_count=None, dist_all=None,
+                   stream=None):
+    """X: cuda bf16 [N,D]; W: cuda bf16 [D,P] or None; ref: cuda fp32 [M,D]."""
+    import torch
+    N, D = X.shape
+    P = W.shape[1] if W is not None else D
+    si = SelectIn(X.data_ptr(), N, D, W.data_ptr() if W is not None else None, P, ref.data_ptr(),
+                  ref.shape[0], exclude.data_ptr() if exclude is not None else None)
+    dev = X.device
+    out_idx = out_idx if out_idx is not None else torch.empty(k, dtype=torch.int32, device=dev)
+    out_dist = out_dist if out_dist is not None else torch.empty(k, dtype=torch.float32, device=dev)
+    out_count = out_count if out_count is not None else torch.empty(1, dtype=torch.int32, device=dev)
+    check(lib().adainf_select_retrain(C.byref(si), int(k), ptr(out_idx), ptr(out_dist), ptr(out_count),
+                                      ptr(dist_all), stream_ptr(stream)))
+    return out_idx, out_dist, out_count
+
+
+# ---- kernel-level (include/adainf_debug.h) ----
+def dbg_conv_fwd(x, w, b, stride, pad, act=0, res=None, out_f32=False, stream=None):
+    import torch
+    n, H, W_, Cc = x.shape
+    Co, KH, KW, _ = w.shape
+    Ho, Wo = (H + 2 * pad - KH) // stride + 1, (W_ + 2 * pad - KW) // stride + 1
+    out = torch.empty((n, Ho, Wo, Co), dtype=torch.float32 if out_f32 else torch.bfloat16, device=x.device)
+    check(lib().adainf_dbg_conv_fwd(ptr(x), n, H, W_, Cc, ptr(w), ptr(b), Co, KH, KW, stride, pad, act, ptr(res),
+                                    ptr(out), int(out_f32), stream_ptr(stream)))
+    return out
+
+
+def dbg_conv_dgrad(dz, w, H, W_, stride, pad, bcast=None, sc=None, yact=None, mask_act=0, stream=None):
+    import torch
+    n = dz.shape[0]
+    Co, KH, KW, Cc = w.shape
+    dx = torch.empty((n, H, W_, Cc), dtype=torch.bfloat16, device=dz.device)
+    check(lib().adainf_dbg_conv_dgrad(ptr(dz), n, H, W_, Cc, ptr(w), Co, KH, KW, stride, pad, ptr(bcast), ptr(sc),
+                                      ptr(yact), mask_act, ptr(dx), stream_ptr(stream)))
+    return dx
+
+
+def dbg_conv_wgrad(x, dz, KH, KW, stride, pad, stream=None):
+    import torch
+    n, H, W_, Cc = x.shape
+    Co = dz.shape[-1]
+    dw = torch.empty((Co, KH, KW, Cc), dtype=torch.float32, device=x.device)
+    db = torch.empty(Co, dtype=torch.float32, device=x.device)
+    check(lib().adainf_dbg_conv_wgrad(ptr(x), ptr(dz), n, H, W_, Cc, Co, KH, KW, stride, pad, ptr(dw), ptr(db),
+                                      stream_ptr(stream)))
+    return dw, db

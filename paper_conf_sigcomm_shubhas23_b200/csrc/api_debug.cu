@@ -1,0 +1,64 @@
+// Kernel-level entry points (include/adainf_debug.h) used by the per-kernel GPU parity tests.
+#include <cstring>
+
+#include "../../include/adainf_debug.h"
+#include "api_common.h"
+#include "runtime.h"
+
+using namespace adainf;
+
+static ConvGeom geom(int H, int W, int C, int Co, int KH, int KW, int s, int p) {
+  ConvGeom g;
+  g.Cin = C;
+  g.Cout = Co;
+  g.KH = KH;
+  g.KW = KW;
+  g.stride = s;
+  g.pad = p;
+  g.H = H;
+  g.W = W;
+  g.Ho = (H + 2 * p - KH) / s + 1;
+  g.Wo = (W + 2 * p - KW) / s + 1;
+  return g;
+}
+
+extern "C" adainf_status adainf_dbg_conv_fwd(const void* x, int32_t n, int32_t H, int32_t W, int32_t C,
+                                             const void* w, const float* b, int32_t Co, int32_t KH, int32_t KW,
+                                             int32_t stride, int32_t pad, int32_t act, const void* res, void* out,
+                                             int32_t out_f32, adainf_stream_t stream) {
+  return guard([&] {
+    if (C % 8 || n <= 0 || KH * KW > 49) throw ShapeError("conv_fwd: C must be a multiple of 8");
+    require_device();
+    ConvGeom g = geom(H, W, C, Co, KH, KW, stride, pad);
+    conv_fwd(g, (const bf16*)x, nullptr, nullptr, n, (const bf16*)w, KH * KW * C, b, (const bf16*)res, nullptr,
+             act, out, out_f32 != 0, (cudaStream_t)stream);
+  });
+}
+
+extern "C" adainf_status adainf_dbg_conv_dgrad(const void* dz, int32_t n, int32_t H, int32_t W, int32_t C,
+                                               const void* w, int32_t Co, int32_t KH, int32_t KW, int32_t stride,
+                                               int32_t pad, const float* bcast, const void* sc, const void* yact,
+                                               int32_t mask_act, void* dx, adainf_stream_t stream) {
+  return guard([&] {
+    if (C % 8 || Co % 8 || n <= 0) throw ShapeError("conv_dgrad: C, Co must be multiples of 8");
+    require_device();
+    ConvGeom g = geom(H, W, C, Co, KH, KW, stride, pad);
+    conv_dgrad(g, (const bf16*)dz, (const bf16*)w, KH * KW * C, n, bcast, (const bf16*)sc, (const bf16*)yact,
+               mask_act, (bf16*)dx, (cudaStream_t)stream);
+  });
+}
+
+extern "C" adainf_status adainf_dbg_conv_wgrad(const void* x, const void* dz, int32_t n, int32_t H, int32_t W,
+                                               int32_t C, int32_t Co, int32_t KH, int32_t KW, int32_t stride,
+                                               int32_t pad, float* dw, float* db, adainf_stream_t stream) {
+  return guard([&] {
+    if (C % 8 || Co % 8 || n <= 0) throw ShapeError("conv_wgrad: C, Co must be multiples of 8");
+    require_device();
+    ConvGeom g = geom(H, W, C, Co, KH, KW, stride, pad);
+    const size_t ws = wgrad_ws_bytes(g, n);
+    float* buf = nullptr;
+    CK(cudaMallocAsync((void**)&buf, ws, (cudaStream_t)stream));
+    conv_wgrad(g, (const bf16*)x, (const bf16*)dz, n, C, buf, ws, dw, db, (cudaStream_t)stream);
+    CK(cudaFreeAsync(buf, (cudaStream_t)stream));
+  });
+}

@@ -1,0 +1,253 @@
+// Host-side launchers for the tcgen05 implicit-GEMM conv kernels (fwd / dgrad phases / wgrad split-K
+// + deterministic reduction) and the bias-gradient column sums.
+#include <algorithm>
+#include <cstdio>
+#include <stdexcept>
+
+#include "conv_gemm.cuh"
+#include "runtime.h"
+
+namespace adainf {
+
+static int g_num_sms = 0;
+int num_sms() {
+  if (!g_num_sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
+    if (g_num_sms <= 0) g_num_sms = 148;
+  }
+  return g_num_sms;
+}
+
+template <int MODE, int BN>
+static void launch_t(const ConvArgs& a, dim3 grid, cudaStream_t st) {
+  using Cfg = ConvCfg<MODE, BN>;
+  static bool attr = false;
+  if (!attr) {
+    CK(cudaFuncSetAttribute(conv_umma_kernel<MODE, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
+    attr = true;
+  }
+  conv_umma_kernel<MODE, BN><<<grid, NUM_THREADS, Cfg::SMEM, st>>>(a);
+  CK(cudaGetLastError());
+}
+
+template <int MODE>
+static void launch_bn(int BN, const ConvArgs& a, dim3 grid, cudaStream_t st) {
+  switch (BN) {
+    case 32:
+      if constexpr (MODE == MODE_FWD) { launch_t<MODE, 32>(a, grid, st); return; }
+      break;
+    case 64: launch_t<MODE, 64>(a, grid, st); return;
+    case 128: launch_t<MODE, 128>(a, grid, st); return;
+    case 256: launch_t<MODE, 256>(a, grid, st); return;
+  }
+  throw std::runtime_error("unsupported BN");
+}
+
+static int pick_bn(int nout, bool mn_major_b) {
+  if (nout <= 32 && !mn_major_b) return 32;
+  if (nout <= 64) return 64;
+  if (nout <= 128) return 128;
+  return 256;
+}
+
+void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* count, int n_static,
+              const bf16* w, int ldb, const float* bias, const bf16* res, const int* res_map, int act, void* out,
+              bool out_f32, cudaStream_t st) {
+  ConvArgs a{};
+  a.src = x;
+  a.src_map = x_map;
+  a.Hs = g.H;
+  a.Ws = g.W;
+  a.Cs = g.Cin;
+  a.count = count;
+  a.n_static = n_static;
+  a.Hg = g.Ho;
+  a.Wg = g.Wo;
+  a.sy = g.stride;
+  a.sx = g.stride;
+  a.ntaps = g.KH * g.KW;
+  if (a.ntaps > MAX_TAPS) throw std::runtime_error("kernel too large");
+  for (int kh = 0; kh < g.KH; ++kh)
+    for (int kw = 0; kw < g.KW; ++kw) {
+      a.ty[kh * g.KW + kw] = (int8_t)(kh - g.pad);
+      a.tx[kh * g.KW + kw] = (int8_t)(kw - g.pad);
+    }
+  a.B = w;
+  a.ldb = ldb;
+  a.K = a.ntaps * g.Cin;
+  a.Nout = g.Cout;
+  a.out = out;
+  a.out_f32 = out_f32;
+  a.Ho = g.Ho;
+  a.Wo = g.Wo;
+  a.oys = a.oxs = 1;
+  a.bias = bias;
+  a.res = res;
+  a.res_map = res_map;
+  a.act = act;
+  const int BN = pick_bn(g.Cout, false);
+  const long long mt = ((long long)n_static * g.Ho * g.Wo + BM - 1) / BM;
+  dim3 grid((unsigned)mt, (g.Cout + BN - 1) / BN, 1);
+  if (mt == 0) return;
+  launch_bn<MODE_FWD>(BN, a, grid, st);
+}
+
+void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n, const float* bcast,
+                const bf16* sc, const bf16* yact, int mask_act, bf16* dx, cudaStream_t st) {
+  // dX[y] = sum_{kh: (y + pad - kh) % s == 0} dZ[(y + pad - kh)/s] W[kh]; split by output phase (py,px)
+  const int s = g.stride;
+  for (int py = 0; py < s; ++py)
+    for (int px = 0; px < s; ++px) {
+      ConvArgs a{};
+      a.src = dz;
+      a.Hs = g.Ho;
+      a.Ws = g.Wo;
+      a.Cs = g.Cout;
+      a.n_static = n;
+      a.Hg = (g.H - py + s - 1) / s;
+      a.Wg = (g.W - px + s - 1) / s;
+      if (a.Hg <= 0 || a.Wg <= 0) continue;
+      a.sy = a.sx = 1;
+      int nt = 0;
+      for (int kh = 0; kh < g.KH; ++kh) {
+        const int qy = py + g.pad - kh;
+        if (((qy % s) + s) % s) continue;
+        for (int kw = 0; kw < g.KW; ++kw) {
+          const int qx = px + g.pad - kw;
+          if (((qx % s) + s) % s) continue;
+          a.ty[nt] = (int8_t)((qy - (((qy % s) + s) % s)) / s);
+          a.tx[nt] = (int8_t)((qx - (((qx % s) + s) % s)) / s);
+          a.btap[nt] = (int16_t)(kh * g.KW + kw);
+          nt++;
+        }
+      }
+      a.ntaps = nt;
+      a.B = w;
+      a.ldb = ldb;
+      a.K = nt * g.Cout;
+      a.Nout = g.Cin;
+      a.out = dx;
+      a.Ho = g.H;
+      a.Wo = g.W;
+      a.oys = s;
+      a.oxs = s;
+      a.oyo = py;
+      a.oxo = px;
+      a.bcast = bcast;
+      a.sc = sc;
+      a.yact = yact;
+      a.mask_act = mask_act;
+      const int BN = pick_bn(g.Cin, true);
+      const long long mt = ((long long)n * a.Hg * a.Wg + BM - 1) / BM;
+      dim3 grid((unsigned)mt, (g.Cin + BN - 1) / BN, 1);
+      launch_bn<MODE_DGRAD>(BN, a, grid, st);
+    }
+}
+
+// partial [S][Kconv][Cout] -> dw [Cout][taps][cin_real] (fp32), summed over S in fixed order
+__global__ void wgrad_reduce_kernel(const float* __restrict__ part, int S, int Kconv, int Cout, int cin_pad,
+                                    int cin_real, float* __restrict__ dw) {
+  __shared__ float tile[32][33];
+  const int k0 = blockIdx.x * 32, c0 = blockIdx.y * 32;
+  const int tx = threadIdx.x, ty = threadIdx.y;  // 32 x 8
+  for (int r = ty; r < 32; r += 8) {
+    const int k = k0 + r, co = c0 + tx;
+    float acc = 0.f;
+    if (k < Kconv && co < Cout)
+      for (int s = 0; s < S; ++s) acc += part[((long long)s * Kconv + k) * Cout + co];
+    tile[r][tx] = acc;
+  }
+  __syncthreads();
+  for (int r = ty; r < 32; r += 8) {
+    const int co = c0 + r, k = k0 + tx;
+    if (k < Kconv && co < Cout) {
+      const int tap = k / cin_pad, ci = k - tap * cin_pad;
+      if (ci < cin_real) {
+        const int ntaps = Kconv / cin_pad;
+        dw[((long long)co * ntaps + tap) * cin_real + ci] = tile[tx][r];
+      }
+    }
+  }
+}
+
+// column sums of dz [P][C] -> db[C], deterministic: per-block fixed-order partials, then fixed-order sum
+__global__ void colsum_partial_kernel(const bf16* __restrict__ dz, long long P, int C, int rows_per_block,
+                                      float* __restrict__ part) {
+  const long long r0 = (long long)blockIdx.x * rows_per_block;
+  const long long r1 = min(P, r0 + rows_per_block);
+  for (int c = threadIdx.x; c < C; c += blockDim.x) {
+    float acc = 0.f;
+    for (long long r = r0; r < r1; ++r) acc += __bfloat162float(dz[r * C + c]);
+    part[(long long)blockIdx.x * C + c] = acc;
+  }
+}
+__global__ void colsum_final_kernel(const float* __restrict__ part, int nb, int C, float* __restrict__ out) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= C) return;
+  float acc = 0.f;
+  for (int b = 0; b < nb; ++b) acc += part[(long long)b * C + c];
+  out[c] = acc;
+}
+
+size_t wgrad_ws_bytes(const ConvGeom& g, int n) {
+  const long long npix = (long long)n * g.Ho * g.Wo;
+  const int nkb = (int)((npix + BK - 1) / BK);
+  const int Kconv = g.KH * g.KW * g.Cin;
+  const int BN = pick_bn(g.Cout, true);
+  const int tiles = ((Kconv + BM - 1) / BM) * ((g.Cout + BN - 1) / BN);
+  int S = std::max(1, std::min(nkb, (2 * num_sms() + tiles - 1) / tiles));
+  const int kbs = (nkb + S - 1) / S;
+  S = (nkb + kbs - 1) / kbs;
+  const long long colsum_blocks = (npix + 255) / 256;
+  return (size_t)S * Kconv * g.Cout * sizeof(float) + (size_t)colsum_blocks * g.Cout * sizeof(float);
+}
+
+void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin_real, float* ws, size_t ws_bytes,
+                float* dw, float* db, cudaStream_t st) {
+  const long long npix = (long long)n * g.Ho * g.Wo;
+  const int nkb = (int)((npix + BK - 1) / BK);
+  const int Kconv = g.KH * g.KW * g.Cin;
+  const int BN = pick_bn(g.Cout, true);
+  const int tiles = ((Kconv + BM - 1) / BM) * ((g.Cout + BN - 1) / BN);
+  int S = std::max(1, std::min(nkb, (2 * num_sms() + tiles - 1) / tiles));
+  const int kbs = (nkb + S - 1) / S;
+  S = (nkb + kbs - 1) / kbs;
+  if (wgrad_ws_bytes(g, n) > ws_bytes) throw std::runtime_error("wgrad workspace too small");
+  ConvArgs a{};
+  a.src = x;
+  a.Hs = g.H;
+  a.Ws = g.W;
+  a.Cs = g.Cin;
+  a.n_static = n;
+  a.Hg = g.Ho;
+  a.Wg = g.Wo;
+  a.sy = a.sx = g.stride;
+  a.ntaps = g.KH * g.KW;
+  for (int kh = 0; kh < g.KH; ++kh)
+    for (int kw = 0; kw < g.KW; ++kw) {
+      a.ty[kh * g.KW + kw] = (int8_t)(kh - g.pad);
+      a.tx[kh * g.KW + kw] = (int8_t)(kw - g.pad);
+    }
+  a.B = dz;
+  a.K = Kconv;
+  a.Nout = g.Cout;
+  a.out = ws;
+  a.kb_per_split = kbs;
+  dim3 grid((Kconv + BM - 1) / BM, (g.Cout + BN - 1) / BN, S);
+  launch_bn<MODE_WGRAD>(BN, a, grid, st);
+  dim3 rg((Kconv + 31) / 32, (g.Cout + 31) / 32);
+  wgrad_reduce_kernel<<<rg, dim3(32, 8), 0, st>>>(ws, S, Kconv, g.Cout, g.Cin, cin_real, dw);
+  CK(cudaGetLastError());
+  if (db) {
+    float* part = ws + (size_t)S * Kconv * g.Cout;
+    const int rpb = 256;
+    const int nb = (int)((npix + rpb - 1) / rpb);
+    colsum_partial_kernel<<<nb, 128, 0, st>>>(dz, npix, g.Cout, rpb, part);
+    colsum_final_kernel<<<(g.Cout + 127) / 128, 128, 0, st>>>(part, nb, g.Cout, db);
+    CK(cudaGetLastError());
+  }
+}
+
+}  // namespace adainf

@@ -1,0 +1,44 @@
+// Internal declarations of the AdaInf B200 runtime (host C++ side of libadainf.so).
+#pragma once
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include <stdexcept>
+#include <string>
+
+namespace adainf {
+
+typedef __nv_bfloat16 bf16;
+
+struct CudaError : std::runtime_error {
+  using std::runtime_error::runtime_error;
+};
+struct ShapeError : std::runtime_error {
+  using std::runtime_error::runtime_error;
+};
+
+#define CK(expr)                                                                                         \
+  do {                                                                                                   \
+    cudaError_t _e = (expr);                                                                             \
+    if (_e != cudaSuccess)                                                                               \
+      throw ::adainf::CudaError(std::string(#expr) + ": " + cudaGetErrorString(_e) + " @" + __FILE__ + ":" + \
+                                std::to_string(__LINE__));                                               \
+  } while (0)
+
+int num_sms();
+
+// conv geometry (Cin = padded input channels as stored, multiple of 8)
+struct ConvGeom {
+  int Cin, Cout, KH, KW, stride, pad, H, W, Ho, Wo;
+};
+
+void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* count, int n_static, const bf16* w,
+              int ldb, const float* bias, const bf16* res, const int* res_map, int act, void* out, bool out_f32,
+              cudaStream_t st);
+void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n, const float* bcast,
+                const bf16* sc, const bf16* yact, int mask_act, bf16* dx, cudaStream_t st);
+size_t wgrad_ws_bytes(const ConvGeom& g, int n);
+void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin_real, float* ws, size_t ws_bytes,
+                float* dw, float* db, cudaStream_t st);
+
+}  // namespace adainf

@@ -1,0 +1,130 @@
+"""Per-kernel GPU parity of the tcgen05 implicit-GEMM conv (fwd / dgrad / wgrad) through the C-ABI
+(include/adainf_debug.h).  Small shapes are checked against the oracle's direct-loop conv (fp64
+accumulation); all shapes against torch fp32 on the same bf16 operands.  Shapes span several M/N tiles,
+ragged tails, stride-2 phases, 1x1 / 3x3 / 7x7 kernels and every BN variant."""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_sigcomm_shubhas23_b200 import binding as B
+
+pytestmark = pytest.mark.gpu
+
+FWD_CASES = [  # n, H, W, C, Co, K, s, p
+    (2, 9, 7, 8, 32, 3, 1, 1),
+    (3, 14, 14, 64, 64, 3, 1, 1),
+    (2, 15, 13, 64, 128, 3, 2, 1),
+    (2, 8, 8, 128, 256, 1, 2, 0),
+    (1, 21, 20, 8, 64, 7, 2, 3),
+    (2, 7, 7, 256, 512, 3, 1, 1),
+    (5, 13, 13, 32, 24, 1, 1, 0),
+]
+
+
+def _rel(a, b):
+    a, b = a.double(), b.double()
+    return float((a - b).norm() / b.norm().clamp_min(1e-30))
+
+
+def _mk(case, seed):
+    n, H, W, C, Co, K, s, p = case
+    g = torch.Generator(device="cpu").manual_seed(seed)
+    x = torch.randn(n, H, W, C, generator=g).to(torch.bfloat16).cuda()
+    w = (torch.randn(Co, K, K, C, generator=g) * (2.0 / (K * K * C)) ** 0.5).to(torch.bfloat16).cuda()
+    b = (torch.randn(Co, generator=g) * 0.1).cuda()
+    return x, w, b
+
+
+def _ref_fwd(x, w, b, s, p):
+    return torch.nn.functional.conv2d(x.float().permute(0, 3, 1, 2), w.float().permute(0, 3, 1, 2), b, stride=s,
+                                      padding=p).permute(0, 2, 3, 1)
+
+
+@pytest.mark.parametrize("case", FWD_CASES)
+@pytest.mark.parametrize("act", [0, 1, 2])
+def test_conv_fwd_vs_torch(case, act):
+    n, H, W, C, Co, K, s, p = case
+    x, w, b = _mk(case, 1)
+    ref = _ref_fwd(x, w, b, s, p)
+    if act == 1:
+        ref = torch.relu(ref)
+    elif act == 2:
+        ref = torch.where(ref > 0, ref, 0.1 * ref)
+    out = B.dbg_conv_fwd(x, w, b, s, p, act=act)
+    torch.cuda.synchronize()
+    assert out.shape == ref.shape
+    assert _rel(out.float(), ref) < 8e-3
+
+
+def test_conv_fwd_residual_and_f32_out():
+    case = (3, 14, 14, 64, 64, 3, 1, 1)
+    x, w, b = _mk(case, 2)
+    res = torch.randn(3, 14, 14, 64).to(torch.bfloat16).cuda()
+    ref = torch.relu(_ref_fwd(x, w, b, 1, 1) + res.float())
+    out = B.dbg_conv_fwd(x, w, b, 1, 1, act=1, res=res)
+    assert _rel(out.float(), ref) < 8e-3
+    case = (4, 13, 13, 64, 21, 1, 1, 0)
+    x, w, b = _mk(case, 3)
+    out = B.dbg_conv_fwd(x, w, b, 1, 0, act=0, out_f32=True)
+    assert out.dtype == torch.float32
+    assert _rel(out, _ref_fwd(x, w, b, 1, 0)) < 1e-4
+
+
+def test_conv_fwd_vs_oracle_exact_small():
+    """fp32 accumulate vs the oracle's fp64 sum, then bf16 rounding on both: nearly all equal."""
+    import oracle as O
+    case = (2, 9, 7, 16, 32, 3, 2, 1)
+    x, w, b = _mk(case, 4)
+    out = B.dbg_conv_fwd(x, w, b, 2, 1, act=0).float().cpu().numpy()
+    xs, ws, bs = x.float().cpu().numpy(), w.float().cpu().numpy(), b.cpu().numpy()
+    for i in range(2):
+        acc = O.conv_acc(xs[i], ws, 2, 1) + bs
+        ref = O.bf16(acc.astype(np.float32))
+        mism = np.mean(ref != out[i])
+        assert mism < 0.01, mism
+        np.testing.assert_allclose(out[i], ref, rtol=1e-2, atol=1e-2)
+
+
+@pytest.mark.parametrize("case", [c for c in FWD_CASES if c[4] % 8 == 0])
+def test_conv_dgrad_vs_torch(case):
+    n, H, W, C, Co, K, s, p = case
+    x, w, b = _mk(case, 5)
+    Ho, Wo = (H + 2 * p - K) // s + 1, (W + 2 * p - K) // s + 1
+    dz = torch.randn(n, Ho, Wo, Co).to(torch.bfloat16).cuda()
+    ref = torch.nn.grad.conv2d_input((n, C, H, W), w.float().permute(0, 3, 1, 2), dz.float().permute(0, 3, 1, 2),
+                                     stride=s, padding=p).permute(0, 2, 3, 1)
+    dx = B.dbg_conv_dgrad(dz, w, H, W, s, p)
+    torch.cuda.synchronize()
+    assert _rel(dx.float(), ref) < 8e-3
+
+
+def test_conv_dgrad_epilogue_terms():
+    case = (2, 14, 14, 64, 128, 3, 2, 1)
+    n, H, W, C, Co, K, s, p = case
+    x, w, b = _mk(case, 6)
+    dz = torch.randn(n, 7, 7, Co).to(torch.bfloat16).cuda()
+    bc = torch.randn(n, C).cuda() * 0.01
+    sc = torch.randn(n, H, W, C).to(torch.bfloat16).cuda()
+    y = torch.randn(n, H, W, C).to(torch.bfloat16).cuda()
+    ref = torch.nn.grad.conv2d_input((n, C, H, W), w.float().permute(0, 3, 1, 2), dz.float().permute(0, 3, 1, 2),
+                                     stride=s, padding=p).permute(0, 2, 3, 1)
+    ref = (ref + bc[:, None, None, :] + sc.float()) * (y.float() > 0)
+    dx = B.dbg_conv_dgrad(dz, w, H, W, s, p, bcast=bc, sc=sc, yact=y, mask_act=1)
+    assert _rel(dx.float(), ref) < 8e-3
+
+
+@pytest.mark.parametrize("case", [c for c in FWD_CASES if c[4] % 8 == 0])
+def test_conv_wgrad_vs_torch(case):
+    n, H, W, C, Co, K, s, p = case
+    x, w, b = _mk(case, 7)
+    Ho, Wo = (H + 2 * p - K) // s + 1, (W + 2 * p - K) // s + 1
+    dz = torch.randn(n, Ho, Wo, Co).to(torch.bfloat16).cuda()
+    ref = torch.nn.grad.conv2d_weight(x.float().permute(0, 3, 1, 2), (Co, C, K, K), dz.float().permute(0, 3, 1, 2),
+                                      stride=s, padding=p).permute(0, 2, 3, 1)
+    dw, db = B.dbg_conv_wgrad(x, dz, K, K, s, p)
+    torch.cuda.synchronize()
+    assert _rel(dw, ref) < 1e-4
+    assert _rel(db, dz.float().sum(dim=(0, 1, 2))) < 1e-5
+    # deterministic: same bits on a second run
+    dw2, db2 = B.dbg_conv_wgrad(x, dz, K, K, s, p)
+    assert torch.equal(dw, dw2) and torch.equal(db, db2)
