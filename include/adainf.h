@@ -111,6 +111,8 @@ adainf_status adainf_model_set_params(adainf_model_t m, const float* host_src, i
 /* device pointer to the flat fp32 gradient of the last retrain step (num_params floats), for
  * inspection and for callers that reduce gradients themselves. */
 adainf_status adainf_model_grad_ptr(adainf_model_t m, float** dev_ptr);
+/* host copy of that gradient (synchronizing) */
+adainf_status adainf_model_get_grads(adainf_model_t m, float* host_dst, int64_t n);
 
 /* ---- Application DAG (Fig. 1): root model first, routing edges between models ---------- */
 typedef enum {

@@ -82,6 +82,7 @@ def lib():
             "adainf_model_get_params": [vp, C.POINTER(C.c_float), i64],
             "adainf_model_set_params": [vp, C.POINTER(C.c_float), i64],
             "adainf_model_grad_ptr": [vp, C.POINTER(vp)],
+            "adainf_model_get_grads": [vp, C.POINTER(C.c_float), i64],
             "adainf_app_create": [C.POINTER(AppSpec), C.POINTER(vp)],
             "adainf_app_destroy": [vp],
             "adainf_infer_dag": [vp, vp, i32, C.POINTER(C.c_float), i32, C.POINTER(ModelOut), vp],
@@ -140,6 +141,16 @@ def make_ops(spec):
     return ops
 
 
+def _exit0_channels(spec):
+    Cc = spec["in_c"]
+    for o in spec["ops"]:
+        if o["kind"] == "conv":
+            Cc = o["cout"]
+        elif o["kind"] == "exit":
+            return Cc
+    return 0
+
+
 class Model:
     """Owns an adainf_model_t."""
 
@@ -162,6 +173,7 @@ class Model:
         self.num_exits = e.value
         self.ncls = next((o["num_classes"] for o in spec["ops"] if o["kind"] == "exit"), 0)
         self.max_batch = max_batch
+        self.exit0_channels = _exit0_channels(spec)
 
     def get_params(self):
         out = np.zeros(self.num_params, np.float32)
@@ -172,18 +184,10 @@ class Model:
         p = np.ascontiguousarray(p, np.float32)
         check(lib().adainf_model_set_params(self.h, p.ctypes.data_as(C.POINTER(C.c_float)), self.num_params))
 
-    def grad(self):
-        import torch
-        vp = C.c_void_p()
-        check(lib().adainf_model_grad_ptr(self.h, C.byref(vp)))
-        # copy out through torch (device -> host) for inspection
-        buf = torch.empty(self.num_params, dtype=torch.float32, device="cuda")
-        C.memmove  # noqa: B018
-        torch.cuda.synchronize()
-        import ctypes
-        cudart = torch.cuda.cudart()
-        cudart.cudaMemcpy(buf.data_ptr(), vp.value, self.num_params * 4, 3)  # D2D
-        return buf
+    def get_grads(self):
+        out = np.zeros(self.num_params, np.float32)
+        check(lib().adainf_model_get_grads(self.h, out.ctypes.data_as(C.POINTER(C.c_float)), self.num_params))
+        return out
 
     def retrain_step(self, samples, labels, n_global=None, lr=0.01, stats=None, stream=None):
         check(lib().adainf_retrain_step(self.h, ptr(samples), ptr(labels), int(samples.shape[0]),
@@ -204,6 +208,30 @@ class Model:
             self.close()
         except Exception:
             pass
+
+
+def alloc_outs(model, rows, max_det=0, n_out_edges=0, max_routed=0, device="cuda"):
+    """Per-model output buffers of adainf_infer_dag as torch tensors (rows = input rows capacity)."""
+    import torch
+    E, NC = model.num_exits, model.ncls
+    o = {}
+    if E:
+        o["exit_id"] = torch.full((rows,), -1, dtype=torch.int8, device=device)
+        o["pred"] = torch.full((rows,), -1, dtype=torch.int32, device=device)
+        o["conf"] = torch.zeros(rows, dtype=torch.float32, device=device)
+        o["entropy"] = torch.zeros(rows, dtype=torch.float32, device=device)
+        o["logits"] = torch.zeros((rows, NC), dtype=torch.float32, device=device)
+        o["exit_counts"] = torch.zeros(E, dtype=torch.int32, device=device)
+        o["surv_idx"] = torch.full((max(E - 1, 1), rows), -1, dtype=torch.int32, device=device)
+        c0 = model.exit0_channels
+        o["embed"] = torch.zeros((rows, c0), dtype=torch.float32, device=device)
+    if max_det:
+        o["n_det"] = torch.zeros(1, dtype=torch.int32, device=device)
+        o["det_table"] = torch.zeros((max_det, 9), dtype=torch.float32, device=device)
+    if n_out_edges:
+        o["route_idx"] = torch.full((n_out_edges, max_routed), -1, dtype=torch.int32, device=device)
+        o["n_routed"] = torch.zeros(n_out_edges, dtype=torch.int32, device=device)
+    return o
 
 
 def nccl_unique_id() -> bytes:

@@ -1,0 +1,478 @@
+// CUDA-core kernels of the AdaInf hot path: input packing, max-pooling (fwd/bwd), the fused early-exit
+// head (GAP -> FC -> softmax confidence / entropy / argmax -> threshold), the stable
+// survivor compaction (ballot + block scan), exit losses and head gradients (a8-a9), and the fused
+// SGD-momentum update with bf16-shadow refresh (a11).  All reductions use a fixed order (deterministic).
+#include <cuda_bf16.h>
+
+#include "common.cuh"
+#include "kernels.cuh"
+
+namespace adainf {
+
+// ------------------------------------------------------------------------------------------------
+__global__ void pack_input_kernel(const bf16* __restrict__ x, const int* __restrict__ map, const int* count,
+                                  int n_static, int HW, int Cin, int Cpad, bf16* __restrict__ y) {
+  const int n_rows = count ? *count : n_static;
+  const long long total = (long long)n_rows * HW;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+    const long long n = i / HW, pix = i - n * HW;
+    const long long src = (map ? map[n] : n) * (long long)HW + pix;
+    bf16* o = y + i * Cpad;
+    for (int c = 0; c < Cpad; ++c) o[c] = c < Cin ? x[src * Cin + c] : __float2bfloat16_rn(0.f);
+  }
+}
+void launch_pack_input(const bf16* x, const int* map, const int* count, int n_static, int H, int W, int Cin, int Cpad,
+                       bf16* y, cudaStream_t st) {
+  const long long total = (long long)n_static * H * W;
+  const int blocks = (int)std::min<long long>((total + 255) / 256, 16LL * num_sms());
+  if (blocks <= 0) return;
+  pack_input_kernel<<<blocks, 256, 0, st>>>(x, map, count, n_static, H * W, Cin, Cpad, y);
+  CK(cudaGetLastError());
+}
+
+// ------------------------------------------------------------------------------------------------
+__global__ void maxpool_fwd_kernel(const bf16* __restrict__ x, const int* __restrict__ map, const int* count,
+                                   int n_static, int H, int W, int C, int K, int s, int p, int Ho, int Wo,
+                                   bf16* __restrict__ y, uint8_t* __restrict__ amax) {
+  const int n_rows = count ? *count : n_static;
+  const int CV = C / 8;
+  const long long total = (long long)n_rows * Ho * Wo * CV;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+    const int cv = (int)(i % CV);
+    long long r = i / CV;
+    const int wo = (int)(r % Wo);
+    r /= Wo;
+    const int ho = (int)(r % Ho);
+    const long long n = r / Ho;
+    const long long sn = map ? map[n] : n;
+    float best[8];
+    uint8_t arg[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      best[q] = -INFINITY;
+      arg[q] = 0;
+    }
+    for (int kh = 0; kh < K; ++kh) {
+      const int ih = ho * s - p + kh;
+      if (ih < 0 || ih >= H) continue;
+      for (int kw = 0; kw < K; ++kw) {
+        const int iw = wo * s - p + kw;
+        if (iw < 0 || iw >= W) continue;
+        const uint4 raw = *(const uint4*)(x + ((sn * H + ih) * W + iw) * C + cv * 8);
+        const bf16* h = (const bf16*)&raw;
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+          const float v = __bfloat162float(h[q]);
+          if (v > best[q]) {  // strict: the FIRST maximal element in row-major window order
+            best[q] = v;
+            arg[q] = (uint8_t)(kh * K + kw);
+          }
+        }
+      }
+    }
+    __align__(16) bf16 o[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) o[q] = __float2bfloat16_rn(best[q]);
+    const long long oi = ((n * Ho + ho) * Wo + wo) * C + cv * 8;
+    *(uint4*)(y + oi) = *(uint4*)o;
+    if (amax) *(uint2*)(amax + oi) = *(uint2*)arg;
+  }
+}
+void launch_maxpool_fwd(const bf16* x, const int* map, const int* count, int n_static, int H, int W, int C, int K,
+                        int s, int p, int Ho, int Wo, bf16* y, uint8_t* amax, cudaStream_t st) {
+  const long long total = (long long)n_static * Ho * Wo * (C / 8);
+  const int blocks = (int)std::min<long long>((total + 255) / 256, 32LL * num_sms());
+  if (blocks <= 0) return;
+  maxpool_fwd_kernel<<<blocks, 256, 0, st>>>(x, map, count, n_static, H, W, C, K, s, p, Ho, Wo, y, amax);
+  CK(cudaGetLastError());
+}
+
+__global__ void maxpool_bwd_kernel(const bf16* __restrict__ dT, const uint8_t* __restrict__ amax,
+                                   const bf16* __restrict__ yact, int act, long long n, int H, int W, int C, int K,
+                                   int s, int p, int Ho, int Wo, bf16* __restrict__ dz) {
+  const long long total = n * H * W * C;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+    const int c = (int)(i % C);
+    long long r = i / C;
+    const int iw = (int)(r % W);
+    r /= W;
+    const int ih = (int)(r % H);
+    const long long b = r / H;
+    // windows ho with ho*s - p <= ih <= ho*s - p + K - 1
+    const int ho_lo = max(0, (ih + p - K + s) / s), ho_hi = min(Ho - 1, (ih + p) / s);
+    const int wo_lo = max(0, (iw + p - K + s) / s), wo_hi = min(Wo - 1, (iw + p) / s);
+    float acc = 0.f;
+    for (int ho = ho_lo; ho <= ho_hi; ++ho) {
+      const int kh = ih - (ho * s - p);
+      if (kh < 0 || kh >= K) continue;
+      for (int wo = wo_lo; wo <= wo_hi; ++wo) {
+        const int kw = iw - (wo * s - p);
+        if (kw < 0 || kw >= K) continue;
+        const long long oi = ((b * Ho + ho) * Wo + wo) * C + c;
+        if (amax[oi] == (uint8_t)(kh * K + kw)) acc = __fadd_rn(acc, __bfloat162float(dT[oi]));
+      }
+    }
+    const float g = __fmul_rn(acc, act_grad(act, __bfloat162float(yact[i])));
+    dz[i] = __float2bfloat16_rn(g);
+  }
+}
+void launch_maxpool_bwd(const bf16* dT, const uint8_t* amax, const bf16* yact, int act, int n, int H, int W, int C,
+                        int K, int s, int p, int Ho, int Wo, bf16* dz, cudaStream_t st) {
+  const long long total = (long long)n * H * W * C;
+  const int blocks = (int)std::min<long long>((total + 255) / 256, 32LL * num_sms());
+  maxpool_bwd_kernel<<<blocks, 256, 0, st>>>(dT, amax, yact, act, n, H, W, C, K, s, p, Ho, Wo, dz);
+  CK(cudaGetLastError());
+}
+
+// ------------------------------------------------------------------------------------------------
+// Fused exit head: one CTA per dense row.  GAP over HW with 16-byte loads (channel vector v = t % (C/8),
+// pixel group t / (C/8)), fixed-order reduction, FC in fp32, softmax statistics with IEEE expf/logf.
+constexpr int EH_THREADS = 256;
+__global__ void __launch_bounds__(EH_THREADS) exit_head_kernel(const ExitHeadArgs a) {
+  const int n_rows = a.count ? *a.count : a.n_static;
+  const int j = blockIdx.x;
+  if (j >= n_rows) return;
+  extern __shared__ float sh[];  // [EH_THREADS/CV][C] partials, then pooled[C], logits[ncls]
+  const int C = a.C, CV = C / 8;
+  const int groups = EH_THREADS / CV;
+  const int t = threadIdx.x;
+  float acc[8];
+#pragma unroll
+  for (int q = 0; q < 8; ++q) acc[q] = 0.f;
+  const int v = t % CV, g0 = t / CV;
+  if (g0 < groups) {
+    const bf16* base = a.fmap + (long long)j * a.HW * C + v * 8;
+    for (int pix = g0; pix < a.HW; pix += groups) {
+      const uint4 raw = __ldg((const uint4*)(base + (long long)pix * C));
+      const bf16* h = (const bf16*)&raw;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) acc[q] += __bfloat162float(h[q]);
+    }
+#pragma unroll
+    for (int q = 0; q < 8; ++q) sh[g0 * C + v * 8 + q] = acc[q];
+  }
+  __syncthreads();
+  float* pooled = sh + groups * C;
+  float* logits = pooled + C;
+  const float inv_hw = 1.0f / (float)a.HW;
+  for (int c = t; c < C; c += EH_THREADS) {
+    float s = 0.f;
+    for (int g = 0; g < groups; ++g) s += sh[g * C + c];
+    pooled[c] = s * inv_hw;
+  }
+  __syncthreads();
+  for (int k = t; k < a.ncls; k += EH_THREADS) {
+    float l = a.bk[k];
+    for (int c = 0; c < C; ++c) l = fmaf(pooled[c], a.Wk[c * a.ncls + k], l);
+    logits[k] = l;
+  }
+  __syncthreads();
+  const int orig = a.orig ? a.orig[j] : j;
+  if (a.embed)
+    for (int c = t; c < C; c += EH_THREADS) a.embed[(long long)orig * C + c] = pooled[c];
+  if (a.pooled_save)
+    for (int c = t; c < C; c += EH_THREADS) a.pooled_save[(long long)j * C + c] = pooled[c];
+  if (a.logits_save)
+    for (int k = t; k < a.ncls; k += EH_THREADS) a.logits_save[(long long)j * a.ncls + k] = logits[k];
+  __shared__ int s_exit;
+  if (t == 0) {
+    int am = 0;
+    for (int k = 1; k < a.ncls; ++k)
+      if (logits[k] > logits[am]) am = k;
+    const float m = logits[am];
+    float s = 0.f, tt = 0.f;
+    for (int k = 0; k < a.ncls; ++k) {
+      const float e = expf(logits[k] - m);
+      s += e;
+      tt += e * (logits[k] - m);
+    }
+    const float conf = 1.0f / s;
+    const float ent = logf(s) - tt / s;
+    const int ex = a.is_final || conf >= a.tau;
+    s_exit = ex;
+    if (a.alive) a.alive[j] = (uint8_t)(!ex);
+    if (ex) {
+      if (a.exit_id) a.exit_id[orig] = (int8_t)a.exit_index;
+      if (a.pred) a.pred[orig] = am;
+      if (a.conf) a.conf[orig] = conf;
+      if (a.entropy) a.entropy[orig] = ent;
+    }
+  }
+  __syncthreads();
+  if (s_exit && a.logits)
+    for (int k = t; k < a.ncls; k += EH_THREADS) a.logits[(long long)orig * a.ncls + k] = logits[k];
+}
+void launch_exit_head(const ExitHeadArgs& a, cudaStream_t st) {
+  if (a.C % 8 || (EH_THREADS % (a.C / 8)) != 0 || a.C / 8 > EH_THREADS)
+    throw ShapeError("exit head: C must be 8 * a power of two <= 2048");
+  const int groups = EH_THREADS / (a.C / 8);
+  const size_t smem = (size_t)(groups * a.C + a.C + a.ncls) * sizeof(float);
+  if (a.n_static <= 0) return;
+  exit_head_kernel<<<a.n_static, EH_THREADS, smem, st>>>(a);
+  CK(cudaGetLastError());
+}
+
+// ------------------------------------------------------------------------------------------------
+// Stable compaction of alive rows (warp ballot + popc, block scan), single CTA, rows in chunks of 1024.
+__global__ void __launch_bounds__(1024) compact_kernel(const uint8_t* __restrict__ alive, const int* count,
+                                                       int n_static, const int* __restrict__ orig,
+                                                       int* __restrict__ pos_next, int* __restrict__ orig_next,
+                                                       int* count_next, int32_t* counts_out, int exit_index,
+                                                       int32_t* surv_out, int32_t* last_count_out, int last_index) {
+  __shared__ int warp_tot[32];
+  __shared__ int base_s;
+  const int n_rows = count ? *count : n_static;
+  const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+  if (t == 0) base_s = 0;
+  __syncthreads();
+  for (int c0 = 0; c0 < n_rows; c0 += 1024) {
+    const int j = c0 + t;
+    const bool f = j < n_rows && alive[j];
+    const unsigned bal = __ballot_sync(0xffffffffu, f);
+    const int wpre = __popc(bal & ((1u << lane) - 1u));
+    if (lane == 0) warp_tot[w] = __popc(bal);
+    __syncthreads();
+    if (w == 0) {
+      int v = warp_tot[lane];
+      for (int o = 1; o < 32; o <<= 1) {
+        const int u = __shfl_up_sync(0xffffffffu, v, o);
+        if (lane >= o) v += u;
+      }
+      warp_tot[lane] = v;  // inclusive
+    }
+    __syncthreads();
+    const int base = base_s;
+    const int wbase = w ? warp_tot[w - 1] : 0;
+    if (f) {
+      const int o = base + wbase + wpre;
+      const int og = orig ? orig[j] : j;
+      pos_next[o] = j;
+      orig_next[o] = og;
+      if (surv_out) surv_out[o] = og;
+    }
+    __syncthreads();
+    if (t == 0) base_s = base + warp_tot[31];
+    __syncthreads();
+  }
+  if (t == 0) {
+    const int nn = base_s;
+    *count_next = nn;
+    if (counts_out) {
+      counts_out[exit_index] = n_rows - nn;
+      if (last_count_out) counts_out[last_index] = nn;
+    }
+  }
+}
+void launch_compact(const uint8_t* alive, const int* count, int n_static, const int* orig, int* pos_next,
+                    int* orig_next, int* count_next, int32_t* counts_out, int exit_index, int32_t* surv_out,
+                    int32_t* last_count_out, int last_index, cudaStream_t st) {
+  compact_kernel<<<1, 1024, 0, st>>>(alive, count, n_static, orig, pos_next, orig_next, count_next, counts_out,
+                                     exit_index, surv_out, last_count_out, last_index);
+  CK(cudaGetLastError());
+}
+
+// ------------------------------------------------------------------------------------------------
+__global__ void exit_loss_kernel(const float* __restrict__ logits, const int32_t* __restrict__ labels, int n,
+                                 int ncls, float w, float inv_n, float* __restrict__ dl, float* __restrict__ loss_rows,
+                                 int accumulate) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const float* l = logits + (long long)i * ncls;
+  float m = l[0];
+  for (int k = 1; k < ncls; ++k) m = fmaxf(m, l[k]);
+  float s = 0.f;
+  for (int k = 0; k < ncls; ++k) s += expf(l[k] - m);
+  const int y = labels[i];
+  for (int k = 0; k < ncls; ++k) {
+    const float p = expf(l[k] - m) / s;
+    dl[(long long)i * ncls + k] = w * (p - (k == y ? 1.f : 0.f)) * inv_n;
+  }
+  const float ce = (logf(s) - (l[y] - m)) * w * inv_n;
+  loss_rows[i] = accumulate ? loss_rows[i] + ce : ce;
+}
+void launch_exit_loss(const float* logits, const int32_t* labels, int n, int ncls, float w, float inv_n, float* dl,
+                      float* loss_rows, int accumulate, cudaStream_t st) {
+  exit_loss_kernel<<<(n + 127) / 128, 128, 0, st>>>(logits, labels, n, ncls, w, inv_n, dl, loss_rows, accumulate);
+  CK(cudaGetLastError());
+}
+
+__global__ void head_dw_kernel(const float* __restrict__ pooled, const float* __restrict__ dl, int n, int C, int ncls,
+                               float* __restrict__ dW, float* __restrict__ db) {
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx < C * ncls) {
+    const int c = idx / ncls, k = idx - c * ncls;
+    float acc = 0.f;
+    for (int i = 0; i < n; ++i) acc = fmaf(pooled[(long long)i * C + c], dl[(long long)i * ncls + k], acc);
+    dW[idx] = acc;
+  } else if (idx < C * ncls + ncls) {
+    const int k = idx - C * ncls;
+    float acc = 0.f;
+    for (int i = 0; i < n; ++i) acc += dl[(long long)i * ncls + k];
+    db[k] = acc;
+  }
+}
+__global__ void head_bcast_kernel(const float* __restrict__ dl, const float* __restrict__ Wk, int n, int C, int ncls,
+                                  float inv_hw, float* __restrict__ bcast) {
+  const long long idx = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+  if (idx >= (long long)n * C) return;
+  const int c = (int)(idx % C);
+  const long long i = idx / C;
+  float acc = 0.f;
+  for (int k = 0; k < ncls; ++k) acc = fmaf(dl[i * ncls + k], Wk[c * ncls + k], acc);
+  bcast[idx] = acc * inv_hw;
+}
+void launch_head_grads(const float* pooled, const float* dl, const float* Wk, int n, int C, int ncls, int HW,
+                       float* dW, float* db, float* bcast, cudaStream_t st) {
+  const int tot = C * ncls + ncls;
+  head_dw_kernel<<<(tot + 127) / 128, 128, 0, st>>>(pooled, dl, n, C, ncls, dW, db);
+  const long long nb = ((long long)n * C + 255) / 256;
+  head_bcast_kernel<<<(unsigned)nb, 256, 0, st>>>(dl, Wk, n, C, ncls, 1.0f / (float)HW, bcast);
+  CK(cudaGetLastError());
+}
+
+__global__ void grad_finalize_kernel(const float* __restrict__ bcast, const bf16* __restrict__ sc,
+                                     const bf16* __restrict__ yact, int act, long long n, int HW, int C,
+                                     bf16* __restrict__ dz) {
+  const long long total = n * HW * C;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+    const int c = (int)(i % C);
+    const long long b = i / ((long long)HW * C);
+    float v = 0.f;
+    if (bcast) v = __fadd_rn(v, bcast[b * C + c]);
+    if (sc) v = __fadd_rn(v, __bfloat162float(sc[i]));
+    v = __fmul_rn(v, act_grad(act, __bfloat162float(yact[i])));
+    dz[i] = __float2bfloat16_rn(v);
+  }
+}
+void launch_grad_finalize(const float* bcast, const bf16* sc, const bf16* yact, int act, int n, int HW, int C,
+                          bf16* dz, cudaStream_t st) {
+  const long long total = (long long)n * HW * C;
+  const int blocks = (int)std::min<long long>((total + 255) / 256, 32LL * num_sms());
+  grad_finalize_kernel<<<blocks, 256, 0, st>>>(bcast, sc, yact, act, n, HW, C, dz);
+  CK(cudaGetLastError());
+}
+
+__global__ void sum_kernel(const float* __restrict__ x, int n, float* out, float scale) {
+  __shared__ float sh[1024];
+  float acc = 0.f;
+  for (int i = threadIdx.x; i < n; i += blockDim.x) acc += x[i];
+  sh[threadIdx.x] = acc;
+  __syncthreads();
+  for (int o = blockDim.x / 2; o > 0; o >>= 1) {
+    if (threadIdx.x < o) sh[threadIdx.x] += sh[threadIdx.x + o];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *out = scale == 0.f ? sh[0] : (scale < 0.f ? sqrtf(sh[0]) : sh[0] * scale);
+}
+void launch_sum(const float* x, int n, float* out, float scale, cudaStream_t st) {
+  sum_kernel<<<1, 1024, 0, st>>>(x, n, out, scale);
+  CK(cudaGetLastError());
+}
+
+// ------------------------------------------------------------------------------------------------
+// Fused SGD + momentum (PyTorch semantics, reading Q9), 128-bit loads/stores of w, v, g, and the bf16
+// shadow written in the GEMM-ready [Cout][ldb] layout for conv weights.  Blocks map to parameter
+// segments through host-built tables so every thread's float4 stays inside one segment.
+constexpr int SGD_THREADS = 256, SGD_VEC = 4, SGD_ITEMS = 4;
+constexpr int SGD_PER_BLOCK = SGD_THREADS * SGD_VEC * SGD_ITEMS;
+
+__device__ __forceinline__ void shadow_store(const SgdSeg& sg, long long local, const float* w4, int cnt) {
+  const int K = sg.taps * sg.cin;
+  for (int q = 0; q < cnt; ++q) {
+    const long long l = local + q;
+    const long long co = l / K;
+    const int rem = (int)(l - co * K);
+    const int tap = rem / sg.cin, ci = rem - tap * sg.cin;
+    sg.shadow[co * sg.ldb + tap * sg.cin_pad + ci] = __float2bfloat16_rn(w4[q]);
+  }
+}
+
+__global__ void __launch_bounds__(SGD_THREADS) sgd_kernel(float* __restrict__ w, float* __restrict__ v,
+                                                          const float* __restrict__ g, float lr, float mu, float wd,
+                                                          const SgdSeg* __restrict__ segs,
+                                                          const int* __restrict__ block_seg,
+                                                          const long long* __restrict__ block_start,
+                                                          float* __restrict__ sq_partial) {
+  const SgdSeg sg = segs[block_seg[blockIdx.x]];
+  const long long start = block_start[blockIdx.x];
+  const long long end = min(sg.off + sg.count, start + (long long)SGD_PER_BLOCK);
+  float sq = 0.f;
+  const bool vec_ok = ((sg.off & 3) == 0);
+#pragma unroll
+  for (int it = 0; it < SGD_ITEMS; ++it) {
+    const long long i = start + ((long long)it * SGD_THREADS + threadIdx.x) * SGD_VEC;
+    if (i >= end) continue;
+    const int cnt = (int)min((long long)SGD_VEC, end - i);
+    float wr[4], vr[4], gr[4];
+    if (vec_ok && cnt == 4) {
+      const float4 a = *(const float4*)(w + i), b = *(const float4*)(v + i), c = __ldg((const float4*)(g + i));
+      wr[0] = a.x, wr[1] = a.y, wr[2] = a.z, wr[3] = a.w;
+      vr[0] = b.x, vr[1] = b.y, vr[2] = b.z, vr[3] = b.w;
+      gr[0] = c.x, gr[1] = c.y, gr[2] = c.z, gr[3] = c.w;
+    } else {
+      for (int q = 0; q < cnt; ++q) wr[q] = w[i + q], vr[q] = v[i + q], gr[q] = g[i + q];
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (q < cnt) {
+        sq = fmaf(gr[q], gr[q], sq);
+        const float d = __fadd_rn(gr[q], __fmul_rn(wd, wr[q]));
+        vr[q] = __fadd_rn(__fmul_rn(mu, vr[q]), d);
+        wr[q] = __fsub_rn(wr[q], __fmul_rn(lr, vr[q]));
+      }
+    }
+    if (vec_ok && cnt == 4) {
+      *(float4*)(w + i) = make_float4(wr[0], wr[1], wr[2], wr[3]);
+      *(float4*)(v + i) = make_float4(vr[0], vr[1], vr[2], vr[3]);
+    } else {
+      for (int q = 0; q < cnt; ++q) w[i + q] = wr[q], v[i + q] = vr[q];
+    }
+    if (sg.shadow) {
+      const long long local = i - sg.off;
+      if (sg.cin == sg.cin_pad && (sg.cin & 3) == 0 && cnt == 4 && (local & 3) == 0) {
+        const int K = sg.taps * sg.cin;
+        const long long co = local / K;
+        const int rem = (int)(local - co * K);
+        __align__(8) bf16 h[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) h[q] = __float2bfloat16_rn(wr[q]);
+        *(uint2*)(sg.shadow + co * sg.ldb + rem) = *(uint2*)h;
+      } else {
+        shadow_store(sg, local, wr, cnt);
+      }
+    }
+  }
+  // fixed-order block reduction of sum g^2 (for the grad-norm statistic)
+  __shared__ float red[SGD_THREADS];
+  red[threadIdx.x] = sq;
+  __syncthreads();
+  for (int o = SGD_THREADS / 2; o > 0; o >>= 1) {
+    if (threadIdx.x < o) red[threadIdx.x] += red[threadIdx.x + o];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0 && sq_partial) sq_partial[blockIdx.x] = red[0];
+}
+void launch_sgd(float* w, float* v, const float* g, long long n, float lr, float mu, float wd, const SgdSeg* segs_dev,
+                int nseg, const int* block_seg_dev, const long long* block_start_dev, int nblocks, float* sq_partial,
+                cudaStream_t st) {
+  (void)n;
+  (void)nseg;
+  sgd_kernel<<<nblocks, SGD_THREADS, 0, st>>>(w, v, g, lr, mu, wd, segs_dev, block_seg_dev, block_start_dev,
+                                               sq_partial);
+  CK(cudaGetLastError());
+}
+
+__global__ void shadow_pack_kernel(const float* __restrict__ w, const SgdSeg* __restrict__ segs) {
+  const SgdSeg sg = segs[blockIdx.y];
+  if (!sg.shadow) return;
+  for (long long l = blockIdx.x * (long long)blockDim.x + threadIdx.x; l < sg.count; l += (long long)gridDim.x * blockDim.x) {
+    const float x = w[sg.off + l];
+    shadow_store(sg, l, &x, 1);
+  }
+}
+void launch_shadow_pack(const float* w, const SgdSeg* segs_dev, int nseg, cudaStream_t st) {
+  shadow_pack_kernel<<<dim3(64, nseg), 256, 0, st>>>(w, segs_dev);
+  CK(cudaGetLastError());
+}
+
+}  // namespace adainf

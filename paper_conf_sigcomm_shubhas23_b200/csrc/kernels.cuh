@@ -1,0 +1,77 @@
+// Declarations of the CUDA-core kernels' host launchers (HBM / latency-bound steps of the hot path).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "runtime.h"
+
+namespace adainf {
+
+// pad channels Cin -> Cpad (zeros), optional row map / device count (a1 ingest)
+void launch_pack_input(const bf16* x, const int* map, const int* count, int n_static, int H, int W, int Cin, int Cpad,
+                       bf16* y, cudaStream_t st);
+
+// maxpool fwd (NHWC bf16); optional input map; optional argmax offsets (uint8) for backward
+void launch_maxpool_fwd(const bf16* x, const int* map, const int* count, int n_static, int H, int W, int C, int K,
+                        int s, int p, int Ho, int Wo, bf16* y, uint8_t* argmax, cudaStream_t st);
+// maxpool bwd fused with the producer's activation mask: dz = bf16(sum_windows dT * [first argmax]) * act'(y)
+void launch_maxpool_bwd(const bf16* dT, const uint8_t* argmax, const bf16* yact, int act, int n, int H, int W, int C,
+                        int K, int s, int p, int Ho, int Wo, bf16* dz, cudaStream_t st);
+
+// ---- exit head (K4) ----
+struct ExitHeadArgs {
+  const bf16* fmap;     // dense [rows][HW][C]
+  const int* count;     // device rows count (nullptr -> n_static)
+  int n_static;
+  int HW, C, ncls;
+  const float* Wk;      // [C][ncls]
+  const float* bk;
+  float tau;            // exit iff conf >= tau (ignored if is_final)
+  int is_final;
+  const int* orig;      // dense row -> original row (nullptr = identity)
+  // outputs scattered to original rows (written only when the row exits here)
+  int8_t* exit_id;
+  int exit_index;
+  int32_t* pred;
+  float* conf;
+  float* entropy;
+  float* logits;        // [R][ncls]
+  float* embed;         // exit-0 pooled features [R][C], all rows
+  uint8_t* alive;       // [rows] 1 = survives past this exit
+  // training mode: all rows, saved pooled / logits
+  float* pooled_save;   // [rows][C]
+  float* logits_save;   // [rows][ncls]
+};
+void launch_exit_head(const ExitHeadArgs& a, cudaStream_t st);
+
+// stable compaction of alive rows: pos_next[j'] = j, orig_next[j'] = orig[j]; count_next; counts[k] += exited;
+// surv_out (optional, user): ascending original rows
+void launch_compact(const uint8_t* alive, const int* count, int n_static, const int* orig, int* pos_next,
+                    int* orig_next, int* count_next, int32_t* counts_out, int exit_index, int32_t* surv_out,
+                    int32_t* last_count_out, int last_index, cudaStream_t st);
+
+// ---- retraining (K8, K9, K10) ----
+// per exit: dl = w (softmax - onehot) / n_global ; loss_rows[n] += w CE
+void launch_exit_loss(const float* logits, const int32_t* labels, int n, int ncls, float w, float inv_n, float* dl,
+                      float* loss_rows, int accumulate, cudaStream_t st);
+// head grads: dW[c][j] = sum_n pooled[n][c] dl[n][j]; db[j] = sum_n dl[n][j]; bcast[n][c] = (sum_j dl W[c][j]) / HW
+void launch_head_grads(const float* pooled, const float* dl, const float* Wk, int n, int C, int ncls, int HW,
+                       float* dW, float* db, float* bcast, cudaStream_t st);
+// dz = bf16((bcast[n][c] + sc) * act'(y))
+void launch_grad_finalize(const float* bcast, const bf16* sc, const bf16* yact, int act, int n, int HW, int C,
+                          bf16* dz, cudaStream_t st);
+// fixed-order sum of a float vector into out[0] (single block)
+void launch_sum(const float* x, int n, float* out, float scale, cudaStream_t st);
+
+struct SgdSeg {
+  long long off;       // flat offset
+  long long count;
+  bf16* shadow;        // conv weight shadow [Cout][ldb] or nullptr
+  int taps, cin, cin_pad, ldb;
+};
+void launch_sgd(float* w, float* v, const float* g, long long n, float lr, float mu, float wd, const SgdSeg* segs_dev,
+                int nseg, const int* block_seg_dev, const long long* block_start_dev, int nblocks, float* sq_partial,
+                cudaStream_t st);
+void launch_shadow_pack(const float* w, const SgdSeg* segs_dev, int nseg, cudaStream_t st);
+
+}  // namespace adainf

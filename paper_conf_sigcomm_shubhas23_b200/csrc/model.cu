@@ -1,0 +1,538 @@
+// Model runtime: IR resolution, parameter storage, inference and retraining orchestration.
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <random>
+
+#include "api_common.h"
+#include "model.h"
+
+namespace adainf {
+
+void DevBuf::alloc(size_t b) {
+  if (p) cudaFree(p);
+  p = nullptr;
+  bytes = b;
+  if (b) {
+    cudaError_t e = cudaMalloc(&p, b);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      p = nullptr;
+      throw CudaError(std::string("cudaMalloc(") + std::to_string(b) + "): " + cudaGetErrorString(e));
+    }
+  }
+}
+void DevBuf::zero(cudaStream_t st) {
+  if (p) CK(cudaMemsetAsync(p, 0, bytes, st));
+}
+DevBuf::~DevBuf() {
+  if (p) cudaFree(p);
+}
+
+static int pad8(int c) { return (c + 7) / 8 * 8; }
+
+// ------------------------------------------------------------------------------------------------
+void Model::build(const adainf_model_spec& s) {
+  if (s.n_ops <= 0 || !s.ops) throw InvalidError("model: empty op list");
+  if (s.in_h <= 0 || s.in_w <= 0 || s.in_c <= 0 || s.max_batch <= 0) throw ShapeError("model: bad input shape");
+  in_h = s.in_h;
+  in_w = s.in_w;
+  in_c = s.in_c;
+  max_batch = s.max_batch;
+  cin_pad = pad8(in_c);
+  pack = cin_pad != in_c;
+  momentum = s.momentum;
+  weight_decay = s.weight_decay;
+  ops.assign(s.ops, s.ops + s.n_ops);
+  device = s.device;
+
+  TensorRt t0;
+  t0.H = in_h;
+  t0.W = in_w;
+  t0.C = cin_pad;
+  T.push_back(t0);
+  int cur = 0, stage = 0;
+  std::vector<int> blocks;
+  op_node.assign(ops.size(), -1);
+  int n_exit_ops = 0;
+  for (auto& o : ops)
+    if (o.kind == ADAINF_OP_EXIT) n_exit_ops++;
+  int seen_exits = 0;
+  long long off = 0;
+  for (size_t i = 0; i < ops.size(); ++i) {
+    const adainf_op& o = ops[i];
+    if (o.kind == ADAINF_OP_CONV || o.kind == ADAINF_OP_BLOCK) {
+      const bool proj = o.kind == ADAINF_OP_BLOCK;
+      if (proj && o.cout <= 0) {
+        blocks.push_back(cur);
+        continue;
+      }
+      NodeRt nd;
+      nd.kind = proj ? N_PROJ : N_CONV;
+      nd.op = (int)i;
+      nd.in = cur;
+      nd.stage = stage;
+      const TensorRt& X = T[cur];
+      if (X.f32) throw InvalidError("conv on an fp32 tensor");
+      const int KH = proj ? 1 : o.kh, KW = proj ? 1 : o.kw, st = o.stride, pd = proj ? 0 : o.pad;
+      if (KH <= 0 || KW <= 0 || st <= 0 || pd < 0 || o.cout <= 0) throw ShapeError("conv: bad geometry");
+      if (KH * KW > 49) throw ShapeError("conv: at most 49 taps");
+      if (o.cout % 8 && !(i + 1 < ops.size() && ops[i + 1].kind == ADAINF_OP_DET_HEAD))
+        throw ShapeError("conv: cout must be a multiple of 8");
+      nd.g.Cin = X.C;
+      nd.g.Cout = o.cout;
+      nd.g.KH = KH;
+      nd.g.KW = KW;
+      nd.g.stride = st;
+      nd.g.pad = pd;
+      nd.g.H = X.H;
+      nd.g.W = X.W;
+      nd.g.Ho = (X.H + 2 * pd - KH) / st + 1;
+      nd.g.Wo = (X.W + 2 * pd - KW) / st + 1;
+      if (nd.g.Ho <= 0 || nd.g.Wo <= 0) throw ShapeError("conv: empty output");
+      nd.cin_real = (cur == 0) ? in_c : X.C;
+      nd.act = proj ? 0 : o.act;
+      nd.w_off = off;
+      off += (long long)o.cout * KH * KW * nd.cin_real;
+      nd.b_off = off;
+      off += o.cout;
+      nd.ldb = KH * KW * X.C;
+      nd.fp32_out = !proj && (i + 1 < ops.size() && ops[i + 1].kind == ADAINF_OP_DET_HEAD);
+      TensorRt Y;
+      Y.H = nd.g.Ho;
+      Y.W = nd.g.Wo;
+      Y.C = o.cout;
+      Y.producer = (int)nodes.size();
+      Y.act = nd.act;
+      Y.stage = stage;
+      Y.f32 = nd.fp32_out;
+      T.push_back(Y);
+      nd.out = (int)T.size() - 1;
+      if (!proj && o.residual) {
+        if (blocks.empty()) throw InvalidError("residual conv without an open block");
+        nd.res = blocks.back();
+        blocks.pop_back();
+        const TensorRt& R = T[nd.res];
+        if (R.H != Y.H || R.W != Y.W || R.C != Y.C) throw ShapeError("residual shape mismatch");
+        if (R.stage != stage) throw InvalidError("a residual block may not span an exit");
+      }
+      const int ni = (int)nodes.size();
+      if (proj) {
+        if (T[cur].proj >= 0) throw InvalidError("tensor used by two projections");
+        T[cur].proj = ni;
+        blocks.push_back(nd.out);
+      } else {
+        if (T[cur].primary >= 0) throw InvalidError("tensor consumed twice on the main path");
+        T[cur].primary = ni;
+        if (nd.res >= 0 && T[nd.res].producer >= 0 && nodes[T[nd.res].producer].kind == N_PROJ) {
+          // shortcut tensor produced by a projection: its gradient is this conv's dZ (handled by the walk)
+        } else if (nd.res >= 0) {
+          T[nd.res].res_of = ni;
+        }
+        cur = nd.out;
+      }
+      op_node[i] = ni;
+      nodes.push_back(std::move(nd));
+    } else if (o.kind == ADAINF_OP_MAXPOOL) {
+      NodeRt nd;
+      nd.kind = N_POOL;
+      nd.op = (int)i;
+      nd.in = cur;
+      nd.stage = stage;
+      const TensorRt& X = T[cur];
+      nd.pk = o.kh;
+      nd.ps = o.stride;
+      nd.pp = o.pad;
+      if (o.kh <= 0 || o.kh != o.kw || o.kh * o.kw > 255 || o.stride <= 0) throw ShapeError("maxpool: bad window");
+      nd.g.H = X.H;
+      nd.g.W = X.W;
+      nd.g.Cin = nd.g.Cout = X.C;
+      nd.g.Ho = (X.H + 2 * o.pad - o.kh) / o.stride + 1;
+      nd.g.Wo = (X.W + 2 * o.pad - o.kw) / o.stride + 1;
+      TensorRt Y;
+      Y.H = nd.g.Ho;
+      Y.W = nd.g.Wo;
+      Y.C = X.C;
+      Y.producer = (int)nodes.size();
+      Y.act = 0;
+      Y.stage = stage;
+      T.push_back(Y);
+      nd.out = (int)T.size() - 1;
+      if (T[cur].primary >= 0) throw InvalidError("tensor consumed twice on the main path");
+      T[cur].primary = (int)nodes.size();
+      cur = nd.out;
+      op_node[i] = (int)nodes.size();
+      nodes.push_back(std::move(nd));
+    } else if (o.kind == ADAINF_OP_EXIT) {
+      if (!blocks.empty()) throw InvalidError("an exit may not sit inside an open residual block");
+      if (o.num_classes <= 0 || o.num_classes > 64) throw ShapeError("exit: num_classes in 1..64");
+      ExitRt e;
+      e.op = (int)i;
+      e.tensor = cur;
+      e.ncls = o.num_classes;
+      e.stage = stage;
+      e.lw = o.loss_weight;
+      const int C = T[cur].C;
+      if (C % 8 || (256 % (C / 8)) || C / 8 > 256) throw ShapeError("exit: channels must be 8 * power of two");
+      e.w_off = off;
+      off += (long long)C * o.num_classes;
+      e.b_off = off;
+      off += o.num_classes;
+      if (!exits.empty() && exits[0].ncls != e.ncls) throw ShapeError("all exits of a model share num_classes");
+      if (T[cur].exit_k >= 0) throw InvalidError("two exits on one tensor");
+      T[cur].exit_k = (int)exits.size();
+      exits.push_back(std::move(e));
+      seen_exits++;
+      if (seen_exits < n_exit_ops) stage++;
+    } else if (o.kind == ADAINF_OP_DET_HEAD) {
+      if (!T[cur].f32) throw InvalidError("DET_HEAD must follow a conv");
+      det.tensor = cur;
+      det.anchors = o.anchors;
+      det.classes = o.det_classes;
+      det.stride = o.grid_stride;
+      if (o.anchors <= 0 || o.anchors > 8 || o.det_classes <= 0 || T[cur].C != o.anchors * (5 + o.det_classes))
+        throw ShapeError("det_head: channels must be anchors*(5+classes)");
+      memcpy(det.anchor_wh, o.anchor_wh, sizeof(det.anchor_wh));
+    } else {
+      throw InvalidError("unknown op kind");
+    }
+  }
+  if (!blocks.empty()) throw InvalidError("unclosed residual block");
+  if (exits.empty() && det.tensor < 0) throw InvalidError("model needs at least one EXIT or a DET_HEAD");
+  if (!exits.empty() && exits.back().op != (int)ops.size() - 1) throw InvalidError("the final EXIT must be the last op");
+  for (auto& nd : nodes)
+    if (nd.kind == N_POOL && (T[nd.in].exit_k >= 0 || T[nd.in].res_of >= 0 || T[nd.in].proj >= 0))
+      throw InvalidError("a pooled tensor may not feed an exit or a shortcut");
+  for (size_t i = 0; i < nodes.size(); ++i) {
+    const NodeRt& nd = nodes[i];
+    if (T[nd.in].stage + 1 < nd.stage) throw InvalidError("tensor read across two exits");
+  }
+  nstages = stage + 1;
+  nparams = off;
+
+  CK(cudaSetDevice(device));
+  // activations
+  for (size_t t = 1; t < T.size(); ++t) {
+    const size_t b = (size_t)max_batch * T[t].row_elems() * (T[t].f32 ? 4 : 2);
+    T[t].own.alloc(b);
+    T[t].buf = T[t].own.as<bf16>();
+  }
+  if (pack) {
+    packed_in.alloc((size_t)max_batch * in_h * in_w * cin_pad * 2);
+    T[0].buf = packed_in.as<bf16>();
+  }
+  for (auto& nd : nodes)
+    if (nd.kind != N_POOL) {
+      nd.shadow.alloc((size_t)nd.g.Cout * nd.ldb * 2);
+      nd.shadow.zero();
+    }
+  params.alloc(nparams * 4);
+  mom.alloc(nparams * 4);
+  grads.alloc(nparams * 4);
+  mom.zero();
+  grads.zero();
+  pos.alloc((size_t)nstages * max_batch * 4);
+  orig.alloc((size_t)nstages * max_batch * 4);
+  counts.alloc((size_t)nstages * 4 + 16);
+  alive.alloc((size_t)max_batch);
+
+  // SGD segment tables (shadow layout per conv weight)
+  std::vector<SgdSeg> segs;
+  auto add_seg = [&](long long o, long long c, bf16* sh, int taps, int cin, int cin_p, int ldb) {
+    SgdSeg s{};
+    s.off = o;
+    s.count = c;
+    s.shadow = sh;
+    s.taps = taps;
+    s.cin = cin;
+    s.cin_pad = cin_p;
+    s.ldb = ldb;
+    segs.push_back(s);
+  };
+  // segments in flat order
+  std::vector<std::pair<long long, int>> order;  // (offset, kind/index)
+  for (size_t i = 0; i < nodes.size(); ++i)
+    if (nodes[i].kind != N_POOL) order.push_back({nodes[i].w_off, (int)i});
+  for (size_t k = 0; k < exits.size(); ++k) order.push_back({exits[k].w_off, -1 - (int)k});
+  std::sort(order.begin(), order.end());
+  for (auto& pr : order) {
+    if (pr.second >= 0) {
+      NodeRt& nd = nodes[pr.second];
+      add_seg(nd.w_off, (long long)nd.g.Cout * nd.g.KH * nd.g.KW * nd.cin_real, nd.shadow.as<bf16>(),
+              nd.g.KH * nd.g.KW, nd.cin_real, nd.g.Cin, nd.ldb);
+      add_seg(nd.b_off, nd.g.Cout, nullptr, 0, 0, 0, 0);
+    } else {
+      ExitRt& e = exits[-1 - pr.second];
+      add_seg(e.w_off, e.b_off + e.ncls - e.w_off, nullptr, 0, 0, 0, 0);
+    }
+  }
+  std::vector<int> bseg;
+  std::vector<long long> bstart;
+  const long long PER = 256 * 4 * 4;
+  for (size_t si = 0; si < segs.size(); ++si)
+    for (long long st = segs[si].off; st < segs[si].off + segs[si].count; st += PER) {
+      bseg.push_back((int)si);
+      bstart.push_back(st);
+    }
+  sgd_nseg = (int)segs.size();
+  sgd_nblocks = (int)bseg.size();
+  sgd_segs.alloc(segs.size() * sizeof(SgdSeg));
+  sgd_block_seg.alloc(bseg.size() * 4);
+  sgd_block_start.alloc(bstart.size() * 8);
+  CK(cudaMemcpy(sgd_segs.p, segs.data(), segs.size() * sizeof(SgdSeg), cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(sgd_block_seg.p, bseg.data(), bseg.size() * 4, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(sgd_block_start.p, bstart.data(), bstart.size() * 8, cudaMemcpyHostToDevice));
+  sq_partial.alloc((size_t)sgd_nblocks * 4 + 64);
+
+  // parameters: caller's, or He-normal from seed (exit heads x4)
+  std::vector<float> host(nparams);
+  if (s.init_params) {
+    memcpy(host.data(), s.init_params, nparams * 4);
+  } else {
+    std::mt19937_64 rng(s.seed);
+    std::normal_distribution<float> nd01(0.f, 1.f);
+    for (auto& nd : nodes) {
+      if (nd.kind == N_POOL) continue;
+      const float sd = std::sqrt(2.0f / (float)(nd.g.KH * nd.g.KW * nd.cin_real));
+      for (long long j = nd.w_off; j < nd.b_off; ++j) host[j] = nd01(rng) * sd;
+      for (int j = 0; j < nd.g.Cout; ++j) host[nd.b_off + j] = 0.01f * nd01(rng);
+    }
+    for (auto& e : exits) {
+      const int C = T[e.tensor].C;
+      const float sd = 4.0f / std::sqrt((float)C);
+      for (long long j = e.w_off; j < e.b_off; ++j) host[j] = nd01(rng) * sd;
+      for (int j = 0; j < e.ncls; ++j) host[e.b_off + j] = 0.1f * nd01(rng);
+    }
+  }
+  CK(cudaMemcpy(params.p, host.data(), nparams * 4, cudaMemcpyHostToDevice));
+  refresh_shadows(0);
+  CK(cudaDeviceSynchronize());
+}
+
+void Model::refresh_shadows(cudaStream_t st) {
+  launch_shadow_pack(params.as<float>(), sgd_segs.as<SgdSeg>(), sgd_nseg, st);
+}
+
+void Model::ensure_training() {
+  if (train_ready) return;
+  if (exits.empty()) throw UnsupportedError("retraining needs an early-exit classifier (detector is not retrained, P:86)");
+  for (size_t t = 1; t < T.size(); ++t) {
+    if (T[t].f32) continue;
+    T[t].own_grad.alloc((size_t)max_batch * T[t].row_elems() * 2);
+    T[t].grad = T[t].own_grad.as<bf16>();
+  }
+  size_t ws = 0;
+  for (auto& nd : nodes) {
+    if (nd.kind == N_POOL) {
+      nd.argmax.alloc((size_t)max_batch * T[nd.out].row_elems());
+    } else {
+      ws = std::max(ws, ::adainf::wgrad_ws_bytes(nd.g, max_batch));
+      if (nd.kind == N_PROJ && nd.in != 0) nd.proj_dx.alloc((size_t)max_batch * T[nd.in].row_elems() * 2);
+    }
+  }
+  wgrad_ws.alloc(ws);
+  wgrad_ws_bytes = ws;
+  for (auto& e : exits) {
+    const int C = T[e.tensor].C;
+    e.pooled.alloc((size_t)max_batch * C * 4);
+    e.logits.alloc((size_t)max_batch * e.ncls * 4);
+    e.dl.alloc((size_t)max_batch * e.ncls * 4);
+    e.bcast.alloc((size_t)max_batch * C * 4);
+  }
+  loss_rows.alloc((size_t)max_batch * 4);
+  stats_tmp.alloc(64);
+  train_ready = true;
+}
+
+// ------------------------------------------------------------------------------------------------
+// Forward over all ops.  Inference: stage s>0 reads tensors of stage s-1 through pos[s] (dense survivor
+// positions) and works on count[s] rows (device-side), outputs are scattered through orig[s].
+// Training: all rows, no exits taken, heads evaluated for every row (SURVEY c.1 step 9).
+void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, int n_static, bool train,
+                          const float* taus, const adainf_model_out* out, cudaStream_t st) {
+  int* posb = pos.as<int>();
+  int* origb = orig.as<int>();
+  int* cnt = counts.as<int>();
+  auto stage_count = [&](int s) -> const int* { return s == 0 ? count0 : cnt + s; };
+  auto stage_orig = [&](int s) -> const int* { return s == 0 ? nullptr : origb + (size_t)s * max_batch; };
+  auto buf_of = [&](int t) -> const bf16* { return t == 0 ? x0 : T[t].buf; };
+  // map used by a node of stage `ns` reading tensor t
+  auto map_for = [&](int t, int ns) -> const int* {
+    if (train) return nullptr;
+    if (t == 0) return ns == 0 ? map0 : nullptr;
+    if (T[t].stage < ns) return posb + (size_t)ns * max_batch;
+    return nullptr;
+  };
+  const int E = (int)exits.size();
+  for (size_t i = 0; i < ops.size(); ++i) {
+    const int ni = op_node[i];
+    if (ni >= 0) {
+      NodeRt& nd = nodes[ni];
+      const int ns = train ? 0 : nd.stage;
+      const int* c = train ? nullptr : stage_count(ns);
+      if (nd.kind == N_POOL) {
+        launch_maxpool_fwd(buf_of(nd.in), map_for(nd.in, ns), c, n_static, nd.g.H, nd.g.W, nd.g.Cin, nd.pk, nd.ps,
+                           nd.pp, nd.g.Ho, nd.g.Wo, T[nd.out].buf, train ? nd.argmax.as<uint8_t>() : nullptr, st);
+      } else {
+        const float* bias = params.as<float>() + nd.b_off;
+        const bf16* res = nd.res >= 0 ? T[nd.res].buf : nullptr;
+        const int* rmap = nd.res >= 0 ? map_for(nd.res, ns) : nullptr;
+        conv_fwd(nd.g, buf_of(nd.in), map_for(nd.in, ns), c, n_static, nd.shadow.as<bf16>(), nd.ldb, bias, res, rmap,
+                 nd.act, T[nd.out].buf, nd.fp32_out, st);
+      }
+      continue;
+    }
+    if (ops[i].kind != ADAINF_OP_EXIT) continue;
+    int k = -1;
+    for (int q = 0; q < E; ++q)
+      if (exits[q].op == (int)i) k = q;
+    ExitRt& e = exits[k];
+    const TensorRt& X = T[e.tensor];
+    ExitHeadArgs a{};
+    a.fmap = buf_of(e.tensor);
+    a.HW = X.H * X.W;
+    a.C = X.C;
+    a.ncls = e.ncls;
+    a.Wk = params.as<float>() + e.w_off;
+    a.bk = params.as<float>() + e.b_off;
+    a.n_static = n_static;
+    if (train) {
+      a.is_final = 1;
+      a.pooled_save = e.pooled.as<float>();
+      a.logits_save = e.logits.as<float>();
+      launch_exit_head(a, st);
+      continue;
+    }
+    const int s = e.stage;
+    a.count = stage_count(s);
+    a.orig = stage_orig(s);
+    a.is_final = (k == E - 1);
+    a.tau = a.is_final ? 0.f : taus[k];
+    a.exit_index = k;
+    a.exit_id = out->exit_id;
+    a.pred = out->pred;
+    a.conf = out->conf;
+    a.entropy = out->entropy;
+    a.logits = out->logits;
+    a.embed = k == 0 ? out->embed : nullptr;
+    a.alive = a.is_final ? nullptr : alive.as<uint8_t>();
+    if (e.tensor == 0 && map0) throw InvalidError("exit directly on a mapped input is not supported");
+    launch_exit_head(a, st);
+    if (!a.is_final) {
+      // survivors of exit k -> stage s+1 (stable, ascending original rows)
+      launch_compact(alive.as<uint8_t>(), a.count, n_static, a.orig, posb + (size_t)(s + 1) * max_batch,
+                     origb + (size_t)(s + 1) * max_batch, cnt + s + 1, out->exit_counts, k,
+                     out->surv_idx ? out->surv_idx + (size_t)k * n_static : nullptr,
+                     (k == E - 2) ? out->exit_counts : nullptr, E - 1, st);
+    }
+  }
+}
+
+void Model::infer(const bf16* x, const int* in_map, const int* in_count, int n_static, const float* taus,
+                  const adainf_model_out& out, cudaStream_t st, bool x_padded) {
+  if (n_static <= 0) return;
+  if (n_static > max_batch) throw ShapeError("batch exceeds max_batch");
+  const bf16* x0 = x;
+  const int* map0 = in_map;
+  if (pack && !x_padded) {
+    launch_pack_input(x, in_map, in_count, n_static, in_h, in_w, in_c, cin_pad, packed_in.as<bf16>(), st);
+    x0 = packed_in.as<bf16>();
+    map0 = nullptr;
+  }
+  if (exits.size() == 1 && out.exit_counts) {
+    // single-exit model: every row leaves at exit 0 -> counts[0] = rows (device count or static)
+    if (in_count)
+      CK(cudaMemcpyAsync(out.exit_counts, in_count, 4, cudaMemcpyDeviceToDevice, st));
+    else
+      CK(cudaMemcpyAsync(out.exit_counts, &n_static, 4, cudaMemcpyHostToDevice, st));
+  }
+  forward_nodes(x0, map0, in_count, n_static, false, taus, &out, st);
+}
+
+// ------------------------------------------------------------------------------------------------
+void Model::train_step(const bf16* x, const int32_t* labels, int n, long long n_global, float lr,
+                       adainf_step_stats* stats, cudaStream_t st) {
+  if (n <= 0 || n > max_batch) throw ShapeError("retrain: n_local must be in 1..max_batch");
+  if (n_global < n) throw ShapeError("retrain: n_global < n_local");
+  ensure_training();
+  const bf16* x0 = x;
+  if (pack) {
+    launch_pack_input(x, nullptr, nullptr, n, in_h, in_w, in_c, cin_pad, packed_in.as<bf16>(), st);
+    x0 = packed_in.as<bf16>();
+  }
+  forward_nodes(x0, nullptr, nullptr, n, true, nullptr, nullptr, st);
+  float* G = grads.as<float>();
+  const float* P = params.as<float>();
+  const float inv_n = (float)(1.0 / (double)n_global);
+  // exit losses and head gradients (K8)
+  for (size_t k = 0; k < exits.size(); ++k) {
+    ExitRt& e = exits[k];
+    const TensorRt& X = T[e.tensor];
+    launch_exit_loss(e.logits.as<float>(), labels, n, e.ncls, e.lw, inv_n, e.dl.as<float>(), loss_rows.as<float>(),
+                     k > 0, st);
+    launch_head_grads(e.pooled.as<float>(), e.dl.as<float>(), P + e.w_off, n, X.C, e.ncls, X.H * X.W, G + e.w_off,
+                      G + e.b_off, e.bcast.as<float>(), st);
+  }
+  auto buf_of = [&](int t) -> const bf16* { return t == 0 ? x0 : T[t].buf; };
+  auto bcast_of = [&](int t) -> const float* { return T[t].exit_k >= 0 ? exits[T[t].exit_k].bcast.as<float>() : nullptr; };
+  auto sc_of = [&](int t) -> const bf16* {
+    if (T[t].res_of >= 0) return T[nodes[T[t].res_of].out].grad;  // identity shortcut: dZ of the residual conv
+    if (T[t].proj >= 0) return nodes[T[t].proj].proj_dx.as<bf16>();
+    return nullptr;
+  };
+  // tensors with no main-path consumer (the final exit's input): gradient = broadcast (+ shortcut)
+  for (size_t t = 1; t < T.size(); ++t)
+    if (T[t].primary < 0 && !T[t].f32 && T[t].producer >= 0 && nodes[T[t].producer].kind != N_PROJ)
+      launch_grad_finalize(bcast_of((int)t), sc_of((int)t), T[t].buf, T[t].act, n, T[t].H * T[t].W, T[t].C,
+                           T[t].grad, st);
+  // reverse walk (K2, K3, K9)
+  auto conv_backward = [&](NodeRt& nd, const bf16* dz) {
+    conv_wgrad(nd.g, buf_of(nd.in), dz, n, nd.cin_real, wgrad_ws.as<float>(), wgrad_ws_bytes, G + nd.w_off,
+               G + nd.b_off, st);
+    if (nd.in == 0) return;  // no input gradient for the first layer
+    const TensorRt& X = T[nd.in];
+    if (nd.kind == N_PROJ) {
+      conv_dgrad(nd.g, dz, nd.shadow.as<bf16>(), nd.ldb, n, nullptr, nullptr, nullptr, 0, nd.proj_dx.as<bf16>(), st);
+    } else {
+      const int prod = X.producer;
+      const int mask = (prod >= 0 && nodes[prod].kind == N_CONV) ? X.act : 0;
+      conv_dgrad(nd.g, dz, nd.shadow.as<bf16>(), nd.ldb, n, bcast_of(nd.in), sc_of(nd.in), mask ? X.buf : nullptr,
+                 mask, T[nd.in].grad, st);
+    }
+  };
+  for (int ni = (int)nodes.size() - 1; ni >= 0; --ni) {
+    NodeRt& nd = nodes[ni];
+    if (nd.kind == N_PROJ) continue;  // handled right after its residual conv
+    if (nd.kind == N_POOL) {
+      const TensorRt& X = T[nd.in];
+      if (nd.in == 0) continue;
+      launch_maxpool_bwd(T[nd.out].grad, nd.argmax.as<uint8_t>(), X.buf, X.act, n, X.H, X.W, X.C, nd.pk, nd.ps, nd.pp,
+                         nd.g.Ho, nd.g.Wo, T[nd.in].grad, st);
+      continue;
+    }
+    const bf16* dz = T[nd.out].grad;
+    if (nd.res >= 0 && T[nd.res].producer >= 0 && nodes[T[nd.res].producer].kind == N_PROJ) {
+      // projection shortcut: its output gradient is this conv's dZ; do it before the block's first conv
+      conv_backward(nd, dz);
+      conv_backward(nodes[T[nd.res].producer], dz);
+    } else {
+      conv_backward(nd, dz);
+    }
+  }
+#ifdef ADAINF_WITH_NCCL
+  if (comm && dp_world > 1) {
+    ncclResult_t r = ncclAllReduce(G, G, (size_t)nparams, ncclFloat, ncclSum, comm, st);
+    if (r != ncclSuccess) throw std::runtime_error(std::string("NCCL: ") + ncclGetErrorString(r));
+  }
+#endif
+  // fused SGD + momentum + shadow refresh (K10)
+  launch_sgd(params.as<float>(), mom.as<float>(), G, nparams, lr, momentum, weight_decay, sgd_segs.as<SgdSeg>(),
+             sgd_nseg, sgd_block_seg.as<int>(), sgd_block_start.as<long long>(), sgd_nblocks, sq_partial.as<float>(),
+             st);
+  if (stats) {
+    launch_sum(loss_rows.as<float>(), n, &stats->loss, 0.f, st);
+    launch_sum(sq_partial.as<float>(), sgd_nblocks, &stats->grad_norm, -1.f, st);
+  }
+}
+
+}  // namespace adainf

@@ -1,0 +1,160 @@
+// Model / app runtime of libadainf.so: the model IR resolved into tensors + GEMM/pool nodes + exit heads,
+// device-resident parameters (fp32 master, momentum, bf16 GEMM-ready shadows) and workspaces sized for
+// max_batch at create time, and the stream-ordered orchestration of inference (stage by stage with
+// device-side survivor counts) and of the retraining step (forward, losses, reverse walk, update).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "../../include/adainf.h"
+#include "kernels.cuh"
+#include "runtime.h"
+
+#ifdef ADAINF_WITH_NCCL
+#include <nccl.h>
+#endif
+
+namespace adainf {
+
+enum NodeKind { N_CONV = 0, N_POOL = 1, N_PROJ = 2 };
+
+struct DevBuf {  // owning device allocation
+  void* p = nullptr;
+  size_t bytes = 0;
+  void alloc(size_t b);
+  void zero(cudaStream_t st = 0);
+  ~DevBuf();
+  template <class T>
+  T* as() const { return (T*)p; }
+};
+
+struct TensorRt {
+  int H, W, C;
+  int producer = -1;  // node index, -1 = model input
+  int act = 0;        // activation of the producing conv (mask for gradients)
+  int stage = 0;
+  bool f32 = false;
+  bf16* buf = nullptr;   // activations (max_batch rows)
+  DevBuf own;
+  // training
+  bf16* grad = nullptr;  // stored gradient (dZ of a conv output / dT of a pool output)
+  DevBuf own_grad;
+  int primary = -1;      // node reading it as main input (conv or pool)
+  int proj = -1;         // projection node reading it
+  int res_of = -1;       // conv node adding it as identity shortcut
+  int exit_k = -1;       // exit attached
+  size_t row_elems() const { return (size_t)H * W * C; }
+};
+
+struct NodeRt {
+  int kind;
+  int op;
+  int in, out, res = -1;
+  int stage;
+  ConvGeom g{};
+  int act = 0;
+  int cin_real = 0;
+  long long w_off = 0, b_off = 0;
+  int ldb = 0;
+  DevBuf shadow;  // bf16 [Cout][ldb]
+  bool fp32_out = false;
+  int pk = 0, ps = 0, pp = 0;  // pool
+  DevBuf argmax;               // pool (training)
+  DevBuf proj_dx;              // proj (training): dgrad into the block input, added as shortcut term
+};
+
+struct ExitRt {
+  int op, tensor, ncls, stage;
+  float lw;
+  long long w_off, b_off;
+  DevBuf pooled, logits, dl, bcast;  // training
+};
+
+struct DetRt {
+  int tensor = -1;
+  int anchors = 0, classes = 0, stride = 0;
+  float anchor_wh[16];
+};
+
+struct Model {
+  int device = 0;
+  int in_h, in_w, in_c, cin_pad, max_batch;
+  bool pack = false;
+  std::vector<adainf_op> ops;
+  std::vector<TensorRt> T;
+  std::vector<NodeRt> nodes;
+  std::vector<int> op_node;  // op index -> node index (or -1)
+  std::vector<ExitRt> exits;
+  DetRt det;
+  int nstages = 1;
+  long long nparams = 0;
+  float momentum = 0.9f, weight_decay = 0.f;
+
+  DevBuf params, mom, grads;
+  DevBuf packed_in;           // [max_batch][H][W][cin_pad]
+  // inference stage bookkeeping
+  DevBuf pos, orig, counts, alive;  // pos/orig: [nstages][max_batch] int; counts [nstages] int
+  // training
+  bool train_ready = false;
+  DevBuf wgrad_ws, loss_rows, stats_tmp, sq_partial;
+  size_t wgrad_ws_bytes = 0;
+  DevBuf sgd_segs, sgd_block_seg, sgd_block_start;
+  int sgd_nblocks = 0, sgd_nseg = 0;
+  int n_out_det_edges = 0;
+#ifdef ADAINF_WITH_NCCL
+  ncclComm_t comm = nullptr;
+#endif
+  int dp_world = 1, dp_rank = 0;
+
+  void build(const adainf_model_spec& s);
+  void refresh_shadows(cudaStream_t st);
+  void ensure_training();
+  // inference of one (possibly routed / device-counted) batch
+  void infer(const bf16* x, const int* in_map, const int* in_count, int n_static, const float* taus,
+             const adainf_model_out& out, cudaStream_t st, bool x_padded = false);
+  void train_step(const bf16* x, const int32_t* labels, int n, long long n_global, float lr,
+                  adainf_step_stats* stats, cudaStream_t st);
+
+ private:
+  void forward_nodes(const bf16* x0, const int* map0, const int* count0, int n_static, bool train, const float* taus,
+                     const adainf_model_out* out, cudaStream_t st);
+};
+
+struct App {
+  std::vector<Model*> models;
+  std::vector<adainf_edge> edges;
+  int max_routed = 0;
+};
+
+// detector decode / routing / crop (detect.cu)
+struct DetRouteArgs {
+  const float* raw;  // [B][G][G][A*(5+NC)]
+  const int* count;  // frames count (device) or nullptr
+  int n_static, G, A, NC, stride, img_w, img_h;
+  float anchor_wh[16];
+  float tau;
+  int n_edges;
+  int edge_class[8];
+  int cap;
+  float* det_table;      // internal, capacity = all candidates
+  float* user_table;     // caller's copy (first user_max rows) or nullptr
+  int user_max;
+  int32_t* n_det;
+  int32_t* route_idx;    // [n_edges][cap]
+  int32_t* n_routed;     // [n_edges] required
+  int32_t* count_clamped;  // [n_edges]
+  int32_t* cap_flag;
+};
+size_t det_route_ws_bytes(int n_static, int G, int A);
+void launch_det_route(const DetRouteArgs& a, void* ws, cudaStream_t st);
+void launch_crops(const bf16* frames, int H, int W, int C, const float* det_table, const int32_t* route_idx,
+                  const int32_t* count_clamped, int edge, int cap, int crop_h, int crop_w, int cout_pad, bf16* dst,
+                  cudaStream_t st);
+// CLASS_WHOLE routing: stable compaction of rows with pred == cls
+void launch_route_class(const int32_t* pred, const int* count, int n_static, int cls, int32_t* list,
+                        int32_t* count_out, int cap, int32_t* cap_flag, cudaStream_t st);
+
+}  // namespace adainf

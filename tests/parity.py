@@ -1,0 +1,95 @@
+"""Shared parity helpers for the GPU tests: run the CUDA path through the C-ABI binding and the oracle
+on the same seeded inputs, and compare under the north_star tolerances (bands per SURVEY §8(c.2))."""
+from __future__ import annotations
+
+import numpy as np
+
+import oracle as O
+from paper_conf_sigcomm_shubhas23_b200 import binding as B
+from paper_conf_sigcomm_shubhas23_b200 import synth
+
+BAND = 1e-3
+
+
+def rel(a, b):
+    a = np.asarray(a, np.float64)
+    b = np.asarray(b, np.float64)
+    return float(np.linalg.norm(a - b) / max(np.linalg.norm(b), 1e-30))
+
+
+def images(spec, B_, seed, num_classes=10, period=0):
+    xb, y = synth.drifted_images(B_, spec["in_h"], spec["in_w"], spec["in_c"], num_classes=num_classes, seed=seed,
+                                 period=period)
+    return xb, y, synth.bf16_bits_to_f32(xb)
+
+
+def to_cuda_bf16(xb):
+    import torch
+    return torch.from_numpy(xb.view(np.int16)).cuda().view(torch.bfloat16)
+
+
+def gpu_infer_single(spec, params, xb, taus, max_batch=None):
+    """Single-model app on the GPU: returns dict of numpy outputs."""
+    import torch
+    n = xb.shape[0]
+    m = B.Model(spec, max_batch or n, params=params)
+    app = B.App([m])
+    outs = B.alloc_outs(m, n)
+    x = to_cuda_bf16(xb)
+    app.infer(x, list(taus), [outs])
+    torch.cuda.synchronize()
+    res = {k: v.cpu().numpy() for k, v in outs.items()}
+    app.close()
+    m.close()
+    return res
+
+
+def banded_rows(conf_all, taus, exit_oracle):
+    """rows whose confidence at any exit k <= e_oracle (k < E-1) lies within BAND of tau_k"""
+    Bn, E = conf_all.shape
+    band = np.zeros(Bn, bool)
+    for k in range(E - 1):
+        band |= (np.abs(conf_all[:, k] - taus[k]) < BAND) & (exit_oracle >= k)
+    return band
+
+
+def check_infer_parity(orc, gpu, taus):
+    """exit ids, survivor lists, counts bit-exact outside the band; logits rel 2e-2; conf within 1e-3."""
+    conf_all = orc["conf"]
+    E = conf_all.shape[1]
+    eid, surv, counts = O.exit_assign(conf_all, taus)
+    band = banded_rows(conf_all, taus, eid)
+    ok = ~band
+    assert (gpu["exit_id"][ok] == eid[ok]).all(), np.nonzero((gpu["exit_id"] != eid) & ok)
+    if not band.any():
+        np.testing.assert_array_equal(gpu["exit_counts"], counts)
+    assert gpu["exit_counts"].sum() == conf_all.shape[0]
+    bad = set(np.nonzero(band)[0].tolist())
+    for k in range(E - 1):
+        n_alive = conf_all.shape[0] - int(gpu["exit_counts"][:k + 1].sum())
+        g = gpu["surv_idx"][k][:n_alive]
+        assert np.all(np.diff(g) > 0), "survivor list not ascending"
+        o = surv[k][surv[k] >= 0]
+        np.testing.assert_array_equal([i for i in g if i not in bad], [i for i in o if i not in bad])
+    rows = np.nonzero(ok)[0]
+    ex = eid[rows]
+    ref_logits = orc["logits"][rows, ex, :]
+    for i, r in enumerate(rows):
+        assert rel(gpu["logits"][r], ref_logits[i]) <= 2e-2, (r, gpu["logits"][r], ref_logits[i])
+    np.testing.assert_allclose(gpu["conf"][rows], conf_all[rows, ex], atol=1e-3)
+    # argmax equal where the top-2 oracle logits are separated
+    srt = np.sort(ref_logits, axis=1)
+    sep = (srt[:, -1] - srt[:, -2]) > 1e-2 * np.maximum(1, np.abs(srt[:, -1]))
+    assert (gpu["pred"][rows][sep] == orc["pred"][rows, ex][sep]).all()
+    return int(band.sum())
+
+
+def check_grads(spec, g_gpu, g_orc, tol=2e-2):
+    from paper_conf_sigcomm_shubhas23_b200 import specs as S
+    worst = 0.0
+    for kind, i, off, shp in S.param_segments(spec):
+        n = int(np.prod(shp))
+        r = rel(g_gpu[off:off + n], g_orc[off:off + n])
+        worst = max(worst, r)
+        assert r <= tol, (kind, i, r)
+    return worst

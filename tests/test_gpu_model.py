@@ -1,0 +1,109 @@
+"""Model-level GPU parity through the C-ABI: early-exit inference (exit ids, compaction order, counts,
+logits), the incremental-retraining SGD step (gradients, updated weights) — CUDA path vs the oracle on
+the same seeded inputs (BASELINE configs 1 and 2, plus reduced-resolution ResNet-18-EE cases that
+span many tiles with ragged tails)."""
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+from paper_conf_sigcomm_shubhas23_b200 import binding as B
+from paper_conf_sigcomm_shubhas23_b200 import specs as S
+from paper_conf_sigcomm_shubhas23_b200 import synth
+
+from parity import check_grads, check_infer_parity, gpu_infer_single, images, rel, to_cuda_bf16
+
+pytestmark = pytest.mark.gpu
+
+
+def _infer_case(spec, Bn, seed, fractions):
+    p = synth.init_params(spec, seed=seed)
+    xb, y, xf = images(spec, Bn, seed)
+    om = O.Model(spec)
+    orc = om.forward(p, xf)
+    taus = synth.calibrate_thresholds(orc["conf"], fractions)
+    gpu = gpu_infer_single(spec, p, xb, taus)
+    nb = check_infer_parity(orc, gpu, taus)
+    # exit-0 pooled features (selection embeddings, Q12)
+    assert rel(gpu["embed"], orc["pooled0"]) <= 2e-2
+    return orc, gpu, taus, nb
+
+
+def test_tiny_cnn_inference_c1():
+    """BASELINE config 1: tiny 3-conv EE CNN, batch 64, tau -> 50% exit."""
+    orc, gpu, taus, nb = _infer_case(S.tiny_cnn_ee(), 64, 1, [0.5])
+    assert nb <= 3
+    assert 20 <= gpu["exit_counts"][0] <= 44
+
+
+@pytest.mark.parametrize("Bn,hw,seed", [(37, 64, 2), (24, 96, 3)])
+def test_resnet18_ee_inference_reduced(Bn, hw, seed):
+    """ResNet-18-EE (4 exits) at reduced resolution: 25/25/25/25 exits, ragged batch."""
+    orc, gpu, taus, nb = _infer_case(S.resnet18_ee(in_hw=hw), Bn, seed, [0.25, 0.25, 0.25])
+    assert nb <= 3
+
+
+def test_resnet18_ee_inference_full_res():
+    """ResNet-18-EE at 224x224 (config 2 geometry), a few samples."""
+    _infer_case(S.resnet18_ee(), 5, 4, [0.2, 0.2, 0.2])
+
+
+def test_threshold_special_cases():
+    """tau <= 0 -> everything exits at exit 0; tau > 1 -> full structure (all at the final exit)."""
+    spec = S.resnet18_ee(in_hw=64)
+    p = synth.init_params(spec, seed=5)
+    xb, _, xf = images(spec, 19, 5)
+    g0 = gpu_infer_single(spec, p, xb, [0.0, 0.0, 0.0])
+    assert (g0["exit_id"] == 0).all() and g0["exit_counts"].tolist() == [19, 0, 0, 0]
+    g1 = gpu_infer_single(spec, p, xb, [1.5, 1.5, 1.5])
+    assert (g1["exit_id"] == 3).all() and g1["exit_counts"].tolist() == [0, 0, 0, 19]
+    orc = O.Model(spec).forward(p, xf)
+    for r in range(19):
+        assert rel(g1["logits"][r], orc["logits"][r, 3]) <= 2e-2
+
+
+def _retrain_case(spec, n, seed, lr, n_global=None):
+    p = synth.init_params(spec, seed=seed)
+    xb, y, xf = images(spec, n, seed, num_classes=spec["ops"][-1]["num_classes"])
+    om = O.Model(spec)
+    p1, v1, g_o, loss_o = om.retrain_step(p, np.zeros_like(p), xf, y, n_global=n_global, lr=lr, mu=0.9)
+    m = B.Model(spec, n, params=p, momentum=0.9)
+    x = to_cuda_bf16(xb)
+    lab = torch.from_numpy(y).cuda()
+    stats = torch.zeros(2, dtype=torch.float32, device="cuda")
+    m.retrain_step(x, lab, n_global=n_global, lr=lr, stats=stats)
+    torch.cuda.synchronize()
+    g_g = m.get_grads()
+    p_g = m.get_params()
+    worst = check_grads(spec, g_g, g_o)
+    assert rel(p_g, p1) <= 1e-3
+    assert rel(p_g - p, p1 - p) <= 2e-2
+    st = stats.cpu().numpy()
+    assert abs(st[0] - loss_o) <= 1e-3 * abs(loss_o)
+    assert abs(st[1] - np.linalg.norm(g_o)) <= 2e-2 * np.linalg.norm(g_o)
+    m.close()
+    return worst
+
+
+def test_tiny_cnn_retrain_step_c1():
+    """BASELINE config 1: one incremental-retraining SGD step on 128 selected samples (lr 0.05)."""
+    _retrain_case(S.tiny_cnn_ee(), 128, 11, 0.05)
+
+
+def test_resnet18_ee_retrain_step_reduced():
+    """ResNet-18-EE backward (dgrad phases, wgrad split-K, projections, maxpool) at 64x64, 12 samples,
+    gradients scaled by 1/n_global with n_global > n_local (a DP shard, reading Q22)."""
+    _retrain_case(S.resnet18_ee(in_hw=64), 12, 12, 0.01, n_global=48)
+
+
+def test_retrain_deterministic():
+    spec = S.tiny_cnn_ee()
+    p = synth.init_params(spec, seed=3)
+    xb, y, _ = images(spec, 64, 3)
+    outs = []
+    for _ in range(2):
+        m = B.Model(spec, 64, params=p)
+        m.retrain_step(to_cuda_bf16(xb), torch.from_numpy(y).cuda(), lr=0.05)
+        outs.append(m.get_params())
+        m.close()
+    assert np.array_equal(outs[0], outs[1])

@@ -1,0 +1,56 @@
+"""GPU parity of retraining-sample selection (P:195/P:239/P:243) vs the oracle: distances, the exact
+top-k index set (ties -> lower index, ascending output), exclusion, k >= #eligible, M > 1 references."""
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+from paper_conf_sigcomm_shubhas23_b200 import binding as B
+from paper_conf_sigcomm_shubhas23_b200 import synth
+
+from parity import BAND
+
+pytestmark = pytest.mark.gpu
+
+
+def _run(N, D, P, M, k, seed, excl_frac=0.1, use_w=True):
+    Xb, Wb, ref = synth.embeddings(N, D, P, seed=seed, M=M)
+    rng = np.random.default_rng(seed)
+    ex = (rng.random(N) < excl_frac).astype(np.uint8)
+    X = torch.from_numpy(Xb.view(np.int16)).cuda().view(torch.bfloat16)
+    W = torch.from_numpy(Wb.view(np.int16)).cuda().view(torch.bfloat16).reshape(D, P) if use_w else None
+    R = torch.from_numpy(ref).cuda()
+    E = torch.from_numpy(ex).cuda()
+    dist = torch.empty(N, dtype=torch.float32, device="cuda")
+    idx, dd, cnt = B.select_retrain(X.reshape(N, D), W, R, k, exclude=E, dist_all=dist)
+    torch.cuda.synchronize()
+    cnt = int(cnt.item())
+    idx, dd, dist = idx.cpu().numpy()[:cnt], dd.cpu().numpy()[:cnt], dist.cpu().numpy()
+    oi, od, oc, odist = O.select(synth.bf16_bits_to_f32(Xb).reshape(N, D),
+                                 synth.bf16_bits_to_f32(Wb).reshape(D, P) if use_w else None, ref, k, exclude=ex)
+    assert cnt == oc
+    el = ex == 0
+    np.testing.assert_allclose(dist[el], odist[el], atol=2e-4, rtol=2e-3)
+    assert (dist[~el] == -1).all()
+    assert np.all(np.diff(idx) > 0)
+    assert not ex[idx].any()
+    # bit-exact index set outside the band around the oracle's k-th distance
+    if oc == k and oc < el.sum():
+        dk = np.sort(odist[el])[::-1][k - 1]
+        banded = np.abs(odist - dk) < BAND
+        sg = set(i for i in idx.tolist() if not banded[i])
+        so = set(i for i in oi.tolist() if not banded[i])
+        assert sg == so
+    else:
+        assert set(idx.tolist()) == set(oi.tolist())
+    np.testing.assert_allclose(dd, dist[idx], rtol=0, atol=0)
+
+
+@pytest.mark.parametrize("N,D,P,M,k", [(4099, 64, 16, 1, 512), (16384, 64, 16, 1, 1024), (3000, 512, 64, 4, 257),
+                                       (1000, 64, 16, 1, 5000)])
+def test_select_vs_oracle(N, D, P, M, k):
+    _run(N, D, P, M, k, seed=N + k)
+
+
+def test_select_identity_projection():
+    _run(2048, 64, 64, 1, 100, seed=9, use_w=False)
