@@ -95,7 +95,7 @@ typedef struct {
   int32_t n_ops;
   const adainf_op* ops;       /* host, copied at create */
   float momentum, weight_decay; /* SGD (PyTorch semantics, reading Q9) */
-  uint64_t seed;              /* He-normal init when init_params == NULL */
+  uint64_t seed;              /* LeCun-normal init when init_params == NULL */
   const float* init_params;   /* host, num_params fp32, or NULL */
   int32_t device;             /* CUDA device ordinal */
 } adainf_model_spec;

@@ -293,7 +293,7 @@ void Model::build(const adainf_model_spec& s) {
     std::normal_distribution<float> nd01(0.f, 1.f);
     for (auto& nd : nodes) {
       if (nd.kind == N_POOL) continue;
-      const float sd = std::sqrt(2.0f / (float)(nd.g.KH * nd.g.KW * nd.cin_real));
+      const float sd = std::sqrt(1.0f / (float)(nd.g.KH * nd.g.KW * nd.cin_real));
       for (long long j = nd.w_off; j < nd.b_off; ++j) host[j] = nd01(rng) * sd;
       for (int j = 0; j < nd.g.Cout; ++j) host[nd.b_off + j] = 0.01f * nd01(rng);
     }
@@ -301,6 +301,12 @@ void Model::build(const adainf_model_spec& s) {
       const int C = T[e.tensor].C;
       const float sd = 4.0f / std::sqrt((float)C);
       for (long long j = e.w_off; j < e.b_off; ++j) host[j] = nd01(rng) * sd;
+      for (int cls = 0; cls < e.ncls; ++cls) {  // zero-mean over channels (see synth.init_params)
+        double mean = 0;
+        for (int c = 0; c < C; ++c) mean += host[e.w_off + (long long)c * e.ncls + cls];
+        mean /= C;
+        for (int c = 0; c < C; ++c) host[e.w_off + (long long)c * e.ncls + cls] -= (float)mean;
+      }
       for (int j = 0; j < e.ncls; ++j) host[e.b_off + j] = 0.1f * nd01(rng);
     }
   }

@@ -8,7 +8,8 @@ they share.  Recipe (DESIGN.md §Input recipe):
   U(-0.3, 0.3), contrast c_p ~ U(0.7, 1.3), occlusion rectangle with prob 0.1 (lighting / occlusion
   drift); label priors pi_p ~ Dirichlet(5) mild / Dirichlet(0.3) heavy (label drift).
 * spectrograms: 128 mel x 128 frames log-energy, class harmonic stripes + 1/f noise (reading Q24).
-* weights: He-normal conv weights, small biases, exit heads x4 to spread confidences.
+* weights: LeCun-normal conv weights, small biases, exit heads x4 and zero-mean over channels to
+  spread confidences.
 * embeddings for selection: old features ~ N(mu_old, I), new features drifted; PCA basis from the old
   features (fitted off the hot path).
 
@@ -127,7 +128,8 @@ def spectrograms(B: int, num_classes: int = 8, F: int = 128, T: int = 128, perio
 
 
 def init_params(spec: dict, seed: int = 0, exit_scale: float = 4.0) -> np.ndarray:
-    """He-normal conv weights, small biases, exit heads scaled x`exit_scale` (fp32 flat vector)."""
+    """LeCun-normal conv weights (sd = 1/sqrt(fan_in): keeps activations O(1) through the BN-free
+    residual stages, reading Q10), small biases, exit heads scaled x`exit_scale` (fp32 flat vector)."""
     rng = np.random.default_rng(seed)
     n = S.num_params(spec)
     p = np.zeros(n, np.float32)
@@ -135,12 +137,15 @@ def init_params(spec: dict, seed: int = 0, exit_scale: float = 4.0) -> np.ndarra
         cnt = int(np.prod(shp))
         if kind in ("conv_w", "proj_w"):
             fan_in = shp[1] * shp[2] * shp[3]
-            p[off:off + cnt] = rng.standard_normal(cnt, dtype=np.float32) * np.float32(np.sqrt(2.0 / fan_in))
+            p[off:off + cnt] = rng.standard_normal(cnt, dtype=np.float32) * np.float32(np.sqrt(1.0 / fan_in))
         elif kind in ("conv_b", "proj_b"):
             p[off:off + cnt] = rng.standard_normal(cnt, dtype=np.float32) * np.float32(0.01)
         elif kind == "exit_w":
-            p[off:off + cnt] = rng.standard_normal(cnt, dtype=np.float32) * np.float32(
-                exit_scale / np.sqrt(shp[0]))
+            w = rng.standard_normal(shp, dtype=np.float32) * np.float32(exit_scale / np.sqrt(shp[0]))
+            # zero-mean over channels per class: cancels the common mode of post-ReLU pooled features
+            # (otherwise every sample gets the same class offsets and the confidences bunch up)
+            w -= w.mean(axis=0, keepdims=True)
+            p[off:off + cnt] = w.reshape(-1)
         elif kind == "exit_b":
             p[off:off + cnt] = rng.standard_normal(cnt, dtype=np.float32) * np.float32(0.1)
     return p
