@@ -1,0 +1,428 @@
+#!/usr/bin/env python
+"""AdaInf hot-path benchmark on B200 (BASELINE.json metric, config 2).
+
+One STEP = one pass of the whole hot path on one batch of synthetic drifted
+input, all through libadainf.so's C-ABI (include/adainf.h):
+  a1-a4  adainf_infer_dag     ResNet-18-EE (4 exits, 10 vehicle classes) on 256 224x224 crops, taus
+                              calibrated once to ~25/25/25/25 exit fractions
+  a7     adainf_select_retrain  16,384-sample window pool (D=64 embeddings -> PCA P=16, cosine distance
+                              to the old mean, 10% already used/excluded) -> k = 1,024
+         adainf_gather_rows   selected samples -> retraining batch (device-resident pool)
+  a8-a11 adainf_retrain_step  one SGD+momentum step on the 1,024 selected samples (lr 0.01, mu 0.9)
+                              (N>1: data-parallel, NCCL all-reduce of the fp32 gradient)
+
+value = (inference samples + retraining samples) of all ranks / max-over-ranks device time per step.
+e2e   = the same step through the same API with the step's inputs copied H2D from pinned host memory
+        (request batch, candidate embeddings, pool labels) and its results read back D2H.
+--impl reference runs the oracle (oracle/, plain C++ fp64) on the box's host cores on a bounded sample
+of the same workload (the reference arm for this tier).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_sigcomm_shubhas23_b200 import specs as S  # noqa: E402
+from paper_conf_sigcomm_shubhas23_b200 import synth  # noqa: E402
+
+METRIC = "DAG inference samples/s + retrain samples/s per B200 (1/2/4/8), % of bf16 peak"
+UNIT = "samples/s"
+INF_B, POOL_N, D_EMB, P_EMB, K_SEL = 256, 16384, 64, 16, 1024
+LR, MU = 0.01, 0.9
+EXIT_FRACTIONS = [0.25, 0.25, 0.25]
+BASE_IMAGES = 2048  # distinct synthetic images; the 16,384-sample pool repeats them (DESIGN.md §Input recipe)
+
+
+def arm_config(world):
+    return {"workload": "BASELINE config 2: ResNet-18-EE (4 exits) vehicle-type classifier, 224x224 crops, "
+                        "inference batch 256 + selection from a 16,384-sample window pool + one retrain step on "
+                        "k=1,024 selected samples",
+            "model": "resnet18_ee", "global_batch": (INF_B + K_SEL) * world, "seq_len": None,
+            "parallelism": f"dp{world}" if world > 1 else "single", "inference_batch": INF_B,
+            "retrain_batch": K_SEL, "pool": POOL_N, "l2": "inputs + activations larger than L2 (no flush)"}
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["bf16_tflops"]), float(p.get("bf16_tflops_sustained", p["bf16_tflops"])), float(
+            p["hbm_gbs"]), "measured"
+    except Exception:
+        return 1590.0, 1400.0, 6650.0, "fallback"
+
+
+def flops_model():
+    """Algorithmic FLOPs: per-stage forward MACs of ResNet-18-EE, retraining = 3x fwd - stem dgrad."""
+    spec = S.resnet18_ee()
+    macs = S.macs_per_sample(spec)
+    stage_macs = [0, 0, 0, 0]
+    st = 0
+    for o, m in zip(spec["ops"], macs):
+        stage_macs[st] += m
+        if o["kind"] == "exit" and st < 3:
+            st += 1
+    conv_macs = sum(m for o, m in zip(spec["ops"], macs) if o["kind"] in ("conv", "block"))
+    stem_macs = macs[0]
+    retrain_flops = 2 * (3 * sum(macs) - stem_macs)
+    retrain_conv_flops = 2 * (3 * conv_macs - stem_macs)
+    return spec, stage_macs, retrain_flops, retrain_conv_flops
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region (B200_PROFILING.md)."""
+
+    def __init__(self, idx):
+        self.idx, self.rows, self.proc = idx, [], None
+
+    def start(self):
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"], stdout=subprocess.PIPE,
+                                         stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) >= 7:
+                self.rows.append(parts)
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[3 + i].lower() in ("active", "1")})
+        loaded = [s for s in sm if s > 0.5 * (max(mx) if mx else 1)] or sm
+        return {"sm_mhz": statistics.median(loaded) if loaded else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(sm)}
+
+
+def dist_setup():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+# ------------------------------------------------------------------------------------------------
+def run_reference(args, world, rank):
+    """Reference arm for this tier: the oracle (plain C++ fp64) on the host cores, bounded sample."""
+    if rank != 0:
+        return 0
+    import oracle as O
+    spec = S.resnet18_ee()
+    om = O.Model(spec)
+    p = synth.init_params(spec, seed=2)
+    n_inf, n_rt = 1, 4  # same 1:4 mix as the GPU step (256 : 1024)
+    xb, y = synth.drifted_images(n_inf + n_rt, 224, 224, 3, seed=2)
+    xf = synth.bf16_bits_to_f32(xb)
+    Xb, Wb, ref = synth.embeddings(2048, D_EMB, P_EMB, seed=3)
+    X = synth.bf16_bits_to_f32(Xb).reshape(2048, D_EMB)
+    W = synth.bf16_bits_to_f32(Wb).reshape(D_EMB, P_EMB)
+
+    def step():
+        r = om.forward(p, xf[:n_inf])
+        O.exit_assign(r["conf"], [0.5, 0.5, 0.5])
+        O.select(X, W, ref, K_SEL // 8)
+        om.retrain_step(p, np.zeros_like(p), xf[n_inf:], y[n_inf:], lr=LR, mu=MU)
+
+    for _ in range(args.warmup):
+        step()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        step()
+    dt = (time.perf_counter() - t0) / args.steps
+    v = (n_inf + n_rt) / dt
+    cores = O.get_threads()
+    sample = (f"per step: {n_inf} inference sample (full depth + exit rule) + selection over 2,048 "
+              f"candidates (k=128) + one retrain step on {n_rt} samples, ResNet-18-EE 224x224")
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": arm_config(world),
+        "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+        "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+    return 0
+
+
+def cpu_baseline_leg():
+    """The oracle as it stands on the box's host cores, bounded sample (~10-30 s)."""
+    import oracle as O
+    spec = S.resnet18_ee()
+    om = O.Model(spec)
+    p = synth.init_params(spec, seed=2)
+    n_inf, n_rt = 4, 16
+    xb, y = synth.drifted_images(n_inf + n_rt, 224, 224, 3, seed=5)
+    xf = synth.bf16_bits_to_f32(xb)
+    Xb, Wb, ref = synth.embeddings(POOL_N, D_EMB, P_EMB, seed=3)
+    t0 = time.perf_counter()
+    r = om.forward(p, xf[:n_inf])
+    O.exit_assign(r["conf"], [0.5, 0.5, 0.5])
+    O.select(synth.bf16_bits_to_f32(Xb).reshape(POOL_N, D_EMB), synth.bf16_bits_to_f32(Wb).reshape(D_EMB, P_EMB),
+             ref, K_SEL)
+    om.retrain_step(p, np.zeros_like(p), xf[n_inf:], y[n_inf:], lr=LR, mu=MU)
+    dt = time.perf_counter() - t0
+    return {"value": (n_inf + n_rt) / dt, "unit": UNIT, "cores": O.get_threads(), "kind": "oracle",
+            "sample": f"{n_inf} inference samples + selection over the {POOL_N}-sample pool (k={K_SEL}) + one "
+                      f"retrain step on {n_rt} samples (ResNet-18-EE 224x224), {dt:.1f} s"}
+
+
+# ------------------------------------------------------------------------------------------------
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="adainf", choices=["adainf", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--profile-steps", type=int, default=None)
+    args = ap.parse_args()
+    world, rank, local = dist_setup()
+    if args.impl == "reference":
+        return run_reference(args, world, rank)
+    args.warmup = max(args.warmup, 3)
+
+    import torch
+    from paper_conf_sigcomm_shubhas23_b200 import binding as B
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    def barrier():
+        if world > 1:
+            torch.distributed.barrier()
+
+    bf16_burst, bf16_sust, hbm_gbs, peak_src = peaks()
+    spec, stage_macs, retrain_flops, retrain_conv_flops = flops_model()
+
+    # ---- synthetic inputs (seeded per rank) ----
+    seed = 100 + rank
+    params = synth.init_params(spec, seed=1)  # identical replicas
+    protos = synth.class_prototypes(10, 224, 224, 3, seed=1244)
+    inf_b, _ = synth.drifted_images(INF_B, 224, 224, 3, seed=seed, period=1, protos=protos)
+    base_b, base_y = synth.drifted_images(BASE_IMAGES, 224, 224, 3, seed=seed, period=0, protos=protos)
+    Xb, Wb, ref = synth.embeddings(POOL_N, D_EMB, P_EMB, seed=seed)
+    excl = (np.random.default_rng(seed).random(POOL_N) < 0.1).astype(np.uint8)
+
+    dev = torch.device("cuda", local)
+
+    def bf(a):
+        return torch.from_numpy(a.view(np.int16)).to(dev).view(torch.bfloat16)
+
+    x_inf = bf(inf_b)
+    base = bf(base_b)
+    reps = (POOL_N + BASE_IMAGES - 1) // BASE_IMAGES
+    pool = base.repeat(reps, 1, 1, 1)[:POOL_N].contiguous()
+    pool_y = torch.from_numpy(np.ascontiguousarray(np.tile(base_y, reps)[:POOL_N])).to(dev)
+    del base
+    X = bf(Xb).reshape(POOL_N, D_EMB)
+    W = bf(Wb).reshape(D_EMB, P_EMB)
+    R = torch.from_numpy(ref).to(dev)
+    E = torch.from_numpy(excl).to(dev)
+
+    m = B.Model(spec, max(INF_B, K_SEL), params=params, momentum=MU)
+    if world > 1:
+        import torch.distributed as dist
+        uid = B.nccl_unique_id() if rank == 0 else b"\0" * 128
+        obj = [uid]
+        dist.broadcast_object_list(obj, src=0)
+        m.dp_attach(obj[0], rank, world)
+    app = B.App([m])
+    outs = B.alloc_outs(m, INF_B)
+    sel_idx = torch.empty(K_SEL, dtype=torch.int32, device=dev)
+    sel_dist = torch.empty(K_SEL, dtype=torch.float32, device=dev)
+    sel_cnt = torch.empty(1, dtype=torch.int32, device=dev)
+    rt_x = torch.empty((K_SEL, 224, 224, 3), dtype=torch.bfloat16, device=dev)
+    rt_y = torch.empty(K_SEL, dtype=torch.int32, device=dev)
+    stats = torch.zeros(2, dtype=torch.float32, device=dev)
+    stream = torch.cuda.current_stream()
+    n_global = K_SEL * world
+
+    # thresholds: calibrated once on the first (untimed) batch from full-depth confidences (all exits
+    # disabled), placed in the widest gap near the 25/25/25 quantiles
+    calib = B.alloc_outs(m, INF_B)
+    conf_all = np.zeros((INF_B, 4), np.float32)
+    for k in range(4):
+        taus = [2.0] * 3
+        if k < 3:
+            taus[k] = 0.0
+            taus[:k] = [2.0] * k
+        app.infer(x_inf, taus, [calib])
+        torch.cuda.synchronize()
+        conf_all[:, k] = calib["conf"].cpu().numpy()
+    taus = [float(t) for t in synth.calibrate_thresholds(conf_all, EXIT_FRACTIONS)]
+    def step_device(out_counts):
+        outs["exit_counts"] = out_counts
+        app.infer(x_inf, taus, [outs])
+        B.select_retrain(X, W, R, K_SEL, exclude=E, out_idx=sel_idx, out_dist=sel_dist, out_count=sel_cnt)
+        B.gather_rows(pool, sel_idx, sel_cnt, K_SEL, rt_x)
+        B.gather_rows(pool_y, sel_idx, sel_cnt, K_SEL, rt_y)
+        m.retrain_step(rt_x, rt_y, n_global=n_global, lr=LR, stats=stats)
+
+    cnt_buf = torch.zeros((max(args.steps, 1) + args.warmup + 64, 4), dtype=torch.int32, device=dev)
+    for i in range(args.warmup):
+        step_device(cnt_buf[-1 - i % 32])
+    torch.cuda.synchronize()
+    barrier()
+
+    # ---- timed region (device time, CUDA events on the launching stream) ----
+    clk = ClockSampler(local)
+    clk.start()
+    time.sleep(0.3)
+    l0 = B.launch_count()
+    barrier()
+    torch.cuda.synchronize()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record(stream)
+    for i in range(args.steps):
+        step_device(cnt_buf[i])
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    launches = B.launch_count() - l0
+    barrier()
+    clocks = clk.stop()
+    ms = ev0.elapsed_time(ev1) / args.steps
+    if world > 1:
+        t = torch.tensor([ms], device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms = float(t.item())
+    counts = cnt_buf[:args.steps].cpu().numpy()
+    samples_per_step = (INF_B + K_SEL) * world
+    value = samples_per_step / (ms / 1e3)
+
+    # algorithmic FLOPs of one step (survivors only): per-stage MACs x samples reaching the stage
+    reach = np.array([INF_B - counts[:, :k].sum(1) for k in range(4)]).T.mean(0)
+    inf_flops = 2 * float(np.dot(reach, stage_macs))
+    sel_flops = 2.0 * POOL_N * D_EMB * P_EMB
+    step_flops = inf_flops + K_SEL * retrain_flops + sel_flops
+    pct_peak = step_flops / (ms / 1e3) / (bf16_sust * 1e12) * 100
+
+    # ---- profiled pass: per-kernel-class device time (events on the launching stream) ----
+    pk = args.profile_steps or args.steps
+    B.prof_reset()
+    B.prof_enable(True)
+    torch.cuda.synchronize()
+    ev2, ev3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev2.record(stream)
+    for i in range(pk):
+        step_device(cnt_buf[-1 - i % 32])
+    ev3.record(stream)
+    torch.cuda.synchronize()
+    prof = B.prof_query()
+    B.prof_enable(False)
+    prof_ms = ev2.elapsed_time(ev3) / pk
+    conv_ms = sum(prof[k][1] for k in ("conv_fwd", "conv_dgrad", "conv_wgrad")) / pk
+    conv_launches = sum(prof[k][0] for k in ("conv_fwd", "conv_dgrad", "conv_wgrad")) / pk
+    conv_flops = inf_flops + K_SEL * retrain_conv_flops + sel_flops  # algorithmic MACs on the tensor cores
+    achieved = conv_flops / (conv_ms / 1e3) / 1e12
+    traffic = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            traffic = json.load(f).get("conv_umma_kernel_bytes_per_launch")
+    except Exception:
+        pass
+    breakdown = {k: round(v[1] / pk, 4) for k, v in sorted(prof.items(), key=lambda kv: -kv[1][1]) if v[0]}
+
+    # ---- e2e: same step, inputs H2D from pinned host memory, results D2H, through the same API ----
+    e2e = None
+    if not args.no_e2e:
+        h_inf = torch.from_numpy(inf_b.view(np.int16)).view(torch.bfloat16).pin_memory()
+        h_X = torch.from_numpy(Xb.view(np.int16)).view(torch.bfloat16).reshape(POOL_N, D_EMB).pin_memory()
+        h_y = pool_y.cpu().pin_memory()
+        h_exit = torch.empty(INF_B, dtype=torch.int8).pin_memory()
+        h_pred = torch.empty(INF_B, dtype=torch.int32).pin_memory()
+        h_stats = torch.empty(2, dtype=torch.float32).pin_memory()
+        h2d = h_inf.numel() * 2 + h_X.numel() * 2 + h_y.numel() * 4
+        d2h = INF_B * 1 + INF_B * 4 + 8
+        torch.cuda.synchronize()
+        barrier()
+        ev4, ev5 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev4.record(stream)
+        for i in range(args.steps):
+            x_inf.view(torch.int16).copy_(h_inf.view(torch.int16), non_blocking=True)
+            X.view(torch.int16).copy_(h_X.view(torch.int16), non_blocking=True)
+            pool_y.copy_(h_y, non_blocking=True)
+            step_device(cnt_buf[-1 - i % 32])
+            h_exit.copy_(outs["exit_id"], non_blocking=True)
+            h_pred.copy_(outs["pred"], non_blocking=True)
+            h_stats.copy_(stats, non_blocking=True)
+        ev5.record(stream)
+        torch.cuda.synchronize()
+        ems = ev4.elapsed_time(ev5) / args.steps
+        if world > 1:
+            t = torch.tensor([ems], device=dev)
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            ems = float(t.item())
+        e2e = {"value": samples_per_step / (ems / 1e3), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+               "d2h_bytes_per_step": int(d2h), "ms_per_step": ems}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        try:
+            cpu = cpu_baseline_leg()
+        except Exception as ex:  # pragma: no cover
+            cpu = {"value": None, "unit": UNIT, "cores": None, "kind": "oracle", "sample": f"failed: {ex}"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
+            "config": dict(arm_config(world), exit_thresholds=taus),
+            "inference_samples_per_s": INF_B * world / (ms / 1e3),
+            "retrain_samples_per_s": K_SEL * world / (ms / 1e3),
+            "exit_counts_mean": counts.mean(0).round(2).tolist(),
+            "algorithmic_tflop_per_step": step_flops / 1e12,
+            "pct_bf16_peak": pct_peak,
+            "pct_bf16_peak_note": f"algorithmic FLOP/s of the whole step / {bf16_sust} TFLOP/s sustained ({peak_src})",
+            "roofline": {"bound": "tensor", "kernel": "conv_umma_kernel (tcgen05 implicit GEMM: fwd+dgrad+wgrad)",
+                         "achieved": achieved, "peak": bf16_sust, "unit": "TFLOP/s", "frac": achieved / bf16_sust,
+                         "traffic": traffic, "peak_kind": f"bf16 sustained ({peak_src})",
+                         "launches_per_step": conv_launches, "kernel_ms_per_step": conv_ms,
+                         "share_of_step": conv_ms / prof_ms},
+            "kernel_ms_per_step": breakdown,
+            "gpu_launches": int(launches),
+            "clocks": clocks,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    app.close()
+    m.close()
+    if world > 1:
+        torch.distributed.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

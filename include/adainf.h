@@ -203,6 +203,12 @@ adainf_status adainf_retrain_step(adainf_model_t m, const void* samples_bf16_nhw
                                   int32_t n_local, int64_t n_global, float lr,
                                   adainf_step_stats* stats_dev, adainf_stream_t stream);
 
+/* Assemble the retraining batch from the device-resident window pool (samples collected in the
+ * previous period): dst[r] = src[idx[r]] for r < min(*count, n) (count device int or NULL -> n);
+ * rows of row_bytes bytes (multiple of 4; 16 for 128-bit copies).  Pairs with adainf_select_retrain's out_idx/out_count. */
+adainf_status adainf_gather_rows(const void* src, const int32_t* idx, const int32_t* count, int32_t n,
+                                 int64_t row_bytes, void* dst, adainf_stream_t stream);
+
 /* Data-parallel retraining: attach an NCCL communicator created from a 128-byte
  * ncclUniqueId (broadcast by the caller, e.g. over torch.distributed); retrain_step then sums the
  * replicas' gradients (each scaled by 1/n_global) with ncclAllReduce before the update, so all

@@ -31,6 +31,20 @@ adainf_status adainf_dbg_conv_wgrad(const void* x, const void* dz, int32_t n, in
                                     int32_t Co, int32_t KH, int32_t KW, int32_t stride, int32_t pad, float* dw,
                                     float* db, adainf_stream_t stream);
 
+/* Launch accounting and per-kernel-class timing (CUDA events on the launching stream).
+ * adainf_launch_count: total kernels launched by the library since load (host-side counter).
+ * adainf_prof_enable(1): bracket every launch class with events; adainf_prof_query (synchronizing)
+ * returns per-class launch counts and summed device milliseconds since the last reset. */
+typedef struct {
+  const char* name;
+  int64_t launches;
+  double total_ms;
+} adainf_prof_entry;
+int64_t adainf_launch_count(void);
+adainf_status adainf_prof_enable(int32_t on);
+adainf_status adainf_prof_reset(void);
+adainf_status adainf_prof_query(adainf_prof_entry* out, int32_t max_entries, int32_t* n_out);
+
 #ifdef __cplusplus
 }
 #endif

@@ -74,6 +74,7 @@ def lib():
         vp, i32, i64 = C.c_void_p, C.c_int32, C.c_int64
         L.adainf_last_error.restype = C.c_char_p
         L.adainf_version.restype = C.c_int32
+        L.adainf_launch_count.restype = C.c_int64
         for name, args in {
             "adainf_model_create": [C.POINTER(ModelSpec), C.POINTER(vp)],
             "adainf_model_destroy": [vp],
@@ -90,6 +91,10 @@ def lib():
             "adainf_retrain_step": [vp, vp, vp, i32, i64, C.c_float, vp, vp],
             "adainf_dp_attach": [vp, vp, i32, i32],
             "adainf_nccl_unique_id": [vp],
+            "adainf_gather_rows": [vp, vp, vp, i32, i64, vp, vp],
+            "adainf_prof_enable": [i32],
+            "adainf_prof_reset": [],
+            "adainf_prof_query": [vp, i32, C.POINTER(i32)],
             "adainf_dbg_conv_fwd": [vp, i32, i32, i32, i32, vp, vp, i32, i32, i32, i32, i32, i32, vp, vp, i32, vp],
             "adainf_dbg_conv_dgrad": [vp, i32, i32, i32, i32, vp, i32, i32, i32, i32, i32, vp, vp, vp, i32, vp,
                                       vp],
@@ -298,6 +303,36 @@ def select_retrain(X, W, ref, k, exclude=None, out_idx=None, out_dist=None, out_
     check(lib().adainf_select_retrain(C.byref(si), int(k), ptr(out_idx), ptr(out_dist), ptr(out_count),
                                       ptr(dist_all), stream_ptr(stream)))
     return out_idx, out_dist, out_count
+
+
+def gather_rows(src, idx, count, n, dst, stream=None):
+    """dst[r] = src[idx[r]] for r < min(count, n) (device count tensor or None)."""
+    row_bytes = src[0].numel() * src.element_size()
+    check(lib().adainf_gather_rows(ptr(src), ptr(idx), ptr(count), int(n), int(row_bytes), ptr(dst),
+                                   stream_ptr(stream)))
+
+
+class ProfEntry(C.Structure):
+    _fields_ = [("name", C.c_char_p), ("launches", C.c_int64), ("total_ms", C.c_double)]
+
+
+def launch_count() -> int:
+    return int(lib().adainf_launch_count())
+
+
+def prof_enable(on: bool):
+    check(lib().adainf_prof_enable(int(on)))
+
+
+def prof_reset():
+    check(lib().adainf_prof_reset())
+
+
+def prof_query():
+    arr = (ProfEntry * 64)()
+    n = C.c_int32()
+    check(lib().adainf_prof_query(arr, 64, C.byref(n)))
+    return {arr[i].name.decode(): (int(arr[i].launches), float(arr[i].total_ms)) for i in range(n.value)}
 
 
 # ---- kernel-level (include/adainf_debug.h) ----

@@ -340,6 +340,15 @@ extern "C" adainf_status adainf_retrain_step(adainf_model_t m, const void* sampl
   });
 }
 
+extern "C" adainf_status adainf_gather_rows(const void* src, const int32_t* idx, const int32_t* count, int32_t n,
+                                            int64_t row_bytes, void* dst, adainf_stream_t stream) {
+  return guard([&] {
+    if (!src || !idx || !dst || n < 0 || row_bytes <= 0) throw InvalidError("gather_rows: bad argument");
+    require_device();
+    launch_gather_rows(src, idx, count, n, row_bytes, dst, (cudaStream_t)stream);
+  });
+}
+
 extern "C" adainf_status adainf_nccl_unique_id(void* out128) {
   return guard([&] {
     if (!out128) throw InvalidError("null argument");

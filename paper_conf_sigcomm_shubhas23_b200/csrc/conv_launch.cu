@@ -5,6 +5,7 @@
 #include <stdexcept>
 
 #include "conv_gemm.cuh"
+#include "prof.h"
 #include "runtime.h"
 
 namespace adainf {
@@ -28,6 +29,7 @@ static void launch_t(const ConvArgs& a, dim3 grid, cudaStream_t st) {
     CK(cudaFuncSetAttribute(conv_umma_kernel<MODE, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
     attr = true;
   }
+  ProfScope ps(MODE == MODE_FWD ? PC_CONV_FWD : (MODE == MODE_DGRAD ? PC_CONV_DGRAD : PC_CONV_WGRAD), st);
   conv_umma_kernel<MODE, BN><<<grid, NUM_THREADS, Cfg::SMEM, st>>>(a);
   CK(cudaGetLastError());
 }
@@ -238,12 +240,16 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
   dim3 grid((Kconv + BM - 1) / BM, (g.Cout + BN - 1) / BN, S);
   launch_bn<MODE_WGRAD>(BN, a, grid, st);
   dim3 rg((Kconv + 31) / 32, (g.Cout + 31) / 32);
+  {
+  ProfScope ps(PC_WGRAD_REDUCE, st);
   wgrad_reduce_kernel<<<rg, dim3(32, 8), 0, st>>>(ws, S, Kconv, g.Cout, g.Cin, cin_real, dw);
   CK(cudaGetLastError());
+  }
   if (db) {
     float* part = ws + (size_t)S * Kconv * g.Cout;
     const int rpb = 256;
     const int nb = (int)((npix + rpb - 1) / rpb);
+    ProfScope ps(PC_BIAS_COLSUM, st, 2);
     colsum_partial_kernel<<<nb, 128, 0, st>>>(dz, npix, g.Cout, rpb, part);
     colsum_final_kernel<<<(g.Cout + 127) / 128, 128, 0, st>>>(part, nb, g.Cout, db);
     CK(cudaGetLastError());

@@ -9,6 +9,7 @@
 //              (half-pixel centres, clamped edges, every fp32 op rounded on its own, reading Q19)
 #include "common.cuh"
 #include "model.h"
+#include "prof.h"
 
 namespace adainf {
 
@@ -167,6 +168,7 @@ void launch_det_route(const DetRouteArgs& a, void* ws, cudaStream_t st) {
   const long long ncand = (long long)a.n_static * a.G * a.G * a.A;
   const int nb = (int)((ncand + DET_PER_BLOCK - 1) / DET_PER_BLOCK);
   int* blk = (int*)ws;
+  ProfScope ps(PC_DET_ROUTE, st, 3);
   det_count_kernel<<<nb, DET_THREADS, 0, st>>>(a, blk);
   det_scan_kernel<<<1, 32 * (1 + MAX_EDGES), 0, st>>>(a, nb, blk);
   det_emit_kernel<<<nb, DET_THREADS, 0, st>>>(a, blk);
@@ -221,6 +223,7 @@ void launch_crops(const bf16* frames, int H, int W, int C, const float* det_tabl
                   const int32_t* count_clamped, int edge, int cap, int crop_h, int crop_w, int cout_pad, bf16* dst,
                   cudaStream_t st) {
   dim3 grid((crop_h * crop_w + 255) / 256, cap);
+  ProfScope ps(PC_CROP, st);
   crop_kernel<<<grid, 256, 0, st>>>(frames, H, W, C, det_table, route_idx, count_clamped, edge, cap, crop_h, crop_w,
                                      cout_pad, dst);
   CK(cudaGetLastError());
@@ -267,6 +270,7 @@ __global__ void __launch_bounds__(1024) route_class_kernel(const int32_t* __rest
 }
 void launch_route_class(const int32_t* pred, const int* count, int n_static, int cls, int32_t* list,
                         int32_t* count_out, int cap, int32_t* cap_flag, cudaStream_t st) {
+  ProfScope ps(PC_ROUTE_CLASS, st);
   route_class_kernel<<<1, 1024, 0, st>>>(pred, count, n_static, cls, list, count_out, cap, cap_flag);
   CK(cudaGetLastError());
 }

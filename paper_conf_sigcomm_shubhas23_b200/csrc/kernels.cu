@@ -6,6 +6,7 @@
 
 #include "common.cuh"
 #include "kernels.cuh"
+#include "prof.h"
 
 namespace adainf {
 
@@ -26,6 +27,7 @@ void launch_pack_input(const bf16* x, const int* map, const int* count, int n_st
   const long long total = (long long)n_static * H * W;
   const int blocks = (int)std::min<long long>((total + 255) / 256, 16LL * num_sms());
   if (blocks <= 0) return;
+  ProfScope ps(PC_PACK, st);
   pack_input_kernel<<<blocks, 256, 0, st>>>(x, map, count, n_static, H * W, Cin, Cpad, y);
   CK(cudaGetLastError());
 }
@@ -83,6 +85,7 @@ void launch_maxpool_fwd(const bf16* x, const int* map, const int* count, int n_s
   const long long total = (long long)n_static * Ho * Wo * (C / 8);
   const int blocks = (int)std::min<long long>((total + 255) / 256, 32LL * num_sms());
   if (blocks <= 0) return;
+  ProfScope ps(PC_POOL_FWD, st);
   maxpool_fwd_kernel<<<blocks, 256, 0, st>>>(x, map, count, n_static, H, W, C, K, s, p, Ho, Wo, y, amax);
   CK(cudaGetLastError());
 }
@@ -120,6 +123,7 @@ void launch_maxpool_bwd(const bf16* dT, const uint8_t* amax, const bf16* yact, i
                         int K, int s, int p, int Ho, int Wo, bf16* dz, cudaStream_t st) {
   const long long total = (long long)n * H * W * C;
   const int blocks = (int)std::min<long long>((total + 255) / 256, 32LL * num_sms());
+  ProfScope ps(PC_POOL_BWD, st);
   maxpool_bwd_kernel<<<blocks, 256, 0, st>>>(dT, amax, yact, act, n, H, W, C, K, s, p, Ho, Wo, dz);
   CK(cudaGetLastError());
 }
@@ -208,6 +212,7 @@ void launch_exit_head(const ExitHeadArgs& a, cudaStream_t st) {
   const int groups = EH_THREADS / (a.C / 8);
   const size_t smem = (size_t)(groups * a.C + a.C + a.ncls) * sizeof(float);
   if (a.n_static <= 0) return;
+  ProfScope ps(PC_EXIT_HEAD, st);
   exit_head_kernel<<<a.n_static, EH_THREADS, smem, st>>>(a);
   CK(cudaGetLastError());
 }
@@ -266,6 +271,7 @@ __global__ void __launch_bounds__(1024) compact_kernel(const uint8_t* __restrict
 void launch_compact(const uint8_t* alive, const int* count, int n_static, const int* orig, int* pos_next,
                     int* orig_next, int* count_next, int32_t* counts_out, int exit_index, int32_t* surv_out,
                     int32_t* last_count_out, int last_index, cudaStream_t st) {
+  ProfScope ps(PC_COMPACT, st);
   compact_kernel<<<1, 1024, 0, st>>>(alive, count, n_static, orig, pos_next, orig_next, count_next, counts_out,
                                      exit_index, surv_out, last_count_out, last_index);
   CK(cudaGetLastError());
@@ -292,6 +298,7 @@ __global__ void exit_loss_kernel(const float* __restrict__ logits, const int32_t
 }
 void launch_exit_loss(const float* logits, const int32_t* labels, int n, int ncls, float w, float inv_n, float* dl,
                       float* loss_rows, int accumulate, cudaStream_t st) {
+  ProfScope ps(PC_EXIT_LOSS, st);
   exit_loss_kernel<<<(n + 127) / 128, 128, 0, st>>>(logits, labels, n, ncls, w, inv_n, dl, loss_rows, accumulate);
   CK(cudaGetLastError());
 }
@@ -324,6 +331,7 @@ __global__ void head_bcast_kernel(const float* __restrict__ dl, const float* __r
 void launch_head_grads(const float* pooled, const float* dl, const float* Wk, int n, int C, int ncls, int HW,
                        float* dW, float* db, float* bcast, cudaStream_t st) {
   const int tot = C * ncls + ncls;
+  ProfScope ps(PC_HEAD_GRADS, st, 2);
   head_dw_kernel<<<(tot + 127) / 128, 128, 0, st>>>(pooled, dl, n, C, ncls, dW, db);
   const long long nb = ((long long)n * C + 255) / 256;
   head_bcast_kernel<<<(unsigned)nb, 256, 0, st>>>(dl, Wk, n, C, ncls, 1.0f / (float)HW, bcast);
@@ -348,6 +356,7 @@ void launch_grad_finalize(const float* bcast, const bf16* sc, const bf16* yact, 
                           bf16* dz, cudaStream_t st) {
   const long long total = (long long)n * HW * C;
   const int blocks = (int)std::min<long long>((total + 255) / 256, 32LL * num_sms());
+  ProfScope ps(PC_GRAD_FINALIZE, st);
   grad_finalize_kernel<<<blocks, 256, 0, st>>>(bcast, sc, yact, act, n, HW, C, dz);
   CK(cudaGetLastError());
 }
@@ -365,6 +374,7 @@ __global__ void sum_kernel(const float* __restrict__ x, int n, float* out, float
   if (threadIdx.x == 0) *out = scale == 0.f ? sh[0] : (scale < 0.f ? sqrtf(sh[0]) : sh[0] * scale);
 }
 void launch_sum(const float* x, int n, float* out, float scale, cudaStream_t st) {
+  ProfScope ps(PC_SUM, st);
   sum_kernel<<<1, 1024, 0, st>>>(x, n, out, scale);
   CK(cudaGetLastError());
 }
@@ -457,6 +467,7 @@ void launch_sgd(float* w, float* v, const float* g, long long n, float lr, float
                 cudaStream_t st) {
   (void)n;
   (void)nseg;
+  ProfScope ps(PC_SGD, st);
   sgd_kernel<<<nblocks, SGD_THREADS, 0, st>>>(w, v, g, lr, mu, wd, segs_dev, block_seg_dev, block_start_dev,
                                                sq_partial);
   CK(cudaGetLastError());
@@ -471,7 +482,44 @@ __global__ void shadow_pack_kernel(const float* __restrict__ w, const SgdSeg* __
   }
 }
 void launch_shadow_pack(const float* w, const SgdSeg* segs_dev, int nseg, cudaStream_t st) {
+  ProfScope ps(PC_SHADOW_PACK, st);
   shadow_pack_kernel<<<dim3(64, nseg), 256, 0, st>>>(w, segs_dev);
+  CK(cudaGetLastError());
+}
+
+// ------------------------------------------------------------------------------------------------
+// row gather by an index list with a device-side count (retraining batch assembly from the window pool)
+__global__ void gather_rows_kernel(const uint4* __restrict__ src, const int32_t* __restrict__ idx, const int32_t* count,
+                                   int n_static, long long row_vec, uint4* __restrict__ dst) {
+  const int n = count ? min(*count, n_static) : n_static;
+  const long long total = (long long)n * row_vec;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+    const long long r = i / row_vec, c = i - r * row_vec;
+    dst[i] = __ldg(src + (long long)idx[r] * row_vec + c);
+  }
+}
+__global__ void gather_rows4_kernel(const uint32_t* __restrict__ src, const int32_t* __restrict__ idx, const int32_t* count,
+                                    int n_static, long long row_words, uint32_t* __restrict__ dst) {
+  const int n = count ? min(*count, n_static) : n_static;
+  const long long total = (long long)n * row_words;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+    const long long r = i / row_words, c = i - r * row_words;
+    dst[i] = __ldg(src + (long long)idx[r] * row_words + c);
+  }
+}
+void launch_gather_rows(const void* src, const int32_t* idx, const int32_t* count, int n_static, long long row_bytes,
+                        void* dst, cudaStream_t st) {
+  if (row_bytes % 4) throw ShapeError("gather_rows: row bytes must be a multiple of 4");
+  const bool v16 = (row_bytes % 16) == 0;
+  const long long total = (long long)n_static * (row_bytes / (v16 ? 16 : 4));
+  const int blocks = (int)std::min<long long>((total + 255) / 256, 32LL * num_sms());
+  if (blocks <= 0) return;
+  ProfScope ps(PC_GATHER, st);
+  if (v16)
+    gather_rows_kernel<<<blocks, 256, 0, st>>>((const uint4*)src, idx, count, n_static, row_bytes / 16, (uint4*)dst);
+  else
+    gather_rows4_kernel<<<blocks, 256, 0, st>>>((const uint32_t*)src, idx, count, n_static, row_bytes / 4,
+                                                (uint32_t*)dst);
   CK(cudaGetLastError());
 }
 

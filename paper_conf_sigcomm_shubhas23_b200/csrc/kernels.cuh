@@ -73,5 +73,7 @@ void launch_sgd(float* w, float* v, const float* g, long long n, float lr, float
                 int nseg, const int* block_seg_dev, const long long* block_start_dev, int nblocks, float* sq_partial,
                 cudaStream_t st);
 void launch_shadow_pack(const float* w, const SgdSeg* segs_dev, int nseg, cudaStream_t st);
+void launch_gather_rows(const void* src, const int32_t* idx, const int32_t* count, int n_static, long long row_bytes,
+                        void* dst, cudaStream_t st);
 
 }  // namespace adainf

@@ -12,6 +12,7 @@
 #include "api_common.h"
 #include "common.cuh"
 #include "model.h"
+#include "prof.h"
 
 namespace adainf {
 
@@ -267,9 +268,11 @@ void select_retrain(const adainf_select_in& in, int k, int32_t* out_idx, float* 
   const long long nb = (N + EMIT_THREADS - 1) / EMIT_THREADS;
   int* blk = (int*)take((size_t)nb * 8);
   int* offs = (int*)take((size_t)nb * 8);
-  project_ref_kernel<<<M, 256, 0, st>>>(in.ref, (const bf16*)in.W_bf16, D, P, M, mu, mun);
+  { ProfScope ps(PC_SELECT_PROJ, st);
+  project_ref_kernel<<<M, 256, 0, st>>>(in.ref, (const bf16*)in.W_bf16, D, P, M, mu, mun); }
   if (in.W_bf16) {
-    transpose_w_kernel<<<(D * P + 255) / 256, 256, 0, st>>>((const bf16*)in.W_bf16, D, P, Wt);
+    { ProfScope ps(PC_SELECT_PROJ, st);
+    transpose_w_kernel<<<(D * P + 255) / 256, 256, 0, st>>>((const bf16*)in.W_bf16, D, P, Wt); }
     CK(cudaMemsetAsync(zb, 0, (size_t)P * 4, st));
     ConvGeom g{};
     g.Cin = D;
@@ -280,13 +283,16 @@ void select_retrain(const adainf_select_in& in, int k, int32_t* out_idx, float* 
     g.H = g.W = g.Ho = g.Wo = 1;
     // Y [N][P] fp32 = X [N][D] . W [D][P] on the tensor cores
     conv_fwd(g, (const bf16*)in.X_bf16, nullptr, nullptr, (int)N, Wt, D, zb, nullptr, nullptr, 0, Y, true, st);
+    ProfScope ps(PC_SELECT_COSINE, st);
     cosine_key_kernel<false><<<(unsigned)((N * 32 + 255) / 256), 256, 0, st>>>(Y, N, P, mu, mun, M, in.exclude, keys,
                                                                               dist_all);
   } else {
+    ProfScope ps(PC_SELECT_COSINE, st);
     cosine_key_kernel<true><<<(unsigned)((N * 32 + 255) / 256), 256, 0, st>>>(in.X_bf16, N, P, mu, mun, M,
                                                                              in.exclude, keys, dist_all);
   }
   const int k_eff = (int)std::min<long long>(k, N);  // the k-th largest must exist
+  ProfScope ps_topk(PC_SELECT_TOPK, st, 12);
   radix_init_kernel<<<1, 256, 0, st>>>(rs, k_eff);
   const int hb = (int)std::min<long long>((N + 1023) / 1024, 4LL * num_sms());
   for (int pass = 0; pass < 4; ++pass) {
