@@ -1,15 +1,23 @@
 // Implicit-GEMM convolution on the 5th-gen tensor cores (tcgen05.mma kind::f16, fp32 accumulator in
-// TMEM), one kernel template for the three contractions of the hot path:
+// TMEM), one persistent warp-specialized kernel template for the three contractions of the hot path
+// (SURVEY §8(a) a2, a9):
 //
 //   FWD   D[pix][co]   = sum_{tap,ci} X[gather(pix,tap)][ci] * W[co][tap][ci]        A K-major, B K-major
 //   DGRAD D[pix'][ci]  = sum_{tap',co} dZ[gather(pix',tap')][co] * W[co][tap(tap')][ci]  A K-major, B MN-major
 //   WGRAD D[kconv][co] = sum_{pix} X[gather(pix,tap(kconv))][ci(kconv)] * dZ[pix][co]   A MN-major, B MN-major
 //
 // "Run one layer for all requests of the batch at once" is inherent: M spans every pixel of
-// every sample of the (compacted) batch.  Operands are gathered by 4 producer warps with 16-byte
-// cp.async (zero-fill for padding / out-of-range taps / rows beyond the device-side sample count) into
-// 128B-swizzled UMMA tiles; one elected thread of warp 4 issues the MMAs; the producer warps then run
-// the fused epilogue (TMEM -> registers -> bias / residual / activation / gradient masks -> HBM).
+// every sample of the (compacted) batch.
+//
+// Structure (one CTA per SM, persistent over output tiles, tile order n-fastest for L2 reuse of A):
+//   warps 0-3  producers: gather A/B 16-byte chunks with cp.async (zero-fill for padding, out-of-range
+//              taps and rows beyond the device-side sample count) into a STAGES-deep ring of
+//              128B-swizzled UMMA tiles; completion tracked by cp.async.mbarrier.arrive.noinc
+//   warp 4     TMEM owner + MMA issuer (one elected lane): 4 x tcgen05.mma (K=16) per 64-wide K-block,
+//              tcgen05.commit frees the smem stage; two TMEM accumulators (double buffer) so the
+//              epilogue of tile i overlaps the MMAs of tile i+1
+//   warps 5-8  epilogue: tcgen05.ld (32 lanes x 32 cols) -> bias / residual / activation / gradient
+//              terms and masks -> 128-bit global stores; frees the accumulator after the last load
 #pragma once
 #include "common.cuh"
 
@@ -48,19 +56,21 @@ struct ConvArgs {
   const bf16* yact;     // DGRAD: stored activation for the act' mask
   int mask_act;         // DGRAD: activation whose derivative masks (0 = none)
   int kb_per_split;     // WGRAD split-K (in 64-pixel blocks)
+  int splits;           // WGRAD number of splits
 };
 
 constexpr int BM = 128, BK = 64;
-constexpr int NUM_THREADS = 160;  // warps 0-3 producers + epilogue, warp 4 MMA issuer / TMEM owner
+constexpr int NUM_THREADS = 288;  // 4 producer warps, 1 MMA warp, 4 epilogue warps
 
 template <int MODE, int BN>
 struct ConvCfg {
-  static constexpr int STAGES = BN >= 256 ? 4 : (BN >= 128 ? 3 : 4);
   static constexpr int A_BYTES = BM * BK * 2;
   static constexpr int B_BYTES = BN * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int STAGES = (200 * 1024) / STAGE_BYTES > 8 ? 8 : (200 * 1024) / STAGE_BYTES;
   static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
-  static constexpr int TMEM_COLS = BN < 32 ? 32 : BN;
+  static constexpr int ACC_COLS = BN < 32 ? 32 : BN;
+  static constexpr int TMEM_COLS = 2 * ACC_COLS;  // double-buffered accumulator
 };
 
 // 128B-swizzle offsets inside a tile (bytes).
@@ -73,6 +83,57 @@ __device__ __forceinline__ uint32_t mnmaj_off(int r, int j) {
   return (uint32_t)((j >> 3) * 8192 + (r >> 3) * 1024 + (r & 7) * 128 + (((j & 7) ^ (r & 7)) << 4));
 }
 
+struct TileInfo {
+  long long m0;
+  int n0, kb0, kb1, z;
+};
+
+template <int MODE, int BN>
+__device__ __forceinline__ int num_tiles(const ConvArgs& a, long long npix, int& mt, int& nt) {
+  nt = (a.Nout + BN - 1) / BN;
+  if (MODE == MODE_WGRAD) {
+    mt = (a.K + BM - 1) / BM;
+    return mt * nt * a.splits;
+  }
+  mt = (int)((npix + BM - 1) / BM);
+  return mt * nt;
+}
+
+template <int MODE, int BN>
+__device__ __forceinline__ TileInfo tile_info(const ConvArgs& a, int t, int mt, int nt, int nkb_total) {
+  TileInfo ti;
+  const int n = t % nt;
+  const int r = t / nt;
+  ti.n0 = n * BN;
+  if (MODE == MODE_WGRAD) {
+    const int m = r % mt;
+    ti.z = r / mt;
+    ti.m0 = (long long)m * BM;
+    ti.kb0 = ti.z * a.kb_per_split;
+    ti.kb1 = min(ti.kb0 + a.kb_per_split, nkb_total);
+  } else {
+    ti.z = 0;
+    ti.m0 = (long long)r * BM;
+    ti.kb0 = 0;
+    ti.kb1 = nkb_total;
+  }
+  if (ti.kb1 < ti.kb0) ti.kb1 = ti.kb0;
+  return ti;
+}
+
+__device__ __forceinline__ void st_bf16x8(bf16* p, const float* v) {
+  __align__(16) bf16 h[8];
+#pragma unroll
+  for (int q = 0; q < 8; ++q) h[q] = __float2bfloat16_rn(v[q]);
+  *(uint4*)p = *(uint4*)h;
+}
+__device__ __forceinline__ void ld_bf16x8(const bf16* p, float* v) {
+  const uint4 raw = __ldg((const uint4*)p);
+  const bf16* h = (const bf16*)&raw;
+#pragma unroll
+  for (int q = 0; q < 8; ++q) v[q] = __bfloat162float(h[q]);
+}
+
 template <int MODE, int BN>
 __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArgs a) {
   using Cfg = ConvCfg<MODE, BN>;
@@ -82,39 +143,28 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint64_t* full = (uint64_t*)(smem + STAGES * Cfg::STAGE_BYTES);
   uint64_t* empty = full + STAGES;
-  uint64_t* tfull = empty + STAGES;
-  uint32_t* tmem_slot = (uint32_t*)(tfull + 1);
+  uint64_t* tfull = empty + STAGES;   // [2]
+  uint64_t* tempty = tfull + 2;       // [2]
+  uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nsamp = a.count ? *a.count : a.n_static;
   const int HWg = a.Hg * a.Wg;
   const long long npix = (long long)nsamp * HWg;
-
-  // tile coordinates
-  long long m0;
-  int n0, kb0, kb1;
+  int mt, nt;
+  const int ntile = num_tiles<MODE, BN>(a, npix, mt, nt);
   const int nkb_total = (MODE == MODE_WGRAD) ? (int)((npix + BK - 1) / BK) : (a.K + BK - 1) / BK;
-  if (MODE == MODE_WGRAD) {
-    m0 = (long long)blockIdx.x * BM;  // kconv
-    n0 = blockIdx.y * BN;             // co
-    kb0 = blockIdx.z * a.kb_per_split;
-    kb1 = min(kb0 + a.kb_per_split, nkb_total);
-    if (m0 >= a.K) return;
-  } else {
-    m0 = (long long)blockIdx.x * BM;  // pixel
-    n0 = blockIdx.y * BN;
-    kb0 = 0;
-    kb1 = nkb_total;
-    if (m0 >= npix) return;           // rows beyond the device-side count: nothing to do
-  }
-  const int nkb = max(kb1 - kb0, 0);
+  if ((int)blockIdx.x >= ntile) return;  // uniform: nothing for this CTA
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&full[s], 128);
       mbar_init(&empty[s], 1);
     }
-    mbar_init(tfull, 1);
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 128);
+    }
     fence_mbar_init();
   }
   if (warp == 4) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
@@ -127,214 +177,144 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
   if (warp < 4) {
     // ================= producers =================
     const int t = threadIdx.x;  // 0..127
-    if (MODE != MODE_WGRAD) {
-      // A: 128 rows (pixels) x 8 chunks; thread -> chunk t&7, rows (t>>3)+16*i
-      const int j = t & 7;
-      long long rowbase[8];
-      int iy0[8], ix0[8];
-#pragma unroll
-      for (int i = 0; i < 8; ++i) {
-        const long long m = m0 + (t >> 3) + 16 * i;
-        if (m < npix) {
-          const int n = (int)(m / HWg);
-          const int pix = (int)(m - (long long)n * HWg);
-          const int gy = pix / a.Wg, gx = pix - (pix / a.Wg) * a.Wg;
-          const int sn = a.src_map ? a.src_map[n] : n;
-          rowbase[i] = (long long)sn * a.Hs * a.Ws;
-          iy0[i] = gy * a.sy;
-          ix0[i] = gx * a.sx;
-        } else {
-          rowbase[i] = -1;
-          iy0[i] = 0;
-          ix0[i] = 0;
-        }
-      }
-      for (int kbi = 0; kbi < nkb; ++kbi) {
-        const int s = kbi % STAGES, u = kbi / STAGES;
-        if (u > 0) mbar_wait(&empty[s], (u - 1) & 1);
-        const uint32_t sa = smem_base + s * Cfg::STAGE_BYTES;
-        const uint32_t sb = sa + Cfg::A_BYTES;
-        const int k = (kb0 + kbi) * BK + j * 8;
-        const int tap = k / a.Cs;
-        const int c = k - tap * a.Cs;
-        const bool kval = k < a.K;
-        const int dy = kval ? a.ty[tap] : 0, dx = kval ? a.tx[tap] : 0;
+    int it = 0;                 // global k-block counter (ring position)
+    for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x) {
+      const TileInfo ti = tile_info<MODE, BN>(a, tile, mt, nt, nkb_total);
+      const int nkb = ti.kb1 - ti.kb0;
+      if (MODE != MODE_WGRAD) {
+        // A: 128 rows (pixels) x 8 chunks; thread -> chunk t&7, rows (t>>3)+16*i
+        const int j = t & 7;
+        long long rowbase[8];
+        int iy0[8], ix0[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
-          const int r = (t >> 3) + 16 * i;
-          const int iy = iy0[i] + dy, ix = ix0[i] + dx;
-          const bool v = kval && rowbase[i] >= 0 && iy >= 0 && iy < a.Hs && ix >= 0 && ix < a.Ws;
-          const bf16* g = v ? a.src + ((rowbase[i] + (long long)iy * a.Ws + ix) * a.Cs + c) : a.src;
-          cp_async16(sa + kmaj_off(r, j), g, v);
-        }
-        // B
-        if (MODE == MODE_FWD) {
-          // W [Nout][ldb] K-major: BN rows x 8 chunks
-          for (int idx = t; idx < BN * 8; idx += 128) {
-            const int r = idx >> 3, jj = idx & 7;
-            const int kk = (kb0 + kbi) * BK + jj * 8;
-            const bool v = (n0 + r) < a.Nout && kk < a.K;
-            const bf16* g = v ? a.B + ((long long)(n0 + r) * a.ldb + kk) : a.B;
-            cp_async16(sb + kmaj_off(r, jj), g, v);
-          }
-        } else {
-          // DGRAD: B MN-major [K=64 (tap',co) rows][BN ci]: element (k=(t',co), n=ci) = W[co][btap[t']][ci]
-          constexpr int CH = BN / 8;
-          for (int idx = t; idx < 64 * CH; idx += 128) {
-            const int r = idx / CH, jj = idx - (idx / CH) * CH;
-            const int kk = (kb0 + kbi) * BK + r;
-            const int tp = kk / a.Cs;
-            const int co = kk - tp * a.Cs;
-            const int ci = n0 + jj * 8;
-            const bool v = kk < a.K && ci < a.Nout;
-            const bf16* g = v ? a.B + ((long long)co * a.ldb + (long long)a.btap[tp] * a.Nout + ci) : a.B;
-            cp_async16(sb + mnmaj_off(r, jj), g, v);
-          }
-        }
-        cp_async_arrive_noinc(&full[s]);
-      }
-    } else {
-      // WGRAD: A MN-major [K=64 pixels][128 kconv]; thread -> kconv chunk j = t&15, pixels (t>>4)+8*i
-      const int j = t & 15;
-      const int kc = (int)m0 + j * 8;
-      const bool mval = kc < a.K;
-      const int tap = mval ? kc / a.Cs : 0;
-      const int c = kc - tap * a.Cs;
-      const int dy = a.ty[tap], dx = a.tx[tap];
-      for (int kbi = 0; kbi < nkb; ++kbi) {
-        const int s = kbi % STAGES, u = kbi / STAGES;
-        if (u > 0) mbar_wait(&empty[s], (u - 1) & 1);
-        const uint32_t sa = smem_base + s * Cfg::STAGE_BYTES;
-        const uint32_t sb = sa + Cfg::A_BYTES;
-        const long long p0 = (long long)(kb0 + kbi) * BK;
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          const int r = (t >> 4) + 8 * i;
-          const long long p = p0 + r;
-          bool v = mval && p < npix;
-          const bf16* g = a.src;
-          if (v) {
-            const int n = (int)(p / HWg);
-            const int pix = (int)(p - (long long)n * HWg);
-            const int gy = pix / a.Wg, gx = pix - (pix / a.Wg) * a.Wg;
-            const int iy = gy * a.sy + dy, ix = gx * a.sx + dx;
-            v = iy >= 0 && iy < a.Hs && ix >= 0 && ix < a.Ws;
-            const int sn = a.src_map ? a.src_map[n] : n;
-            if (v) g = a.src + ((((long long)sn * a.Hs + iy) * a.Ws + ix) * a.Cs + c);
-          }
-          cp_async16(sa + mnmaj_off(r, j), g, v);
-        }
-        // B: dZ [pix][Nout] MN-major [64 pixels][BN co]
-        constexpr int CH = BN / 8;
-        for (int idx = t; idx < 64 * CH; idx += 128) {
-          const int r = idx / CH, jj = idx - (idx / CH) * CH;
-          const long long p = p0 + r;
-          const bool v = p < npix && (n0 + jj * 8) < a.Nout;
-          const bf16* g = v ? a.B + (p * a.Nout + n0 + jj * 8) : a.B;
-          cp_async16(sb + mnmaj_off(r, jj), g, v);
-        }
-        cp_async_arrive_noinc(&full[s]);
-      }
-    }
-
-    // ================= epilogue =================
-    mbar_wait(tfull, 0);
-    tc_fence_after();
-    const int row = warp * 32 + lane;
-    const long long m = m0 + row;
-    const uint32_t trow = tmem + ((uint32_t)(warp * 32) << 16);
-    if (MODE == MODE_WGRAD) {
-      float* outp = (float*)a.out + ((long long)blockIdx.z * a.K + m) * a.Nout + n0;
-      for (int c0 = 0; c0 < BN; c0 += 32) {
-        float v[32];
-        if (nkb > 0) tmem_ld32(trow + c0, v);  // whole warp (.sync.aligned), stores predicated below
-        else
-#pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] = 0.f;
-        if (m >= a.K) continue;
-        if (n0 + c0 + 32 <= a.Nout && (a.Nout & 3) == 0) {
-#pragma unroll
-          for (int i = 0; i < 32; i += 4)
-            *(float4*)(outp + c0 + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
-        } else {
-          for (int i = 0; i < 32; ++i)
-            if (n0 + c0 + i < a.Nout) outp[c0 + i] = v[i];
-        }
-      }
-    } else {
-      const bool rv = m < npix;
-      long long orow = 0;
-      int n = 0;
-      if (rv) {
-        n = (int)(m / HWg);
-        const int pix = (int)(m - (long long)n * HWg);
-        const int gy = pix / a.Wg, gx = pix - (pix / a.Wg) * a.Wg;
-        orow = ((long long)n * a.Ho + gy * a.oys + a.oyo) * a.Wo + gx * a.oxs + a.oxo;
-      }
-      for (int c0 = 0; c0 < BN; c0 += 32) {
-        float v[32];
-        if (nkb > 0) tmem_ld32(trow + c0, v);
-        else
-#pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] = 0.f;
-        if (!rv) continue;
-        const int cb = n0 + c0;
-        if (cb >= a.Nout) continue;
-        const bool full32 = (cb + 32 <= a.Nout) && ((a.Nout & 7) == 0);
-        if (MODE == MODE_FWD) {
-          long long rrow = 0;
-          if (a.res) {
-            const long long pix_o = orow - (long long)n * a.Ho * a.Wo;
-            const int rn = a.res_map ? a.res_map[n] : n;
-            rrow = (long long)rn * a.Ho * a.Wo + pix_o;
-          }
-#pragma unroll
-          for (int i = 0; i < 32; ++i) {
-            const int ch = cb + i;
-            if (!full32 && ch >= a.Nout) break;
-            float x = __fadd_rn(v[i], a.bias[ch]);
-            if (a.res) x = __fadd_rn(x, __bfloat162float(a.res[rrow * a.Nout + ch]));
-            v[i] = act_apply(a.act, x);
-          }
-          if (a.out_f32) {
-            float* o = (float*)a.out + orow * a.Nout + cb;
-            for (int i = 0; i < 32; ++i)
-              if (cb + i < a.Nout) o[i] = v[i];
+          const long long m = ti.m0 + (t >> 3) + 16 * i;
+          if (m < npix) {
+            const int n = (int)(m / HWg);
+            const int pix = (int)(m - (long long)n * HWg);
+            const int gy = pix / a.Wg, gx = pix - gy * a.Wg;
+            const int sn = a.src_map ? __ldg(a.src_map + n) : n;
+            rowbase[i] = (long long)sn * a.Hs * a.Ws;
+            iy0[i] = gy * a.sy;
+            ix0[i] = gx * a.sx;
           } else {
-            bf16* o = (bf16*)a.out + orow * a.Nout + cb;
-            if (full32) {
+            rowbase[i] = 0;
+            iy0[i] = -100000;
+            ix0[i] = 0;
+          }
+        }
+        for (int kbi = 0; kbi < nkb; ++kbi, ++it) {
+          const int s = it % STAGES, u = it / STAGES;
+          if (u > 0) mbar_wait(&empty[s], (u - 1) & 1);
+          const uint32_t sa = smem_base + s * Cfg::STAGE_BYTES;
+          const uint32_t sb = sa + Cfg::A_BYTES;
+          const int k = (ti.kb0 + kbi) * BK + j * 8;
+          const int tap = k / a.Cs;
+          const int c = k - tap * a.Cs;
+          const bool kval = k < a.K;
+          const int dy = kval ? a.ty[tap] : -100000, dx = kval ? a.tx[tap] : 0;
 #pragma unroll
-              for (int i = 0; i < 32; i += 8) {
-                __align__(16) bf16 h[8];
+          for (int i = 0; i < 8; ++i) {
+            const int r = (t >> 3) + 16 * i;
+            const int iy = iy0[i] + dy, ix = ix0[i] + dx;
+            const bool v = (unsigned)iy < (unsigned)a.Hs && (unsigned)ix < (unsigned)a.Ws;
+            const bf16* g = v ? a.src + ((rowbase[i] + (long long)iy * a.Ws + ix) * a.Cs + c) : a.src;
+            cp_async16(sa + kmaj_off(r, j), g, v);
+          }
+          if (MODE == MODE_FWD) {
+            // W [Nout][ldb] K-major: BN rows x 8 chunks
 #pragma unroll
-                for (int q = 0; q < 8; ++q) h[q] = __float2bfloat16_rn(v[i + q]);
-                *(uint4*)(o + i) = *(uint4*)h;
-              }
-            } else {
-              for (int i = 0; i < 32; ++i)
-                if (cb + i < a.Nout) o[i] = __float2bfloat16_rn(v[i]);
+            for (int idx = t; idx < BN * 8; idx += 128) {
+              const int r = idx >> 3, jj = idx & 7;
+              const int kk = (ti.kb0 + kbi) * BK + jj * 8;
+              const bool v = (ti.n0 + r) < a.Nout && kk < a.K;
+              const bf16* g = v ? a.B + ((long long)(ti.n0 + r) * a.ldb + kk) : a.B;
+              cp_async16(sb + kmaj_off(r, jj), g, v);
+            }
+          } else {
+            // DGRAD: B MN-major [K=64 (tap',co) rows][BN ci]: element (k=(t',co), n=ci) = W[co][btap[t']][ci]
+            constexpr int CH = BN / 8;
+#pragma unroll
+            for (int idx = t; idx < 64 * CH; idx += 128) {
+              const int r = idx / CH, jj = idx - (idx / CH) * CH;
+              const int kk = (ti.kb0 + kbi) * BK + r;
+              const int tp = kk / a.Cs;
+              const int co = kk - tp * a.Cs;
+              const int ci = ti.n0 + jj * 8;
+              const bool v = kk < a.K && ci < a.Nout;
+              const bf16* g = v ? a.B + ((long long)co * a.ldb + (long long)a.btap[tp] * a.Nout + ci) : a.B;
+              cp_async16(sb + mnmaj_off(r, jj), g, v);
             }
           }
-        } else {  // DGRAD epilogue: + bcast + shortcut, x act'(y), -> bf16
-          bf16* o = (bf16*)a.out + orow * a.Nout + cb;
-          for (int i = 0; i < 32; ++i) {
-            const int ch = cb + i;
-            if (ch >= a.Nout) break;
-            float x = v[i];
-            if (a.bcast) x = __fadd_rn(x, a.bcast[(long long)n * a.Nout + ch]);
-            if (a.sc) x = __fadd_rn(x, __bfloat162float(a.sc[orow * a.Nout + ch]));
-            if (a.mask_act) x = __fmul_rn(x, act_grad(a.mask_act, __bfloat162float(a.yact[orow * a.Nout + ch])));
-            o[i] = __float2bfloat16_rn(x);
+          cp_async_arrive_noinc(&full[s]);
+        }
+      } else {
+        // WGRAD: A MN-major [K=64 pixels][128 kconv]; thread -> pixel row r = t>>1 (one pixel decomposition
+        // per K-block), kconv chunks j = (t&1)*8 .. +8 (taps / channels fixed per tile)
+        const int r = t >> 1;
+        const int j0 = (t & 1) * 8;
+        int dyj[8], dxj[8], cj[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+          const int kc = (int)ti.m0 + (j0 + q) * 8;
+          const bool mval = kc < a.K;
+          const int tap = mval ? kc / a.Cs : 0;
+          cj[q] = kc - tap * a.Cs;
+          dyj[q] = mval ? a.ty[tap] : -100000;
+          dxj[q] = a.tx[tap];
+        }
+        for (int kbi = 0; kbi < nkb; ++kbi, ++it) {
+          const int s = it % STAGES, u = it / STAGES;
+          if (u > 0) mbar_wait(&empty[s], (u - 1) & 1);
+          const uint32_t sa = smem_base + s * Cfg::STAGE_BYTES;
+          const uint32_t sb = sa + Cfg::A_BYTES;
+          const long long p0 = (long long)(ti.kb0 + kbi) * BK;
+          const long long p = p0 + r;
+          long long base = 0;
+          int gy0 = -100000, gx0 = 0;
+          if (p < npix) {
+            const int n = (int)(p / HWg);
+            const int pix = (int)(p - (long long)n * HWg);
+            gy0 = pix / a.Wg;
+            gx0 = pix - gy0 * a.Wg;
+            gy0 *= a.sy;
+            gx0 *= a.sx;
+            base = (long long)(a.src_map ? __ldg(a.src_map + n) : n) * a.Hs * a.Ws;
           }
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            const int iy = gy0 + dyj[q], ix = gx0 + dxj[q];
+            const bool v = (unsigned)iy < (unsigned)a.Hs && (unsigned)ix < (unsigned)a.Ws;
+            const bf16* g = v ? a.src + ((base + (long long)iy * a.Ws + ix) * a.Cs + cj[q]) : a.src;
+            cp_async16(sa + mnmaj_off(r, j0 + q), g, v);
+          }
+          // B: dZ [pix][Nout] MN-major [64 pixels][BN co]
+          constexpr int CH = BN / 8;
+#pragma unroll
+          for (int idx = t; idx < 64 * CH; idx += 128) {
+            const int r = idx / CH, jj = idx - (idx / CH) * CH;
+            const long long p = p0 + r;
+            const bool v = p < npix && (ti.n0 + jj * 8) < a.Nout;
+            const bf16* g = v ? a.B + (p * a.Nout + ti.n0 + jj * 8) : a.B;
+            cp_async16(sb + mnmaj_off(r, jj), g, v);
+          }
+          cp_async_arrive_noinc(&full[s]);
         }
       }
     }
   } else if (warp == 4) {
     // ================= MMA issuer =================
-    if (nkb > 0) {
-      constexpr uint32_t IDESC = make_idesc(BM, BN, MODE == MODE_WGRAD ? 1 : 0, MODE == MODE_FWD ? 0 : 1);
-      for (int kbi = 0; kbi < nkb; ++kbi) {
-        const int s = kbi % STAGES, u = kbi / STAGES;
+    constexpr uint32_t IDESC = make_idesc(BM, BN, MODE == MODE_WGRAD ? 1 : 0, MODE == MODE_FWD ? 0 : 1);
+    int it = 0, lt = 0;
+    for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++lt) {
+      const TileInfo ti = tile_info<MODE, BN>(a, tile, mt, nt, nkb_total);
+      const int nkb = ti.kb1 - ti.kb0;
+      const int b = lt & 1, ub = lt >> 1;
+      if (ub > 0) mbar_wait(&tempty[b], (ub - 1) & 1);  // epilogue drained this accumulator
+      tc_fence_after();
+      const uint32_t dacc = tmem + (uint32_t)(b * Cfg::ACC_COLS);
+      for (int kbi = 0; kbi < nkb; ++kbi, ++it) {
+        const int s = it % STAGES, u = it / STAGES;
         mbar_wait(&full[s], u & 1);
         fence_proxy_async_smem();
         tc_fence_after();
@@ -348,17 +328,165 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
             else ad = make_sdesc(sa + kk * 32, 16, 1024);
             if (MODE == MODE_FWD) bd = make_sdesc(sb + kk * 32, 16, 1024);
             else bd = make_sdesc(sb + kk * 2048, 8192, 1024);
-            umma_bf16(tmem, ad, bd, IDESC, (kbi | kk) != 0);
+            umma_bf16(dacc, ad, bd, IDESC, (kbi | kk) != 0);
           }
           umma_commit(&empty[s]);
-          if (kbi == nkb - 1) umma_commit(tfull);
+          if (kbi == nkb - 1) umma_commit(&tfull[b]);
         }
         __syncwarp();
       }
-    } else if (lane == 0) {
-      mbar_arrive(tfull);
+      if (nkb == 0 && lane == 0) mbar_arrive(&tfull[b]);
+      __syncwarp();
     }
-    __syncwarp();
+  } else {
+    // ================= epilogue =================
+    const int q = warp & 3;  // TMEM lane quadrant of this warp
+    const int row = q * 32 + lane;
+    int lt = 0;
+    for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++lt) {
+      const TileInfo ti = tile_info<MODE, BN>(a, tile, mt, nt, nkb_total);
+      const int nkb = ti.kb1 - ti.kb0;
+      const int b = lt & 1, ub = lt >> 1;
+      mbar_wait(&tfull[b], ub & 1);
+      tc_fence_after();
+      const uint32_t trow = tmem + (uint32_t)(b * Cfg::ACC_COLS) + ((uint32_t)(q * 32) << 16);
+      const long long m = ti.m0 + row;
+      if (MODE == MODE_WGRAD) {
+        float* outp = (float*)a.out + ((long long)ti.z * a.K + m) * a.Nout + ti.n0;
+#pragma unroll 1
+        for (int c0 = 0; c0 < BN; c0 += 32) {
+          float v[32];
+          if (nkb > 0) tmem_ld32(trow + c0, v);
+          else
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] = 0.f;
+          if (c0 + 32 >= BN) {
+            tc_fence_before();
+            mbar_arrive(&tempty[b]);
+          }
+          if (m >= a.K) continue;
+          if (ti.n0 + c0 + 32 <= a.Nout && (a.Nout & 3) == 0) {
+#pragma unroll
+            for (int i = 0; i < 32; i += 4)
+              *(float4*)(outp + c0 + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+          } else {
+            for (int i = 0; i < 32; ++i)
+              if (ti.n0 + c0 + i < a.Nout) outp[c0 + i] = v[i];
+          }
+        }
+      } else {
+        const bool rv = m < npix;
+        long long orow = 0, rrow = 0;
+        int n = 0;
+        if (rv) {
+          n = (int)(m / HWg);
+          const int pix = (int)(m - (long long)n * HWg);
+          const int gy = pix / a.Wg, gx = pix - gy * a.Wg;
+          orow = ((long long)n * a.Ho + gy * a.oys + a.oyo) * a.Wo + gx * a.oxs + a.oxo;
+          if (MODE == MODE_FWD && a.res) {
+            const int rn = a.res_map ? __ldg(a.res_map + n) : n;
+            rrow = (long long)rn * a.Ho * a.Wo + (orow - (long long)n * a.Ho * a.Wo);
+          }
+        }
+#pragma unroll 1
+        for (int c0 = 0; c0 < BN; c0 += 32) {
+          float v[32];
+          if (nkb > 0) tmem_ld32(trow + c0, v);
+          else
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] = 0.f;
+          if (c0 + 32 >= BN) {
+            tc_fence_before();
+            mbar_arrive(&tempty[b]);  // accumulator free for the tile after next
+          }
+          const int cb = ti.n0 + c0;
+          if (!rv || cb >= a.Nout) continue;
+          const bool vec = (cb + 32 <= a.Nout) && ((a.Nout & 7) == 0);
+          if (MODE == MODE_FWD) {
+            if (vec) {
+#pragma unroll
+              for (int i = 0; i < 32; ++i) v[i] = __fadd_rn(v[i], __ldg(a.bias + cb + i));  // flat params: 4B-aligned
+              if (a.res) {
+#pragma unroll
+                for (int i = 0; i < 32; i += 8) {
+                  float r8[8];
+                  ld_bf16x8(a.res + rrow * a.Nout + cb + i, r8);
+#pragma unroll
+                  for (int qq = 0; qq < 8; ++qq) v[i + qq] = __fadd_rn(v[i + qq], r8[qq]);
+                }
+              }
+#pragma unroll
+              for (int i = 0; i < 32; ++i) v[i] = act_apply(a.act, v[i]);
+              if (a.out_f32) {
+                float* o = (float*)a.out + orow * a.Nout + cb;
+#pragma unroll
+                for (int i = 0; i < 32; i += 4) *(float4*)(o + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+              } else {
+                bf16* o = (bf16*)a.out + orow * a.Nout + cb;
+#pragma unroll
+                for (int i = 0; i < 32; i += 8) st_bf16x8(o + i, v + i);
+              }
+            } else {
+              for (int i = 0; i < 32; ++i) {
+                const int ch = cb + i;
+                if (ch >= a.Nout) break;
+                float x = __fadd_rn(v[i], a.bias[ch]);
+                if (a.res) x = __fadd_rn(x, __bfloat162float(a.res[rrow * a.Nout + ch]));
+                x = act_apply(a.act, x);
+                if (a.out_f32) ((float*)a.out)[orow * a.Nout + ch] = x;
+                else ((bf16*)a.out)[orow * a.Nout + ch] = __float2bfloat16_rn(x);
+              }
+            }
+          } else {  // DGRAD epilogue: + bcast + shortcut, x act'(y), -> bf16
+            if (vec) {
+              if (a.bcast) {
+#pragma unroll
+                for (int i = 0; i < 32; i += 4) {
+                  const float4 bb = __ldg((const float4*)(a.bcast + (long long)n * a.Nout + cb + i));
+                  v[i] = __fadd_rn(v[i], bb.x);
+                  v[i + 1] = __fadd_rn(v[i + 1], bb.y);
+                  v[i + 2] = __fadd_rn(v[i + 2], bb.z);
+                  v[i + 3] = __fadd_rn(v[i + 3], bb.w);
+                }
+              }
+              if (a.sc) {
+#pragma unroll
+                for (int i = 0; i < 32; i += 8) {
+                  float r8[8];
+                  ld_bf16x8(a.sc + orow * a.Nout + cb + i, r8);
+#pragma unroll
+                  for (int qq = 0; qq < 8; ++qq) v[i + qq] = __fadd_rn(v[i + qq], r8[qq]);
+                }
+              }
+              if (a.mask_act) {
+#pragma unroll
+                for (int i = 0; i < 32; i += 8) {
+                  float y8[8];
+                  ld_bf16x8(a.yact + orow * a.Nout + cb + i, y8);
+#pragma unroll
+                  for (int qq = 0; qq < 8; ++qq) v[i + qq] = __fmul_rn(v[i + qq], act_grad(a.mask_act, y8[qq]));
+                }
+              }
+              bf16* o = (bf16*)a.out + orow * a.Nout + cb;
+#pragma unroll
+              for (int i = 0; i < 32; i += 8) st_bf16x8(o + i, v + i);
+            } else {
+              bf16* o = (bf16*)a.out + orow * a.Nout + cb;
+              for (int i = 0; i < 32; ++i) {
+                const int ch = cb + i;
+                if (ch >= a.Nout) break;
+                float x = v[i];
+                if (a.bcast) x = __fadd_rn(x, a.bcast[(long long)n * a.Nout + ch]);
+                if (a.sc) x = __fadd_rn(x, __bfloat162float(a.sc[orow * a.Nout + ch]));
+                if (a.mask_act)
+                  x = __fmul_rn(x, act_grad(a.mask_act, __bfloat162float(a.yact[orow * a.Nout + ch])));
+                o[i] = __float2bfloat16_rn(x);
+              }
+            }
+          }
+        }
+      }
+    }
   }
 
   tc_fence_before();

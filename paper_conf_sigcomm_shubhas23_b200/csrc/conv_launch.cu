@@ -21,8 +21,10 @@ int num_sms() {
   return g_num_sms;
 }
 
+// persistent launch: one CTA per SM (or fewer when there are fewer tiles)
 template <int MODE, int BN>
-static void launch_t(const ConvArgs& a, dim3 grid, cudaStream_t st) {
+static void launch_t(const ConvArgs& a, long long max_tiles, cudaStream_t st) {
+  dim3 grid((unsigned)std::max(1LL, std::min<long long>(max_tiles, num_sms())));
   using Cfg = ConvCfg<MODE, BN>;
   static bool attr = false;
   if (!attr) {
@@ -35,14 +37,14 @@ static void launch_t(const ConvArgs& a, dim3 grid, cudaStream_t st) {
 }
 
 template <int MODE>
-static void launch_bn(int BN, const ConvArgs& a, dim3 grid, cudaStream_t st) {
+static void launch_bn(int BN, const ConvArgs& a, long long max_tiles, cudaStream_t st) {
   switch (BN) {
     case 32:
-      if constexpr (MODE == MODE_FWD) { launch_t<MODE, 32>(a, grid, st); return; }
+      if constexpr (MODE == MODE_FWD) { launch_t<MODE, 32>(a, max_tiles, st); return; }
       break;
-    case 64: launch_t<MODE, 64>(a, grid, st); return;
-    case 128: launch_t<MODE, 128>(a, grid, st); return;
-    case 256: launch_t<MODE, 256>(a, grid, st); return;
+    case 64: launch_t<MODE, 64>(a, max_tiles, st); return;
+    case 128: launch_t<MODE, 128>(a, max_tiles, st); return;
+    case 256: launch_t<MODE, 256>(a, max_tiles, st); return;
   }
   throw std::runtime_error("unsupported BN");
 }
@@ -91,9 +93,8 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
   a.act = act;
   const int BN = pick_bn(g.Cout, false);
   const long long mt = ((long long)n_static * g.Ho * g.Wo + BM - 1) / BM;
-  dim3 grid((unsigned)mt, (g.Cout + BN - 1) / BN, 1);
   if (mt == 0) return;
-  launch_bn<MODE_FWD>(BN, a, grid, st);
+  launch_bn<MODE_FWD>(BN, a, mt * ((g.Cout + BN - 1) / BN), st);
 }
 
 void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n, const float* bcast,
@@ -143,8 +144,7 @@ void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n
       a.mask_act = mask_act;
       const int BN = pick_bn(g.Cin, true);
       const long long mt = ((long long)n * a.Hg * a.Wg + BM - 1) / BM;
-      dim3 grid((unsigned)mt, (g.Cin + BN - 1) / BN, 1);
-      launch_bn<MODE_DGRAD>(BN, a, grid, st);
+      launch_bn<MODE_DGRAD>(BN, a, mt * ((g.Cin + BN - 1) / BN), st);
     }
 }
 
@@ -174,15 +174,36 @@ __global__ void wgrad_reduce_kernel(const float* __restrict__ part, int S, int K
   }
 }
 
-// column sums of dz [P][C] -> db[C], deterministic: per-block fixed-order partials, then fixed-order sum
-__global__ void colsum_partial_kernel(const bf16* __restrict__ dz, long long P, int C, int rows_per_block,
-                                      float* __restrict__ part) {
+// column sums of dz [P][C] -> db[C], deterministic: each block reduces a contiguous row range with
+// 128-bit loads (thread = 8-channel vector x row group), fixed-order smem reduction -> part[block][C];
+// then a fixed-order sum over blocks.
+constexpr int CS_THREADS = 256;
+__global__ void __launch_bounds__(CS_THREADS) colsum_partial_kernel(const bf16* __restrict__ dz, long long P, int C,
+                                                                     long long rows_per_block,
+                                                                     float* __restrict__ part) {
+  extern __shared__ float red[];  // [groups][C]
+  const int CV = C / 8, groups = CS_THREADS / CV;
+  const int v = threadIdx.x % CV, g = threadIdx.x / CV;
   const long long r0 = (long long)blockIdx.x * rows_per_block;
   const long long r1 = min(P, r0 + rows_per_block);
-  for (int c = threadIdx.x; c < C; c += blockDim.x) {
-    float acc = 0.f;
-    for (long long r = r0; r < r1; ++r) acc += __bfloat162float(dz[r * C + c]);
-    part[(long long)blockIdx.x * C + c] = acc;
+  float acc[8];
+#pragma unroll
+  for (int q = 0; q < 8; ++q) acc[q] = 0.f;
+  if (g < groups)
+    for (long long r = r0 + g; r < r1; r += groups) {
+      const uint4 raw = __ldg((const uint4*)(dz + r * C + v * 8));
+      const bf16* h = (const bf16*)&raw;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) acc[q] += __bfloat162float(h[q]);
+    }
+  if (g < groups)
+#pragma unroll
+    for (int q = 0; q < 8; ++q) red[g * C + v * 8 + q] = acc[q];
+  __syncthreads();
+  for (int c = threadIdx.x; c < C; c += CS_THREADS) {
+    float s = 0.f;
+    for (int q = 0; q < groups; ++q) s += red[q * C + c];
+    part[(long long)blockIdx.x * C + c] = s;
   }
 }
 __global__ void colsum_final_kernel(const float* __restrict__ part, int nb, int C, float* __restrict__ out) {
@@ -192,6 +213,14 @@ __global__ void colsum_final_kernel(const float* __restrict__ part, int nb, int 
   for (int b = 0; b < nb; ++b) acc += part[(long long)b * C + c];
   out[c] = acc;
 }
+static int colsum_blocks(long long P) { return (int)std::max(1LL, std::min<long long>((P + 63) / 64, 4LL * num_sms())); }
+
+// split-K factor: one balanced wave of persistent CTAs (units = tiles * S <= #SMs), each unit a contiguous
+// range of 64-pixel K-blocks; the fp32 partials are reduced in fixed order (deterministic)
+static int wgrad_splits(int tiles, int nkb) {
+  if (tiles >= num_sms()) return 1;
+  return std::max(1, std::min(nkb, num_sms() / tiles));
+}
 
 size_t wgrad_ws_bytes(const ConvGeom& g, int n) {
   const long long npix = (long long)n * g.Ho * g.Wo;
@@ -199,11 +228,10 @@ size_t wgrad_ws_bytes(const ConvGeom& g, int n) {
   const int Kconv = g.KH * g.KW * g.Cin;
   const int BN = pick_bn(g.Cout, true);
   const int tiles = ((Kconv + BM - 1) / BM) * ((g.Cout + BN - 1) / BN);
-  int S = std::max(1, std::min(nkb, (2 * num_sms() + tiles - 1) / tiles));
+  int S = wgrad_splits(tiles, nkb);
   const int kbs = (nkb + S - 1) / S;
   S = (nkb + kbs - 1) / kbs;
-  const long long colsum_blocks = (npix + 255) / 256;
-  return (size_t)S * Kconv * g.Cout * sizeof(float) + (size_t)colsum_blocks * g.Cout * sizeof(float);
+  return (size_t)S * Kconv * g.Cout * sizeof(float) + (size_t)colsum_blocks(npix) * g.Cout * sizeof(float);
 }
 
 void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin_real, float* ws, size_t ws_bytes,
@@ -213,7 +241,7 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
   const int Kconv = g.KH * g.KW * g.Cin;
   const int BN = pick_bn(g.Cout, true);
   const int tiles = ((Kconv + BM - 1) / BM) * ((g.Cout + BN - 1) / BN);
-  int S = std::max(1, std::min(nkb, (2 * num_sms() + tiles - 1) / tiles));
+  int S = wgrad_splits(tiles, nkb);
   const int kbs = (nkb + S - 1) / S;
   S = (nkb + kbs - 1) / kbs;
   if (wgrad_ws_bytes(g, n) > ws_bytes) throw std::runtime_error("wgrad workspace too small");
@@ -237,8 +265,8 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
   a.Nout = g.Cout;
   a.out = ws;
   a.kb_per_split = kbs;
-  dim3 grid((Kconv + BM - 1) / BM, (g.Cout + BN - 1) / BN, S);
-  launch_bn<MODE_WGRAD>(BN, a, grid, st);
+  a.splits = S;
+  launch_bn<MODE_WGRAD>(BN, a, (long long)tiles * S, st);
   dim3 rg((Kconv + 31) / 32, (g.Cout + 31) / 32);
   {
   ProfScope ps(PC_WGRAD_REDUCE, st);
@@ -247,10 +275,12 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
   }
   if (db) {
     float* part = ws + (size_t)S * Kconv * g.Cout;
-    const int rpb = 256;
-    const int nb = (int)((npix + rpb - 1) / rpb);
+    const int nb = colsum_blocks(npix);
+    const long long rpb = (npix + nb - 1) / nb;
+    if (g.Cout % 8 || g.Cout / 8 > CS_THREADS) throw ShapeError("colsum: Cout must be a multiple of 8, <= 2048");
+    const int groups = CS_THREADS / (g.Cout / 8);
     ProfScope ps(PC_BIAS_COLSUM, st, 2);
-    colsum_partial_kernel<<<nb, 128, 0, st>>>(dz, npix, g.Cout, rpb, part);
+    colsum_partial_kernel<<<nb, CS_THREADS, (size_t)groups * g.Cout * 4, st>>>(dz, npix, g.Cout, rpb, part);
     colsum_final_kernel<<<(g.Cout + 127) / 128, 128, 0, st>>>(part, nb, g.Cout, db);
     CK(cudaGetLastError());
   }

@@ -90,39 +90,55 @@ void launch_maxpool_fwd(const bf16* x, const int* map, const int* count, int n_s
   CK(cudaGetLastError());
 }
 
+// one thread per (n, ih, iw, 8-channel vector): sums dT over the windows whose FIRST argmax is this
+// element (fixed window order), then the producer's activation mask; 128-bit loads / stores
 __global__ void maxpool_bwd_kernel(const bf16* __restrict__ dT, const uint8_t* __restrict__ amax,
                                    const bf16* __restrict__ yact, int act, long long n, int H, int W, int C, int K,
                                    int s, int p, int Ho, int Wo, bf16* __restrict__ dz) {
-  const long long total = n * H * W * C;
+  const int CV = C / 8;
+  const long long total = n * H * W * CV;
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
-    const int c = (int)(i % C);
-    long long r = i / C;
+    const int cv = (int)(i % CV);
+    long long r = i / CV;
     const int iw = (int)(r % W);
     r /= W;
     const int ih = (int)(r % H);
     const long long b = r / H;
-    // windows ho with ho*s - p <= ih <= ho*s - p + K - 1
     const int ho_lo = max(0, (ih + p - K + s) / s), ho_hi = min(Ho - 1, (ih + p) / s);
     const int wo_lo = max(0, (iw + p - K + s) / s), wo_hi = min(Wo - 1, (iw + p) / s);
-    float acc = 0.f;
+    float acc[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) acc[q] = 0.f;
     for (int ho = ho_lo; ho <= ho_hi; ++ho) {
       const int kh = ih - (ho * s - p);
       if (kh < 0 || kh >= K) continue;
       for (int wo = wo_lo; wo <= wo_hi; ++wo) {
         const int kw = iw - (wo * s - p);
         if (kw < 0 || kw >= K) continue;
-        const long long oi = ((b * Ho + ho) * Wo + wo) * C + c;
-        if (amax[oi] == (uint8_t)(kh * K + kw)) acc = __fadd_rn(acc, __bfloat162float(dT[oi]));
+        const long long oi = ((b * Ho + ho) * Wo + wo) * C + cv * 8;
+        const uint2 am = __ldg((const uint2*)(amax + oi));
+        const uint8_t* a8 = (const uint8_t*)&am;
+        const uint4 dv = __ldg((const uint4*)(dT + oi));
+        const bf16* d8 = (const bf16*)&dv;
+        const uint8_t me = (uint8_t)(kh * K + kw);
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+          if (a8[q] == me) acc[q] = __fadd_rn(acc[q], __bfloat162float(d8[q]));
       }
     }
-    const float g = __fmul_rn(acc, act_grad(act, __bfloat162float(yact[i])));
-    dz[i] = __float2bfloat16_rn(g);
+    const long long xi = ((b * H + ih) * W + iw) * C + cv * 8;
+    const uint4 yv = __ldg((const uint4*)(yact + xi));
+    const bf16* y8 = (const bf16*)&yv;
+    __align__(16) bf16 o[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) o[q] = __float2bfloat16_rn(__fmul_rn(acc[q], act_grad(act, __bfloat162float(y8[q]))));
+    *(uint4*)(dz + xi) = *(uint4*)o;
   }
 }
 void launch_maxpool_bwd(const bf16* dT, const uint8_t* amax, const bf16* yact, int act, int n, int H, int W, int C,
                         int K, int s, int p, int Ho, int Wo, bf16* dz, cudaStream_t st) {
-  const long long total = (long long)n * H * W * C;
-  const int blocks = (int)std::min<long long>((total + 255) / 256, 32LL * num_sms());
+  const long long total = (long long)n * H * W * (C / 8);
+  const int blocks = (int)std::min<long long>((total + 255) / 256, 64LL * num_sms());
   ProfScope ps(PC_POOL_BWD, st);
   maxpool_bwd_kernel<<<blocks, 256, 0, st>>>(dT, amax, yact, act, n, H, W, C, K, s, p, Ho, Wo, dz);
   CK(cudaGetLastError());
