@@ -268,19 +268,24 @@ def main():
     stream = torch.cuda.current_stream()
     n_global = K_SEL * world
 
-    # thresholds: calibrated once on the first (untimed) batch from full-depth confidences (all exits
-    # disabled), placed in the widest gap near the 25/25/25 quantiles
+    # thresholds: calibrated on the request batch from full-depth confidences (all exits disabled),
+    # placed in the widest gap near the 25/25/25 quantiles; re-done after warm-up because the warm-up
+    # retraining steps move the exit confidences
     calib = B.alloc_outs(m, INF_B)
-    conf_all = np.zeros((INF_B, 4), np.float32)
-    for k in range(4):
-        taus = [2.0] * 3
-        if k < 3:
-            taus[k] = 0.0
-            taus[:k] = [2.0] * k
-        app.infer(x_inf, taus, [calib])
-        torch.cuda.synchronize()
-        conf_all[:, k] = calib["conf"].cpu().numpy()
-    taus = [float(t) for t in synth.calibrate_thresholds(conf_all, EXIT_FRACTIONS)]
+
+    def calibrate():
+        conf_all = np.zeros((INF_B, 4), np.float32)
+        for k in range(4):
+            tk = [2.0] * 3
+            if k < 3:
+                tk[k] = 0.0
+            app.infer(x_inf, tk, [calib])
+            torch.cuda.synchronize()
+            conf_all[:, k] = calib["conf"].cpu().numpy()
+        return [float(t) for t in synth.calibrate_thresholds(conf_all, EXIT_FRACTIONS)]
+
+    taus = calibrate()
+
     def step_device(out_counts):
         outs["exit_counts"] = out_counts
         app.infer(x_inf, taus, [outs])
@@ -293,6 +298,7 @@ def main():
     for i in range(args.warmup):
         step_device(cnt_buf[-1 - i % 32])
     torch.cuda.synchronize()
+    taus[:] = calibrate()
     barrier()
 
     # ---- timed region (device time, CUDA events on the launching stream) ----

@@ -31,6 +31,10 @@ adainf_status adainf_dbg_conv_wgrad(const void* x, const void* dz, int32_t n, in
                                     int32_t Co, int32_t KH, int32_t KW, int32_t stride, int32_t pad, float* dw,
                                     float* db, adainf_stream_t stream);
 
+/* Conv kernel selection for A/B tests: 0 = generic gather kernel only, 1 = default routing (window
+ * kernel for stride-1 3x3 dgrad at H <= 14), 2 = window kernel for every eligible stride-1 3x3 fwd/dgrad. */
+adainf_status adainf_dbg_set_win_mode(int32_t mode);
+
 /* Launch accounting and per-kernel-class timing (CUDA events on the launching stream).
  * adainf_launch_count: total kernels launched by the library since load (host-side counter).
  * adainf_prof_enable(1): bracket every launch class with events; adainf_prof_query (synchronizing)

@@ -92,6 +92,7 @@ def lib():
             "adainf_dp_attach": [vp, vp, i32, i32],
             "adainf_nccl_unique_id": [vp],
             "adainf_gather_rows": [vp, vp, vp, i32, i64, vp, vp],
+            "adainf_dbg_set_win_mode": [i32],
             "adainf_prof_enable": [i32],
             "adainf_prof_reset": [],
             "adainf_prof_query": [vp, i32, C.POINTER(i32)],
@@ -336,6 +337,10 @@ def prof_query():
 
 
 # ---- kernel-level (include/adainf_debug.h) ----
+def dbg_set_win_mode(mode: int):
+    check(lib().adainf_dbg_set_win_mode(int(mode)))
+
+
 def dbg_conv_fwd(x, w, b, stride, pad, act=0, res=None, out_f32=False, stream=None):
     import torch
     n, H, W_, Cc = x.shape

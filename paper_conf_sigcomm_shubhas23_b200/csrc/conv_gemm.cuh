@@ -234,16 +234,30 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
           } else {
             // DGRAD: B MN-major [K=64 (tap',co) rows][BN ci]: element (k=(t',co), n=ci) = W[co][btap[t']][ci]
             constexpr int CH = BN / 8;
+            const int kb64 = (ti.kb0 + kbi) * BK;
+            if ((a.Cs & 63) == 0) {  // the whole K-block lies in one tap: one division per K-block
+              const int tp = kb64 / a.Cs;
+              const int co0 = kb64 - tp * a.Cs;
+              const bf16* wb = a.B + (long long)co0 * a.ldb + (long long)a.btap[tp] * a.Nout + ti.n0;
 #pragma unroll
-            for (int idx = t; idx < 64 * CH; idx += 128) {
-              const int r = idx / CH, jj = idx - (idx / CH) * CH;
-              const int kk = (ti.kb0 + kbi) * BK + r;
-              const int tp = kk / a.Cs;
-              const int co = kk - tp * a.Cs;
-              const int ci = ti.n0 + jj * 8;
-              const bool v = kk < a.K && ci < a.Nout;
-              const bf16* g = v ? a.B + ((long long)co * a.ldb + (long long)a.btap[tp] * a.Nout + ci) : a.B;
-              cp_async16(sb + mnmaj_off(r, jj), g, v);
+              for (int idx = t; idx < 64 * CH; idx += 128) {
+                const int r = idx / CH, jj = idx % CH;
+                const bool v = (ti.n0 + jj * 8) < a.Nout;
+                const bf16* g = v ? wb + (long long)r * a.ldb + jj * 8 : a.B;
+                cp_async16(sb + mnmaj_off(r, jj), g, v);
+              }
+            } else {
+#pragma unroll
+              for (int idx = t; idx < 64 * CH; idx += 128) {
+                const int r = idx / CH, jj = idx % CH;
+                const int kk = kb64 + r;
+                const int tp = kk / a.Cs;
+                const int co = kk - tp * a.Cs;
+                const int ci = ti.n0 + jj * 8;
+                const bool v = kk < a.K && ci < a.Nout;
+                const bf16* g = v ? a.B + ((long long)co * a.ldb + (long long)a.btap[tp] * a.Nout + ci) : a.B;
+                cp_async16(sb + mnmaj_off(r, jj), g, v);
+              }
             }
           }
           cp_async_arrive_noinc(&full[s]);

@@ -4,7 +4,10 @@
 #include <cstdio>
 #include <stdexcept>
 
+#include <cstdlib>
+
 #include "conv_gemm.cuh"
+#include "conv_win.cuh"
 #include "prof.h"
 #include "runtime.h"
 
@@ -49,6 +52,48 @@ static void launch_bn(int BN, const ConvArgs& a, long long max_tiles, cudaStream
   throw std::runtime_error("unsupported BN");
 }
 
+// ---- window kernel (stride-1 3x3 pad-1) ----
+static int g_win_mode = -1;  // -1 unset, 0 disabled, 1 base-offset 0, 2 base-offset phase
+int win_mode() {
+  if (g_win_mode < 0) {
+    const char* e = getenv("ADAINF_WIN");
+    g_win_mode = e ? atoi(e) : 1;
+  }
+  return g_win_mode;
+}
+void set_win_mode(int m) { g_win_mode = m; }
+
+static bool win_ok(const ConvGeom& g) {
+  return win_mode() > 0 && g.KH == 3 && g.KW == 3 && g.stride == 1 && g.pad == 1 && g.Cin % 64 == 0 &&
+         g.Cout % 64 == 0 && g.W <= 56 && g.H == g.Ho && g.W == g.Wo;
+}
+
+template <int BN>
+static void launch_win_t(const WinArgs& w, long long max_tiles, cudaStream_t st) {
+  using Cfg = WinCfg<BN>;
+  static bool attr = false;
+  if (!attr) {
+    CK(cudaFuncSetAttribute(conv_win_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
+    attr = true;
+  }
+  dim3 grid((unsigned)std::max(1LL, std::min<long long>(max_tiles, num_sms())));
+  ProfScope ps(w.dgrad ? PC_CONV_DGRAD : PC_CONV_FWD, st);
+  conv_win_kernel<BN><<<grid, NUM_THREADS, Cfg::SMEM, st>>>(w);
+  CK(cudaGetLastError());
+}
+
+static void launch_win(WinArgs& w, int nstatic, int nout, cudaStream_t st) {
+  const int BN = nout >= 256 ? 256 : (nout >= 128 ? 128 : 64);
+  const long long Q = (long long)nstatic * (w.c.Hs + 1) * (w.c.Ws + 1);
+  const long long tiles = ((Q + BM - 1) / BM) * ((nout + BN - 1) / BN);
+  w.base_off = 0;  // the 128B swizzle follows absolute smem address bits: no phase in the descriptor
+  switch (BN) {
+    case 64: launch_win_t<64>(w, tiles, st); break;
+    case 128: launch_win_t<128>(w, tiles, st); break;
+    default: launch_win_t<256>(w, tiles, st); break;
+  }
+}
+
 static int pick_bn(int nout, bool mn_major_b) {
   if (nout <= 32 && !mn_major_b) return 32;
   if (nout <= 64) return 64;
@@ -91,6 +136,19 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
   a.res = res;
   a.res_map = res_map;
   a.act = act;
+  if (n_static <= 0) return;
+  if (win_ok(g) && !out_f32 && win_mode() >= 2) {  // measured slower than the gather kernel for FWD (r1)
+    WinArgs w{};
+    w.c = a;
+    w.dgrad = 0;
+    for (int kh = 0; kh < 3; ++kh)
+      for (int kw = 0; kw < 3; ++kw) {
+        w.tap_off[kh * 3 + kw] = kh * (g.W + 1) + kw;
+        w.btap[kh * 3 + kw] = kh * 3 + kw;
+      }
+    launch_win(w, n_static, g.Cout, st);
+    return;
+  }
   const int BN = pick_bn(g.Cout, false);
   const long long mt = ((long long)n_static * g.Ho * g.Wo + BM - 1) / BM;
   if (mt == 0) return;
@@ -100,6 +158,33 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
 void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n, const float* bcast,
                 const bf16* sc, const bf16* yact, int mask_act, bf16* dx, cudaStream_t st) {
   // dX[y] = sum_{kh: (y + pad - kh) % s == 0} dZ[(y + pad - kh)/s] W[kh]; split by output phase (py,px)
+  if (win_ok(g) && (g.H <= 14 || win_mode() >= 2)) {  // stride 1: one window launch with flipped taps (faster at H<=14)
+    WinArgs wa{};
+    ConvArgs& a = wa.c;
+    a.src = dz;
+    a.Hs = g.Ho;
+    a.Ws = g.Wo;
+    a.Cs = g.Cout;
+    a.n_static = n;
+    a.B = w;
+    a.ldb = ldb;
+    a.Nout = g.Cin;
+    a.out = dx;
+    a.Ho = g.H;
+    a.Wo = g.W;
+    a.bcast = bcast;
+    a.sc = sc;
+    a.yact = yact;
+    a.mask_act = mask_act;
+    wa.dgrad = 1;
+    for (int kh = 0; kh < 3; ++kh)
+      for (int kw = 0; kw < 3; ++kw) {
+        wa.tap_off[kh * 3 + kw] = (2 - kh) * (g.W + 1) + (2 - kw);
+        wa.btap[kh * 3 + kw] = kh * 3 + kw;
+      }
+    launch_win(wa, n, g.Cin, st);
+    return;
+  }
   const int s = g.stride;
   for (int py = 0; py < s; ++py)
     for (int px = 0; px < s; ++px) {

@@ -135,12 +135,81 @@ __global__ void maxpool_bwd_kernel(const bf16* __restrict__ dT, const uint8_t* _
     *(uint4*)(dz + xi) = *(uint4*)o;
   }
 }
+// stride-2 fast path: one thread per (n, 2x2 input block, 8-channel vector); each window touching the
+// block is read once (argmax + dT, 128-bit), its gradient routed to the block element it selected; the
+// per-element window order is the same as the gather kernel's (ho, then wo ascending)
+__global__ void maxpool_bwd_s2_kernel(const bf16* __restrict__ dT, const uint8_t* __restrict__ amax,
+                                      const bf16* __restrict__ yact, int act, long long n, int H, int W, int C, int K,
+                                      int p, int Ho, int Wo, bf16* __restrict__ dz) {
+  const int CV = C / 8;
+  const int BH = (H + 1) / 2, BW = (W + 1) / 2;
+  const long long total = n * BH * BW * CV;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+    const int cv = (int)(i % CV);
+    long long r = i / CV;
+    const int bj = (int)(r % BW);
+    r /= BW;
+    const int bi = (int)(r % BH);
+    const long long b = r / BH;
+    const int ih0 = 2 * bi, iw0 = 2 * bj;
+    float acc[2][2][8];
+#pragma unroll
+    for (int u = 0; u < 2; ++u)
+#pragma unroll
+      for (int v = 0; v < 2; ++v)
+#pragma unroll
+        for (int q = 0; q < 8; ++q) acc[u][v][q] = 0.f;
+    const int ho_lo = max(0, (ih0 + p - K + 2) / 2), ho_hi = min(Ho - 1, (ih0 + 1 + p) / 2);
+    const int wo_lo = max(0, (iw0 + p - K + 2) / 2), wo_hi = min(Wo - 1, (iw0 + 1 + p) / 2);
+    for (int ho = ho_lo; ho <= ho_hi; ++ho)
+      for (int wo = wo_lo; wo <= wo_hi; ++wo) {
+        const long long oi = ((b * Ho + ho) * Wo + wo) * C + cv * 8;
+        const uint2 am = __ldg((const uint2*)(amax + oi));
+        const uint8_t* a8 = (const uint8_t*)&am;
+        const uint4 dv = __ldg((const uint4*)(dT + oi));
+        const bf16* d8 = (const bf16*)&dv;
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+          const int kh = a8[q] / K, kw = a8[q] - (a8[q] / K) * K;
+          const int u = ho * 2 - p + kh - ih0, v = wo * 2 - p + kw - iw0;
+          const float g = __bfloat162float(d8[q]);
+#pragma unroll
+          for (int uu = 0; uu < 2; ++uu)
+#pragma unroll
+            for (int vv = 0; vv < 2; ++vv)
+              if (u == uu && v == vv) acc[uu][vv][q] = __fadd_rn(acc[uu][vv][q], g);
+        }
+      }
+#pragma unroll
+    for (int u = 0; u < 2; ++u)
+#pragma unroll
+      for (int v = 0; v < 2; ++v) {
+        const int ih = ih0 + u, iw = iw0 + v;
+        if (ih >= H || iw >= W) continue;
+        const long long xi = ((b * H + ih) * W + iw) * C + cv * 8;
+        const uint4 yv = __ldg((const uint4*)(yact + xi));
+        const bf16* y8 = (const bf16*)&yv;
+        __align__(16) bf16 o[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+          o[q] = __float2bfloat16_rn(__fmul_rn(acc[u][v][q], act_grad(act, __bfloat162float(y8[q]))));
+        *(uint4*)(dz + xi) = *(uint4*)o;
+      }
+  }
+}
+
 void launch_maxpool_bwd(const bf16* dT, const uint8_t* amax, const bf16* yact, int act, int n, int H, int W, int C,
                         int K, int s, int p, int Ho, int Wo, bf16* dz, cudaStream_t st) {
-  const long long total = (long long)n * H * W * (C / 8);
-  const int blocks = (int)std::min<long long>((total + 255) / 256, 64LL * num_sms());
   ProfScope ps(PC_POOL_BWD, st);
-  maxpool_bwd_kernel<<<blocks, 256, 0, st>>>(dT, amax, yact, act, n, H, W, C, K, s, p, Ho, Wo, dz);
+  if (s == 2) {
+    const long long total = (long long)n * ((H + 1) / 2) * ((W + 1) / 2) * (C / 8);
+    const int blocks = (int)std::min<long long>((total + 255) / 256, 64LL * num_sms());
+    maxpool_bwd_s2_kernel<<<blocks, 256, 0, st>>>(dT, amax, yact, act, n, H, W, C, K, p, Ho, Wo, dz);
+  } else {
+    const long long total = (long long)n * H * W * (C / 8);
+    const int blocks = (int)std::min<long long>((total + 255) / 256, 64LL * num_sms());
+    maxpool_bwd_kernel<<<blocks, 256, 0, st>>>(dT, amax, yact, act, n, H, W, C, K, s, p, Ho, Wo, dz);
+  }
   CK(cudaGetLastError());
 }
 
@@ -319,19 +388,40 @@ void launch_exit_loss(const float* logits, const int32_t* labels, int n, int ncl
   CK(cudaGetLastError());
 }
 
+// dW[c][k] = sum_n pooled[n][c] dl[n][k] (+ db): one CTA per 32-channel slab, threads over (n-slice, c),
+// fixed-order partials in smem -> deterministic
 __global__ void head_dw_kernel(const float* __restrict__ pooled, const float* __restrict__ dl, int n, int C, int ncls,
                                float* __restrict__ dW, float* __restrict__ db) {
-  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx < C * ncls) {
-    const int c = idx / ncls, k = idx - c * ncls;
-    float acc = 0.f;
-    for (int i = 0; i < n; ++i) acc = fmaf(pooled[(long long)i * C + c], dl[(long long)i * ncls + k], acc);
-    dW[idx] = acc;
-  } else if (idx < C * ncls + ncls) {
-    const int k = idx - C * ncls;
-    float acc = 0.f;
-    for (int i = 0; i < n; ++i) acc += dl[(long long)i * ncls + k];
-    db[k] = acc;
+  __shared__ float part[8][32][33];
+  const int c = blockIdx.x * 32 + (threadIdx.x & 31);
+  const int sl = threadIdx.x >> 5;  // 8 n-slices
+  const bool bias_blk = blockIdx.x == (C + 31) / 32;
+  for (int k0 = 0; k0 < ncls; k0 += 32) {
+    float acc[32];
+#pragma unroll
+    for (int k = 0; k < 32; ++k) acc[k] = 0.f;
+    for (int i = sl; i < n; i += 8) {
+      const float pv = bias_blk ? 1.f : (c < C ? pooled[(long long)i * C + c] : 0.f);
+      const float* d = dl + (long long)i * ncls + k0;
+#pragma unroll
+      for (int k = 0; k < 32; ++k)
+        if (k0 + k < ncls) acc[k] = fmaf(pv, __ldg(d + k), acc[k]);
+    }
+#pragma unroll
+    for (int k = 0; k < 32; ++k) part[sl][threadIdx.x & 31][k] = acc[k];
+    __syncthreads();
+    if (sl == 0) {
+      for (int k = 0; k < 32 && k0 + k < ncls; ++k) {
+        float s = 0.f;
+        for (int q = 0; q < 8; ++q) s += part[q][threadIdx.x & 31][k];
+        if (bias_blk) {
+          if ((threadIdx.x & 31) == 0) db[k0 + k] = s;
+        } else if (c < C) {
+          dW[(long long)c * ncls + k0 + k] = s;
+        }
+      }
+    }
+    __syncthreads();
   }
 }
 __global__ void head_bcast_kernel(const float* __restrict__ dl, const float* __restrict__ Wk, int n, int C, int ncls,
@@ -346,9 +436,8 @@ __global__ void head_bcast_kernel(const float* __restrict__ dl, const float* __r
 }
 void launch_head_grads(const float* pooled, const float* dl, const float* Wk, int n, int C, int ncls, int HW,
                        float* dW, float* db, float* bcast, cudaStream_t st) {
-  const int tot = C * ncls + ncls;
   ProfScope ps(PC_HEAD_GRADS, st, 2);
-  head_dw_kernel<<<(tot + 127) / 128, 128, 0, st>>>(pooled, dl, n, C, ncls, dW, db);
+  head_dw_kernel<<<(C + 31) / 32 + 1, 256, 0, st>>>(pooled, dl, n, C, ncls, dW, db);
   const long long nb = ((long long)n * C + 255) / 256;
   head_bcast_kernel<<<(unsigned)nb, 256, 0, st>>>(dl, Wk, n, C, ncls, 1.0f / (float)HW, bcast);
   CK(cudaGetLastError());

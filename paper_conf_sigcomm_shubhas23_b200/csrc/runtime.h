@@ -26,6 +26,8 @@ struct ShapeError : std::runtime_error {
   } while (0)
 
 int num_sms();
+int win_mode();
+void set_win_mode(int m);  // 0 off, 1 window kernel (base offset 0), 2 window kernel (base-offset phase)
 
 // conv geometry (Cin = padded input channels as stored, multiple of 8)
 struct ConvGeom {

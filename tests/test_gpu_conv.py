@@ -128,3 +128,33 @@ def test_conv_wgrad_vs_torch(case):
     # deterministic: same bits on a second run
     dw2, db2 = B.dbg_conv_wgrad(x, dz, K, K, s, p)
     assert torch.equal(dw, dw2) and torch.equal(db, db2)
+
+
+WIN_CASES = [(2, 14, 14, 64, 64), (3, 7, 7, 128, 256), (2, 28, 28, 64, 128), (1, 56, 56, 64, 64), (5, 9, 11, 64, 64)]
+
+
+@pytest.mark.parametrize("mode", [2])
+@pytest.mark.parametrize("case", WIN_CASES)
+def test_window_kernel_fwd_dgrad(case, mode):
+    """Window implicit GEMM (stride-1 3x3) vs torch: tap A operands are row-shifted views of one window
+    (mode 2 forces the window kernel for every eligible fwd/dgrad shape; the default routes by size)."""
+    n, H, W, C, Co = case
+    B.dbg_set_win_mode(mode)
+    try:
+        x, w, b = _mk((n, H, W, C, Co, 3, 1, 1), 11)
+        res = torch.randn(n, H, W, Co).to(torch.bfloat16).cuda()
+        ref = torch.relu(_ref_fwd(x, w, b, 1, 1) + res.float())
+        out = B.dbg_conv_fwd(x, w, b, 1, 1, act=1, res=res)
+        torch.cuda.synchronize()
+        assert _rel(out.float(), ref) < 8e-3, ("fwd", mode)
+        dz = torch.randn(n, H, W, Co).to(torch.bfloat16).cuda()
+        y = torch.randn(n, H, W, C).to(torch.bfloat16).cuda()
+        bc = torch.randn(n, C).cuda() * 0.01
+        refd = torch.nn.grad.conv2d_input((n, C, H, W), w.float().permute(0, 3, 1, 2), dz.float().permute(0, 3, 1, 2),
+                                          stride=1, padding=1).permute(0, 2, 3, 1)
+        refd = (refd + bc[:, None, None, :]) * (y.float() > 0)
+        dx = B.dbg_conv_dgrad(dz, w, H, W, 1, 1, bcast=bc, yact=y, mask_act=1)
+        torch.cuda.synchronize()
+        assert _rel(dx.float(), refd) < 8e-3, ("dgrad", mode)
+    finally:
+        B.dbg_set_win_mode(1)

@@ -1,0 +1,26 @@
+"""Time single conv launches (fwd/dgrad/wgrad) with CUDA events at ResNet-18 training shapes."""
+import sys, os
+sys.path.insert(0, os.path.join(os.path.dirname(os.path.abspath(__file__)), ".."))
+import torch
+from paper_conf_sigcomm_shubhas23_b200 import binding as B
+n = int(os.environ.get("N", "1024"))
+modes = [int(m) for m in os.environ.get("MODES", "0,1").split(",")]
+shapes = [(56, 64, 64), (28, 128, 128), (14, 256, 256), (7, 512, 512)]
+for (H, C, Co) in shapes:
+    x = torch.randn(n, H, H, C, device="cuda").to(torch.bfloat16)
+    w = (torch.randn(Co, 3, 3, C, device="cuda") * 0.05).to(torch.bfloat16)
+    b = torch.zeros(Co, device="cuda")
+    dz = torch.randn(n, H, H, Co, device="cuda").to(torch.bfloat16)
+    fl = 2 * n * H * H * Co * 9 * C
+    for m in modes:
+        B.dbg_set_win_mode(m)
+        for name, fn in [("fwd", lambda: B.dbg_conv_fwd(x, w, b, 1, 1, act=1)),
+                         ("dgrad", lambda: B.dbg_conv_dgrad(dz, w, H, H, 1, 1))]:
+            fn(); torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            for _ in range(5): fn()
+            e1.record(); torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1) / 5
+            print(f"H={H:3d} C={C:3d} mode={m} {name:6s} {ms*1e3:8.1f} us {fl/ms/1e9:7.1f} TFLOP/s", flush=True)
+B.dbg_set_win_mode(1)
