@@ -27,11 +27,21 @@ extern "C" adainf_status adainf_dbg_conv_fwd(const void* x, int32_t n, int32_t H
                                              int32_t stride, int32_t pad, int32_t act, const void* res, void* out,
                                              int32_t out_f32, adainf_stream_t stream) {
   return guard([&] {
-    if (C % 8 || n <= 0 || KH * KW > 49) throw ShapeError("conv_fwd: C must be a multiple of 8");
+    if ((C % 8 && C != 4) || n <= 0 || KH * KW > 49) throw ShapeError("conv_fwd: C must be 4 or a multiple of 8");
     require_device();
     ConvGeom g = geom(H, W, C, Co, KH, KW, stride, pad);
-    conv_fwd(g, (const bf16*)x, nullptr, nullptr, n, (const bf16*)w, KH * KW * C, b, (const bf16*)res, nullptr,
-             act, out, out_f32 != 0, (cudaStream_t)stream);
+    const int K = KH * KW * C, ldb = (K + 7) / 8 * 8;  // GEMM-ready rows are 16-byte aligned
+    const bf16* wp = (const bf16*)w;
+    bf16* tmp = nullptr;
+    cudaStream_t st = (cudaStream_t)stream;
+    if (ldb != K) {
+      CK(cudaMallocAsync((void**)&tmp, (size_t)Co * ldb * 2, st));
+      CK(cudaMemsetAsync(tmp, 0, (size_t)Co * ldb * 2, st));
+      CK(cudaMemcpy2DAsync(tmp, ldb * 2, w, K * 2, K * 2, Co, cudaMemcpyDeviceToDevice, st));
+      wp = tmp;
+    }
+    conv_fwd(g, (const bf16*)x, nullptr, nullptr, n, wp, ldb, b, (const bf16*)res, nullptr, act, out, out_f32 != 0, st);
+    if (tmp) CK(cudaFreeAsync(tmp, st));
   });
 }
 
@@ -52,7 +62,7 @@ extern "C" adainf_status adainf_dbg_conv_wgrad(const void* x, const void* dz, in
                                                int32_t C, int32_t Co, int32_t KH, int32_t KW, int32_t stride,
                                                int32_t pad, float* dw, float* db, adainf_stream_t stream) {
   return guard([&] {
-    if (C % 8 || Co % 8 || n <= 0) throw ShapeError("conv_wgrad: C, Co must be multiples of 8");
+    if ((C % 8 && C != 4) || Co % 8 || n <= 0) throw ShapeError("conv_wgrad: C must be 4 or a multiple of 8, Co of 8");
     require_device();
     ConvGeom g = geom(H, W, C, Co, KH, KW, stride, pad);
     const size_t ws = wgrad_ws_bytes(g, n);

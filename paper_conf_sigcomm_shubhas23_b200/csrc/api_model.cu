@@ -167,7 +167,7 @@ extern "C" adainf_status adainf_app_create(const adainf_app_spec* spec, adainf_a
       for (size_t e = 0; e < a.edges.size(); ++e)
         if (a.edges[e].kind == ADAINF_ROUTE_DET_CROP) {
           Model* dst = a.models[a.edges[e].dst_model];
-          I.routed_in[e].alloc((size_t)a.max_routed * dst->in_h * dst->in_w * dst->cin_pad * 2);
+          I.routed_in[e].alloc((size_t)a.max_routed * dst->in_h * dst->in_w * dst->in_c * 2);
         }
       I.route_list.alloc((size_t)std::max<size_t>(1, a.edges.size()) * std::max(1, a.max_routed) * 4);
       I.route_cnt.alloc((size_t)std::max<size_t>(1, a.edges.size()) * 4 + 16);
@@ -253,8 +253,7 @@ extern "C" adainf_status adainf_infer_dag(adainf_app_t app, const void* batch, i
         rows = a.max_routed;
         cnt = I.route_cnt.as<int>() + e;
         if (ed.kind == ADAINF_ROUTE_DET_CROP) {
-          x = I.routed_in[e].as<bf16>();
-          padded = true;
+          x = I.routed_in[e].as<bf16>();  // crops in the destination's own input layout (ingested like a batch)
         } else {
           // whole-input routing: read the source model's own input rows through the route list
           if (ed.src_model != 0) throw UnsupportedError("CLASS_WHOLE routing from a routed model");
@@ -294,7 +293,7 @@ extern "C" adainf_status adainf_infer_dag(adainf_app_t app, const void* batch, i
           Model* dst = a.models[a.edges[e].dst_model];
           CK(cudaMemcpyAsync(I.route_cnt.as<int>() + e, S.cnt_clamped.as<int>() + q, 4, cudaMemcpyDeviceToDevice, st));
           launch_crops(x, m->in_h, m->in_w, m->in_c, S.det_table.as<float>(), S.route_idx.as<int32_t>(),
-                       S.cnt_clamped.as<int32_t>(), q, d.cap, a.edges[e].crop_h, a.edges[e].crop_w, dst->cin_pad,
+                       S.cnt_clamped.as<int32_t>(), q, d.cap, a.edges[e].crop_h, a.edges[e].crop_w, dst->in_c,
                        I.routed_in[e].as<bf16>(), st);
         }
         if (o.route_idx && d.n_edges)

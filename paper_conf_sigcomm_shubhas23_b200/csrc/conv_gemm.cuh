@@ -209,17 +209,35 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
           const uint32_t sa = smem_base + s * Cfg::STAGE_BYTES;
           const uint32_t sb = sa + Cfg::A_BYTES;
           const int k = (ti.kb0 + kbi) * BK + j * 8;
-          const int tap = k / a.Cs;
-          const int c = k - tap * a.Cs;
-          const bool kval = k < a.K;
-          const int dy = kval ? a.ty[tap] : -100000, dx = kval ? a.tx[tap] : 0;
+          if (a.Cs == 4) {
+            // 4-channel (8-byte) pixels: each 16-byte chunk = taps t0, t0+1 -> two 8-byte cp.async
+            const int t0 = k >> 2;
+            const bool k0 = t0 < a.ntaps, k1 = t0 + 1 < a.ntaps;
+            const int dy0 = k0 ? a.ty[t0] : -100000, dx0 = k0 ? a.tx[t0] : 0;
+            const int dy1 = k1 ? a.ty[t0 + 1] : -100000, dx1 = k1 ? a.tx[t0 + 1] : 0;
 #pragma unroll
-          for (int i = 0; i < 8; ++i) {
-            const int r = (t >> 3) + 16 * i;
-            const int iy = iy0[i] + dy, ix = ix0[i] + dx;
-            const bool v = (unsigned)iy < (unsigned)a.Hs && (unsigned)ix < (unsigned)a.Ws;
-            const bf16* g = v ? a.src + ((rowbase[i] + (long long)iy * a.Ws + ix) * a.Cs + c) : a.src;
-            cp_async16(sa + kmaj_off(r, j), g, v);
+            for (int i = 0; i < 8; ++i) {
+              const int r = (t >> 3) + 16 * i;
+              const int iya = iy0[i] + dy0, ixa = ix0[i] + dx0, iyb = iy0[i] + dy1, ixb = ix0[i] + dx1;
+              const bool va = (unsigned)iya < (unsigned)a.Hs && (unsigned)ixa < (unsigned)a.Ws;
+              const bool vb = (unsigned)iyb < (unsigned)a.Hs && (unsigned)ixb < (unsigned)a.Ws;
+              const uint32_t d = sa + kmaj_off(r, j);
+              cp_async8(d, va ? a.src + ((rowbase[i] + (long long)iya * a.Ws + ixa) << 2) : a.src, va);
+              cp_async8(d + 8, vb ? a.src + ((rowbase[i] + (long long)iyb * a.Ws + ixb) << 2) : a.src, vb);
+            }
+          } else {
+            const int tap = k / a.Cs;
+            const int c = k - tap * a.Cs;
+            const bool kval = k < a.K;
+            const int dy = kval ? a.ty[tap] : -100000, dx = kval ? a.tx[tap] : 0;
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              const int r = (t >> 3) + 16 * i;
+              const int iy = iy0[i] + dy, ix = ix0[i] + dx;
+              const bool v = (unsigned)iy < (unsigned)a.Hs && (unsigned)ix < (unsigned)a.Ws;
+              const bf16* g = v ? a.src + ((rowbase[i] + (long long)iy * a.Ws + ix) * a.Cs + c) : a.src;
+              cp_async16(sa + kmaj_off(r, j), g, v);
+            }
           }
           if (MODE == MODE_FWD) {
             // W [Nout][ldb] K-major: BN rows x 8 chunks
@@ -267,7 +285,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
         // per K-block), kconv chunks j = (t&1)*8 .. +8 (taps / channels fixed per tile)
         const int r = t >> 1;
         const int j0 = (t & 1) * 8;
-        int dyj[8], dxj[8], cj[8];
+        const bool c4 = a.Cs == 4;  // 4-channel input: each 8-kconv chunk = two taps (8-byte halves)
+        int dyj[8], dxj[8], cj[8], dyk[8], dxk[8];
 #pragma unroll
         for (int q = 0; q < 8; ++q) {
           const int kc = (int)ti.m0 + (j0 + q) * 8;
@@ -276,6 +295,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
           cj[q] = kc - tap * a.Cs;
           dyj[q] = mval ? a.ty[tap] : -100000;
           dxj[q] = a.tx[tap];
+          const bool m1 = c4 && tap + 1 < a.ntaps && mval;
+          dyk[q] = m1 ? a.ty[tap + 1] : -100000;
+          dxk[q] = m1 ? a.tx[tap + 1] : 0;
         }
         for (int kbi = 0; kbi < nkb; ++kbi, ++it) {
           const int s = it % STAGES, u = it / STAGES;
@@ -295,12 +317,24 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
             gx0 *= a.sx;
             base = (long long)(a.src_map ? __ldg(a.src_map + n) : n) * a.Hs * a.Ws;
           }
+          if (c4) {
 #pragma unroll
-          for (int q = 0; q < 8; ++q) {
-            const int iy = gy0 + dyj[q], ix = gx0 + dxj[q];
-            const bool v = (unsigned)iy < (unsigned)a.Hs && (unsigned)ix < (unsigned)a.Ws;
-            const bf16* g = v ? a.src + ((base + (long long)iy * a.Ws + ix) * a.Cs + cj[q]) : a.src;
-            cp_async16(sa + mnmaj_off(r, j0 + q), g, v);
+            for (int q = 0; q < 8; ++q) {
+              const int iya = gy0 + dyj[q], ixa = gx0 + dxj[q], iyb = gy0 + dyk[q], ixb = gx0 + dxk[q];
+              const bool va = (unsigned)iya < (unsigned)a.Hs && (unsigned)ixa < (unsigned)a.Ws;
+              const bool vb = (unsigned)iyb < (unsigned)a.Hs && (unsigned)ixb < (unsigned)a.Ws;
+              const uint32_t d = sa + mnmaj_off(r, j0 + q);
+              cp_async8(d, va ? a.src + ((base + (long long)iya * a.Ws + ixa) << 2) : a.src, va);
+              cp_async8(d + 8, vb ? a.src + ((base + (long long)iyb * a.Ws + ixb) << 2) : a.src, vb);
+            }
+          } else {
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+              const int iy = gy0 + dyj[q], ix = gx0 + dxj[q];
+              const bool v = (unsigned)iy < (unsigned)a.Hs && (unsigned)ix < (unsigned)a.Ws;
+              const bf16* g = v ? a.src + ((base + (long long)iy * a.Ws + ix) * a.Cs + cj[q]) : a.src;
+              cp_async16(sa + mnmaj_off(r, j0 + q), g, v);
+            }
           }
           // B: dZ [pix][Nout] MN-major [64 pixels][BN co]
           constexpr int CH = BN / 8;

@@ -19,7 +19,14 @@ __global__ void pack_input_kernel(const bf16* __restrict__ x, const int* __restr
     const long long n = i / HW, pix = i - n * HW;
     const long long src = (map ? map[n] : n) * (long long)HW + pix;
     bf16* o = y + i * Cpad;
-    for (int c = 0; c < Cpad; ++c) o[c] = c < Cin ? x[src * Cin + c] : __float2bfloat16_rn(0.f);
+    if (Cpad == 4) {
+      __align__(8) bf16 v[4];
+#pragma unroll
+      for (int c = 0; c < 4; ++c) v[c] = c < Cin ? x[src * Cin + c] : __float2bfloat16_rn(0.f);
+      *(uint2*)o = *(uint2*)v;
+    } else {
+      for (int c = 0; c < Cpad; ++c) o[c] = c < Cin ? x[src * Cin + c] : __float2bfloat16_rn(0.f);
+    }
   }
 }
 void launch_pack_input(const bf16* x, const int* map, const int* count, int n_static, int H, int W, int Cin, int Cpad,

@@ -39,7 +39,9 @@ void Model::build(const adainf_model_spec& s) {
   in_w = s.in_w;
   in_c = s.in_c;
   max_batch = s.max_batch;
-  cin_pad = pad8(in_c);
+  // few-channel inputs (images 3, spectrograms 1) are padded to 4 channels (8-byte pixels) and gathered
+  // by the conv producers with 8-byte cp.async (one tap per half chunk); others to a multiple of 8
+  cin_pad = in_c <= 4 ? 4 : pad8(in_c);
   pack = cin_pad != in_c;
   momentum = s.momentum;
   weight_decay = s.weight_decay;
@@ -96,7 +98,7 @@ void Model::build(const adainf_model_spec& s) {
       off += (long long)o.cout * KH * KW * nd.cin_real;
       nd.b_off = off;
       off += o.cout;
-      nd.ldb = KH * KW * X.C;
+      nd.ldb = pad8(KH * KW * X.C);  // 16-byte aligned shadow rows (4-channel stems: 49*4 -> 200)
       nd.fp32_out = !proj && (i + 1 < ops.size() && ops[i + 1].kind == ADAINF_OP_DET_HEAD);
       TensorRt Y;
       Y.H = nd.g.Ho;
@@ -218,7 +220,7 @@ void Model::build(const adainf_model_spec& s) {
     T[t].buf = T[t].own.as<bf16>();
   }
   if (pack) {
-    packed_in.alloc((size_t)max_batch * in_h * in_w * cin_pad * 2);
+    packed_in.alloc((size_t)max_batch * T[0].row_elems() * 2);
     T[0].buf = packed_in.as<bf16>();
   }
   for (auto& nd : nodes)
@@ -313,6 +315,11 @@ void Model::build(const adainf_model_spec& s) {
   CK(cudaMemcpy(params.p, host.data(), nparams * 4, cudaMemcpyHostToDevice));
   refresh_shadows(0);
   CK(cudaDeviceSynchronize());
+}
+
+// a1 ingest: channel padding (to 4 for few-channel inputs, else to a multiple of 8)
+void Model::ingest(const bf16* x, const int* map, const int* count, int n_static, cudaStream_t st) {
+  launch_pack_input(x, map, count, n_static, in_h, in_w, in_c, cin_pad, packed_in.as<bf16>(), st);
 }
 
 void Model::refresh_shadows(cudaStream_t st) {
@@ -441,7 +448,7 @@ void Model::infer(const bf16* x, const int* in_map, const int* in_count, int n_s
   const bf16* x0 = x;
   const int* map0 = in_map;
   if (pack && !x_padded) {
-    launch_pack_input(x, in_map, in_count, n_static, in_h, in_w, in_c, cin_pad, packed_in.as<bf16>(), st);
+    ingest(x, in_map, in_count, n_static, st);
     x0 = packed_in.as<bf16>();
     map0 = nullptr;
   }
@@ -463,7 +470,7 @@ void Model::train_step(const bf16* x, const int32_t* labels, int n, long long n_
   ensure_training();
   const bf16* x0 = x;
   if (pack) {
-    launch_pack_input(x, nullptr, nullptr, n, in_h, in_w, in_c, cin_pad, packed_in.as<bf16>(), st);
+    ingest(x, nullptr, nullptr, n, st);
     x0 = packed_in.as<bf16>();
   }
   forward_nodes(x0, nullptr, nullptr, n, true, nullptr, nullptr, st);

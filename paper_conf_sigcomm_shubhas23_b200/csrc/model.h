@@ -111,6 +111,7 @@ struct Model {
 
   void build(const adainf_model_spec& s);
   void refresh_shadows(cudaStream_t st);
+  void ingest(const bf16* x, const int* map, const int* count, int n_static, cudaStream_t st);
   void ensure_training();
   // inference of one (possibly routed / device-counted) batch
   void infer(const bf16* x, const int* in_map, const int* in_count, int n_static, const float* taus,
