@@ -57,6 +57,7 @@ struct ConvArgs {
   int mask_act;         // DGRAD: activation whose derivative masks (0 = none)
   int kb_per_split;     // WGRAD split-K (in 64-pixel blocks)
   int splits;           // WGRAD number of splits
+  int exp_flags;        // experiments only (ADAINF_EXP): bit0 skip epilogue stores, bit1 skip bias/res loads
 };
 
 constexpr int BM = 128, BK = 64;
@@ -448,12 +449,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
             mbar_arrive(&tempty[b]);  // accumulator free for the tile after next
           }
           const int cb = ti.n0 + c0;
-          if (!rv || cb >= a.Nout) continue;
+          if (!rv || cb >= a.Nout || (a.exp_flags & 1)) continue;
           const bool vec = (cb + 32 <= a.Nout) && ((a.Nout & 7) == 0);
           if (MODE == MODE_FWD) {
             if (vec) {
 #pragma unroll
-              for (int i = 0; i < 32; ++i) v[i] = __fadd_rn(v[i], __ldg(a.bias + cb + i));  // flat params: 4B-aligned
+              if (!(a.exp_flags & 2))
+                for (int i = 0; i < 32; ++i) v[i] = __fadd_rn(v[i], __ldg(a.bias + cb + i));  // flat params: 4B-aligned
               if (a.res) {
 #pragma unroll
                 for (int i = 0; i < 32; i += 8) {

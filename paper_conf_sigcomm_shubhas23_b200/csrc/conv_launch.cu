@@ -83,6 +83,20 @@ static void launch_win_t(const WinArgs& w, long long max_tiles, cudaStream_t st)
 }
 
 static void launch_win(WinArgs& w, int nstatic, int nout, cudaStream_t st) {
+  if (w.c.Cs == 64 && nout == 64) {  // weight-stationary 64x64 variant (ResNet layer1)
+    static bool attr = false;
+    if (!attr) {
+      CK(cudaFuncSetAttribute(conv_win_ws_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, WinWsCfg::SMEM));
+      attr = true;
+    }
+    const long long Q = (long long)nstatic * (w.c.Hs + 1) * (w.c.Ws + 1);
+    const long long tiles = (Q + BM - 1) / BM;
+    dim3 grid((unsigned)std::max(1LL, std::min<long long>(tiles, num_sms())));
+    ProfScope ps(w.dgrad ? PC_CONV_DGRAD : PC_CONV_FWD, st);
+    conv_win_ws_kernel<<<grid, WS_THREADS, WinWsCfg::SMEM, st>>>(w);
+    CK(cudaGetLastError());
+    return;
+  }
   const int BN = nout >= 256 ? 256 : (nout >= 128 ? 128 : 64);
   const long long Q = (long long)nstatic * (w.c.Hs + 1) * (w.c.Ws + 1);
   const long long tiles = ((Q + BM - 1) / BM) * ((nout + BN - 1) / BN);
@@ -137,7 +151,8 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
   a.res_map = res_map;
   a.act = act;
   if (n_static <= 0) return;
-  if (win_ok(g) && !out_f32 && win_mode() >= 2) {  // measured slower than the gather kernel for FWD (r1)
+  if (win_ok(g) && !out_f32 && (win_mode() >= 2 || (g.Cin == 64 && g.Cout == 64))) {
+    // window kernel: weight-stationary 64x64 variant by default; the general window FWD measured slower
     WinArgs w{};
     w.c = a;
     w.dgrad = 0;
@@ -149,6 +164,14 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
     launch_win(w, n_static, g.Cout, st);
     return;
   }
+  {
+    static int expf = -1;
+    if (expf < 0) {
+      const char* e = getenv("ADAINF_EXP");
+      expf = e ? atoi(e) : 0;
+    }
+    a.exp_flags = expf;
+  }
   const int BN = pick_bn(g.Cout, false);
   const long long mt = ((long long)n_static * g.Ho * g.Wo + BM - 1) / BM;
   if (mt == 0) return;
@@ -158,7 +181,8 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
 void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n, const float* bcast,
                 const bf16* sc, const bf16* yact, int mask_act, bf16* dx, cudaStream_t st) {
   // dX[y] = sum_{kh: (y + pad - kh) % s == 0} dZ[(y + pad - kh)/s] W[kh]; split by output phase (py,px)
-  if (win_ok(g) && (g.H <= 14 || win_mode() >= 2)) {  // stride 1: one window launch with flipped taps (faster at H<=14)
+  if (win_ok(g) && (g.H <= 14 || win_mode() >= 2 || (g.Cin == 64 && g.Cout == 64))) {
+    // stride 1: one window launch with flipped taps (faster at H<=14; weight-stationary at 64x64)
     WinArgs wa{};
     ConvArgs& a = wa.c;
     a.src = dz;

@@ -310,3 +310,282 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_win_kernel(const WinArgs 
 }
 
 }  // namespace adainf
+
+namespace adainf {
+
+// ------------------------------------------------------------------------------------------------
+// Weight-stationary variant for 64-channel 3x3 layers (ResNet layer1: Cin = Cout = 64): all 9 tap tiles
+// of B (9 x 64 x 64 bf16 = 72 KB) are loaded into shared memory ONCE per persistent CTA, so the only
+// per-tile traffic is the input window (~31 KB at 56x56) instead of 9 im2col A tiles + 9 B tiles
+// (216 KB) in the gather kernel.
+struct WinWsCfg {
+  static constexpr int WIN_BYTES = ((WIN_MAX_L + 7) / 8) * 1024;
+  static constexpr int WSTAGES = 2;
+  static constexpr int B_BYTES = 64 * 64 * 2;
+  static constexpr int STAGE_E = 2 * 128 * 256;  // epilogue staging: 2 groups x 128 rows x (2 x 128 B)
+  static constexpr int SMEM = WSTAGES * WIN_BYTES + 9 * B_BYTES + STAGE_E + 1024 + 512;
+  static constexpr int ACC_COLS = 64;
+  static constexpr int TMEM_COLS = 128;
+};
+
+constexpr int WS_THREADS = 416;  // 4 producer warps, 1 MMA warp, 2 x 4 epilogue warps (alternate tiles)
+
+__global__ void __launch_bounds__(WS_THREADS, 1) conv_win_ws_kernel(const WinArgs w) {
+  using Cfg = WinWsCfg;
+  const ConvArgs& a = w.c;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* win_base = smem;
+  uint8_t* b_base = smem + Cfg::WSTAGES * Cfg::WIN_BYTES;
+  uint8_t* e_base = b_base + 9 * Cfg::B_BYTES;
+  uint64_t* bars = (uint64_t*)(e_base + Cfg::STAGE_E);
+  uint64_t* wfull = bars;
+  uint64_t* wempty = wfull + Cfg::WSTAGES;
+  uint64_t* bready = wempty + Cfg::WSTAGES;
+  uint64_t* tfull = bready + 1;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+  float* s_bias = (float*)(tmem_slot + 4);  // 64 floats (FWD bias, staged once per CTA)
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int H = a.Hs, W = a.Ws, Wp = W + 1, Hp = H + 1;
+  const int nsamp = a.count ? *a.count : a.n_static;
+  const int Qimg = Hp * Wp;
+  const long long Q = (long long)nsamp * Qimg;
+  const int ntile = (int)((Q + BM - 1) / BM);
+  const int L = BM + 2 * Wp + 2;
+  if ((int)blockIdx.x >= ntile) return;
+  if (threadIdx.x < 64) s_bias[threadIdx.x] = (!w.dgrad && a.bias) ? a.bias[threadIdx.x] : 0.f;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < Cfg::WSTAGES; ++s) {
+      mbar_init(&wfull[s], 128);
+      mbar_init(&wempty[s], 1);
+    }
+    mbar_init(bready, 128);
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 128);
+    }
+    fence_mbar_init();
+  }
+  if (warp == 4) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  const uint32_t wsm = smem_u32(win_base), bsm = smem_u32(b_base);
+
+  if (warp < 4) {
+    const int t = threadIdx.x;
+    const int j = t & 7;
+    // ---- resident B: 9 tap tiles ----
+    for (int tp = 0; tp < 9; ++tp) {
+      const uint32_t sb = bsm + tp * Cfg::B_BYTES;
+      if (!w.dgrad) {
+        const bf16* wb = a.B + (long long)w.btap[tp] * 64;
+#pragma unroll
+        for (int idx = t; idx < 64 * 8; idx += 128) {
+          const int r = idx >> 3, jj = idx & 7;
+          cp_async16(sb + kmaj_off(r, jj), wb + (long long)r * a.ldb + jj * 8, true);
+        }
+      } else {
+        const bf16* wb = a.B + (long long)w.btap[tp] * 64;
+#pragma unroll
+        for (int idx = t; idx < 64 * 8; idx += 128) {
+          const int r = idx >> 3, jj = idx & 7;
+          cp_async16(sb + mnmaj_off(r, jj), wb + (long long)r * a.ldb + jj * 8, true);
+        }
+      }
+    }
+    cp_async_arrive_noinc(bready);
+    // ---- windows ----
+    constexpr int RPT = (WIN_MAX_L + 15) / 16;
+    int wit = 0;
+    for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++wit) {
+      const long long q0 = (long long)tile * BM;
+      const int s = wit % Cfg::WSTAGES, u = wit / Cfg::WSTAGES;
+      // decode the first row of this thread once, then step by 16 rows with carries
+      long long qs = q0 - Wp - 1 + (t >> 3);
+      int n = 0, h = 0, x = 0;
+      if (qs >= 0) {
+        n = (int)(qs / Qimg);
+        const int rem = (int)(qs - (long long)n * Qimg);
+        h = rem / Wp;
+        x = rem - h * Wp;
+      }
+      if (u > 0) mbar_wait(&wempty[s], (u - 1) & 1);
+      const uint32_t sw = wsm + s * Cfg::WIN_BYTES;
+#pragma unroll
+      for (int i = 0; i < RPT; ++i) {
+        const int r = (t >> 3) + 16 * i;
+        if (r < L) {
+          const bool v = qs >= 0 && qs < Q && h < H && x < W;
+          const bf16* g = a.src;
+          if (v) {
+            const int sn = a.src_map ? __ldg(a.src_map + n) : n;
+            g = a.src + ((long long)((sn * H + h) * W + x) * 64 + j * 8);
+          }
+          cp_async16(sw + kmaj_off(r, j), g, v);
+        }
+        // advance 16 rows
+        qs += 16;
+        if (qs >= 0) {
+          if (qs < 16) {  // crossed from negative: decode afresh
+            n = 0;
+            h = (int)qs / Wp;
+            x = (int)qs - h * Wp;
+          } else {
+            x += 16;
+            while (x >= Wp) {  // Wp may be < 16 (small maps): possibly several carries
+              x -= Wp;
+              if (++h >= Hp) {
+                h = 0;
+                ++n;
+              }
+            }
+          }
+        }
+      }
+      cp_async_arrive_noinc(&wfull[s]);
+    }
+  } else if (warp == 4) {
+    const uint32_t IDESC = make_idesc(BM, 64, 0, w.dgrad ? 1 : 0);
+    mbar_wait(bready, 0);
+    int wit = 0;
+    for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++wit) {
+      const int b = wit & 1, ub = wit >> 1;
+      if (ub > 0) mbar_wait(&tempty[b], (ub - 1) & 1);
+      tc_fence_after();
+      const uint32_t dacc = tmem + (uint32_t)(b * Cfg::ACC_COLS);
+      const int s = wit % Cfg::WSTAGES, u = wit / Cfg::WSTAGES;
+      mbar_wait(&wfull[s], u & 1);
+      fence_proxy_async_smem();
+      tc_fence_after();
+      if (lane == 0) {
+        const uint32_t sw = wsm + s * Cfg::WIN_BYTES;
+#pragma unroll 1
+        for (int tp = 0; tp < 9; ++tp) {
+          const uint32_t sb = bsm + tp * Cfg::B_BYTES;
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk) {
+            const uint64_t ad = make_sdesc_rows(sw, w.tap_off[tp], kk, 0);
+            const uint64_t bd = w.dgrad ? make_sdesc(sb + kk * 2048, 8192, 1024) : make_sdesc(sb + kk * 32, 16, 1024);
+            umma_bf16(dacc, ad, bd, IDESC, (tp | kk) != 0);
+          }
+        }
+        umma_commit(&wempty[s]);
+        umma_commit(&tfull[b]);
+      }
+      __syncwarp();
+    }
+  } else {
+    const int grp = (warp - 5) >> 2;  // 0: even local tiles (accumulator 0), 1: odd (accumulator 1)
+    const int qd = warp & 3;
+    const int row = qd * 32 + lane;
+    int lt = grp;
+    for (int tile = blockIdx.x + grp * gridDim.x; tile < ntile; tile += 2 * gridDim.x, lt += 2) {
+      const long long q = (long long)tile * BM + row;
+      const int b = grp, ub = lt >> 1;
+      bool rv = q < Q;
+      int n = 0, h = 0, x = 0;
+      if (rv) {
+        n = (int)(q / Qimg);
+        const int rem = (int)(q - (long long)n * Qimg);
+        h = rem / Wp;
+        x = rem - h * Wp;
+        rv = h < H && x < W;
+      }
+      const long long orow = ((long long)n * H + h) * W + x;
+      long long rrow = orow;
+      if (!w.dgrad && a.res && rv) rrow = ((long long)(a.res_map ? __ldg(a.res_map + n) : n) * H + h) * W + x;
+      // stage this row's epilogue operands (residual / shortcut-gradient, stored activation) into shared
+      // memory with cp.async before waiting for the accumulator (hides the global-load latency)
+      const bf16* p0 = nullptr;
+      const bf16* p1 = nullptr;
+      if (rv) {
+        if (!w.dgrad) p0 = a.res ? a.res + rrow * 64 : nullptr;
+        else {
+          p0 = a.sc ? a.sc + orow * 64 : nullptr;
+          p1 = a.mask_act ? a.yact + orow * 64 : nullptr;
+        }
+      }
+      const uint32_t est = smem_u32(e_base) + (uint32_t)((grp * 128 + row) * 256);
+      if (p0)
+#pragma unroll
+        for (int i = 0; i < 8; ++i) cp_async16(est + i * 16, p0 + i * 8, true);
+      if (p1)
+#pragma unroll
+        for (int i = 0; i < 8; ++i) cp_async16(est + 128 + i * 16, p1 + i * 8, true);
+      asm volatile("cp.async.commit_group;" ::: "memory");
+      mbar_wait(&tfull[b], ub & 1);
+      tc_fence_after();
+      const uint32_t trow = tmem + (uint32_t)(b * Cfg::ACC_COLS) + ((uint32_t)(qd * 32) << 16);
+      float v[64];
+      tmem_ld32(trow, v);
+      tmem_ld32(trow + 32, v + 32);
+      tc_fence_before();
+      mbar_arrive(&tempty[b]);
+      asm volatile("cp.async.wait_all;" ::: "memory");
+      if (!rv) continue;
+      const uint8_t* es = e_base + (grp * 128 + row) * 256;
+      if (!w.dgrad) {
+#pragma unroll
+        for (int i = 0; i < 64; ++i) v[i] = __fadd_rn(v[i], s_bias[i]);
+        if (p0) {
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const uint4 e = *(const uint4*)(es + i * 16);
+            const bf16* hh = (const bf16*)&e;
+#pragma unroll
+            for (int qq = 0; qq < 8; ++qq) v[i * 8 + qq] = __fadd_rn(v[i * 8 + qq], __bfloat162float(hh[qq]));
+          }
+        }
+#pragma unroll
+        for (int i = 0; i < 64; ++i) v[i] = act_apply(a.act, v[i]);
+      } else {
+        if (a.bcast) {
+#pragma unroll
+          for (int i = 0; i < 64; i += 4) {
+            const float4 bb = __ldg((const float4*)(a.bcast + (long long)n * 64 + i));
+            v[i] = __fadd_rn(v[i], bb.x);
+            v[i + 1] = __fadd_rn(v[i + 1], bb.y);
+            v[i + 2] = __fadd_rn(v[i + 2], bb.z);
+            v[i + 3] = __fadd_rn(v[i + 3], bb.w);
+          }
+        }
+        if (p0) {
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const uint4 e = *(const uint4*)(es + i * 16);
+            const bf16* hh = (const bf16*)&e;
+#pragma unroll
+            for (int qq = 0; qq < 8; ++qq) v[i * 8 + qq] = __fadd_rn(v[i * 8 + qq], __bfloat162float(hh[qq]));
+          }
+        }
+        if (p1) {
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const uint4 e = *(const uint4*)(es + 128 + i * 16);
+            const bf16* hh = (const bf16*)&e;
+#pragma unroll
+            for (int qq = 0; qq < 8; ++qq)
+              v[i * 8 + qq] = __fmul_rn(v[i * 8 + qq], act_grad(a.mask_act, __bfloat162float(hh[qq])));
+          }
+        }
+      }
+      bf16* o = (bf16*)a.out + orow * 64;
+#pragma unroll
+      for (int i = 0; i < 64; i += 8) st_bf16x8(o + i, v + i);
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 4) {
+    tc_fence_after();
+    tmem_dealloc<Cfg::TMEM_COLS>(tmem);
+  }
+}
+
+}  // namespace adainf
