@@ -191,8 +191,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
         for (int i = 0; i < 8; ++i) {
           const long long m = ti.m0 + (t >> 3) + 16 * i;
           if (m < npix) {
-            const int n = (int)(m / HWg);
-            const int pix = (int)(m - (long long)n * HWg);
+            const int mi = (int)m;  // pixel counts < 2^31 (host-checked)
+            const int n = mi / HWg;
+            const int pix = mi - n * HWg;
             const int gy = pix / a.Wg, gx = pix - gy * a.Wg;
             const int sn = a.src_map ? __ldg(a.src_map + n) : n;
             rowbase[i] = (long long)sn * a.Hs * a.Ws;
@@ -310,8 +311,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
           long long base = 0;
           int gy0 = -100000, gx0 = 0;
           if (p < npix) {
-            const int n = (int)(p / HWg);
-            const int pix = (int)(p - (long long)n * HWg);
+            const int pi = (int)p;
+            const int n = pi / HWg;
+            const int pix = pi - n * HWg;
             gy0 = pix / a.Wg;
             gx0 = pix - gy0 * a.Wg;
             gy0 *= a.sy;
@@ -428,8 +430,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
         long long orow = 0, rrow = 0;
         int n = 0;
         if (rv) {
-          n = (int)(m / HWg);
-          const int pix = (int)(m - (long long)n * HWg);
+          n = (int)m / HWg;
+          const int pix = (int)m - n * HWg;
           const int gy = pix / a.Wg, gx = pix - gy * a.Wg;
           orow = ((long long)n * a.Ho + gy * a.oys + a.oyo) * a.Wo + gx * a.oxs + a.oxo;
           if (MODE == MODE_FWD && a.res) {

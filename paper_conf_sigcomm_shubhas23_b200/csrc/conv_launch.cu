@@ -115,9 +115,14 @@ static int pick_bn(int nout, bool mn_major_b) {
   return 256;
 }
 
+static void check_extent(long long pixels) {
+  if (pixels >= (1LL << 31) - (1LL << 20)) throw ShapeError("conv: more than 2^31 output positions");
+}
+
 void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* count, int n_static,
               const bf16* w, int ldb, const float* bias, const bf16* res, const int* res_map, int act, void* out,
               bool out_f32, cudaStream_t st) {
+  check_extent((long long)n_static * (g.H + 1) * (g.W + 1));
   ConvArgs a{};
   a.src = x;
   a.src_map = x_map;
@@ -180,6 +185,7 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
 
 void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n, const float* bcast,
                 const bf16* sc, const bf16* yact, int mask_act, bf16* dx, cudaStream_t st) {
+  check_extent((long long)n * (g.H + 1) * (g.W + 1));
   // dX[y] = sum_{kh: (y + pad - kh) % s == 0} dZ[(y + pad - kh)/s] W[kh]; split by output phase (py,px)
   if (win_ok(g) && (g.H <= 14 || win_mode() >= 2 || (g.Cin == 64 && g.Cout == 64))) {
     // stride 1: one window launch with flipped taps (faster at H<=14; weight-stationary at 64x64)
@@ -340,11 +346,70 @@ size_t wgrad_ws_bytes(const ConvGeom& g, int n) {
   int S = wgrad_splits(tiles, nkb);
   const int kbs = (nkb + S - 1) / S;
   S = (nkb + kbs - 1) / kbs;
-  return (size_t)S * Kconv * g.Cout * sizeof(float) + (size_t)colsum_blocks(npix) * g.Cout * sizeof(float);
+  size_t need = (size_t)S * Kconv * g.Cout * sizeof(float) + (size_t)colsum_blocks(npix) * g.Cout * sizeof(float);
+  if (g.KH == 3 && g.KW == 3 && g.stride == 1 && g.Cin == 64 && g.Cout == 64)  // window variant
+    need = std::max(need, (size_t)num_sms() * 576 * 64 * 4 + (size_t)colsum_blocks(npix) * g.Cout * 4);
+  return need;
+}
+
+static bool win_wgrad_ok(const ConvGeom& g) {
+  return win_mode() > 0 && g.KH == 3 && g.KW == 3 && g.stride == 1 && g.pad == 1 && g.Cin == 64 && g.Cout == 64 &&
+         g.W <= 56 && g.H == g.Ho && g.W == g.Wo;
 }
 
 void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin_real, float* ws, size_t ws_bytes,
                 float* dw, float* db, cudaStream_t st) {
+  check_extent((long long)n * (g.H + 1) * (g.W + 1));
+  if (win_wgrad_ok(g)) {
+    // one K-range of 64-position blocks per persistent CTA; partials [S][576][64] reduced in fixed order
+    const long long Q = (long long)n * (g.H + 1) * (g.W + 1);
+    const int nkb = (int)((Q + 63) / 64);
+    int S = std::min(num_sms(), nkb);
+    const int kbs = (nkb + S - 1) / S;
+    S = (nkb + kbs - 1) / kbs;
+    if ((size_t)S * 576 * 64 * 4 + (size_t)colsum_blocks((long long)n * g.Ho * g.Wo) * g.Cout * 4 > ws_bytes)
+      throw std::runtime_error("wgrad workspace too small (window)");
+    WinArgs w{};
+    w.c.src = x;
+    w.c.Hs = g.H;
+    w.c.Ws = g.W;
+    w.c.Cs = 64;
+    w.c.n_static = n;
+    w.c.B = dz;
+    w.c.Nout = 64;
+    w.c.out = ws;
+    w.c.kb_per_split = kbs;
+    for (int kh = 0; kh < 3; ++kh)
+      for (int kw = 0; kw < 3; ++kw) w.tap_off[kh * 3 + kw] = kh * (g.W + 1) + kw;
+    static bool attr = false;
+    if (!attr) {
+      CK(cudaFuncSetAttribute(conv_win_wgrad_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, WinWgCfg::SMEM));
+      attr = true;
+    }
+    {
+      ProfScope ps(PC_CONV_WGRAD, st);
+      conv_win_wgrad_kernel<<<S, NUM_THREADS, WinWgCfg::SMEM, st>>>(w);
+      CK(cudaGetLastError());
+    }
+    {
+      dim3 rg((576 + 31) / 32, 2);
+      ProfScope ps(PC_WGRAD_REDUCE, st);
+      wgrad_reduce_kernel<<<rg, dim3(32, 8), 0, st>>>(ws, S, 576, 64, 64, cin_real, dw);
+      CK(cudaGetLastError());
+    }
+    if (db) {
+      const long long npix = (long long)n * g.Ho * g.Wo;
+      float* part = ws + (size_t)S * 576 * 64;
+      const int nb = colsum_blocks(npix);
+      const long long rpb = (npix + nb - 1) / nb;
+      const int groups = CS_THREADS / (g.Cout / 8);
+      ProfScope ps(PC_BIAS_COLSUM, st, 2);
+      colsum_partial_kernel<<<nb, CS_THREADS, (size_t)groups * g.Cout * 4, st>>>(dz, npix, g.Cout, rpb, part);
+      colsum_final_kernel<<<(g.Cout + 127) / 128, 128, 0, st>>>(part, nb, g.Cout, db);
+      CK(cudaGetLastError());
+    }
+    return;
+  }
   const long long npix = (long long)n * g.Ho * g.Wo;
   const int nkb = (int)((npix + BK - 1) / BK);
   const int Kconv = g.KH * g.KW * g.Cin;

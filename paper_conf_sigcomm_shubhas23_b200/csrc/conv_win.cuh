@@ -589,3 +589,201 @@ __global__ void __launch_bounds__(WS_THREADS, 1) conv_win_ws_kernel(const WinArg
 }
 
 }  // namespace adainf
+
+namespace adainf {
+
+// ------------------------------------------------------------------------------------------------
+// Window WGRAD for 64-channel stride-1 3x3 layers (ResNet layer1):
+//   dW[(tap, ci)][co] = sum_q X[q + off(tap)][ci] * dZ[q][co]    (q on the padded flattened grid)
+// Per 64-position K-block the CTA loads ONE window of X rows (64 + 2(W+1) + 2) and the 64 dZ rows; the
+// A operand of tap pair (t, t+1) is the window viewed MN-major at row offset off(t) with the second MN
+// atom LBO = (off(t+1) - off(t)) rows away (tap 8 pairs with a zero atom).  Five TMEM accumulators
+// (5 x 64 columns) cover all 576 kconv rows, so each K-block's operands are used by 20 MMAs.  Each CTA
+// reduces a contiguous range of K-blocks into fp32 partials [split][576][64] (fixed-order reduction
+// afterwards: deterministic).
+struct WinWgCfg {
+  static constexpr int WROWS = 64 + 2 * 57 + 2;                       // <= W 56
+  static constexpr int WIN_BYTES = ((WROWS + 7) / 8) * 1024;            // 23 KB
+  static constexpr int B_BYTES = 64 * 64 * 2;                           // dZ block, MN-major
+  static constexpr int STAGE_BYTES = WIN_BYTES + B_BYTES;
+  static constexpr int STAGES = 5;
+  static constexpr int ZERO_BYTES = 2048;                               // zero MN atom for tap 8
+  static constexpr int SMEM = STAGES * STAGE_BYTES + ZERO_BYTES + 1024 + 256;
+  static constexpr int TMEM_COLS = 512;                                 // 5 x 64 used
+};
+
+__global__ void __launch_bounds__(NUM_THREADS, 1) conv_win_wgrad_kernel(const WinArgs w) {
+  using Cfg = WinWgCfg;
+  const ConvArgs& a = w.c;  // src = X (Cs = 64), B = dZ (Nout = 64), out = partial, kb_per_split
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* zero = smem + Cfg::STAGES * Cfg::STAGE_BYTES;
+  uint64_t* full = (uint64_t*)(zero + Cfg::ZERO_BYTES);
+  uint64_t* empty = full + Cfg::STAGES;
+  uint64_t* tfull = empty + Cfg::STAGES;
+  uint32_t* tmem_slot = (uint32_t*)(tfull + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int H = a.Hs, W = a.Ws, Wp = W + 1, Hp = H + 1;
+  const int nsamp = a.n_static;
+  const int Qimg = Hp * Wp;
+  const int Q = nsamp * Qimg;
+  const int nkb = (Q + 63) / 64;
+  const int kb0 = blockIdx.x * a.kb_per_split;
+  const int kb1 = min(kb0 + a.kb_per_split, nkb);
+  const int L = 64 + 2 * Wp + 2;
+
+  for (int i = threadIdx.x; i < Cfg::ZERO_BYTES / 16; i += blockDim.x) ((uint4*)zero)[i] = make_uint4(0, 0, 0, 0);
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < Cfg::STAGES; ++s) {
+      mbar_init(&full[s], 128);
+      mbar_init(&empty[s], 1);
+    }
+    mbar_init(tfull, 1);
+    fence_mbar_init();
+  }
+  if (warp == 4) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
+  fence_proxy_async_smem();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  const uint32_t sbase = smem_u32(smem);
+
+  if (warp < 4) {
+    const int t = threadIdx.x, j = t & 7;
+    constexpr int RPT = (Cfg::WROWS + 15) / 16;
+    int it = 0;
+    for (int kb = kb0; kb < kb1; ++kb, ++it) {
+      const int s = it % Cfg::STAGES, u = it / Cfg::STAGES;
+      if (u > 0) mbar_wait(&empty[s], (u - 1) & 1);
+      const uint32_t sw = sbase + s * Cfg::STAGE_BYTES;
+      const uint32_t sb = sw + Cfg::WIN_BYTES;
+      const int q0 = kb * 64;  // Q < 2^31 (asserted on the host)
+      // X window rows [q0 - Wp - 1, q0 - Wp - 1 + L): decode the first row, then step 16 with carries
+      {
+        int qs = q0 - Wp - 1 + (t >> 3);
+        int n = 0, h = 0, x = 0;
+        if (qs >= 0) {
+          n = qs / Qimg;
+          const int rem = qs - n * Qimg;
+          h = rem / Wp;
+          x = rem - h * Wp;
+        }
+#pragma unroll
+        for (int i = 0; i < RPT; ++i) {
+          const int r = (t >> 3) + 16 * i;
+          if (r < L) {
+            const bool v = qs >= 0 && qs < Q && h < H && x < W;
+            const bf16* g = v ? a.src + ((long long)((n * H + h) * W + x) * 64 + j * 8) : a.src;
+            cp_async16(sw + kmaj_off(r, j), g, v);
+          }
+          qs += 16;
+          if (qs >= 0) {
+            if (qs < 16) {
+              n = 0;
+              h = qs / Wp;
+              x = qs - h * Wp;
+            } else {
+              x += 16;
+              while (x >= Wp) {
+                x -= Wp;
+                if (++h >= Hp) {
+                  h = 0;
+                  ++n;
+                }
+              }
+            }
+          }
+        }
+      }
+      // dZ rows q0 .. q0+63 (zero at padding positions)
+      {
+        int q = q0 + (t >> 3);
+        int n = q / Qimg;
+        const int rem = q - n * Qimg;
+        int h = rem / Wp, x = rem - h * Wp;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int r = (t >> 3) + 16 * i;
+          const bool v = q < Q && h < H && x < W;
+          const bf16* g = v ? a.B + ((long long)((n * H + h) * W + x) * 64 + j * 8) : a.B;
+          cp_async16(sb + kmaj_off(r, j), g, v);  // == MN-major layout for a single 64-wide atom
+          q += 16;
+          x += 16;
+          while (x >= Wp) {
+            x -= Wp;
+            if (++h >= Hp) {
+              h = 0;
+              ++n;
+            }
+          }
+        }
+      }
+      cp_async_arrive_noinc(&full[s]);
+    }
+  } else if (warp == 4) {
+    const uint32_t IDESC = make_idesc(BM, 64, 1, 1);
+    const uint32_t zaddr = smem_u32(zero);
+    int it = 0;
+    for (int kb = kb0; kb < kb1; ++kb, ++it) {
+      const int s = it % Cfg::STAGES, u = it / Cfg::STAGES;
+      mbar_wait(&full[s], u & 1);
+      fence_proxy_async_smem();
+      tc_fence_after();
+      if (lane == 0) {
+        const uint32_t sw = sbase + s * Cfg::STAGE_BYTES;
+        const uint32_t sb = sw + Cfg::WIN_BYTES;
+#pragma unroll
+        for (int p = 0; p < 5; ++p) {
+          const int t0 = 2 * p;
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk) {
+            const uint32_t a0 = sw + (uint32_t)(w.tap_off[t0] + kk * 16) * 128u;
+            const uint32_t a1 = (t0 + 1 < 9) ? sw + (uint32_t)(w.tap_off[t0 + 1] + kk * 16) * 128u : zaddr;
+            const uint64_t ad = make_sdesc(a0, a1 - a0, 1024);
+            const uint64_t bd = make_sdesc(sb + kk * 2048, 8192, 1024);
+            umma_bf16(tmem + (uint32_t)(p * 64), ad, bd, IDESC, (it | kk) != 0);
+          }
+        }
+        umma_commit(&empty[s]);
+      }
+      __syncwarp();
+    }
+    if (lane == 0) {
+      if (kb1 > kb0) umma_commit(tfull);
+      else mbar_arrive(tfull);
+    }
+    __syncwarp();
+  } else {
+    const int qd = warp & 3;
+    const int row = qd * 32 + lane;
+    mbar_wait(tfull, 0);
+    tc_fence_after();
+    const uint32_t trow = tmem + ((uint32_t)(qd * 32) << 16);
+    for (int p = 0; p < 5; ++p) {
+      const int kconv = p * 128 + row;
+      float* outp = (float*)a.out + ((long long)blockIdx.x * 576 + kconv) * 64;
+#pragma unroll 1
+      for (int c0 = 0; c0 < 64; c0 += 32) {
+        float v[32];
+        if (kb1 > kb0) tmem_ld32(trow + p * 64 + c0, v);
+        else
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = 0.f;
+        if (kconv < 576)
+#pragma unroll
+          for (int i = 0; i < 32; i += 4) *(float4*)(outp + c0 + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+      }
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 4) {
+    tc_fence_after();
+    tmem_dealloc<Cfg::TMEM_COLS>(tmem);
+  }
+}
+
+}  // namespace adainf

@@ -24,3 +24,19 @@ for (H, C, Co) in shapes:
             ms = e0.elapsed_time(e1) / 5
             print(f"H={H:3d} C={C:3d} mode={m} {name:6s} {ms*1e3:8.1f} us {fl/ms/1e9:7.1f} TFLOP/s", flush=True)
 B.dbg_set_win_mode(1)
+# wgrad timing
+if os.environ.get("WGRAD", "1") == "1":
+    for (H, C, Co) in shapes:
+        x = torch.randn(n, H, H, C, device="cuda").to(torch.bfloat16)
+        dz = torch.randn(n, H, H, Co, device="cuda").to(torch.bfloat16)
+        fl = 2 * n * H * H * Co * 9 * C
+        for m in modes:
+            B.dbg_set_win_mode(m)
+            B.dbg_conv_wgrad(x, dz, 3, 3, 1, 1); torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            for _ in range(5): B.dbg_conv_wgrad(x, dz, 3, 3, 1, 1)
+            e1.record(); torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1) / 5
+            print(f"H={H:3d} C={C:3d} mode={m} wgrad  {ms*1e3:8.1f} us {fl/ms/1e9:7.1f} TFLOP/s (incl. reduce+colsum+alloc)", flush=True)
+    B.dbg_set_win_mode(1)
