@@ -76,3 +76,4 @@ extern "C" adainf_status adainf_dbg_conv_wgrad(const void* x, const void* dz, in
 extern "C" adainf_status adainf_dbg_set_win_mode(int32_t mode) {
   return guard([&] { set_win_mode(mode); });
 }
+

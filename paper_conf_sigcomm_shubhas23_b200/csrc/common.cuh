@@ -43,6 +43,20 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
+// ---- optional role timing (compile with -DADAINF_TIMING): per-CTA cycle counters of barrier waits ----
+#ifdef ADAINF_TIMING
+__device__ unsigned long long g_wait_cycles[4096][8];
+#define TIMED_WAIT(slot, expr)                                                         \
+  do {                                                                                 \
+    const long long _t0 = clock64();                                                   \
+    expr;                                                                              \
+    if ((threadIdx.x & 31) == 0)                                                       \
+      atomicAdd(&g_wait_cycles[blockIdx.x & 4095][slot], (unsigned long long)(clock64() - _t0)); \
+  } while (0)
+#else
+#define TIMED_WAIT(slot, expr) expr
+#endif
+
 // ---- cp.async (LDGSTS) -------------------------------------------------------------------------
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, bool valid) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(valid ? 16 : 0)

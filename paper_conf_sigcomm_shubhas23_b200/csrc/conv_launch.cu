@@ -8,6 +8,7 @@
 
 #include "conv_gemm.cuh"
 #include "conv_win.cuh"
+#include "conv_tma.cuh"
 #include "prof.h"
 #include "runtime.h"
 
@@ -82,7 +83,65 @@ static void launch_win_t(const WinArgs& w, long long max_tiles, cudaStream_t st)
   CK(cudaGetLastError());
 }
 
+// TMA weight-stationary 64x64 window conv (FWD: e0 = residual; DGRAD: e0 = shortcut grad, e1 = activation)
+static void launch_ws_tma(const ConvArgs& c, bool dgrad, int nstatic, cudaStream_t st) {
+  static WsTmaArgs a;  // host staging (copied into the launch parameters)
+  a = WsTmaArgs{};
+  const int H = c.Hs, W = c.Ws;
+  int Wp = 1;
+  while (Wp < W + 1) Wp <<= 1;
+  const int R = std::max(1, 128 / Wp);
+  a.H = H;
+  a.W = W;
+  a.Wp = Wp;
+  a.R = R;
+  a.tpi = (H + R - 1) / R;
+  a.smap = c.src_map;
+  a.count = c.count;
+  a.n_static = nstatic;
+  a.B = c.B;
+  a.ldb = c.ldb;
+  a.dgrad = dgrad;
+  a.act = c.act;
+  a.mask_act = c.mask_act;
+  a.bias = c.bias;
+  a.bcast = c.bcast;
+  a.out = (bf16*)c.out;
+  for (int kh = 0; kh < 3; ++kh)
+    for (int kw = 0; kw < 3; ++kw) {
+      a.tap_off[kh * 3 + kw] = dgrad ? 8 + (2 - kh) * Wp + (1 - kw) : 8 + kh * Wp + kw - 1;
+      a.btap[kh * 3 + kw] = kh * 3 + kw;
+    }
+  a.win_map = make_tmap_nhwc(c.src, nstatic, H, W, 64, 64, Wp, R + 2);
+  const bf16* e0 = dgrad ? c.sc : c.res;
+  const bf16* e1 = dgrad && c.mask_act ? c.yact : nullptr;
+  a.has_e0 = e0 != nullptr;
+  a.has_e1 = e1 != nullptr;
+  if (e0) a.e0_map = make_tmap_nhwc(e0, nstatic, H, W, 64, 64, Wp, R);
+  if (e1) a.e1_map = make_tmap_nhwc(e1, nstatic, H, W, 64, 64, Wp, R);
+  if (!dgrad && c.res_map && c.res_map != c.src_map) throw std::runtime_error("ws_tma: residual map differs");
+  a.win_bytes = ((16 + (R + 2) * Wp) * 128 + 1023) / 1024 * 1024;
+  const int fixed = 9 * 8192 + 2 * (a.has_e0 + a.has_e1) * 16384 + 1024 /*align*/ + 512 /*barriers*/;
+  a.wstages = std::min(8, (227 * 1024 - fixed) / a.win_bytes);
+  if (a.wstages < 2) throw std::runtime_error("ws_tma: shared memory");
+  const int smem = a.wstages * a.win_bytes + fixed;
+  static bool attr = false;
+  if (!attr) {
+    CK(cudaFuncSetAttribute(conv_ws_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    attr = true;
+  }
+  const long long tiles = (long long)nstatic * a.tpi;
+  dim3 grid((unsigned)std::max(1LL, std::min<long long>(tiles, num_sms())));
+  ProfScope ps(dgrad ? PC_CONV_DGRAD : PC_CONV_FWD, st);
+  conv_ws_tma_kernel<<<grid, TMA_WS_THREADS, smem, st>>>(a);
+  CK(cudaGetLastError());
+}
+
 static void launch_win(WinArgs& w, int nstatic, int nout, cudaStream_t st) {
+  if (w.c.Cs == 64 && nout == 64 && win_mode() != 4) {  // TMA weight-stationary (mode 4: cp.async variant)
+    launch_ws_tma(w.c, w.dgrad != 0, nstatic, st);
+    return;
+  }
   if (w.c.Cs == 64 && nout == 64) {  // weight-stationary 64x64 variant (ResNet layer1)
     static bool attr = false;
     if (!attr) {
@@ -461,3 +520,16 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
 }
 
 }  // namespace adainf
+
+#ifdef ADAINF_TIMING
+// instrumented builds only (tools/build_timing.sh): per-CTA barrier-wait cycle counters of this TU's kernels
+extern "C" int adainf_dbg_wait_cycles(unsigned long long* host_out /* 4096*8 */, int reset) {
+  cudaDeviceSynchronize();
+  cudaMemcpyFromSymbol(host_out, adainf::g_wait_cycles, sizeof(unsigned long long) * 4096 * 8);
+  if (reset) {
+    static unsigned long long z[4096][8];
+    cudaMemcpyToSymbol(adainf::g_wait_cycles, z, sizeof(z));
+  }
+  return 0;
+}
+#endif

@@ -1,0 +1,246 @@
+// Weight-stationary window conv for 64-channel stride-1 3x3 layers (ResNet layer1), operands moved by
+// TMA (cp.async.bulk.tensor) instead of per-thread cp.async.
+//
+// Why TMA: the cp.async gather keeps only a bounded number of 16-byte requests in flight per SM, so for
+// DRAM-resident activations it delivered ~3-5 B/cycle/SM (producers spent 75% of their time issuing);
+// one bulk tensor copy per window moves 32 KB with a single instruction and an mbarrier transaction count.
+//
+// Tiling: a tile is R = 128 / Wp consecutive image rows of ONE image on a padded row pitch Wp (power of
+// two >= W+1, the columns x >= W are the zero padding the TMA box reads out of bounds).  The window of a
+// tile is the TMA box {64 ch, Wp px, R+2 rows} starting at row h0-1 (row -1 / H are out of bounds ->
+// zeros), so every tap (dy, dx) of the 3x3 stencil is the window viewed at row offset 8 + (dy+1)Wp + dx
+// (8 zero rows lead the box in shared memory).  B (9 tap tiles, 72 KB) stays resident in shared memory;
+// the epilogue operands (residual / shortcut-gradient / stored activation) are staged by TMA too.
+#pragma once
+#include "conv_gemm.cuh"
+#include "tma.cuh"
+
+namespace adainf {
+
+struct WsTmaArgs {
+  CUtensorMap win_map;  // source activations, box {64, Wp, R+2, 1}
+  CUtensorMap e0_map;   // FWD: residual; DGRAD: shortcut gradient   (box {64, Wp, R, 1})
+  CUtensorMap e1_map;   // DGRAD: stored activation for the act' mask (box {64, Wp, R, 1})
+  const int* smap;      // optional sample map for the window / residual (inference stages)
+  const int* count;
+  int n_static;
+  int H, W, Wp, R, tpi;  // tiles per image = ceil(H / R)
+  const bf16* B;
+  int ldb;
+  int tap_off[9], btap[9];
+  int dgrad, has_e0, has_e1, act, mask_act;
+  const float* bias;
+  const float* bcast;
+  bf16* out;
+  int wstages, win_bytes;
+};
+
+constexpr int TMA_WS_THREADS = 416;  // warp 0 TMA producer (+ warps 1-3 help load B), warp 4 MMA, 8 epilogue warps
+
+__global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __grid_constant__ WsTmaArgs a) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  const int WS = a.wstages;
+  uint8_t* win = smem;
+  uint8_t* bres = win + WS * a.win_bytes;               // 9 x 8 KB
+  const int ntens = a.has_e0 + a.has_e1;
+  uint8_t* stg = bres + 9 * 8192;                        // [2 groups][ntens tensors][16 KB]
+  uint64_t* bars = (uint64_t*)(stg + 2 * ntens * 16384);
+  uint64_t* wfull = bars;          // [WS]
+  uint64_t* wempty = wfull + 8;    // [WS]
+  uint64_t* tfull = wempty + 8;    // [2]
+  uint64_t* tempty = tfull + 2;    // [2]
+  uint64_t* efull = tempty + 2;    // [2]
+  uint64_t* bready = efull + 2;
+  uint32_t* tmem_slot = (uint32_t*)(bready + 1);
+  float* s_bias = (float*)(tmem_slot + 4);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nsamp = a.count ? *a.count : a.n_static;
+  const int ntile = nsamp * a.tpi;
+  if ((int)blockIdx.x >= ntile) return;
+  const int Wp = a.Wp, R = a.R, H = a.H, W = a.W;
+
+  // zero the 8 lead / 8 trail rows of every window buffer (the TMA never writes them)
+  for (int i = threadIdx.x; i < WS * 2 * 64; i += blockDim.x) {
+    const int s = i / 128, k = i % 128;
+    const int rows = 8 + (R + 2) * Wp;
+    uint4* p = (uint4*)(win + s * a.win_bytes + (k < 64 ? k * 16 : rows * 128 + (k - 64) * 16));
+    *p = make_uint4(0, 0, 0, 0);
+  }
+  if (threadIdx.x < 64) s_bias[threadIdx.x] = (!a.dgrad && a.bias) ? a.bias[threadIdx.x] : 0.f;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < WS; ++s) {
+      mbar_init(&wfull[s], 1);
+      mbar_init(&wempty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 128);
+      mbar_init(&efull[b], 1);
+    }
+    mbar_init(bready, 128);
+    fence_mbar_init();
+    tma_prefetch_desc(&a.win_map);
+  }
+  if (warp == 4) tmem_alloc<128>(tmem_slot);
+  fence_proxy_async_smem();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  const uint32_t wsm = smem_u32(win), bsm = smem_u32(bres), ssm = smem_u32(stg);
+  const uint32_t box_bytes = 64u * 2u * Wp * (R + 2);
+  const uint32_t ebox_bytes = 64u * 2u * Wp * R;
+
+  if (warp < 4) {
+    // ---- resident B (once per CTA, cp.async by all 128 producer threads) ----
+    const int t = threadIdx.x;
+    for (int tp = 0; tp < 9; ++tp) {
+      const uint32_t sb = bsm + tp * 8192;
+      const bf16* wb = a.B + (long long)a.btap[tp] * 64;
+#pragma unroll
+      for (int idx = t; idx < 64 * 8; idx += 128) {
+        const int r = idx >> 3, jj = idx & 7;
+        const uint32_t off = a.dgrad ? mnmaj_off(r, jj) : kmaj_off(r, jj);
+        cp_async16(sb + off, wb + (long long)r * a.ldb + jj * 8, true);
+      }
+    }
+    cp_async_arrive_noinc(bready);
+    // ---- windows: one TMA box per tile, issued by one thread ----
+    if (warp == 0 && lane == 0) {
+      int it = 0;
+      for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++it) {
+        const int n = tile / a.tpi, h0 = (tile - n * a.tpi) * R;
+        const int sn = a.smap ? __ldg(a.smap + n) : n;
+        const int s = it % WS, u = it / WS;
+        if (u > 0) mbar_wait(&wempty[s], (u - 1) & 1);
+        mbar_expect_tx(&wfull[s], box_bytes);
+        tma_load_4d(wsm + s * a.win_bytes + 1024, &a.win_map, &wfull[s], 0, 0, h0 - 1, sn);
+      }
+    }
+  } else if (warp == 4) {
+    // ---- MMA issuer ----
+    const uint32_t IDESC = make_idesc(BM, 64, 0, a.dgrad ? 1 : 0);
+    mbar_wait(bready, 0);
+    fence_proxy_async_smem();
+    int it = 0;
+    for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++it) {
+      const int b = it & 1, ub = it >> 1;
+      if (ub > 0) mbar_wait(&tempty[b], (ub - 1) & 1);
+      const int s = it % WS, u = it / WS;
+      mbar_wait(&wfull[s], u & 1);
+      tc_fence_after();
+      if (lane == 0) {
+        const uint32_t sw = wsm + s * a.win_bytes;
+        const uint32_t dacc = tmem + (uint32_t)(b * 64);
+#pragma unroll 1
+        for (int tp = 0; tp < 9; ++tp) {
+          const uint32_t sb = bsm + tp * 8192;
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk) {
+            const uint64_t ad = make_sdesc(sw + (uint32_t)a.tap_off[tp] * 128u + kk * 32, 16, 1024);
+            const uint64_t bd = a.dgrad ? make_sdesc(sb + kk * 2048, 8192, 1024) : make_sdesc(sb + kk * 32, 16, 1024);
+            umma_bf16(dacc, ad, bd, IDESC, (tp | kk) != 0);
+          }
+        }
+        umma_commit(&wempty[s]);
+        umma_commit(&tfull[b]);
+      }
+      __syncwarp();
+    }
+  } else {
+    // ---- epilogue: 2 groups of 4 warps, group g handles this CTA's local tiles g, g+2, ... ----
+    const int grp = (warp - 5) >> 2;
+    const int qd = warp & 3;
+    const int row = qd * 32 + lane;  // output position p within the tile
+    const bool leader = (warp == 5 + 4 * grp) && lane == 0;
+    const uint32_t sg = ssm + grp * ntens * 16384;
+    int lt = grp, use = 0;
+    for (int tile = blockIdx.x + grp * gridDim.x; tile < ntile; tile += 2 * gridDim.x, lt += 2, ++use) {
+      const int n = tile / a.tpi, h0 = (tile - n * a.tpi) * R;
+      const int h = h0 + row / Wp, x = row % Wp;
+      const bool rv = h < H && x < W;
+      const long long orow = ((long long)n * H + h) * W + x;
+      if (ntens && leader) {  // stage the epilogue operands of this tile (buffer freed by the group barrier)
+        mbar_expect_tx(&efull[grp], ntens * ebox_bytes);
+        const int sn = (!a.dgrad && a.smap) ? __ldg(a.smap + n) : n;
+        if (a.has_e0) tma_load_4d(sg, &a.e0_map, &efull[grp], 0, 0, h0, sn);
+        if (a.has_e1) tma_load_4d(sg + a.has_e0 * 16384, &a.e1_map, &efull[grp], 0, 0, h0, n);
+      }
+      const int b = grp, ub = lt >> 1;
+      mbar_wait(&tfull[b], ub & 1);
+      tc_fence_after();
+      const uint32_t trow = tmem + (uint32_t)(b * 64) + ((uint32_t)(qd * 32) << 16);
+      float v[64];
+      tmem_ld32(trow, v);
+      tmem_ld32(trow + 32, v + 32);
+      tc_fence_before();
+      mbar_arrive(&tempty[b]);
+      if (ntens) mbar_wait(&efull[grp], use & 1);
+      const uint8_t* e0 = stg + (grp * ntens) * 16384 + row * 128;
+      const uint8_t* e1 = e0 + a.has_e0 * 16384;
+      if (rv) {
+        if (!a.dgrad) {
+#pragma unroll
+          for (int i = 0; i < 64; ++i) v[i] = __fadd_rn(v[i], s_bias[i]);
+          if (a.has_e0) {
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              const uint4 e = *(const uint4*)(e0 + ((i ^ (row & 7)) << 4));
+              const bf16* hh = (const bf16*)&e;
+#pragma unroll
+              for (int qq = 0; qq < 8; ++qq) v[i * 8 + qq] = __fadd_rn(v[i * 8 + qq], __bfloat162float(hh[qq]));
+            }
+          }
+#pragma unroll
+          for (int i = 0; i < 64; ++i) v[i] = act_apply(a.act, v[i]);
+        } else {
+          if (a.bcast) {
+#pragma unroll
+            for (int i = 0; i < 64; i += 4) {
+              const float4 bb = __ldg((const float4*)(a.bcast + (long long)n * 64 + i));
+              v[i] = __fadd_rn(v[i], bb.x);
+              v[i + 1] = __fadd_rn(v[i + 1], bb.y);
+              v[i + 2] = __fadd_rn(v[i + 2], bb.z);
+              v[i + 3] = __fadd_rn(v[i + 3], bb.w);
+            }
+          }
+          if (a.has_e0) {
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              const uint4 e = *(const uint4*)(e0 + ((i ^ (row & 7)) << 4));
+              const bf16* hh = (const bf16*)&e;
+#pragma unroll
+              for (int qq = 0; qq < 8; ++qq) v[i * 8 + qq] = __fadd_rn(v[i * 8 + qq], __bfloat162float(hh[qq]));
+            }
+          }
+          if (a.has_e1) {
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              const uint4 e = *(const uint4*)(e1 + ((i ^ (row & 7)) << 4));
+              const bf16* hh = (const bf16*)&e;
+#pragma unroll
+              for (int qq = 0; qq < 8; ++qq)
+                v[i * 8 + qq] = __fmul_rn(v[i * 8 + qq], act_grad(a.mask_act, __bfloat162float(hh[qq])));
+            }
+          }
+        }
+        bf16* o = a.out + orow * 64;
+#pragma unroll
+        for (int i = 0; i < 64; i += 8) st_bf16x8(o + i, v + i);
+      }
+      // all threads of the group are done with the staging buffer before the next TMA overwrites it
+      asm volatile("bar.sync %0, 128;" ::"r"(1 + grp) : "memory");
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 4) {
+    tc_fence_after();
+    tmem_dealloc<128>(tmem);
+  }
+}
+
+}  // namespace adainf

@@ -414,8 +414,11 @@ __global__ void __launch_bounds__(WS_THREADS, 1) conv_win_ws_kernel(const WinArg
         h = rem / Wp;
         x = rem - h * Wp;
       }
-      if (u > 0) mbar_wait(&wempty[s], (u - 1) & 1);
+      if (u > 0) TIMED_WAIT(0, mbar_wait(&wempty[s], (u - 1) & 1));
       const uint32_t sw = wsm + s * Cfg::WIN_BYTES;
+#ifdef ADAINF_TIMING
+      const long long _ti0 = clock64();
+#endif
 #pragma unroll
       for (int i = 0; i < RPT; ++i) {
         const int r = (t >> 3) + 16 * i;
@@ -448,6 +451,9 @@ __global__ void __launch_bounds__(WS_THREADS, 1) conv_win_ws_kernel(const WinArg
         }
       }
       cp_async_arrive_noinc(&wfull[s]);
+#ifdef ADAINF_TIMING
+      if ((threadIdx.x & 31) == 0) atomicAdd(&g_wait_cycles[blockIdx.x & 4095][4], (unsigned long long)(clock64() - _ti0));
+#endif
     }
   } else if (warp == 4) {
     const uint32_t IDESC = make_idesc(BM, 64, 0, w.dgrad ? 1 : 0);
@@ -455,11 +461,11 @@ __global__ void __launch_bounds__(WS_THREADS, 1) conv_win_ws_kernel(const WinArg
     int wit = 0;
     for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++wit) {
       const int b = wit & 1, ub = wit >> 1;
-      if (ub > 0) mbar_wait(&tempty[b], (ub - 1) & 1);
+      if (ub > 0) TIMED_WAIT(1, mbar_wait(&tempty[b], (ub - 1) & 1));
       tc_fence_after();
       const uint32_t dacc = tmem + (uint32_t)(b * Cfg::ACC_COLS);
       const int s = wit % Cfg::WSTAGES, u = wit / Cfg::WSTAGES;
-      mbar_wait(&wfull[s], u & 1);
+      TIMED_WAIT(2, mbar_wait(&wfull[s], u & 1));
       fence_proxy_async_smem();
       tc_fence_after();
       if (lane == 0) {
@@ -518,7 +524,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1) conv_win_ws_kernel(const WinArg
 #pragma unroll
         for (int i = 0; i < 8; ++i) cp_async16(est + 128 + i * 16, p1 + i * 8, true);
       asm volatile("cp.async.commit_group;" ::: "memory");
-      mbar_wait(&tfull[b], ub & 1);
+      TIMED_WAIT(3, mbar_wait(&tfull[b], ub & 1));
       tc_fence_after();
       const uint32_t trow = tmem + (uint32_t)(b * Cfg::ACC_COLS) + ((uint32_t)(qd * 32) << 16);
       float v[64];

@@ -1,0 +1,40 @@
+// TMA (cp.async.bulk.tensor) helpers: host-side tensor-map encoding through the driver entry point (no
+// -lcuda link) and device-side bulk tensor loads completing on an mbarrier (transaction bytes).
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include "common.cuh"
+#include "runtime.h"
+
+namespace adainf {
+
+// 4-D tiled map over a dense NHWC bf16 tensor [N][H][W][C]: dims (innermost first) {C, W, H, N},
+// box {bc, bw, bh, 1}, 128B swizzle (bc * 2 bytes must be <= 128), out-of-bounds -> zeros.
+CUtensorMap make_tmap_nhwc(const void* base, int N, int H, int W, int C, int bc, int bw, int bh);
+// 2-D tiled map over a row-major [rows][cols] bf16 matrix (row pitch ld elements), box {bcols, brows}.
+CUtensorMap make_tmap_2d(const void* base, long long rows, int cols, int ld, int bcols, int brows);
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void tma_load_4d(uint32_t dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1, int c2,
+                                            int c3) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], "
+      "[%6];" ::"r"(dst),
+      "l"(map), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
+          dst),
+      "l"(map), "r"(c0), "r"(c1), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void tma_prefetch_desc(const CUtensorMap* map) {
+  asm volatile("prefetch.tensormap [%0];" ::"l"(map) : "memory");
+}
+
+}  // namespace adainf
