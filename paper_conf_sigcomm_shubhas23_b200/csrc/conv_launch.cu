@@ -137,7 +137,84 @@ static void launch_ws_tma(const ConvArgs& c, bool dgrad, int nstatic, cudaStream
   CK(cudaGetLastError());
 }
 
+// general TMA window conv (Cin multiple of 64, BN 128/256, W <= 28)
+template <int BN>
+static void launch_win_tma_t(WinTmaArgs& a, int nstatic, cudaStream_t st) {
+  constexpr int B_BYTES = BN * 128;
+  const int fixed = 1024 + 1024;
+  const int budget = 227 * 1024 - fixed;
+  a.wstages = 2;
+  a.bstages = std::min(16, (budget - 2 * a.win_bytes) / B_BYTES);
+  if (a.bstages < 3) {
+    a.wstages = 1;
+    a.bstages = std::min(16, (budget - a.win_bytes) / B_BYTES);
+  }
+  if (a.bstages < 2) throw std::runtime_error("win_tma: shared memory");
+  const int smem = a.wstages * a.win_bytes + a.bstages * B_BYTES + fixed;
+  static bool attr = false;
+  if (!attr) {
+    CK(cudaFuncSetAttribute(conv_win_tma_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    attr = true;
+  }
+  const long long tiles = (long long)nstatic * a.tpi * ((a.Nout + BN - 1) / BN);
+  dim3 grid((unsigned)std::max(1LL, std::min<long long>(tiles, num_sms())));
+  ProfScope ps(a.dgrad ? PC_CONV_DGRAD : PC_CONV_FWD, st);
+  conv_win_tma_kernel<BN><<<grid, NUM_THREADS, smem, st>>>(a);
+  CK(cudaGetLastError());
+}
+
+static bool win_tma_ok(const ConvArgs& c, int nout) {
+  return c.Cs % 64 == 0 && nout % 128 == 0 && c.Ws <= 28 && c.Ws >= 8 && win_mode() != 4;
+}
+
+static void launch_win_tma(const ConvArgs& c, bool dgrad, int nstatic, int nout, cudaStream_t st) {
+  static WinTmaArgs a;
+  a = WinTmaArgs{};
+  const int H = c.Hs, W = c.Ws;
+  int Wp = 1;
+  while (Wp < W + 1) Wp <<= 1;
+  const int R = std::max(1, 128 / Wp);
+  a.H = H;
+  a.W = W;
+  a.Wp = Wp;
+  a.R = R;
+  a.tpi = (H + R - 1) / R;
+  a.ncb = c.Cs / 64;
+  a.Nout = nout;
+  a.smap = c.src_map;
+  a.count = c.count;
+  a.n_static = nstatic;
+  a.dgrad = dgrad;
+  a.act = c.act;
+  a.mask_act = c.mask_act;
+  a.bias = c.bias;
+  a.res = c.res;
+  a.bcast = c.bcast;
+  a.sc = c.sc;
+  a.yact = c.yact;
+  a.out = (bf16*)c.out;
+  if (!dgrad && c.res && c.res_map != c.src_map) throw std::runtime_error("win_tma: residual map differs");
+  for (int kh = 0; kh < 3; ++kh)
+    for (int kw = 0; kw < 3; ++kw) {
+      a.tap_off[kh * 3 + kw] = dgrad ? 8 + (2 - kh) * Wp + (1 - kw) : 8 + kh * Wp + kw - 1;
+      a.btap[kh * 3 + kw] = kh * 3 + kw;
+    }
+  a.win_map = make_tmap_nhwc(c.src, nstatic, H, W, c.Cs, 64, Wp, R + 2);
+  const int BN = nout >= 256 ? 256 : 128;
+  // weights shadow rows: FWD [Cout = nout][ldb]; DGRAD [Cout = Cs][ldb] read MN-major
+  const long long wrows = dgrad ? c.Cs : nout;
+  if (!dgrad) a.b_map = make_tmap_2d(c.B, wrows, c.ldb, c.ldb, 64, BN);
+  else a.b_map = make_tmap_2d(c.B, wrows, c.ldb, c.ldb, 64, 64);
+  a.win_bytes = ((16 + (R + 2) * Wp) * 128 + 1023) / 1024 * 1024;
+  if (BN == 256) launch_win_tma_t<256>(a, nstatic, st);
+  else launch_win_tma_t<128>(a, nstatic, st);
+}
+
 static void launch_win(WinArgs& w, int nstatic, int nout, cudaStream_t st) {
+  if (win_tma_ok(w.c, nout) && !(w.c.Cs == 64 && nout == 64)) {
+    launch_win_tma(w.c, w.dgrad != 0, nstatic, nout, st);
+    return;
+  }
   if (w.c.Cs == 64 && nout == 64 && win_mode() != 4) {  // TMA weight-stationary (mode 4: cp.async variant)
     launch_ws_tma(w.c, w.dgrad != 0, nstatic, st);
     return;
@@ -215,7 +292,8 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
   a.res_map = res_map;
   a.act = act;
   if (n_static <= 0) return;
-  if (win_ok(g) && !out_f32 && (win_mode() >= 2 || (g.Cin == 64 && g.Cout == 64))) {
+  if (win_ok(g) && !out_f32 &&
+      (win_mode() >= 2 || (g.Cin == 64 && g.Cout == 64) || (win_mode() != 4 && g.W <= 28 && g.W >= 8 && g.Cout % 128 == 0))) {
     // window kernel: weight-stationary 64x64 variant by default; the general window FWD measured slower
     WinArgs w{};
     w.c = a;
@@ -246,7 +324,7 @@ void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n
                 const bf16* sc, const bf16* yact, int mask_act, bf16* dx, cudaStream_t st) {
   check_extent((long long)n * (g.H + 1) * (g.W + 1));
   // dX[y] = sum_{kh: (y + pad - kh) % s == 0} dZ[(y + pad - kh)/s] W[kh]; split by output phase (py,px)
-  if (win_ok(g) && (g.H <= 14 || win_mode() >= 2 || (g.Cin == 64 && g.Cout == 64))) {
+  if (win_ok(g) && (g.H <= 14 || win_mode() >= 2 || (g.Cin == 64 && g.Cout == 64) || (g.W <= 28 && g.Cin % 128 == 0))) {
     // stride 1: one window launch with flipped taps (faster at H<=14; weight-stationary at 64x64)
     WinArgs wa{};
     ConvArgs& a = wa.c;

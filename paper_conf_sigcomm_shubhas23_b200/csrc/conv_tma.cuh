@@ -244,3 +244,237 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
 }
 
 }  // namespace adainf
+
+namespace adainf {
+
+// ------------------------------------------------------------------------------------------------
+// General TMA window conv for stride-1 3x3 layers with Cin = 64*ncb and BN in {128, 256} (ResNet layers
+// 2-3): per tile and 64-channel block, one window box {64, Wp, R+2, 1} and nine B boxes (FWD: K-major
+// {64 K, BN co} from the [Cout][9*Cin] shadow; DGRAD: MN-major, BN/64 boxes {64 ci, 64 co} per tap), all
+// issued by one thread and completed on mbarrier transaction counts.  Epilogue as in conv_gemm.cuh
+// (4 warps, double-buffered TMEM accumulators, 128-bit global loads / stores).
+struct WinTmaArgs {
+  CUtensorMap win_map;  // source activations, box {64, Wp, R+2, 1}
+  CUtensorMap b_map;    // weights shadow [Cout][ldb] (2-D): FWD box {64, BN}; DGRAD box {64, 64}
+  const int* smap;
+  const int* count;
+  int n_static;
+  int H, W, Wp, R, tpi, ncb, Nout;
+  int tap_off[9], btap[9];
+  int dgrad, act, mask_act;
+  const float* bias;
+  const bf16* res;
+  const float* bcast;
+  const bf16* sc;
+  const bf16* yact;
+  bf16* out;
+  int wstages, bstages, win_bytes;
+};
+
+template <int BN>
+__global__ void __launch_bounds__(NUM_THREADS, 1) conv_win_tma_kernel(const __grid_constant__ WinTmaArgs a) {
+  constexpr int B_BYTES = BN * 128;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  const int WS = a.wstages, BS = a.bstages;
+  uint8_t* win = smem;
+  uint8_t* bb = win + WS * a.win_bytes;
+  uint64_t* bars = (uint64_t*)(bb + BS * B_BYTES);
+  uint64_t* wfull = bars;
+  uint64_t* wempty = wfull + 8;
+  uint64_t* bfull = wempty + 8;
+  uint64_t* bempty = bfull + 16;
+  uint64_t* tfull = bempty + 16;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nsamp = a.count ? *a.count : a.n_static;
+  const int nt = (a.Nout + BN - 1) / BN;
+  const int ntile = nsamp * a.tpi * nt;
+  if ((int)blockIdx.x >= ntile) return;
+  const int Wp = a.Wp, R = a.R, H = a.H, W = a.W;
+
+  for (int i = threadIdx.x; i < WS * 2 * 64; i += blockDim.x) {
+    const int s = i / 128, k = i % 128;
+    const int rows = 8 + (R + 2) * Wp;
+    *(uint4*)(win + s * a.win_bytes + (k < 64 ? k * 16 : rows * 128 + (k - 64) * 16)) = make_uint4(0, 0, 0, 0);
+  }
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < WS; ++s) {
+      mbar_init(&wfull[s], 1);
+      mbar_init(&wempty[s], 1);
+    }
+    for (int s = 0; s < BS; ++s) {
+      mbar_init(&bfull[s], 1);
+      mbar_init(&bempty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 128);
+    }
+    fence_mbar_init();
+    tma_prefetch_desc(&a.win_map);
+    tma_prefetch_desc(&a.b_map);
+  }
+  if (warp == 4) tmem_alloc<2 * BN>(tmem_slot);
+  fence_proxy_async_smem();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  const uint32_t wsm = smem_u32(win), bsm = smem_u32(bb);
+  const uint32_t box_bytes = 64u * 2u * Wp * (R + 2);
+
+  if (warp == 0) {
+    if (lane == 0) {
+      int wit = 0, bit = 0;
+      for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x) {
+        const int nb = tile % nt, r = tile / nt;
+        const int n = r / a.tpi, h0 = (r - n * a.tpi) * R;
+        const int n0 = nb * BN;
+        const int sn = a.smap ? __ldg(a.smap + n) : n;
+        for (int cb = 0; cb < a.ncb; ++cb, ++wit) {
+          const int s = wit % WS, u = wit / WS;
+          if (u > 0) mbar_wait(&wempty[s], (u - 1) & 1);
+          mbar_expect_tx(&wfull[s], box_bytes);
+          tma_load_4d(wsm + s * a.win_bytes + 1024, &a.win_map, &wfull[s], cb * 64, 0, h0 - 1, sn);
+          for (int tp = 0; tp < 9; ++tp, ++bit) {
+            const int bs = bit % BS, bu = bit / BS;
+            if (bu > 0) mbar_wait(&bempty[bs], (bu - 1) & 1);
+            mbar_expect_tx(&bfull[bs], B_BYTES);
+            const uint32_t dst = bsm + bs * B_BYTES;
+            if (!a.dgrad) {
+              // K-major: rows co = n0.., columns btap*Cin + cb*64 ..
+              tma_load_2d(dst, &a.b_map, &bfull[bs], a.btap[tp] * a.ncb * 64 + cb * 64, n0);
+            } else {
+              // MN-major: atom j = ci block n0 + 64j, rows co = cb*64 .. +64
+#pragma unroll
+              for (int j = 0; j < BN / 64; ++j)
+                tma_load_2d(dst + j * 8192, &a.b_map, &bfull[bs], a.btap[tp] * a.Nout + n0 + j * 64, cb * 64);
+            }
+          }
+        }
+      }
+    }
+  } else if (warp == 4) {
+    const uint32_t IDESC = make_idesc(BM, BN, 0, a.dgrad ? 1 : 0);
+    int wit = 0, bit = 0, lt = 0;
+    for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++lt) {
+      const int b = lt & 1, ub = lt >> 1;
+      if (ub > 0) mbar_wait(&tempty[b], (ub - 1) & 1);
+      tc_fence_after();
+      const uint32_t dacc = tmem + (uint32_t)(b * BN);
+      for (int cb = 0; cb < a.ncb; ++cb, ++wit) {
+        const int s = wit % WS, u = wit / WS;
+        mbar_wait(&wfull[s], u & 1);
+        const uint32_t sw = wsm + s * a.win_bytes;
+        for (int tp = 0; tp < 9; ++tp, ++bit) {
+          const int bs = bit % BS, bu = bit / BS;
+          mbar_wait(&bfull[bs], bu & 1);
+          tc_fence_after();
+          if (lane == 0) {
+            const uint32_t sb = bsm + bs * B_BYTES;
+#pragma unroll
+            for (int kk = 0; kk < 4; ++kk) {
+              const uint64_t ad = make_sdesc(sw + (uint32_t)a.tap_off[tp] * 128u + kk * 32, 16, 1024);
+              const uint64_t bd = a.dgrad ? make_sdesc(sb + kk * 2048, 8192, 1024) : make_sdesc(sb + kk * 32, 16, 1024);
+              umma_bf16(dacc, ad, bd, IDESC, (cb | tp | kk) != 0);
+            }
+            umma_commit(&bempty[bs]);
+            if (tp == 8) {
+              umma_commit(&wempty[s]);
+              if (cb == a.ncb - 1) umma_commit(&tfull[b]);
+            }
+          }
+          __syncwarp();
+        }
+      }
+    }
+  } else if (warp >= 5) {
+    const int qd = warp & 3;
+    const int row = qd * 32 + lane;
+    int lt = 0;
+    for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++lt) {
+      const int nb = tile % nt, r = tile / nt;
+      const int n = r / a.tpi, h0 = (r - n * a.tpi) * R;
+      const int n0 = nb * BN;
+      const int h = h0 + row / Wp, x = row % Wp;
+      const bool rv = h < H && x < W;
+      const long long orow = ((long long)n * H + h) * W + x;
+      long long rrow = orow;
+      if (!a.dgrad && a.res && rv && a.smap) rrow = ((long long)__ldg(a.smap + n) * H + h) * W + x;
+      const int b = lt & 1, ub = lt >> 1;
+      mbar_wait(&tfull[b], ub & 1);
+      tc_fence_after();
+      const uint32_t trow = tmem + (uint32_t)(b * BN) + ((uint32_t)(qd * 32) << 16);
+#pragma unroll 1
+      for (int c0 = 0; c0 < BN; c0 += 32) {
+        float v[32];
+        tmem_ld32(trow + c0, v);
+        if (c0 + 32 >= BN) {
+          tc_fence_before();
+          mbar_arrive(&tempty[b]);
+        }
+        const int cbase = n0 + c0;
+        if (!rv || cbase >= a.Nout) continue;
+        if (!a.dgrad) {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = __fadd_rn(v[i], __ldg(a.bias + cbase + i));
+          if (a.res) {
+#pragma unroll
+            for (int i = 0; i < 32; i += 8) {
+              float r8[8];
+              ld_bf16x8(a.res + rrow * a.Nout + cbase + i, r8);
+#pragma unroll
+              for (int qq = 0; qq < 8; ++qq) v[i + qq] = __fadd_rn(v[i + qq], r8[qq]);
+            }
+          }
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = act_apply(a.act, v[i]);
+        } else {
+          if (a.bcast) {
+#pragma unroll
+            for (int i = 0; i < 32; i += 4) {
+              const float4 q4 = __ldg((const float4*)(a.bcast + (long long)n * a.Nout + cbase + i));
+              v[i] = __fadd_rn(v[i], q4.x);
+              v[i + 1] = __fadd_rn(v[i + 1], q4.y);
+              v[i + 2] = __fadd_rn(v[i + 2], q4.z);
+              v[i + 3] = __fadd_rn(v[i + 3], q4.w);
+            }
+          }
+          if (a.sc) {
+#pragma unroll
+            for (int i = 0; i < 32; i += 8) {
+              float r8[8];
+              ld_bf16x8(a.sc + orow * a.Nout + cbase + i, r8);
+#pragma unroll
+              for (int qq = 0; qq < 8; ++qq) v[i + qq] = __fadd_rn(v[i + qq], r8[qq]);
+            }
+          }
+          if (a.mask_act) {
+#pragma unroll
+            for (int i = 0; i < 32; i += 8) {
+              float y8[8];
+              ld_bf16x8(a.yact + orow * a.Nout + cbase + i, y8);
+#pragma unroll
+              for (int qq = 0; qq < 8; ++qq) v[i + qq] = __fmul_rn(v[i + qq], act_grad(a.mask_act, y8[qq]));
+            }
+          }
+        }
+        bf16* o = a.out + orow * a.Nout + cbase;
+#pragma unroll
+        for (int i = 0; i < 32; i += 8) st_bf16x8(o + i, v + i);
+      }
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 4) {
+    tc_fence_after();
+    tmem_dealloc<2 * BN>(tmem);
+  }
+}
+
+}  // namespace adainf

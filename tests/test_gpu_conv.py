@@ -132,10 +132,11 @@ def test_conv_wgrad_vs_torch(case):
     assert torch.equal(dw, dw2) and torch.equal(db, db2)
 
 
-WIN_CASES = [(2, 14, 14, 64, 64), (3, 7, 7, 128, 256), (2, 28, 28, 64, 128), (1, 56, 56, 64, 64), (5, 9, 11, 64, 64)]
+WIN_CASES = [(2, 14, 14, 64, 64), (3, 7, 7, 128, 256), (2, 28, 28, 64, 128), (1, 56, 56, 64, 64), (5, 9, 11, 64, 64),
+             (2, 14, 14, 256, 256), (3, 28, 28, 128, 128), (2, 12, 20, 128, 128), (2, 9, 13, 128, 256)]
 
 
-@pytest.mark.parametrize("mode", [2])
+@pytest.mark.parametrize("mode", [1, 2])
 @pytest.mark.parametrize("case", WIN_CASES)
 def test_window_kernel_fwd_dgrad(case, mode):
     """Window implicit GEMM (stride-1 3x3) vs torch: tap A operands are row-shifted views of one window
