@@ -494,9 +494,82 @@ static bool win_wgrad_ok(const ConvGeom& g) {
          g.W <= 56 && g.H == g.Ho && g.W == g.Wo;
 }
 
+template <int BN>
+static void launch_wgrad_tma_t(WgTmaArgs& a, cudaStream_t st) {
+  constexpr int STAGE = 16384 + BN * 128;
+  a.stages = std::min(16, (225 * 1024 - 2048) / STAGE);
+  const int smem = a.stages * STAGE + 2048;
+  static bool attr = false;
+  if (!attr) {
+    CK(cudaFuncSetAttribute(conv_wgrad_tma_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    attr = true;
+  }
+  const long long units = (long long)((a.Kconv + 127) / 128) * ((a.Cout + BN - 1) / BN) * a.splits;
+  dim3 grid((unsigned)std::max(1LL, std::min<long long>(units, num_sms())));
+  ProfScope ps(PC_CONV_WGRAD, st);
+  conv_wgrad_tma_kernel<BN><<<grid, NUM_THREADS, smem, st>>>(a);
+  CK(cudaGetLastError());
+}
+
+static bool wgrad_tma_ok(const ConvGeom& g) {
+  return win_mode() != 4 && win_mode() != 5 && g.Cin % 64 == 0 && g.Cout % 64 == 0 && g.Wo <= 64 && g.stride <= 2;
+}
+
 void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin_real, float* ws, size_t ws_bytes,
                 float* dw, float* db, cudaStream_t st) {
   check_extent((long long)n * (g.H + 1) * (g.W + 1));
+  if (wgrad_tma_ok(g)) {
+    static WgTmaArgs a;
+    a = WgTmaArgs{};
+    int Wp = 8;
+    while (Wp < g.Wo) Wp <<= 1;
+    a.n = n;
+    a.Ho = g.Ho;
+    a.Wo = g.Wo;
+    a.Wp = Wp;
+    a.Rk = 64 / Wp;
+    a.rg = (g.Ho + a.Rk - 1) / a.Rk;
+    a.KW = g.KW;
+    a.stride = g.stride;
+    a.pad = g.pad;
+    a.ncb = g.Cin / 64;
+    a.Kconv = g.KH * g.KW * g.Cin;
+    a.Cout = g.Cout;
+    const int BN = g.Cout <= 64 ? 64 : (g.Cout <= 128 ? 128 : 256);
+    const int nkb = n * a.rg;
+    const int tiles = ((a.Kconv + 127) / 128) * ((g.Cout + BN - 1) / BN);
+    int S = wgrad_splits(tiles, nkb);
+    const int kbs = (nkb + S - 1) / S;
+    S = (nkb + kbs - 1) / kbs;
+    a.kb_per_split = kbs;
+    a.splits = S;
+    if ((size_t)S * a.Kconv * g.Cout * 4 + (size_t)colsum_blocks((long long)n * g.Ho * g.Wo) * g.Cout * 4 > ws_bytes)
+      throw std::runtime_error("wgrad workspace too small (tma)");
+    a.out = ws;
+    a.x_map = make_tmap_nhwc(x, n, g.H, g.W, g.Cin, 64, Wp, a.Rk, g.stride);
+    a.dz_map = make_tmap_nhwc(dz, n, g.Ho, g.Wo, g.Cout, 64, Wp, a.Rk, 1);
+    if (BN == 64) launch_wgrad_tma_t<64>(a, st);
+    else if (BN == 128) launch_wgrad_tma_t<128>(a, st);
+    else launch_wgrad_tma_t<256>(a, st);
+    {
+      dim3 rg((a.Kconv + 31) / 32, (g.Cout + 31) / 32);
+      ProfScope ps(PC_WGRAD_REDUCE, st);
+      wgrad_reduce_kernel<<<rg, dim3(32, 8), 0, st>>>(ws, S, a.Kconv, g.Cout, g.Cin, cin_real, dw);
+      CK(cudaGetLastError());
+    }
+    if (db) {
+      const long long npix = (long long)n * g.Ho * g.Wo;
+      float* part = ws + (size_t)S * a.Kconv * g.Cout;
+      const int nb = colsum_blocks(npix);
+      const long long rpb = (npix + nb - 1) / nb;
+      const int groups = CS_THREADS / (g.Cout / 8);
+      ProfScope ps(PC_BIAS_COLSUM, st, 2);
+      colsum_partial_kernel<<<nb, CS_THREADS, (size_t)groups * g.Cout * 4, st>>>(dz, npix, g.Cout, rpb, part);
+      colsum_final_kernel<<<(g.Cout + 127) / 128, 128, 0, st>>>(part, nb, g.Cout, db);
+      CK(cudaGetLastError());
+    }
+    return;
+  }
   if (win_wgrad_ok(g)) {
     // one K-range of 64-position blocks per persistent CTA; partials [S][576][64] reduced in fixed order
     const long long Q = (long long)n * (g.H + 1) * (g.W + 1);

@@ -478,3 +478,161 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_win_tma_kernel(const __gr
 }
 
 }  // namespace adainf
+
+namespace adainf {
+
+// ------------------------------------------------------------------------------------------------
+// TMA weight-gradient GEMM for convs with Cin % 64 == 0 (any kernel size / stride / pad):
+//   dW[(tap, ci)][co] = sum_{positions} X[s*oh + kh - p][s*ow + kw - p][ci] * dZ[oh][ow][co]
+// K-blocks are R_k = 64 / Wp output rows of one image on a padded pitch Wp (power of two >= Wo).  Per
+// K-block and M tile (128 kconv = two (tap, 64-ci) atoms) the A atoms are TMA boxes {64 ci, Wp, R_k}
+// of X started at the tap's offset (element stride s; out-of-bounds -> 0) and the B atoms are boxes
+// {64 co, Wp, R_k} of dZ (positions x >= Wo are out of bounds -> 0, so they contribute nothing).  Both
+// land directly in the MN-major 128B-swizzled UMMA layout.  Split-K units write fp32 partials.
+struct WgTmaArgs {
+  CUtensorMap x_map;    // X [N][H][W][Cin], box {64, Wp, R_k} with element stride s
+  CUtensorMap dz_map;   // dZ [N][Ho][Wo][Cout], box {64, Wp, R_k}
+  int n, Ho, Wo, Wp, Rk, rg;  // rg = row groups per image = ceil(Ho / Rk)
+  int KW, stride, pad, ncb;   // ncb = Cin / 64
+  int Kconv, Cout;
+  int kb_per_split, splits;
+  float* out;           // partials [split][Kconv][Cout]
+  int stages;
+};
+
+template <int BN>
+__global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __grid_constant__ WgTmaArgs a) {
+  constexpr int A_BYTES = 16384, B_BYTES = BN * 128, STAGE = A_BYTES + B_BYTES;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  const int ST = a.stages;
+  uint64_t* full = (uint64_t*)(smem + ST * STAGE);
+  uint64_t* empty = full + 16;
+  uint64_t* tfull = empty + 16;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int mt = (a.Kconv + 127) / 128, nt = (a.Cout + BN - 1) / BN;
+  const int ntile = mt * nt * a.splits;
+  const int nkb = a.n * a.rg;
+  if ((int)blockIdx.x >= ntile) return;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < ST; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 128);
+    }
+    fence_mbar_init();
+    tma_prefetch_desc(&a.x_map);
+    tma_prefetch_desc(&a.dz_map);
+  }
+  if (warp == 4) tmem_alloc<2 * BN>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  const uint32_t sbase = smem_u32(smem);
+
+  if (warp == 0) {
+    if (lane == 0) {
+      int it = 0;
+      for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x) {
+        const int nb = tile % nt, r = tile / nt, m = r % mt, z = r / mt;
+        const int kb0 = z * a.kb_per_split, kb1 = min(kb0 + a.kb_per_split, nkb);
+        // the two A atoms of this M tile: (tap, ci block) = divmod(m*2 + i, ncb)
+        int ax[2], ay[2], ac[2];
+        bool av[2];
+        for (int i = 0; i < 2; ++i) {
+          const int at = m * 2 + i;
+          const int tap = at / a.ncb, cb = at - tap * a.ncb;
+          av[i] = at * 64 < a.Kconv;
+          ac[i] = cb * 64;
+          ax[i] = (tap % a.KW) - a.pad;
+          ay[i] = (tap / a.KW) - a.pad;
+        }
+        for (int kb = kb0; kb < kb1; ++kb, ++it) {
+          const int s = it % ST, u = it / ST;
+          if (u > 0) mbar_wait(&empty[s], (u - 1) & 1);
+          const int img = kb / a.rg, h0 = (kb - img * a.rg) * a.Rk;
+          const uint32_t sa = sbase + s * STAGE, sb = sa + A_BYTES;
+          const int nA = av[1] ? 2 : 1;
+          mbar_expect_tx(&full[s], nA * 8192 + (BN / 64) * 8192);
+          for (int i = 0; i < nA; ++i)
+            tma_load_4d(sa + i * 8192, &a.x_map, &full[s], ac[i], ax[i], h0 * a.stride + ay[i], img);
+#pragma unroll
+          for (int j = 0; j < BN / 64; ++j) tma_load_4d(sb + j * 8192, &a.dz_map, &full[s], nb * BN + j * 64, 0, h0, img);
+        }
+      }
+    }
+  } else if (warp == 4) {
+    constexpr uint32_t IDESC = make_idesc(BM, BN, 1, 1);
+    int it = 0, lt = 0;
+    for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++lt) {
+      const int r = tile / nt, z = r / mt;
+      const int kb0 = z * a.kb_per_split, kb1 = min(kb0 + a.kb_per_split, nkb);
+      const int b = lt & 1, ub = lt >> 1;
+      if (ub > 0) mbar_wait(&tempty[b], (ub - 1) & 1);
+      tc_fence_after();
+      const uint32_t dacc = tmem + (uint32_t)(b * BN);
+      for (int kb = kb0; kb < kb1; ++kb, ++it) {
+        const int s = it % ST, u = it / ST;
+        mbar_wait(&full[s], u & 1);
+        tc_fence_after();
+        if (lane == 0) {
+          const uint32_t sa = sbase + s * STAGE, sb = sa + A_BYTES;
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk)
+            umma_bf16(dacc, make_sdesc(sa + kk * 2048, 8192, 1024), make_sdesc(sb + kk * 2048, 8192, 1024), IDESC,
+                      (kb != kb0 || kk != 0));
+          umma_commit(&empty[s]);
+          if (kb == kb1 - 1) umma_commit(&tfull[b]);
+        }
+        __syncwarp();
+      }
+      if (kb1 <= kb0 && lane == 0) mbar_arrive(&tfull[b]);
+      __syncwarp();
+    }
+  } else if (warp >= 5) {
+    const int qd = warp & 3;
+    const int row = qd * 32 + lane;
+    int lt = 0;
+    for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++lt) {
+      const int nb = tile % nt, r = tile / nt, m = r % mt, z = r / mt;
+      const int kb0 = z * a.kb_per_split, kb1 = min(kb0 + a.kb_per_split, nkb);
+      const int b = lt & 1, ub = lt >> 1;
+      mbar_wait(&tfull[b], ub & 1);
+      tc_fence_after();
+      const uint32_t trow = tmem + (uint32_t)(b * BN) + ((uint32_t)(qd * 32) << 16);
+      const int kc = m * 128 + row;
+      float* outp = a.out + ((long long)z * a.Kconv + kc) * a.Cout + nb * BN;
+#pragma unroll 1
+      for (int c0 = 0; c0 < BN; c0 += 32) {
+        float v[32];
+        if (kb1 > kb0) tmem_ld32(trow + c0, v);
+        else
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = 0.f;
+        if (c0 + 32 >= BN) {
+          tc_fence_before();
+          mbar_arrive(&tempty[b]);
+        }
+        if (kc < a.Kconv && nb * BN + c0 < a.Cout)
+#pragma unroll
+          for (int i = 0; i < 32; i += 4) *(float4*)(outp + c0 + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+      }
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 4) {
+    tc_fence_after();
+    tmem_dealloc<2 * BN>(tmem);
+  }
+}
+
+}  // namespace adainf

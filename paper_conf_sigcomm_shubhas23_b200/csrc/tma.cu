@@ -21,12 +21,13 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   return fn;
 }
 
-CUtensorMap make_tmap_nhwc(const void* base, int N, int H, int W, int C, int bc, int bw, int bh) {
+// stride > 1: the box traverses W and H with that element stride (bw, bh are the ELEMENT counts loaded)
+CUtensorMap make_tmap_nhwc(const void* base, int N, int H, int W, int C, int bc, int bw, int bh, int stride) {
   CUtensorMap m;
   const cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
   const cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2, (cuuint64_t)H * W * C * 2};
-  const cuuint32_t box[4] = {(cuuint32_t)bc, (cuuint32_t)bw, (cuuint32_t)bh, 1};
-  const cuuint32_t es[4] = {1, 1, 1, 1};
+  const cuuint32_t box[4] = {(cuuint32_t)bc, (cuuint32_t)(bw * stride), (cuuint32_t)(bh * stride), 1};
+  const cuuint32_t es[4] = {1, (cuuint32_t)stride, (cuuint32_t)stride, 1};
   CUresult r = encode_fn()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(base), dims, strides, box, es,
                            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
                            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);

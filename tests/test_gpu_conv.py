@@ -115,7 +115,13 @@ def test_conv_dgrad_epilogue_terms():
     assert _rel(dx.float(), ref) < 8e-3
 
 
-@pytest.mark.parametrize("case", [c for c in FWD_CASES if c[4] % 8 == 0])
+# extra wgrad shapes for the TMA path: Wo up to 64 (Wp=64, one row per K-block), odd channel blocks
+# (a half-empty last M tile), stride-2 3x3 and 1x1 with ragged spatial tails
+WG_CASES = [(3, 56, 56, 64, 64, 3, 1, 1), (2, 28, 28, 128, 128, 3, 1, 1), (4, 29, 27, 192, 64, 3, 1, 1),
+            (2, 17, 17, 64, 128, 1, 2, 0), (3, 31, 29, 64, 128, 3, 2, 1), (2, 33, 64, 64, 256, 3, 1, 1)]
+
+
+@pytest.mark.parametrize("case", [c for c in FWD_CASES if c[4] % 8 == 0] + WG_CASES)
 def test_conv_wgrad_vs_torch(case):
     n, H, W, C, Co, K, s, p = case
     x, w, b = _mk(case, 7)

@@ -26,17 +26,21 @@ for (H, C, Co) in shapes:
 B.dbg_set_win_mode(1)
 # wgrad timing
 if os.environ.get("WGRAD", "1") == "1":
-    for (H, C, Co) in shapes:
+    wshapes = [(56, 64, 64, 3, 1), (28, 128, 128, 3, 1), (14, 256, 256, 3, 1), (7, 512, 512, 3, 1),
+               (56, 64, 128, 3, 2), (28, 128, 256, 3, 2), (14, 256, 512, 3, 2),
+               (56, 64, 128, 1, 2), (28, 128, 256, 1, 2), (14, 256, 512, 1, 2)]
+    for (H, C, Co, K, s) in wshapes:
+        Ho = (H + 2 * (K // 2) - K) // s + 1
         x = torch.randn(n, H, H, C, device="cuda").to(torch.bfloat16)
-        dz = torch.randn(n, H, H, Co, device="cuda").to(torch.bfloat16)
-        fl = 2 * n * H * H * Co * 9 * C
+        dz = torch.randn(n, Ho, Ho, Co, device="cuda").to(torch.bfloat16)
+        fl = 2 * n * Ho * Ho * Co * K * K * C
         for m in modes:
             B.dbg_set_win_mode(m)
-            B.dbg_conv_wgrad(x, dz, 3, 3, 1, 1); torch.cuda.synchronize()
+            B.dbg_conv_wgrad(x, dz, K, K, s, K // 2); torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
-            for _ in range(5): B.dbg_conv_wgrad(x, dz, 3, 3, 1, 1)
+            for _ in range(5): B.dbg_conv_wgrad(x, dz, K, K, s, K // 2)
             e1.record(); torch.cuda.synchronize()
             ms = e0.elapsed_time(e1) / 5
-            print(f"H={H:3d} C={C:3d} mode={m} wgrad  {ms*1e3:8.1f} us {fl/ms/1e9:7.1f} TFLOP/s (incl. reduce+colsum+alloc)", flush=True)
+            print(f"H={H:3d} C={C:3d} Co={Co:3d} K={K} s={s} mode={m} wgrad {ms*1e3:8.1f} us {fl/ms/1e9:7.1f} TFLOP/s (incl. reduce+colsum+alloc)", flush=True)
     B.dbg_set_win_mode(1)
