@@ -31,8 +31,14 @@ adainf_status adainf_dbg_conv_wgrad(const void* x, const void* dz, int32_t n, in
                                     int32_t Co, int32_t KH, int32_t KW, int32_t stride, int32_t pad, float* dw,
                                     float* db, adainf_stream_t stream);
 
-/* Conv kernel selection for A/B tests: 0 = generic gather kernel only, 1 = default routing (window
- * kernel for stride-1 3x3 dgrad at H <= 14), 2 = window kernel for every eligible stride-1 3x3 fwd/dgrad. */
+/* Conv kernel selection for A/B tests (process-wide, not thread-safe; tests restore 1):
+ *   0 = generic cp.async gather kernels only
+ *   1 = default routing (TMA window kernels for stride-1 3x3, TMA generic wgrad, cp.async elsewhere)
+ *   2 = window kernel for every eligible stride-1 3x3 fwd/dgrad
+ *   4 = cp.async warp-specialised window variant, no TMA
+ *   5 = no TMA weight-gradient kernels (cp.async window for 64x64 3x3, else generic)
+ *   6 = TMA generic weight gradient even where the window variant applies
+ *   7 = TMA window weight gradient forced for every eligible shape (any width) */
 adainf_status adainf_dbg_set_win_mode(int32_t mode);
 
 /* Launch accounting and per-kernel-class timing (CUDA events on the launching stream).

@@ -43,6 +43,17 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
+// one lane of a converged warp (elect.sync): the single-thread issue guard for tcgen05.mma / TMA
+__device__ __forceinline__ bool elect_one() {
+  uint32_t pred = 0;
+  asm volatile(
+      "{\n\t.reg .pred P;\n\t"
+      "elect.sync _|P, 0xffffffff;\n\t"
+      "selp.b32 %0, 1, 0, P;\n\t}"
+      : "=r"(pred));
+  return pred != 0;
+}
+
 // ---- optional role timing (compile with -DADAINF_TIMING): per-CTA cycle counters of barrier waits ----
 #ifdef ADAINF_TIMING
 __device__ unsigned long long g_wait_cycles[4096][8];

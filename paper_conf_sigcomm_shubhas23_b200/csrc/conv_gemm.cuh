@@ -369,7 +369,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
         mbar_wait(&full[s], u & 1);
         fence_proxy_async_smem();
         tc_fence_after();
-        if (lane == 0) {
+        if (elect_one()) {
           const uint32_t sa = smem_base + s * Cfg::STAGE_BYTES;
           const uint32_t sb = sa + Cfg::A_BYTES;
 #pragma unroll

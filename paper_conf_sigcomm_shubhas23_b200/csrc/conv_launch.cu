@@ -401,6 +401,25 @@ void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n
 }
 
 // partial [S][Kconv][Cout] -> dw [Cout][taps][cin_real] (fp32), summed over S in fixed order
+// stage 1 of the split-K reduction when there are many splits: group g sums splits [g*SG, (g+1)*SG) in
+// order (float4 per thread); stage 2 (wgrad_reduce_kernel) sums the groups in order and transposes.
+constexpr int WG_SG = 8;
+__global__ void wgrad_reduce_groups_kernel(const float4* __restrict__ part, int S, long long n4,
+                                           float4* __restrict__ out) {
+  const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n4) return;
+  const int s0 = blockIdx.y * WG_SG, s1 = min(S, s0 + WG_SG);
+  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int s = s0; s < s1; ++s) {
+    const float4 v = __ldg(part + (long long)s * n4 + i);
+    acc.x += v.x;
+    acc.y += v.y;
+    acc.z += v.z;
+    acc.w += v.w;
+  }
+  out[(long long)blockIdx.y * n4 + i] = acc;
+}
+
 __global__ void wgrad_reduce_kernel(const float* __restrict__ part, int S, int Kconv, int Cout, int cin_pad,
                                     int cin_real, float* __restrict__ dw) {
   __shared__ float tile[32][33];
@@ -474,31 +493,124 @@ static int wgrad_splits(int tiles, int nkb) {
   return std::max(1, std::min(nkb, num_sms() / tiles));
 }
 
-size_t wgrad_ws_bytes(const ConvGeom& g, int n) {
-  const long long npix = (long long)n * g.Ho * g.Wo;
-  const int nkb = (int)((npix + BK - 1) / BK);
-  const int Kconv = g.KH * g.KW * g.Cin;
-  const int BN = pick_bn(g.Cout, true);
-  const int tiles = ((Kconv + BM - 1) / BM) * ((g.Cout + BN - 1) / BN);
-  int S = wgrad_splits(tiles, nkb);
-  const int kbs = (nkb + S - 1) / S;
-  S = (nkb + kbs - 1) / kbs;
-  size_t need = (size_t)S * Kconv * g.Cout * sizeof(float) + (size_t)colsum_blocks(npix) * g.Cout * sizeof(float);
-  if (g.KH == 3 && g.KW == 3 && g.stride == 1 && g.Cin == 64 && g.Cout == 64)  // window variant
-    need = std::max(need, (size_t)num_sms() * 576 * 64 * 4 + (size_t)colsum_blocks(npix) * g.Cout * 4);
-  return need;
-}
+// Weight-gradient execution plan, shared by the workspace query and the launcher so both agree on the
+// split-K factor.  Paths: TMA window (stride-1 3x3, 64-aligned channels), TMA generic (64-aligned
+// channels, Wo <= 64), cp.async window (64x64 3x3, when TMA is disabled by the debug mode), generic.
+enum WgPath { WG_GENERIC = 0, WG_WIN_CPASYNC = 1, WG_TMA = 2, WG_WIN_TMA = 3 };
+struct WgPlan {
+  WgPath path;
+  int S, kbs, nkb, Kconv, tiles;
+  int BN;          // WG_TMA / WG_GENERIC
+  int Wp, R, rg;   // TMA paths
+};
 
 static bool win_wgrad_ok(const ConvGeom& g) {
   return win_mode() > 0 && g.KH == 3 && g.KW == 3 && g.stride == 1 && g.pad == 1 && g.Cin == 64 && g.Cout == 64 &&
          g.W <= 56 && g.H == g.Ho && g.W == g.Wo;
 }
+static bool tma_wgrad_allowed() { return win_mode() != 4 && win_mode() != 5; }
+static bool win_tma_wgrad_ok(const ConvGeom& g) {
+  return tma_wgrad_allowed() && win_mode() != 6 && g.KH == 3 && g.KW == 3 && g.stride == 1 && g.pad == 1 &&
+         g.Cin % 64 == 0 && g.Cout % 64 == 0 && g.H == g.Ho && g.W == g.Wo && g.W <= 127 &&
+         (g.W >= 14 || win_mode() == 7);  // below 14 columns the padded window wastes too much (mode 7 forces)
+}
+static bool wgrad_tma_ok(const ConvGeom& g) {
+  return tma_wgrad_allowed() && g.Cin % 64 == 0 && g.Cout % 64 == 0 && g.Wo <= 64 && g.stride <= 2;
+}
+
+static void finish_splits(WgPlan& p) {
+  p.S = wgrad_splits(p.tiles, p.nkb);
+  p.kbs = (p.nkb + p.S - 1) / p.S;
+  p.S = (p.nkb + p.kbs - 1) / p.kbs;
+}
+
+static int win_wg_stage_bytes(int Wp, int R) { return (16 + (R + 2) * Wp) * 128 + R * Wp * 128; }
+
+static WgPlan plan_wgrad(const ConvGeom& g, int n) {
+  WgPlan p{};
+  p.Kconv = g.KH * g.KW * g.Cin;
+  if (win_tma_wgrad_ok(g)) {
+    p.path = WG_WIN_TMA;
+    int Wp = 8;
+    while (Wp < g.W + 1) Wp <<= 1;
+    // R rows per K-block: K = R*Wp pixels a multiple of 16 and <= 256, >= 3 pipeline stages; least padded
+    // rows (R * ceil(H/R)) first, then the largest K
+    int bestR = 0;
+    long long best_rows = 0;
+    for (int R = 1; R * Wp <= 256; ++R) {
+      if ((R * Wp) % 16) continue;
+      if (3 * win_wg_stage_bytes(Wp, R) + 4096 > 225 * 1024) continue;
+      const long long rows = (long long)R * ((g.H + R - 1) / R);
+      if (!bestR || rows < best_rows || (rows == best_rows && R > bestR)) {
+        bestR = R;
+        best_rows = rows;
+      }
+    }
+    if (bestR) {
+      p.Wp = Wp;
+      p.R = bestR;
+      p.rg = (g.H + bestR - 1) / bestR;
+      p.nkb = n * p.rg;
+      p.tiles = (g.Cin / 64) * (g.Cout / 64);
+      finish_splits(p);
+      return p;
+    }
+  }
+  if (wgrad_tma_ok(g)) {
+    p.path = WG_TMA;
+    int Wp = 8;
+    while (Wp < g.Wo) Wp <<= 1;
+    p.Wp = Wp;
+    p.R = 64 / Wp;
+    p.rg = (g.Ho + p.R - 1) / p.R;
+    p.nkb = n * p.rg;
+    p.BN = g.Cout <= 64 ? 64 : (g.Cout <= 128 ? 128 : 256);
+    p.tiles = ((p.Kconv + 127) / 128) * ((g.Cout + p.BN - 1) / p.BN);
+    finish_splits(p);
+    return p;
+  }
+  if (win_wgrad_ok(g)) {
+    p.path = WG_WIN_CPASYNC;
+    const long long Q = (long long)n * (g.H + 1) * (g.W + 1);
+    p.nkb = (int)((Q + 63) / 64);
+    p.tiles = 1;
+    p.S = std::min(num_sms(), p.nkb);
+    p.kbs = (p.nkb + p.S - 1) / p.S;
+    p.S = (p.nkb + p.kbs - 1) / p.kbs;
+    return p;
+  }
+  p.path = WG_GENERIC;
+  const long long npix = (long long)n * g.Ho * g.Wo;
+  p.nkb = (int)((npix + BK - 1) / BK);
+  p.BN = pick_bn(g.Cout, true);
+  p.tiles = ((p.Kconv + BM - 1) / BM) * ((g.Cout + p.BN - 1) / p.BN);
+  finish_splits(p);
+  return p;
+}
+
+// workspace: [S][Kconv][Cout] split partials, then column-sum partials [max(S, colsum blocks)][Cout], then
+// the grouped partials [ceil(S / WG_SG)][Kconv][Cout] of the two-stage reduction
+static size_t wgrad_ws_floats(const WgPlan& p, const ConvGeom& g, int n, size_t* cs_off, size_t* grp_off) {
+  const long long npix = (long long)n * g.Ho * g.Wo;
+  const size_t kc = (size_t)p.Kconv * g.Cout;
+  const size_t a = (size_t)p.S * kc;
+  const size_t b = (size_t)std::max(p.S * ((p.Kconv + 127) / 128), colsum_blocks(npix)) * g.Cout;
+  const size_t grp = p.S > WG_SG ? (size_t)((p.S + WG_SG - 1) / WG_SG) * kc : 0;
+  if (cs_off) *cs_off = a;
+  if (grp_off) *grp_off = (a + b + 3) / 4 * 4;
+  return (a + b + 3) / 4 * 4 + grp;
+}
+
+size_t wgrad_ws_bytes(const ConvGeom& g, int n) {
+  const WgPlan p = plan_wgrad(g, n);
+  return wgrad_ws_floats(p, g, n, nullptr, nullptr) * sizeof(float);
+}
 
 template <int BN>
 static void launch_wgrad_tma_t(WgTmaArgs& a, cudaStream_t st) {
   constexpr int STAGE = 16384 + BN * 128;
-  a.stages = std::min(16, (225 * 1024 - 2048) / STAGE);
-  const int smem = a.stages * STAGE + 2048;
+  a.stages = std::min(16, (225 * 1024 - 5120) / STAGE);
+  const int smem = a.stages * STAGE + 2048 + 3072;
   static bool attr = false;
   if (!attr) {
     CK(cudaFuncSetAttribute(conv_wgrad_tma_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
@@ -511,74 +623,76 @@ static void launch_wgrad_tma_t(WgTmaArgs& a, cudaStream_t st) {
   CK(cudaGetLastError());
 }
 
-static bool wgrad_tma_ok(const ConvGeom& g) {
-  return win_mode() != 4 && win_mode() != 5 && g.Cin % 64 == 0 && g.Cout % 64 == 0 && g.Wo <= 64 && g.stride <= 2;
-}
-
 void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin_real, float* ws, size_t ws_bytes,
                 float* dw, float* db, cudaStream_t st) {
   check_extent((long long)n * (g.H + 1) * (g.W + 1));
-  if (wgrad_tma_ok(g)) {
+  const WgPlan p = plan_wgrad(g, n);
+  const long long npix = (long long)n * g.Ho * g.Wo;
+  size_t cs_off = 0, grp_off = 0;
+  if (wgrad_ws_floats(p, g, n, &cs_off, &grp_off) * sizeof(float) > ws_bytes)
+    throw std::runtime_error("wgrad workspace too small");
+  float* cs_part = ws + cs_off;
+  const bool fused_cs = db && (p.path == WG_WIN_TMA || p.path == WG_TMA);
+  if (db && (g.Cout % 8 || g.Cout / 8 > CS_THREADS)) throw ShapeError("colsum: Cout must be a multiple of 8, <= 2048");
+  const int S = p.S;
+
+  if (p.path == WG_WIN_TMA) {
+    static WinWgTmaArgs a;
+    a = WinWgTmaArgs{};
+    a.n = n;
+    a.H = g.H;
+    a.Wp = p.Wp;
+    a.R = p.R;
+    a.rg = p.rg;
+    a.ncb = g.Cin / 64;
+    a.nnb = g.Cout / 64;
+    a.Cin = g.Cin;
+    a.Cout = g.Cout;
+    a.kb_per_split = p.kbs;
+    a.splits = S;
+    a.out = ws;
+    a.a_bytes = (16 + (p.R + 2) * p.Wp) * 128;
+    a.cs_part = fused_cs ? cs_part : nullptr;
+    const int stage = win_wg_stage_bytes(p.Wp, p.R);
+    a.stages = std::min(8, (225 * 1024 - 7168) / stage);
+    const int smem = a.stages * stage + 2048 + 1024 + 256 + 3072;
+    a.x_map = make_tmap_nhwc(x, n, g.H, g.W, g.Cin, 64, p.Wp, p.R + 2);
+    a.dz_map = make_tmap_nhwc(dz, n, g.H, g.W, g.Cout, 64, p.Wp, p.R);
+    static bool attr = false;
+    if (!attr) {
+      CK(cudaFuncSetAttribute(conv_wgrad_win_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+      attr = true;
+    }
+    const int units = p.tiles * S;
+    ProfScope ps(PC_CONV_WGRAD, st);
+    conv_wgrad_win_tma_kernel<<<std::max(1, std::min(units, num_sms())), NUM_THREADS, smem, st>>>(a);
+    CK(cudaGetLastError());
+  } else if (p.path == WG_TMA) {
     static WgTmaArgs a;
     a = WgTmaArgs{};
-    int Wp = 8;
-    while (Wp < g.Wo) Wp <<= 1;
     a.n = n;
     a.Ho = g.Ho;
     a.Wo = g.Wo;
-    a.Wp = Wp;
-    a.Rk = 64 / Wp;
-    a.rg = (g.Ho + a.Rk - 1) / a.Rk;
+    a.Wp = p.Wp;
+    a.Rk = p.R;
+    a.rg = p.rg;
     a.KW = g.KW;
     a.stride = g.stride;
     a.pad = g.pad;
     a.ncb = g.Cin / 64;
-    a.Kconv = g.KH * g.KW * g.Cin;
+    a.Kconv = p.Kconv;
     a.Cout = g.Cout;
-    const int BN = g.Cout <= 64 ? 64 : (g.Cout <= 128 ? 128 : 256);
-    const int nkb = n * a.rg;
-    const int tiles = ((a.Kconv + 127) / 128) * ((g.Cout + BN - 1) / BN);
-    int S = wgrad_splits(tiles, nkb);
-    const int kbs = (nkb + S - 1) / S;
-    S = (nkb + kbs - 1) / kbs;
-    a.kb_per_split = kbs;
+    a.kb_per_split = p.kbs;
     a.splits = S;
-    if ((size_t)S * a.Kconv * g.Cout * 4 + (size_t)colsum_blocks((long long)n * g.Ho * g.Wo) * g.Cout * 4 > ws_bytes)
-      throw std::runtime_error("wgrad workspace too small (tma)");
     a.out = ws;
-    a.x_map = make_tmap_nhwc(x, n, g.H, g.W, g.Cin, 64, Wp, a.Rk, g.stride);
-    a.dz_map = make_tmap_nhwc(dz, n, g.Ho, g.Wo, g.Cout, 64, Wp, a.Rk, 1);
-    if (BN == 64) launch_wgrad_tma_t<64>(a, st);
-    else if (BN == 128) launch_wgrad_tma_t<128>(a, st);
+    a.cs_part = fused_cs ? cs_part : nullptr;
+    a.x_map = make_tmap_nhwc(x, n, g.H, g.W, g.Cin, 64, p.Wp, p.R, g.stride);
+    a.dz_map = make_tmap_nhwc(dz, n, g.Ho, g.Wo, g.Cout, 64, p.Wp, p.R, 1);
+    if (p.BN == 64) launch_wgrad_tma_t<64>(a, st);
+    else if (p.BN == 128) launch_wgrad_tma_t<128>(a, st);
     else launch_wgrad_tma_t<256>(a, st);
-    {
-      dim3 rg((a.Kconv + 31) / 32, (g.Cout + 31) / 32);
-      ProfScope ps(PC_WGRAD_REDUCE, st);
-      wgrad_reduce_kernel<<<rg, dim3(32, 8), 0, st>>>(ws, S, a.Kconv, g.Cout, g.Cin, cin_real, dw);
-      CK(cudaGetLastError());
-    }
-    if (db) {
-      const long long npix = (long long)n * g.Ho * g.Wo;
-      float* part = ws + (size_t)S * a.Kconv * g.Cout;
-      const int nb = colsum_blocks(npix);
-      const long long rpb = (npix + nb - 1) / nb;
-      const int groups = CS_THREADS / (g.Cout / 8);
-      ProfScope ps(PC_BIAS_COLSUM, st, 2);
-      colsum_partial_kernel<<<nb, CS_THREADS, (size_t)groups * g.Cout * 4, st>>>(dz, npix, g.Cout, rpb, part);
-      colsum_final_kernel<<<(g.Cout + 127) / 128, 128, 0, st>>>(part, nb, g.Cout, db);
-      CK(cudaGetLastError());
-    }
-    return;
-  }
-  if (win_wgrad_ok(g)) {
+  } else if (p.path == WG_WIN_CPASYNC) {
     // one K-range of 64-position blocks per persistent CTA; partials [S][576][64] reduced in fixed order
-    const long long Q = (long long)n * (g.H + 1) * (g.W + 1);
-    const int nkb = (int)((Q + 63) / 64);
-    int S = std::min(num_sms(), nkb);
-    const int kbs = (nkb + S - 1) / S;
-    S = (nkb + kbs - 1) / kbs;
-    if ((size_t)S * 576 * 64 * 4 + (size_t)colsum_blocks((long long)n * g.Ho * g.Wo) * g.Cout * 4 > ws_bytes)
-      throw std::runtime_error("wgrad workspace too small (window)");
     WinArgs w{};
     w.c.src = x;
     w.c.Hs = g.H;
@@ -588,7 +702,7 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
     w.c.B = dz;
     w.c.Nout = 64;
     w.c.out = ws;
-    w.c.kb_per_split = kbs;
+    w.c.kb_per_split = p.kbs;
     for (int kh = 0; kh < 3; ++kh)
       for (int kw = 0; kw < 3; ++kw) w.tap_off[kh * 3 + kw] = kh * (g.W + 1) + kw;
     static bool attr = false;
@@ -596,76 +710,59 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
       CK(cudaFuncSetAttribute(conv_win_wgrad_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, WinWgCfg::SMEM));
       attr = true;
     }
-    {
-      ProfScope ps(PC_CONV_WGRAD, st);
-      conv_win_wgrad_kernel<<<S, NUM_THREADS, WinWgCfg::SMEM, st>>>(w);
-      CK(cudaGetLastError());
-    }
-    {
-      dim3 rg((576 + 31) / 32, 2);
-      ProfScope ps(PC_WGRAD_REDUCE, st);
-      wgrad_reduce_kernel<<<rg, dim3(32, 8), 0, st>>>(ws, S, 576, 64, 64, cin_real, dw);
-      CK(cudaGetLastError());
-    }
-    if (db) {
-      const long long npix = (long long)n * g.Ho * g.Wo;
-      float* part = ws + (size_t)S * 576 * 64;
-      const int nb = colsum_blocks(npix);
-      const long long rpb = (npix + nb - 1) / nb;
-      const int groups = CS_THREADS / (g.Cout / 8);
-      ProfScope ps(PC_BIAS_COLSUM, st, 2);
-      colsum_partial_kernel<<<nb, CS_THREADS, (size_t)groups * g.Cout * 4, st>>>(dz, npix, g.Cout, rpb, part);
-      colsum_final_kernel<<<(g.Cout + 127) / 128, 128, 0, st>>>(part, nb, g.Cout, db);
-      CK(cudaGetLastError());
-    }
-    return;
+    ProfScope ps(PC_CONV_WGRAD, st);
+    conv_win_wgrad_kernel<<<S, NUM_THREADS, WinWgCfg::SMEM, st>>>(w);
+    CK(cudaGetLastError());
+  } else {
+    ConvArgs a{};
+    a.src = x;
+    a.Hs = g.H;
+    a.Ws = g.W;
+    a.Cs = g.Cin;
+    a.n_static = n;
+    a.Hg = g.Ho;
+    a.Wg = g.Wo;
+    a.sy = a.sx = g.stride;
+    a.ntaps = g.KH * g.KW;
+    for (int kh = 0; kh < g.KH; ++kh)
+      for (int kw = 0; kw < g.KW; ++kw) {
+        a.ty[kh * g.KW + kw] = (int8_t)(kh - g.pad);
+        a.tx[kh * g.KW + kw] = (int8_t)(kw - g.pad);
+      }
+    a.B = dz;
+    a.K = p.Kconv;
+    a.Nout = g.Cout;
+    a.out = ws;
+    a.kb_per_split = p.kbs;
+    a.splits = S;
+    launch_bn<MODE_WGRAD>(p.BN, a, (long long)p.tiles * S, st);
   }
-  const long long npix = (long long)n * g.Ho * g.Wo;
-  const int nkb = (int)((npix + BK - 1) / BK);
-  const int Kconv = g.KH * g.KW * g.Cin;
-  const int BN = pick_bn(g.Cout, true);
-  const int tiles = ((Kconv + BM - 1) / BM) * ((g.Cout + BN - 1) / BN);
-  int S = wgrad_splits(tiles, nkb);
-  const int kbs = (nkb + S - 1) / S;
-  S = (nkb + kbs - 1) / kbs;
-  if (wgrad_ws_bytes(g, n) > ws_bytes) throw std::runtime_error("wgrad workspace too small");
-  ConvArgs a{};
-  a.src = x;
-  a.Hs = g.H;
-  a.Ws = g.W;
-  a.Cs = g.Cin;
-  a.n_static = n;
-  a.Hg = g.Ho;
-  a.Wg = g.Wo;
-  a.sy = a.sx = g.stride;
-  a.ntaps = g.KH * g.KW;
-  for (int kh = 0; kh < g.KH; ++kh)
-    for (int kw = 0; kw < g.KW; ++kw) {
-      a.ty[kh * g.KW + kw] = (int8_t)(kh - g.pad);
-      a.tx[kh * g.KW + kw] = (int8_t)(kw - g.pad);
-    }
-  a.B = dz;
-  a.K = Kconv;
-  a.Nout = g.Cout;
-  a.out = ws;
-  a.kb_per_split = kbs;
-  a.splits = S;
-  launch_bn<MODE_WGRAD>(BN, a, (long long)tiles * S, st);
-  dim3 rg((Kconv + 31) / 32, (g.Cout + 31) / 32);
   {
-  ProfScope ps(PC_WGRAD_REDUCE, st);
-  wgrad_reduce_kernel<<<rg, dim3(32, 8), 0, st>>>(ws, S, Kconv, g.Cout, g.Cin, cin_real, dw);
-  CK(cudaGetLastError());
+    ProfScope ps(PC_WGRAD_REDUCE, st, S > WG_SG ? 2 : 1);
+    const float* src = ws;
+    int S2 = S;
+    if (S > WG_SG) {
+      const long long n4 = (long long)p.Kconv * g.Cout / 4;  // Cout % 8 == 0
+      const int G = (S + WG_SG - 1) / WG_SG;
+      dim3 gg((unsigned)((n4 + 255) / 256), G);
+      wgrad_reduce_groups_kernel<<<gg, 256, 0, st>>>((const float4*)ws, S, n4, (float4*)(ws + grp_off));
+      src = ws + grp_off;
+      S2 = G;
+    }
+    dim3 rg((p.Kconv + 31) / 32, (g.Cout + 31) / 32);
+    wgrad_reduce_kernel<<<rg, dim3(32, 8), 0, st>>>(src, S2, p.Kconv, g.Cout, g.Cin, cin_real, dw);
+    CK(cudaGetLastError());
   }
   if (db) {
-    float* part = ws + (size_t)S * Kconv * g.Cout;
-    const int nb = colsum_blocks(npix);
-    const long long rpb = (npix + nb - 1) / nb;
-    if (g.Cout % 8 || g.Cout / 8 > CS_THREADS) throw ShapeError("colsum: Cout must be a multiple of 8, <= 2048");
-    const int groups = CS_THREADS / (g.Cout / 8);
-    ProfScope ps(PC_BIAS_COLSUM, st, 2);
-    colsum_partial_kernel<<<nb, CS_THREADS, (size_t)groups * g.Cout * 4, st>>>(dz, npix, g.Cout, rpb, part);
-    colsum_final_kernel<<<(g.Cout + 127) / 128, 128, 0, st>>>(part, nb, g.Cout, db);
+    ProfScope ps(PC_BIAS_COLSUM, st, fused_cs ? 1 : 2);
+    int nb = p.path == WG_TMA ? S * ((p.Kconv + 127) / 128) : S;  // fused partial rows
+    if (!fused_cs) {
+      nb = colsum_blocks(npix);
+      const long long rpb = (npix + nb - 1) / nb;
+      const int groups = CS_THREADS / (g.Cout / 8);
+      colsum_partial_kernel<<<nb, CS_THREADS, (size_t)groups * g.Cout * 4, st>>>(dz, npix, g.Cout, rpb, cs_part);
+    }
+    colsum_final_kernel<<<(g.Cout + 127) / 128, 128, 0, st>>>(cs_part, nb, g.Cout, db);
     CK(cudaGetLastError());
   }
 }

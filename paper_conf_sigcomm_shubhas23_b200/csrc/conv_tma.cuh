@@ -131,7 +131,7 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
       const int s = it % WS, u = it / WS;
       mbar_wait(&wfull[s], u & 1);
       tc_fence_after();
-      if (lane == 0) {
+      if (elect_one()) {
         const uint32_t sw = wsm + s * a.win_bytes;
         const uint32_t dacc = tmem + (uint32_t)(b * 64);
 #pragma unroll 1
@@ -373,7 +373,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_win_tma_kernel(const __gr
           const int bs = bit % BS, bu = bit / BS;
           mbar_wait(&bfull[bs], bu & 1);
           tc_fence_after();
-          if (lane == 0) {
+          if (elect_one()) {
             const uint32_t sb = bsm + bs * B_BYTES;
 #pragma unroll
             for (int kk = 0; kk < 4; ++kk) {
@@ -481,6 +481,66 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_win_tma_kernel(const __gr
 
 namespace adainf {
 
+// Bias gradient fused into the weight-gradient pipeline: warps 1-3 (idle otherwise) sum the columns of
+// every dZ tile while it sits in shared memory, so dZ is not read a second time from HBM.  Tile layout is
+// the MN-major 128B-swizzled one TMA writes: row = pixel, 64 channels per 128-byte row, 16-byte chunk j of
+// row r stored at chunk j ^ (r & 7); atoms of 64 channels are 8192 B apart (64-row atoms) when the tile is
+// wider than 64.  Each thread owns one 8-channel chunk column and a strided subset of rows; the per-thread
+// sums are combined in a fixed order at the end of the unit (deterministic).
+constexpr int CS_WORKERS = 96;
+template <int BN>
+struct TileColsum {
+  static constexpr int NCH = BN / 8, NPH = CS_WORKERS / NCH;
+  float acc[8];
+  int cc, ph;
+  __device__ __forceinline__ void init(int t) {
+    cc = t % NCH;
+    ph = t / NCH;
+  }
+  __device__ __forceinline__ void zero() {
+#pragma unroll
+    for (int q = 0; q < 8; ++q) acc[q] = 0.f;
+  }
+  // rows: valid rows per 64-channel atom (64 for the generic path, R*Wp for the window path)
+  __device__ __forceinline__ void add(const uint8_t* tile, int rows) {
+    if (ph >= NPH) return;
+    const uint8_t* at = tile + (cc >> 3) * 8192;
+    const int j = cc & 7;
+    // four rows per batch: independent shared loads in flight before the adds
+    for (int r0 = ph; r0 < rows; r0 += 4 * NPH) {
+      uint4 raw[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int r = r0 + i * NPH;
+        raw[i] = r < rows ? *(const uint4*)(at + r * 128 + ((j ^ (r & 7)) << 4)) : make_uint4(0, 0, 0, 0);
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const __nv_bfloat162* h = (const __nv_bfloat162*)&raw[i];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const float2 f = __bfloat1622float2(h[q]);
+          acc[2 * q] += f.x;
+          acc[2 * q + 1] += f.y;
+        }
+      }
+    }
+  }
+  // combine the NPH row phases (fixed order) and write `lim` (<= BN) channel sums to out
+  __device__ __forceinline__ void finish(float* red, float* out, int lim, int t) {
+    if (ph < NPH)
+#pragma unroll
+      for (int q = 0; q < 8; ++q) red[ph * BN + cc * 8 + q] = acc[q];
+    asm volatile("bar.sync 1, %0;" ::"n"(CS_WORKERS) : "memory");
+    for (int ch = t; ch < BN; ch += CS_WORKERS) {
+      float s = 0.f;
+      for (int p = 0; p < NPH; ++p) s += red[p * BN + ch];
+      if (ch < lim) out[ch] = s;
+    }
+    asm volatile("bar.sync 1, %0;" ::"n"(CS_WORKERS) : "memory");
+  }
+};
+
 // ------------------------------------------------------------------------------------------------
 // TMA weight-gradient GEMM for convs with Cin % 64 == 0 (any kernel size / stride / pad):
 //   dW[(tap, ci)][co] = sum_{positions} X[s*oh + kh - p][s*ow + kw - p][ci] * dZ[oh][ow][co]
@@ -497,6 +557,7 @@ struct WgTmaArgs {
   int Kconv, Cout;
   int kb_per_split, splits;
   float* out;           // partials [split][Kconv][Cout]
+  float* cs_part;       // bias-gradient partials [split][Cout] (nullptr: not fused)
   int stages;
 };
 
@@ -511,6 +572,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
   uint64_t* tfull = empty + 16;
   uint64_t* tempty = tfull + 2;
   uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+  float* cs_red = (float*)((uint8_t*)full + 512);  // [NPH][BN] column-sum combine scratch (3 KB)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int mt = (a.Kconv + 127) / 128, nt = (a.Cout + BN - 1) / BN;
@@ -520,7 +582,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
   if (threadIdx.x == 0) {
     for (int s = 0; s < ST; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&empty[s], 1);
+      mbar_init(&empty[s], a.cs_part ? 4 : 1);  // MMA commit (+ one arrive per column-sum warp)
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&tfull[b], 1);
@@ -582,7 +644,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
         const int s = it % ST, u = it / ST;
         mbar_wait(&full[s], u & 1);
         tc_fence_after();
-        if (lane == 0) {
+        if (elect_one()) {
           const uint32_t sa = sbase + s * STAGE, sb = sa + A_BYTES;
 #pragma unroll
           for (int kk = 0; kk < 4; ++kk)
@@ -595,6 +657,28 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
       }
       if (kb1 <= kb0 && lane == 0) mbar_arrive(&tfull[b]);
       __syncwarp();
+    }
+  } else if (warp >= 1 && warp <= 3) {
+    if (a.cs_part) {
+      // fused bias gradient: the mt M tiles of one (co block, split) see the same dZ K-blocks; M tile m
+      // sums the K-blocks with kb % mt == m into partial row z * mt + m
+      TileColsum<BN> cs;
+      const int t = threadIdx.x - 32;
+      cs.init(t);
+      int it = 0;
+      for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x) {
+        const int nb = tile % nt, r = tile / nt, m = r % mt, z = r / mt;
+        const int kb0 = z * a.kb_per_split, kb1 = min(kb0 + a.kb_per_split, nkb);
+        cs.zero();
+        for (int kb = kb0; kb < kb1; ++kb, ++it) {
+          const int s = it % ST, u = it / ST;
+          mbar_wait(&full[s], u & 1);
+          if (kb % mt == m) cs.add(smem + s * STAGE + A_BYTES, 64);
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&empty[s]);
+        }
+        cs.finish(cs_red, a.cs_part + ((long long)z * mt + m) * a.Cout + nb * BN, a.Cout - nb * BN, t);
+      }
     }
   } else if (warp >= 5) {
     const int qd = warp & 3;
@@ -632,6 +716,197 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
   if (warp == 4) {
     tc_fence_after();
     tmem_dealloc<2 * BN>(tmem);
+  }
+}
+
+
+// ---- window weight gradient (stride-1 3x3, pad 1), TMA-fed --------------------------------------------
+// dW[tap][ci][co] = sum_pix X(pix + tap) * dZ(pix).  K = output pixels of R rows of one image on a padded
+// grid of Wp (>= W+1) columns; the X window (R+2 rows, 8 zero rows before and after) serves all nine taps
+// as row-shifted MN-major A operands, so each dZ tile is loaded once for 9 taps.  M = (tap pair, 64 ci):
+// five TMEM accumulators of 128 x 64 (the tenth slot reads a zero atom), N = 64 co.
+struct WinWgTmaArgs {
+  CUtensorMap x_map;    // X [N][H][W][Cin], box {64, Wp, R+2, 1}
+  CUtensorMap dz_map;   // dZ [N][H][W][Cout], box {64, Wp, R, 1}
+  int n, H, Wp, R, rg;  // rg = ceil(H / R) row groups per image
+  int ncb, nnb, Cin, Cout;
+  int kb_per_split, splits;
+  float* out;           // partials [split][9*Cin][Cout]
+  float* cs_part;       // bias-gradient partials [split][Cout] (nullptr: not fused)
+  int stages, a_bytes;  // a_bytes = (16 + (R+2)*Wp) * 128
+};
+
+__global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_win_tma_kernel(const __grid_constant__ WinWgTmaArgs a) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  const int ST = a.stages, Wp = a.Wp, R = a.R;
+  const int b_bytes = R * Wp * 128;
+  const int stage_bytes = a.a_bytes + b_bytes;
+  uint8_t* zero = smem + ST * stage_bytes;
+  uint64_t* full = (uint64_t*)(zero + 2048);
+  uint64_t* empty = full + 8;
+  uint64_t* tfull = empty + 8;
+  uint64_t* tempty = tfull + 1;
+  uint32_t* tmem_slot = (uint32_t*)(tempty + 1);
+  float* cs_red = (float*)(zero + 2048 + 256);  // [12][64] column-sum combine scratch (3 KB)
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int tiles = a.ncb * a.nnb;
+  const int nunit = tiles * a.splits;
+  const int nkb = a.n * a.rg;
+  if ((int)blockIdx.x >= nunit) return;
+  // zero: 8 lead + 8 trail rows of every A stage, and the zero atom
+  const int wrows = 8 + (R + 2) * Wp;
+  for (int i = threadIdx.x; i < ST * 128 + 128; i += blockDim.x) {
+    const int s = i / 128, k = i % 128;
+    uint8_t* d = s < ST ? smem + s * stage_bytes + (k < 64 ? k * 16 : wrows * 128 + (k - 64) * 16) : zero + k * 16;
+    *(uint4*)d = make_uint4(0, 0, 0, 0);
+  }
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < ST; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], a.cs_part ? 4 : 1);  // MMA commit (+ one arrive per column-sum warp)
+    }
+    mbar_init(tfull, 1);
+    mbar_init(tempty, 128);
+    fence_mbar_init();
+    tma_prefetch_desc(&a.x_map);
+    tma_prefetch_desc(&a.dz_map);
+  }
+  if (warp == 4) tmem_alloc<512>(tmem_slot);
+  fence_proxy_async_smem();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  const uint32_t sbase = smem_u32(smem);
+
+  if (warp == 0) {
+    if (lane == 0) {
+      const uint32_t xbytes = 64u * 2u * Wp * (R + 2), zbytes = (uint32_t)b_bytes;
+      int it = 0;
+      for (int u = blockIdx.x; u < nunit; u += gridDim.x) {
+        const int t = u % tiles, z = u / tiles;
+        const int cb = t % a.ncb, nb = t / a.ncb;
+        const int kb0 = z * a.kb_per_split, kb1 = min(kb0 + a.kb_per_split, nkb);
+        for (int kb = kb0; kb < kb1; ++kb, ++it) {
+          const int s = it % ST, ph = it / ST;
+          if (ph > 0) mbar_wait(&empty[s], (ph - 1) & 1);
+          const int img = kb / a.rg, h0 = (kb - img * a.rg) * R;
+          const uint32_t sa = sbase + s * stage_bytes;
+          mbar_expect_tx(&full[s], xbytes + zbytes);
+          tma_load_4d(sa + 1024, &a.x_map, &full[s], cb * 64, 0, h0 - 1, img);
+          tma_load_4d(sa + a.a_bytes, &a.dz_map, &full[s], nb * 64, 0, h0, img);
+        }
+      }
+    }
+  } else if (warp == 4) {
+    constexpr uint32_t IDESC = make_idesc(BM, 64, 1, 1);
+    const uint32_t zaddr = smem_u32(zero);
+    const int ksteps = R * Wp / 16;
+    int off[10];
+#pragma unroll
+    for (int tp = 0; tp < 9; ++tp) off[tp] = (8 + (tp / 3) * Wp + (tp % 3) - 1) * 128;
+    int it = 0, lt = 0;
+    for (int u = blockIdx.x; u < nunit; u += gridDim.x, ++lt) {
+      const int z = u / tiles;
+      const int kb0 = z * a.kb_per_split, kb1 = min(kb0 + a.kb_per_split, nkb);
+      if (lt > 0) mbar_wait(tempty, (lt - 1) & 1);
+      tc_fence_after();
+      for (int kb = kb0; kb < kb1; ++kb, ++it) {
+        const int s = it % ST, ph = it / ST;
+        mbar_wait(&full[s], ph & 1);
+        tc_fence_after();
+        if (elect_one()) {
+          const uint32_t sa = sbase + s * stage_bytes, sb = sa + a.a_bytes;
+          // descriptors for K-step 0; each further K-step (16 pixel rows = 2048 B) adds 128 to the address field
+          uint64_t da[5];
+#pragma unroll
+          for (int p = 0; p < 5; ++p) {
+            const uint32_t a0 = sa + off[2 * p];
+            const uint32_t a1 = p < 4 ? sa + off[2 * p + 1] : zaddr;
+            da[p] = make_sdesc(a0, a1 - a0, 1024);
+          }
+          const uint64_t db0 = make_sdesc(sb, 8192, 1024);
+          const uint32_t acc0 = kb != kb0;
+#pragma unroll
+          for (int p = 0; p < 5; ++p) umma_bf16(tmem + (uint32_t)(p * 64), da[p], db0, IDESC, acc0);
+          for (int kk = 1; kk < ksteps; ++kk) {
+            const uint64_t inc = (uint64_t)(kk * 128);
+#pragma unroll
+            for (int p = 0; p < 4; ++p) umma_bf16(tmem + (uint32_t)(p * 64), da[p] + inc, db0 + inc, IDESC, 1u);
+            // the tenth atom (zero) stays in place: LBO shrinks by the same 2048 B per K-step
+            umma_bf16(tmem + 256u, da[4] + inc - ((uint64_t)(kk * 128) << 16), db0 + inc, IDESC, 1u);
+          }
+          umma_commit(&empty[s]);
+          if (kb == kb1 - 1) umma_commit(tfull);
+        }
+        __syncwarp();
+      }
+      if (kb1 <= kb0 && lane == 0) mbar_arrive(tfull);
+      __syncwarp();
+    }
+  } else if (warp >= 1 && warp <= 3) {
+    if (a.cs_part) {
+      // fused bias gradient: tiles with cb == 0 see every (pixel, co) of their co block exactly once
+      TileColsum<64> cs;
+      const int t = threadIdx.x - 32;
+      cs.init(t);
+      int it = 0;
+      for (int u = blockIdx.x; u < nunit; u += gridDim.x) {
+        const int tl = u % tiles, z = u / tiles;
+        const int cb = tl % a.ncb, nb = tl / a.ncb;
+        const int kb0 = z * a.kb_per_split, kb1 = min(kb0 + a.kb_per_split, nkb);
+        cs.zero();
+        for (int kb = kb0; kb < kb1; ++kb, ++it) {
+          const int s = it % ST, ph = it / ST;
+          mbar_wait(&full[s], ph & 1);
+          if (cb == 0) cs.add(smem + s * stage_bytes + a.a_bytes, R * Wp);
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&empty[s]);
+        }
+        if (cb == 0) cs.finish(cs_red, a.cs_part + (long long)z * a.Cout + nb * 64, 64, t);
+      }
+    }
+  } else if (warp >= 5) {
+    const int qd = warp & 3;
+    const int row = qd * 32 + lane;
+    const int Kconv = 9 * a.Cin;
+    int lt = 0;
+    for (int u = blockIdx.x; u < nunit; u += gridDim.x, ++lt) {
+      const int t = u % tiles, z = u / tiles;
+      const int cb = t % a.ncb, nb = t / a.ncb;
+      const int kb0 = z * a.kb_per_split, kb1 = min(kb0 + a.kb_per_split, nkb);
+      mbar_wait(tfull, lt & 1);
+      tc_fence_after();
+      const uint32_t trow = tmem + ((uint32_t)(qd * 32) << 16);
+#pragma unroll 1
+      for (int p = 0; p < 5; ++p) {
+        const int tap = 2 * p + (row >> 6);
+        const int kc = tap * a.Cin + cb * 64 + (row & 63);
+        float* outp = a.out + ((long long)z * Kconv + kc) * a.Cout + nb * 64;
+#pragma unroll 1
+        for (int c0 = 0; c0 < 64; c0 += 32) {
+          float v[32];
+          if (kb1 > kb0) tmem_ld32(trow + p * 64 + c0, v);
+          else
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] = 0.f;
+          if (tap < 9)
+#pragma unroll
+            for (int i = 0; i < 32; i += 4) *(float4*)(outp + c0 + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(tempty);
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 4) {
+    tc_fence_after();
+    tmem_dealloc<512>(tmem);
   }
 }
 

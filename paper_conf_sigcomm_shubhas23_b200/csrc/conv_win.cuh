@@ -195,7 +195,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_win_kernel(const WinArgs 
           mbar_wait(&bfull[s], u & 1);
           fence_proxy_async_smem();
           tc_fence_after();
-          if (lane == 0) {
+          if (elect_one()) {
             const uint32_t sb = bsm + s * Cfg::B_BYTES;
 #pragma unroll
             for (int kk = 0; kk < 4; ++kk) {
@@ -468,7 +468,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1) conv_win_ws_kernel(const WinArg
       TIMED_WAIT(2, mbar_wait(&wfull[s], u & 1));
       fence_proxy_async_smem();
       tc_fence_after();
-      if (lane == 0) {
+      if (elect_one()) {
         const uint32_t sw = wsm + s * Cfg::WIN_BYTES;
 #pragma unroll 1
         for (int tp = 0; tp < 9; ++tp) {
@@ -737,7 +737,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_win_wgrad_kernel(const Wi
       mbar_wait(&full[s], u & 1);
       fence_proxy_async_smem();
       tc_fence_after();
-      if (lane == 0) {
+      if (elect_one()) {
         const uint32_t sw = sbase + s * Cfg::STAGE_BYTES;
         const uint32_t sb = sw + Cfg::WIN_BYTES;
 #pragma unroll

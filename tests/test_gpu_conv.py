@@ -167,3 +167,25 @@ def test_window_kernel_fwd_dgrad(case, mode):
         assert _rel(dx.float(), refd) < 8e-3, ("dgrad", mode)
     finally:
         B.dbg_set_win_mode(1)
+
+
+@pytest.mark.parametrize("mode", [1, 5, 6, 7])
+@pytest.mark.parametrize("case", WIN_CASES)
+def test_window_wgrad(case, mode):
+    """Stride-1 3x3 weight gradient through each routing: 1 = default (TMA window from 14 columns up, else
+    TMA generic), 7 = TMA window forced (nine taps from one X window), 6 = TMA generic (one tap pair per
+    M tile), 5 = no TMA (cp.async window for 64x64, else generic).  The bias gradient is fused into the
+    TMA kernels and a separate pass otherwise."""
+    n, H, W, C, Co = case
+    B.dbg_set_win_mode(mode)
+    try:
+        x, _, _ = _mk((n, H, W, C, Co, 3, 1, 1), 12)
+        dz = torch.randn(n, H, W, Co).to(torch.bfloat16).cuda()
+        ref = torch.nn.grad.conv2d_weight(x.float().permute(0, 3, 1, 2), (Co, C, 3, 3), dz.float().permute(0, 3, 1, 2),
+                                          stride=1, padding=1).permute(0, 2, 3, 1)
+        dw, db = B.dbg_conv_wgrad(x, dz, 3, 3, 1, 1)
+        torch.cuda.synchronize()
+        assert _rel(dw, ref) < 1e-4, mode
+        assert _rel(db, dz.float().sum(dim=(0, 1, 2))) < 1e-5
+    finally:
+        B.dbg_set_win_mode(1)

@@ -6,7 +6,7 @@ from paper_conf_sigcomm_shubhas23_b200 import binding as B
 n = int(os.environ.get("N", "1024"))
 modes = [int(m) for m in os.environ.get("MODES", "0,1").split(",")]
 shapes = [(56, 64, 64), (28, 128, 128), (14, 256, 256), (7, 512, 512)]
-for (H, C, Co) in shapes:
+for (H, C, Co) in (shapes if os.environ.get("FWD", "1") == "1" else []):
     x = torch.randn(n, H, H, C, device="cuda").to(torch.bfloat16)
     w = (torch.randn(Co, 3, 3, C, device="cuda") * 0.05).to(torch.bfloat16)
     b = torch.zeros(Co, device="cuda")
@@ -37,10 +37,13 @@ if os.environ.get("WGRAD", "1") == "1":
         for m in modes:
             B.dbg_set_win_mode(m)
             B.dbg_conv_wgrad(x, dz, K, K, s, K // 2); torch.cuda.synchronize()
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record()
+            B.prof_enable(True); B.prof_reset()
             for _ in range(5): B.dbg_conv_wgrad(x, dz, K, K, s, K // 2)
-            e1.record(); torch.cuda.synchronize()
-            ms = e0.elapsed_time(e1) / 5
-            print(f"H={H:3d} C={C:3d} Co={Co:3d} K={K} s={s} mode={m} wgrad {ms*1e3:8.1f} us {fl/ms/1e9:7.1f} TFLOP/s (incl. reduce+colsum+alloc)", flush=True)
+            torch.cuda.synchronize()
+            q = B.prof_query(); B.prof_enable(False)
+            ms = q["conv_wgrad"][1] / 5
+            red = q.get("wgrad_reduce", (0, 0.0))[1] / 5
+            cs = q.get("bias_colsum", (0, 0.0))[1] / 5
+            print(f"H={H:3d} C={C:3d} Co={Co:3d} K={K} s={s} mode={m} wgrad {ms*1e3:8.1f} us {fl/ms/1e9:7.1f} TFLOP/s"
+                  f"  reduce {red*1e3:6.1f} us  colsum {cs*1e3:6.1f} us", flush=True)
     B.dbg_set_win_mode(1)
