@@ -38,8 +38,22 @@ adainf_status adainf_dbg_conv_wgrad(const void* x, const void* dz, int32_t n, in
  *   4 = cp.async warp-specialised window variant, no TMA
  *   5 = no TMA weight-gradient kernels (cp.async window for 64x64 3x3, else generic)
  *   6 = TMA generic weight gradient even where the window variant applies
- *   7 = TMA window weight gradient forced for every eligible shape (any width) */
+ *   7 = TMA window weight gradient forced for every eligible shape (any width)
+ *   8 = default routing, but models created while it is set keep the unfused stem (generic 7x7 conv +
+ *       separate max-pool) instead of the space-to-depth stem kernels */
 adainf_status adainf_dbg_set_win_mode(int32_t mode);
+
+/* ResNet stem (7x7/2 pad 3 conv, <= 4 input channels, 64 outputs, ReLU, then 3x3/2 pad 1 max-pool) through
+ * the space-to-depth kernels (stem.cuh):
+ *   stem_fwd  : x [n][H][W][cin] bf16 (H, W even, W/2 <= 125), w [64][7][7][cin] bf16, b [64] fp32 ->
+ *               pooled [n][Hp][Wp][64] bf16 (Hp = (H/2 - 1)/2 + 1), argmax [n][Hp][Wp][64] uint8 (window
+ *               index kh*3 + kw of the FIRST maximum in row-major order; nullable)
+ *   stem_wgrad: x as above, dz [n][H/2][W/2][64] bf16 -> dw [64][7][7][cin] fp32, db [64] fp32 (nullable)
+ * Device pointers; temporaries are allocated stream-ordered.  Errors: ADAINF_ERR_SHAPE for ineligible shapes. */
+adainf_status adainf_dbg_stem_fwd(const void* x, int32_t n, int32_t H, int32_t W, int32_t cin, const void* w,
+                                  const float* b, void* pooled, uint8_t* argmax, adainf_stream_t stream);
+adainf_status adainf_dbg_stem_wgrad(const void* x, const void* dz, int32_t n, int32_t H, int32_t W, int32_t cin,
+                                    float* dw, float* db, adainf_stream_t stream);
 
 /* Launch accounting and per-kernel-class timing (CUDA events on the launching stream).
  * adainf_launch_count: total kernels launched by the library since load (host-side counter).

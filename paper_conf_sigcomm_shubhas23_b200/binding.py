@@ -100,6 +100,8 @@ def lib():
             "adainf_dbg_conv_dgrad": [vp, i32, i32, i32, i32, vp, i32, i32, i32, i32, i32, vp, vp, vp, i32, vp,
                                       vp],
             "adainf_dbg_conv_wgrad": [vp, vp, i32, i32, i32, i32, i32, i32, i32, i32, i32, vp, vp, vp],
+            "adainf_dbg_stem_fwd": [vp, i32, i32, i32, i32, vp, vp, vp, vp, vp],
+            "adainf_dbg_stem_wgrad": [vp, vp, i32, i32, i32, i32, vp, vp, vp],
         }.items():
             f = getattr(L, name, None)
             if f is not None:
@@ -360,6 +362,26 @@ def dbg_conv_dgrad(dz, w, H, W_, stride, pad, bcast=None, sc=None, yact=None, ma
     check(lib().adainf_dbg_conv_dgrad(ptr(dz), n, H, W_, Cc, ptr(w), Co, KH, KW, stride, pad, ptr(bcast), ptr(sc),
                                       ptr(yact), mask_act, ptr(dx), stream_ptr(stream)))
     return dx
+
+
+def dbg_stem_fwd(x, w, b, stream=None, want_argmax=True):
+    """Space-to-depth stem: conv 7x7/2 pad 3 + bias + ReLU + maxpool 3x3/2 pad 1 (include/adainf_debug.h)."""
+    import torch
+    n, H, W_, cin = x.shape
+    Hp, Wp = (H // 2 - 1) // 2 + 1, (W_ // 2 - 1) // 2 + 1
+    pooled = torch.empty((n, Hp, Wp, 64), dtype=torch.bfloat16, device=x.device)
+    am = torch.empty((n, Hp, Wp, 64), dtype=torch.uint8, device=x.device) if want_argmax else None
+    check(lib().adainf_dbg_stem_fwd(ptr(x), n, H, W_, cin, ptr(w), ptr(b), ptr(pooled), ptr(am), stream_ptr(stream)))
+    return pooled, am
+
+
+def dbg_stem_wgrad(x, dz, stream=None):
+    import torch
+    n, H, W_, cin = x.shape
+    dw = torch.empty((64, 7, 7, cin), dtype=torch.float32, device=x.device)
+    db = torch.empty(64, dtype=torch.float32, device=x.device)
+    check(lib().adainf_dbg_stem_wgrad(ptr(x), ptr(dz), n, H, W_, cin, ptr(dw), ptr(db), stream_ptr(stream)))
+    return dw, db
 
 
 def dbg_conv_wgrad(x, dz, KH, KW, stride, pad, stream=None):

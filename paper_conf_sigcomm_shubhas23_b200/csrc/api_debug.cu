@@ -4,6 +4,7 @@
 #include "../../include/adainf_debug.h"
 #include "api_common.h"
 #include "runtime.h"
+#include "stem.cuh"
 
 using namespace adainf;
 
@@ -70,6 +71,49 @@ extern "C" adainf_status adainf_dbg_conv_wgrad(const void* x, const void* dz, in
     CK(cudaMallocAsync((void**)&buf, ws, (cudaStream_t)stream));
     conv_wgrad(g, (const bf16*)x, (const bf16*)dz, n, C, buf, ws, dw, db, (cudaStream_t)stream);
     CK(cudaFreeAsync(buf, (cudaStream_t)stream));
+  });
+}
+
+extern "C" adainf_status adainf_dbg_stem_fwd(const void* x, int32_t n, int32_t H, int32_t W, int32_t cin,
+                                             const void* w, const float* b, void* pooled, uint8_t* argmax,
+                                             adainf_stream_t stream) {
+  return guard([&] {
+    if (n <= 0 || !stem_s2d_ok(H, W, cin, 64, 7, 7, 2, 3)) throw ShapeError("stem_fwd: ineligible shape");
+    require_device();
+    cudaStream_t st = (cudaStream_t)stream;
+    // GEMM-ready shadow [64][200] (K = (kh*7 + kw)*4 + c, zero-padded channels), then the per-tap layout
+    bf16 *shadow = nullptr, *wprep = nullptr, *s = nullptr;
+    CK(cudaMallocAsync((void**)&shadow, 64 * 200 * 2, st));
+    CK(cudaMallocAsync((void**)&wprep, 16 * 2 * 64 * 8 * 2, st));
+    CK(cudaMallocAsync((void**)&s, (size_t)n * H * W * 4 * 2, st));
+    CK(cudaMemsetAsync(shadow, 0, 64 * 200 * 2, st));
+    for (int co = 0; co < 64; ++co)  // 49 taps of cin channels -> 8-byte slots, rows of 200 elements
+      CK(cudaMemcpy2DAsync(shadow + co * 200, 8, (const bf16*)w + (size_t)co * 49 * cin, cin * 2, cin * 2, 49,
+                           cudaMemcpyDeviceToDevice, st));
+    launch_pack_s2d((const bf16*)x, nullptr, nullptr, n, H, W, cin, s, st);
+    launch_stem_wprep(shadow, 200, wprep, st);
+    stem_fwd(s, nullptr, n, H / 2, W / 2, wprep, b, (bf16*)pooled, argmax, st);
+    CK(cudaFreeAsync(s, st));
+    CK(cudaFreeAsync(wprep, st));
+    CK(cudaFreeAsync(shadow, st));
+  });
+}
+
+extern "C" adainf_status adainf_dbg_stem_wgrad(const void* x, const void* dz, int32_t n, int32_t H, int32_t W,
+                                               int32_t cin, float* dw, float* db, adainf_stream_t stream) {
+  return guard([&] {
+    if (n <= 0 || !stem_s2d_ok(H, W, cin, 64, 7, 7, 2, 3)) throw ShapeError("stem_wgrad: ineligible shape");
+    require_device();
+    cudaStream_t st = (cudaStream_t)stream;
+    bf16* s = nullptr;
+    float* ws = nullptr;
+    const size_t wsb = stem_wgrad_ws_bytes(n);
+    CK(cudaMallocAsync((void**)&s, (size_t)n * H * W * 4 * 2, st));
+    CK(cudaMallocAsync((void**)&ws, wsb, st));
+    launch_pack_s2d((const bf16*)x, nullptr, nullptr, n, H, W, cin, s, st);
+    stem_wgrad(s, (const bf16*)dz, n, H / 2, W / 2, cin, ws, wsb, dw, db, st);
+    CK(cudaFreeAsync(ws, st));
+    CK(cudaFreeAsync(s, st));
   });
 }
 

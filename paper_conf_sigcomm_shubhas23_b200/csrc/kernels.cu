@@ -97,10 +97,12 @@ void launch_maxpool_fwd(const bf16* x, const int* map, const int* count, int n_s
   CK(cudaGetLastError());
 }
 
-// one thread per (n, ih, iw, 8-channel vector): sums dT over the windows whose FIRST argmax is this
-// element (fixed window order), then the producer's activation mask; 128-bit loads / stores
+// Max-pool backward through the producer's activation: dz(pos) = act'(y(pos)) * sum of dT(w) over the windows
+// w whose FIRST argmax is pos.  y(pos) equals the pooled value of any such window, so the activation mask
+// is read from the pooled tensor P [n][Ho][Wo][C] (4x smaller than y for the 3x3/2 stem pool) instead of y.
+// One thread per (n, ih, iw, 8-channel vector), fixed window order (ho, then wo ascending), 128-bit I/O.
 __global__ void maxpool_bwd_kernel(const bf16* __restrict__ dT, const uint8_t* __restrict__ amax,
-                                   const bf16* __restrict__ yact, int act, long long n, int H, int W, int C, int K,
+                                   const bf16* __restrict__ pooled, int act, long long n, int H, int W, int C, int K,
                                    int s, int p, int Ho, int Wo, bf16* __restrict__ dz) {
   const int CV = C / 8;
   const long long total = n * H * W * CV;
@@ -113,9 +115,9 @@ __global__ void maxpool_bwd_kernel(const bf16* __restrict__ dT, const uint8_t* _
     const long long b = r / H;
     const int ho_lo = max(0, (ih + p - K + s) / s), ho_hi = min(Ho - 1, (ih + p) / s);
     const int wo_lo = max(0, (iw + p - K + s) / s), wo_hi = min(Wo - 1, (iw + p) / s);
-    float acc[8];
+    float acc[8], m[8];
 #pragma unroll
-    for (int q = 0; q < 8; ++q) acc[q] = 0.f;
+    for (int q = 0; q < 8; ++q) acc[q] = 0.f, m[q] = 0.f;
     for (int ho = ho_lo; ho <= ho_hi; ++ho) {
       const int kh = ih - (ho * s - p);
       if (kh < 0 || kh >= K) continue;
@@ -127,27 +129,30 @@ __global__ void maxpool_bwd_kernel(const bf16* __restrict__ dT, const uint8_t* _
         const uint8_t* a8 = (const uint8_t*)&am;
         const uint4 dv = __ldg((const uint4*)(dT + oi));
         const bf16* d8 = (const bf16*)&dv;
+        const uint4 pv = __ldg((const uint4*)(pooled + oi));
+        const bf16* p8 = (const bf16*)&pv;
         const uint8_t me = (uint8_t)(kh * K + kw);
 #pragma unroll
         for (int q = 0; q < 8; ++q)
-          if (a8[q] == me) acc[q] = __fadd_rn(acc[q], __bfloat162float(d8[q]));
+          if (a8[q] == me) {
+            acc[q] = __fadd_rn(acc[q], __bfloat162float(d8[q]));
+            m[q] = act_grad(act, __bfloat162float(p8[q]));
+          }
       }
     }
     const long long xi = ((b * H + ih) * W + iw) * C + cv * 8;
-    const uint4 yv = __ldg((const uint4*)(yact + xi));
-    const bf16* y8 = (const bf16*)&yv;
     __align__(16) bf16 o[8];
 #pragma unroll
-    for (int q = 0; q < 8; ++q) o[q] = __float2bfloat16_rn(__fmul_rn(acc[q], act_grad(act, __bfloat162float(y8[q]))));
+    for (int q = 0; q < 8; ++q) o[q] = __float2bfloat16_rn(__fmul_rn(acc[q], m[q]));
     *(uint4*)(dz + xi) = *(uint4*)o;
   }
 }
 // stride-2 fast path: one thread per (n, 2x2 input block, 8-channel vector); each window touching the
-// block is read once (argmax + dT, 128-bit), its gradient routed to the block element it selected; the
-// per-element window order is the same as the gather kernel's (ho, then wo ascending)
+// block is read once (argmax + dT + pooled value, 128-bit), its gradient routed to the block element it
+// selected; the per-element window order is the same as the gather kernel's (ho, then wo ascending)
 __global__ void maxpool_bwd_s2_kernel(const bf16* __restrict__ dT, const uint8_t* __restrict__ amax,
-                                      const bf16* __restrict__ yact, int act, long long n, int H, int W, int C, int K,
-                                      int p, int Ho, int Wo, bf16* __restrict__ dz) {
+                                      const bf16* __restrict__ pooled, int act, long long n, int H, int W, int C,
+                                      int K, int p, int Ho, int Wo, bf16* __restrict__ dz) {
   const int CV = C / 8;
   const int BH = (H + 1) / 2, BW = (W + 1) / 2;
   const long long total = n * BH * BW * CV;
@@ -159,13 +164,13 @@ __global__ void maxpool_bwd_s2_kernel(const bf16* __restrict__ dT, const uint8_t
     const int bi = (int)(r % BH);
     const long long b = r / BH;
     const int ih0 = 2 * bi, iw0 = 2 * bj;
-    float acc[2][2][8];
+    float acc[2][2][8], m[2][2][8];
 #pragma unroll
     for (int u = 0; u < 2; ++u)
 #pragma unroll
       for (int v = 0; v < 2; ++v)
 #pragma unroll
-        for (int q = 0; q < 8; ++q) acc[u][v][q] = 0.f;
+        for (int q = 0; q < 8; ++q) acc[u][v][q] = 0.f, m[u][v][q] = 0.f;
     const int ho_lo = max(0, (ih0 + p - K + 2) / 2), ho_hi = min(Ho - 1, (ih0 + 1 + p) / 2);
     const int wo_lo = max(0, (iw0 + p - K + 2) / 2), wo_hi = min(Wo - 1, (iw0 + 1 + p) / 2);
     for (int ho = ho_lo; ho <= ho_hi; ++ho)
@@ -175,16 +180,22 @@ __global__ void maxpool_bwd_s2_kernel(const bf16* __restrict__ dT, const uint8_t
         const uint8_t* a8 = (const uint8_t*)&am;
         const uint4 dv = __ldg((const uint4*)(dT + oi));
         const bf16* d8 = (const bf16*)&dv;
+        const uint4 pv = __ldg((const uint4*)(pooled + oi));
+        const bf16* p8 = (const bf16*)&pv;
 #pragma unroll
         for (int q = 0; q < 8; ++q) {
           const int kh = a8[q] / K, kw = a8[q] - (a8[q] / K) * K;
           const int u = ho * 2 - p + kh - ih0, v = wo * 2 - p + kw - iw0;
           const float g = __bfloat162float(d8[q]);
+          const float mg = act_grad(act, __bfloat162float(p8[q]));
 #pragma unroll
           for (int uu = 0; uu < 2; ++uu)
 #pragma unroll
             for (int vv = 0; vv < 2; ++vv)
-              if (u == uu && v == vv) acc[uu][vv][q] = __fadd_rn(acc[uu][vv][q], g);
+              if (u == uu && v == vv) {
+                acc[uu][vv][q] = __fadd_rn(acc[uu][vv][q], g);
+                m[uu][vv][q] = mg;
+              }
         }
       }
 #pragma unroll
@@ -194,28 +205,25 @@ __global__ void maxpool_bwd_s2_kernel(const bf16* __restrict__ dT, const uint8_t
         const int ih = ih0 + u, iw = iw0 + v;
         if (ih >= H || iw >= W) continue;
         const long long xi = ((b * H + ih) * W + iw) * C + cv * 8;
-        const uint4 yv = __ldg((const uint4*)(yact + xi));
-        const bf16* y8 = (const bf16*)&yv;
         __align__(16) bf16 o[8];
 #pragma unroll
-        for (int q = 0; q < 8; ++q)
-          o[q] = __float2bfloat16_rn(__fmul_rn(acc[u][v][q], act_grad(act, __bfloat162float(y8[q]))));
+        for (int q = 0; q < 8; ++q) o[q] = __float2bfloat16_rn(__fmul_rn(acc[u][v][q], m[u][v][q]));
         *(uint4*)(dz + xi) = *(uint4*)o;
       }
   }
 }
 
-void launch_maxpool_bwd(const bf16* dT, const uint8_t* amax, const bf16* yact, int act, int n, int H, int W, int C,
+void launch_maxpool_bwd(const bf16* dT, const uint8_t* amax, const bf16* pooled, int act, int n, int H, int W, int C,
                         int K, int s, int p, int Ho, int Wo, bf16* dz, cudaStream_t st) {
   ProfScope ps(PC_POOL_BWD, st);
   if (s == 2) {
     const long long total = (long long)n * ((H + 1) / 2) * ((W + 1) / 2) * (C / 8);
     const int blocks = (int)std::min<long long>((total + 255) / 256, 64LL * num_sms());
-    maxpool_bwd_s2_kernel<<<blocks, 256, 0, st>>>(dT, amax, yact, act, n, H, W, C, K, p, Ho, Wo, dz);
+    maxpool_bwd_s2_kernel<<<blocks, 256, 0, st>>>(dT, amax, pooled, act, n, H, W, C, K, p, Ho, Wo, dz);
   } else {
     const long long total = (long long)n * H * W * (C / 8);
     const int blocks = (int)std::min<long long>((total + 255) / 256, 64LL * num_sms());
-    maxpool_bwd_kernel<<<blocks, 256, 0, st>>>(dT, amax, yact, act, n, H, W, C, K, s, p, Ho, Wo, dz);
+    maxpool_bwd_kernel<<<blocks, 256, 0, st>>>(dT, amax, pooled, act, n, H, W, C, K, s, p, Ho, Wo, dz);
   }
   CK(cudaGetLastError());
 }

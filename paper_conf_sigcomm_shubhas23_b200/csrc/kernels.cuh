@@ -14,8 +14,9 @@ void launch_pack_input(const bf16* x, const int* map, const int* count, int n_st
 // maxpool fwd (NHWC bf16); optional input map; optional argmax offsets (uint8) for backward
 void launch_maxpool_fwd(const bf16* x, const int* map, const int* count, int n_static, int H, int W, int C, int K,
                         int s, int p, int Ho, int Wo, bf16* y, uint8_t* argmax, cudaStream_t st);
-// maxpool bwd fused with the producer's activation mask: dz = bf16(sum_windows dT * [first argmax]) * act'(y)
-void launch_maxpool_bwd(const bf16* dT, const uint8_t* argmax, const bf16* yact, int act, int n, int H, int W, int C,
+// maxpool bwd fused with the producer's activation mask: dz = bf16(sum_windows dT * [first argmax]) * act'(y),
+// the mask taken from the pooled output P (= y at the selected position)
+void launch_maxpool_bwd(const bf16* dT, const uint8_t* argmax, const bf16* pooled, int act, int n, int H, int W, int C,
                         int K, int s, int p, int Ho, int Wo, bf16* dz, cudaStream_t st);
 
 // ---- exit head (K4) ----

@@ -6,6 +6,7 @@
 
 #include "api_common.h"
 #include "model.h"
+#include "stem.cuh"
 
 namespace adainf {
 
@@ -212,9 +213,25 @@ void Model::build(const adainf_model_spec& s) {
   nstages = stage + 1;
   nparams = off;
 
+  // fused space-to-depth stem: conv 7x7/2 (ReLU) whose only consumer is a 3x3/2 pad-1 max-pool
+  stem_s2d = false;
+  if (!nodes.empty() && nodes[0].kind == N_CONV && nodes[0].in == 0 && win_mode() != 8) {
+    const NodeRt& c0 = nodes[0];
+    const TensorRt& Y = T[c0.out];
+    const int po = Y.primary;
+    if (po >= 0 && nodes[po].kind == N_POOL && nodes[po].pk == 3 && nodes[po].ps == 2 && nodes[po].pp == 1 &&
+        nodes[po].stage == c0.stage && c0.act == 1 && !c0.fp32_out && c0.res < 0 && Y.exit_k < 0 &&
+        Y.res_of < 0 && Y.proj < 0 && stem_s2d_ok(in_h, in_w, in_c, c0.g.Cout, c0.g.KH, c0.g.KW, c0.g.stride, c0.g.pad)) {
+      stem_s2d = true;
+      stem_pool = po;
+      pack = true;
+    }
+  }
+
   CK(cudaSetDevice(device));
   // activations
   for (size_t t = 1; t < T.size(); ++t) {
+    if (stem_s2d && (int)t == nodes[0].out) continue;  // the fused stem never materialises its conv output
     const size_t b = (size_t)max_batch * T[t].row_elems() * (T[t].f32 ? 4 : 2);
     T[t].own.alloc(b);
     T[t].buf = T[t].own.as<bf16>();
@@ -228,6 +245,7 @@ void Model::build(const adainf_model_spec& s) {
       nd.shadow.alloc((size_t)nd.g.Cout * nd.ldb * 2);
       nd.shadow.zero();
     }
+  if (stem_s2d) stem_wprep.alloc(16 * 2 * 64 * 8 * 2);
   params.alloc(nparams * 4);
   mom.alloc(nparams * 4);
   grads.alloc(nparams * 4);
@@ -319,6 +337,10 @@ void Model::build(const adainf_model_spec& s) {
 
 // a1 ingest: channel padding (to 4 for few-channel inputs, else to a multiple of 8)
 void Model::ingest(const bf16* x, const int* map, const int* count, int n_static, cudaStream_t st) {
+  if (stem_s2d) {
+    launch_pack_s2d(x, map, count, n_static, in_h, in_w, in_c, packed_in.as<bf16>(), st);
+    return;
+  }
   launch_pack_input(x, map, count, n_static, in_h, in_w, in_c, cin_pad, packed_in.as<bf16>(), st);
 }
 
@@ -340,6 +362,7 @@ void Model::ensure_training() {
       nd.argmax.alloc((size_t)max_batch * T[nd.out].row_elems());
     } else {
       ws = std::max(ws, ::adainf::wgrad_ws_bytes(nd.g, max_batch));
+      if (stem_s2d && &nd == &nodes[0]) ws = std::max(ws, stem_wgrad_ws_bytes(max_batch));
       if (nd.kind == N_PROJ && nd.in != 0) nd.proj_dx.alloc((size_t)max_batch * T[nd.in].row_elems() * 2);
     }
   }
@@ -383,7 +406,16 @@ void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, in
       NodeRt& nd = nodes[ni];
       const int ns = train ? 0 : nd.stage;
       const int* c = train ? nullptr : stage_count(ns);
+      if (stem_s2d && ni == 0) {
+        if (map_for(0, ns)) throw InvalidError("stem: mapped input rows must be ingested first");
+        const NodeRt& pl = nodes[stem_pool];
+        launch_stem_wprep(nd.shadow.as<bf16>(), nd.ldb, stem_wprep.as<bf16>(), st);
+        stem_fwd(buf_of(0), c, n_static, in_h / 2, in_w / 2, stem_wprep.as<bf16>(), params.as<float>() + nd.b_off,
+                 T[pl.out].buf, train ? pl.argmax.as<uint8_t>() : nullptr, st);
+        continue;
+      }
       if (nd.kind == N_POOL) {
+        if (stem_s2d && ni == stem_pool) continue;  // produced by the fused stem
         launch_maxpool_fwd(buf_of(nd.in), map_for(nd.in, ns), c, n_static, nd.g.H, nd.g.W, nd.g.Cin, nd.pk, nd.ps,
                            nd.pp, nd.g.Ho, nd.g.Wo, T[nd.out].buf, train ? nd.argmax.as<uint8_t>() : nullptr, st);
       } else {
@@ -500,6 +532,11 @@ void Model::train_step(const bf16* x, const int32_t* labels, int n, long long n_
                            T[t].grad, st);
   // reverse walk (K2, K3, K9)
   auto conv_backward = [&](NodeRt& nd, const bf16* dz) {
+    if (stem_s2d && &nd == &nodes[0]) {
+      stem_wgrad(buf_of(0), dz, n, in_h / 2, in_w / 2, nd.cin_real, wgrad_ws.as<float>(), wgrad_ws_bytes,
+                 G + nd.w_off, G + nd.b_off, st);
+      return;
+    }
     conv_wgrad(nd.g, buf_of(nd.in), dz, n, nd.cin_real, wgrad_ws.as<float>(), wgrad_ws_bytes, G + nd.w_off,
                G + nd.b_off, st);
     if (nd.in == 0) return;  // no input gradient for the first layer
@@ -519,7 +556,7 @@ void Model::train_step(const bf16* x, const int32_t* labels, int n, long long n_
     if (nd.kind == N_POOL) {
       const TensorRt& X = T[nd.in];
       if (nd.in == 0) continue;
-      launch_maxpool_bwd(T[nd.out].grad, nd.argmax.as<uint8_t>(), X.buf, X.act, n, X.H, X.W, X.C, nd.pk, nd.ps, nd.pp,
+      launch_maxpool_bwd(T[nd.out].grad, nd.argmax.as<uint8_t>(), T[nd.out].buf, X.act, n, X.H, X.W, X.C, nd.pk, nd.ps, nd.pp,
                          nd.g.Ho, nd.g.Wo, T[nd.in].grad, st);
       continue;
     }

@@ -94,7 +94,11 @@ struct Model {
   float momentum = 0.9f, weight_decay = 0.f;
 
   DevBuf params, mom, grads;
-  DevBuf packed_in;           // [max_batch][H][W][cin_pad]
+  DevBuf packed_in;           // [max_batch][H][W][cin_pad], or S2D [max_batch][H/2][W/2][16] (stem_s2d)
+  // ResNet stem (7x7/2 conv + ReLU + 3x3/2 max-pool) run by the fused space-to-depth kernels (stem.cuh)
+  bool stem_s2d = false;
+  int stem_pool = -1;         // node index of the pool fused into the stem
+  DevBuf stem_wprep;          // per-tap bf16 weights [16][2][64][8], rebuilt from the shadow every forward
   // inference stage bookkeeping
   DevBuf pos, orig, counts, alive;  // pos/orig: [nstages][max_batch] int; counts [nstages] int
   // training

@@ -13,7 +13,8 @@ static const char* kNames[PROF_NCLASS] = {"conv_fwd",     "conv_dgrad", "conv_wg
                                           "pack_input",   "maxpool_fwd", "maxpool_bwd", "exit_head",    "compact",
                                           "exit_loss",    "head_grads",  "grad_finalize", "sum",        "sgd_update",
                                           "shadow_pack",  "select_proj", "select_cosine", "select_topk", "det_route",
-                                          "crop",         "route_class", "gather_rows"};
+                                          "crop",         "route_class", "gather_rows", "stem_fwd",   "stem_wgrad",
+                                          "stem_aux"};
 
 struct Prof {
   std::mutex mu;

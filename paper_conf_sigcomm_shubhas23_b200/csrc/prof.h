@@ -28,6 +28,9 @@ enum ProfClass {
   PC_CROP,
   PC_ROUTE_CLASS,
   PC_GATHER,
+  PC_STEM_FWD,
+  PC_STEM_WGRAD,
+  PC_STEM_AUX,
   PROF_NCLASS
 };
 

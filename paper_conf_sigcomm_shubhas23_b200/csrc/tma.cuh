@@ -12,6 +12,8 @@ namespace adainf {
 // 4-D tiled map over a dense NHWC bf16 tensor [N][H][W][C]: dims (innermost first) {C, W, H, N},
 // box {bc, bw, bh, 1}, 128B swizzle (bc * 2 bytes must be <= 128), out-of-bounds -> zeros.
 CUtensorMap make_tmap_nhwc(const void* base, int N, int H, int W, int C, int bc, int bw, int bh, int stride = 1);
+// same, no swizzle: the box lands row-major (bc * 2 bytes per (w, h) position, a multiple of 16)
+CUtensorMap make_tmap_nhwc_plain(const void* base, int N, int H, int W, int C, int bc, int bw, int bh);
 // 2-D tiled map over a row-major [rows][cols] bf16 matrix (row pitch ld elements), box {bcols, brows}.
 CUtensorMap make_tmap_2d(const void* base, long long rows, int cols, int ld, int bcols, int brows);
 
