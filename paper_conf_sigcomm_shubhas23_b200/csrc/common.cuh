@@ -158,6 +158,16 @@ __device__ __forceinline__ uint64_t make_sdesc_plain(uint32_t saddr, uint32_t lb
   d |= (uint64_t)1 << 46;
   return d;
 }
+// UMMA shared-memory descriptor, SWIZZLE_32B (layout type 6): 32-byte rows, 8-row groups of 256 B (SBO)
+__device__ __forceinline__ uint64_t make_sdesc_sw32(uint32_t saddr, uint32_t lbo_bytes, uint32_t sbo_bytes) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFFu);
+  d |= (uint64_t)((lbo_bytes >> 4) & 0x3FFFu) << 16;
+  d |= (uint64_t)((sbo_bytes >> 4) & 0x3FFFu) << 32;
+  d |= (uint64_t)1 << 46;
+  d |= (uint64_t)6 << 61;
+  return d;
+}
 // instruction descriptor, kind::f16: D f32, A/B bf16, majors, N, M
 __host__ __device__ constexpr uint32_t make_idesc(int M, int N, int a_mn_major, int b_mn_major) {
   return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)a_mn_major << 15) | ((uint32_t)b_mn_major << 16) |

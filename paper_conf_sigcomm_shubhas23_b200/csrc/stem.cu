@@ -97,15 +97,15 @@ static void pick_bands(int n, int rows, int halo, int* bands, int* band_rows) {
 // =====================================================================================================
 constexpr int SF_THREADS = 416;  // warp 0 TMA, warp 4 MMA, warps 5..12 epilogue (two per TMEM lane quadrant)
 constexpr int SLOTS = 128;       // padded columns of one output row = the M tile
-constexpr int SF_PLANE = (4 * SLOTS + 8) * 16;  // 4 window rows x 128 positions x 16 B (+ 8 trail rows)
-constexpr int SF_STAGE = 2 * SF_PLANE;
+// window: 4 s2d rows x 128 positions x 32 B (SWIZZLE_32B: 16-byte chunk ^= row bit 2), + 8 trail rows
+constexpr int SF_STAGE = ((4 * SLOTS + 8) * 32 + 1023) / 1024 * 1024;
 constexpr int SF_STAGES = 6;
 constexpr int SF_W_BYTES = 16 * 2048;
 constexpr int SF_RING = 4;  // conv-row ring: bf16 [SLOTS][64], 16-byte chunk k of column x at k ^ (x & 7)
 constexpr int SF_SMEM = 1024 + SF_W_BYTES + SF_STAGES * SF_STAGE + SF_RING * SLOTS * 128 + 256;
 
 struct StemFwdArgs {
-  CUtensorMap s_map;  // S2D [n][Hs][Ws][16], box {8, 128, 4, 1}, no swizzle
+  CUtensorMap s_map;  // S2D [n][Hs][Ws][16], box {16, 128, 4, 1}, 32B swizzle
   const bf16* wprep;
   const float* bias;
   const int* count;
@@ -176,10 +176,8 @@ __global__ void __launch_bounds__(SF_THREADS, 1) stem_fwd_kernel(const __grid_co
         for (int r = su.r0; r <= su.r1; ++r, ++it) {
           const int s = it % SF_STAGES, ph = it / SF_STAGES;
           if (ph > 0) mbar_wait(&empty[s], (ph - 1) & 1);
-          mbar_expect_tx(&full[s], 2 * 4 * SLOTS * 16);
-          const uint32_t dst = st_base + s * SF_STAGE;
-          tma_load_4d(dst, &a.s_map, &full[s], 0, -2, r - 2, su.img);
-          tma_load_4d(dst + SF_PLANE, &a.s_map, &full[s], 8, -2, r - 2, su.img);
+          mbar_expect_tx(&full[s], 4 * SLOTS * 32);
+          tma_load_4d(st_base + s * SF_STAGE, &a.s_map, &full[s], 0, -2, r - 2, su.img);
         }
       }
     }
@@ -196,11 +194,14 @@ __global__ void __launch_bounds__(SF_THREADS, 1) stem_fwd_kernel(const __grid_co
         mbar_wait(&full[s], ph & 1);
         tc_fence_after();
         if (elect_one()) {
-          const uint64_t adesc0 = make_sdesc_plain(st_base + s * SF_STAGE, SF_PLANE, 128);
+          // K-major SWIZZLE_32B: one 32-byte row (16 channels = K) per position, 8-row groups 256 B apart;
+          // tap (ah, aw) = the window shifted by (ah+2)*128 + (aw+2) rows (swizzle follows address bits)
+          const uint64_t adesc0 = make_sdesc_sw32(st_base + s * SF_STAGE, 16, 256);
 #pragma unroll
           for (int t = 0; t < 16; ++t) {
-            const uint32_t row_off = (uint32_t)((t >> 2) * SLOTS + (t & 3));  // window row of tap (ah, aw)
-            umma_bf16(tmem + (uint32_t)(b * 64), adesc0 + row_off, bdesc0 + (uint64_t)(t * 128), IDESC, t > 0);
+            const uint32_t row_off = (uint32_t)((t >> 2) * SLOTS + (t & 3));
+            umma_bf16(tmem + (uint32_t)(b * 64), adesc0 + (uint64_t)(row_off * 2), bdesc0 + (uint64_t)(t * 128), IDESC,
+                      t > 0);
           }
           umma_commit(&empty[s]);
           umma_commit(&tfull[b]);
@@ -249,44 +250,45 @@ __global__ void __launch_bounds__(SF_THREADS, 1) stem_fwd_kernel(const __grid_co
         if (po < su.po0 || po >= su.po1) continue;
         for (int item = t; item < a.Wp * 8; item += 256) {
           const int pw = item >> 3, k = item & 7;
-          float best[8];
-          uint32_t arg[2] = {0u, 0u};
-#pragma unroll
-          for (int q = 0; q < 8; ++q) best[q] = -INFINITY;
+          // the 3x3 window (bf16x2 x 4 per position; -inf outside the conv output)
+          uint4 wv[9];
 #pragma unroll
           for (int kh = 0; kh < 3; ++kh) {
             const int rr = 2 * po - 1 + kh;
-            if (rr < 0 || rr >= a.Hs) continue;
             const uint8_t* slot = ring + (rr & 3) * SLOTS * 128;
 #pragma unroll
             for (int kw = 0; kw < 3; ++kw) {
               const int cc = 2 * pw - 1 + kw;
-              if (cc < 0 || cc >= a.Ws) continue;
-              const uint4 raw = *(const uint4*)(slot + cc * 128 + ((k ^ (cc & 7)) << 4));
-              const __nv_bfloat162* h = (const __nv_bfloat162*)&raw;
-#pragma unroll
-              for (int q = 0; q < 4; ++q) {
-                const float2 f = __bfloat1622float2(h[q]);
-                // strict: the FIRST maximal element in row-major window order (as maxpool_fwd_kernel)
-                if (f.x > best[2 * q]) {
-                  best[2 * q] = f.x;
-                  const int sh = ((2 * q) & 3) * 8;
-                  arg[q >> 1] = (arg[q >> 1] & ~(0xFFu << sh)) | ((uint32_t)(kh * 3 + kw) << sh);
-                }
-                if (f.y > best[2 * q + 1]) {
-                  best[2 * q + 1] = f.y;
-                  const int sh = ((2 * q + 1) & 3) * 8;
-                  arg[q >> 1] = (arg[q >> 1] & ~(0xFFu << sh)) | ((uint32_t)(kh * 3 + kw) << sh);
-                }
-              }
+              wv[kh * 3 + kw] = (rr >= 0 && rr < a.Hs && cc >= 0 && cc < a.Ws)
+                                    ? *(const uint4*)(slot + cc * 128 + ((k ^ (cc & 7)) << 4))
+                                    : make_uint4(0xFF80FF80u, 0xFF80FF80u, 0xFF80FF80u, 0xFF80FF80u);
             }
           }
-          __align__(16) __nv_bfloat162 o[4];
+          __nv_bfloat162 best[4];
 #pragma unroll
-          for (int q = 0; q < 4; ++q) o[q] = __floats2bfloat162_rn(best[2 * q], best[2 * q + 1]);
+          for (int q = 0; q < 4; ++q) best[q] = ((const __nv_bfloat162*)&wv[0])[q];
+#pragma unroll
+          for (int p = 1; p < 9; ++p)
+#pragma unroll
+            for (int q = 0; q < 4; ++q) best[q] = __hmax2(best[q], ((const __nv_bfloat162*)&wv[p])[q]);
           const long long oi = (((long long)su.img * a.Hp + po) * a.Wp + pw) * 64 + k * 8;
-          *(uint4*)(a.pooled + oi) = *(const uint4*)o;
-          if (a.argmax) *(uint2*)(a.argmax + oi) = make_uint2(arg[0], arg[1]);
+          *(uint4*)(a.pooled + oi) = *(const uint4*)best;
+          if (a.argmax) {
+            // FIRST maximal position in row-major window order: scan backwards, the last match written wins
+            uint32_t arg[2] = {0u, 0u};
+#pragma unroll
+            for (int p = 8; p >= 0; --p) {
+              const uint32_t kk = 0x01010101u * (uint32_t)p;
+#pragma unroll
+              for (int w = 0; w < 2; ++w) {
+                const uint32_t m0 = __heq2_mask(((const __nv_bfloat162*)&wv[p])[2 * w], best[2 * w]);
+                const uint32_t m1 = __heq2_mask(((const __nv_bfloat162*)&wv[p])[2 * w + 1], best[2 * w + 1]);
+                const uint32_t pm = __byte_perm(m0, m1, 0x6420);  // one byte per channel
+                arg[w] = (arg[w] & ~pm) | (kk & pm);
+              }
+            }
+            *(uint2*)(a.argmax + oi) = make_uint2(arg[0], arg[1]);
+          }
         }
       }
     }
@@ -306,7 +308,7 @@ void stem_fwd(const bf16* s, const int* count, int n_static, int Hs, int Ws, con
   if (Ws > 125) throw ShapeError("stem: width/2 must be <= 125");
   static StemFwdArgs a;
   a = StemFwdArgs{};
-  a.s_map = make_tmap_nhwc_plain(s, n_static, Hs, Ws, 16, 8, SLOTS, 4);
+  a.s_map = make_tmap_nhwc_swz(s, n_static, Hs, Ws, 16, 16, SLOTS, 4, 32);
   a.wprep = wprep;
   a.bias = bias;
   a.count = count;
@@ -333,43 +335,51 @@ void stem_fwd(const bf16* s, const int* count, int n_static, int Hs, int Ws, con
 // weight gradient
 // =====================================================================================================
 constexpr int SW_THREADS = 288;  // warp 0 TMA, warps 1-3 bias column sums, warp 4 MMA, warps 5-8 epilogue
-constexpr int SW_NS = 8;         // dZ ring slots: 128 positions (col -1 .. 126) x 64 co, 128B swizzle
-constexpr int SW_SS = 8;         // S stages: two planes of 128 positions x 8 channels
-constexpr int SW_SLOT = SLOTS * 128;
-constexpr int SW_SSTAGE = 2 * SLOTS * 16;
-constexpr int SW_SMEM = 1024 + SW_NS * SW_SLOT + 1024 + SW_SS * SW_SSTAGE + 256 + 3072;
+constexpr int SW_DZ_STAGE = 2 * SLOTS * 128;  // dZ rows i, i+1: 128 positions x 64 co each, 128B swizzle
+constexpr int SW_ND = 3;                      // dZ row-pair stages
+constexpr int SW_S_SLOT = SLOTS * 32;         // one S row: 128 positions (cols -2..125) x 16 ch, 32B swizzle
+constexpr int SW_NS = 16;                     // S row ring
+constexpr int SW_SMEM = 1024 + SW_ND * SW_DZ_STAGE + SW_NS * SW_S_SLOT + 1024 + 512 + 3072;
 
+// dW[ah][aw][ch][co] = sum_q dZ(i, q)[co] * S(i + ah, q + aw)[ch], output rows taken in pairs (i, i+1):
+// A = the two dZ rows (M = 2 x 64 co, MN-major, atoms 16 KB apart), B = one S row rho = i - 2 + o shifted
+// by aw = -2..1 (N = 4 x 16 ch: MN-major SWIZZLE_32B atoms one 32-byte position apart), K = 16 positions.
+// Accumulator o (64 TMEM columns) collects tap ah = o - 2 in its top half (row i) and ah = o - 3 in its
+// bottom half (row i + 1); the finish kernel adds the two halves of each tap.
 struct StemWgArgs {
-  CUtensorMap s_map;   // S2D [n][Hs][Ws][16], box {8, 128, 1, 1}, no swizzle
-  CUtensorMap dz_map;  // dZ [n][Hs][Ws][64], box {64, 128, 1, 1}, 128B swizzle
-  int n, Hs, Ws, bands, band_rows;
-  float* part;     // [gridDim.x][256][64]
+  CUtensorMap s_map;   // S2D [n][Hs][Ws][16], box {16, 128, 1, 1}, 32B swizzle
+  CUtensorMap dz_map;  // dZ [n][Hs][Ws][64], box {64, 128, 2, 1}, 128B swizzle
+  int n, Hs, Ws, bands, band_rows;  // band_rows even
+  float* part;     // [gridDim.x][2][256][64]
   float* cs_part;  // [gridDim.x][64] or nullptr
 };
 
 __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_constant__ StemWgArgs a) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-  uint8_t* ring = smem;
-  uint8_t* guard = ring + SW_NS * SW_SLOT;  // zero rows read (for invalid positions only) past the last slot
-  uint8_t* sst = guard + 1024;
-  uint64_t* dz_full = (uint64_t*)(sst + SW_SS * SW_SSTAGE);
-  uint64_t* dz_empty = dz_full + SW_NS;
-  uint64_t* s_full = dz_empty + SW_NS;
-  uint64_t* s_empty = s_full + SW_SS;
-  uint64_t* tfull = s_empty + SW_SS;
+  uint8_t* dzst = smem;
+  uint8_t* sring = dzst + SW_ND * SW_DZ_STAGE;
+  uint8_t* guard = sring + SW_NS * SW_S_SLOT;  // finite rows read past the last S slot (invalid positions only)
+  uint64_t* dz_full = (uint64_t*)(guard + 1024);
+  uint64_t* dz_empty = dz_full + SW_ND;
+  uint64_t* s_full = dz_empty + SW_ND;
+  uint64_t* s_empty = s_full + SW_NS;
+  uint64_t* tfull = s_empty + SW_NS;
   uint32_t* tmem_slot = (uint32_t*)(tfull + 1);
-  float* cs_red = (float*)((uint8_t*)dz_full + 256);
+  float* cs_red = (float*)((uint8_t*)dz_full + 512);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nunits = a.n * a.bands;
-  for (int i = threadIdx.x; i < 1024 / 16; i += blockDim.x) ((uint4*)guard)[i] = make_uint4(0, 0, 0, 0);
+  // zero the S ring and the guard: B rows past the end of a slot (positions >= 125, where dZ is zero) read
+  // the next slot, which must hold finite values even before its first load (0 * NaN = NaN)
+  for (int i = threadIdx.x; i < (SW_NS * SW_S_SLOT + 1024) / 16; i += blockDim.x)
+    ((uint4*)sring)[i] = make_uint4(0, 0, 0, 0);
   if (threadIdx.x == 0) {
-    for (int s = 0; s < SW_NS; ++s) {
+    for (int s = 0; s < SW_ND; ++s) {
       mbar_init(&dz_full[s], 1);
       mbar_init(&dz_empty[s], a.cs_part ? 4 : 1);  // MMA commit (+ one arrive per column-sum warp)
     }
-    for (int s = 0; s < SW_SS; ++s) {
+    for (int s = 0; s < SW_NS; ++s) {
       mbar_init(&s_full[s], 1);
       mbar_init(&s_empty[s], 1);
     }
@@ -378,39 +388,38 @@ __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_
     tma_prefetch_desc(&a.s_map);
     tma_prefetch_desc(&a.dz_map);
   }
-  if (warp == 4) tmem_alloc<128>(tmem_slot);
+  if (warp == 4) tmem_alloc<512>(tmem_slot);
   fence_proxy_async_smem();
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
-  const uint32_t ring_u = smem_u32(ring), sst_u = smem_u32(sst);
+  const uint32_t dz_u = smem_u32(dzst), s_u = smem_u32(sring);
 
   auto unit_rows = [&](int u, int& img, int& i0, int& i1) {
     img = u / a.bands;
     i0 = (u - img * a.bands) * a.band_rows;
-    i1 = min(a.Hs, i0 + a.band_rows);
+    i1 = min(a.Hs, i0 + a.band_rows);  // pairs (i, i+1) for i = i0, i0+2, ..; i+1 may be Hs (zero rows)
   };
 
   if (warp == 0) {
     if (lane == 0) {
-      int L = 0, it = 0;
+      int L = 0, P = 0;  // S rows loaded, dZ pairs loaded
       for (int u = blockIdx.x; u < nunits; u += gridDim.x) {
         int img, i0, i1;
         unit_rows(u, img, i0, i1);
-        int nd = i0 - 1;
-        for (int i = i0; i < i1; ++i, ++it) {
-          for (; nd <= i + 2; ++nd, ++L) {
+        int nr = i0 - 2;  // next S row
+        for (int i = i0; i < i1; i += 2, ++P) {
+          for (; nr <= i + 2; ++nr, ++L) {
             const int slot = L % SW_NS, ph = L / SW_NS;
-            if (ph > 0) mbar_wait(&dz_empty[slot], (ph - 1) & 1);
-            mbar_expect_tx(&dz_full[slot], SW_SLOT);
-            tma_load_4d(ring_u + slot * SW_SLOT, &a.dz_map, &dz_full[slot], 0, -1, nd, img);
+            if (ph > 0) mbar_wait(&s_empty[slot], (ph - 1) & 1);
+            mbar_expect_tx(&s_full[slot], SW_S_SLOT);
+            tma_load_4d(s_u + slot * SW_S_SLOT, &a.s_map, &s_full[slot], 0, -2, nr, img);
           }
-          const int s = it % SW_SS, ph = it / SW_SS;
-          if (ph > 0) mbar_wait(&s_empty[s], (ph - 1) & 1);
-          mbar_expect_tx(&s_full[s], SW_SSTAGE);
-          tma_load_4d(sst_u + s * SW_SSTAGE, &a.s_map, &s_full[s], 0, 0, i, img);
-          tma_load_4d(sst_u + s * SW_SSTAGE + SLOTS * 16, &a.s_map, &s_full[s], 8, 0, i, img);
+          const int st = P % SW_ND, ph = P / SW_ND;
+          if (ph > 0) mbar_wait(&dz_empty[st], (ph - 1) & 1);
+          mbar_expect_tx(&dz_full[st], SW_DZ_STAGE);
+          tma_load_4d(dz_u + st * SW_DZ_STAGE, &a.dz_map, &dz_full[st], 0, 0, i, img);
         }
       }
     }
@@ -420,63 +429,59 @@ __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_
       const int t = threadIdx.x - 32;
       cs.init(t);
       cs.zero();
-      int L = 0;
+      int P = 0;
       for (int u = blockIdx.x; u < nunits; u += gridDim.x) {
         int img, i0, i1;
         unit_rows(u, img, i0, i1);
-        for (int rho = i0 - 1; rho <= i1 + 1; ++rho, ++L) {
-          const int slot = L % SW_NS;
-          mbar_wait(&dz_full[slot], (L / SW_NS) & 1);
-          if (rho >= i0 && rho < i1) cs.add(ring + slot * SW_SLOT, SLOTS);
+        for (int i = i0; i < i1; i += 2, ++P) {
+          const int st = P % SW_ND;
+          mbar_wait(&dz_full[st], (P / SW_ND) & 1);
+          cs.add(dzst + st * SW_DZ_STAGE, 2 * SLOTS);  // rows >= Hs and columns >= Ws are zero-filled
           __syncwarp();
-          if (lane == 0) mbar_arrive(&dz_empty[slot]);
+          if (lane == 0) mbar_arrive(&dz_empty[st]);
         }
       }
       cs.finish(cs_red, a.cs_part + (long long)blockIdx.x * 64, 64, t);
     }
   } else if (warp == 4) {
-    constexpr uint32_t IDESC = make_idesc(128, 16, 1, 1);
-    int L = 0, it = 0;
+    constexpr uint32_t IDESC = make_idesc(128, 64, 1, 1);
+    int L = 0, P = 0;
     bool first = true;
     for (int u = blockIdx.x; u < nunits; u += gridDim.x) {
       int img, i0, i1;
       unit_rows(u, img, i0, i1);
-      const int Lb = L;
-      for (int i = i0; i < i1; ++i, ++it) {
-        for (int q = (i == i0 ? 0 : 3); q <= 3; ++q) {
+      const int Lb = L;  // load index of S row i0 - 2
+      for (int i = i0; i < i1; i += 2, ++P) {
+        // S rows up to i + 2 (load index Lb + (i + 2) - (i0 - 2))
+        for (int q = (i == i0 ? 0 : 3); q <= 4; ++q) {
           const int Lx = Lb + (i - i0) + q;
-          mbar_wait(&dz_full[Lx % SW_NS], (Lx / SW_NS) & 1);
+          mbar_wait(&s_full[Lx % SW_NS], (Lx / SW_NS) & 1);
         }
-        const int s = it % SW_SS;
-        mbar_wait(&s_full[s], (it / SW_SS) & 1);
+        const int st = P % SW_ND;
+        mbar_wait(&dz_full[st], (P / SW_ND) & 1);
         tc_fence_after();
         if (elect_one()) {
-          // MN-major, no swizzle: LBO = K-direction stride of 8-row groups, SBO = N-direction (plane) stride
-          const uint64_t bdesc0 = make_sdesc_plain(sst_u + s * SW_SSTAGE, 128, SLOTS * 16);
+          const uint64_t adesc0 = make_sdesc(dz_u + st * SW_DZ_STAGE, SLOTS * 128, 1024);
+          uint64_t bdesc[5];
 #pragma unroll
-          for (int ah = -2; ah <= 1; ++ah) {
-            const int Lr = Lb + (i - ah) - (i0 - 1);  // load index of dZ row i - ah
-            const uint32_t base = ring_u + (Lr % SW_NS) * SW_SLOT;
+          for (int o = 0; o < 5; ++o)
+            bdesc[o] = make_sdesc_sw32(s_u + ((Lb + (i - i0) + o) % SW_NS) * SW_S_SLOT, 32, 256);
+#pragma unroll 1
+          for (int kk = 0; kk < 8; ++kk) {
 #pragma unroll
-            for (int pr = 0; pr < 2; ++pr) {
-              // atoms: aw = 1 - 2*pr (row offset 2*pr), aw = -2*pr (row offset 2*pr + 1); LBO = one row
-              const uint64_t adesc0 = make_sdesc(base + pr * 256, 128, 1024);
-              const uint32_t acc = (uint32_t)(((ah + 2) * 2 + pr) * 16);
-#pragma unroll
-              for (int kk = 0; kk < 8; ++kk)
-                umma_bf16(tmem + acc, adesc0 + (uint64_t)(kk * 128), bdesc0 + (uint64_t)(kk * 16), IDESC,
-                          (!first || kk > 0) ? 1u : 0u);
-            }
+            for (int o = 0; o < 5; ++o)
+              umma_bf16(tmem + (uint32_t)(o * 64), adesc0 + (uint64_t)(kk * 128), bdesc[o] + (uint64_t)(kk * 32),
+                        IDESC, (!first || kk > 0) ? 1u : 0u);
           }
-          umma_commit(&s_empty[s]);
-          umma_commit(&dz_empty[(Lb + (i - i0)) % SW_NS]);  // dZ row i - 1: no later use
-          if (i == i1 - 1)
-            for (int q = 1; q <= 3; ++q) umma_commit(&dz_empty[(Lb + (i - i0) + q) % SW_NS]);
+          umma_commit(&dz_empty[st]);
+          // S rows i - 2, i - 1 are not used by the next pair; the unit's last pair releases all five
+          const int nrel = (i + 2 >= i1) ? 5 : 2;
+          for (int q = 0; q < nrel; ++q) umma_commit(&s_empty[(Lb + (i - i0) + q) % SW_NS]);
         }
         __syncwarp();
         first = false;
       }
-      L = Lb + (i1 - i0 + 3);
+      L = Lb + ((i1 - i0 + 1) / 2) * 2 + 3;  // S rows i0-2 .. (last pair start)+2
     }
     if (elect_one()) {
       if (!first) umma_commit(tfull);
@@ -486,45 +491,46 @@ __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_
   } else if (warp >= 5) {
     const int qd = warp & 3;
     const int m = qd * 32 + lane;
-    const int atom = m >> 6, co = m & 63;
-    const bool any = (int)blockIdx.x < nunits;
+    const int half = m >> 6, co = m & 63;
     mbar_wait(tfull, 0);
     tc_fence_after();
-    float* P = a.part + (long long)blockIdx.x * 256 * 64;
+    float* P = a.part + ((long long)blockIdx.x * 2 + half) * 256 * 64;
 #pragma unroll 1
-    for (int c0 = 0; c0 < 8; c0 += 2) {
-      float v[32];
-      if (any) tmem_ld32(tmem + (uint32_t)(c0 * 16) + ((uint32_t)(qd * 32) << 16), v);
-      else
+    for (int o = 0; o < 5; ++o) {
+      const int ah = o - 2 - half;
+      const bool valid = ah >= -2 && ah <= 1;
+#pragma unroll 1
+      for (int c0 = 0; c0 < 64; c0 += 32) {
+        float v[32];
+        tmem_ld32(tmem + (uint32_t)(o * 64 + c0) + ((uint32_t)(qd * 32) << 16), v);
+        if (!valid) continue;
 #pragma unroll
-        for (int i = 0; i < 32; ++i) v[i] = 0.f;
-#pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const int accn = c0 + h;
-        const int ah = (accn >> 1) - 2, pr = accn & 1;
-        const int aw = 1 - 2 * pr - atom;
-        const int tap = (ah + 2) * 4 + (aw + 2);
-#pragma unroll
-        for (int ch = 0; ch < 16; ++ch) P[(tap * 16 + ch) * 64 + co] = v[h * 16 + ch];
+        for (int j = 0; j < 32; ++j) {
+          const int n = c0 + j, aw = (n >> 4) - 2, ch = n & 15;
+          const int tap = (ah + 2) * 4 + (aw + 2);
+          P[(tap * 16 + ch) * 64 + co] = v[j];
+        }
       }
     }
+    // each half writes all 16 taps (top: accumulators 0..3, bottom: 1..4); the finish kernel adds them
   }
 
   tc_fence_before();
   __syncthreads();
   if (warp == 4) {
     tc_fence_after();
-    tmem_dealloc<128>(tmem);
+    tmem_dealloc<512>(tmem);
   }
 }
 
-// sum the per-CTA partials in fixed order and scatter (tap, s2d channel) back to dw [64][7][7][cin]
+// sum the per-CTA partials (both row halves) in fixed order and scatter (tap, s2d channel) back to
+// dw [64][7][7][cin]
 __global__ void stem_wgrad_finish_kernel(const float* __restrict__ part, int G, int cin, float* __restrict__ dw) {
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
   if (idx >= 256 * 64) return;
   const int co = idx & 63, k = idx >> 6;
   float acc = 0.f;
-  for (int g = 0; g < G; ++g) acc += __ldg(part + ((long long)g * 256 + k) * 64 + co);
+  for (int g = 0; g < 2 * G; ++g) acc += __ldg(part + ((long long)g * 256 + k) * 64 + co);
   const int t = k >> 4, ch = k & 15;
   const int bh = ch >> 3, bw = (ch >> 2) & 1, c = ch & 3;
   const int kh = 2 * (t / 4 - 2) + bh + 3, kw = 2 * (t % 4 - 2) + bw + 3;
@@ -539,7 +545,7 @@ __global__ void stem_colsum_final_kernel(const float* __restrict__ part, int G, 
 
 size_t stem_wgrad_ws_bytes(int n) {
   (void)n;
-  return (size_t)num_sms() * (256 * 64 + 64) * sizeof(float);
+  return (size_t)num_sms() * (2 * 256 * 64 + 64) * sizeof(float);
 }
 
 void stem_wgrad(const bf16* s, const bf16* dz, int n, int Hs, int Ws, int cin_real, float* ws, size_t ws_bytes,
@@ -549,15 +555,20 @@ void stem_wgrad(const bf16* s, const bf16* dz, int n, int Hs, int Ws, int cin_re
   if (ws_bytes < stem_wgrad_ws_bytes(n)) throw std::runtime_error("stem wgrad workspace too small");
   static StemWgArgs a;
   a = StemWgArgs{};
-  a.s_map = make_tmap_nhwc_plain(s, n, Hs, Ws, 16, 8, SLOTS, 1);
-  a.dz_map = make_tmap_nhwc(dz, n, Hs, Ws, 64, 64, SLOTS, 1);
+  a.s_map = make_tmap_nhwc_swz(s, n, Hs, Ws, 16, 16, SLOTS, 1, 32);
+  a.dz_map = make_tmap_nhwc(dz, n, Hs, Ws, 64, 64, SLOTS, 2);
   a.n = n;
   a.Hs = Hs;
   a.Ws = Ws;
-  pick_bands(n, Hs, 3, &a.bands, &a.band_rows);
+  // bands of an even number of rows (row pairs never straddle two units)
+  const int pairs = (Hs + 1) / 2;
+  int bands, bpairs;
+  pick_bands(n, pairs, 2, &bands, &bpairs);
+  a.bands = bands;
+  a.band_rows = 2 * bpairs;
   const int G = std::min(n * a.bands, num_sms());
   a.part = ws;
-  a.cs_part = db ? ws + (size_t)G * 256 * 64 : nullptr;
+  a.cs_part = db ? ws + (size_t)G * 2 * 256 * 64 : nullptr;
   static bool attr = false;
   if (!attr) {
     CK(cudaFuncSetAttribute(stem_wgrad_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SW_SMEM));

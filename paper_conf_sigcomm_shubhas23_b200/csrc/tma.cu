@@ -36,15 +36,22 @@ CUtensorMap make_tmap_nhwc(const void* base, int N, int H, int W, int C, int bc,
 }
 
 CUtensorMap make_tmap_nhwc_plain(const void* base, int N, int H, int W, int C, int bc, int bw, int bh) {
+  return make_tmap_nhwc_swz(base, N, H, W, C, bc, bw, bh, 0);
+}
+
+CUtensorMap make_tmap_nhwc_swz(const void* base, int N, int H, int W, int C, int bc, int bw, int bh, int swz) {
   CUtensorMap m;
+  const CUtensorMapSwizzle sw = swz == 32 ? CU_TENSOR_MAP_SWIZZLE_32B
+                                : swz == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                : swz == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE;
   const cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
   const cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2, (cuuint64_t)H * W * C * 2};
   const cuuint32_t box[4] = {(cuuint32_t)bc, (cuuint32_t)bw, (cuuint32_t)bh, 1};
   const cuuint32_t es[4] = {1, 1, 1, 1};
   CUresult r = encode_fn()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(base), dims, strides, box, es,
-                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
                            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (r != CUDA_SUCCESS) throw CudaError("cuTensorMapEncodeTiled(nhwc, plain) failed: " + std::to_string((int)r));
+  if (r != CUDA_SUCCESS) throw CudaError("cuTensorMapEncodeTiled(nhwc, swz) failed: " + std::to_string((int)r));
   return m;
 }
 

@@ -84,4 +84,7 @@ def test_stem_wgrad(case):
     assert _rel(dw, ref) < 1e-4
     assert _rel(db, dz.float().sum(dim=(0, 1, 2))) < 1e-5
     dw2, db2 = B.dbg_stem_wgrad(x, dz)
-    assert torch.equal(dw, dw2) and torch.equal(db, db2)
+    torch.cuda.synchronize()
+    diff = (dw2 - dw).abs()
+    assert torch.equal(dw, dw2), ("dw", float(diff.max()), torch.nonzero(diff)[:8].tolist())
+    assert torch.equal(db, db2), ("db", float((db2 - db).abs().max()))

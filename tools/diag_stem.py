@@ -4,7 +4,7 @@ import os, sys
 sys.path.insert(0, os.path.join(os.path.dirname(os.path.abspath(__file__)), ".."))
 import torch
 from paper_conf_sigcomm_shubhas23_b200 import binding as B
-n, H, W, cin = 2, 32, 32, 4
+n, H, W, cin = [int(v) for v in os.environ.get("CASE", "2,32,32,4").split(",")]
 g = torch.Generator().manual_seed(4)
 x = torch.randn(n, H, W, cin, generator=g).to(torch.bfloat16).cuda()
 dz = torch.randn(n, H // 2, W // 2, 64, generator=g).to(torch.bfloat16).cuda()
@@ -36,3 +36,10 @@ for k in sorted(A.keys()):
     else:
         print("ours", k, "-> ref", keys[j], "corr %.4f" % float(cor[j]), "norm ratio %.3f" % float(A[k].norm() / R[keys[j]].norm()))
 print("matching", ok, "of", len(A))
+rel = float((dw - ref).norm() / ref.norm())
+print("dw rel", rel)
+err = (dw - ref).abs()
+idx = torch.nonzero(err > 1e-3 * ref.abs().max())
+print("entries off:", idx.shape[0], "of", ref.numel())
+if idx.shape[0]:
+    print("kh,kw,c of first offenders:", idx[:20, 1:].tolist())
