@@ -42,7 +42,7 @@ void launch_pack_input(const bf16* x, const int* map, const int* count, int n_st
 // ------------------------------------------------------------------------------------------------
 __global__ void maxpool_fwd_kernel(const bf16* __restrict__ x, const int* __restrict__ map, const int* count,
                                    int n_static, int H, int W, int C, int K, int s, int p, int Ho, int Wo,
-                                   bf16* __restrict__ y, uint8_t* __restrict__ amax) {
+                                   bf16* __restrict__ y, uint8_t* __restrict__ amax, int fold_relu) {
   const int n_rows = count ? *count : n_static;
   const int CV = C / 8;
   const long long total = (long long)n_rows * Ho * Wo * CV;
@@ -84,16 +84,20 @@ __global__ void maxpool_fwd_kernel(const bf16* __restrict__ x, const int* __rest
     for (int q = 0; q < 8; ++q) o[q] = __float2bfloat16_rn(best[q]);
     const long long oi = ((n * Ho + ho) * Wo + wo) * C + cv * 8;
     *(uint4*)(y + oi) = *(uint4*)o;
+    if (fold_relu)  // ReLU producer: a window whose max is not > 0 routes no gradient (act'(y) = 0)
+#pragma unroll
+      for (int q = 0; q < 8; ++q)
+        if (!(best[q] > 0.f)) arg[q] = AMAX_MASKED;
     if (amax) *(uint2*)(amax + oi) = *(uint2*)arg;
   }
 }
 void launch_maxpool_fwd(const bf16* x, const int* map, const int* count, int n_static, int H, int W, int C, int K,
-                        int s, int p, int Ho, int Wo, bf16* y, uint8_t* amax, cudaStream_t st) {
+                        int s, int p, int Ho, int Wo, bf16* y, uint8_t* amax, int fold_relu, cudaStream_t st) {
   const long long total = (long long)n_static * Ho * Wo * (C / 8);
   const int blocks = (int)std::min<long long>((total + 255) / 256, 32LL * num_sms());
   if (blocks <= 0) return;
   ProfScope ps(PC_POOL_FWD, st);
-  maxpool_fwd_kernel<<<blocks, 256, 0, st>>>(x, map, count, n_static, H, W, C, K, s, p, Ho, Wo, y, amax);
+  maxpool_fwd_kernel<<<blocks, 256, 0, st>>>(x, map, count, n_static, H, W, C, K, s, p, Ho, Wo, y, amax, fold_relu);
   CK(cudaGetLastError());
 }
 
@@ -129,14 +133,15 @@ __global__ void maxpool_bwd_kernel(const bf16* __restrict__ dT, const uint8_t* _
         const uint8_t* a8 = (const uint8_t*)&am;
         const uint4 dv = __ldg((const uint4*)(dT + oi));
         const bf16* d8 = (const bf16*)&dv;
-        const uint4 pv = __ldg((const uint4*)(pooled + oi));
+        uint4 pv = make_uint4(0u, 0u, 0u, 0u);
+        if (act != 1) pv = __ldg((const uint4*)(pooled + oi));  // ReLU: mask folded into the codes
         const bf16* p8 = (const bf16*)&pv;
         const uint8_t me = (uint8_t)(kh * K + kw);
 #pragma unroll
         for (int q = 0; q < 8; ++q)
           if (a8[q] == me) {
             acc[q] = __fadd_rn(acc[q], __bfloat162float(d8[q]));
-            m[q] = act_grad(act, __bfloat162float(p8[q]));
+            m[q] = act == 1 ? 1.f : act_grad(act, __bfloat162float(p8[q]));
           }
       }
     }
@@ -180,14 +185,16 @@ __global__ void maxpool_bwd_s2_kernel(const bf16* __restrict__ dT, const uint8_t
         const uint8_t* a8 = (const uint8_t*)&am;
         const uint4 dv = __ldg((const uint4*)(dT + oi));
         const bf16* d8 = (const bf16*)&dv;
-        const uint4 pv = __ldg((const uint4*)(pooled + oi));
+        uint4 pv = make_uint4(0u, 0u, 0u, 0u);
+        if (act != 1) pv = __ldg((const uint4*)(pooled + oi));  // ReLU: mask folded into the codes
         const bf16* p8 = (const bf16*)&pv;
 #pragma unroll
         for (int q = 0; q < 8; ++q) {
+          if (a8[q] == AMAX_MASKED) continue;
           const int kh = a8[q] / K, kw = a8[q] - (a8[q] / K) * K;
           const int u = ho * 2 - p + kh - ih0, v = wo * 2 - p + kw - iw0;
           const float g = __bfloat162float(d8[q]);
-          const float mg = act_grad(act, __bfloat162float(p8[q]));
+          const float mg = act == 1 ? 1.f : act_grad(act, __bfloat162float(p8[q]));
 #pragma unroll
           for (int uu = 0; uu < 2; ++uu)
 #pragma unroll
@@ -213,10 +220,76 @@ __global__ void maxpool_bwd_s2_kernel(const bf16* __restrict__ dT, const uint8_t
   }
 }
 
+// 3x3 / stride 2 / pad 1 (the ResNet stem pool) with the ReLU mask folded into the codes (or no activation):
+// one thread per (n, 2x2 input block, 8-channel vector).  Block (bi, bj) is covered by windows (bi|bi+1, bj|bj+1)
+// only; each of its four positions has a fixed set of (window, code) pairs that can select it:
+//   (0,0): w00 code 4     (0,1): w00 5, w01 3     (1,0): w00 7, w10 1     (1,1): w00 8, w01 6, w10 2, w11 0
+// summed in window order (ho, then wo ascending) like the generic kernels.  128-bit dT loads, 64-bit codes,
+// no reads of the pooled tensor.
+__global__ void __launch_bounds__(256) maxpool_bwd_k3s2_kernel(const bf16* __restrict__ dT,
+                                                               const uint8_t* __restrict__ amax, long long n, int H,
+                                                               int W, int C, int Ho, int Wo, bf16* __restrict__ dz) {
+  const int CV = C / 8;
+  const int BH = (H + 1) / 2, BW = (W + 1) / 2;
+  const long long total = n * BH * BW * CV;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+    const int cv = (int)(i % CV);
+    long long r = i / CV;
+    const int bj = (int)(r % BW);
+    r /= BW;
+    const int bi = (int)(r % BH);
+    const long long b = r / BH;
+    uint2 cw[4];
+    uint4 gw[4];
+#pragma unroll
+    for (int wq = 0; wq < 4; ++wq) {
+      const int ho = bi + (wq >> 1), wo = bj + (wq & 1);
+      if (ho < Ho && wo < Wo) {
+        const long long oi = ((b * Ho + ho) * Wo + wo) * C + cv * 8;
+        cw[wq] = __ldg((const uint2*)(amax + oi));
+        gw[wq] = __ldg((const uint4*)(dT + oi));
+      } else {
+        cw[wq] = make_uint2(0xFFFFFFFFu, 0xFFFFFFFFu);
+        gw[wq] = make_uint4(0u, 0u, 0u, 0u);
+      }
+    }
+    __align__(16) bf16 o00[8], o01[8], o10[8], o11[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const uint32_t c00 = ((const uint8_t*)&cw[0])[q], c01 = ((const uint8_t*)&cw[1])[q];
+      const uint32_t c10 = ((const uint8_t*)&cw[2])[q], c11 = ((const uint8_t*)&cw[3])[q];
+      const float g00 = __bfloat162float(((const bf16*)&gw[0])[q]), g01 = __bfloat162float(((const bf16*)&gw[1])[q]);
+      const float g10 = __bfloat162float(((const bf16*)&gw[2])[q]), g11 = __bfloat162float(((const bf16*)&gw[3])[q]);
+      const float a00 = c00 == 4 ? g00 : 0.f;
+      const float a01 = __fadd_rn(c00 == 5 ? g00 : 0.f, c01 == 3 ? g01 : 0.f);
+      const float a10 = __fadd_rn(c00 == 7 ? g00 : 0.f, c10 == 1 ? g10 : 0.f);
+      const float a11 = __fadd_rn(__fadd_rn(__fadd_rn(c00 == 8 ? g00 : 0.f, c01 == 6 ? g01 : 0.f), c10 == 2 ? g10 : 0.f),
+                                  c11 == 0 ? g11 : 0.f);
+      o00[q] = __float2bfloat16_rn(a00);
+      o01[q] = __float2bfloat16_rn(a01);
+      o10[q] = __float2bfloat16_rn(a10);
+      o11[q] = __float2bfloat16_rn(a11);
+    }
+    const int ih = 2 * bi, iw = 2 * bj;
+    bf16* d0 = dz + ((b * H + ih) * W + iw) * C + cv * 8;
+    *(uint4*)d0 = *(const uint4*)o00;
+    if (iw + 1 < W) *(uint4*)(d0 + C) = *(const uint4*)o01;
+    if (ih + 1 < H) {
+      bf16* d1 = d0 + (long long)W * C;
+      *(uint4*)d1 = *(const uint4*)o10;
+      if (iw + 1 < W) *(uint4*)(d1 + C) = *(const uint4*)o11;
+    }
+  }
+}
+
 void launch_maxpool_bwd(const bf16* dT, const uint8_t* amax, const bf16* pooled, int act, int n, int H, int W, int C,
                         int K, int s, int p, int Ho, int Wo, bf16* dz, cudaStream_t st) {
   ProfScope ps(PC_POOL_BWD, st);
-  if (s == 2) {
+  if (K == 3 && s == 2 && p == 1 && (act == 0 || act == 1)) {
+    const long long total = (long long)n * ((H + 1) / 2) * ((W + 1) / 2) * (C / 8);
+    const int blocks = (int)std::min<long long>((total + 255) / 256, 16LL * num_sms());
+    maxpool_bwd_k3s2_kernel<<<blocks, 256, 0, st>>>(dT, amax, n, H, W, C, Ho, Wo, dz);
+  } else if (s == 2) {
     const long long total = (long long)n * ((H + 1) / 2) * ((W + 1) / 2) * (C / 8);
     const int blocks = (int)std::min<long long>((total + 255) / 256, 64LL * num_sms());
     maxpool_bwd_s2_kernel<<<blocks, 256, 0, st>>>(dT, amax, pooled, act, n, H, W, C, K, p, Ho, Wo, dz);
@@ -403,41 +476,52 @@ void launch_exit_loss(const float* logits, const int32_t* labels, int n, int ncl
   CK(cudaGetLastError());
 }
 
-// dW[c][k] = sum_n pooled[n][c] dl[n][k] (+ db): one CTA per 32-channel slab, threads over (n-slice, c),
-// fixed-order partials in smem -> deterministic
-__global__ void head_dw_kernel(const float* __restrict__ pooled, const float* __restrict__ dl, int n, int C, int ncls,
-                               float* __restrict__ dW, float* __restrict__ db) {
-  __shared__ float part[8][32][33];
+// dW[c][k] = sum_n pooled[n][c] dl[n][k] (+ db = sum_n dl[n][k]): stage 1, CTA (32-channel slab, sample split)
+// writes fixed-order partials part[split][c][k] (c == C is the bias row); stage 2 sums the splits in order.
+constexpr int HEAD_SPLIT_ROWS = 32;
+__global__ void head_dw_partial_kernel(const float* __restrict__ pooled, const float* __restrict__ dl, int n, int C,
+                                       int ncls, int chunk, float* __restrict__ part) {
+  __shared__ float red[8][32][33];
   const int c = blockIdx.x * 32 + (threadIdx.x & 31);
-  const int sl = threadIdx.x >> 5;  // 8 n-slices
+  const int sl = threadIdx.x >> 5;  // 8 sample slices
   const bool bias_blk = blockIdx.x == (C + 31) / 32;
+  const int i0 = blockIdx.y * chunk, i1 = min(n, i0 + chunk);
+  float* out = part + (long long)blockIdx.y * (C + 1) * ncls;
   for (int k0 = 0; k0 < ncls; k0 += 32) {
     float acc[32];
 #pragma unroll
     for (int k = 0; k < 32; ++k) acc[k] = 0.f;
-    for (int i = sl; i < n; i += 8) {
-      const float pv = bias_blk ? 1.f : (c < C ? pooled[(long long)i * C + c] : 0.f);
+    for (int i = i0 + sl; i < i1; i += 8) {
+      const float pv = bias_blk ? 1.f : (c < C ? __ldg(pooled + (long long)i * C + c) : 0.f);
       const float* d = dl + (long long)i * ncls + k0;
 #pragma unroll
       for (int k = 0; k < 32; ++k)
         if (k0 + k < ncls) acc[k] = fmaf(pv, __ldg(d + k), acc[k]);
     }
 #pragma unroll
-    for (int k = 0; k < 32; ++k) part[sl][threadIdx.x & 31][k] = acc[k];
+    for (int k = 0; k < 32; ++k) red[sl][threadIdx.x & 31][k] = acc[k];
     __syncthreads();
-    if (sl == 0) {
-      for (int k = 0; k < 32 && k0 + k < ncls; ++k) {
-        float s = 0.f;
-        for (int q = 0; q < 8; ++q) s += part[q][threadIdx.x & 31][k];
-        if (bias_blk) {
-          if ((threadIdx.x & 31) == 0) db[k0 + k] = s;
-        } else if (c < C) {
-          dW[(long long)c * ncls + k0 + k] = s;
-        }
-      }
+    for (int e = threadIdx.x; e < 32 * 32; e += 256) {
+      const int cc = e >> 5, k = e & 31;
+      const int ch = bias_blk ? C : blockIdx.x * 32 + cc;
+      if (k0 + k >= ncls || (bias_blk ? cc != 0 : ch >= C)) continue;
+      float sum = 0.f;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) sum += red[q][cc][k];
+      out[(long long)ch * ncls + k0 + k] = sum;
     }
     __syncthreads();
   }
+}
+__global__ void head_dw_final_kernel(const float* __restrict__ part, int splits, int C, int ncls,
+                                     float* __restrict__ dW, float* __restrict__ db) {
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  const int per = (C + 1) * ncls;
+  if (e >= per) return;
+  float sum = 0.f;
+  for (int sp = 0; sp < splits; ++sp) sum += __ldg(part + (long long)sp * per + e);
+  if (e < C * ncls) dW[e] = sum;
+  else db[e - C * ncls] = sum;
 }
 __global__ void head_bcast_kernel(const float* __restrict__ dl, const float* __restrict__ Wk, int n, int C, int ncls,
                                   float inv_hw, float* __restrict__ bcast) {
@@ -449,18 +533,53 @@ __global__ void head_bcast_kernel(const float* __restrict__ dl, const float* __r
   for (int k = 0; k < ncls; ++k) acc = fmaf(dl[i * ncls + k], Wk[c * ncls + k], acc);
   bcast[idx] = acc * inv_hw;
 }
+size_t head_grads_ws_bytes(int n, int C, int ncls) {
+  const int splits = std::max(1, std::min(64, (n + HEAD_SPLIT_ROWS - 1) / HEAD_SPLIT_ROWS));
+  return (size_t)splits * (C + 1) * ncls * sizeof(float);
+}
 void launch_head_grads(const float* pooled, const float* dl, const float* Wk, int n, int C, int ncls, int HW,
-                       float* dW, float* db, float* bcast, cudaStream_t st) {
-  ProfScope ps(PC_HEAD_GRADS, st, 2);
-  head_dw_kernel<<<(C + 31) / 32 + 1, 256, 0, st>>>(pooled, dl, n, C, ncls, dW, db);
+                       float* dW, float* db, float* bcast, float* ws, cudaStream_t st) {
+  ProfScope ps(PC_HEAD_GRADS, st, 3);
+  const int splits = std::max(1, std::min(64, (n + HEAD_SPLIT_ROWS - 1) / HEAD_SPLIT_ROWS));
+  const int chunk = (n + splits - 1) / splits;
+  head_dw_partial_kernel<<<dim3((C + 31) / 32 + 1, splits), 256, 0, st>>>(pooled, dl, n, C, ncls, chunk, ws);
+  head_dw_final_kernel<<<((C + 1) * ncls + 255) / 256, 256, 0, st>>>(ws, splits, C, ncls, dW, db);
   const long long nb = ((long long)n * C + 255) / 256;
   head_bcast_kernel<<<(unsigned)nb, 256, 0, st>>>(dl, Wk, n, C, ncls, 1.0f / (float)HW, bcast);
   CK(cudaGetLastError());
 }
 
+// one thread per 8-channel vector (C % 8 == 0): 128-bit bf16 loads / stores, float4 bcast loads
 __global__ void grad_finalize_kernel(const float* __restrict__ bcast, const bf16* __restrict__ sc,
                                      const bf16* __restrict__ yact, int act, long long n, int HW, int C,
                                      bf16* __restrict__ dz) {
+  const int CV = C / 8;
+  const long long total = n * HW * CV;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+    const int cv = (int)(i % CV);
+    const long long b = i / ((long long)HW * CV);
+    float v[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) v[q] = 0.f;
+    if (bcast) {
+      const float4 b0 = __ldg((const float4*)(bcast + b * C + cv * 8)), b1 = __ldg((const float4*)(bcast + b * C + cv * 8 + 4));
+      v[0] = b0.x, v[1] = b0.y, v[2] = b0.z, v[3] = b0.w, v[4] = b1.x, v[5] = b1.y, v[6] = b1.z, v[7] = b1.w;
+    }
+    if (sc) {
+      const uint4 r = __ldg((const uint4*)(sc + i * 8));
+#pragma unroll
+      for (int q = 0; q < 8; ++q) v[q] = __fadd_rn(v[q], __bfloat162float(((const bf16*)&r)[q]));
+    }
+    const uint4 y = __ldg((const uint4*)(yact + i * 8));
+    __align__(16) bf16 o[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) o[q] = __float2bfloat16_rn(__fmul_rn(v[q], act_grad(act, __bfloat162float(((const bf16*)&y)[q]))));
+    *(uint4*)(dz + i * 8) = *(const uint4*)o;
+  }
+}
+__global__ void grad_finalize_scalar_kernel(const float* __restrict__ bcast, const bf16* __restrict__ sc,
+                                            const bf16* __restrict__ yact, int act, long long n, int HW, int C,
+                                            bf16* __restrict__ dz) {
   const long long total = n * HW * C;
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
     const int c = (int)(i % C);
@@ -477,7 +596,12 @@ void launch_grad_finalize(const float* bcast, const bf16* sc, const bf16* yact, 
   const long long total = (long long)n * HW * C;
   const int blocks = (int)std::min<long long>((total + 255) / 256, 32LL * num_sms());
   ProfScope ps(PC_GRAD_FINALIZE, st);
-  grad_finalize_kernel<<<blocks, 256, 0, st>>>(bcast, sc, yact, act, n, HW, C, dz);
+  if (C % 8 == 0) {
+    const int vb = (int)std::min<long long>((total / 8 + 255) / 256, 32LL * num_sms());
+    grad_finalize_kernel<<<vb, 256, 0, st>>>(bcast, sc, yact, act, n, HW, C, dz);
+  } else {
+    grad_finalize_scalar_kernel<<<blocks, 256, 0, st>>>(bcast, sc, yact, act, n, HW, C, dz);
+  }
   CK(cudaGetLastError());
 }
 

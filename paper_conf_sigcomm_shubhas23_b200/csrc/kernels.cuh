@@ -11,11 +11,15 @@ namespace adainf {
 void launch_pack_input(const bf16* x, const int* map, const int* count, int n_static, int H, int W, int Cin, int Cpad,
                        bf16* y, cudaStream_t st);
 
-// maxpool fwd (NHWC bf16); optional input map; optional argmax offsets (uint8) for backward
+// argmax code of a window whose ReLU producer output is not > 0: routes no gradient (act' = 0)
+constexpr uint8_t AMAX_MASKED = 0xFF;
+// maxpool fwd (NHWC bf16); optional input map; optional argmax offsets (uint8, kh*K+kw of the FIRST maximum)
+// for backward; fold_relu (producer activation ReLU) stores AMAX_MASKED where the window max is not > 0
 void launch_maxpool_fwd(const bf16* x, const int* map, const int* count, int n_static, int H, int W, int C, int K,
-                        int s, int p, int Ho, int Wo, bf16* y, uint8_t* argmax, cudaStream_t st);
-// maxpool bwd fused with the producer's activation mask: dz = bf16(sum_windows dT * [first argmax]) * act'(y),
-// the mask taken from the pooled output P (= y at the selected position)
+                        int s, int p, int Ho, int Wo, bf16* y, uint8_t* argmax, int fold_relu, cudaStream_t st);
+// maxpool bwd fused with the producer's activation mask: dz = bf16(sum_windows dT * [first argmax]) * act'(y).
+// act == 1 (ReLU): the mask is folded into the argmax codes (AMAX_MASKED) and `pooled` is not read;
+// otherwise the mask is taken from the pooled output P (= y at the selected position)
 void launch_maxpool_bwd(const bf16* dT, const uint8_t* argmax, const bf16* pooled, int act, int n, int H, int W, int C,
                         int K, int s, int p, int Ho, int Wo, bf16* dz, cudaStream_t st);
 
@@ -56,8 +60,11 @@ void launch_compact(const uint8_t* alive, const int* count, int n_static, const 
 void launch_exit_loss(const float* logits, const int32_t* labels, int n, int ncls, float w, float inv_n, float* dl,
                       float* loss_rows, int accumulate, cudaStream_t st);
 // head grads: dW[c][j] = sum_n pooled[n][c] dl[n][j]; db[j] = sum_n dl[n][j]; bcast[n][c] = (sum_j dl W[c][j]) / HW
+// exit-head gradients: dW = pooled^T dl, db = colsum(dl) (deterministic split over samples, partials in `ws`
+// of head_grads_ws_bytes), bcast = dl Wk^T / HW (the GAP broadcast added to the exit tensor's gradient)
+size_t head_grads_ws_bytes(int n, int C, int ncls);
 void launch_head_grads(const float* pooled, const float* dl, const float* Wk, int n, int C, int ncls, int HW,
-                       float* dW, float* db, float* bcast, cudaStream_t st);
+                       float* dW, float* db, float* bcast, float* ws, cudaStream_t st);
 // dz = bf16((bcast[n][c] + sc) * act'(y))
 void launch_grad_finalize(const float* bcast, const bf16* sc, const bf16* yact, int act, int n, int HW, int C,
                           bf16* dz, cudaStream_t st);

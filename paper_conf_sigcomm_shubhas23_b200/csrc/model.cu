@@ -366,6 +366,7 @@ void Model::ensure_training() {
       if (nd.kind == N_PROJ && nd.in != 0) nd.proj_dx.alloc((size_t)max_batch * T[nd.in].row_elems() * 2);
     }
   }
+  for (auto& e : exits) ws = std::max(ws, head_grads_ws_bytes(max_batch, T[e.tensor].C, e.ncls));
   wgrad_ws.alloc(ws);
   wgrad_ws_bytes = ws;
   for (auto& e : exits) {
@@ -417,7 +418,8 @@ void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, in
       if (nd.kind == N_POOL) {
         if (stem_s2d && ni == stem_pool) continue;  // produced by the fused stem
         launch_maxpool_fwd(buf_of(nd.in), map_for(nd.in, ns), c, n_static, nd.g.H, nd.g.W, nd.g.Cin, nd.pk, nd.ps,
-                           nd.pp, nd.g.Ho, nd.g.Wo, T[nd.out].buf, train ? nd.argmax.as<uint8_t>() : nullptr, st);
+                           nd.pp, nd.g.Ho, nd.g.Wo, T[nd.out].buf, train ? nd.argmax.as<uint8_t>() : nullptr,
+                           nd.in > 0 && T[nd.in].act == 1, st);
       } else {
         const float* bias = params.as<float>() + nd.b_off;
         const bf16* res = nd.res >= 0 ? T[nd.res].buf : nullptr;
@@ -516,7 +518,7 @@ void Model::train_step(const bf16* x, const int32_t* labels, int n, long long n_
     launch_exit_loss(e.logits.as<float>(), labels, n, e.ncls, e.lw, inv_n, e.dl.as<float>(), loss_rows.as<float>(),
                      k > 0, st);
     launch_head_grads(e.pooled.as<float>(), e.dl.as<float>(), P + e.w_off, n, X.C, e.ncls, X.H * X.W, G + e.w_off,
-                      G + e.b_off, e.bcast.as<float>(), st);
+                      G + e.b_off, e.bcast.as<float>(), wgrad_ws.as<float>(), st);
   }
   auto buf_of = [&](int t) -> const bf16* { return t == 0 ? x0 : T[t].buf; };
   auto bcast_of = [&](int t) -> const float* { return T[t].exit_k >= 0 ? exits[T[t].exit_k].bcast.as<float>() : nullptr; };

@@ -287,6 +287,13 @@ __global__ void __launch_bounds__(SF_THREADS, 1) stem_fwd_kernel(const __grid_co
                 arg[w] = (arg[w] & ~pm) | (kk & pm);
               }
             }
+            // ReLU producer: a window whose max is 0 routes no gradient -> AMAX_MASKED (0xFF) code
+#pragma unroll
+            for (int w = 0; w < 2; ++w) {
+              const __nv_bfloat162 z2 = __float2bfloat162_rn(0.f);
+              const uint32_t z0 = __heq2_mask(best[2 * w], z2), z1 = __heq2_mask(best[2 * w + 1], z2);
+              arg[w] |= __byte_perm(z0, z1, 0x6420);
+            }
             *(uint2*)(a.argmax + oi) = make_uint2(arg[0], arg[1]);
           }
         }
