@@ -54,6 +54,14 @@ extern "C" adainf_status adainf_dbg_conv_dgrad(const void* dz, int32_t n, int32_
     if (C % 8 || Co % 8 || n <= 0) throw ShapeError("conv_dgrad: C, Co must be multiples of 8");
     require_device();
     ConvGeom g = geom(H, W, C, Co, KH, KW, stride, pad);
+    if (dgrad_sp_ok(g)) {  // the runtime's route for stride-2 3x3 layers (one sub-pixel GEMM)
+      bf16* wsp = nullptr;
+      CK(cudaMallocAsync((void**)&wsp, dgrad_sp_ws_bytes(g), (cudaStream_t)stream));
+      conv_dgrad_sp(g, (const bf16*)dz, (const bf16*)w, KH * KW * C, wsp, n, bcast, (const bf16*)sc, false,
+                    (const bf16*)yact, mask_act, (bf16*)dx, (cudaStream_t)stream);
+      CK(cudaFreeAsync(wsp, (cudaStream_t)stream));
+      return;
+    }
     conv_dgrad(g, (const bf16*)dz, (const bf16*)w, KH * KW * C, n, bcast, (const bf16*)sc, (const bf16*)yact,
                mask_act, (bf16*)dx, (cudaStream_t)stream);
   });

@@ -20,10 +20,20 @@
 //              terms and masks -> 128-bit global stores; frees the accumulator after the last load
 #pragma once
 #include "common.cuh"
+#include "tma.cuh"
 
 namespace adainf {
 
-enum { MODE_FWD = 0, MODE_DGRAD = 1, MODE_WGRAD = 2 };
+enum { MODE_FWD = 0, MODE_DGRAD = 1, MODE_WGRAD = 2, MODE_DGRAD_SP = 3 };
+// MODE_DGRAD_SP: stride-2 dgrad as ONE sub-pixel GEMM over the dZ grid (instead of 4 output-phase launches):
+//   D[(n,y',x')][(py,px,ci)] = sum_{(a,b) in {0,1}^2, co} dZ[n][y'+a][x'+b][co] * Bsp[(py,px,ci)][(a,b,co)]
+//   with Bsp = W[co][kh = py+p-2a][kw = px+p-2b][ci] (zero where the tap does not exist); the epilogue writes
+//   column block (py,px) to dX[n][2y'+py][2x'+px].  N = 4*Cin instead of Cin: 4x fewer A-operand loads per MMA.
+template <int MODE>
+struct ModeTraits {
+  static constexpr bool B_KMAJ = MODE == MODE_FWD || MODE == MODE_DGRAD_SP;  // B K-major ([N][K] rows)
+  static constexpr bool DG_EPI = MODE == MODE_DGRAD || MODE == MODE_DGRAD_SP;
+};
 constexpr int MAX_TAPS = 49;
 
 struct ConvArgs {
@@ -58,6 +68,13 @@ struct ConvArgs {
   int kb_per_split;     // WGRAD split-K (in 64-pixel blocks)
   int splits;           // WGRAD number of splits
   int exp_flags;        // experiments only (ADAINF_EXP): bit0 skip epilogue stores, bit1 skip bias/res loads
+  // ---- optional TMA for the B (weight) operand of FWD / DGRAD: one elected producer thread issues the
+  // bulk tensor loads (FWD: one {64 K, BN rows} box of the K-major shadow; DGRAD: BN/64 {64 ci, 64 co} boxes
+  // that land as the MN-major SW128 atoms) instead of 128 threads issuing BN*8 cp.async each K-block ----
+  int b_tma;
+  int sp_cin;           // DGRAD_SP: Cin of the output (column block width); sp_sc_compact: sc is indexed by
+  int sp_sc_compact;    // the dZ-grid row m and applies to phase (0,0) only (compact projection dgrad)
+  CUtensorMap b_map;
 };
 
 constexpr int BM = 128, BK = 64;
@@ -136,9 +153,9 @@ __device__ __forceinline__ void ld_bf16x8(const bf16* p, float* v) {
 }
 
 template <int MODE, int BN>
-__global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArgs a) {
+__global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_constant__ ConvArgs a) {
   using Cfg = ConvCfg<MODE, BN>;
-  static_assert(MODE == MODE_FWD || BN >= 64, "MN-major SW128 B tiles need >= 64 columns");
+  static_assert(ModeTraits<MODE>::B_KMAJ || BN >= 64, "MN-major SW128 B tiles need >= 64 columns");
   constexpr int STAGES = Cfg::STAGES;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -158,8 +175,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
   if ((int)blockIdx.x >= ntile) return;  // uniform: nothing for this CTA
 
   if (threadIdx.x == 0) {
+    const bool btma = MODE != MODE_WGRAD && a.b_tma;
     for (int s = 0; s < STAGES; ++s) {
-      mbar_init(&full[s], 128);
+      mbar_init(&full[s], btma ? 129 : 128);  // 128 cp.async arrivals (+1 expect_tx arrival of the B TMA)
       mbar_init(&empty[s], 1);
     }
     for (int b = 0; b < 2; ++b) {
@@ -241,7 +259,21 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
               cp_async16(sa + kmaj_off(r, j), g, v);
             }
           }
-          if (MODE == MODE_FWD) {
+          if (a.b_tma) {
+            if (t == 0) {
+              mbar_expect_tx(&full[s], (uint32_t)Cfg::B_BYTES);
+              const int kb64 = (ti.kb0 + kbi) * BK;
+              if (ModeTraits<MODE>::B_KMAJ) {
+                tma_load_2d(sb, &a.b_map, &full[s], kb64, ti.n0);
+              } else {
+                const int tp = kb64 / a.Cs;  // host guarantees Cs % 64 == 0: the K-block lies in one tap
+                const int co0 = kb64 - tp * a.Cs;
+#pragma unroll
+                for (int b = 0; b < BN / 64; ++b)
+                  tma_load_2d(sb + b * 8192, &a.b_map, &full[s], a.btap[tp] * a.Nout + ti.n0 + b * 64, co0);
+              }
+            }
+          } else if (ModeTraits<MODE>::B_KMAJ) {
             // W [Nout][ldb] K-major: BN rows x 8 chunks
 #pragma unroll
             for (int idx = t; idx < BN * 8; idx += 128) {
@@ -355,7 +387,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
     }
   } else if (warp == 4) {
     // ================= MMA issuer =================
-    constexpr uint32_t IDESC = make_idesc(BM, BN, MODE == MODE_WGRAD ? 1 : 0, MODE == MODE_FWD ? 0 : 1);
+    constexpr uint32_t IDESC = make_idesc(BM, BN, MODE == MODE_WGRAD ? 1 : 0, ModeTraits<MODE>::B_KMAJ ? 0 : 1);
     int it = 0, lt = 0;
     for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++lt) {
       const TileInfo ti = tile_info<MODE, BN>(a, tile, mt, nt, nkb_total);
@@ -377,7 +409,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
             uint64_t ad, bd;
             if (MODE == MODE_WGRAD) ad = make_sdesc(sa + kk * 2048, 8192, 1024);
             else ad = make_sdesc(sa + kk * 32, 16, 1024);
-            if (MODE == MODE_FWD) bd = make_sdesc(sb + kk * 32, 16, 1024);
+            if (ModeTraits<MODE>::B_KMAJ) bd = make_sdesc(sb + kk * 32, 16, 1024);
             else bd = make_sdesc(sb + kk * 2048, 8192, 1024);
             umma_bf16(dacc, ad, bd, IDESC, (kbi | kk) != 0);
           }
@@ -490,22 +522,40 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
               }
             }
           } else {  // DGRAD epilogue: + bcast + shortcut, x act'(y), -> bf16
+            int ocol = cb;         // channel within the output row
+            long long srow = orow;  // row of the shortcut term
+            const bf16* scp = a.sc;
+            if (MODE == MODE_DGRAD_SP) {
+              const int ph = cb / a.sp_cin;
+              ocol = cb - ph * a.sp_cin;
+              const int pix = (int)m - n * HWg;
+              const int gy = pix / a.Wg, gx = pix - gy * a.Wg;
+              const int oy = 2 * gy + (ph >> 1), ox = 2 * gx + (ph & 1);
+              if (oy >= a.Ho || ox >= a.Wo) continue;
+              orow = ((long long)n * a.Ho + oy) * a.Wo + ox;
+              srow = orow;
+              if (a.sp_sc_compact) {
+                srow = m;
+                if (ph != 0) scp = nullptr;
+              }
+            }
+            const int NO = MODE == MODE_DGRAD_SP ? a.sp_cin : a.Nout;  // output row pitch (channels)
             if (vec) {
               if (a.bcast) {
 #pragma unroll
                 for (int i = 0; i < 32; i += 4) {
-                  const float4 bb = __ldg((const float4*)(a.bcast + (long long)n * a.Nout + cb + i));
+                  const float4 bb = __ldg((const float4*)(a.bcast + (long long)n * NO + ocol + i));
                   v[i] = __fadd_rn(v[i], bb.x);
                   v[i + 1] = __fadd_rn(v[i + 1], bb.y);
                   v[i + 2] = __fadd_rn(v[i + 2], bb.z);
                   v[i + 3] = __fadd_rn(v[i + 3], bb.w);
                 }
               }
-              if (a.sc) {
+              if (scp) {
 #pragma unroll
                 for (int i = 0; i < 32; i += 8) {
                   float r8[8];
-                  ld_bf16x8(a.sc + orow * a.Nout + cb + i, r8);
+                  ld_bf16x8(scp + srow * NO + ocol + i, r8);
 #pragma unroll
                   for (int qq = 0; qq < 8; ++qq) v[i + qq] = __fadd_rn(v[i + qq], r8[qq]);
                 }
@@ -514,24 +564,24 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const ConvArg
 #pragma unroll
                 for (int i = 0; i < 32; i += 8) {
                   float y8[8];
-                  ld_bf16x8(a.yact + orow * a.Nout + cb + i, y8);
+                  ld_bf16x8(a.yact + orow * NO + ocol + i, y8);
 #pragma unroll
                   for (int qq = 0; qq < 8; ++qq) v[i + qq] = __fmul_rn(v[i + qq], act_grad(a.mask_act, y8[qq]));
                 }
               }
-              bf16* o = (bf16*)a.out + orow * a.Nout + cb;
+              bf16* o = (bf16*)a.out + orow * NO + ocol;
 #pragma unroll
               for (int i = 0; i < 32; i += 8) st_bf16x8(o + i, v + i);
             } else {
-              bf16* o = (bf16*)a.out + orow * a.Nout + cb;
+              bf16* o = (bf16*)a.out + orow * NO + ocol;
               for (int i = 0; i < 32; ++i) {
-                const int ch = cb + i;
-                if (ch >= a.Nout) break;
+                if (cb + i >= a.Nout) break;
+                const int ch = ocol + i;
                 float x = v[i];
-                if (a.bcast) x = __fadd_rn(x, a.bcast[(long long)n * a.Nout + ch]);
-                if (a.sc) x = __fadd_rn(x, __bfloat162float(a.sc[orow * a.Nout + ch]));
+                if (a.bcast) x = __fadd_rn(x, a.bcast[(long long)n * NO + ch]);
+                if (scp) x = __fadd_rn(x, __bfloat162float(scp[srow * NO + ch]));
                 if (a.mask_act)
-                  x = __fmul_rn(x, act_grad(a.mask_act, __bfloat162float(a.yact[orow * a.Nout + ch])));
+                  x = __fmul_rn(x, act_grad(a.mask_act, __bfloat162float(a.yact[orow * NO + ch])));
                 o[i] = __float2bfloat16_rn(x);
               }
             }

@@ -35,7 +35,7 @@ static void launch_t(const ConvArgs& a, long long max_tiles, cudaStream_t st) {
     CK(cudaFuncSetAttribute(conv_umma_kernel<MODE, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
     attr = true;
   }
-  ProfScope ps(MODE == MODE_FWD ? PC_CONV_FWD : (MODE == MODE_DGRAD ? PC_CONV_DGRAD : PC_CONV_WGRAD), st);
+  ProfScope ps(MODE == MODE_FWD ? PC_CONV_FWD : (ModeTraits<MODE>::DG_EPI ? PC_CONV_DGRAD : PC_CONV_WGRAD), st);
   conv_umma_kernel<MODE, BN><<<grid, NUM_THREADS, Cfg::SMEM, st>>>(a);
   CK(cudaGetLastError());
 }
@@ -244,6 +244,16 @@ static void launch_win(WinArgs& w, int nstatic, int nout, cudaStream_t st) {
   }
 }
 
+// TMA for the weight operand of the generic kernel (ADAINF_BTMA=0 restores the cp.async B path)
+static int g_btma = -1;
+static bool btma_on() {
+  if (g_btma < 0) {
+    const char* e = getenv("ADAINF_BTMA");
+    g_btma = e ? atoi(e) : 1;
+  }
+  return g_btma != 0;
+}
+
 static int pick_bn(int nout, bool mn_major_b) {
   if (nout <= 32 && !mn_major_b) return 32;
   if (nout <= 64) return 64;
@@ -317,6 +327,10 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
   const int BN = pick_bn(g.Cout, false);
   const long long mt = ((long long)n_static * g.Ho * g.Wo + BM - 1) / BM;
   if (mt == 0) return;
+  if (btma_on() && ldb % 8 == 0 && ((uintptr_t)w & 15) == 0) {
+    a.b_tma = 1;
+    a.b_map = make_tmap_2d(w, g.Cout, a.K, ldb, 64, BN);  // K-major [Cout][K]; k >= K and rows >= Cout read 0
+  }
   launch_bn<MODE_FWD>(BN, a, mt * ((g.Cout + BN - 1) / BN), st);
 }
 
@@ -324,7 +338,10 @@ void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n
                 const bf16* sc, const bf16* yact, int mask_act, bf16* dx, cudaStream_t st) {
   check_extent((long long)n * (g.H + 1) * (g.W + 1));
   // dX[y] = sum_{kh: (y + pad - kh) % s == 0} dZ[(y + pad - kh)/s] W[kh]; split by output phase (py,px)
-  if (win_ok(g) && (g.H <= 14 || win_mode() >= 2 || (g.Cin == 64 && g.Cout == 64) || (g.W <= 28 && g.Cin % 128 == 0))) {
+  // W < 8 (ResNet layer 4): the generic kernel with TMA weight boxes beats the cp.async window kernel
+  const bool small_w_generic = g.W < 8 && btma_on() && g.Cout % 64 == 0 && g.Cin % 64 == 0 && win_mode() < 2;
+  if (win_ok(g) && !small_w_generic &&
+      (g.H <= 14 || win_mode() >= 2 || (g.Cin == 64 && g.Cout == 64) || (g.W <= 28 && g.Cin % 128 == 0))) {
     // stride 1: one window launch with flipped taps (faster at H<=14; weight-stationary at 64x64)
     WinArgs wa{};
     ConvArgs& a = wa.c;
@@ -396,8 +413,91 @@ void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n
       a.mask_act = mask_act;
       const int BN = pick_bn(g.Cin, true);
       const long long mt = ((long long)n * a.Hg * a.Wg + BM - 1) / BM;
+      if (btma_on() && g.Cout % 64 == 0 && g.Cin % 64 == 0 && BN % 64 == 0 && ldb % 8 == 0 &&
+          ((uintptr_t)w & 15) == 0) {
+        a.b_tma = 1;
+        a.b_map = make_tmap_2d(w, g.Cout, ldb, ldb, 64, 64);  // rows co, cols (tap, ci): MN-major boxes
+      }
       launch_bn<MODE_DGRAD>(BN, a, mt * ((g.Cin + BN - 1) / BN), st);
     }
+}
+
+// ---- stride-2 dgrad as one sub-pixel GEMM (see MODE_DGRAD_SP in conv_gemm.cuh) ----
+bool dgrad_sp_ok(const ConvGeom& g) {
+  return btma_on() && g.stride == 2 && g.KH == 3 && g.KW == 3 && g.pad == 1 && g.Cin % 64 == 0 &&
+         g.Cout % 64 == 0 && g.H <= 2 * g.Ho && g.W <= 2 * g.Wo && getenv("ADAINF_NO_SP") == nullptr;
+}
+size_t dgrad_sp_ws_bytes(const ConvGeom& g) { return (size_t)4 * g.Cin * 4 * g.Cout * 2; }
+
+// Bsp[(py,px,ci)][(a,b,co)] = W[co][kh = py+p-2a][kw = px+p-2b][ci], 0 where the tap does not exist.
+// One thread per (a,b,co) column and 8-channel ci vector: a 16-byte read of the shadow row, 8 strided writes.
+__global__ void sp_weight_kernel(const bf16* __restrict__ w, int ldb, int Cin, int Cout, int K, int pad,
+                                 bf16* __restrict__ bsp) {
+  const int CV = Cin / 8;
+  const long long total = 4LL * Cout * CV * 4;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+    const int cv = (int)(i % CV);
+    long long r = i / CV;
+    const int ph = (int)(r % 4);
+    const int kcol = (int)(r / 4);  // (a,b,co)
+    const int ab = kcol / Cout, co = kcol - ab * Cout;
+    const int py = ph >> 1, px = ph & 1, aa = ab >> 1, bb = ab & 1;
+    const int kh = py + pad - 2 * aa, kw = px + pad - 2 * bb;
+    uint4 v = make_uint4(0u, 0u, 0u, 0u);
+    if (kh >= 0 && kh < K && kw >= 0 && kw < K)
+      v = __ldg((const uint4*)(w + (long long)co * ldb + (kh * K + kw) * Cin + cv * 8));
+    const bf16* h = (const bf16*)&v;
+    const long long K4 = 4LL * Cout;
+#pragma unroll
+    for (int q = 0; q < 8; ++q) bsp[((long long)ph * Cin + cv * 8 + q) * K4 + kcol] = h[q];
+  }
+}
+
+void conv_dgrad_sp(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, bf16* wsp, int n, const float* bcast,
+                   const bf16* sc, bool sc_compact, const bf16* yact, int mask_act, bf16* dx, cudaStream_t st) {
+  if (!dgrad_sp_ok(g)) throw ShapeError("conv_dgrad_sp: unsupported geometry");
+  check_extent((long long)n * (g.H + 1) * (g.W + 1));
+  if (n <= 0) return;
+  {
+    ProfScope ps(PC_CONV_DGRAD_PREP, st);
+    const long long total = 16LL * g.Cout * (g.Cin / 8);
+    const int blocks = (int)std::min<long long>((total + 255) / 256, 8LL * num_sms());
+    sp_weight_kernel<<<blocks, 256, 0, st>>>(w, ldb, g.Cin, g.Cout, 3, g.pad, wsp);
+    CK(cudaGetLastError());
+  }
+  static ConvArgs a;
+  a = ConvArgs{};
+  a.src = dz;
+  a.Hs = g.Ho;
+  a.Ws = g.Wo;
+  a.Cs = g.Cout;
+  a.n_static = n;
+  a.Hg = g.Ho;
+  a.Wg = g.Wo;
+  a.sy = a.sx = 1;
+  a.ntaps = 4;
+  for (int t = 0; t < 4; ++t) {
+    a.ty[t] = (int8_t)(t >> 1);
+    a.tx[t] = (int8_t)(t & 1);
+  }
+  a.B = wsp;
+  a.ldb = 4 * g.Cout;
+  a.K = 4 * g.Cout;
+  a.Nout = 4 * g.Cin;
+  a.out = dx;
+  a.Ho = g.H;
+  a.Wo = g.W;
+  a.oys = a.oxs = 1;
+  a.bcast = bcast;
+  a.sc = sc;
+  a.yact = yact;
+  a.mask_act = mask_act;
+  a.sp_cin = g.Cin;
+  a.sp_sc_compact = sc_compact ? 1 : 0;
+  a.b_tma = 1;
+  a.b_map = make_tmap_2d(wsp, a.Nout, a.K, a.ldb, 64, 256);
+  const long long mt = ((long long)n * g.Ho * g.Wo + BM - 1) / BM;
+  launch_t<MODE_DGRAD_SP, 256>(a, mt * ((a.Nout + 255) / 256), st);
 }
 
 // partial [S][Kconv][Cout] -> dw [Cout][taps][cin_real] (fp32), summed over S in fixed order

@@ -338,10 +338,16 @@ __global__ void __launch_bounds__(EH_THREADS) exit_head_kernel(const ExitHeadArg
     pooled[c] = s * inv_hw;
   }
   __syncthreads();
-  for (int k = t; k < a.ncls; k += EH_THREADS) {
-    float l = a.bk[k];
-    for (int c = 0; c < C; ++c) l = fmaf(pooled[c], a.Wk[c * a.ncls + k], l);
-    logits[k] = l;
+  // FC: one warp per class, lanes stride the channels, fixed xor-tree reduction (deterministic)
+  {
+    const int wp = t >> 5, ln = t & 31;
+    for (int k = wp; k < a.ncls; k += EH_THREADS / 32) {
+      float l = 0.f;
+      for (int c = ln; c < C; c += 32) l = fmaf(pooled[c], __ldg(a.Wk + c * a.ncls + k), l);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) l += __shfl_xor_sync(0xffffffffu, l, o);
+      if (ln == 0) logits[k] = __fadd_rn(l, a.bk[k]);
+    }
   }
   __syncthreads();
   const int orig = a.orig ? a.orig[j] : j;
@@ -652,17 +658,28 @@ __global__ void __launch_bounds__(SGD_THREADS) sgd_kernel(float* __restrict__ w,
   const long long end = min(sg.off + sg.count, start + (long long)SGD_PER_BLOCK);
   float sq = 0.f;
   const bool vec_ok = ((sg.off & 3) == 0);
+  // issue every 128-bit load of the thread's items first (12 loads in flight), then update and store
+  float4 wl[SGD_ITEMS], vl[SGD_ITEMS], gl[SGD_ITEMS];
+#pragma unroll
+  for (int it = 0; it < SGD_ITEMS; ++it) {
+    const long long i = start + ((long long)it * SGD_THREADS + threadIdx.x) * SGD_VEC;
+    if (vec_ok && i + SGD_VEC <= end) {
+      wl[it] = *(const float4*)(w + i);
+      vl[it] = *(const float4*)(v + i);
+      gl[it] = __ldg((const float4*)(g + i));
+    }
+  }
 #pragma unroll
   for (int it = 0; it < SGD_ITEMS; ++it) {
     const long long i = start + ((long long)it * SGD_THREADS + threadIdx.x) * SGD_VEC;
     if (i >= end) continue;
     const int cnt = (int)min((long long)SGD_VEC, end - i);
+    const bool full = vec_ok && cnt == 4;
     float wr[4], vr[4], gr[4];
-    if (vec_ok && cnt == 4) {
-      const float4 a = *(const float4*)(w + i), b = *(const float4*)(v + i), c = __ldg((const float4*)(g + i));
-      wr[0] = a.x, wr[1] = a.y, wr[2] = a.z, wr[3] = a.w;
-      vr[0] = b.x, vr[1] = b.y, vr[2] = b.z, vr[3] = b.w;
-      gr[0] = c.x, gr[1] = c.y, gr[2] = c.z, gr[3] = c.w;
+    if (full) {
+      wr[0] = wl[it].x, wr[1] = wl[it].y, wr[2] = wl[it].z, wr[3] = wl[it].w;
+      vr[0] = vl[it].x, vr[1] = vl[it].y, vr[2] = vl[it].z, vr[3] = vl[it].w;
+      gr[0] = gl[it].x, gr[1] = gl[it].y, gr[2] = gl[it].z, gr[3] = gl[it].w;
     } else {
       for (int q = 0; q < cnt; ++q) wr[q] = w[i + q], vr[q] = v[i + q], gr[q] = g[i + q];
     }
@@ -675,7 +692,7 @@ __global__ void __launch_bounds__(SGD_THREADS) sgd_kernel(float* __restrict__ w,
         wr[q] = __fsub_rn(wr[q], __fmul_rn(lr, vr[q]));
       }
     }
-    if (vec_ok && cnt == 4) {
+    if (full) {
       *(float4*)(w + i) = make_float4(wr[0], wr[1], wr[2], wr[3]);
       *(float4*)(v + i) = make_float4(vr[0], vr[1], vr[2], vr[3]);
     } else {

@@ -357,13 +357,23 @@ void Model::ensure_training() {
     T[t].grad = T[t].own_grad.as<bf16>();
   }
   size_t ws = 0;
+  for (auto& nd : nodes)
+    if (nd.kind == N_CONV && nd.in != 0 && dgrad_sp_ok(nd.g)) {
+      nd.sp = true;
+      nd.wsp.alloc(dgrad_sp_ws_bytes(nd.g));
+    }
   for (auto& nd : nodes) {
     if (nd.kind == N_POOL) {
       nd.argmax.alloc((size_t)max_batch * T[nd.out].row_elems());
     } else {
       ws = std::max(ws, ::adainf::wgrad_ws_bytes(nd.g, max_batch));
       if (stem_s2d && &nd == &nodes[0]) ws = std::max(ws, stem_wgrad_ws_bytes(max_batch));
-      if (nd.kind == N_PROJ && nd.in != 0) nd.proj_dx.alloc((size_t)max_batch * T[nd.in].row_elems() * 2);
+      if (nd.kind == N_PROJ && nd.in != 0) {
+        for (const auto& c : nodes)
+          if (c.kind == N_CONV && c.in == nd.in && c.sp && c.g.Ho == nd.g.Ho && c.g.Wo == nd.g.Wo) nd.proj_compact = true;
+        const size_t rows = nd.proj_compact ? (size_t)nd.g.Ho * nd.g.Wo * nd.g.Cin : T[nd.in].row_elems();
+        nd.proj_dx.alloc((size_t)max_batch * rows * 2);
+      }
     }
   }
   for (auto& e : exits) ws = std::max(ws, head_grads_ws_bytes(max_batch, T[e.tensor].C, e.ncls));
@@ -544,12 +554,24 @@ void Model::train_step(const bf16* x, const int32_t* labels, int n, long long n_
     if (nd.in == 0) return;  // no input gradient for the first layer
     const TensorRt& X = T[nd.in];
     if (nd.kind == N_PROJ) {
-      conv_dgrad(nd.g, dz, nd.shadow.as<bf16>(), nd.ldb, n, nullptr, nullptr, nullptr, 0, nd.proj_dx.as<bf16>(), st);
+      ConvGeom g = nd.g;
+      if (nd.proj_compact) {  // only the even input positions receive gradient: a plain 1x1 GEMM on the dZ grid
+        g.stride = 1;
+        g.H = g.Ho;
+        g.W = g.Wo;
+      }
+      conv_dgrad(g, dz, nd.shadow.as<bf16>(), nd.ldb, n, nullptr, nullptr, nullptr, 0, nd.proj_dx.as<bf16>(), st);
     } else {
       const int prod = X.producer;
       const int mask = (prod >= 0 && nodes[prod].kind == N_CONV) ? X.act : 0;
-      conv_dgrad(nd.g, dz, nd.shadow.as<bf16>(), nd.ldb, n, bcast_of(nd.in), sc_of(nd.in), mask ? X.buf : nullptr,
-                 mask, T[nd.in].grad, st);
+      if (nd.sp) {
+        const bool sc_compact = X.res_of < 0 && X.proj >= 0 && nodes[X.proj].proj_compact;
+        conv_dgrad_sp(nd.g, dz, nd.shadow.as<bf16>(), nd.ldb, nd.wsp.as<bf16>(), n, bcast_of(nd.in), sc_of(nd.in),
+                      sc_compact, mask ? X.buf : nullptr, mask, T[nd.in].grad, st);
+      } else {
+        conv_dgrad(nd.g, dz, nd.shadow.as<bf16>(), nd.ldb, n, bcast_of(nd.in), sc_of(nd.in), mask ? X.buf : nullptr,
+                   mask, T[nd.in].grad, st);
+      }
     }
   };
   for (int ni = (int)nodes.size() - 1; ni >= 0; --ni) {

@@ -64,6 +64,10 @@ struct NodeRt {
   int pk = 0, ps = 0, pp = 0;  // pool
   DevBuf argmax;               // pool (training)
   DevBuf proj_dx;              // proj (training): dgrad into the block input, added as shortcut term
+  bool proj_compact = false;   // proj: proj_dx stored on the output grid (only the (0,0) phase is nonzero),
+                               // consumed by the sibling's sub-pixel dgrad epilogue
+  bool sp = false;             // stride-2 3x3 conv whose dgrad runs as one sub-pixel GEMM (MODE_DGRAD_SP)
+  DevBuf wsp;                  // its packed sub-pixel weights bf16 [4*Cin][4*Cout]
 };
 
 struct ExitRt {

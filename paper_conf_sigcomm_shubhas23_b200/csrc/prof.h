@@ -31,6 +31,7 @@ enum ProfClass {
   PC_STEM_FWD,
   PC_STEM_WGRAD,
   PC_STEM_AUX,
+  PC_CONV_DGRAD_PREP,
   PROF_NCLASS
 };
 

@@ -100,6 +100,32 @@ def test_conv_dgrad_vs_torch(case):
     assert _rel(dx.float(), ref) < 8e-3
 
 
+# stride-2 3x3 layers take the sub-pixel dgrad (one GEMM over the dZ grid, N = 4 * Cin): ResNet shapes at small
+# batch, odd spatial sizes (the last output row / column phase is dropped), a ragged last M tile
+SP_CASES = [(3, 56, 56, 64, 128, 3, 2, 1), (2, 28, 28, 128, 256, 3, 2, 1), (2, 14, 14, 256, 512, 3, 2, 1),
+            (3, 7, 9, 128, 64, 3, 2, 1), (1, 13, 11, 64, 192, 3, 2, 1)]
+
+
+@pytest.mark.parametrize("case", SP_CASES)
+def test_conv_dgrad_subpixel_vs_torch(case):
+    n, H, W, C, Co, K, s, p = case
+    x, w, b = _mk(case, 7)
+    Ho, Wo = (H + 2 * p - K) // s + 1, (W + 2 * p - K) // s + 1
+    g = torch.Generator(device="cpu").manual_seed(8)
+    dz = torch.randn(n, Ho, Wo, Co, generator=g).to(torch.bfloat16).cuda()
+    bc = torch.randn(n, C, generator=g).cuda() * 0.01
+    sc = torch.randn(n, H, W, C, generator=g).to(torch.bfloat16).cuda()
+    y = torch.randn(n, H, W, C, generator=g).to(torch.bfloat16).cuda()
+    ref = torch.nn.grad.conv2d_input((n, C, H, W), w.float().permute(0, 3, 1, 2), dz.float().permute(0, 3, 1, 2),
+                                     stride=s, padding=p).permute(0, 2, 3, 1)
+    dx = B.dbg_conv_dgrad(dz, w, H, W, s, p)
+    torch.cuda.synchronize()
+    assert _rel(dx.float(), ref) < 8e-3
+    ref2 = (ref + bc[:, None, None, :] + sc.float()) * (y.float() > 0)
+    dx2 = B.dbg_conv_dgrad(dz, w, H, W, s, p, bcast=bc, sc=sc, yact=y, mask_act=1)
+    assert _rel(dx2.float(), ref2) < 8e-3
+
+
 def test_conv_dgrad_epilogue_terms():
     case = (2, 14, 14, 64, 128, 3, 2, 1)
     n, H, W, C, Co, K, s, p = case
