@@ -303,17 +303,27 @@ def main():
 
     # ---- timed region (device time, CUDA events on the launching stream) ----
     clk = ClockSampler(local)
-    clk.start()
-    time.sleep(0.3)
+    if os.environ.get("ADAINF_BENCH_NO_CLOCKS") != "1":
+        # nvidia-smi's NVML start-up stalls the GPU for tens of ms: wait until it is sampling steadily
+        # (two samples) so the start-up falls before the timed region, not inside its first step
+        clk.start()
+        t_wait = time.time()
+        while len(clk.rows) < 2 and time.time() - t_wait < 10.0:
+            time.sleep(0.05)
+        time.sleep(0.2)
     l0 = B.launch_count()
     barrier()
     torch.cuda.synchronize()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
     ev0.record(stream)
+    evs[0].record(stream)
     for i in range(args.steps):
         step_device(cnt_buf[i])
+        evs[i + 1].record(stream)
     ev1.record(stream)
     torch.cuda.synchronize()
+    step_ms = [round(evs[i].elapsed_time(evs[i + 1]), 3) for i in range(args.steps)]
     launches = B.launch_count() - l0
     barrier()
     clocks = clk.stop()
@@ -418,6 +428,7 @@ def main():
                          "share_of_step": conv_ms / prof_ms},
             "kernel_ms_per_step": breakdown,
             "gpu_launches": int(launches),
+            "step_ms": step_ms,
             "clocks": clocks,
             "e2e": e2e,
             "cpu_baseline": cpu,

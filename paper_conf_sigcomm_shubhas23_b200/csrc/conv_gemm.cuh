@@ -85,8 +85,11 @@ struct ConvCfg {
   static constexpr int A_BYTES = BM * BK * 2;
   static constexpr int B_BYTES = BN * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int STAGES = (200 * 1024) / STAGE_BYTES > 8 ? 8 : (200 * 1024) / STAGE_BYTES;
-  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+  // coalescing buffers of the bf16 epilogue: 4 warps x 2 x (32 rows x 128 B)
+  static constexpr int EPI_BYTES = (MODE != 2 && BN >= 64) ? 4 * 8192 : 0;
+  static constexpr int STAGES_FIT = (220 * 1024 - EPI_BYTES - 1280) / STAGE_BYTES;
+  static constexpr int STAGES = STAGES_FIT > 8 ? 8 : STAGES_FIT;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/ + EPI_BYTES;
   static constexpr int ACC_COLS = BN < 32 ? 32 : BN;
   static constexpr int TMEM_COLS = 2 * ACC_COLS;  // double-buffered accumulator
 };
@@ -152,6 +155,177 @@ __device__ __forceinline__ void ld_bf16x8(const bf16* p, float* v) {
   for (int q = 0; q < 8; ++q) v[q] = __bfloat162float(h[q]);
 }
 
+// ---- coalesced bf16 epilogue (FWD / DGRAD / DGRAD_SP with Nout % 64 == 0) ----
+// Per 64-column block: the warp's 32 accumulator rows (thread = row) are combined with their epilogue
+// operands and written through a per-warp 32 x 128 B shared buffer (16-byte chunks XOR-swizzled by row), so
+// every global access is a lane group of 8 covering one row's 128 contiguous bytes (4 rows per instruction)
+// instead of 32 rows x 16 B per instruction.  Same arithmetic and order as the per-thread path.
+__device__ __forceinline__ uint32_t stg_off(int r, int j) { return (uint32_t)(r * 128 + ((j ^ (r & 7)) << 4)); }
+
+// cooperative cp.async of 32 rows x 64 bf16 (row r of the warp at base + prow(r) * pitch; rows with ok = 0
+// zero-filled) into a staging buffer: no register staging, one commit group per call
+__device__ __forceinline__ void stage_issue(uint8_t* stg, const bf16* base, long long prow, bool ok, int pitch,
+                                            int lane) {
+  const int j = lane & 7;
+#pragma unroll
+  for (int it = 0; it < 8; ++it) {
+    const int r = it * 4 + (lane >> 3);
+    const long long pr = __shfl_sync(0xffffffffu, prow, r);
+    const int okr = __shfl_sync(0xffffffffu, (int)ok, r);
+    cp_async16(smem_u32(stg + stg_off(r, j)), okr ? (const void*)(base + pr * pitch + j * 8) : (const void*)base, okr);
+  }
+}
+__device__ __forceinline__ void stage_wait() {
+  asm volatile("cp.async.commit_group;" ::: "memory");
+  asm volatile("cp.async.wait_group 0;" ::: "memory");
+  __syncwarp();
+}
+// each lane applies op to its own row of a staged buffer
+template <class Op>
+__device__ __forceinline__ void stage_apply(const uint8_t* stg, int lane, float* v, Op op) {
+#pragma unroll
+  for (int jj = 0; jj < 8; ++jj) {
+    const uint4 x = *(const uint4*)(stg + stg_off(lane, jj));
+    const bf16* h = (const bf16*)&x;
+#pragma unroll
+    for (int qq = 0; qq < 8; ++qq) v[jj * 8 + qq] = op(v[jj * 8 + qq], __bfloat162float(h[qq]));
+  }
+}
+template <class Op>
+__device__ __forceinline__ void stage_rows_in(uint8_t* stg, const bf16* base, long long prow, bool ok, int pitch,
+                                              int lane, float* v, Op op) {
+  stage_issue(stg, base, prow, ok, pitch, lane);
+  stage_wait();
+  stage_apply(stg, lane, v, op);
+  __syncwarp();
+}
+__device__ __forceinline__ void prefetch_l2(const void* p) {
+  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+}
+// two operands with one memory latency: first into stg, second into stg + 4096
+template <class Op0, class Op1>
+__device__ __forceinline__ void stage_rows_in2(uint8_t* stg, const bf16* base0, long long prow0, const bf16* base1,
+                                               long long prow1, bool ok, int pitch, int lane, float* v, Op0 op0,
+                                               Op1 op1) {
+  stage_issue(stg, base0, prow0, ok, pitch, lane);
+  stage_issue(stg + 4096, base1, prow1, ok, pitch, lane);
+  stage_wait();
+  stage_apply(stg, lane, v, op0);
+  stage_apply(stg + 4096, lane, v, op1);
+  __syncwarp();
+}
+
+template <int MODE, int BN>
+__device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const TileInfo& ti, uint32_t trow,
+                                                   uint64_t* tempty_b, int nkb, long long m, bool rv, int n,
+                                                   long long orow, long long rrow, int HWg, uint8_t* stg, int lane) {
+  int gy = 0, gx = 0;
+  if (MODE == MODE_DGRAD_SP && rv) {
+    const int pix = (int)m - n * HWg;
+    gy = pix / a.Wg;
+    gx = pix - gy * a.Wg;
+  }
+  // L2 prefetch of this row's epilogue operands for the column blocks after the first (the first block's
+  // loads are issued right away; later blocks then hit L2 instead of DRAM)
+  if (MODE != MODE_DGRAD_SP && rv) {
+    const bf16* p0 = MODE == MODE_FWD ? a.res : a.sc;
+    const bf16* p1 = MODE == MODE_FWD ? nullptr : (a.mask_act ? a.yact : nullptr);
+    const long long r0 = MODE == MODE_FWD ? rrow : orow;
+#pragma unroll 1
+    for (int c = 64; c < BN; c += 64) {
+      if (ti.n0 + c >= a.Nout) break;
+      if (p0) prefetch_l2(p0 + r0 * a.Nout + ti.n0 + c);
+      if (p1) prefetch_l2(p1 + orow * a.Nout + ti.n0 + c);
+    }
+  }
+#pragma unroll 1
+  for (int c0 = 0; c0 < BN; c0 += 64) {
+    float v[64];
+    if (nkb > 0) {
+      tmem_ld32(trow + c0, v);
+      tmem_ld32(trow + c0 + 32, v + 32);
+    } else {
+#pragma unroll
+      for (int i = 0; i < 64; ++i) v[i] = 0.f;
+    }
+    if (c0 + 64 >= BN) {
+      tc_fence_before();
+      mbar_arrive(tempty_b);  // accumulator free for the tile after next
+    }
+    const int cb = ti.n0 + c0;
+    if (cb >= a.Nout) continue;  // warp-uniform
+    int ocol = cb, NO = a.Nout;
+    bool ok = rv;
+    long long orow_b = orow, srow = orow;
+    const bf16* scp = a.sc;
+    if (MODE == MODE_DGRAD_SP) {
+      const int ph = cb / a.sp_cin;
+      ocol = cb - ph * a.sp_cin;
+      NO = a.sp_cin;
+      const int oy = 2 * gy + (ph >> 1), ox = 2 * gx + (ph & 1);
+      ok = rv && oy < a.Ho && ox < a.Wo;
+      orow_b = ((long long)n * a.Ho + oy) * a.Wo + ox;
+      srow = orow_b;
+      if (a.sp_sc_compact) {
+        srow = m;
+        if (ph != 0) scp = nullptr;
+      }
+    }
+    if (MODE == MODE_FWD) {
+      if (!(a.exp_flags & 2)) {
+#pragma unroll
+        for (int i = 0; i < 64; ++i) v[i] = __fadd_rn(v[i], __ldg(a.bias + cb + i));  // flat params: 4B-aligned
+      }
+      if (a.res)
+        stage_rows_in(stg, a.res + ocol, rrow, ok, NO, lane, v, [](float x, float r) { return __fadd_rn(x, r); });
+#pragma unroll
+      for (int i = 0; i < 64; ++i) v[i] = act_apply(a.act, v[i]);
+    } else {
+      if (a.bcast && ok) {
+#pragma unroll
+        for (int i = 0; i < 64; i += 4) {
+          const float4 bb = __ldg((const float4*)(a.bcast + (long long)n * NO + ocol + i));
+          v[i] = __fadd_rn(v[i], bb.x);
+          v[i + 1] = __fadd_rn(v[i + 1], bb.y);
+          v[i + 2] = __fadd_rn(v[i + 2], bb.z);
+          v[i + 3] = __fadd_rn(v[i + 3], bb.w);
+        }
+      }
+      const int ma = a.mask_act;
+      if (scp && ma) {
+        stage_rows_in2(stg, scp + ocol, srow, a.yact + ocol, orow_b, ok, NO, lane, v,
+                       [](float x, float r) { return __fadd_rn(x, r); },
+                       [ma](float x, float y) { return __fmul_rn(x, act_grad(ma, y)); });
+      } else if (scp) {
+        stage_rows_in(stg, scp + ocol, srow, ok, NO, lane, v, [](float x, float r) { return __fadd_rn(x, r); });
+      } else if (ma) {
+        stage_rows_in(stg, a.yact + ocol, orow_b, ok, NO, lane, v,
+                      [ma](float x, float y) { return __fmul_rn(x, act_grad(ma, y)); });
+      }
+    }
+    // own row -> staging (bf16), then 8 coalesced 16-byte stores per lane
+#pragma unroll
+    for (int jj = 0; jj < 8; ++jj) {
+      __align__(16) bf16 h[8];
+#pragma unroll
+      for (int qq = 0; qq < 8; ++qq) h[qq] = __float2bfloat16_rn(v[jj * 8 + qq]);
+      *(uint4*)(stg + stg_off(lane, jj)) = *(const uint4*)h;
+    }
+    __syncwarp();
+    const int j = lane & 7;
+    bf16* ob = (bf16*)a.out + ocol;
+#pragma unroll
+    for (int it = 0; it < 8; ++it) {
+      const int r = it * 4 + (lane >> 3);
+      const long long pr = __shfl_sync(0xffffffffu, orow_b, r);
+      const int okr = __shfl_sync(0xffffffffu, (int)ok, r);
+      const uint4 x = *(const uint4*)(stg + stg_off(r, j));
+      if (okr) *((uint4*)(ob + pr * NO) + j) = x;
+    }
+    __syncwarp();
+  }
+}
+
 template <int MODE, int BN>
 __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_constant__ ConvArgs a) {
   using Cfg = ConvCfg<MODE, BN>;
@@ -164,6 +338,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
   uint64_t* tfull = empty + STAGES;   // [2]
   uint64_t* tempty = tfull + 2;       // [2]
   uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+  uint8_t* epi_smem = smem + STAGES * Cfg::STAGE_BYTES + 256;  // Cfg::EPI_BYTES (non-WGRAD, BN >= 64)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nsamp = a.count ? *a.count : a.n_static;
@@ -469,6 +644,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
           if (MODE == MODE_FWD && a.res) {
             const int rn = a.res_map ? __ldg(a.res_map + n) : n;
             rrow = (long long)rn * a.Ho * a.Wo + (orow - (long long)n * a.Ho * a.Wo);
+          }
+        }
+        if constexpr (Cfg::EPI_BYTES > 0) {
+          if (!a.out_f32 && (a.Nout & 63) == 0 && !(a.exp_flags & 1)) {
+            epilogue_coalesced<MODE, BN>(a, ti, trow, &tempty[b], nkb, m, rv, n, orow, rrow, HWg,
+                                          epi_smem + q * 8192, lane);
+            continue;
           }
         }
 #pragma unroll 1
