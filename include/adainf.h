@@ -179,7 +179,7 @@ typedef struct {
   const void* W_bf16;     /* device [D * P] bf16 PCA basis (row-major), or NULL -> identity (P == D) */
   int32_t P;              /* 16..256, multiple of 16                                    */
   const float* ref;       /* device [M * D] fp32 reference rows (M = 1: mean of old samples) */
-  int32_t M;              /* 1..64 */
+  int32_t M;              /* 1..4096 (M > 4: lanes stride the reference rows) */
   const uint8_t* exclude; /* device [N] nonzero = already used / in use, or NULL */
 } adainf_select_in;
 

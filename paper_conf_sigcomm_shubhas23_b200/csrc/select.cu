@@ -82,6 +82,51 @@ __global__ void cosine_key_kernel(const void* __restrict__ Yv, long long N, int 
   }
 }
 
+// many reference rows (M > 4, the GEMM-shaped variant of reading Q14): one warp per candidate row, the row's
+// projected vector staged in shared memory, lanes stride the reference rows (each lane a full P-length dot in
+// fixed order), min-reduced over lanes
+template <bool FROM_BF16>
+__global__ void __launch_bounds__(256) cosine_key_multi_kernel(const void* __restrict__ Yv, long long N, int P,
+                                                               const float* __restrict__ mu,
+                                                               const float* __restrict__ mun, int M,
+                                                               const uint8_t* __restrict__ exclude,
+                                                               uint32_t* __restrict__ keys, float* __restrict__ dist_all) {
+  __shared__ float ys[8][256];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const long long row = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+  if (row >= N) return;
+  float nn = 0.f;
+  for (int p = lane; p < P; p += 32) {
+    const float v = FROM_BF16 ? __bfloat162float(((const bf16*)Yv)[row * P + p]) : ((const float*)Yv)[row * P + p];
+    ys[w][p] = v;
+    nn = fmaf(v, v, nn);
+  }
+  for (int o = 16; o > 0; o >>= 1) nn += __shfl_xor_sync(0xffffffffu, nn, o);
+  __syncwarp();
+  const float yn = sqrtf(nn);
+  float best = FLT_MAX;
+  for (int r = lane; r < M; r += 32) {
+    const float* m = mu + (long long)r * P;
+    float dot = 0.f;
+    for (int p = 0; p < P; p += 4) {
+      const float4 q = __ldg((const float4*)(m + p));
+      dot = fmaf(ys[w][p], q.x, dot);
+      dot = fmaf(ys[w][p + 1], q.y, dot);
+      dot = fmaf(ys[w][p + 2], q.z, dot);
+      dot = fmaf(ys[w][p + 3], q.w, dot);
+    }
+    const float cs = dot / fmaxf(yn * mun[r], 1e-12f);
+    best = fminf(best, 1.0f - cs);
+  }
+  for (int o = 16; o > 0; o >>= 1) best = fminf(best, __shfl_xor_sync(0xffffffffu, best, o));
+  if (lane == 0) {
+    const bool ex = exclude && exclude[row];
+    const float d = fmaxf(best, 0.f);
+    keys[row] = ex ? 0u : (__float_as_uint(d) + 1u);
+    if (dist_all) dist_all[row] = ex ? -1.f : d;
+  }
+}
+
 // ---- radix select state: [0] prefix, [1] k remaining, [2] pass, hist[256] ----
 struct RadixState {
   uint32_t prefix;
@@ -245,8 +290,8 @@ void select_retrain(const adainf_select_in& in, int k, int32_t* out_idx, float* 
   const long long N = in.N;
   const int D = in.D, P = in.W_bf16 ? in.P : in.D, M = in.M;
   if (N <= 0 || N > (1LL << 31) - 1 || D <= 0 || D % 8 || D > 1024 || P <= 0 || P > 256 || P % 16 || M <= 0 ||
-      M > 64 || k <= 0)
-    throw ShapeError("select: N in 1..2^31, D multiple of 8 <= 1024, P multiple of 16 <= 256, M in 1..64, k > 0");
+      M > 4096 || k <= 0)
+    throw ShapeError("select: N in 1..2^31, D multiple of 8 <= 1024, P multiple of 16 <= 256, M in 1..4096, k > 0");
   if (!in.X_bf16 || !in.ref) throw InvalidError("select: X and ref are required");
   SelectWs sw;
   void* wsp = nullptr;
@@ -284,12 +329,20 @@ void select_retrain(const adainf_select_in& in, int k, int32_t* out_idx, float* 
     // Y [N][P] fp32 = X [N][D] . W [D][P] on the tensor cores
     conv_fwd(g, (const bf16*)in.X_bf16, nullptr, nullptr, (int)N, Wt, D, zb, nullptr, nullptr, 0, Y, true, st);
     ProfScope ps(PC_SELECT_COSINE, st);
-    cosine_key_kernel<false><<<(unsigned)((N * 32 + 255) / 256), 256, 0, st>>>(Y, N, P, mu, mun, M, in.exclude, keys,
-                                                                              dist_all);
+    if (M > 4)
+      cosine_key_multi_kernel<false><<<(unsigned)((N * 32 + 255) / 256), 256, 0, st>>>(Y, N, P, mu, mun, M,
+                                                                                      in.exclude, keys, dist_all);
+    else
+      cosine_key_kernel<false><<<(unsigned)((N * 32 + 255) / 256), 256, 0, st>>>(Y, N, P, mu, mun, M, in.exclude,
+                                                                                keys, dist_all);
   } else {
     ProfScope ps(PC_SELECT_COSINE, st);
-    cosine_key_kernel<true><<<(unsigned)((N * 32 + 255) / 256), 256, 0, st>>>(in.X_bf16, N, P, mu, mun, M,
-                                                                             in.exclude, keys, dist_all);
+    if (M > 4)
+      cosine_key_multi_kernel<true><<<(unsigned)((N * 32 + 255) / 256), 256, 0, st>>>(in.X_bf16, N, P, mu, mun, M,
+                                                                                     in.exclude, keys, dist_all);
+    else
+      cosine_key_kernel<true><<<(unsigned)((N * 32 + 255) / 256), 256, 0, st>>>(in.X_bf16, N, P, mu, mun, M,
+                                                                               in.exclude, keys, dist_all);
   }
   const int k_eff = (int)std::min<long long>(k, N);  // the k-th largest must exist
   ProfScope ps_topk(PC_SELECT_TOPK, st, 12);

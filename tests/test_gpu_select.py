@@ -47,7 +47,7 @@ def _run(N, D, P, M, k, seed, excl_frac=0.1, use_w=True):
 
 
 @pytest.mark.parametrize("N,D,P,M,k", [(4099, 64, 16, 1, 512), (16384, 64, 16, 1, 1024), (3000, 512, 64, 4, 257),
-                                       (1000, 64, 16, 1, 5000)])
+                                       (1000, 64, 16, 1, 5000), (5001, 64, 16, 33, 700), (2048, 512, 64, 256, 300)])
 def test_select_vs_oracle(N, D, P, M, k):
     _run(N, D, P, M, k, seed=N + k)
 
