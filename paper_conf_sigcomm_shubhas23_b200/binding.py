@@ -56,6 +56,15 @@ class ModelOut(C.Structure):
                 ("route_idx", C.c_void_p), ("n_routed", C.c_void_p)]
 
 
+class RetrainProfile(C.Structure):
+    _fields_ = [("n", C.c_int32), ("batch", C.POINTER(C.c_int32)), ("step_ms", C.POINTER(C.c_double))]
+
+
+class RetrainPlan(C.Structure):
+    _fields_ = [("samples", C.c_int32), ("batch", C.c_int32), ("steps", C.c_int32), ("epochs", C.c_int32),
+                ("est_ms", C.c_double)]
+
+
 class SelectIn(C.Structure):
     _fields_ = [("X_bf16", C.c_void_p), ("N", C.c_int64), ("D", C.c_int32), ("W_bf16", C.c_void_p),
                 ("P", C.c_int32), ("ref", C.c_void_p), ("M", C.c_int32), ("exclude", C.c_void_p)]
@@ -92,6 +101,14 @@ def lib():
             "adainf_dp_attach": [vp, vp, i32, i32],
             "adainf_nccl_unique_id": [vp],
             "adainf_gather_rows": [vp, vp, vp, i32, i64, vp, vp],
+            "adainf_time_split": [C.c_double, C.POINTER(C.c_double), i32, C.POINTER(C.c_double), i32,
+                                  C.POINTER(C.c_double), C.POINTER(C.c_double)],
+            "adainf_retrain_setting": [C.c_double, C.POINTER(RetrainProfile), i64, i32, C.POINTER(RetrainPlan)],
+            "adainf_model_average": [vp, C.POINTER(vp), i32, vp],
+            "adainf_dp_average": [vp, vp],
+            "adainf_mark_used": [vp, vp, vp, i32, vp],
+            "adainf_count_correct": [vp, vp, i32, vp, vp],
+            "adainf_drift_should_stop": [C.POINTER(C.c_uint64), i32, i32, C.POINTER(i32)],
             "adainf_dbg_set_win_mode": [i32],
             "adainf_prof_enable": [i32],
             "adainf_prof_reset": [],
@@ -393,3 +410,54 @@ def dbg_conv_wgrad(x, dz, KH, KW, stride, pad, stream=None):
     check(lib().adainf_dbg_conv_wgrad(ptr(x), ptr(dz), n, H, W_, Cc, Co, KH, KW, stride, pad, ptr(dw), ptr(db),
                                       stream_ptr(stream)))
     return dw, db
+
+
+# ---- incremental-retraining support (include/adainf_sched.h) ----
+def time_split(slo_ms, infer_ms, impact):
+    """T_r = max(0, L_s - sum l_k) and its split by impact degree.  Host arithmetic."""
+    li = (C.c_double * max(1, len(infer_ms)))(*infer_ms)
+    di = (C.c_double * max(1, len(impact)))(*impact)
+    out = (C.c_double * max(1, len(impact)))()
+    tr = C.c_double()
+    check(lib().adainf_time_split(float(slo_ms), li, len(infer_ms), di, len(impact), C.byref(tr), out))
+    return tr.value, [out[j] for j in range(len(impact))]
+
+
+def retrain_setting(alloc_ms, batches, step_ms, eligible, max_batch):
+    """Retraining setting a time allocation affords under a measured step profile."""
+    bi = (C.c_int32 * len(batches))(*batches)
+    ti = (C.c_double * len(step_ms))(*step_ms)
+    prof = RetrainProfile(len(batches), bi, ti)
+    out = RetrainPlan()
+    check(lib().adainf_retrain_setting(float(alloc_ms), C.byref(prof), int(eligible), int(max_batch), C.byref(out)))
+    return {"samples": out.samples, "batch": out.batch, "steps": out.steps, "epochs": out.epochs, "est_ms": out.est_ms}
+
+
+def model_average(dst, versions, stream=None):
+    """dst <- mean of the versions' fp32 parameters, momentum reset (reading Q23)."""
+    arr = (C.c_void_p * len(versions))(*[v.h for v in versions])
+    check(lib().adainf_model_average(dst.h, arr, len(versions), stream_ptr(stream)))
+
+
+def dp_average(model, stream=None):
+    check(lib().adainf_dp_average(model.h, stream_ptr(stream)))
+
+
+def mark_used(exclude, idx, count=None, stream=None):
+    """exclude[idx[:count]] = 1 (samples used by one job are not reused by another)."""
+    check(lib().adainf_mark_used(ptr(exclude), ptr(idx), ptr(count), int(idx.numel()), stream_ptr(stream)))
+
+
+def count_correct(pred, labels, stream=None):
+    import torch
+    out = torch.empty(1, dtype=torch.int32, device=pred.device)
+    check(lib().adainf_count_correct(ptr(pred), ptr(labels), int(pred.numel()), ptr(out), stream_ptr(stream)))
+    return out
+
+
+def drift_should_stop(results, n=4):
+    """Stop rule of the drift-impact detection (Table 2): the last n impacted-set results agree."""
+    arr = (C.c_uint64 * max(1, len(results)))(*results)
+    out = C.c_int32()
+    check(lib().adainf_drift_should_stop(arr, len(results), int(n), C.byref(out)))
+    return bool(out.value)

@@ -13,12 +13,7 @@ void select_retrain(const adainf_select_in& in, int k, int32_t* out_idx, float* 
 
 using namespace adainf;
 
-struct adainf_model {
-  Model m;
-};
-struct adainf_app {
-  App a;
-};
+#include "api_handles.h"
 
 extern "C" adainf_status adainf_model_create(const adainf_model_spec* spec, adainf_model_t* out) {
   return guard([&] {

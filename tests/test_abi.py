@@ -12,7 +12,7 @@ LIB = os.path.join(ROOT, "paper_conf_sigcomm_shubhas23_b200", "libadainf.so")
 
 def declared_symbols():
     names = set()
-    for h in ("adainf.h", "adainf_debug.h"):
+    for h in ("adainf.h", "adainf_debug.h", "adainf_sched.h"):
         txt = open(os.path.join(ROOT, "include", h)).read()
         names |= set(re.findall(r"\b(adainf_[a-z0-9_]+)\s*\(", txt))
     return names

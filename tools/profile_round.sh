@@ -17,5 +17,11 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 3000 --
   --log-file $O/${TAG}_bench_launch_list.csv python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline \
   > $O/${TAG}_bench_under_ncu.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on --nvtx --nvtx-include "profiled/" -k "$KRE" -c ${NFULL:-6} \
-  -o $O/${TAG}_full -f python tools/profile_step.py --steps 2 > $O/${TAG}_full.log 2>&1
+  -o $O/${TAG}_full -f python tools/profile_step.py --train-only --steps 2 > $O/${TAG}_full.log 2>&1
+
+# keep the bring-back small: export the full capture's raw metrics (+ per-kernel SASS stall tops) as CSV and
+# drop the report unless it is small
+ncu -i $O/${TAG}_full.ncu-rep --page raw --csv > $O/${TAG}_full_raw.csv 2>/dev/null
+sz=$(stat -c %s $O/${TAG}_full.ncu-rep 2>/dev/null || echo 0)
+if [ "$sz" -gt 30000000 ]; then rm -f $O/${TAG}_full.ncu-rep; fi
 echo done
