@@ -85,8 +85,9 @@ struct ConvCfg {
   static constexpr int A_BYTES = BM * BK * 2;
   static constexpr int B_BYTES = BN * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  // coalescing buffers of the bf16 epilogue: 4 warps x 2 x (32 rows x 128 B)
-  static constexpr int EPI_BYTES = (MODE != 2 && BN >= 64) ? 4 * 8192 : 0;
+  // coalescing buffers of the bf16 epilogue: 4 warps x 2 operands x (32 rows x 128 B), double-buffered in
+  // the sub-pixel dgrad mode
+  static constexpr int EPI_BYTES = (MODE != 2 && BN >= 64) ? (MODE == 3 ? 4 * 16384 : 4 * 8192) : 0;
   static constexpr int STAGES_FIT = (220 * 1024 - EPI_BYTES - 1280) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_FIT > 8 ? 8 : STAGES_FIT;
   static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/ + EPI_BYTES;
@@ -175,11 +176,6 @@ __device__ __forceinline__ void stage_issue(uint8_t* stg, const bf16* base, long
     cp_async16(smem_u32(stg + stg_off(r, j)), okr ? (const void*)(base + pr * pitch + j * 8) : (const void*)base, okr);
   }
 }
-__device__ __forceinline__ void stage_wait() {
-  asm volatile("cp.async.commit_group;" ::: "memory");
-  asm volatile("cp.async.wait_group 0;" ::: "memory");
-  __syncwarp();
-}
 // each lane applies op to its own row of a staged buffer
 template <class Op>
 __device__ __forceinline__ void stage_apply(const uint8_t* stg, int lane, float* v, Op op) {
@@ -191,45 +187,73 @@ __device__ __forceinline__ void stage_apply(const uint8_t* stg, int lane, float*
     for (int qq = 0; qq < 8; ++qq) v[jj * 8 + qq] = op(v[jj * 8 + qq], __bfloat162float(h[qq]));
   }
 }
-template <class Op>
-__device__ __forceinline__ void stage_rows_in(uint8_t* stg, const bf16* base, long long prow, bool ok, int pitch,
-                                              int lane, float* v, Op op) {
-  stage_issue(stg, base, prow, ok, pitch, lane);
-  stage_wait();
-  stage_apply(stg, lane, v, op);
-  __syncwarp();
-}
 __device__ __forceinline__ void prefetch_l2(const void* p) {
   asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
 }
-// two operands with one memory latency: first into stg, second into stg + 4096
-template <class Op0, class Op1>
-__device__ __forceinline__ void stage_rows_in2(uint8_t* stg, const bf16* base0, long long prow0, const bf16* base1,
-                                               long long prow1, bool ok, int pitch, int lane, float* v, Op0 op0,
-                                               Op1 op1) {
-  stage_issue(stg, base0, prow0, ok, pitch, lane);
-  stage_issue(stg + 4096, base1, prow1, ok, pitch, lane);
-  stage_wait();
-  stage_apply(stg, lane, v, op0);
-  stage_apply(stg + 4096, lane, v, op1);
-  __syncwarp();
+// Column-block geometry of the coalesced epilogue: where a row's 64 channels of this block come from / go to
+struct EpiBlk {
+  bool ok;              // row valid for this block (inside the batch; SP: output pixel inside the image)
+  long long orow, srow;  // output / shortcut-term row
+  const bf16* scp;       // shortcut term source (SP compact: phase 0 only)
+  int ocol, NO;          // channel offset within the output row, output row pitch (channels)
+};
+
+template <int MODE>
+__device__ __forceinline__ EpiBlk epi_block(const ConvArgs& a, int cb, long long m, bool rv, int n, long long orow,
+                                            int gy, int gx) {
+  EpiBlk e;
+  e.ok = rv;
+  e.orow = e.srow = orow;
+  e.scp = a.sc;
+  e.ocol = cb;
+  e.NO = a.Nout;
+  if (MODE == MODE_DGRAD_SP) {
+    const int ph = cb / a.sp_cin;
+    e.ocol = cb - ph * a.sp_cin;
+    e.NO = a.sp_cin;
+    const int oy = 2 * gy + (ph >> 1), ox = 2 * gx + (ph & 1);
+    e.ok = rv && oy < a.Ho && ox < a.Wo;
+    e.orow = e.srow = ((long long)n * a.Ho + oy) * a.Wo + ox;
+    if (a.sp_sc_compact) {
+      e.srow = m;
+      if (ph != 0) e.scp = nullptr;
+    }
+  }
+  return e;
 }
 
+// Coalesced epilogue.  Operands (FWD: residual; DGRAD: shortcut term and activation) are staged with cp.async
+// into per-warp buffers; in the sub-pixel mode (short K, epilogue-heavy tiles) they are double-buffered: the
+// first block's operands are requested before waiting for the accumulator, block c+1's while block c is
+// combined, so the epilogue does not pay a memory latency per column block.
 template <int MODE, int BN>
 __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const TileInfo& ti, uint32_t trow,
-                                                   uint64_t* tempty_b, int nkb, long long m, bool rv, int n,
-                                                   long long orow, long long rrow, int HWg, uint8_t* stg, int lane) {
+                                                   uint64_t* tfull_b, uint32_t tpar, uint64_t* tempty_b, int nkb,
+                                                   long long m, bool rv, int n, long long orow, long long rrow,
+                                                   int HWg, uint8_t* stg, int lane) {
+  constexpr bool PIPE = MODE == MODE_DGRAD_SP;
   int gy = 0, gx = 0;
   if (MODE == MODE_DGRAD_SP && rv) {
     const int pix = (int)m - n * HWg;
     gy = pix / a.Wg;
     gx = pix - gy * a.Wg;
   }
-  // L2 prefetch of this row's epilogue operands for the column blocks after the first (the first block's
-  // loads are issued right away; later blocks then hit L2 instead of DRAM)
-  if (MODE != MODE_DGRAD_SP && rv) {
+  const int ma = MODE == MODE_FWD ? 0 : a.mask_act;
+  // operand 0: FWD residual / DGRAD shortcut term; operand 1: DGRAD activation (mask)
+  auto issue = [&](const EpiBlk& e, int par) {
+    uint8_t* s0 = stg + (PIPE ? par * 8192 : 0);
+    if (MODE == MODE_FWD) {
+      if (a.res) stage_issue(s0, a.res + e.ocol, rrow, e.ok, e.NO, lane);
+    } else {
+      if (e.scp) stage_issue(s0, e.scp + e.ocol, e.srow, e.ok, e.NO, lane);
+      if (ma) stage_issue(s0 + 4096, a.yact + e.ocol, e.orow, e.ok, e.NO, lane);
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  // L2 prefetch of this row's operands for the later column blocks (non-pipelined modes)
+  if (!PIPE && rv) {
     const bf16* p0 = MODE == MODE_FWD ? a.res : a.sc;
-    const bf16* p1 = MODE == MODE_FWD ? nullptr : (a.mask_act ? a.yact : nullptr);
+    const bf16* p1 = MODE == MODE_FWD ? nullptr : (ma ? a.yact : nullptr);
     const long long r0 = MODE == MODE_FWD ? rrow : orow;
 #pragma unroll 1
     for (int c = 64; c < BN; c += 64) {
@@ -238,8 +262,13 @@ __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const Tile
       if (p1) prefetch_l2(p1 + orow * a.Nout + ti.n0 + c);
     }
   }
+  EpiBlk cur = epi_block<MODE>(a, ti.n0, m, rv, n, orow, gy, gx);
+  if (PIPE) issue(cur, 0);
+  mbar_wait(tfull_b, tpar);
+  tc_fence_after();
+  int it = 0;
 #pragma unroll 1
-  for (int c0 = 0; c0 < BN; c0 += 64) {
+  for (int c0 = 0; c0 < BN; c0 += 64, ++it) {
     float v[64];
     if (nkb > 0) {
       tmem_ld32(trow + c0, v);
@@ -253,76 +282,69 @@ __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const Tile
       mbar_arrive(tempty_b);  // accumulator free for the tile after next
     }
     const int cb = ti.n0 + c0;
-    if (cb >= a.Nout) continue;  // warp-uniform
-    int ocol = cb, NO = a.Nout;
-    bool ok = rv;
-    long long orow_b = orow, srow = orow;
-    const bf16* scp = a.sc;
-    if (MODE == MODE_DGRAD_SP) {
-      const int ph = cb / a.sp_cin;
-      ocol = cb - ph * a.sp_cin;
-      NO = a.sp_cin;
-      const int oy = 2 * gy + (ph >> 1), ox = 2 * gx + (ph & 1);
-      ok = rv && oy < a.Ho && ox < a.Wo;
-      orow_b = ((long long)n * a.Ho + oy) * a.Wo + ox;
-      srow = orow_b;
-      if (a.sp_sc_compact) {
-        srow = m;
-        if (ph != 0) scp = nullptr;
+    if (cb >= a.Nout) continue;  // warp-uniform (Nout % 64 == 0); keep looping: the last block frees the accumulator
+    const bool has_next = c0 + 64 < BN && cb + 64 < a.Nout;
+    if (!PIPE) cur = epi_block<MODE>(a, cb, m, rv, n, orow, gy, gx);
+    EpiBlk nxt = cur;
+    if (PIPE) {
+      if (has_next) {
+        nxt = epi_block<MODE>(a, cb + 64, m, rv, n, orow, gy, gx);
+        issue(nxt, (it + 1) & 1);
+        asm volatile("cp.async.wait_group 1;" ::: "memory");
+      } else {
+        asm volatile("cp.async.wait_group 0;" ::: "memory");
       }
+    } else {
+      issue(cur, 0);
+      asm volatile("cp.async.wait_group 0;" ::: "memory");
     }
+    __syncwarp();
+    uint8_t* s0 = stg + (PIPE ? (it & 1) * 8192 : 0);
+    const auto add = [](float x, float r) { return __fadd_rn(x, r); };
     if (MODE == MODE_FWD) {
       if (!(a.exp_flags & 2)) {
 #pragma unroll
         for (int i = 0; i < 64; ++i) v[i] = __fadd_rn(v[i], __ldg(a.bias + cb + i));  // flat params: 4B-aligned
       }
-      if (a.res)
-        stage_rows_in(stg, a.res + ocol, rrow, ok, NO, lane, v, [](float x, float r) { return __fadd_rn(x, r); });
+      if (a.res) stage_apply(s0, lane, v, add);
 #pragma unroll
       for (int i = 0; i < 64; ++i) v[i] = act_apply(a.act, v[i]);
     } else {
-      if (a.bcast && ok) {
+      if (a.bcast && cur.ok) {
 #pragma unroll
         for (int i = 0; i < 64; i += 4) {
-          const float4 bb = __ldg((const float4*)(a.bcast + (long long)n * NO + ocol + i));
+          const float4 bb = __ldg((const float4*)(a.bcast + (long long)n * cur.NO + cur.ocol + i));
           v[i] = __fadd_rn(v[i], bb.x);
           v[i + 1] = __fadd_rn(v[i + 1], bb.y);
           v[i + 2] = __fadd_rn(v[i + 2], bb.z);
           v[i + 3] = __fadd_rn(v[i + 3], bb.w);
         }
       }
-      const int ma = a.mask_act;
-      if (scp && ma) {
-        stage_rows_in2(stg, scp + ocol, srow, a.yact + ocol, orow_b, ok, NO, lane, v,
-                       [](float x, float r) { return __fadd_rn(x, r); },
-                       [ma](float x, float y) { return __fmul_rn(x, act_grad(ma, y)); });
-      } else if (scp) {
-        stage_rows_in(stg, scp + ocol, srow, ok, NO, lane, v, [](float x, float r) { return __fadd_rn(x, r); });
-      } else if (ma) {
-        stage_rows_in(stg, a.yact + ocol, orow_b, ok, NO, lane, v,
-                      [ma](float x, float y) { return __fmul_rn(x, act_grad(ma, y)); });
-      }
+      if (cur.scp) stage_apply(s0, lane, v, add);
+      if (ma) stage_apply(s0 + 4096, lane, v, [ma](float x, float y) { return __fmul_rn(x, act_grad(ma, y)); });
     }
+    __syncwarp();
     // own row -> staging (bf16), then 8 coalesced 16-byte stores per lane
 #pragma unroll
     for (int jj = 0; jj < 8; ++jj) {
       __align__(16) bf16 h[8];
 #pragma unroll
       for (int qq = 0; qq < 8; ++qq) h[qq] = __float2bfloat16_rn(v[jj * 8 + qq]);
-      *(uint4*)(stg + stg_off(lane, jj)) = *(const uint4*)h;
+      *(uint4*)(s0 + stg_off(lane, jj)) = *(const uint4*)h;
     }
     __syncwarp();
     const int j = lane & 7;
-    bf16* ob = (bf16*)a.out + ocol;
+    bf16* ob = (bf16*)a.out + cur.ocol;
 #pragma unroll
-    for (int it = 0; it < 8; ++it) {
-      const int r = it * 4 + (lane >> 3);
-      const long long pr = __shfl_sync(0xffffffffu, orow_b, r);
-      const int okr = __shfl_sync(0xffffffffu, (int)ok, r);
-      const uint4 x = *(const uint4*)(stg + stg_off(r, j));
-      if (okr) *((uint4*)(ob + pr * NO) + j) = x;
+    for (int q8 = 0; q8 < 8; ++q8) {
+      const int r = q8 * 4 + (lane >> 3);
+      const long long pr = __shfl_sync(0xffffffffu, cur.orow, r);
+      const int okr = __shfl_sync(0xffffffffu, (int)cur.ok, r);
+      const uint4 x = *(const uint4*)(s0 + stg_off(r, j));
+      if (okr) *((uint4*)(ob + pr * cur.NO) + j) = x;
     }
     __syncwarp();
+    cur = nxt;
   }
 }
 
@@ -605,8 +627,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
       const TileInfo ti = tile_info<MODE, BN>(a, tile, mt, nt, nkb_total);
       const int nkb = ti.kb1 - ti.kb0;
       const int b = lt & 1, ub = lt >> 1;
-      mbar_wait(&tfull[b], ub & 1);
-      tc_fence_after();
+      bool coalesced = false;
+      if constexpr (Cfg::EPI_BYTES > 0)
+        coalesced = MODE != MODE_WGRAD && !a.out_f32 && (a.Nout & 63) == 0 && !(a.exp_flags & 1);
+      if (!coalesced) {  // the coalesced epilogue waits itself, after requesting its first operands
+        mbar_wait(&tfull[b], ub & 1);
+        tc_fence_after();
+      }
       const uint32_t trow = tmem + (uint32_t)(b * Cfg::ACC_COLS) + ((uint32_t)(q * 32) << 16);
       const long long m = ti.m0 + row;
       if (MODE == MODE_WGRAD) {
@@ -647,9 +674,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
           }
         }
         if constexpr (Cfg::EPI_BYTES > 0) {
-          if (!a.out_f32 && (a.Nout & 63) == 0 && !(a.exp_flags & 1)) {
-            epilogue_coalesced<MODE, BN>(a, ti, trow, &tempty[b], nkb, m, rv, n, orow, rrow, HWg,
-                                          epi_smem + q * 8192, lane);
+          if (coalesced) {
+            epilogue_coalesced<MODE, BN>(a, ti, trow, &tfull[b], ub & 1, &tempty[b], nkb, m, rv, n, orow, rrow,
+                                          HWg, epi_smem + q * (Cfg::EPI_BYTES / 4), lane);
             continue;
           }
         }
