@@ -23,7 +23,8 @@ for d in data.values():
     c[2] += f(d.get("dram__bytes_read.sum")) + f(d.get("dram__bytes_write.sum"))
     c[3] += f(d.get("sm__pipe_tensor_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed")) * f(d.get("gpu__time_duration.sum"))
 tot_t = sum(c[1] for c in cls.values())
-out = [f"# {tag}: one ResNet-18-EE step (infer 256 + retrain 1024), ncu launch metrics (cold, serialised)\n",
+out = [f"# {tag}: one ResNet-18-EE step (infer 256 + retrain 1024), ncu launch metrics (cold, serialised: "
+       f"compare shares, not absolutes)\n",
        "| kernel | launches | time ms | share | DRAM GB | avg GB/s | tensor-pipe % (time-weighted) |",
        "|---|---|---|---|---|---|---|"]
 for k, c in sorted(cls.items(), key=lambda kv: -kv[1][1]):
@@ -31,7 +32,7 @@ for k, c in sorted(cls.items(), key=lambda kv: -kv[1][1]):
     unit = 1e9 if max(c[2], 1) > 1e6 else 1.0
     out.append(f"| `{k[:60]}` | {c[0]} | {c[1]/1e6:.3f} | {c[1]/tot_t*100:.1f}% | {c[2]/1e9:.3f} | "
                f"{c[2]/max(c[1],1):.0f} | {c[3]/max(c[1],1):.1f} |")
-conv = [d for d in data.values() if d["name"].startswith(("void conv_umma_kernel", "conv_win"))]
+conv = [d for d in data.values() if d["name"].startswith(("void conv_", "conv_"))]
 conv_bytes = sum(f(d.get("dram__bytes_read.sum")) + f(d.get("dram__bytes_write.sum")) for d in conv)
 conv_t = sum(f(d.get("gpu__time_duration.sum")) for d in conv)
 out.append(f"\nconv GEMM (all variants): {len(conv)} launches, {conv_t/1e6:.3f} ms, DRAM {conv_bytes/1e9:.3f} GB "
@@ -40,12 +41,14 @@ json.dump({"tag": tag, "conv_umma_kernel_bytes_per_launch": conv_bytes / max(len
            "conv_launches": len(conv), "conv_time_ms": conv_t / 1e6, "source": traffic_csv},
           open("profiles/ncu_traffic.json", "w"), indent=1)
 # full capture: key metrics per profiled kernel
-raw = subprocess.run(["ncu", "-i", full_rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+raw = open(full_rep).read() if full_rep.endswith(".csv") else subprocess.run(
+    ["ncu", "-i", full_rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
 rr = list(csv.reader(raw.splitlines()))
 h = rr[0]
 keys = ["gpu__time_duration.sum", "TPC.TriageCompute.sm__pipe_tensor_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed",
         "dram__bytes_read.sum", "dram__bytes_write.sum", "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed",
         "smsp__issue_active.avg.pct_of_peak_sustained_active", "lts__t_sectors.avg.pct_of_peak_sustained_elapsed",
+        "l1tex__data_pipe_tc_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed",
         "launch__registers_per_thread", "sm__warps_active.avg.pct_of_peak_sustained_active"]
 out.append("## ncu --set full captures (key metrics)\n")
 out.append("| kernel | " + " | ".join(k.split(".")[-3] if k.startswith("TPC") else k for k in keys) + " |")
