@@ -174,15 +174,15 @@ __host__ __device__ constexpr uint32_t make_idesc(int M, int N, int a_mn_major, 
          ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
 }
 
+// Branch-free (select) forms: the activation kind is a runtime layer attribute, and a per-element branch on it
+// costs the single epilogue warp of each TMEM lane quadrant more than the arithmetic itself.
 __device__ __forceinline__ float act_apply(int act, float v) {
-  if (act == 1) return v > 0.f ? v : 0.f;
-  if (act == 2) return v > 0.f ? v : __fmul_rn(0.1f, v);
-  return v;
+  const float neg = act == 2 ? __fmul_rn(0.1f, v) : 0.f;
+  return (act == 0 || v > 0.f) ? v : neg;
 }
 __device__ __forceinline__ float act_grad(int act, float y) {
-  if (act == 1) return y > 0.f ? 1.f : 0.f;
-  if (act == 2) return y > 0.f ? 1.f : 0.1f;
-  return 1.f;
+  const float neg = act == 2 ? 0.1f : 0.f;
+  return (act == 0 || y > 0.f) ? 1.f : neg;
 }
 
 }  // namespace adainf

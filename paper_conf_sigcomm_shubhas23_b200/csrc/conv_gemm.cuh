@@ -75,6 +75,12 @@ struct ConvArgs {
   int sp_cin;           // DGRAD_SP: Cin of the output (column block width); sp_sc_compact: sc is indexed by
   int sp_sc_compact;    // the dZ-grid row m and applies to phase (0,0) only (compact projection dgrad)
   CUtensorMap b_map;
+  // ---- optional TMA im2col for the A operand of FWD / DGRAD / DGRAD_SP (dense source, Cs % 64 == 0, square
+  // geometry): one elected producer thread issues one im2col load per K-block (128 GEMM rows x 64 channels
+  // of one tap) instead of 128 threads decoding rows and issuing 8 cp.async each; requires b_tma ----
+  int a_tma;
+  int a_lo;             // base pixel = (g * stride + a_lo); tap offset = t{y,x}[tap] - a_lo >= 0
+  CUtensorMap a_map;
 };
 
 constexpr int BM = 128, BK = 64;
@@ -90,7 +96,8 @@ struct ConvCfg {
   static constexpr int EPI_BYTES = (MODE != 2 && BN >= 64) ? (MODE == 3 ? 4 * 16384 : 4 * 8192) : 0;
   static constexpr int STAGES_FIT = (220 * 1024 - EPI_BYTES - 1280) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_FIT > 8 ? 8 : STAGES_FIT;
-  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/ + EPI_BYTES;
+  static constexpr int BIAS_BYTES = (MODE == 0 && EPI_BYTES > 0) ? 4096 : 0;  // FWD bias vector (Nout <= 1024)
+  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/ + EPI_BYTES + BIAS_BYTES;
   static constexpr int ACC_COLS = BN < 32 ? 32 : BN;
   static constexpr int TMEM_COLS = 2 * ACC_COLS;  // double-buffered accumulator
 };
@@ -230,7 +237,7 @@ template <int MODE, int BN>
 __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const TileInfo& ti, uint32_t trow,
                                                    uint64_t* tfull_b, uint32_t tpar, uint64_t* tempty_b, int nkb,
                                                    long long m, bool rv, int n, long long orow, long long rrow,
-                                                   int HWg, uint8_t* stg, int lane) {
+                                                   int HWg, uint8_t* stg, int lane, const float* bias_s) {
   constexpr bool PIPE = MODE == MODE_DGRAD_SP;
   int gy = 0, gx = 0;
   if (MODE == MODE_DGRAD_SP && rv) {
@@ -303,8 +310,19 @@ __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const Tile
     const auto add = [](float x, float r) { return __fadd_rn(x, r); };
     if (MODE == MODE_FWD) {
       if (!(a.exp_flags & 2)) {
+        if (bias_s) {  // staged once per CTA: 16 broadcast LDS.128 instead of 64 uniform global loads
 #pragma unroll
-        for (int i = 0; i < 64; ++i) v[i] = __fadd_rn(v[i], __ldg(a.bias + cb + i));  // flat params: 4B-aligned
+          for (int i = 0; i < 64; i += 4) {
+            const float4 bb = *(const float4*)(bias_s + cb + i);
+            v[i] = __fadd_rn(v[i], bb.x);
+            v[i + 1] = __fadd_rn(v[i + 1], bb.y);
+            v[i + 2] = __fadd_rn(v[i + 2], bb.z);
+            v[i + 3] = __fadd_rn(v[i + 3], bb.w);
+          }
+        } else {
+#pragma unroll
+          for (int i = 0; i < 64; ++i) v[i] = __fadd_rn(v[i], __ldg(a.bias + cb + i));  // flat params: 4B-aligned
+        }
       }
       if (a.res) stage_apply(s0, lane, v, add);
 #pragma unroll
@@ -361,6 +379,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
   uint64_t* tempty = tfull + 2;       // [2]
   uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
   uint8_t* epi_smem = smem + STAGES * Cfg::STAGE_BYTES + 256;  // Cfg::EPI_BYTES (non-WGRAD, BN >= 64)
+  float* bias_s = nullptr;  // FWD: the layer's bias vector, staged once per CTA
+  if (Cfg::BIAS_BYTES > 0 && a.bias && a.Nout <= Cfg::BIAS_BYTES / 4) {
+    bias_s = (float*)(epi_smem + Cfg::EPI_BYTES);
+    for (int i = threadIdx.x; i < a.Nout; i += NUM_THREADS) bias_s[i] = __ldg(a.bias + i);
+  }
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nsamp = a.count ? *a.count : a.n_static;
@@ -374,7 +397,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
   if (threadIdx.x == 0) {
     const bool btma = MODE != MODE_WGRAD && a.b_tma;
     for (int s = 0; s < STAGES; ++s) {
-      mbar_init(&full[s], btma ? 129 : 128);  // 128 cp.async arrivals (+1 expect_tx arrival of the B TMA)
+      // 128 cp.async arrivals (+1 expect_tx arrival of the B TMA); A by TMA: the single expect_tx arrival
+      mbar_init(&full[s], (btma && a.a_tma) ? 1 : (btma ? 129 : 128));
       mbar_init(&empty[s], 1);
     }
     for (int b = 0; b < 2; ++b) {
@@ -397,7 +421,36 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
     for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x) {
       const TileInfo ti = tile_info<MODE, BN>(a, tile, mt, nt, nkb_total);
       const int nkb = ti.kb1 - ti.kb0;
-      if (MODE != MODE_WGRAD) {
+      if (MODE != MODE_WGRAD && a.a_tma) {
+        // A and B by TMA: one thread issues both loads of every K-block
+        if (t == 0) {
+          const int n0 = (int)(ti.m0 / HWg);
+          const int pix = (int)ti.m0 - n0 * HWg;
+          const int gy = pix / a.Wg, gx = pix - gy * a.Wg;
+          const int bw = gx * a.sx + a.a_lo, bh = gy * a.sy + a.a_lo;
+          int k = ti.kb0 * BK;
+          int tap = k / a.Cs, c = k - tap * a.Cs;
+          for (int kbi = 0; kbi < nkb; ++kbi, ++it) {
+            const int s = it % STAGES, u = it / STAGES;
+            if (u > 0) mbar_wait(&empty[s], (u - 1) & 1);
+            const uint32_t sa = smem_base + s * Cfg::STAGE_BYTES;
+            const uint32_t sb = sa + Cfg::A_BYTES;
+            mbar_expect_tx(&full[s], (uint32_t)(Cfg::A_BYTES + Cfg::B_BYTES));
+            tma_load_im2col_4d(sa, &a.a_map, &full[s], c, bw, bh, n0, (uint16_t)(a.tx[tap] - a.a_lo),
+                               (uint16_t)(a.ty[tap] - a.a_lo));
+            const int kb64 = (ti.kb0 + kbi) * BK;
+            if (ModeTraits<MODE>::B_KMAJ) {
+              tma_load_2d(sb, &a.b_map, &full[s], kb64, ti.n0);
+            } else {
+#pragma unroll
+              for (int b = 0; b < BN / 64; ++b)
+                tma_load_2d(sb + b * 8192, &a.b_map, &full[s], a.btap[tap] * a.Nout + ti.n0 + b * 64, c);
+            }
+            c += BK;
+            if (c >= a.Cs) c = 0, ++tap;
+          }
+        }
+      } else if (MODE != MODE_WGRAD) {
         // A: 128 rows (pixels) x 8 chunks; thread -> chunk t&7, rows (t>>3)+16*i
         const int j = t & 7;
         long long rowbase[8];
@@ -676,7 +729,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
         if constexpr (Cfg::EPI_BYTES > 0) {
           if (coalesced) {
             epilogue_coalesced<MODE, BN>(a, ti, trow, &tfull[b], ub & 1, &tempty[b], nkb, m, rv, n, orow, rrow,
-                                          HWg, epi_smem + q * (Cfg::EPI_BYTES / 4), lane);
+                                          HWg, epi_smem + q * (Cfg::EPI_BYTES / 4), lane, bias_s);
             continue;
           }
         }

@@ -254,6 +254,31 @@ static bool btma_on() {
   return g_btma != 0;
 }
 
+// TMA im2col for the A operand of the generic kernel (ADAINF_ATMA=0 restores the cp.async gather)
+static int g_atma = -1;
+static bool atma_on() {
+  if (g_atma < 0) {
+    const char* e = getenv("ADAINF_ATMA");
+    g_atma = e ? atoi(e) : 1;
+  }
+  return g_atma != 0;
+}
+// Switch the A operand to im2col TMA loads when the gather is a plain strided window over a dense source:
+// the base pixel of GEMM row (n, gy, gx) is (gy * s + lo, gx * s + lo) and every tap offset is >= 0 from it.
+static void try_a_tma(ConvArgs& a) {
+  if (!atma_on() || !a.b_tma || a.src_map || a.Cs % 64 != 0 || a.Hs != a.Ws || a.Hg != a.Wg || a.sy != a.sx ||
+      a.sy > 8 || a.ntaps <= 0)
+    return;
+  int loy = 127, lox = 127;
+  for (int t = 0; t < a.ntaps; ++t) loy = std::min(loy, (int)a.ty[t]), lox = std::min(lox, (int)a.tx[t]);
+  if (loy != lox) return;
+  const int lo = loy, up = lo + (a.Hg - 1) * a.sy - (a.Hs - 1);
+  if (lo < -128 || up < -128 || up > 127) return;
+  a.a_map = make_tmap_im2col(a.src, a.n_static, a.Hs, a.Ws, a.Cs, lo, up, a.sy, 64, BM);
+  a.a_lo = lo;
+  a.a_tma = 1;
+}
+
 static int pick_bn(int nout, bool mn_major_b) {
   if (nout <= 32 && !mn_major_b) return 32;
   if (nout <= 64) return 64;
@@ -302,8 +327,12 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
   a.res_map = res_map;
   a.act = act;
   if (n_static <= 0) return;
+  // the generic kernel with im2col TMA operands beats the window kernels except at 64x64 (BN = 64); the window
+  // kernels still serve survivor-mapped sources (x_map), which im2col TMA cannot gather
+  const bool gen_tma = atma_on() && btma_on() && !x_map && g.Cin % 64 == 0 && g.H == g.W;
   if (win_ok(g) && !out_f32 &&
-      (win_mode() >= 2 || (g.Cin == 64 && g.Cout == 64) || (win_mode() != 4 && g.W <= 28 && g.W >= 8 && g.Cout % 128 == 0))) {
+      (win_mode() >= 2 || (g.Cin == 64 && g.Cout == 64) ||
+       (!gen_tma && win_mode() != 4 && g.W <= 28 && g.W >= 8 && g.Cout % 128 == 0))) {
     // window kernel: weight-stationary 64x64 variant by default; the general window FWD measured slower
     WinArgs w{};
     w.c = a;
@@ -330,6 +359,7 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
   if (btma_on() && ldb % 8 == 0 && ((uintptr_t)w & 15) == 0) {
     a.b_tma = 1;
     a.b_map = make_tmap_2d(w, g.Cout, a.K, ldb, 64, BN);  // K-major [Cout][K]; k >= K and rows >= Cout read 0
+    try_a_tma(a);
   }
   launch_bn<MODE_FWD>(BN, a, mt * ((g.Cout + BN - 1) / BN), st);
 }
@@ -340,8 +370,10 @@ void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n
   // dX[y] = sum_{kh: (y + pad - kh) % s == 0} dZ[(y + pad - kh)/s] W[kh]; split by output phase (py,px)
   // W < 8 (ResNet layer 4): the generic kernel with TMA weight boxes beats the cp.async window kernel
   const bool small_w_generic = g.W < 8 && btma_on() && g.Cout % 64 == 0 && g.Cin % 64 == 0 && win_mode() < 2;
+  const bool gen_tma = atma_on() && btma_on() && g.Cout % 64 == 0 && g.Cin % 64 == 0 && g.H == g.W;
   if (win_ok(g) && !small_w_generic &&
-      (g.H <= 14 || win_mode() >= 2 || (g.Cin == 64 && g.Cout == 64) || (g.W <= 28 && g.Cin % 128 == 0))) {
+      (win_mode() >= 2 || (g.Cin == 64 && g.Cout == 64) ||
+       (!gen_tma && (g.H <= 14 || (g.W <= 28 && g.Cin % 128 == 0))))) {
     // stride 1: one window launch with flipped taps (faster at H<=14; weight-stationary at 64x64)
     WinArgs wa{};
     ConvArgs& a = wa.c;
@@ -417,6 +449,7 @@ void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n
           ((uintptr_t)w & 15) == 0) {
         a.b_tma = 1;
         a.b_map = make_tmap_2d(w, g.Cout, ldb, ldb, 64, 64);  // rows co, cols (tap, ci): MN-major boxes
+        try_a_tma(a);
       }
       launch_bn<MODE_DGRAD>(BN, a, mt * ((g.Cin + BN - 1) / BN), st);
     }
@@ -496,6 +529,7 @@ void conv_dgrad_sp(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, bf
   a.sp_sc_compact = sc_compact ? 1 : 0;
   a.b_tma = 1;
   a.b_map = make_tmap_2d(wsp, a.Nout, a.K, a.ldb, 64, 256);
+  try_a_tma(a);
   const long long mt = ((long long)n * g.Ho * g.Wo + BM - 1) / BM;
   launch_t<MODE_DGRAD_SP, 256>(a, mt * ((a.Nout + 255) / 256), st);
 }

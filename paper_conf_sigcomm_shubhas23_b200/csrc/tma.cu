@@ -55,6 +55,37 @@ CUtensorMap make_tmap_nhwc_swz(const void* base, int N, int H, int W, int C, int
   return m;
 }
 
+static PFN_cuTensorMapEncodeIm2col_v12000 encode_im2col_fn() {
+  static PFN_cuTensorMapEncodeIm2col_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeIm2col", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (PFN_cuTensorMapEncodeIm2col_v12000)p;
+  });
+  if (!fn) throw CudaError("cuTensorMapEncodeIm2col unavailable");
+  return fn;
+}
+
+// im2col map over NHWC [N][H][W][C] bf16: 128B swizzle, `pixels` pixel rows of `ch` channels per load.
+// The pixel bounding box is [lo, dim - 1 + up] in H and W (same for both), traversed with `stride`.
+CUtensorMap make_tmap_im2col(const void* base, int N, int H, int W, int C, int lo, int up, int stride, int ch,
+                             int pixels) {
+  CUtensorMap m;
+  const cuuint64_t dims[4] = {(cuuint64_t)C, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
+  const cuuint64_t strides[3] = {(cuuint64_t)C * 2, (cuuint64_t)W * C * 2, (cuuint64_t)H * W * C * 2};
+  const int lower[2] = {lo, lo}, upper[2] = {up, up};
+  const cuuint32_t es[4] = {1, (cuuint32_t)stride, (cuuint32_t)stride, 1};
+  CUresult r = encode_im2col_fn()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(base), dims, strides,
+                                  lower, upper, (cuuint32_t)ch, (cuuint32_t)pixels, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                  CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) throw CudaError("cuTensorMapEncodeIm2col failed: " + std::to_string((int)r));
+  return m;
+}
+
 CUtensorMap make_tmap_2d(const void* base, long long rows, int cols, int ld, int bcols, int brows) {
   CUtensorMap m;
   const cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};

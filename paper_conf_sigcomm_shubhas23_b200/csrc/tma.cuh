@@ -18,6 +18,11 @@ CUtensorMap make_tmap_nhwc_plain(const void* base, int N, int H, int W, int C, i
 CUtensorMap make_tmap_nhwc_swz(const void* base, int N, int H, int W, int C, int bc, int bw, int bh, int swz);
 // 2-D tiled map over a row-major [rows][cols] bf16 matrix (row pitch ld elements), box {bcols, brows}.
 CUtensorMap make_tmap_2d(const void* base, long long rows, int cols, int ld, int bcols, int brows);
+// im2col map over NHWC [N][H][W][C] bf16 (128B swizzle): one load = `pixels` consecutive GEMM rows (output
+// positions, W fastest then H then N, base positions [lo, dim-1+up] stepped by `stride`) x `ch` channels of the
+// filter tap given by the load's offsets; elements outside the tensor read 0.
+CUtensorMap make_tmap_im2col(const void* base, int N, int H, int W, int C, int lo, int up, int stride, int ch,
+                             int pixels);
 
 __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
@@ -28,6 +33,15 @@ __device__ __forceinline__ void tma_load_4d(uint32_t dst, const CUtensorMap* map
       "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], "
       "[%6];" ::"r"(dst),
       "l"(map), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(smem_u32(bar))
+      : "memory");
+}
+// im2col load: coordinates {c, w, h, n} of the first row's base pixel, filter-tap offsets (ow, oh) >= 0
+__device__ __forceinline__ void tma_load_im2col_4d(uint32_t dst, const CUtensorMap* map, uint64_t* bar, int c, int w,
+                                                   int h, int n, uint16_t ow, uint16_t oh) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.im2col.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], "
+      "[%6], {%7, %8};" ::"r"(dst),
+      "l"(map), "r"(c), "r"(w), "r"(h), "r"(n), "r"(smem_u32(bar)), "h"(ow), "h"(oh)
       : "memory");
 }
 __device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1) {
