@@ -304,7 +304,7 @@ void launch_maxpool_bwd(const bf16* dT, const uint8_t* amax, const bf16* pooled,
 // ------------------------------------------------------------------------------------------------
 // Fused exit head: one CTA per dense row.  GAP over HW with 16-byte loads (channel vector v = t % (C/8),
 // pixel group t / (C/8)), fixed-order reduction, FC in fp32, softmax statistics with IEEE expf/logf.
-constexpr int EH_THREADS = 256;
+constexpr int EH_THREADS = 128;  // 128-thread CTAs: a 1,024-row exit fits one wave (12 CTAs / SM)
 __global__ void __launch_bounds__(EH_THREADS) exit_head_kernel(const ExitHeadArgs a) {
   const int n_rows = a.count ? *a.count : a.n_static;
   const int j = blockIdx.x;
@@ -319,7 +319,20 @@ __global__ void __launch_bounds__(EH_THREADS) exit_head_kernel(const ExitHeadArg
   const int v = t % CV, g0 = t / CV;
   if (g0 < groups) {
     const bf16* base = a.fmap + (long long)j * a.HW * C + v * 8;
-    for (int pix = g0; pix < a.HW; pix += groups) {
+    // eight independent 16-byte loads in flight per thread, accumulated in the same (ascending pixel) order
+    int pix = g0;
+    for (; pix + 7 * groups < a.HW; pix += 8 * groups) {
+      uint4 raw[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) raw[u] = __ldg((const uint4*)(base + (long long)(pix + u * groups) * C));
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const bf16* h = (const bf16*)&raw[u];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) acc[q] += __bfloat162float(h[q]);
+      }
+    }
+    for (; pix < a.HW; pix += groups) {
       const uint4 raw = __ldg((const uint4*)(base + (long long)pix * C));
       const bf16* h = (const bf16*)&raw;
 #pragma unroll
@@ -633,17 +646,20 @@ void launch_sum(const float* x, int n, float* out, float scale, cudaStream_t st)
 // Fused SGD + momentum (PyTorch semantics, reading Q9), 128-bit loads/stores of w, v, g, and the bf16
 // shadow written in the GEMM-ready [Cout][ldb] layout for conv weights.  Blocks map to parameter
 // segments through host-built tables so every thread's float4 stays inside one segment.
-constexpr int SGD_THREADS = 256, SGD_VEC = 4, SGD_ITEMS = 4;
+constexpr int SGD_THREADS = 256, SGD_VEC = 4, SGD_ITEMS = 2;  // 2048-element units: < 10% last-wave tail
 constexpr int SGD_PER_BLOCK = SGD_THREADS * SGD_VEC * SGD_ITEMS;
+static_assert(SGD_PER_BLOCK == SGD_BLOCK_ELEMS, "host partition unit");
 
 __device__ __forceinline__ void shadow_store(const SgdSeg& sg, long long local, const float* w4, int cnt) {
   const int K = sg.taps * sg.cin;
-  for (int q = 0; q < cnt; ++q) {
-    const long long l = local + q;
-    const long long co = l / K;
-    const int rem = (int)(l - co * K);
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {  // fully unrolled with a predicate: w4 stays in registers
+    if (q >= cnt) break;
+    const unsigned l = (unsigned)(local + q);
+    const unsigned co = l / (unsigned)K;
+    const int rem = (int)(l - co * (unsigned)K);
     const int tap = rem / sg.cin, ci = rem - tap * sg.cin;
-    sg.shadow[co * sg.ldb + tap * sg.cin_pad + ci] = __float2bfloat16_rn(w4[q]);
+    sg.shadow[(long long)co * sg.ldb + tap * sg.cin_pad + ci] = __float2bfloat16_rn(w4[q]);
   }
 }
 
@@ -681,7 +697,12 @@ __global__ void __launch_bounds__(SGD_THREADS) sgd_kernel(float* __restrict__ w,
       vr[0] = vl[it].x, vr[1] = vl[it].y, vr[2] = vl[it].z, vr[3] = vl[it].w;
       gr[0] = gl[it].x, gr[1] = gl[it].y, gr[2] = gl[it].z, gr[3] = gl[it].w;
     } else {
-      for (int q = 0; q < cnt; ++q) wr[q] = w[i + q], vr[q] = v[i + q], gr[q] = g[i + q];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {  // unrolled + predicated (a runtime trip count would demote wr/vr/gr to local memory)
+        wr[q] = q < cnt ? w[i + q] : 0.f;
+        vr[q] = q < cnt ? v[i + q] : 0.f;
+        gr[q] = q < cnt ? g[i + q] : 0.f;
+      }
     }
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
@@ -696,18 +717,20 @@ __global__ void __launch_bounds__(SGD_THREADS) sgd_kernel(float* __restrict__ w,
       *(float4*)(w + i) = make_float4(wr[0], wr[1], wr[2], wr[3]);
       *(float4*)(v + i) = make_float4(vr[0], vr[1], vr[2], vr[3]);
     } else {
-      for (int q = 0; q < cnt; ++q) w[i + q] = wr[q], v[i + q] = vr[q];
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+        if (q < cnt) w[i + q] = wr[q], v[i + q] = vr[q];
     }
     if (sg.shadow) {
       const long long local = i - sg.off;
       if (sg.cin == sg.cin_pad && (sg.cin & 3) == 0 && cnt == 4 && (local & 3) == 0) {
-        const int K = sg.taps * sg.cin;
-        const long long co = local / K;
-        const int rem = (int)(local - co * K);
+        const unsigned K = (unsigned)(sg.taps * sg.cin);  // segment-local offsets < 2^31: 32-bit division
+        const unsigned co = (unsigned)local / K;
+        const int rem = (int)((unsigned)local - co * K);
         __align__(8) bf16 h[4];
 #pragma unroll
         for (int q = 0; q < 4; ++q) h[q] = __float2bfloat16_rn(wr[q]);
-        *(uint2*)(sg.shadow + co * sg.ldb + rem) = *(uint2*)h;
+        *(uint2*)(sg.shadow + (long long)co * sg.ldb + rem) = *(uint2*)h;
       } else {
         shadow_store(sg, local, wr, cnt);
       }

@@ -77,6 +77,8 @@ struct SgdSeg {
   bf16* shadow;        // conv weight shadow [Cout][ldb] or nullptr
   int taps, cin, cin_pad, ldb;
 };
+// elements per sgd_kernel block (the host partitions the parameter segments into units of this size)
+constexpr int SGD_BLOCK_ELEMS = 256 * 4 * 2;
 void launch_sgd(float* w, float* v, const float* g, long long n, float lr, float mu, float wd, const SgdSeg* segs_dev,
                 int nseg, const int* block_seg_dev, const long long* block_start_dev, int nblocks, float* sq_partial,
                 cudaStream_t st);

@@ -288,7 +288,7 @@ void Model::build(const adainf_model_spec& s) {
   }
   std::vector<int> bseg;
   std::vector<long long> bstart;
-  const long long PER = 256 * 4 * 4;
+  const long long PER = SGD_BLOCK_ELEMS;
   for (size_t si = 0; si < segs.size(); ++si)
     for (long long st = segs[si].off; st < segs[si].off + segs[si].count; st += PER) {
       bseg.push_back((int)si);
