@@ -654,15 +654,12 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
         if (elect_one()) {
           const uint32_t sa = smem_base + s * Cfg::STAGE_BYTES;
           const uint32_t sb = sa + Cfg::A_BYTES;
+          // descriptors are linear in the start address (16-byte units): base + per-k-step offset
+          const uint64_t ad0 = MODE == MODE_WGRAD ? make_sdesc(sa, 8192, 1024) : make_sdesc(sa, 16, 1024);
+          const uint64_t bd0 = ModeTraits<MODE>::B_KMAJ ? make_sdesc(sb, 16, 1024) : make_sdesc(sb, 8192, 1024);
+          constexpr uint32_t A_KK = MODE == MODE_WGRAD ? 128u : 2u, B_KK = ModeTraits<MODE>::B_KMAJ ? 2u : 128u;
 #pragma unroll
-          for (int kk = 0; kk < BK / 16; ++kk) {
-            uint64_t ad, bd;
-            if (MODE == MODE_WGRAD) ad = make_sdesc(sa + kk * 2048, 8192, 1024);
-            else ad = make_sdesc(sa + kk * 32, 16, 1024);
-            if (ModeTraits<MODE>::B_KMAJ) bd = make_sdesc(sb + kk * 32, 16, 1024);
-            else bd = make_sdesc(sb + kk * 2048, 8192, 1024);
-            umma_bf16(dacc, ad, bd, IDESC, (kbi | kk) != 0);
-          }
+          for (int kk = 0; kk < BK / 16; ++kk) umma_bf16(dacc, ad0 + kk * A_KK, bd0 + kk * B_KK, IDESC, (kbi | kk) != 0);
           umma_commit(&empty[s]);
           if (kbi == nkb - 1) umma_commit(&tfull[b]);
         }

@@ -112,7 +112,16 @@ static void launch_ws_tma(const ConvArgs& c, bool dgrad, int nstatic, cudaStream
       a.tap_off[kh * 3 + kw] = dgrad ? 8 + (2 - kh) * Wp + (1 - kw) : 8 + kh * Wp + kw - 1;
       a.btap[kh * 3 + kw] = kh * 3 + kw;
     }
-  a.win_map = make_tmap_nhwc(c.src, nstatic, H, W, 64, 64, Wp, R + 2);
+  // one box per image row when the padded pitch exceeds W (ADAINF_ROWBOX=0: one {64, Wp, R+2} box with
+  // out-of-bounds columns)
+  static int rowbox = -1;
+  if (rowbox < 0) {
+    const char* e = getenv("ADAINF_ROWBOX");
+    rowbox = e ? atoi(e) : 1;
+  }
+  a.rowbox = rowbox && Wp > W && W % 8 == 0 && W <= 256;
+  a.win_map = a.rowbox ? make_tmap_nhwc(c.src, nstatic, H, W, 64, 64, W, 1)
+                       : make_tmap_nhwc(c.src, nstatic, H, W, 64, 64, Wp, R + 2);
   const bf16* e0 = dgrad ? c.sc : c.res;
   const bf16* e1 = dgrad && c.mask_act ? c.yact : nullptr;
   a.has_e0 = e0 != nullptr;
@@ -123,6 +132,7 @@ static void launch_ws_tma(const ConvArgs& c, bool dgrad, int nstatic, cudaStream
   a.win_bytes = ((16 + (R + 2) * Wp) * 128 + 1023) / 1024 * 1024;
   const int fixed = 9 * 8192 + 2 * (a.has_e0 + a.has_e1) * 16384 + 1024 /*align*/ + 512 /*barriers*/;
   a.wstages = std::min(8, (227 * 1024 - fixed) / a.win_bytes);
+  if (const char* e = getenv("ADAINF_WS_STAGES")) a.wstages = std::min(a.wstages, std::max(1, atoi(e)));
   if (a.wstages < 2) throw std::runtime_error("ws_tma: shared memory");
   const int smem = a.wstages * a.win_bytes + fixed;
   static bool attr = false;

@@ -34,6 +34,8 @@ struct WsTmaArgs {
   const float* bcast;
   bf16* out;
   int wstages, win_bytes;
+  int rowbox;  // 1: the window is R+2 boxes {64, W, 1, 1} (one per image row, no out-of-bounds columns); the
+               // pad columns W..Wp-1 of every row slot are zeroed once and never written by the TMA
 };
 
 constexpr int TMA_WS_THREADS = 416;  // warp 0 TMA producer (+ warps 1-3 help load B), warp 4 MMA, 8 epilogue warps
@@ -68,6 +70,15 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
     const int rows = 8 + (R + 2) * Wp;
     uint4* p = (uint4*)(win + s * a.win_bytes + (k < 64 ? k * 16 : rows * 128 + (k - 64) * 16));
     *p = make_uint4(0, 0, 0, 0);
+  }
+  if (a.rowbox) {
+    const int padc = Wp - W, per_stage = (R + 2) * padc * 8;
+    for (int i = threadIdx.x; i < WS * per_stage; i += blockDim.x) {
+      const int s = i / per_stage, k = i - s * per_stage;
+      const int j = k / (padc * 8), rem = k - j * (padc * 8);
+      const int x = W + rem / 8, c = rem % 8;
+      *(uint4*)(win + s * a.win_bytes + 1024 + (j * Wp + x) * 128 + c * 16) = make_uint4(0, 0, 0, 0);
+    }
   }
   if (threadIdx.x < 64) s_bias[threadIdx.x] = (!a.dgrad && a.bias) ? a.bias[threadIdx.x] : 0.f;
   if (threadIdx.x == 0) {
@@ -116,13 +127,26 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
         const int sn = a.smap ? __ldg(a.smap + n) : n;
         const int s = it % WS, u = it / WS;
         if (u > 0) mbar_wait(&wempty[s], (u - 1) & 1);
-        mbar_expect_tx(&wfull[s], box_bytes);
-        tma_load_4d(wsm + s * a.win_bytes + 1024, &a.win_map, &wfull[s], 0, 0, h0 - 1, sn);
+        if (a.rowbox) {
+          mbar_expect_tx(&wfull[s], 64u * 2u * W * (R + 2));
+          for (int j = 0; j < R + 2; ++j)
+            tma_load_4d(wsm + s * a.win_bytes + 1024 + j * Wp * 128, &a.win_map, &wfull[s], 0, 0, h0 - 1 + j, sn);
+        } else {
+          mbar_expect_tx(&wfull[s], box_bytes);
+          tma_load_4d(wsm + s * a.win_bytes + 1024, &a.win_map, &wfull[s], 0, 0, h0 - 1, sn);
+        }
       }
     }
   } else if (warp == 4) {
     // ---- MMA issuer ----
     const uint32_t IDESC = make_idesc(BM, 64, 0, a.dgrad ? 1 : 0);
+    // descriptors are linear in the start address (16-byte units, < 2^14): build the bases once and add
+    // per-(tap, k-step) offsets, so the single issuing thread spends ~3 uniform ops per MMA instead of ~18
+    const uint64_t b_base = a.dgrad ? make_sdesc(bsm, 8192, 1024) : make_sdesc(bsm, 16, 1024);
+    const uint32_t b_kk = a.dgrad ? 128u : 2u;
+    uint32_t toff[9];
+#pragma unroll
+    for (int tp = 0; tp < 9; ++tp) toff[tp] = (uint32_t)a.tap_off[tp] * 8u;
     mbar_wait(bready, 0);
     fence_proxy_async_smem();
     int it = 0;
@@ -135,15 +159,13 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
       if (elect_one()) {
         const uint32_t sw = wsm + s * a.win_bytes;
         const uint32_t dacc = tmem + (uint32_t)(b * 64);
-#pragma unroll 1
-        for (int tp = 0; tp < 9; ++tp) {
-          const uint32_t sb = bsm + tp * 8192;
+        const uint64_t a_base = make_sdesc(sw, 16, 1024);
 #pragma unroll
-          for (int kk = 0; kk < 4; ++kk) {
-            const uint64_t ad = make_sdesc(sw + (uint32_t)a.tap_off[tp] * 128u + kk * 32, 16, 1024);
-            const uint64_t bd = a.dgrad ? make_sdesc(sb + kk * 2048, 8192, 1024) : make_sdesc(sb + kk * 32, 16, 1024);
-            umma_bf16(dacc, ad, bd, IDESC, (tp | kk) != 0);
-          }
+        for (int tp = 0; tp < 9; ++tp) {
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk)
+            umma_bf16(dacc, a_base + (toff[tp] + 2u * kk), b_base + (uint32_t)(tp * 512 + kk * b_kk), IDESC,
+                      (tp | kk) != 0);
         }
         umma_commit(&wempty[s]);
         umma_commit(&tfull[b]);
@@ -376,12 +398,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_win_tma_kernel(const __gr
           tc_fence_after();
           if (elect_one()) {
             const uint32_t sb = bsm + bs * B_BYTES;
+            const uint64_t ad0 = make_sdesc(sw + (uint32_t)a.tap_off[tp] * 128u, 16, 1024);
+            const uint64_t bd0 = a.dgrad ? make_sdesc(sb, 8192, 1024) : make_sdesc(sb, 16, 1024);
+            const uint32_t bkk = a.dgrad ? 128u : 2u;
 #pragma unroll
-            for (int kk = 0; kk < 4; ++kk) {
-              const uint64_t ad = make_sdesc(sw + (uint32_t)a.tap_off[tp] * 128u + kk * 32, 16, 1024);
-              const uint64_t bd = a.dgrad ? make_sdesc(sb + kk * 2048, 8192, 1024) : make_sdesc(sb + kk * 32, 16, 1024);
-              umma_bf16(dacc, ad, bd, IDESC, (cb | tp | kk) != 0);
-            }
+            for (int kk = 0; kk < 4; ++kk) umma_bf16(dacc, ad0 + 2u * kk, bd0 + kk * bkk, IDESC, (cb | tp | kk) != 0);
             umma_commit(&bempty[bs]);
             if (tp == 8) {
               umma_commit(&wempty[s]);
@@ -588,10 +609,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
         tc_fence_after();
         if (elect_one()) {
           const uint32_t sa = sbase + s * STAGE, sb = sa + A_BYTES;
+          const uint64_t ad0 = make_sdesc(sa, 8192, 1024), bd0 = make_sdesc(sb, 8192, 1024);
 #pragma unroll
           for (int kk = 0; kk < 4; ++kk)
-            umma_bf16(dacc, make_sdesc(sa + kk * 2048, 8192, 1024), make_sdesc(sb + kk * 2048, 8192, 1024), IDESC,
-                      (kb != kb0 || kk != 0));
+            umma_bf16(dacc, ad0 + kk * 128u, bd0 + kk * 128u, IDESC, (kb != kb0 || kk != 0));
           umma_commit(&empty[s]);
           if (kb == kb1 - 1) umma_commit(&tfull[b]);
         }

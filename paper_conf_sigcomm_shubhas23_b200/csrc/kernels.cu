@@ -304,7 +304,9 @@ void launch_maxpool_bwd(const bf16* dT, const uint8_t* amax, const bf16* pooled,
 // ------------------------------------------------------------------------------------------------
 // Fused exit head: one CTA per dense row.  GAP over HW with 16-byte loads (channel vector v = t % (C/8),
 // pixel group t / (C/8)), fixed-order reduction, FC in fp32, softmax statistics with IEEE expf/logf.
-constexpr int EH_THREADS = 128;  // 128-thread CTAs: a 1,024-row exit fits one wave (12 CTAs / SM)
+// EH_THREADS = 128 for large batches (a 1,024-row exit fits one wave, 12 CTAs / SM), 512 when the rows alone
+// cannot fill the SMs (each row then has 4x the loads in flight)
+template <int EH_THREADS>
 __global__ void __launch_bounds__(EH_THREADS) exit_head_kernel(const ExitHeadArgs a) {
   const int n_rows = a.count ? *a.count : a.n_static;
   const int j = blockIdx.x;
@@ -399,13 +401,16 @@ __global__ void __launch_bounds__(EH_THREADS) exit_head_kernel(const ExitHeadArg
     for (int k = t; k < a.ncls; k += EH_THREADS) a.logits[(long long)orig * a.ncls + k] = logits[k];
 }
 void launch_exit_head(const ExitHeadArgs& a, cudaStream_t st) {
-  if (a.C % 8 || (EH_THREADS % (a.C / 8)) != 0 || a.C / 8 > EH_THREADS)
-    throw ShapeError("exit head: C must be 8 * a power of two <= 2048");
-  const int groups = EH_THREADS / (a.C / 8);
-  const size_t smem = (size_t)(groups * a.C + a.C + a.ncls) * sizeof(float);
   if (a.n_static <= 0) return;
+  const bool wide = a.n_static < 4 * num_sms();
+  const int T = wide ? 512 : 128;
+  if (a.C % 8 || (T % (a.C / 8)) != 0 || a.C / 8 > 128)
+    throw ShapeError("exit head: C must be 8 * a power of two <= 1024");
+  const int groups = T / (a.C / 8);
+  const size_t smem = (size_t)(groups * a.C + a.C + a.ncls) * sizeof(float);
   ProfScope ps(PC_EXIT_HEAD, st);
-  exit_head_kernel<<<a.n_static, EH_THREADS, smem, st>>>(a);
+  if (wide) exit_head_kernel<512><<<a.n_static, 512, smem, st>>>(a);
+  else exit_head_kernel<128><<<a.n_static, 128, smem, st>>>(a);
   CK(cudaGetLastError());
 }
 
