@@ -6,6 +6,7 @@
 
 #include "common.cuh"
 #include "kernels.cuh"
+#include "pool_bwd.cuh"
 #include "prof.h"
 
 namespace adainf {
@@ -241,43 +242,17 @@ __global__ void __launch_bounds__(256) maxpool_bwd_k3s2_kernel(const bf16* __res
     const long long b = r / BH;
     uint2 cw[4];
     uint4 gw[4];
-#pragma unroll
-    for (int wq = 0; wq < 4; ++wq) {
-      const int ho = bi + (wq >> 1), wo = bj + (wq & 1);
-      if (ho < Ho && wo < Wo) {
-        const long long oi = ((b * Ho + ho) * Wo + wo) * C + cv * 8;
-        cw[wq] = __ldg((const uint2*)(amax + oi));
-        gw[wq] = __ldg((const uint4*)(dT + oi));
-      } else {
-        cw[wq] = make_uint2(0xFFFFFFFFu, 0xFFFFFFFFu);
-        gw[wq] = make_uint4(0u, 0u, 0u, 0u);
-      }
-    }
-    __align__(16) bf16 o00[8], o01[8], o10[8], o11[8];
-#pragma unroll
-    for (int q = 0; q < 8; ++q) {
-      const uint32_t c00 = ((const uint8_t*)&cw[0])[q], c01 = ((const uint8_t*)&cw[1])[q];
-      const uint32_t c10 = ((const uint8_t*)&cw[2])[q], c11 = ((const uint8_t*)&cw[3])[q];
-      const float g00 = __bfloat162float(((const bf16*)&gw[0])[q]), g01 = __bfloat162float(((const bf16*)&gw[1])[q]);
-      const float g10 = __bfloat162float(((const bf16*)&gw[2])[q]), g11 = __bfloat162float(((const bf16*)&gw[3])[q]);
-      const float a00 = c00 == 4 ? g00 : 0.f;
-      const float a01 = __fadd_rn(c00 == 5 ? g00 : 0.f, c01 == 3 ? g01 : 0.f);
-      const float a10 = __fadd_rn(c00 == 7 ? g00 : 0.f, c10 == 1 ? g10 : 0.f);
-      const float a11 = __fadd_rn(__fadd_rn(__fadd_rn(c00 == 8 ? g00 : 0.f, c01 == 6 ? g01 : 0.f), c10 == 2 ? g10 : 0.f),
-                                  c11 == 0 ? g11 : 0.f);
-      o00[q] = __float2bfloat16_rn(a00);
-      o01[q] = __float2bfloat16_rn(a01);
-      o10[q] = __float2bfloat16_rn(a10);
-      o11[q] = __float2bfloat16_rn(a11);
-    }
+    pool_bwd_k3s2_load(dT, amax, b, bi, bj, cv, C, Ho, Wo, cw, gw);
+    uint4 ob[4];
+    pool_bwd_k3s2_block(cw, gw, ob);
     const int ih = 2 * bi, iw = 2 * bj;
     bf16* d0 = dz + ((b * H + ih) * W + iw) * C + cv * 8;
-    *(uint4*)d0 = *(const uint4*)o00;
-    if (iw + 1 < W) *(uint4*)(d0 + C) = *(const uint4*)o01;
+    *(uint4*)d0 = ob[0];
+    if (iw + 1 < W) *(uint4*)(d0 + C) = ob[1];
     if (ih + 1 < H) {
       bf16* d1 = d0 + (long long)W * C;
-      *(uint4*)d1 = *(const uint4*)o10;
-      if (iw + 1 < W) *(uint4*)(d1 + C) = *(const uint4*)o11;
+      *(uint4*)d1 = ob[2];
+      if (iw + 1 < W) *(uint4*)(d1 + C) = ob[3];
     }
   }
 }

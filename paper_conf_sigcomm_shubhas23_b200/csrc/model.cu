@@ -543,10 +543,29 @@ void Model::train_step(const bf16* x, const int32_t* labels, int n, long long n_
       launch_grad_finalize(bcast_of((int)t), sc_of((int)t), T[t].buf, T[t].act, n, T[t].H * T[t].W, T[t].C,
                            T[t].grad, st);
   // reverse walk (K2, K3, K9)
+  // the stem's max-pool backward is fused into its weight gradient when the stem output feeds only the pool
+  static int fuse_env = -1;
+  if (fuse_env < 0) {
+    const char* e = getenv("ADAINF_STEM_POOL_FUSE");
+    fuse_env = e ? atoi(e) : 1;
+  }
+  bool stem_pool_fused = false;
+  if (stem_s2d && fuse_env) {
+    const NodeRt& pl = nodes[stem_pool];
+    const TensorRt& X = T[pl.in];
+    stem_pool_fused = pl.in == nodes[0].out && pl.pk == 3 && pl.ps == 2 && pl.pp == 1 && X.C == 64 &&
+                      (X.act == 0 || X.act == 1) && X.exit_k < 0 && X.res_of < 0 && X.proj < 0;
+  }
   auto conv_backward = [&](NodeRt& nd, const bf16* dz) {
     if (stem_s2d && &nd == &nodes[0]) {
-      stem_wgrad(buf_of(0), dz, n, in_h / 2, in_w / 2, nd.cin_real, wgrad_ws.as<float>(), wgrad_ws_bytes,
-                 G + nd.w_off, G + nd.b_off, st);
+      if (stem_pool_fused) {
+        const NodeRt& pl = nodes[stem_pool];
+        stem_wgrad_pooled(buf_of(0), T[pl.out].grad, pl.argmax.as<uint8_t>(), pl.g.Ho, pl.g.Wo, n, in_h / 2,
+                          in_w / 2, nd.cin_real, wgrad_ws.as<float>(), wgrad_ws_bytes, G + nd.w_off, G + nd.b_off, st);
+      } else {
+        stem_wgrad(buf_of(0), dz, n, in_h / 2, in_w / 2, nd.cin_real, wgrad_ws.as<float>(), wgrad_ws_bytes,
+                   G + nd.w_off, G + nd.b_off, st);
+      }
       return;
     }
     conv_wgrad(nd.g, buf_of(nd.in), dz, n, nd.cin_real, wgrad_ws.as<float>(), wgrad_ws_bytes, G + nd.w_off,
@@ -580,6 +599,7 @@ void Model::train_step(const bf16* x, const int32_t* labels, int n, long long n_
     if (nd.kind == N_POOL) {
       const TensorRt& X = T[nd.in];
       if (nd.in == 0) continue;
+      if (stem_pool_fused && ni == stem_pool) continue;  // inside the stem weight gradient
       launch_maxpool_bwd(T[nd.out].grad, nd.argmax.as<uint8_t>(), T[nd.out].buf, X.act, n, X.H, X.W, X.C, nd.pk, nd.ps, nd.pp,
                          nd.g.Ho, nd.g.Wo, T[nd.in].grad, st);
       continue;

@@ -4,6 +4,7 @@
 
 #include "colsum_tile.cuh"
 #include "conv_gemm.cuh"
+#include "pool_bwd.cuh"
 #include "prof.h"
 #include "runtime.h"
 #include "stem.cuh"
@@ -346,7 +347,11 @@ constexpr int SW_DZ_STAGE = 2 * SLOTS * 128;  // dZ rows i, i+1: 128 positions x
 constexpr int SW_ND = 3;                      // dZ row-pair stages
 constexpr int SW_S_SLOT = SLOTS * 32;         // one S row: 128 positions (cols -2..125) x 16 ch, 32B swizzle
 constexpr int SW_NS = 16;                     // S row ring
-constexpr int SW_SMEM = 1024 + SW_ND * SW_DZ_STAGE + SW_NS * SW_S_SLOT + 1024 + 512 + 3072;
+// fused pool backward: pooled rows (bi, bi+1) of dT (bf16) and codes (u8), box width 64 >= Wp + 1
+constexpr int SW_PT_BYTES = 2 * 64 * 64 * 2, SW_PC_BYTES = 2 * 64 * 64, SW_PSTAGE = SW_PT_BYTES + SW_PC_BYTES;
+constexpr int SW_NP = 2;
+constexpr int SW_BUILDERS = 224;  // warps 1-3 and 5-8 build dZ (fused mode)
+constexpr int SW_SMEM = 1024 + SW_ND * SW_DZ_STAGE + SW_NS * SW_S_SLOT + 1024 + SW_NP * SW_PSTAGE + 512 + 3072;
 
 // dW[ah][aw][ch][co] = sum_q dZ(i, q)[co] * S(i + ah, q + aw)[ch], output rows taken in pairs (i, i+1):
 // A = the two dZ rows (M = 2 x 64 co, MN-major, atoms 16 KB apart), B = one S row rho = i - 2 + o shifted
@@ -359,6 +364,14 @@ struct StemWgArgs {
   int n, Hs, Ws, bands, band_rows;  // band_rows even
   float* part;     // [gridDim.x][2][256][64]
   float* cs_part;  // [gridDim.x][64] or nullptr
+  // fused max-pool backward (pool_dT != nullptr): dZ is never materialised; warps 5-8 build each dZ row pair
+  // in shared memory from the pooled-output gradient [n][Hp][Wp][64] and the argmax codes (pool_bwd.cuh),
+  // in the layout the dZ TMA box would have produced
+  const bf16* pool_dT;
+  const uint8_t* pool_codes;
+  int Hp, Wp;
+  CUtensorMap pt_map;  // dT [n][Hp][Wp][64] bf16, box {64, 64, 2, 1}
+  CUtensorMap pc_map;  // codes [n][Hp][Wp][64] u8, box {64, 64, 2, 1}
 };
 
 __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_constant__ StemWgArgs a) {
@@ -367,12 +380,15 @@ __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_
   uint8_t* dzst = smem;
   uint8_t* sring = dzst + SW_ND * SW_DZ_STAGE;
   uint8_t* guard = sring + SW_NS * SW_S_SLOT;  // finite rows read past the last S slot (invalid positions only)
-  uint64_t* dz_full = (uint64_t*)(guard + 1024);
+  uint8_t* pring = guard + 1024;  // [SW_NP][dT rows | code rows] (fused pool backward)
+  uint64_t* dz_full = (uint64_t*)(pring + SW_NP * SW_PSTAGE);
   uint64_t* dz_empty = dz_full + SW_ND;
   uint64_t* s_full = dz_empty + SW_ND;
   uint64_t* s_empty = s_full + SW_NS;
   uint64_t* tfull = s_empty + SW_NS;
-  uint32_t* tmem_slot = (uint32_t*)(tfull + 1);
+  uint64_t* p_full = tfull + 1;   // [SW_NP]
+  uint64_t* p_empty = p_full + SW_NP;
+  uint32_t* tmem_slot = (uint32_t*)(p_empty + SW_NP);
   float* cs_red = (float*)((uint8_t*)dz_full + 512);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -381,16 +397,30 @@ __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_
   // the next slot, which must hold finite values even before its first load (0 * NaN = NaN)
   for (int i = threadIdx.x; i < (SW_NS * SW_S_SLOT + 1024) / 16; i += blockDim.x)
     ((uint4*)sring)[i] = make_uint4(0, 0, 0, 0);
+  if (a.pool_dT) {  // columns >= Ws of both rows of every dZ stage stay zero (never written by the builders)
+    const int padc = SLOTS - a.Ws, per = 2 * padc * 8;
+    for (int i = threadIdx.x; i < SW_ND * per; i += blockDim.x) {
+      const int st = i / per, k = i - st * per;
+      const int r = k / (padc * 8), rem = k - r * (padc * 8);
+      const int x = a.Ws + rem / 8, j = rem % 8;
+      *(uint4*)(dzst + st * SW_DZ_STAGE + (r * SLOTS + x) * 128 + ((j ^ (x & 7)) << 4)) = make_uint4(0, 0, 0, 0);
+    }
+  }
   if (threadIdx.x == 0) {
     for (int s = 0; s < SW_ND; ++s) {
-      mbar_init(&dz_full[s], 1);
-      mbar_init(&dz_empty[s], a.cs_part ? 4 : 1);  // MMA commit (+ one arrive per column-sum warp)
+      mbar_init(&dz_full[s], a.pool_dT ? SW_BUILDERS : 1);  // TMA transaction, or the dZ-building threads
+      // MMA commit (+ one arrive per column-sum warp; the builders sum the columns themselves in fused mode)
+      mbar_init(&dz_empty[s], (a.cs_part && !a.pool_dT) ? 4 : 1);
     }
     for (int s = 0; s < SW_NS; ++s) {
       mbar_init(&s_full[s], 1);
       mbar_init(&s_empty[s], 1);
     }
     mbar_init(tfull, 1);
+    for (int s = 0; s < SW_NP; ++s) {
+      mbar_init(&p_full[s], 1);
+      mbar_init(&p_empty[s], SW_BUILDERS);
+    }
     fence_mbar_init();
     tma_prefetch_desc(&a.s_map);
     tma_prefetch_desc(&a.dz_map);
@@ -409,6 +439,84 @@ __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_
     i1 = min(a.Hs, i0 + a.band_rows);  // pairs (i, i+1) for i = i0, i0+2, ..; i+1 may be Hs (zero rows)
   };
 
+  // ---- fused pool backward: warps 1-3 and 5-8 build each dZ row pair (2x2 blocks (i/2, bj), 8 channels per
+  // item, two items per thread) from the staged pooled rows, sum its columns for the bias gradient, and hand it
+  // to the MMA warp; the column partials are reduced in fixed order once all MMAs are done ----
+  auto build_dz = [&]() {
+    const int t = warp < 4 ? threadIdx.x - 32 : threadIdx.x - 64;  // 0..223
+    const int j = t & 7;                                             // channel chunk (same for both items)
+    const int BW = (a.Ws + 1) / 2, nitems = BW * 8;
+    float csum[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) csum[q] = 0.f;
+    int P = 0;
+    for (int u = blockIdx.x; u < nunits; u += gridDim.x) {
+      int img, i0, i1;
+      unit_rows(u, img, i0, i1);
+      for (int i = i0; i < i1; i += 2, ++P) {
+        const int st = P % SW_ND, ph = P / SW_ND;
+        const int ps = P % SW_NP;
+        mbar_wait(&p_full[ps], (P / SW_NP) & 1);
+        const uint8_t* pt = pring + ps * SW_PSTAGE;
+        const uint8_t* pc = pt + SW_PT_BYTES;
+        uint4 ob[2][4];
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+          const int item = t + SW_BUILDERS * q;
+          if (item >= nitems) continue;
+          const int bj = item >> 3;
+          uint2 cw[4];
+          uint4 gw[4];
+#pragma unroll
+          for (int wq = 0; wq < 4; ++wq) {  // rows bi, bi+1 of the box; columns >= Wp / rows >= Hp read 0
+            const int r = wq >> 1, c = bj + (wq & 1);
+            cw[wq] = *(const uint2*)(pc + (r * 64 + c) * 64 + j * 8);
+            gw[wq] = *(const uint4*)(pt + (r * 64 + c) * 128 + j * 16);
+          }
+          pool_bwd_k3s2_block(cw, gw, ob[q]);
+        }
+        mbar_arrive(&p_empty[ps]);
+        if (ph > 0) mbar_wait(&dz_empty[st], (ph - 1) & 1);
+        uint8_t* base = dzst + st * SW_DZ_STAGE;
+        const uint4 z = make_uint4(0u, 0u, 0u, 0u);
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+          const int item = t + SW_BUILDERS * q;
+          if (item >= nitems) continue;
+          const int bj = item >> 3;
+#pragma unroll
+          for (int p = 0; p < 4; ++p) {
+            const int r = p >> 1, x = 2 * bj + (p & 1);
+            if (x >= a.Ws) continue;  // pad columns: zeroed once
+            const uint4 v = i + r < a.Hs ? ob[q][p] : z;
+            *(uint4*)(base + (r * SLOTS + x) * 128 + ((j ^ (x & 7)) << 4)) = v;
+            const bf16* h = (const bf16*)&v;
+#pragma unroll
+            for (int c = 0; c < 8; ++c) csum[c] += __bfloat162float(h[c]);
+          }
+        }
+        fence_proxy_async_smem();  // generic-proxy writes -> visible to the tensor core
+        mbar_arrive(&dz_full[st]);
+      }
+    }
+    if (a.cs_part) {
+      // all MMAs done -> the dZ stages are free scratch: [224 threads][8] partials, summed per channel in
+      // thread order
+      mbar_wait(tfull, 0);
+      float* red = (float*)dzst;
+#pragma unroll
+      for (int c = 0; c < 8; ++c) red[t * 8 + c] = csum[c];
+      asm volatile("bar.sync 3, %0;" ::"n"(SW_BUILDERS) : "memory");
+      if (t < 64) {
+        const int jj = t >> 3, c = t & 7;
+        float acc = 0.f;
+        for (int tt = jj; tt < SW_BUILDERS; tt += 8) acc += red[tt * 8 + c];
+        a.cs_part[(long long)blockIdx.x * 64 + t] = acc;
+      }
+      asm volatile("bar.sync 3, %0;" ::"n"(SW_BUILDERS) : "memory");
+    }
+  };
+
   if (warp == 0) {
     if (lane == 0) {
       int L = 0, P = 0;  // S rows loaded, dZ pairs loaded
@@ -423,6 +531,15 @@ __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_
             mbar_expect_tx(&s_full[slot], SW_S_SLOT);
             tma_load_4d(s_u + slot * SW_S_SLOT, &a.s_map, &s_full[slot], 0, -2, nr, img);
           }
+          if (a.pool_dT) {  // dZ pairs are built on chip: stage their pooled rows bi, bi+1 instead
+            const int ps = P % SW_NP, pph = P / SW_NP;
+            if (pph > 0) mbar_wait(&p_empty[ps], (pph - 1) & 1);
+            mbar_expect_tx(&p_full[ps], SW_PSTAGE);
+            const uint32_t pd = smem_u32(pring + ps * SW_PSTAGE);
+            tma_load_4d(pd, &a.pt_map, &p_full[ps], 0, 0, i >> 1, img);
+            tma_load_4d(pd + SW_PT_BYTES, &a.pc_map, &p_full[ps], 0, 0, i >> 1, img);
+            continue;
+          }
           const int st = P % SW_ND, ph = P / SW_ND;
           if (ph > 0) mbar_wait(&dz_empty[st], (ph - 1) & 1);
           mbar_expect_tx(&dz_full[st], SW_DZ_STAGE);
@@ -430,6 +547,8 @@ __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_
         }
       }
     }
+  } else if (warp >= 1 && warp <= 3 && a.pool_dT) {
+    build_dz();
   } else if (warp >= 1 && warp <= 3) {
     if (a.cs_part) {
       TileColsum<64> cs;
@@ -496,6 +615,7 @@ __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_
     }
     __syncwarp();
   } else if (warp >= 5) {
+    if (a.pool_dT) build_dz();
     const int qd = warp & 3;
     const int m = qd * 32 + lane;
     const int half = m >> 6, co = m & 63;
@@ -555,15 +675,38 @@ size_t stem_wgrad_ws_bytes(int n) {
   return (size_t)num_sms() * (2 * 256 * 64 + 64) * sizeof(float);
 }
 
+static void stem_wgrad_impl(const bf16* s, const bf16* dz, const bf16* pool_dT, const uint8_t* pool_codes, int Hp,
+                            int Wp, int n, int Hs, int Ws, int cin_real, float* ws, size_t ws_bytes, float* dw, float* db,
+                            cudaStream_t st);
 void stem_wgrad(const bf16* s, const bf16* dz, int n, int Hs, int Ws, int cin_real, float* ws, size_t ws_bytes,
                 float* dw, float* db, cudaStream_t st) {
+  stem_wgrad_impl(s, dz, nullptr, nullptr, 0, 0, n, Hs, Ws, cin_real, ws, ws_bytes, dw, db, st);
+}
+void stem_wgrad_pooled(const bf16* s, const bf16* pool_dT, const uint8_t* pool_codes, int Hp, int Wp, int n, int Hs,
+                       int Ws, int cin_real, float* ws, size_t ws_bytes, float* dw, float* db, cudaStream_t st) {
+  if (Hp != (Hs - 1) / 2 + 1 || Wp != (Ws - 1) / 2 + 1) throw ShapeError("stem_wgrad_pooled: pool geometry");
+  stem_wgrad_impl(s, nullptr, pool_dT, pool_codes, Hp, Wp, n, Hs, Ws, cin_real, ws, ws_bytes, dw, db, st);
+}
+static void stem_wgrad_impl(const bf16* s, const bf16* dz, const bf16* pool_dT, const uint8_t* pool_codes, int Hp,
+                            int Wp, int n, int Hs, int Ws, int cin_real, float* ws, size_t ws_bytes, float* dw, float* db,
+                            cudaStream_t st) {
   if (n <= 0) return;
   if (Ws > 125) throw ShapeError("stem: width/2 must be <= 125");
   if (ws_bytes < stem_wgrad_ws_bytes(n)) throw std::runtime_error("stem wgrad workspace too small");
   static StemWgArgs a;
   a = StemWgArgs{};
   a.s_map = make_tmap_nhwc_swz(s, n, Hs, Ws, 16, 16, SLOTS, 1, 32);
-  a.dz_map = make_tmap_nhwc(dz, n, Hs, Ws, 64, 64, SLOTS, 2);
+  if (pool_dT) {
+    a.pool_dT = pool_dT;
+    a.pool_codes = pool_codes;
+    a.Hp = Hp;
+    a.Wp = Wp;
+    if (Wp + 1 > 64) throw ShapeError("stem_wgrad_pooled: pooled width must be < 64");
+    a.pt_map = make_tmap_nhwc_plain(pool_dT, n, Hp, Wp, 64, 64, 64, 2);  // row-major [2][64][64] in smem
+    a.pc_map = make_tmap_nhwc_u8(pool_codes, n, Hp, Wp, 64, 64, 64, 2);
+  } else {
+    a.dz_map = make_tmap_nhwc(dz, n, Hs, Ws, 64, 64, SLOTS, 2);
+  }
   a.n = n;
   a.Hs = Hs;
   a.Ws = Ws;

@@ -40,5 +40,9 @@ void stem_fwd(const bf16* s, const int* count, int n_static, int Hs, int Ws, con
 size_t stem_wgrad_ws_bytes(int n);
 void stem_wgrad(const bf16* s, const bf16* dz, int n, int Hs, int Ws, int cin_real, float* ws, size_t ws_bytes,
                 float* dw, float* db, cudaStream_t st);
+// same, with the stem's 3x3/2 max-pool backward fused in: dZ is built on chip from the pooled-output gradient
+// pool_dT [n][Hp][Wp][64] and the forward's argmax codes (ReLU mask folded in), never written to HBM
+void stem_wgrad_pooled(const bf16* s, const bf16* pool_dT, const uint8_t* pool_codes, int Hp, int Wp, int n, int Hs,
+                       int Ws, int cin_real, float* ws, size_t ws_bytes, float* dw, float* db, cudaStream_t st);
 
 }  // namespace adainf

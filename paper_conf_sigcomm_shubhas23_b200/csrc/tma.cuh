@@ -16,6 +16,8 @@ CUtensorMap make_tmap_nhwc(const void* base, int N, int H, int W, int C, int bc,
 CUtensorMap make_tmap_nhwc_plain(const void* base, int N, int H, int W, int C, int bc, int bw, int bh);
 // same with a chosen swizzle: swz in {0, 32, 64, 128} bytes (bc * 2 must not exceed it)
 CUtensorMap make_tmap_nhwc_swz(const void* base, int N, int H, int W, int C, int bc, int bw, int bh, int swz);
+// 4-D tiled map over a dense NHWC uint8 tensor, no swizzle (bc bytes per (w, h) position, a multiple of 16)
+CUtensorMap make_tmap_nhwc_u8(const void* base, int N, int H, int W, int C, int bc, int bw, int bh);
 // 2-D tiled map over a row-major [rows][cols] bf16 matrix (row pitch ld elements), box {bcols, brows}.
 CUtensorMap make_tmap_2d(const void* base, long long rows, int cols, int ld, int bcols, int brows);
 // im2col map over NHWC [N][H][W][C] bf16 (128B swizzle): one load = `pixels` consecutive GEMM rows (output
