@@ -322,12 +322,15 @@ def main():
     evs = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
     ev0.record(stream)
     evs[0].record(stream)
+    host_t = [time.perf_counter()]
     for i in range(args.steps):
         step_device(cnt_buf[i])
         evs[i + 1].record(stream)
+        host_t.append(time.perf_counter())
     ev1.record(stream)
     torch.cuda.synchronize()
     step_ms = [round(evs[i].elapsed_time(evs[i + 1]), 3) for i in range(args.steps)]
+    host_enqueue_ms = [round((host_t[i + 1] - host_t[i]) * 1e3, 3) for i in range(args.steps)]
     launches = B.launch_count() - l0
     barrier()
     clocks = clk.stop()
@@ -458,6 +461,7 @@ def main():
             "hbm_kernels": {"peak_gbs": hbm_gbs, "peak_kind": f"HBM copy ({peak_src})", "kernels": hbm_kernels},
             "gpu_launches": int(launches),
             "step_ms": step_ms,
+            "host_enqueue_ms": host_enqueue_ms,
             "clocks": clocks,
             "e2e": e2e,
             "cpu_baseline": cpu,

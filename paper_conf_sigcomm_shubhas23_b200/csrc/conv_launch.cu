@@ -572,8 +572,19 @@ __global__ void wgrad_reduce_kernel(const float* __restrict__ part, int S, int K
   for (int r = ty; r < 32; r += 8) {
     const int k = k0 + r, co = c0 + tx;
     float acc = 0.f;
-    if (k < Kconv && co < Cout)
-      for (int s = 0; s < S; ++s) acc += part[((long long)s * Kconv + k) * Cout + co];
+    if (k < Kconv && co < Cout) {  // eight independent loads in flight, summed in ascending split order
+      const float* pp = part + (long long)k * Cout + co;
+      const long long sstride = (long long)Kconv * Cout;
+      int s = 0;
+      for (; s + 8 <= S; s += 8) {
+        float v[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) v[u] = __ldg(pp + (s + u) * sstride);
+#pragma unroll
+        for (int u = 0; u < 8; ++u) acc += v[u];
+      }
+      for (; s < S; ++s) acc += __ldg(pp + s * sstride);
+    }
     tile[r][tx] = acc;
   }
   __syncthreads();
@@ -624,8 +635,17 @@ __global__ void __launch_bounds__(CS_THREADS) colsum_partial_kernel(const bf16* 
 __global__ void colsum_final_kernel(const float* __restrict__ part, int nb, int C, float* __restrict__ out) {
   const int c = blockIdx.x * blockDim.x + threadIdx.x;
   if (c >= C) return;
+  // eight independent loads in flight, summed in the same ascending order
   float acc = 0.f;
-  for (int b = 0; b < nb; ++b) acc += part[(long long)b * C + c];
+  int b = 0;
+  for (; b + 8 <= nb; b += 8) {
+    float v[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) v[u] = __ldg(part + (long long)(b + u) * C + c);
+#pragma unroll
+    for (int u = 0; u < 8; ++u) acc += v[u];
+  }
+  for (; b < nb; ++b) acc += __ldg(part + (long long)b * C + c);
   out[c] = acc;
 }
 static int colsum_blocks(long long P) { return (int)std::max(1LL, std::min<long long>((P + 63) / 64, 4LL * num_sms())); }

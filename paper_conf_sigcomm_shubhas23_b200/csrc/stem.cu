@@ -656,8 +656,16 @@ __global__ void stem_wgrad_finish_kernel(const float* __restrict__ part, int G, 
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
   if (idx >= 256 * 64) return;
   const int co = idx & 63, k = idx >> 6;
-  float acc = 0.f;
-  for (int g = 0; g < 2 * G; ++g) acc += __ldg(part + ((long long)g * 256 + k) * 64 + co);
+  float acc = 0.f;  // eight independent loads in flight, summed in ascending order
+  int g = 0;
+  for (; g + 8 <= 2 * G; g += 8) {
+    float v[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) v[u] = __ldg(part + ((long long)(g + u) * 256 + k) * 64 + co);
+#pragma unroll
+    for (int u = 0; u < 8; ++u) acc += v[u];
+  }
+  for (; g < 2 * G; ++g) acc += __ldg(part + ((long long)g * 256 + k) * 64 + co);
   const int t = k >> 4, ch = k & 15;
   const int bh = ch >> 3, bw = (ch >> 2) & 1, c = ch & 3;
   const int kh = 2 * (t / 4 - 2) + bh + 3, kw = 2 * (t % 4 - 2) + bw + 3;
@@ -666,7 +674,15 @@ __global__ void stem_wgrad_finish_kernel(const float* __restrict__ part, int G, 
 __global__ void stem_colsum_final_kernel(const float* __restrict__ part, int G, float* __restrict__ db) {
   const int c = threadIdx.x;
   float acc = 0.f;
-  for (int g = 0; g < G; ++g) acc += part[g * 64 + c];
+  int g = 0;
+  for (; g + 8 <= G; g += 8) {
+    float v[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) v[u] = __ldg(part + (g + u) * 64 + c);
+#pragma unroll
+    for (int u = 0; u < 8; ++u) acc += v[u];
+  }
+  for (; g < G; ++g) acc += __ldg(part + g * 64 + c);
   db[c] = acc;
 }
 
