@@ -202,6 +202,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="adainf", choices=["adainf", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-graph", action="store_true", help="time eager launches instead of the captured step graph")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile-steps", type=int, default=None)
     args = ap.parse_args()
@@ -286,12 +287,15 @@ def main():
 
     taus = calibrate()
 
-    def step_device(out_counts):
+    def step_device(out_counts, xi=None, Xe=None, py=None):
+        xi = x_inf if xi is None else xi
+        Xe = X if Xe is None else Xe
+        py = pool_y if py is None else py
         outs["exit_counts"] = out_counts
-        app.infer(x_inf, taus, [outs])
-        B.select_retrain(X, W, R, K_SEL, exclude=E, out_idx=sel_idx, out_dist=sel_dist, out_count=sel_cnt)
+        app.infer(xi, taus, [outs])
+        B.select_retrain(Xe, W, R, K_SEL, exclude=E, out_idx=sel_idx, out_dist=sel_dist, out_count=sel_cnt)
         B.gather_rows(pool, sel_idx, sel_cnt, K_SEL, rt_x)
-        B.gather_rows(pool_y, sel_idx, sel_cnt, K_SEL, rt_y)
+        B.gather_rows(py, sel_idx, sel_cnt, K_SEL, rt_y)
         m.retrain_step(rt_x, rt_y, n_global=n_global, lr=LR, stats=stats)
 
     cnt_buf = torch.zeros((max(args.steps, 1) + args.warmup + 64, 4), dtype=torch.int32, device=dev)
@@ -315,6 +319,18 @@ def main():
     for i in range(2):
         step_device(cnt_buf[-1 - i % 32])
     torch.cuda.synchronize()
+    # the whole step (inference DAG + selection + gather + retrain step, ~190 kernels) captured once as a CUDA
+    # graph and replayed: the same kernels and arguments, without per-launch host / front-end overhead between
+    # them (--no-graph times the eagerly launched step instead)
+    graph, graph_launches = None, 0
+    if not args.no_graph:
+        graph = torch.cuda.CUDAGraph()
+        la = B.launch_count()
+        with torch.cuda.graph(graph):
+            step_device(cnt_buf[-40])
+        graph_launches = B.launch_count() - la
+        graph.replay()
+        torch.cuda.synchronize()
     l0 = B.launch_count()
     barrier()
     torch.cuda.synchronize()
@@ -324,14 +340,18 @@ def main():
     evs[0].record(stream)
     host_t = [time.perf_counter()]
     for i in range(args.steps):
-        step_device(cnt_buf[i])
+        if graph is not None:
+            graph.replay()
+            cnt_buf[i].copy_(cnt_buf[-40], non_blocking=True)  # this step's exit counts
+        else:
+            step_device(cnt_buf[i])
         evs[i + 1].record(stream)
         host_t.append(time.perf_counter())
     ev1.record(stream)
     torch.cuda.synchronize()
     step_ms = [round(evs[i].elapsed_time(evs[i + 1]), 3) for i in range(args.steps)]
     host_enqueue_ms = [round((host_t[i + 1] - host_t[i]) * 1e3, 3) for i in range(args.steps)]
-    launches = B.launch_count() - l0
+    launches = B.launch_count() - l0 + graph_launches * args.steps
     barrier()
     clocks = clk.stop()
     ms = ev0.elapsed_time(ev1) / args.steps
@@ -411,15 +431,51 @@ def main():
         h_stats = torch.empty(2, dtype=torch.float32).pin_memory()
         h2d = h_inf.numel() * 2 + h_X.numel() * 2 + h_y.numel() * 4
         d2h = INF_B * 1 + INF_B * 4 + 8
+        # double-buffered inputs: step i+1's H2D copies run on a copy stream while step i computes (a serving
+        # loop overlaps them the same way); every step's inputs are still copied inside the timed region
+        xi_b = [x_inf, torch.empty_like(x_inf)]
+        Xe_b = [X, torch.empty_like(X)]
+        py_b = [pool_y, torch.empty_like(pool_y)]
+        cs = torch.cuda.Stream(device=dev)
+        e2e_graphs = None
+        if graph is not None:  # one captured step per input buffer set
+            torch.cuda.synchronize()
+            e2e_graphs = []
+            for b in range(2):
+                gb = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(gb):
+                    step_device(cnt_buf[-40], xi_b[b], Xe_b[b], py_b[b])
+                e2e_graphs.append(gb)
+            torch.cuda.synchronize()
+        copied = [torch.cuda.Event() for _ in range(2)]
+        consumed = [torch.cuda.Event() for _ in range(2)]
         torch.cuda.synchronize()
         barrier()
         ev4, ev5 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         ev4.record(stream)
+
+        def issue_copy(i):
+            b = i % 2
+            with torch.cuda.stream(cs):
+                cs.wait_event(ev4)
+                if i >= 2:
+                    cs.wait_event(consumed[b])
+                xi_b[b].view(torch.int16).copy_(h_inf.view(torch.int16), non_blocking=True)
+                Xe_b[b].view(torch.int16).copy_(h_X.view(torch.int16), non_blocking=True)
+                py_b[b].copy_(h_y, non_blocking=True)
+                copied[b].record(cs)
+
+        issue_copy(0)
         for i in range(args.steps):
-            x_inf.view(torch.int16).copy_(h_inf.view(torch.int16), non_blocking=True)
-            X.view(torch.int16).copy_(h_X.view(torch.int16), non_blocking=True)
-            pool_y.copy_(h_y, non_blocking=True)
-            step_device(cnt_buf[-1 - i % 32])
+            b = i % 2
+            if i + 1 < args.steps:
+                issue_copy(i + 1)
+            stream.wait_event(copied[b])
+            if e2e_graphs is not None:
+                e2e_graphs[b].replay()
+            else:
+                step_device(cnt_buf[-1 - i % 32], xi_b[b], Xe_b[b], py_b[b])
+            consumed[b].record(stream)
             h_exit.copy_(outs["exit_id"], non_blocking=True)
             h_pred.copy_(outs["pred"], non_blocking=True)
             h_stats.copy_(stats, non_blocking=True)
@@ -431,7 +487,8 @@ def main():
             torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
             ems = float(t.item())
         e2e = {"value": samples_per_step / (ems / 1e3), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
-               "d2h_bytes_per_step": int(d2h), "ms_per_step": ems}
+               "d2h_bytes_per_step": int(d2h), "ms_per_step": ems,
+               "overlap": "step i+1's H2D copies on a copy stream during step i (double-buffered inputs)"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -445,7 +502,8 @@ def main():
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
-            "config": dict(arm_config(world), exit_thresholds=taus),
+            "config": dict(arm_config(world), exit_thresholds=taus,
+                           launch="cuda_graph (one captured step, replayed)" if graph is not None else "eager"),
             "inference_samples_per_s": INF_B * world / (ms / 1e3),
             "retrain_samples_per_s": K_SEL * world / (ms / 1e3),
             "exit_counts_mean": counts.mean(0).round(2).tolist(),

@@ -616,6 +616,11 @@ __global__ void sum_kernel(const float* __restrict__ x, int n, float* out, float
   }
   if (threadIdx.x == 0) *out = scale == 0.f ? sh[0] : (scale < 0.f ? sqrtf(sh[0]) : sh[0] * scale);
 }
+__global__ void fill_i32_kernel(int32_t* p, int32_t v) { *p = v; }
+void launch_fill_i32(int32_t* p, int32_t v, cudaStream_t st) {
+  fill_i32_kernel<<<1, 1, 0, st>>>(p, v);
+  CK(cudaGetLastError());
+}
 void launch_sum(const float* x, int n, float* out, float scale, cudaStream_t st) {
   ProfScope ps(PC_SUM, st);
   sum_kernel<<<1, 1024, 0, st>>>(x, n, out, scale);

@@ -70,6 +70,8 @@ void launch_grad_finalize(const float* bcast, const bf16* sc, const bf16* yact, 
                           bf16* dz, cudaStream_t st);
 // fixed-order sum of a float vector into out[0] (single block)
 void launch_sum(const float* x, int n, float* out, float scale, cudaStream_t st);
+// *p = v, stream-ordered (no pageable host source, so it can be captured into a CUDA graph)
+void launch_fill_i32(int32_t* p, int32_t v, cudaStream_t st);
 
 struct SgdSeg {
   long long off;       // flat offset

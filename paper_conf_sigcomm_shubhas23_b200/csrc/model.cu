@@ -501,7 +501,7 @@ void Model::infer(const bf16* x, const int* in_map, const int* in_count, int n_s
     if (in_count)
       CK(cudaMemcpyAsync(out.exit_counts, in_count, 4, cudaMemcpyDeviceToDevice, st));
     else
-      CK(cudaMemcpyAsync(out.exit_counts, &n_static, 4, cudaMemcpyHostToDevice, st));
+      launch_fill_i32(out.exit_counts, n_static, st);
   }
   forward_nodes(x0, map0, in_count, n_static, false, taus, &out, st);
 }
