@@ -84,16 +84,20 @@ struct ConvArgs {
 };
 
 constexpr int BM = 128, BK = 64;
-constexpr int NUM_THREADS = 288;  // 4 producer warps, 1 MMA warp, 4 epilogue warps
+constexpr int NUM_THREADS = 288;  // 4 producer warps, 1 MMA warp, 4 epilogue warps (window / wgrad kernels)
+// conv_umma_kernel<.., EW>: 4 producer warps, 1 MMA warp, 4*EW epilogue warps.  EW = 2 (two warps per TMEM lane
+// quadrant, alternating 64-column blocks) for epilogue-heavy short-K launches, which one epilogue warp per
+// quadrant would bound; EW = 1 keeps more smem stages and registers for long-K launches
+__host__ __device__ constexpr int gemm_threads(int EW) { return 160 + 128 * EW; }
 
-template <int MODE, int BN>
+template <int MODE, int BN, int EW = 1>
 struct ConvCfg {
   static constexpr int A_BYTES = BM * BK * 2;
   static constexpr int B_BYTES = BN * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   // coalescing buffers of the bf16 epilogue: 4 warps x 2 operands x (32 rows x 128 B), double-buffered in
   // the sub-pixel dgrad mode
-  static constexpr int EPI_BYTES = (MODE != 2 && BN >= 64) ? (MODE == 3 ? 4 * 16384 : 4 * 8192) : 0;
+  static constexpr int EPI_BYTES = (MODE != 2 && BN >= 64) ? (MODE == 3 && EW == 1 ? 4 * 16384 : 4 * EW * 8192) : 0;
   static constexpr int STAGES_FIT = (220 * 1024 - EPI_BYTES - 1280) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_FIT > 8 ? 8 : STAGES_FIT;
   static constexpr int BIAS_BYTES = (MODE == 0 && EPI_BYTES > 0) ? 4096 : 0;  // FWD bias vector (Nout <= 1024)
@@ -233,12 +237,23 @@ __device__ __forceinline__ EpiBlk epi_block(const ConvArgs& a, int cb, long long
 // into per-warp buffers; in the sub-pixel mode (short K, epilogue-heavy tiles) they are double-buffered: the
 // first block's operands are requested before waiting for the accumulator, block c+1's while block c is
 // combined, so the epilogue does not pay a memory latency per column block.
-template <int MODE, int BN>
+template <int MODE, int BN, int EW>
 __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const TileInfo& ti, uint32_t trow,
                                                    uint64_t* tfull_b, uint32_t tpar, uint64_t* tempty_b, int nkb,
                                                    long long m, bool rv, int n, long long orow, long long rrow,
-                                                   int HWg, uint8_t* stg, int lane, const float* bias_s) {
-  constexpr bool PIPE = MODE == MODE_DGRAD_SP;
+                                                   int HWg, uint8_t* stg, int lane, const float* bias_s, int h) {
+  // EW warps per lane quadrant: this warp takes column blocks h*64, h*64 + 64*EW, ...; with two warps the
+  // staging is single-buffered (the other warp of the quadrant overlaps its latency)
+  constexpr bool PIPE = MODE == MODE_DGRAD_SP && EW == 1;
+  constexpr int STEP = 64 * EW;
+  const int first = h * 64;
+  if (first >= BN) {  // no block for this warp: release the accumulator in order
+    mbar_wait(tfull_b, tpar);
+    tc_fence_after();
+    tc_fence_before();
+    mbar_arrive(tempty_b);
+    return;
+  }
   int gy = 0, gx = 0;
   if (MODE == MODE_DGRAD_SP && rv) {
     const int pix = (int)m - n * HWg;
@@ -263,19 +278,19 @@ __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const Tile
     const bf16* p1 = MODE == MODE_FWD ? nullptr : (ma ? a.yact : nullptr);
     const long long r0 = MODE == MODE_FWD ? rrow : orow;
 #pragma unroll 1
-    for (int c = 64; c < BN; c += 64) {
+    for (int c = first + STEP; c < BN; c += STEP) {
       if (ti.n0 + c >= a.Nout) break;
       if (p0) prefetch_l2(p0 + r0 * a.Nout + ti.n0 + c);
       if (p1) prefetch_l2(p1 + orow * a.Nout + ti.n0 + c);
     }
   }
-  EpiBlk cur = epi_block<MODE>(a, ti.n0, m, rv, n, orow, gy, gx);
+  EpiBlk cur = epi_block<MODE>(a, ti.n0 + first, m, rv, n, orow, gy, gx);
   if (PIPE) issue(cur, 0);
   mbar_wait(tfull_b, tpar);
   tc_fence_after();
   int it = 0;
 #pragma unroll 1
-  for (int c0 = 0; c0 < BN; c0 += 64, ++it) {
+  for (int c0 = first; c0 < BN; c0 += STEP, ++it) {
     float v[64];
     if (nkb > 0) {
       tmem_ld32(trow + c0, v);
@@ -284,18 +299,18 @@ __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const Tile
 #pragma unroll
       for (int i = 0; i < 64; ++i) v[i] = 0.f;
     }
-    if (c0 + 64 >= BN) {
+    if (c0 + STEP >= BN) {
       tc_fence_before();
       mbar_arrive(tempty_b);  // accumulator free for the tile after next
     }
     const int cb = ti.n0 + c0;
     if (cb >= a.Nout) continue;  // warp-uniform (Nout % 64 == 0); keep looping: the last block frees the accumulator
-    const bool has_next = c0 + 64 < BN && cb + 64 < a.Nout;
+    const bool has_next = c0 + STEP < BN && cb + STEP < a.Nout;
     if (!PIPE) cur = epi_block<MODE>(a, cb, m, rv, n, orow, gy, gx);
     EpiBlk nxt = cur;
     if (PIPE) {
       if (has_next) {
-        nxt = epi_block<MODE>(a, cb + 64, m, rv, n, orow, gy, gx);
+        nxt = epi_block<MODE>(a, cb + STEP, m, rv, n, orow, gy, gx);
         issue(nxt, (it + 1) & 1);
         asm volatile("cp.async.wait_group 1;" ::: "memory");
       } else {
@@ -366,9 +381,9 @@ __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const Tile
   }
 }
 
-template <int MODE, int BN>
-__global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_constant__ ConvArgs a) {
-  using Cfg = ConvCfg<MODE, BN>;
+template <int MODE, int BN, int EW>
+__global__ void __launch_bounds__(gemm_threads(EW), 1) conv_umma_kernel(const __grid_constant__ ConvArgs a) {
+  using Cfg = ConvCfg<MODE, BN, EW>;
   static_assert(ModeTraits<MODE>::B_KMAJ || BN >= 64, "MN-major SW128 B tiles need >= 64 columns");
   constexpr int STAGES = Cfg::STAGES;
   extern __shared__ uint8_t smem_raw[];
@@ -382,7 +397,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
   float* bias_s = nullptr;  // FWD: the layer's bias vector, staged once per CTA
   if (Cfg::BIAS_BYTES > 0 && a.bias && a.Nout <= Cfg::BIAS_BYTES / 4) {
     bias_s = (float*)(epi_smem + Cfg::EPI_BYTES);
-    for (int i = threadIdx.x; i < a.Nout; i += NUM_THREADS) bias_s[i] = __ldg(a.bias + i);
+    for (int i = threadIdx.x; i < a.Nout; i += gemm_threads(EW)) bias_s[i] = __ldg(a.bias + i);
   }
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -403,7 +418,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&tfull[b], 1);
-      mbar_init(&tempty[b], 128);
+      mbar_init(&tempty[b], 128 * EW);
     }
     fence_mbar_init();
   }
@@ -671,6 +686,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
   } else {
     // ================= epilogue =================
     const int q = warp & 3;  // TMEM lane quadrant of this warp
+    const int h = (warp - 5) >> 2;  // which of the quadrant's two epilogue warps
     const int row = q * 32 + lane;
     int lt = 0;
     for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++lt) {
@@ -688,14 +704,18 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
       const long long m = ti.m0 + row;
       if (MODE == MODE_WGRAD) {
         float* outp = (float*)a.out + ((long long)ti.z * a.K + m) * a.Nout + ti.n0;
+        if (h * 32 >= BN) {  // no chunk for this warp
+          tc_fence_before();
+          mbar_arrive(&tempty[b]);
+        }
 #pragma unroll 1
-        for (int c0 = 0; c0 < BN; c0 += 32) {
+        for (int c0 = h * 32; c0 < BN; c0 += 32 * EW) {
           float v[32];
           if (nkb > 0) tmem_ld32(trow + c0, v);
           else
 #pragma unroll
             for (int i = 0; i < 32; ++i) v[i] = 0.f;
-          if (c0 + 32 >= BN) {
+          if (c0 + 32 * EW >= BN) {
             tc_fence_before();
             mbar_arrive(&tempty[b]);
           }
@@ -725,19 +745,23 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_umma_kernel(const __grid_
         }
         if constexpr (Cfg::EPI_BYTES > 0) {
           if (coalesced) {
-            epilogue_coalesced<MODE, BN>(a, ti, trow, &tfull[b], ub & 1, &tempty[b], nkb, m, rv, n, orow, rrow,
-                                          HWg, epi_smem + q * (Cfg::EPI_BYTES / 4), lane, bias_s);
+            epilogue_coalesced<MODE, BN, EW>(a, ti, trow, &tfull[b], ub & 1, &tempty[b], nkb, m, rv, n, orow, rrow,
+                                          HWg, epi_smem + (warp - 5) * (Cfg::EPI_BYTES / (4 * EW)), lane, bias_s, h);
             continue;
           }
         }
+        if (h * 32 >= BN) {  // no chunk for this warp
+          tc_fence_before();
+          mbar_arrive(&tempty[b]);
+        }
 #pragma unroll 1
-        for (int c0 = 0; c0 < BN; c0 += 32) {
+        for (int c0 = h * 32; c0 < BN; c0 += 32 * EW) {
           float v[32];
           if (nkb > 0) tmem_ld32(trow + c0, v);
           else
 #pragma unroll
             for (int i = 0; i < 32; ++i) v[i] = 0.f;
-          if (c0 + 32 >= BN) {
+          if (c0 + 32 * EW >= BN) {
             tc_fence_before();
             mbar_arrive(&tempty[b]);  // accumulator free for the tile after next
           }

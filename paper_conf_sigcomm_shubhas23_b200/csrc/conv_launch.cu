@@ -26,18 +26,32 @@ int num_sms() {
 }
 
 // persistent launch: one CTA per SM (or fewer when there are fewer tiles)
-template <int MODE, int BN>
-static void launch_t(const ConvArgs& a, long long max_tiles, cudaStream_t st) {
+template <int MODE, int BN, int EW>
+static void launch_t_ew(const ConvArgs& a, long long max_tiles, cudaStream_t st) {
   dim3 grid((unsigned)std::max(1LL, std::min<long long>(max_tiles, num_sms())));
-  using Cfg = ConvCfg<MODE, BN>;
+  using Cfg = ConvCfg<MODE, BN, EW>;
   static bool attr = false;
   if (!attr) {
-    CK(cudaFuncSetAttribute(conv_umma_kernel<MODE, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
+    CK(cudaFuncSetAttribute(conv_umma_kernel<MODE, BN, EW>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
     attr = true;
   }
   ProfScope ps(MODE == MODE_FWD ? PC_CONV_FWD : (ModeTraits<MODE>::DG_EPI ? PC_CONV_DGRAD : PC_CONV_WGRAD), st);
-  conv_umma_kernel<MODE, BN><<<grid, NUM_THREADS, Cfg::SMEM, st>>>(a);
+  conv_umma_kernel<MODE, BN, EW><<<grid, gemm_threads(EW), Cfg::SMEM, st>>>(a);
   CK(cudaGetLastError());
+}
+// persistent launch: one CTA per SM (or fewer when there are fewer tiles).  Short-K forward tiles (<= 4
+// K-blocks: the 1x1 projections) are epilogue-bound: they get two epilogue warps per TMEM lane quadrant.
+template <int MODE, int BN>
+static void launch_t(const ConvArgs& a, long long max_tiles, cudaStream_t st) {
+  // (measured: the dgrad modes lose more to the 128-register cap of the wider CTA than they gain)
+  const bool wide_epi = MODE == MODE_FWD && BN >= 64 && a.K <= 4 * BK;
+  if constexpr (MODE == MODE_FWD && BN >= 64) {
+    if (wide_epi) {
+      launch_t_ew<MODE, BN, 2>(a, max_tiles, st);
+      return;
+    }
+  }
+  launch_t_ew<MODE, BN, 1>(a, max_tiles, st);
 }
 
 template <int MODE>

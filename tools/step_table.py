@@ -6,7 +6,10 @@ rows = list(csv.DictReader(io.StringIO("\n".join(lines[i:]))))
 per = collections.OrderedDict()
 for r in rows:
     key = (int(r['ID']), r['Kernel Name'][:38], r['Grid Size'])
-    per.setdefault(key, {})[r['Metric Name']] = float(r['Metric Value'].replace(',', '') or 0)
+    try:
+        per.setdefault(key, {})[r['Metric Name']] = float(r['Metric Value'].replace(',', '') or 0)
+    except ValueError:
+        per.setdefault(key, {})
 ids = sorted(set(k[0] for k in per))
 lo = int(sys.argv[2]) if len(sys.argv) > 2 else 0
 tot = 0
