@@ -28,6 +28,21 @@ __global__ void pack_s2d_kernel(const bf16* __restrict__ x, const int* __restric
     const int rem = (int)(i - n * Hs * Ws);
     const int si = rem / Ws, sj = rem - si * Ws;
     const long long src = map ? map[n] : n;
+    if (cin == 3) {
+      // the two pixels of one input row are 12 contiguous, 4-byte aligned bytes (W even): three 32-bit loads
+      // per row; channel 3 of each pixel is the zero pad
+      uint4 o2[2];
+#pragma unroll
+      for (int bh = 0; bh < 2; ++bh) {
+        const uint32_t* pw = (const uint32_t*)(x + ((src * H + 2 * si + bh) * W + 2 * sj) * 3);
+        const uint32_t w0 = __ldg(pw), w1 = __ldg(pw + 1), w2 = __ldg(pw + 2);
+        o2[bh] = make_uint4(w0, w1 & 0xFFFFu, (w1 >> 16) | (w2 << 16), w2 >> 16);
+      }
+      uint4* o = (uint4*)(s + i * 16);
+      o[0] = o2[0];
+      o[1] = o2[1];
+      continue;
+    }
     __align__(16) bf16 v[16];
 #pragma unroll
     for (int bh = 0; bh < 2; ++bh)
