@@ -324,13 +324,19 @@ def main():
     # them (--no-graph times the eagerly launched step instead)
     graph, graph_launches = None, 0
     if not args.no_graph:
-        graph = torch.cuda.CUDAGraph()
-        la = B.launch_count()
-        with torch.cuda.graph(graph):
-            step_device(cnt_buf[-40])
-        graph_launches = B.launch_count() - la
-        graph.replay()
-        torch.cuda.synchronize()
+        try:
+            graph = torch.cuda.CUDAGraph()
+            la = B.launch_count()
+            with torch.cuda.graph(graph):
+                step_device(cnt_buf[-40])
+            graph_launches = B.launch_count() - la
+            graph.replay()
+            torch.cuda.synchronize()
+        except Exception as ex:  # capture unsupported here (e.g. a collective): time eager launches
+            print(f"[bench] graph capture failed ({type(ex).__name__}: {ex}); timing eager launches",
+                  file=sys.stderr)
+            graph, graph_launches = None, 0
+            torch.cuda.synchronize()
     l0 = B.launch_count()
     barrier()
     torch.cuda.synchronize()
