@@ -683,6 +683,7 @@ struct WgPlan {
   int S, kbs, nkb, Kconv, tiles;
   int BN;          // WG_TMA / WG_GENERIC
   int Wp, R, rg;   // TMA paths
+  int i2c;         // WG_TMA: K-blocks of 64 consecutive output pixels via im2col TMA
 };
 
 static bool win_wgrad_ok(const ConvGeom& g) {
@@ -697,6 +698,17 @@ static bool win_tma_wgrad_ok(const ConvGeom& g) {
 }
 static bool wgrad_tma_ok(const ConvGeom& g) {
   return tma_wgrad_allowed() && g.Cin % 64 == 0 && g.Cout % 64 == 0 && g.Wo <= 64 && g.stride <= 2;
+}
+
+// im2col TMA for the weight-gradient A operand (ADAINF_WG_I2C=0: padded-pitch boxes)
+static bool wgrad_i2c_ok(const ConvGeom& g) {
+  static int env = -1;
+  if (env < 0) {
+    const char* e = getenv("ADAINF_WG_I2C");
+    env = e ? atoi(e) : 1;
+  }
+  const int lo = -g.pad, up = lo + (g.Ho - 1) * g.stride - (g.H - 1);
+  return env && atma_on() && g.H == g.W && g.Ho == g.Wo && g.KH == g.KW && lo >= -128 && up >= -128 && up <= 127;
 }
 
 static void finish_splits(WgPlan& p) {
@@ -745,6 +757,10 @@ static WgPlan plan_wgrad(const ConvGeom& g, int n) {
     p.R = 64 / Wp;
     p.rg = (g.Ho + p.R - 1) / p.R;
     p.nkb = n * p.rg;
+    if (wgrad_i2c_ok(g)) {  // K-blocks of 64 consecutive output pixels: no pitch padding
+      p.i2c = 1;
+      p.nkb = (int)(((long long)n * g.Ho * g.Wo + 63) / 64);
+    }
     p.BN = g.Cout <= 64 ? 64 : (g.Cout <= 128 ? 128 : 256);
     p.tiles = ((p.Kconv + 127) / 128) * ((g.Cout + p.BN - 1) / p.BN);
     finish_splits(p);
@@ -867,8 +883,18 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
     a.splits = S;
     a.out = ws;
     a.cs_part = fused_cs ? cs_part : nullptr;
-    a.x_map = make_tmap_nhwc(x, n, g.H, g.W, g.Cin, 64, p.Wp, p.R, g.stride);
-    a.dz_map = make_tmap_nhwc(dz, n, g.Ho, g.Wo, g.Cout, 64, p.Wp, p.R, 1);
+    if (p.i2c) {
+      a.i2c = 1;
+      a.lo = -g.pad;
+      a.n = p.nkb;  // K-blocks (rg = 1)
+      a.rg = 1;
+      a.x_map = make_tmap_im2col(x, n, g.H, g.W, g.Cin, -g.pad, -g.pad + (g.Ho - 1) * g.stride - (g.H - 1), g.stride,
+                                 64, 64);
+      a.dz_map = make_tmap_2d(dz, (long long)n * g.Ho * g.Wo, g.Cout, g.Cout, 64, 64);
+    } else {
+      a.x_map = make_tmap_nhwc(x, n, g.H, g.W, g.Cin, 64, p.Wp, p.R, g.stride);
+      a.dz_map = make_tmap_nhwc(dz, n, g.Ho, g.Wo, g.Cout, 64, p.Wp, p.R, 1);
+    }
     if (p.BN == 64) launch_wgrad_tma_t<64>(a, st);
     else if (p.BN == 128) launch_wgrad_tma_t<128>(a, st);
     else launch_wgrad_tma_t<256>(a, st);

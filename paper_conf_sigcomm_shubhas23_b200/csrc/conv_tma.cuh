@@ -522,6 +522,10 @@ struct WgTmaArgs {
   float* out;           // partials [split][Kconv][Cout]
   float* cs_part;       // bias-gradient partials [split][Cout] (nullptr: not fused)
   int stages;
+  // i2c = 1: K-blocks are 64 consecutive output pixels (no pitch padding): x_map is an im2col map (64 pixels x
+  // 64 channels per load, base pixel = output position * stride + lo, tap offsets (kw, kh)), dz_map a 2-D map
+  // over dZ as [n*Ho*Wo][Cout] with box {64 co, 64 pixels}; n = #K-blocks and rg = 1 so nkb = n * rg
+  int i2c, lo;
 };
 
 template <int BN>
@@ -582,10 +586,22 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
         for (int kb = kb0; kb < kb1; ++kb, ++it) {
           const int s = it % ST, u = it / ST;
           if (u > 0) mbar_wait(&empty[s], (u - 1) & 1);
-          const int img = kb / a.rg, h0 = (kb - img * a.rg) * a.Rk;
           const uint32_t sa = sbase + s * STAGE, sb = sa + A_BYTES;
           const int nA = av[1] ? 2 : 1;
           mbar_expect_tx(&full[s], nA * 8192 + (BN / 64) * 8192);
+          if (a.i2c) {
+            const int p0 = kb * 64, HWo = a.Ho * a.Wo;
+            const int n0 = p0 / HWo, rem = p0 - n0 * HWo;
+            const int oy = rem / a.Wo, ox = rem - oy * a.Wo;
+            const int bw = ox * a.stride + a.lo, bh = oy * a.stride + a.lo;
+            for (int i = 0; i < nA; ++i)
+              tma_load_im2col_4d(sa + i * 8192, &a.x_map, &full[s], ac[i], bw, bh, n0, (uint16_t)(ax[i] - a.lo),
+                                 (uint16_t)(ay[i] - a.lo));
+#pragma unroll
+            for (int j = 0; j < BN / 64; ++j) tma_load_2d(sb + j * 8192, &a.dz_map, &full[s], nb * BN + j * 64, p0);
+            continue;
+          }
+          const int img = kb / a.rg, h0 = (kb - img * a.rg) * a.Rk;
           for (int i = 0; i < nA; ++i)
             tma_load_4d(sa + i * 8192, &a.x_map, &full[s], ac[i], ax[i], h0 * a.stride + ay[i], img);
 #pragma unroll
