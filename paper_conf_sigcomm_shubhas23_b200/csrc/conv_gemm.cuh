@@ -241,7 +241,13 @@ template <int MODE, int BN, int EW>
 __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const TileInfo& ti, uint32_t trow,
                                                    uint64_t* tfull_b, uint32_t tpar, uint64_t* tempty_b, int nkb,
                                                    long long m, bool rv, int n, long long orow, long long rrow,
-                                                   int HWg, uint8_t* stg, int lane, const float* bias_s, int h) {
+                                                   int HWg, uint8_t* stg, int lane, const float* bias_s, int h,
+                                                   uint32_t tempty_remote = 0) {
+  // tempty_remote != 0: the accumulator-free arrival goes to the pair leader's barrier (CTA-pair kernel)
+  auto release = [&]() {
+    if (tempty_remote) mbar_arrive_cluster(tempty_remote);
+    else mbar_arrive(tempty_b);
+  };
   // EW warps per lane quadrant: this warp takes column blocks h*64, h*64 + 64*EW, ...; with two warps the
   // staging is single-buffered (the other warp of the quadrant overlaps its latency)
   constexpr bool PIPE = MODE == MODE_DGRAD_SP && EW == 1;
@@ -251,7 +257,7 @@ __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const Tile
     mbar_wait(tfull_b, tpar);
     tc_fence_after();
     tc_fence_before();
-    mbar_arrive(tempty_b);
+    release();
     return;
   }
   int gy = 0, gx = 0;
@@ -301,7 +307,7 @@ __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const Tile
     }
     if (c0 + STEP >= BN) {
       tc_fence_before();
-      mbar_arrive(tempty_b);  // accumulator free for the tile after next
+      release();  // accumulator free for the tile after next
     }
     const int cb = ti.n0 + c0;
     if (cb >= a.Nout) continue;  // warp-uniform (Nout % 64 == 0); keep looping: the last block frees the accumulator

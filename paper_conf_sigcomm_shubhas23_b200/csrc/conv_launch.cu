@@ -9,6 +9,7 @@
 #include "conv_gemm.cuh"
 #include "conv_win.cuh"
 #include "conv_tma.cuh"
+#include "conv_pair.cuh"
 #include "prof.h"
 #include "runtime.h"
 
@@ -52,6 +53,52 @@ static void launch_t(const ConvArgs& a, long long max_tiles, cudaStream_t st) {
     }
   }
   launch_t_ew<MODE, BN, 1>(a, max_tiles, st);
+}
+
+// ---- CTA-pair kernel (cta_group::2, M = 256 tiles) ----
+// Off by default (ADAINF_PAIR=1 enables): it is parity-green but measured ~2x slower than the single-CTA kernel
+// on ResNet layer 2 (the peer's per-stage completion forwarding and remote epilogue releases are cluster-scope
+// release operations on the critical path); see DESIGN.md section 11.
+static int g_pair = -1;
+static bool pair_on() {
+  if (g_pair < 0) {
+    const char* e = getenv("ADAINF_PAIR");
+    g_pair = e ? atoi(e) : 0;
+  }
+  return g_pair != 0;
+}
+template <int MODE, int BN>
+static void launch_pair_t(const ConvArgs& a, long long pair_tiles, cudaStream_t st) {
+  using Cfg = PairCfg<MODE, BN>;
+  static bool attr = false;
+  if (!attr) {
+    CK(cudaFuncSetAttribute(conv_pair_kernel<MODE, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
+    attr = true;
+  }
+  const long long pairs = std::max(1LL, std::min<long long>(pair_tiles, num_sms() / 2));
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(2 * pairs));
+  cfg.blockDim = dim3(NUM_THREADS);
+  cfg.dynamicSmemBytes = Cfg::SMEM;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = 2;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  ProfScope ps(MODE == MODE_FWD ? PC_CONV_FWD : PC_CONV_DGRAD, st);
+  CK(cudaLaunchKernelEx(&cfg, conv_pair_kernel<MODE, BN>, a));
+}
+// pair launch when eligible: all-TMA operands, BN in {128, 256}; returns false otherwise
+template <int MODE>
+static bool try_launch_pair(int BN, const ConvArgs& a, long long npix_static, cudaStream_t st) {
+  if (!pair_on() || !a.a_tma || !a.b_tma || (BN != 128 && BN != 256)) return false;
+  const long long pt = ((npix_static + 2 * BM - 1) / (2 * BM)) * ((a.Nout + BN - 1) / BN);
+  if (BN == 128) launch_pair_t<MODE, 128>(a, pt, st);
+  else launch_pair_t<MODE, 256>(a, pt, st);
+  return true;
 }
 
 template <int MODE>
@@ -387,6 +434,10 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
     a.b_tma = 1;
     a.b_map = make_tmap_2d(w, g.Cout, a.K, ldb, 64, BN);  // K-major [Cout][K]; k >= K and rows >= Cout read 0
     try_a_tma(a);
+    if (a.a_tma && pair_on() && (BN == 128 || BN == 256) && a.K > 4 * BK) {
+      a.b_map = make_tmap_2d(w, g.Cout, a.K, ldb, 64, BN / 2);  // each CTA of the pair loads half the N rows
+      if (try_launch_pair<MODE_FWD>(BN, a, (long long)n_static * g.Ho * g.Wo, st)) return;
+    }
   }
   launch_bn<MODE_FWD>(BN, a, mt * ((g.Cout + BN - 1) / BN), st);
 }
@@ -477,6 +528,7 @@ void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n
         a.b_tma = 1;
         a.b_map = make_tmap_2d(w, g.Cout, ldb, ldb, 64, 64);  // rows co, cols (tap, ci): MN-major boxes
         try_a_tma(a);
+        if (s == 1 && a.K > 4 * BK && try_launch_pair<MODE_DGRAD>(BN, a, (long long)n * a.Hg * a.Wg, st)) continue;
       }
       launch_bn<MODE_DGRAD>(BN, a, mt * ((g.Cin + BN - 1) / BN), st);
     }

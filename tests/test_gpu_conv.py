@@ -215,3 +215,34 @@ def test_window_wgrad(case, mode):
         assert _rel(db, dz.float().sum(dim=(0, 1, 2))) < 1e-5
     finally:
         B.dbg_set_win_mode(1)
+
+
+@pytest.mark.parametrize("H,C,Co", [(28, 128, 128), (14, 256, 256)])
+def test_pair_kernel_fwd_dgrad_vs_single(H, C, Co, monkeypatch):
+    """CTA-pair (tcgen05.mma.cta_group::2, M = 256) kernel: bit-identical to the single-CTA kernel's output
+    (same K order per row), for forward and stride-1 dgrad (opt-in path, ADAINF_PAIR)."""
+    import subprocess, sys, os, json
+    code = f"""
+import json, os, sys, torch
+sys.path.insert(0, {os.path.dirname(os.path.dirname(os.path.abspath(__file__)))!r})
+from paper_conf_sigcomm_shubhas23_b200 import binding as B
+torch.manual_seed(0)
+n = 6
+x = torch.randn(n, {H}, {H}, {C}, device="cuda").to(torch.bfloat16)
+w = (torch.randn({Co}, 3, 3, {C}, device="cuda") * 0.05).to(torch.bfloat16)
+b = torch.randn({Co}, device="cuda") * 0.1
+dz = torch.randn(n, {H}, {H}, {Co}, device="cuda").to(torch.bfloat16)
+y = B.dbg_conv_fwd(x, w, b, 1, 1, act=1)
+dx = B.dbg_conv_dgrad(dz, w, {H}, {H}, 1, 1)
+torch.cuda.synchronize()
+torch.save({{"y": y.cpu(), "dx": dx.cpu()}}, sys.argv[1])
+"""
+    outs = []
+    for pair in ("0", "1"):
+        path = f"/tmp/pair_{pair}_{H}.pt"
+        env = dict(os.environ, ADAINF_PAIR=pair, ADAINF_WIN="4")
+        r = subprocess.run([sys.executable, "-c", code, path], env=env, capture_output=True, text=True, timeout=300)
+        assert r.returncode == 0, r.stderr[-2000:]
+        outs.append(torch.load(path))
+    assert torch.equal(outs[0]["y"], outs[1]["y"])
+    assert torch.equal(outs[0]["dx"], outs[1]["dx"])
