@@ -10,6 +10,7 @@
 #include "conv_win.cuh"
 #include "conv_tma.cuh"
 #include "conv_pair.cuh"
+#include "conv_dualm.cuh"
 #include "prof.h"
 #include "runtime.h"
 
@@ -98,6 +99,32 @@ static bool try_launch_pair(int BN, const ConvArgs& a, long long npix_static, cu
   const long long pt = ((npix_static + 2 * BM - 1) / (2 * BM)) * ((a.Nout + BN - 1) / BN);
   if (BN == 128) launch_pair_t<MODE, 128>(a, pt, st);
   else launch_pair_t<MODE, 256>(a, pt, st);
+  return true;
+}
+
+// ---- dual-M kernel (two 128-row tiles share each weight tile; ADAINF_DUALM=0 disables) ----
+static int g_dualm = -1;
+static bool dualm_on() {
+  if (g_dualm < 0) {
+    const char* e = getenv("ADAINF_DUALM");
+    g_dualm = e ? atoi(e) : 1;
+  }
+  return g_dualm != 0;
+}
+template <int MODE>
+static bool try_launch_dualm(int BN, const ConvArgs& a, long long npix_static, cudaStream_t st) {
+  if (!dualm_on() || !a.a_tma || !a.b_tma || BN != 128 || a.K <= 4 * BK) return false;
+  using Cfg = DualMCfg<MODE>;
+  static bool attr = false;
+  if (!attr) {
+    CK(cudaFuncSetAttribute(conv_dualm_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
+    attr = true;
+  }
+  const long long tiles = ((npix_static + 2 * BM - 1) / (2 * BM)) * ((a.Nout + BN - 1) / BN);
+  dim3 grid((unsigned)std::max(1LL, std::min<long long>(tiles, num_sms())));
+  ProfScope ps(MODE == MODE_FWD ? PC_CONV_FWD : PC_CONV_DGRAD, st);
+  conv_dualm_kernel<MODE><<<grid, DUALM_THREADS, Cfg::SMEM, st>>>(a);
+  CK(cudaGetLastError());
   return true;
 }
 
@@ -434,6 +461,7 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
     a.b_tma = 1;
     a.b_map = make_tmap_2d(w, g.Cout, a.K, ldb, 64, BN);  // K-major [Cout][K]; k >= K and rows >= Cout read 0
     try_a_tma(a);
+    if (try_launch_dualm<MODE_FWD>(BN, a, (long long)n_static * g.Ho * g.Wo, st)) return;
     if (a.a_tma && pair_on() && (BN == 128 || BN == 256) && a.K > 4 * BK) {
       a.b_map = make_tmap_2d(w, g.Cout, a.K, ldb, 64, BN / 2);  // each CTA of the pair loads half the N rows
       if (try_launch_pair<MODE_FWD>(BN, a, (long long)n_static * g.Ho * g.Wo, st)) return;
@@ -528,6 +556,7 @@ void conv_dgrad(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, int n
         a.b_tma = 1;
         a.b_map = make_tmap_2d(w, g.Cout, ldb, ldb, 64, 64);  // rows co, cols (tap, ci): MN-major boxes
         try_a_tma(a);
+        if (s == 1 && try_launch_dualm<MODE_DGRAD>(BN, a, (long long)n * a.Hg * a.Wg, st)) continue;
         if (s == 1 && a.K > 4 * BK && try_launch_pair<MODE_DGRAD>(BN, a, (long long)n * a.Hg * a.Wg, st)) continue;
       }
       launch_bn<MODE_DGRAD>(BN, a, mt * ((g.Cin + BN - 1) / BN), st);
