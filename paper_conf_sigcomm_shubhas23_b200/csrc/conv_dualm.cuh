@@ -11,9 +11,12 @@ namespace adainf {
 
 constexpr int DUALM_THREADS = 416;
 
-template <int MODE>
+// BN = 128: accumulators double-buffered (4 x 128 TMEM columns); BN = 256 (layers 3-4): single-buffered
+// (2 x 256 columns), the epilogue of a tile is short next to its 36+ K-blocks of MMAs
+template <int MODE, int BN_>
 struct DualMCfg {
-  static constexpr int BN = 128;
+  static constexpr int BN = BN_;
+  static constexpr int NBUF = BN == 128 ? 2 : 1;
   static constexpr int A_BYTES = 2 * BM * BK * 2;  // two 128-row tiles
   static constexpr int B_BYTES = BN * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
@@ -24,10 +27,11 @@ struct DualMCfg {
   static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 512 + EPI_BYTES + BIAS_BYTES;
 };
 
-template <int MODE>
+template <int MODE, int BN_>
 __global__ void __launch_bounds__(DUALM_THREADS, 1) conv_dualm_kernel(const __grid_constant__ ConvArgs a) {
   static_assert(MODE == MODE_FWD || MODE == MODE_DGRAD, "dual-M kernel: FWD / DGRAD");
-  using Cfg = DualMCfg<MODE>;
+  using Cfg = DualMCfg<MODE, BN_>;
+  constexpr int NBUF = Cfg::NBUF;
   constexpr int BN = Cfg::BN;
   constexpr int STAGES = Cfg::STAGES;
   extern __shared__ uint8_t smem_raw[];
@@ -65,7 +69,7 @@ __global__ void __launch_bounds__(DUALM_THREADS, 1) conv_dualm_kernel(const __gr
     }
     fence_mbar_init();
   }
-  if (warp == 4) tmem_alloc<4 * BN>(tmem_slot);
+  if (warp == 4) tmem_alloc<2 * BN * NBUF>(tmem_slot);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -114,7 +118,7 @@ __global__ void __launch_bounds__(DUALM_THREADS, 1) conv_dualm_kernel(const __gr
     constexpr uint32_t IDESC = make_idesc(BM, BN, 0, MODE == MODE_FWD ? 0 : 1);
     int it = 0, lt = 0;
     for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++lt) {
-      const int b = lt & 1, ub = lt >> 1;
+      const int b = NBUF == 2 ? (lt & 1) : 0, ub = NBUF == 2 ? (lt >> 1) : lt;
       if (ub > 0) mbar_wait(&tempty[b], (ub - 1) & 1);
       tc_fence_after();
       const uint32_t dacc = tmem + (uint32_t)(b * 2 * BN);
@@ -151,7 +155,7 @@ __global__ void __launch_bounds__(DUALM_THREADS, 1) conv_dualm_kernel(const __gr
       ti.kb0 = 0;
       ti.kb1 = nkb;
       ti.z = 0;
-      const int b = lt & 1, ub = lt >> 1;
+      const int b = NBUF == 2 ? (lt & 1) : 0, ub = NBUF == 2 ? (lt >> 1) : lt;
       const uint32_t trow = tmem + (uint32_t)(b * 2 * BN + half * BN) + ((uint32_t)(q * 32) << 16);
       const long long m = ti.m0 + row;
       const bool rv = m < npix;
@@ -176,7 +180,7 @@ __global__ void __launch_bounds__(DUALM_THREADS, 1) conv_dualm_kernel(const __gr
   __syncthreads();
   if (warp == 4) {
     tc_fence_after();
-    tmem_dealloc<4 * BN>(tmem);
+    tmem_dealloc<2 * BN * NBUF>(tmem);
   }
 }
 

@@ -111,20 +111,27 @@ static bool dualm_on() {
   }
   return g_dualm != 0;
 }
-template <int MODE>
-static bool try_launch_dualm(int BN, const ConvArgs& a, long long npix_static, cudaStream_t st) {
-  if (!dualm_on() || !a.a_tma || !a.b_tma || BN != 128 || a.K <= 4 * BK) return false;
-  using Cfg = DualMCfg<MODE>;
+template <int MODE, int BN>
+static void launch_dualm_t(const ConvArgs& a, long long tiles, cudaStream_t st) {
+  using Cfg = DualMCfg<MODE, BN>;
   static bool attr = false;
   if (!attr) {
-    CK(cudaFuncSetAttribute(conv_dualm_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
+    CK(cudaFuncSetAttribute(conv_dualm_kernel<MODE, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
     attr = true;
   }
-  const long long tiles = ((npix_static + 2 * BM - 1) / (2 * BM)) * ((a.Nout + BN - 1) / BN);
   dim3 grid((unsigned)std::max(1LL, std::min<long long>(tiles, num_sms())));
   ProfScope ps(MODE == MODE_FWD ? PC_CONV_FWD : PC_CONV_DGRAD, st);
-  conv_dualm_kernel<MODE><<<grid, DUALM_THREADS, Cfg::SMEM, st>>>(a);
+  conv_dualm_kernel<MODE, BN><<<grid, DUALM_THREADS, Cfg::SMEM, st>>>(a);
   CK(cudaGetLastError());
+}
+template <int MODE>
+static bool try_launch_dualm(int BN, const ConvArgs& a, long long npix_static, cudaStream_t st) {
+  if (!dualm_on() || !a.a_tma || !a.b_tma || (BN != 128 && BN != 256) || a.K <= 4 * BK) return false;
+  // BN = 256 (single-buffered accumulators, 2 smem stages) measured slower than the generic kernel: opt-in only
+  if (BN == 256 && !(getenv("ADAINF_DUALM256") && atoi(getenv("ADAINF_DUALM256")) == 1)) return false;
+  const long long tiles = ((npix_static + 2 * BM - 1) / (2 * BM)) * ((a.Nout + BN - 1) / BN);
+  if (BN == 128) launch_dualm_t<MODE, 128>(a, tiles, st);
+  else launch_dualm_t<MODE, 256>(a, tiles, st);
   return true;
 }
 

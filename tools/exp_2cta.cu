@@ -89,7 +89,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(128, 1) pair_gemm(co
   }
 }
 
-template <int CG>
+template <int CG, int NN = N>
 __global__ void __launch_bounds__(128, 1) mma_rate(const __grid_constant__ Args a, int iters, long long* cycles) {
   __shared__ __align__(1024) uint8_t sA[128 * 128];
   __shared__ __align__(1024) uint8_t sB[128 * 128];
@@ -123,12 +123,12 @@ __global__ void __launch_bounds__(128, 1) mma_rate(const __grid_constant__ Args 
 #pragma unroll
       for (int kk = 0; kk < 4; ++kk) {
         if (CG == 2) {
-          constexpr uint32_t IDESC = make_idesc(256, N, 0, 0);
+          constexpr uint32_t IDESC = make_idesc(256, NN, 0, 0);
           asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
                        "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
                        "l"(ad + 2u * kk), "l"(bd + 2u * kk), "r"(IDESC), "r"(1u) : "memory");
         } else {
-          constexpr uint32_t IDESC = make_idesc(128, N, 0, 0);
+          constexpr uint32_t IDESC = make_idesc(128, NN, 0, 0);
           asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
                        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
                        "l"(ad + 2u * kk), "l"(bd + 2u * kk), "r"(IDESC), "r"(1u) : "memory");
@@ -227,6 +227,28 @@ int main(int argc, char** argv) {
       printf("cta_group::%d M=%d N=%d: %.3f ms (%s) -> %.1f TFLOP/s, cycles/MMA (leader 0) %.1f\n", cg, 128 * cg, N, ms,
              cudaGetErrorString(er), flop / ms / 1e9, (double)hc[0] / (iters * 4));
     }
+  }
+  {
+    long long* cyc2;
+    cudaMalloc(&cyc2, 8 * 296);
+    auto run1 = [&](auto kern, int nn) {
+      cudaEvent_t e0, e1;
+      cudaEventCreate(&e0);
+      cudaEventCreate(&e1);
+      cudaEventRecord(e0);
+      kern<<<148, 128>>>(a, 20000, cyc2);
+      cudaEventRecord(e1);
+      cudaEventSynchronize(e1);
+      float ms = 0;
+      cudaEventElapsedTime(&ms, e0, e1);
+      long long hc[1];
+      cudaMemcpy(hc, cyc2, 8, cudaMemcpyDeviceToHost);
+      printf("cta_group::1 M=128 N=%d K=16: %.1f cycles per MMA, %.1f TFLOP/s\n", nn, (double)hc[0] / 80000,
+             2.0 * 148 * 80000.0 * 128 * nn * 16 / ms / 1e9);
+    };
+    run1(mma_rate<1, 64>, 64);
+    run1(mma_rate<1, 128>, 128);
+    run1(mma_rate<1, 256>, 256);
   }
   {
     for (int smem_kb : {0, 100, 200}) {
