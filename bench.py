@@ -323,7 +323,9 @@ def main():
     # graph and replayed: the same kernels and arguments, without per-launch host / front-end overhead between
     # them (--no-graph times the eagerly launched step instead)
     graph, graph_launches = None, 0
-    if not args.no_graph:
+    # (single process only: with N > 1 the step contains the NCCL gradient all-reduce, and a capture that
+    # failed on one rank but not another would leave the ranks' collectives out of step)
+    if not args.no_graph and world == 1:
         try:
             graph = torch.cuda.CUDAGraph()
             la = B.launch_count()
