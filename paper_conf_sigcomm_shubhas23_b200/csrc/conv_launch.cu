@@ -463,7 +463,12 @@ void conv_fwd(const ConvGeom& g, const bf16* x, const int* x_map, const int* cou
   if (mt == 0) return;
   // small batches (early-exit survivors; the device-side count is at most n_static): narrower N tiles until the
   // full-batch tile count covers two waves, so a partial survivor set still spreads over the SMs
-  while (BN > 64 && mt * ((g.Cout + BN - 1) / BN) < 2 * num_sms()) BN /= 2;
+  static int narrow = -1;  // ADAINF_NARROW=0 keeps the full BN (tests use it to reach the wide-tile kernels)
+  if (narrow < 0) {
+    const char* e = getenv("ADAINF_NARROW");
+    narrow = e ? atoi(e) : 1;
+  }
+  while (narrow && BN > 64 && mt * ((g.Cout + BN - 1) / BN) < 2 * num_sms()) BN /= 2;
   if (btma_on() && ldb % 8 == 0 && ((uintptr_t)w & 15) == 0) {
     a.b_tma = 1;
     a.b_map = make_tmap_2d(w, g.Cout, a.K, ldb, 64, BN);  // K-major [Cout][K]; k >= K and rows >= Cout read 0
