@@ -678,8 +678,9 @@ __global__ void wgrad_reduce_kernel(const float* __restrict__ part, int S, int K
                                     int cin_real, float* __restrict__ dw) {
   __shared__ float tile[32][33];
   const int k0 = blockIdx.x * 32, c0 = blockIdx.y * 32;
-  const int tx = threadIdx.x, ty = threadIdx.y;  // 32 x 8
-  for (int r = ty; r < 32; r += 8) {
+  const int tx = threadIdx.x, ty = threadIdx.y;  // 32 x (8 or 32)
+  const int ry = blockDim.y;
+  for (int r = ty; r < 32; r += ry) {
     const int k = k0 + r, co = c0 + tx;
     float acc = 0.f;
     if (k < Kconv && co < Cout) {  // eight independent loads in flight, summed in ascending split order
@@ -698,7 +699,7 @@ __global__ void wgrad_reduce_kernel(const float* __restrict__ part, int S, int K
     tile[r][tx] = acc;
   }
   __syncthreads();
-  for (int r = ty; r < 32; r += 8) {
+  for (int r = ty; r < 32; r += ry) {
     const int co = c0 + r, k = k0 + tx;
     if (k < Kconv && co < Cout) {
       const int tap = k / cin_pad, ci = k - tap * cin_pad;
@@ -1050,7 +1051,9 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
       S2 = G;
     }
     dim3 rg((p.Kconv + 31) / 32, (g.Cout + 31) / 32);
-    wgrad_reduce_kernel<<<rg, dim3(32, 8), 0, st>>>(src, S2, p.Kconv, g.Cout, g.Cin, cin_real, dw);
+    // small weight tensors: one thread per element of the 32x32 tile (more loads in flight per SM)
+    const dim3 rb(32, (long long)rg.x * rg.y < 2LL * num_sms() ? 32 : 8);
+    wgrad_reduce_kernel<<<rg, rb, 0, st>>>(src, S2, p.Kconv, g.Cout, g.Cin, cin_real, dw);
     CK(cudaGetLastError());
   }
   if (db) {
