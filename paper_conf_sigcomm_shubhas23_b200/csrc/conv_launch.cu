@@ -743,21 +743,33 @@ __global__ void __launch_bounds__(CS_THREADS) colsum_partial_kernel(const bf16* 
     part[(long long)blockIdx.x * C + c] = s;
   }
 }
-__global__ void colsum_final_kernel(const float* __restrict__ part, int nb, int C, float* __restrict__ out) {
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= C) return;
-  // eight independent loads in flight, summed in the same ascending order
+// out[c] = sum over nb partial rows, deterministic: 8 row groups per channel (rows g, g+8, ... in order, eight
+// loads in flight), then the 8 group sums in group order
+__global__ void __launch_bounds__(256) colsum_final_kernel(const float* __restrict__ part, int nb, int C,
+                                                           float* __restrict__ out) {
+  __shared__ float red[8][33];
+  const int cx = threadIdx.x & 31, gy = threadIdx.x >> 5;
+  const int c = blockIdx.x * 32 + cx;
   float acc = 0.f;
-  int b = 0;
-  for (; b + 8 <= nb; b += 8) {
-    float v[8];
+  if (c < C) {
+    int b = gy;
+    for (; b + 56 < nb; b += 64) {
+      float v[8];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) v[u] = __ldg(part + (long long)(b + u) * C + c);
+      for (int u = 0; u < 8; ++u) v[u] = __ldg(part + (long long)(b + 8 * u) * C + c);
 #pragma unroll
-    for (int u = 0; u < 8; ++u) acc += v[u];
+      for (int u = 0; u < 8; ++u) acc += v[u];
+    }
+    for (; b < nb; b += 8) acc += __ldg(part + (long long)b * C + c);
   }
-  for (; b < nb; ++b) acc += __ldg(part + (long long)b * C + c);
-  out[c] = acc;
+  red[gy][cx] = acc;
+  __syncthreads();
+  if (gy == 0 && c < C) {
+    float t = red[0][cx];
+#pragma unroll
+    for (int g = 1; g < 8; ++g) t += red[g][cx];
+    out[c] = t;
+  }
 }
 static int colsum_blocks(long long P) { return (int)std::max(1LL, std::min<long long>((P + 63) / 64, 4LL * num_sms())); }
 
@@ -1065,7 +1077,7 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
       const int groups = CS_THREADS / (g.Cout / 8);
       colsum_partial_kernel<<<nb, CS_THREADS, (size_t)groups * g.Cout * 4, st>>>(dz, npix, g.Cout, rpb, cs_part);
     }
-    colsum_final_kernel<<<(g.Cout + 127) / 128, 128, 0, st>>>(cs_part, nb, g.Cout, db);
+    colsum_final_kernel<<<(g.Cout + 31) / 32, 256, 0, st>>>(cs_part, nb, g.Cout, db);
     CK(cudaGetLastError());
   }
 }
