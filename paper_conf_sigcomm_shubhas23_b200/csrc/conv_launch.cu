@@ -583,26 +583,26 @@ bool dgrad_sp_ok(const ConvGeom& g) {
 size_t dgrad_sp_ws_bytes(const ConvGeom& g) { return (size_t)4 * g.Cin * 4 * g.Cout * 2; }
 
 // Bsp[(py,px,ci)][(a,b,co)] = W[co][kh = py+p-2a][kw = px+p-2b][ci], 0 where the tap does not exist.
-// One thread per (a,b,co) column and 8-channel ci vector: a 16-byte read of the shadow row, 8 strided writes.
+// One thread per 8 consecutive output columns (8 co of one (a,b)): eight 2-byte gathers from the (L2-resident)
+// shadow, one coalesced 16-byte store.
 __global__ void sp_weight_kernel(const bf16* __restrict__ w, int ldb, int Cin, int Cout, int K, int pad,
                                  bf16* __restrict__ bsp) {
-  const int CV = Cin / 8;
-  const long long total = 4LL * Cout * CV * 4;
+  const int K4 = 4 * Cout, KV = K4 / 8;
+  const long long total = 4LL * Cin * KV;
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
-    const int cv = (int)(i % CV);
-    long long r = i / CV;
-    const int ph = (int)(r % 4);
-    const int kcol = (int)(r / 4);  // (a,b,co)
-    const int ab = kcol / Cout, co = kcol - ab * Cout;
+    const int kv = (int)(i % KV);
+    const long long r = i / KV;  // output row (ph, ci)
+    const int ci = (int)(r % Cin), ph = (int)(r / Cin);
+    const int kcol0 = kv * 8;
+    const int ab = kcol0 / Cout, co0 = kcol0 - ab * Cout;
     const int py = ph >> 1, px = ph & 1, aa = ab >> 1, bb = ab & 1;
     const int kh = py + pad - 2 * aa, kw = px + pad - 2 * bb;
-    uint4 v = make_uint4(0u, 0u, 0u, 0u);
-    if (kh >= 0 && kh < K && kw >= 0 && kw < K)
-      v = __ldg((const uint4*)(w + (long long)co * ldb + (kh * K + kw) * Cin + cv * 8));
-    const bf16* h = (const bf16*)&v;
-    const long long K4 = 4LL * Cout;
+    __align__(16) bf16 h[8];
+    const bool ok = kh >= 0 && kh < K && kw >= 0 && kw < K;
 #pragma unroll
-    for (int q = 0; q < 8; ++q) bsp[((long long)ph * Cin + cv * 8 + q) * K4 + kcol] = h[q];
+    for (int q = 0; q < 8; ++q)
+      h[q] = ok ? w[(long long)(co0 + q) * ldb + (kh * K + kw) * Cin + ci] : __float2bfloat16_rn(0.f);
+    *(uint4*)(bsp + r * K4 + kcol0) = *(const uint4*)h;
   }
 }
 
@@ -613,7 +613,7 @@ void conv_dgrad_sp(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, bf
   if (n <= 0) return;
   {
     ProfScope ps(PC_CONV_DGRAD_PREP, st);
-    const long long total = 16LL * g.Cout * (g.Cin / 8);
+    const long long total = 4LL * g.Cin * (4 * g.Cout / 8);
     const int blocks = (int)std::min<long long>((total + 255) / 256, 8LL * num_sms());
     sp_weight_kernel<<<blocks, 256, 0, st>>>(w, ldb, g.Cin, g.Cout, 3, g.pad, wsp);
     CK(cudaGetLastError());
