@@ -667,24 +667,35 @@ __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_
 
 // sum the per-CTA partials (both row halves) in fixed order and scatter (tap, s2d channel) back to
 // dw [64][7][7][cin]
-__global__ void stem_wgrad_finish_kernel(const float* __restrict__ part, int G, int cin, float* __restrict__ dw) {
-  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= 256 * 64) return;
+// 8 partial-row groups per output (groups g, g+8, ... summed in order, eight loads in flight), combined in group
+// order through shared memory: 256 threads = 32 outputs x 8 groups
+__global__ void __launch_bounds__(256) stem_wgrad_finish_kernel(const float* __restrict__ part, int G, int cin,
+                                                                float* __restrict__ dw) {
+  __shared__ float red[8][33];
+  const int ox = threadIdx.x & 31, gy = threadIdx.x >> 5;
+  const int idx = blockIdx.x * 32 + ox;  // < 256 * 64 (grid = 512 blocks)
   const int co = idx & 63, k = idx >> 6;
-  float acc = 0.f;  // eight independent loads in flight, summed in ascending order
-  int g = 0;
-  for (; g + 8 <= 2 * G; g += 8) {
+  float acc = 0.f;
+  const int NG = 2 * G;
+  int g = gy;
+  for (; g + 56 < NG; g += 64) {
     float v[8];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) v[u] = __ldg(part + ((long long)(g + u) * 256 + k) * 64 + co);
+    for (int u = 0; u < 8; ++u) v[u] = __ldg(part + ((long long)(g + 8 * u) * 256 + k) * 64 + co);
 #pragma unroll
     for (int u = 0; u < 8; ++u) acc += v[u];
   }
-  for (; g < 2 * G; ++g) acc += __ldg(part + ((long long)g * 256 + k) * 64 + co);
-  const int t = k >> 4, ch = k & 15;
+  for (; g < NG; g += 8) acc += __ldg(part + ((long long)g * 256 + k) * 64 + co);
+  red[gy][ox] = acc;
+  __syncthreads();
+  if (gy != 0) return;
+  float t = red[0][ox];
+#pragma unroll
+  for (int q = 1; q < 8; ++q) t += red[q][ox];
+  const int tap = k >> 4, ch = k & 15;
   const int bh = ch >> 3, bw = (ch >> 2) & 1, c = ch & 3;
-  const int kh = 2 * (t / 4 - 2) + bh + 3, kw = 2 * (t % 4 - 2) + bw + 3;
-  if (kh >= 0 && kh < 7 && kw >= 0 && kw < 7 && c < cin) dw[((co * 7 + kh) * 7 + kw) * cin + c] = acc;
+  const int kh = 2 * (tap / 4 - 2) + bh + 3, kw = 2 * (tap % 4 - 2) + bw + 3;
+  if (kh >= 0 && kh < 7 && kw >= 0 && kw < 7 && c < cin) dw[((co * 7 + kh) * 7 + kw) * cin + c] = t;
 }
 __global__ void stem_colsum_final_kernel(const float* __restrict__ part, int G, float* __restrict__ db) {
   const int c = threadIdx.x;
@@ -761,7 +772,7 @@ static void stem_wgrad_impl(const bf16* s, const bf16* dz, const bf16* pool_dT, 
     CK(cudaGetLastError());
   }
   ProfScope ps(PC_STEM_AUX, st, db ? 2 : 1);
-  stem_wgrad_finish_kernel<<<64, 256, 0, st>>>(ws, G, cin_real, dw);
+  stem_wgrad_finish_kernel<<<256 * 64 / 32, 256, 0, st>>>(ws, G, cin_real, dw);
   if (db) stem_colsum_final_kernel<<<1, 64, 0, st>>>(a.cs_part, G, db);
   CK(cudaGetLastError());
 }
