@@ -767,6 +767,28 @@ __global__ void gather_rows_kernel(const uint4* __restrict__ src, const int32_t*
     dst[i] = __ldg(src + (long long)idx[r] * row_vec + c);
   }
 }
+// one row per grid.y, 4 x 16 bytes per thread (no per-element division); rows past the device count return
+__global__ void __launch_bounds__(256) gather_rows2d_kernel(const uint4* __restrict__ src, const int32_t* __restrict__ idx,
+                                                            const int32_t* count, int n_static, long long row_vec,
+                                                            uint4* __restrict__ dst) {
+  const int r = blockIdx.y;
+  const int n = count ? min(*count, n_static) : n_static;
+  if (r >= n) return;
+  const uint4* s = src + (long long)__ldg(idx + r) * row_vec;
+  uint4* d = dst + (long long)r * row_vec;
+  const long long c0 = (long long)blockIdx.x * 1024 + threadIdx.x;
+  uint4 v[4];
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    const long long c = c0 + u * 256;
+    if (c < row_vec) v[u] = __ldg(s + c);
+  }
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    const long long c = c0 + u * 256;
+    if (c < row_vec) d[c] = v[u];
+  }
+}
 __global__ void gather_rows4_kernel(const uint32_t* __restrict__ src, const int32_t* __restrict__ idx, const int32_t* count,
                                     int n_static, long long row_words, uint32_t* __restrict__ dst) {
   const int n = count ? min(*count, n_static) : n_static;
@@ -777,14 +799,18 @@ __global__ void gather_rows4_kernel(const uint32_t* __restrict__ src, const int3
   }
 }
 void launch_gather_rows(const void* src, const int32_t* idx, const int32_t* count, int n_static, long long row_bytes,
-                        void* dst, cudaStream_t st) {
+                        void* dst, cudaStream_t st, int prof_class) {
   if (row_bytes % 4) throw ShapeError("gather_rows: row bytes must be a multiple of 4");
   const bool v16 = (row_bytes % 16) == 0;
   const long long total = (long long)n_static * (row_bytes / (v16 ? 16 : 4));
   const int blocks = (int)std::min<long long>((total + 255) / 256, 32LL * num_sms());
   if (blocks <= 0) return;
-  ProfScope ps(PC_GATHER, st);
-  if (v16)
+  ProfScope ps(prof_class, st);
+  if (v16 && row_bytes >= 16 * 1024 && n_static <= 65535) {  // large rows: 2-D grid, one row per grid.y
+    const long long rv = row_bytes / 16;
+    dim3 g((unsigned)((rv + 1023) / 1024), (unsigned)n_static);
+    gather_rows2d_kernel<<<g, 256, 0, st>>>((const uint4*)src, idx, count, n_static, rv, (uint4*)dst);
+  } else if (v16)
     gather_rows_kernel<<<blocks, 256, 0, st>>>((const uint4*)src, idx, count, n_static, row_bytes / 16, (uint4*)dst);
   else
     gather_rows4_kernel<<<blocks, 256, 0, st>>>((const uint32_t*)src, idx, count, n_static, row_bytes / 4,

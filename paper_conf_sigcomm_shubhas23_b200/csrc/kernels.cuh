@@ -1,5 +1,6 @@
 // Declarations of the CUDA-core kernels' host launchers (HBM / latency-bound steps of the hot path).
 #pragma once
+#include "prof.h"
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -86,6 +87,6 @@ void launch_sgd(float* w, float* v, const float* g, long long n, float lr, float
                 cudaStream_t st);
 void launch_shadow_pack(const float* w, const SgdSeg* segs_dev, int nseg, cudaStream_t st);
 void launch_gather_rows(const void* src, const int32_t* idx, const int32_t* count, int n_static, long long row_bytes,
-                        void* dst, cudaStream_t st);
+                        void* dst, cudaStream_t st, int prof_class = PC_GATHER);
 
 }  // namespace adainf

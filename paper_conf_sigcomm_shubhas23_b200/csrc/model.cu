@@ -246,6 +246,11 @@ void Model::build(const adainf_model_spec& s) {
       nd.shadow.zero();
     }
   if (stem_s2d) stem_wprep.alloc(16 * 2 * 64 * 8 * 2);
+  for (size_t k = 0; k + 1 < exits.size(); ++k) {  // dense survivor copies of the stage-boundary tensors
+    const TensorRt& X = T[exits[k].tensor];
+    if (!X.f32 && exits[k].tensor > 0 && (X.row_elems() * 2) % 16 == 0)
+      exits[k].dense_next.alloc((size_t)max_batch * X.row_elems() * 2);
+  }
   params.alloc(nparams * 4);
   mom.alloc(nparams * 4);
   grads.alloc(nparams * 4);
@@ -402,11 +407,14 @@ void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, in
   int* cnt = counts.as<int>();
   auto stage_count = [&](int s) -> const int* { return s == 0 ? count0 : cnt + s; };
   auto stage_orig = [&](int s) -> const int* { return s == 0 ? nullptr : origb + (size_t)s * max_batch; };
-  auto buf_of = [&](int t) -> const bf16* { return t == 0 ? x0 : T[t].buf; };
+  // inference: stage-boundary tensors whose survivors have been gathered densely (per tensor, after compaction)
+  std::vector<const bf16*> dense_t(T.size(), nullptr);
+  auto buf_of = [&](int t) -> const bf16* { return t == 0 ? x0 : (dense_t[t] ? dense_t[t] : T[t].buf); };
   // map used by a node of stage `ns` reading tensor t
   auto map_for = [&](int t, int ns) -> const int* {
     if (train) return nullptr;
     if (t == 0) return ns == 0 ? map0 : nullptr;
+    if (dense_t[t]) return nullptr;
     if (T[t].stage < ns) return posb + (size_t)ns * max_batch;
     return nullptr;
   };
@@ -432,7 +440,7 @@ void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, in
                            nd.in > 0 && T[nd.in].act == 1, st);
       } else {
         const float* bias = params.as<float>() + nd.b_off;
-        const bf16* res = nd.res >= 0 ? T[nd.res].buf : nullptr;
+        const bf16* res = nd.res >= 0 ? buf_of(nd.res) : nullptr;
         const int* rmap = nd.res >= 0 ? map_for(nd.res, ns) : nullptr;
         conv_fwd(nd.g, buf_of(nd.in), map_for(nd.in, ns), c, n_static, nd.shadow.as<bf16>(), nd.ldb, bias, res, rmap,
                  nd.act, T[nd.out].buf, nd.fp32_out, st);
@@ -481,6 +489,11 @@ void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, in
                      origb + (size_t)(s + 1) * max_batch, cnt + s + 1, out->exit_counts, k,
                      out->surv_idx ? out->surv_idx + (size_t)k * n_static : nullptr,
                      (k == E - 2) ? out->exit_counts : nullptr, E - 1, st);
+      if (e.dense_next.p) {
+        launch_gather_rows(T[e.tensor].buf, posb + (size_t)(s + 1) * max_batch, cnt + s + 1, n_static,
+                           (long long)X.row_elems() * 2, e.dense_next.p, st, PC_SURVIVOR_GATHER);
+        dense_t[e.tensor] = e.dense_next.as<bf16>();
+      }
     }
   }
 }

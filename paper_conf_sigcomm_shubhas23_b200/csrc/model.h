@@ -75,6 +75,9 @@ struct ExitRt {
   float lw;
   long long w_off, b_off;
   DevBuf pooled, logits, dl, bcast;  // training
+  // inference: the survivors' rows of this exit's tensor gathered densely after the compaction, so the next
+  // stage's convolutions read a dense source (TMA im2col operands) instead of gathering through the row map
+  DevBuf dense_next;
 };
 
 struct DetRt {

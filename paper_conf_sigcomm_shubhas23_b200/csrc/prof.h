@@ -32,6 +32,7 @@ enum ProfClass {
   PC_STEM_WGRAD,
   PC_STEM_AUX,
   PC_CONV_DGRAD_PREP,
+  PC_SURVIVOR_GATHER,
   PROF_NCLASS
 };
 

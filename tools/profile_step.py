@@ -10,6 +10,7 @@ ap.add_argument("--train-only", action="store_true")
 ap.add_argument("--steps", type=int, default=2)
 ap.add_argument("--batch", type=int, default=256)
 ap.add_argument("--k", type=int, default=1024)
+ap.add_argument("--taus", type=str, default="0.3,0.5,0.7", help="exit thresholds (bench-calibrated: 0.43,0.23,0.26)")
 a = ap.parse_args()
 spec = S.resnet18_ee()
 p = synth.init_params(spec, seed=1)
@@ -25,7 +26,7 @@ for i in range(a.steps):
         torch.cuda.synchronize()
         torch.cuda.nvtx.range_push("profiled")
     if not a.train_only:
-        app.infer(x[:a.batch], [0.3, 0.5, 0.7], [outs])
+        app.infer(x[:a.batch], [float(t) for t in a.taus.split(",")], [outs])
     if not a.infer_only:
         m.retrain_step(x[:a.k], lab[:a.k], lr=0.01)
     if last:
