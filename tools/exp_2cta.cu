@@ -154,6 +154,46 @@ __global__ void __launch_bounds__(128, 1) mma_rate(const __grid_constant__ Args 
   }
 }
 
+// per-tile commit cost: `per` MMAs (N=64) per tile into alternating accumulators, then a commit to an mbarrier
+// (as the window conv kernels do); measures cycles per MMA including the per-tile commit
+template <int NB, int NC = 1>
+__global__ void __launch_bounds__(128, 1) mma_commit_rate(int tiles, int per, long long* cycles) {
+  __shared__ __align__(1024) uint8_t sA[128 * 128];
+  __shared__ __align__(1024) uint8_t sB[128 * 128];
+  __shared__ uint64_t bar[NB], bar2[NB];
+  __shared__ uint32_t tmem_slot;
+  const int warp = threadIdx.x >> 5;
+  if (threadIdx.x == 0) {
+    for (int q = 0; q < NB; ++q) mbar_init(&bar[q], 1), mbar_init(&bar2[q], 1);
+    fence_mbar_init();
+  }
+  if (warp == 0) tmem_alloc<NB * 64 < 32 ? 32 : NB * 64>(&tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_slot;
+  if (threadIdx.x == 0) {
+    const long long t0 = clock64();
+    const uint64_t ad = make_sdesc(smem_u32(sA), 16, 1024), bd = make_sdesc(smem_u32(sB), 16, 1024);
+    constexpr uint32_t IDESC = make_idesc(128, 64, 0, 0);
+    for (int t = 0; t < tiles; ++t) {
+      const int b = t % NB;
+      if (t >= NB) mbar_wait(&bar[b], ((t / NB) - 1) & 1);  // accumulator b drained (no epilogue: commit only)
+      for (int i = 0; i < per; ++i) umma_bf16(tmem + b * 64, ad + 2u * (i & 3), bd + 2u * (i & 3), IDESC, i > 0);
+      if (NC == 2) umma_commit(&bar2[b]);
+      umma_commit(&bar[b]);
+    }
+    mbar_wait(&bar[(tiles - 1) % NB], ((tiles - 1) / NB) & 1);
+    cycles[blockIdx.x] = clock64() - t0;
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) {
+    tc_fence_after();
+    tmem_dealloc<NB * 64 < 32 ? 32 : NB * 64>(tmem);
+  }
+}
+
 static float bf(uint16_t h) {
   uint32_t u = (uint32_t)h << 16;
   float f;
@@ -247,6 +287,26 @@ int main(int argc, char** argv) {
              2.0 * 148 * 80000.0 * 128 * nn * 16 / ms / 1e9);
     };
     run1(mma_rate<1, 64>, 64);
+    for (int per : {36}) {
+      const int tiles = 80000 / per;
+      mma_commit_rate<2, 2><<<148, 128>>>(tiles, per, cyc2);
+      cudaDeviceSynchronize();
+      long long hc[1];
+      cudaMemcpy(hc, cyc2, 8, cudaMemcpyDeviceToHost);
+      printf("N=64, 2 accumulators, TWO commits per tile, %d MMAs per tile: %.1f cycles per MMA\n", per,
+             (double)hc[0] / (tiles * per));
+    }
+    for (int nbuf : {2, 4})
+      for (int per : {36, 72, 144}) {
+        const int tiles = 80000 / per;
+        if (nbuf == 2) mma_commit_rate<2><<<148, 128>>>(tiles, per, cyc2);
+        else mma_commit_rate<4><<<148, 128>>>(tiles, per, cyc2);
+        cudaDeviceSynchronize();
+        long long hc[1];
+        cudaMemcpy(hc, cyc2, 8, cudaMemcpyDeviceToHost);
+        printf("N=64, %d accumulators, %d MMAs per committed tile: %.1f cycles per MMA\n", nbuf, per,
+               (double)hc[0] / (tiles * per));
+      }
     run1(mma_rate<1, 128>, 128);
     run1(mma_rate<1, 256>, 256);
   }
