@@ -156,7 +156,7 @@ __global__ void __launch_bounds__(128, 1) mma_rate(const __grid_constant__ Args 
 
 // per-tile commit cost: `per` MMAs (N=64) per tile into alternating accumulators, then a commit to an mbarrier
 // (as the window conv kernels do); measures cycles per MMA including the per-tile commit
-template <int NB, int NC = 1>
+template <int NB, int NC = 1, int MODE = 0>
 __global__ void __launch_bounds__(128, 1) mma_commit_rate(int tiles, int per, long long* cycles) {
   __shared__ __align__(1024) uint8_t sA[128 * 128];
   __shared__ __align__(1024) uint8_t sB[128 * 128];
@@ -177,13 +177,22 @@ __global__ void __launch_bounds__(128, 1) mma_commit_rate(int tiles, int per, lo
     const uint64_t ad = make_sdesc(smem_u32(sA), 16, 1024), bd = make_sdesc(smem_u32(sB), 16, 1024);
     constexpr uint32_t IDESC = make_idesc(128, 64, 0, 0);
     for (int t = 0; t < tiles; ++t) {
-      const int b = t % NB;
-      if (t >= NB) mbar_wait(&bar[b], ((t / NB) - 1) & 1);  // accumulator b drained (no epilogue: commit only)
-      for (int i = 0; i < per; ++i) umma_bf16(tmem + b * 64, ad + 2u * (i & 3), bd + 2u * (i & 3), IDESC, i > 0);
-      if (NC == 2) umma_commit(&bar2[b]);
-      umma_commit(&bar[b]);
+      const int b = MODE == 1 ? 0 : t % NB;
+      if (MODE == 0 && t >= NB) mbar_wait(&bar[b], ((t / NB) - 1) & 1);  // accumulator b drained
+      // MODE 3: commit every tile but never wait (the barrier phase is simply overrun; timing only)
+      if (MODE == 1 && t >= 1) mbar_wait(&bar[0], (t - 1) & 1);
+      for (int i = 0; i < per; ++i)
+        umma_bf16(tmem + b * 64, ad + 2u * (i & 3), bd + 2u * (i & 3), IDESC, MODE == 1 ? 1 : (i > 0));
+      if (MODE != 2) {
+        if (NC == 2) umma_commit(&bar2[b]);
+        umma_commit(&bar[b]);
+      }
     }
-    mbar_wait(&bar[(tiles - 1) % NB], ((tiles - 1) / NB) & 1);
+    if (MODE == 2 || MODE == 3) umma_commit(&bar2[0]);
+    if (MODE == 2 || MODE == 3) mbar_wait(&bar2[0], 0);
+    else if (MODE == 0) mbar_wait(&bar[(tiles - 1) % NB], ((tiles - 1) / NB) & 1);
+    else if (MODE == 1) mbar_wait(&bar[0], (tiles - 1) & 1);
+
     cycles[blockIdx.x] = clock64() - t0;
   }
   tc_fence_before();
@@ -294,6 +303,23 @@ int main(int argc, char** argv) {
       long long hc[1];
       cudaMemcpy(hc, cyc2, 8, cudaMemcpyDeviceToHost);
       printf("N=64, 2 accumulators, TWO commits per tile, %d MMAs per tile: %.1f cycles per MMA\n", per,
+             (double)hc[0] / (tiles * per));
+    }
+    {
+      const int per = 36, tiles = 80000 / per;
+      long long hc[1];
+      mma_commit_rate<2, 1, 1><<<148, 128>>>(tiles, per, cyc2);
+      cudaDeviceSynchronize();
+      cudaMemcpy(hc, cyc2, 8, cudaMemcpyDeviceToHost);
+      printf("N=64, ONE accumulator, commit + wait every 36 MMAs: %.1f cycles per MMA\n", (double)hc[0] / (tiles * per));
+      mma_commit_rate<2, 1, 3><<<148, 128>>>(tiles, per, cyc2);
+      cudaDeviceSynchronize();
+      cudaMemcpy(hc, cyc2, 8, cudaMemcpyDeviceToHost);
+      printf("N=64, commit every 36 MMAs, never waited on: %.1f cycles per MMA\n", (double)hc[0] / (tiles * per));
+      mma_commit_rate<2, 1, 2><<<148, 128>>>(tiles, per, cyc2);
+      cudaDeviceSynchronize();
+      cudaMemcpy(hc, cyc2, 8, cudaMemcpyDeviceToHost);
+      printf("N=64, switch accumulator every 36 MMAs (fresh accumulate), no commit: %.1f cycles per MMA\n",
              (double)hc[0] / (tiles * per));
     }
     for (int nbuf : {2, 4})
