@@ -412,8 +412,10 @@ def main():
     hbm_bytes = {
         # w, v, g read (12 B), w, v written (8 B), bf16 GEMM-layout shadow of conv weights written (2 B)
         "sgd_update": nparams * 20 + conv_params * 2,
-        # GAP reads the exit tensor of every row reaching the exit (inference survivors + all retrain rows)
-        "exit_head": float(np.dot(reach, exit_bytes_row)) + K_SEL * sum(exit_bytes_row),
+        # inference: GAP reads the exit tensor of every row reaching the exit (survivors only)
+        "exit_head": float(np.dot(reach, exit_bytes_row)),
+        # retraining forward: every exit head reads its tensor for all selected rows
+        "exit_head_train": K_SEL * sum(exit_bytes_row),
         # dT (bf16) + argmax codes read, dZ written at 112x112x64 (stem pool backward)
         "maxpool_bwd": K_SEL * (56 * 56 * 64 * 3 + 112 * 112 * 64 * 2),
         # selected rows read from the pool and written to the retrain batch (+ labels)

@@ -375,7 +375,7 @@ __global__ void __launch_bounds__(EH_THREADS) exit_head_kernel(const ExitHeadArg
   if (s_exit && a.logits)
     for (int k = t; k < a.ncls; k += EH_THREADS) a.logits[(long long)orig * a.ncls + k] = logits[k];
 }
-void launch_exit_head(const ExitHeadArgs& a, cudaStream_t st) {
+void launch_exit_head(const ExitHeadArgs& a, cudaStream_t st, int prof_class) {
   if (a.n_static <= 0) return;
   const bool wide = a.n_static < 4 * num_sms();
   const int T = wide ? 512 : 128;
@@ -383,7 +383,7 @@ void launch_exit_head(const ExitHeadArgs& a, cudaStream_t st) {
     throw ShapeError("exit head: C must be 8 * a power of two <= 1024");
   const int groups = T / (a.C / 8);
   const size_t smem = (size_t)(groups * a.C + a.C + a.ncls) * sizeof(float);
-  ProfScope ps(PC_EXIT_HEAD, st);
+  ProfScope ps(prof_class, st);
   if (wide) exit_head_kernel<512><<<a.n_static, 512, smem, st>>>(a);
   else exit_head_kernel<128><<<a.n_static, 128, smem, st>>>(a);
   CK(cudaGetLastError());

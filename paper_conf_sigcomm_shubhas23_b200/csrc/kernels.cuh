@@ -48,7 +48,7 @@ struct ExitHeadArgs {
   float* pooled_save;   // [rows][C]
   float* logits_save;   // [rows][ncls]
 };
-void launch_exit_head(const ExitHeadArgs& a, cudaStream_t st);
+void launch_exit_head(const ExitHeadArgs& a, cudaStream_t st, int prof_class = PC_EXIT_HEAD);
 
 // stable compaction of alive rows: pos_next[j'] = j, orig_next[j'] = orig[j]; count_next; counts[k] += exited;
 // surv_out (optional, user): ascending original rows

@@ -465,7 +465,7 @@ void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, in
       a.is_final = 1;
       a.pooled_save = e.pooled.as<float>();
       a.logits_save = e.logits.as<float>();
-      launch_exit_head(a, st);
+      launch_exit_head(a, st, PC_EXIT_HEAD_TRAIN);
       continue;
     }
     const int s = e.stage;

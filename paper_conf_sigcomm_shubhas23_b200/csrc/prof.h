@@ -33,6 +33,7 @@ enum ProfClass {
   PC_STEM_AUX,
   PC_CONV_DGRAD_PREP,
   PC_SURVIVOR_GATHER,
+  PC_EXIT_HEAD_TRAIN,
   PROF_NCLASS
 };
 
