@@ -180,7 +180,7 @@ static void launch_win_t(const WinArgs& w, long long max_tiles, cudaStream_t st)
 
 // TMA weight-stationary 64x64 window conv (FWD: e0 = residual; DGRAD: e0 = shortcut grad, e1 = activation)
 static void launch_ws_tma(const ConvArgs& c, bool dgrad, int nstatic, cudaStream_t st) {
-  static WsTmaArgs a;  // host staging (copied into the launch parameters)
+  thread_local WsTmaArgs a;  // host staging (copied into the launch parameters); per thread: handles are independent
   a = WsTmaArgs{};
   const int H = c.Hs, W = c.Ws;
   int Wp = 1;
@@ -273,7 +273,7 @@ static bool win_tma_ok(const ConvArgs& c, int nout) {
 }
 
 static void launch_win_tma(const ConvArgs& c, bool dgrad, int nstatic, int nout, cudaStream_t st) {
-  static WinTmaArgs a;
+  thread_local WinTmaArgs a;
   a = WinTmaArgs{};
   const int H = c.Hs, W = c.Ws;
   int Wp = 1;
@@ -618,7 +618,7 @@ void conv_dgrad_sp(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, bf
     sp_weight_kernel<<<blocks, 256, 0, st>>>(w, ldb, g.Cin, g.Cout, 3, g.pad, wsp);
     CK(cudaGetLastError());
   }
-  static ConvArgs a;
+  thread_local ConvArgs a;
   a = ConvArgs{};
   a.src = dz;
   a.Hs = g.Ho;
@@ -940,7 +940,7 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
   const int S = p.S;
 
   if (p.path == WG_WIN_TMA) {
-    static WinWgTmaArgs a;
+    thread_local WinWgTmaArgs a;
     a = WinWgTmaArgs{};
     a.n = n;
     a.H = g.H;
@@ -971,7 +971,7 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
     conv_wgrad_win_tma_kernel<<<std::max(1, std::min(units, num_sms())), NUM_THREADS, smem, st>>>(a);
     CK(cudaGetLastError());
   } else if (p.path == WG_TMA) {
-    static WgTmaArgs a;
+    thread_local WgTmaArgs a;
     a = WgTmaArgs{};
     a.n = n;
     a.Ho = g.Ho;

@@ -329,7 +329,7 @@ void stem_fwd(const bf16* s, const int* count, int n_static, int Hs, int Ws, con
               bf16* pooled, uint8_t* argmax, cudaStream_t st) {
   if (n_static <= 0) return;
   if (Ws > 125) throw ShapeError("stem: width/2 must be <= 125");
-  static StemFwdArgs a;
+  thread_local StemFwdArgs a;
   a = StemFwdArgs{};
   a.s_map = make_tmap_nhwc_swz(s, n_static, Hs, Ws, 16, 16, SLOTS, 4, 32);
   a.wprep = wprep;
@@ -735,7 +735,7 @@ static void stem_wgrad_impl(const bf16* s, const bf16* dz, const bf16* pool_dT, 
   if (n <= 0) return;
   if (Ws > 125) throw ShapeError("stem: width/2 must be <= 125");
   if (ws_bytes < stem_wgrad_ws_bytes(n)) throw std::runtime_error("stem wgrad workspace too small");
-  static StemWgArgs a;
+  thread_local StemWgArgs a;
   a = StemWgArgs{};
   a.s_map = make_tmap_nhwc_swz(s, n, Hs, Ws, 16, 16, SLOTS, 1, 32);
   if (pool_dT) {
