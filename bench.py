@@ -7,8 +7,8 @@ input, all through libadainf.so's C-ABI (include/adainf.h):
                               calibrated once to ~25/25/25/25 exit fractions
   a7     adainf_select_retrain  16,384-sample window pool (D=64 embeddings -> PCA P=16, cosine distance
                               to the old mean, 10% already used/excluded) -> k = 1,024
-         adainf_gather_rows   selected samples -> retraining batch (device-resident pool)
-  a8-a11 adainf_retrain_step  one SGD+momentum step on the 1,024 selected samples (lr 0.01, mu 0.9)
+  a8-a11 adainf_retrain_step_rows  one SGD+momentum step on the 1,024 selected rows of the device-resident
+                              window pool, packed straight from the pool (lr 0.01, mu 0.9)
                               (N>1: data-parallel, NCCL all-reduce of the fp32 gradient)
 
 value = (inference samples + retraining samples) of all ranks / max-over-ranks device time per step.
@@ -263,8 +263,6 @@ def main():
     sel_idx = torch.empty(K_SEL, dtype=torch.int32, device=dev)
     sel_dist = torch.empty(K_SEL, dtype=torch.float32, device=dev)
     sel_cnt = torch.empty(1, dtype=torch.int32, device=dev)
-    rt_x = torch.empty((K_SEL, 224, 224, 3), dtype=torch.bfloat16, device=dev)
-    rt_y = torch.empty(K_SEL, dtype=torch.int32, device=dev)
     stats = torch.zeros(2, dtype=torch.float32, device=dev)
     stream = torch.cuda.current_stream()
     n_global = K_SEL * world
@@ -294,9 +292,8 @@ def main():
         outs["exit_counts"] = out_counts
         app.infer(xi, taus, [outs])
         B.select_retrain(Xe, W, R, K_SEL, exclude=E, out_idx=sel_idx, out_dist=sel_dist, out_count=sel_cnt)
-        B.gather_rows(pool, sel_idx, sel_cnt, K_SEL, rt_x)
-        B.gather_rows(py, sel_idx, sel_cnt, K_SEL, rt_y)
-        m.retrain_step(rt_x, rt_y, n_global=n_global, lr=LR, stats=stats)
+        # (the pool keeps >= K_SEL eligible rows, so sel_idx holds K_SEL valid rows)
+        m.retrain_step_rows(pool, py, sel_idx, n_global=n_global, lr=LR, stats=stats)
 
     cnt_buf = torch.zeros((max(args.steps, 1) + args.warmup + 64, 4), dtype=torch.int32, device=dev)
     for i in range(args.warmup):
@@ -418,9 +415,7 @@ def main():
         "exit_head_train": K_SEL * sum(exit_bytes_row),
         # dT (bf16) + argmax codes read, dZ written at 112x112x64 (stem pool backward)
         "maxpool_bwd": K_SEL * (56 * 56 * 64 * 3 + 112 * 112 * 64 * 2),
-        # selected rows read from the pool and written to the retrain batch (+ labels)
-        "gather_rows": K_SEL * (224 * 224 * 3 * 2 * 2 + 8),
-        # raw NHWC bf16 in, space-to-depth packed rows out (inference + retraining batches)
+        # raw NHWC bf16 in, space-to-depth packed rows out (inference batch + the selected pool rows)
         "pack_input": (INF_B + K_SEL) * (224 * 224 * 3 * 2 + 112 * 112 * 16 * 2),
     }
     hbm_kernels = {}

@@ -203,6 +203,16 @@ adainf_status adainf_retrain_step(adainf_model_t m, const void* samples_bf16_nhw
                                   int32_t n_local, int64_t n_global, float lr,
                                   adainf_step_stats* stats_dev, adainf_stream_t stream);
 
+/* The retraining step on rows of a device-resident window pool (samples collected in the previous
+ * period), without materialising the batch: sample r of the step is pool row row_idx[r] (device int32[n_local],
+ * every entry a valid row, e.g. adainf_select_retrain's out_idx when out_count == k) and its label
+ * pool_labels[row_idx[r]].  The rows are read once, straight into the model's packed input layout.
+ * Same semantics, results and errors as adainf_retrain_step on the gathered batch; models whose input is used
+ * unpacked (in_c a multiple of 8) return ADAINF_ERR_UNSUPPORTED. */
+adainf_status adainf_retrain_step_rows(adainf_model_t m, const void* pool_bf16_nhwc, const int32_t* pool_labels,
+                                       const int32_t* row_idx, int32_t n_local, int64_t n_global, float lr,
+                                       adainf_step_stats* stats_dev, adainf_stream_t stream);
+
 /* Assemble the retraining batch from the device-resident window pool (samples collected in the
  * previous period): dst[r] = src[idx[r]] for r < min(*count, n) (count device int or NULL -> n);
  * rows of row_bytes bytes (multiple of 4; 16 for 128-bit copies).  Pairs with adainf_select_retrain's out_idx/out_count. */

@@ -98,6 +98,7 @@ def lib():
             "adainf_infer_dag": [vp, vp, i32, C.POINTER(C.c_float), i32, C.POINTER(ModelOut), vp],
             "adainf_select_retrain": [C.POINTER(SelectIn), i32, vp, vp, vp, vp, vp],
             "adainf_retrain_step": [vp, vp, vp, i32, i64, C.c_float, vp, vp],
+            "adainf_retrain_step_rows": [vp, vp, vp, vp, i32, i64, C.c_float, vp, vp],
             "adainf_dp_attach": [vp, vp, i32, i32],
             "adainf_nccl_unique_id": [vp],
             "adainf_gather_rows": [vp, vp, vp, i32, i64, vp, vp],
@@ -218,6 +219,12 @@ class Model:
         check(lib().adainf_retrain_step(self.h, ptr(samples), ptr(labels), int(samples.shape[0]),
                                         int(n_global or samples.shape[0]), float(lr), ptr(stats),
                                         stream_ptr(stream)))
+
+    def retrain_step_rows(self, pool, pool_labels, row_idx, n_global=None, lr=0.01, stats=None, stream=None):
+        """Retraining step on pool rows row_idx (device int32[n]) with labels pool_labels[row_idx]."""
+        n = int(row_idx.shape[0])
+        check(lib().adainf_retrain_step_rows(self.h, ptr(pool), ptr(pool_labels), ptr(row_idx), n,
+                                             int(n_global or n), float(lr), ptr(stats), stream_ptr(stream)))
 
     def dp_attach(self, uid: bytes, rank: int, world: int):
         buf = C.create_string_buffer(uid, 128)

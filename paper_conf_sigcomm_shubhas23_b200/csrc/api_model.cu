@@ -334,6 +334,17 @@ extern "C" adainf_status adainf_retrain_step(adainf_model_t m, const void* sampl
   });
 }
 
+extern "C" adainf_status adainf_retrain_step_rows(adainf_model_t m, const void* pool, const int32_t* pool_labels,
+                                                  const int32_t* row_idx, int32_t n_local, int64_t n_global, float lr,
+                                                  adainf_step_stats* stats, adainf_stream_t stream) {
+  return guard([&] {
+    if (!m || !pool || !pool_labels || !row_idx) throw InvalidError("retrain_step_rows: null argument");
+    if (!(lr == lr)) throw InvalidError("retrain: NaN lr");
+    require_device();
+    m->m.train_step_rows((const bf16*)pool, pool_labels, row_idx, n_local, n_global, lr, stats, (cudaStream_t)stream);
+  });
+}
+
 extern "C" adainf_status adainf_gather_rows(const void* src, const int32_t* idx, const int32_t* count, int32_t n,
                                             int64_t row_bytes, void* dst, adainf_stream_t stream) {
   return guard([&] {

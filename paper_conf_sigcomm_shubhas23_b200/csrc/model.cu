@@ -520,15 +520,31 @@ void Model::infer(const bf16* x, const int* in_map, const int* in_count, int n_s
 }
 
 // ------------------------------------------------------------------------------------------------
+void Model::train_step_rows(const bf16* pool, const int32_t* pool_labels, const int32_t* idx, int n,
+                            long long n_global, float lr, adainf_step_stats* stats, cudaStream_t st) {
+  if (!pack) throw UnsupportedError("retrain_step_rows: the model reads its input unpacked (in_c % 8 == 0)");
+  if (n <= 0 || n > max_batch) throw ShapeError("retrain: n_local must be in 1..max_batch");
+  if (!row_labels.p) row_labels.alloc((size_t)max_batch * 4);
+  launch_gather_rows(pool_labels, idx, nullptr, n, 4, row_labels.p, st);
+  train_step_impl(pool, idx, row_labels.as<int32_t>(), n, n_global, lr, stats, st);
+}
+
 void Model::train_step(const bf16* x, const int32_t* labels, int n, long long n_global, float lr,
                        adainf_step_stats* stats, cudaStream_t st) {
+  train_step_impl(x, nullptr, labels, n, n_global, lr, stats, st);
+}
+
+void Model::train_step_impl(const bf16* x, const int32_t* row_map, const int32_t* labels, int n, long long n_global,
+                            float lr, adainf_step_stats* stats, cudaStream_t st) {
   if (n <= 0 || n > max_batch) throw ShapeError("retrain: n_local must be in 1..max_batch");
   if (n_global < n) throw ShapeError("retrain: n_global < n_local");
   ensure_training();
   const bf16* x0 = x;
   if (pack) {
-    ingest(x, nullptr, nullptr, n, st);
+    ingest(x, row_map, nullptr, n, st);  // row_map: rows of a pool, packed straight into the model layout
     x0 = packed_in.as<bf16>();
+  } else if (row_map) {
+    throw UnsupportedError("retrain: row-mapped input needs a packed model input");
   }
   forward_nodes(x0, nullptr, nullptr, n, true, nullptr, nullptr, st);
   float* G = grads.as<float>();

@@ -129,6 +129,12 @@ struct Model {
              const adainf_model_out& out, cudaStream_t st, bool x_padded = false);
   void train_step(const bf16* x, const int32_t* labels, int n, long long n_global, float lr,
                   adainf_step_stats* stats, cudaStream_t st);
+  // the same step on pool rows idx[0..n) (packed straight from the pool; labels gathered from pool_labels)
+  void train_step_rows(const bf16* pool, const int32_t* pool_labels, const int32_t* idx, int n, long long n_global,
+                       float lr, adainf_step_stats* stats, cudaStream_t st);
+  DevBuf row_labels;  // labels of the rows of train_step_rows
+  void train_step_impl(const bf16* x, const int32_t* row_map, const int32_t* labels, int n, long long n_global,
+                       float lr, adainf_step_stats* stats, cudaStream_t st);
 
  private:
   void forward_nodes(const bf16* x0, const int* map0, const int* count0, int n_static, bool train, const float* taus,

@@ -109,3 +109,30 @@ def test_retrain_deterministic():
         outs.append(m.get_params())
         m.close()
     assert np.array_equal(outs[0], outs[1])
+
+
+def test_retrain_step_rows_equals_gathered_batch():
+    """adainf_retrain_step_rows (pool rows packed straight into the model layout, labels gathered on device)
+    gives bit-identical weights and statistics to gathering the rows and calling adainf_retrain_step."""
+    spec = S.resnet18_ee()
+    p = synth.init_params(spec, seed=21)
+    pool_b, pool_y = synth.drifted_images(40, 224, 224, 3, seed=21)
+    pool = torch.from_numpy(pool_b.view(np.int16)).cuda().view(torch.bfloat16)
+    labels = torch.from_numpy(pool_y).cuda()
+    idx = torch.tensor([3, 17, 0, 39, 22, 8, 8, 30, 11, 5, 26, 14], dtype=torch.int32, device="cuda")
+    n = idx.numel()
+    outs = []
+    for rows in (False, True):
+        m = B.Model(spec, n, params=p)
+        st = torch.zeros(2, dtype=torch.float32, device="cuda")
+        for _ in range(2):
+            if rows:
+                m.retrain_step_rows(pool, labels, idx, n_global=3 * n, lr=0.05, stats=st)
+            else:
+                m.retrain_step(pool[idx.long()].contiguous(), labels[idx.long()].contiguous(), n_global=3 * n, lr=0.05,
+                               stats=st)
+        torch.cuda.synchronize()
+        outs.append((m.get_params().copy(), st.cpu().clone()))
+        m.close()
+    assert np.array_equal(outs[0][0], outs[1][0])
+    assert torch.equal(outs[0][1], outs[1][1])
