@@ -126,7 +126,10 @@ static void launch_dualm_t(const ConvArgs& a, long long tiles, cudaStream_t st) 
 }
 template <int MODE>
 static bool try_launch_dualm(int BN, const ConvArgs& a, long long npix_static, cudaStream_t st) {
-  if (!dualm_on() || !a.a_tma || !a.b_tma || (BN != 128 && BN != 256) || a.K <= 4 * BK) return false;
+  if (!dualm_on() || !a.a_tma || !a.b_tma || (BN != 128 && BN != 256)) return false;
+  // short-K (1x1) launches are bound by per-tile waits / commits: sharing them between two M tiles helps too
+  // (layer-2 1x1/2 projection forward 137 -> 106 us); ADAINF_DUALM_SHORTK=0 restores the generic kernel
+  if (a.K <= 4 * BK && getenv("ADAINF_DUALM_SHORTK") && atoi(getenv("ADAINF_DUALM_SHORTK")) == 0) return false;
   // BN = 256 (single-buffered accumulators, 2 smem stages) measured slower than the generic kernel: opt-in only
   if (BN == 256 && !(getenv("ADAINF_DUALM256") && atoi(getenv("ADAINF_DUALM256")) == 1)) return false;
   const long long tiles = ((npix_static + 2 * BM - 1) / (2 * BM)) * ((a.Nout + BN - 1) / BN);

@@ -270,3 +270,37 @@ torch.save({{"y": y.cpu(), "dx": dx.cpu()}}, sys.argv[1])
     for name in ("dualm", "pair"):
         assert torch.equal(outs[name]["y"], outs["generic"]["y"]), name
         assert torch.equal(outs[name]["dx"], outs["generic"]["dx"]), name
+
+
+def test_dualm_short_k_projection_vs_torch():
+    """1x1 / stride-2 projection (K = 64, one K-block per tile) through the dual-M kernel (ADAINF_NARROW=0 keeps
+    BN = 128), against torch and bit-identical to the generic kernel (ADAINF_DUALM=0)."""
+    import os, subprocess, sys
+    code = f"""
+import sys, torch
+sys.path.insert(0, {os.path.dirname(os.path.dirname(os.path.abspath(__file__)))!r})
+from paper_conf_sigcomm_shubhas23_b200 import binding as B
+g = torch.Generator().manual_seed(3)
+x = torch.randn(5, 30, 30, 64, generator=g).to(torch.bfloat16).cuda()
+w = (torch.randn(128, 1, 1, 64, generator=g) * 0.1).to(torch.bfloat16).cuda()
+b = (torch.randn(128, generator=g) * 0.1).cuda()
+y = B.dbg_conv_fwd(x, w, b, 2, 0, act=0)
+torch.cuda.synchronize()
+torch.save(y.cpu(), sys.argv[1])
+"""
+    outs = {}
+    for name, extra in {"generic": {"ADAINF_DUALM": "0"}, "dualm": {"ADAINF_DUALM": "1"}}.items():
+        path = f"/tmp/proj_{name}.pt"
+        env = dict(os.environ, ADAINF_NARROW="0", **extra)
+        r = subprocess.run([sys.executable, "-c", code, path], env=env, capture_output=True, text=True, timeout=300)
+        assert r.returncode == 0, r.stderr[-2000:]
+        outs[name] = torch.load(path)
+    g = torch.Generator().manual_seed(3)
+    x = torch.randn(5, 30, 30, 64, generator=g).to(torch.bfloat16)
+    w = (torch.randn(128, 1, 1, 64, generator=g) * 0.1).to(torch.bfloat16)
+    b = torch.randn(128, generator=g) * 0.1
+    ref = torch.nn.functional.conv2d(x.float().permute(0, 3, 1, 2), w.float().permute(0, 3, 1, 2), b,
+                                     stride=2).permute(0, 2, 3, 1)
+    for o in outs.values():
+        assert (o.float() - ref).norm() / ref.norm() < 1e-2
+    assert torch.equal(outs["dualm"], outs["generic"])
