@@ -793,6 +793,7 @@ struct WgPlan {
   int BN;          // WG_TMA / WG_GENERIC
   int Wp, R, rg;   // TMA paths
   int i2c;         // WG_TMA: K-blocks of 64 consecutive output pixels via im2col TMA
+  int pm = 1;      // WG_TMA: 128-row M tiles per tile (2: two M tiles share each dZ K-block)
 };
 
 static bool win_wgrad_ok(const ConvGeom& g) {
@@ -871,7 +872,15 @@ static WgPlan plan_wgrad(const ConvGeom& g, int n) {
       p.nkb = (int)(((long long)n * g.Ho * g.Wo + 63) / 64);
     }
     p.BN = g.Cout <= 64 ? 64 : (g.Cout <= 128 ? 128 : 256);
-    p.tiles = ((p.Kconv + 127) / 128) * ((g.Cout + p.BN - 1) / p.BN);
+    {
+      static int env_pm = -1;  // ADAINF_WG_PM=1 keeps one M tile per tile
+      if (env_pm < 0) {
+        const char* e = getenv("ADAINF_WG_PM");
+        env_pm = e ? atoi(e) : 2;
+      }
+      p.pm = (env_pm == 2 && p.BN >= 128 && (p.Kconv + 127) / 128 >= 3) ? 2 : 1;  // 1x1 (<= 2 M tiles): 1
+    }
+    p.tiles = (((p.Kconv + 127) / 128 + p.pm - 1) / p.pm) * ((g.Cout + p.BN - 1) / p.BN);
     finish_splits(p);
     return p;
   }
@@ -912,20 +921,21 @@ size_t wgrad_ws_bytes(const ConvGeom& g, int n) {
   return wgrad_ws_floats(p, g, n, nullptr, nullptr) * sizeof(float);
 }
 
-template <int BN>
+template <int BN, int PM>
 static void launch_wgrad_tma_t(WgTmaArgs& a, cudaStream_t st) {
-  constexpr int STAGE = 16384 + BN * 128;
+  constexpr int STAGE = PM * 16384 + BN * 128;
   a.stages = std::min(16, (225 * 1024 - 5120) / STAGE);
   const int smem = a.stages * STAGE + 2048 + 3072;
   static bool attr = false;
   if (!attr) {
-    CK(cudaFuncSetAttribute(conv_wgrad_tma_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    CK(cudaFuncSetAttribute(conv_wgrad_tma_kernel<BN, PM>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
     attr = true;
   }
-  const long long units = (long long)((a.Kconv + 127) / 128) * ((a.Cout + BN - 1) / BN) * a.splits;
+  const long long units =
+      (long long)(((a.Kconv + 127) / 128 + PM - 1) / PM) * ((a.Cout + BN - 1) / BN) * a.splits;
   dim3 grid((unsigned)std::max(1LL, std::min<long long>(units, num_sms())));
   ProfScope ps(PC_CONV_WGRAD, st);
-  conv_wgrad_tma_kernel<BN><<<grid, NUM_THREADS, smem, st>>>(a);
+  conv_wgrad_tma_kernel<BN, PM><<<grid, NUM_THREADS, smem, st>>>(a);
   CK(cudaGetLastError());
 }
 
@@ -1004,9 +1014,14 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
       a.x_map = make_tmap_nhwc(x, n, g.H, g.W, g.Cin, 64, p.Wp, p.R, g.stride);
       a.dz_map = make_tmap_nhwc(dz, n, g.Ho, g.Wo, g.Cout, 64, p.Wp, p.R, 1);
     }
-    if (p.BN == 64) launch_wgrad_tma_t<64>(a, st);
-    else if (p.BN == 128) launch_wgrad_tma_t<128>(a, st);
-    else launch_wgrad_tma_t<256>(a, st);
+    if (p.BN == 64) launch_wgrad_tma_t<64, 1>(a, st);
+    else if (p.BN == 128) {
+      if (p.pm == 2) launch_wgrad_tma_t<128, 2>(a, st);
+      else launch_wgrad_tma_t<128, 1>(a, st);
+    } else {
+      if (p.pm == 2) launch_wgrad_tma_t<256, 2>(a, st);
+      else launch_wgrad_tma_t<256, 1>(a, st);
+    }
   } else if (p.path == WG_WIN_CPASYNC) {
     // one K-range of 64-position blocks per persistent CTA; partials [S][576][64] reduced in fixed order
     WinArgs w{};
@@ -1073,7 +1088,7 @@ void conv_wgrad(const ConvGeom& g, const bf16* x, const bf16* dz, int n, int cin
   }
   if (db) {
     ProfScope ps(PC_BIAS_COLSUM, st, fused_cs ? 1 : 2);
-    int nb = p.path == WG_TMA ? S * ((p.Kconv + 127) / 128) : S;  // fused partial rows
+    int nb = p.path == WG_TMA ? S * (((p.Kconv + 127) / 128 + p.pm - 1) / p.pm) : S;  // fused partial rows
     if (!fused_cs) {
       nb = colsum_blocks(npix);
       const long long rpb = (npix + nb - 1) / nb;

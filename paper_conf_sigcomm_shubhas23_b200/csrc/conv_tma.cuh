@@ -528,9 +528,13 @@ struct WgTmaArgs {
   int i2c, lo;
 };
 
-template <int BN>
+// PM = M tiles (128 kconv rows each) per tile: PM = 2 shares each dZ (B) K-block between two M tiles (fewer TMA
+// bytes per MAC; 8 MMAs per full-barrier wait / commit); accumulators double-buffered when they fit in TMEM.
+template <int BN, int PM = 1>
 __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __grid_constant__ WgTmaArgs a) {
-  constexpr int A_BYTES = 16384, B_BYTES = BN * 128, STAGE = A_BYTES + B_BYTES;
+  constexpr int A_BYTES = PM * 16384, B_BYTES = BN * 128, STAGE = A_BYTES + B_BYTES;
+  constexpr int NBUF = 2 * PM * BN <= 512 ? 2 : 1;  // accumulator buffers
+  constexpr int TCOLS = PM * BN * NBUF;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   const int ST = a.stages;
@@ -542,7 +546,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
   float* cs_red = (float*)((uint8_t*)full + 512);  // [NPH][BN] column-sum combine scratch (3 KB)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int mt = (a.Kconv + 127) / 128, nt = (a.Cout + BN - 1) / BN;
+  const int mt1 = (a.Kconv + 127) / 128;        // 128-row M tiles
+  const int mt = (mt1 + PM - 1) / PM, nt = (a.Cout + BN - 1) / BN;
   const int ntile = mt * nt * a.splits;
   const int nkb = a.n * a.rg;
   if ((int)blockIdx.x >= ntile) return;
@@ -559,7 +564,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
     tma_prefetch_desc(&a.x_map);
     tma_prefetch_desc(&a.dz_map);
   }
-  if (warp == 4) tmem_alloc<2 * BN>(tmem_slot);
+  if (warp == 4) tmem_alloc<TCOLS>(tmem_slot);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -572,22 +577,23 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
       for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x) {
         const int nb = tile % nt, r = tile / nt, m = r % mt, z = r / mt;
         const int kb0 = z * a.kb_per_split, kb1 = min(kb0 + a.kb_per_split, nkb);
-        // the two A atoms of this M tile: (tap, ci block) = divmod(m*2 + i, ncb)
-        int ax[2], ay[2], ac[2];
-        bool av[2];
-        for (int i = 0; i < 2; ++i) {
-          const int at = m * 2 + i;
+        // the 2*PM A atoms of this tile: (tap, ci block) = divmod(m*2*PM + i, ncb)
+        int ax[2 * PM], ay[2 * PM], ac[2 * PM];
+        bool av[2 * PM];
+        for (int i = 0; i < 2 * PM; ++i) {
+          const int at = m * 2 * PM + i;
           const int tap = at / a.ncb, cb = at - tap * a.ncb;
           av[i] = at * 64 < a.Kconv;
           ac[i] = cb * 64;
           ax[i] = (tap % a.KW) - a.pad;
           ay[i] = (tap / a.KW) - a.pad;
         }
+        int nA = 0;
+        for (int i = 0; i < 2 * PM; ++i) nA += av[i] ? 1 : 0;
         for (int kb = kb0; kb < kb1; ++kb, ++it) {
           const int s = it % ST, u = it / ST;
           if (u > 0) mbar_wait(&empty[s], (u - 1) & 1);
           const uint32_t sa = sbase + s * STAGE, sb = sa + A_BYTES;
-          const int nA = av[1] ? 2 : 1;
           mbar_expect_tx(&full[s], nA * 8192 + (BN / 64) * 8192);
           if (a.i2c) {
             const int p0 = kb * 64, HWo = a.Ho * a.Wo;
@@ -613,12 +619,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
     constexpr uint32_t IDESC = make_idesc(BM, BN, 1, 1);
     int it = 0, lt = 0;
     for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++lt) {
-      const int r = tile / nt, z = r / mt;
+      const int r = tile / nt, m = r % mt, z = r / mt;
       const int kb0 = z * a.kb_per_split, kb1 = min(kb0 + a.kb_per_split, nkb);
-      const int b = lt & 1, ub = lt >> 1;
+      const int b = NBUF == 2 ? (lt & 1) : 0, ub = NBUF == 2 ? (lt >> 1) : lt;
       if (ub > 0) mbar_wait(&tempty[b], (ub - 1) & 1);
       tc_fence_after();
-      const uint32_t dacc = tmem + (uint32_t)(b * BN);
+      const uint32_t dacc = tmem + (uint32_t)(b * PM * BN);
+      const bool second = PM == 2 && (m * 2 + 1) < mt1;  // the second M tile exists
       for (int kb = kb0; kb < kb1; ++kb, ++it) {
         const int s = it % ST, u = it / ST;
         mbar_wait(&full[s], u & 1);
@@ -627,8 +634,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
           const uint32_t sa = sbase + s * STAGE, sb = sa + A_BYTES;
           const uint64_t ad0 = make_sdesc(sa, 8192, 1024), bd0 = make_sdesc(sb, 8192, 1024);
 #pragma unroll
-          for (int kk = 0; kk < 4; ++kk)
+          for (int kk = 0; kk < 4; ++kk) {
             umma_bf16(dacc, ad0 + kk * 128u, bd0 + kk * 128u, IDESC, (kb != kb0 || kk != 0));
+            if (PM == 2 && second)  // A atoms 2, 3 (16 KB further): the second M tile
+              umma_bf16(dacc + BN, ad0 + (16384u >> 4) + kk * 128u, bd0 + kk * 128u, IDESC, (kb != kb0 || kk != 0));
+          }
           umma_commit(&empty[s]);
           if (kb == kb1 - 1) umma_commit(&tfull[b]);
         }
@@ -639,8 +649,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
     }
   } else if (warp >= 1 && warp <= 3) {
     if (a.cs_part) {
-      // fused bias gradient: the mt M tiles of one (co block, split) see the same dZ K-blocks; M tile m
-      // sums the K-blocks with kb % mt == m into partial row z * mt + m
+      // fused bias gradient: the mt tiles of one (co block, split) see the same dZ K-blocks; tile m sums the
+      // K-blocks with kb % mt == m into partial row z * mt + m
       TileColsum<BN> cs;
       const int t = threadIdx.x - 32;
       cs.init(t);
@@ -666,26 +676,30 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
     for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++lt) {
       const int nb = tile % nt, r = tile / nt, m = r % mt, z = r / mt;
       const int kb0 = z * a.kb_per_split, kb1 = min(kb0 + a.kb_per_split, nkb);
-      const int b = lt & 1, ub = lt >> 1;
+      const int b = NBUF == 2 ? (lt & 1) : 0, ub = NBUF == 2 ? (lt >> 1) : lt;
       mbar_wait(&tfull[b], ub & 1);
       tc_fence_after();
-      const uint32_t trow = tmem + (uint32_t)(b * BN) + ((uint32_t)(qd * 32) << 16);
-      const int kc = m * 128 + row;
-      float* outp = a.out + ((long long)z * a.Kconv + kc) * a.Cout + nb * BN;
 #pragma unroll 1
-      for (int c0 = 0; c0 < BN; c0 += 32) {
-        float v[32];
-        if (kb1 > kb0) tmem_ld32(trow + c0, v);
-        else
+      for (int h = 0; h < PM; ++h) {
+        const uint32_t trow = tmem + (uint32_t)(b * PM * BN + h * BN) + ((uint32_t)(qd * 32) << 16);
+        const int kc = (m * PM + h) * 128 + row;
+        float* outp = a.out + ((long long)z * a.Kconv + kc) * a.Cout + nb * BN;
+#pragma unroll 1
+        for (int c0 = 0; c0 < BN; c0 += 32) {
+          float v[32];
+          const bool live = kb1 > kb0 && (h == 0 || (m * PM + h) < mt1);
+          if (live) tmem_ld32(trow + c0, v);
+          else
 #pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] = 0.f;
-        if (c0 + 32 >= BN) {
-          tc_fence_before();
-          mbar_arrive(&tempty[b]);
+            for (int i = 0; i < 32; ++i) v[i] = 0.f;
+          if (h == PM - 1 && c0 + 32 >= BN) {
+            tc_fence_before();
+            mbar_arrive(&tempty[b]);
+          }
+          if (kc < a.Kconv && nb * BN + c0 < a.Cout)
+#pragma unroll
+            for (int i = 0; i < 32; i += 4) *(float4*)(outp + c0 + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
         }
-        if (kc < a.Kconv && nb * BN + c0 < a.Cout)
-#pragma unroll
-          for (int i = 0; i < 32; i += 4) *(float4*)(outp + c0 + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
       }
     }
   }
@@ -694,10 +708,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
   __syncthreads();
   if (warp == 4) {
     tc_fence_after();
-    tmem_dealloc<2 * BN>(tmem);
+    tmem_dealloc<TCOLS>(tmem);
   }
 }
-
 
 // ---- window weight gradient (stride-1 3x3, pad 1), TMA-fed --------------------------------------------
 // dW[tap][ci][co] = sum_pix X(pix + tap) * dZ(pix).  K = output pixels of R rows of one image on a padded
