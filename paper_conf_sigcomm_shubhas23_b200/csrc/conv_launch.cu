@@ -804,7 +804,8 @@ static bool tma_wgrad_allowed() { return win_mode() != 4 && win_mode() != 5; }
 static bool win_tma_wgrad_ok(const ConvGeom& g) {
   return tma_wgrad_allowed() && win_mode() != 6 && g.KH == 3 && g.KW == 3 && g.stride == 1 && g.pad == 1 &&
          g.Cin % 64 == 0 && g.Cout % 64 == 0 && g.H == g.Ho && g.W == g.Wo && g.W <= 127 &&
-         (g.W >= 14 || win_mode() == 7);  // below 14 columns the padded window wastes too much (mode 7 forces)
+         ((g.W >= 14 && g.Cout < 256) || win_mode() == 7);  // below 14 columns the padded window wastes too much;
+  // from Cout = 256 the two-M-tile TMA GEMM (N = 256) beats the N = 64 window kernel (181 vs 263 us, layer 3)
 }
 static bool wgrad_tma_ok(const ConvGeom& g) {
   return tma_wgrad_allowed() && g.Cin % 64 == 0 && g.Cout % 64 == 0 && g.Wo <= 64 && g.stride <= 2;
