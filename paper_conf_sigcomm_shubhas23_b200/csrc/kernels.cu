@@ -378,13 +378,15 @@ __global__ void __launch_bounds__(EH_THREADS) exit_head_kernel(const ExitHeadArg
 void launch_exit_head(const ExitHeadArgs& a, cudaStream_t st, int prof_class) {
   if (a.n_static <= 0) return;
   const bool wide = a.n_static < 4 * num_sms();
-  const int T = wide ? 512 : 128;
+  const bool widest = a.n_static <= 2 * num_sms();  // a row per CTA cannot fill the SMs: 1,024 threads per row
+  const int T = widest ? 1024 : (wide ? 512 : 128);
   if (a.C % 8 || (T % (a.C / 8)) != 0 || a.C / 8 > 128)
     throw ShapeError("exit head: C must be 8 * a power of two <= 1024");
   const int groups = T / (a.C / 8);
   const size_t smem = (size_t)(groups * a.C + a.C + a.ncls) * sizeof(float);
   ProfScope ps(prof_class, st);
-  if (wide) exit_head_kernel<512><<<a.n_static, 512, smem, st>>>(a);
+  if (widest) exit_head_kernel<1024><<<a.n_static, 1024, smem, st>>>(a);
+  else if (wide) exit_head_kernel<512><<<a.n_static, 512, smem, st>>>(a);
   else exit_head_kernel<128><<<a.n_static, 128, smem, st>>>(a);
   CK(cudaGetLastError());
 }
