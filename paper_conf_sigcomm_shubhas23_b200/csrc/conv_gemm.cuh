@@ -97,7 +97,8 @@ struct ConvCfg {
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   // coalescing buffers of the bf16 epilogue: 4 warps x 2 operands x (32 rows x 128 B), double-buffered in
   // the sub-pixel dgrad mode
-  static constexpr int EPI_BYTES = (MODE != 2 && BN >= 64) ? (MODE == 3 && EW == 1 ? 4 * 16384 : 4 * EW * 8192) : 0;
+  static constexpr int EPI_BYTES =
+      (MODE != 2 && BN >= 64) ? ((MODE == 3 || MODE == 1) && EW == 1 ? 4 * 16384 : 4 * EW * 8192) : 0;
   static constexpr int STAGES_FIT = (220 * 1024 - EPI_BYTES - 1280) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_FIT > 8 ? 8 : STAGES_FIT;
   static constexpr int BIAS_BYTES = (MODE == 0 && EPI_BYTES > 0) ? 4096 : 0;  // FWD bias vector (Nout <= 1024)
@@ -237,7 +238,7 @@ __device__ __forceinline__ EpiBlk epi_block(const ConvArgs& a, int cb, long long
 // into per-warp buffers; in the sub-pixel mode (short K, epilogue-heavy tiles) they are double-buffered: the
 // first block's operands are requested before waiting for the accumulator, block c+1's while block c is
 // combined, so the epilogue does not pay a memory latency per column block.
-template <int MODE, int BN, int EW>
+template <int MODE, int BN, int EW, bool PIPE_DG = false>
 __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const TileInfo& ti, uint32_t trow,
                                                    uint64_t* tfull_b, uint32_t tpar, uint64_t* tempty_b, int nkb,
                                                    long long m, bool rv, int n, long long orow, long long rrow,
@@ -250,7 +251,7 @@ __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const Tile
   };
   // EW warps per lane quadrant: this warp takes column blocks h*64, h*64 + 64*EW, ...; with two warps the
   // staging is single-buffered (the other warp of the quadrant overlaps its latency)
-  constexpr bool PIPE = MODE == MODE_DGRAD_SP && EW == 1;
+  constexpr bool PIPE = (MODE == MODE_DGRAD_SP || (MODE == MODE_DGRAD && PIPE_DG)) && EW == 1;
   constexpr int STEP = 64 * EW;
   const int first = h * 64;
   if (first >= BN) {  // no block for this warp: release the accumulator in order
@@ -751,7 +752,7 @@ __global__ void __launch_bounds__(gemm_threads(EW), 1) conv_umma_kernel(const __
         }
         if constexpr (Cfg::EPI_BYTES > 0) {
           if (coalesced) {
-            epilogue_coalesced<MODE, BN, EW>(a, ti, trow, &tfull[b], ub & 1, &tempty[b], nkb, m, rv, n, orow, rrow,
+            epilogue_coalesced<MODE, BN, EW, true>(a, ti, trow, &tfull[b], ub & 1, &tempty[b], nkb, m, rv, n, orow, rrow,
                                           HWg, epi_smem + (warp - 5) * (Cfg::EPI_BYTES / (4 * EW)), lane, bias_s, h);
             continue;
           }
