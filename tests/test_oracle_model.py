@@ -30,14 +30,37 @@ def test_param_counts_match_survey():
     assert abs(sum(S.macs_per_sample(S.tiny_yolo_det())) / 1e6 - 1693.6) < 2.0
 
 
-def torch_forward(spec, params, x, exact):
-    """Independent fp64 interpreter built from torch.nn.functional (NCHW), bf16 rounding emulated at
-    the storage points (activations, conv weights) unless exact."""
+class _GradRound(torch.autograd.Function):
+    """Identity forward; backward rounds the incoming gradient to bf16 (a gradient storage point,
+    DESIGN.md §Readings "Gradient storage points")."""
+
+    @staticmethod
+    def forward(ctx, x):
+        return x.clone()
+
+    @staticmethod
+    def backward(ctx, g):
+        return g.float().to(torch.bfloat16).double()
+
+
+def torch_forward(spec, params, x, exact, want_det=False):
+    """Independent fp64 interpreter built from torch.nn.functional (NCHW).  Unless ``exact``, bf16 / fp32
+    rounding is emulated at the storage points (activations, conv weights) by straight-through rounding,
+    and the backward rounds to bf16 where the method stores gradients (dZ after the activation mask, the
+    pooled tensor's gradient before the max-pool routing, the projection shortcut's dgrad), so autograd
+    yields the bf16-storage gradient the oracle's hand-written backward computes.  Leaky-ReLU slope is
+    the fp32 0.1f product (c.1 step 2); a conv followed by DET_HEAD keeps its fp32 output."""
+    def ste(t, fn):
+        return t if exact else t + (fn(t) - t).detach()
+
     def R(t):
-        return t if exact else t.float().to(torch.bfloat16).double()
+        return ste(t, lambda u: u.float().to(torch.bfloat16).double())
 
     def Fp(t):
-        return t if exact else t.float().double()
+        return ste(t, lambda u: u.float().double())
+
+    def GR(t):
+        return t if exact else _GradRound.apply(t)
 
     segs = {(k, i): (off, shp) for k, i, off, shp in S.param_segments(spec)}
 
@@ -46,39 +69,70 @@ def torch_forward(spec, params, x, exact):
         return params[off:off + int(np.prod(shp))].reshape(shp)
 
     cur = R(x.permute(0, 3, 1, 2))
-    blocks, outs = [], []
-    for i, o in enumerate(spec["ops"]):
+    blocks, outs, det = [], [], None
+    ops = spec["ops"]
+    for i, o in enumerate(ops):
         k = o["kind"]
         if k == "conv":
-            w = seg("conv_w", i).permute(0, 3, 1, 2)
-            w = w if exact else w.float().to(torch.bfloat16).double()
+            w = R(seg("conv_w", i).permute(0, 3, 1, 2))
             v = Fp(Fp(F.conv2d(cur, w, stride=o["stride"], padding=o["pad"])) + seg("conv_b", i)[None, :, None, None])
             if o["residual"]:
                 v = Fp(v + blocks.pop())
+            v = GR(v)
             if o["act"] == 1:
                 v = torch.relu(v)
             elif o["act"] == 2:
-                v = torch.where(v > 0, v, 0.1 * v)
-            cur = R(v)
+                neg = 0.1 * v if exact else (v.float() * torch.tensor(0.1, dtype=torch.float32)).double()
+                neg = neg if exact else v * 0.1 + (neg - v * 0.1).detach()
+                v = torch.where(v > 0, v, neg)
+            fp32_out = i + 1 < len(ops) and ops[i + 1]["kind"] == "det_head"
+            cur = Fp(v) if fp32_out else R(v)
         elif k == "maxpool":
-            cur = F.max_pool2d(cur, o["kh"], o["stride"], o["pad"])
+            cur = GR(F.max_pool2d(cur, o["kh"], o["stride"], o["pad"]))
         elif k == "block":
             if o["cout"] > 0:
-                w = seg("proj_w", i).permute(0, 3, 1, 2)
-                w = w if exact else w.float().to(torch.bfloat16).double()
-                blocks.append(R(Fp(Fp(F.conv2d(cur, w, stride=o["stride"])) + seg("proj_b", i)[None, :, None, None])))
+                w = R(seg("proj_w", i).permute(0, 3, 1, 2))
+                blocks.append(R(Fp(Fp(F.conv2d(GR(cur), w, stride=o["stride"])) +
+                                   seg("proj_b", i)[None, :, None, None])))
             else:
                 blocks.append(cur)
         elif k == "exit":
-            pooled = cur.mean(dim=(2, 3))
-            outs.append(pooled @ seg("exit_w", i) + seg("exit_b", i))
-    return outs
+            pooled = Fp(cur.mean(dim=(2, 3)))
+            outs.append(Fp(pooled @ seg("exit_w", i) + seg("exit_b", i)))
+        elif k == "det_head":
+            det = cur.permute(0, 2, 3, 1)
+    return (outs, det) if want_det else outs
 
 
-@pytest.mark.parametrize("which", ["mini", "tiny"])
+def stem_spec():
+    """ResNet stem geometry (7x7/2 pad-3 conv + ReLU, padded 3x3/2/1 max-pool with first-max routing),
+    a leaky-ReLU conv, identity and projection residual blocks, two exits."""
+    ops = [S.conv(7, 8, stride=2, pad=3), S.maxpool(3, 2, 1), S.exit_(4), S.block(0), S.conv(3, 8, act=S.LEAKY),
+           S.conv(3, 8, residual=True), S.block(12, 2), S.conv(3, 12, stride=2, act=S.LEAKY),
+           S.conv(3, 12, residual=True), S.exit_(4)]
+    return {"name": "stem", "in_h": 19, "in_w": 21, "in_c": 3, "ops": ops}
+
+
+def det_spec():
+    """TinyYOLOv3-like detector in miniature (reading Q18): leaky-ReLU convs, 2x2/2 and 3x3/1/1 pools,
+    fp32 1x1 head output into DET_HEAD."""
+    ops = [S.conv(3, 8, act=S.LEAKY), S.maxpool(2, 2), S.conv(3, 16, act=S.LEAKY), S.maxpool(3, 1, 1),
+           S.conv(1, 16, act=S.LEAKY), S.conv(3, 16, act=S.LEAKY), S.conv(1, 2 * (5 + 2), act=S.NONE),
+           {"kind": "det_head", "anchors": 2, "det_classes": 2, "grid_stride": 2, "anchor_wh": [3.0, 4.0, 6.0, 5.0]}]
+    return {"name": "det", "in_h": 12, "in_w": 12, "in_c": 3, "ops": ops}
+
+
+SPECS = {"mini": mini_spec, "tiny": S.tiny_cnn_ee, "stem": stem_spec,
+         "resnet32": lambda: S.resnet18_ee(in_hw=32), "resnet64": lambda: S.resnet18_ee(in_hw=64)}
+
+
+@pytest.mark.parametrize("which", ["mini", "tiny", "stem", "resnet32", "resnet64"])
 def test_forward_vs_torch_interpreter(which):
-    spec = mini_spec() if which == "mini" else S.tiny_cnn_ee()
-    B = 6
+    """c.1 steps 2-3 at model level, including the ResNet stem geometry (7x7/2/3 conv, 3x3/2/1 padded
+    max-pool), leaky-ReLU and every residual form: a padding, pool-window or slope mistake in the
+    oracle's own loops (Engine::forward, separate from the pinned primitives) fails here."""
+    spec = SPECS[which]()
+    B = 3 if which == "resnet64" else 6
     p = synth.init_params(spec, seed=3)
     xb, _ = synth.drifted_images(B, spec["in_h"], spec["in_w"], 3, num_classes=4, seed=1)
     x = synth.bf16_bits_to_f32(xb)
@@ -91,14 +145,42 @@ def test_forward_vs_torch_interpreter(which):
         np.testing.assert_allclose(got["conf"][:, k], pr.max(1).values.numpy(), rtol=1e-3, atol=1e-3)
 
 
-def test_exact_grad_vs_autograd_and_fd():
-    """c.1 steps 10-11: the backward derivation (CE over all exits, head grads, GAP broadcast, ReLU
-    mask, first-max maxpool routing, residual copy, projection dgrad, conv dgrad/wgrad) against
-    torch.autograd (fp64, exact arithmetic) and central finite differences."""
-    spec = mini_spec()
+def test_forward_detector_vs_torch_interpreter():
+    """Leaky-ReLU (fp32 0.1f slope) detector backbone and the fp32 (un-rounded) head output that feeds
+    DET_HEAD (c.1 steps 2 and 6, reading Q18): the oracle's det_raw against the torch interpreter."""
+    spec = det_spec()
+    p = synth.init_params(spec, seed=4)
+    xb, _ = synth.drifted_images(4, 12, 12, 3, num_classes=4, seed=6)
+    x = synth.bf16_bits_to_f32(xb)
+    got = O.Model(spec).forward(p, x, want_det=True)["det"]
+    _, det = torch_forward(spec, torch.from_numpy(p.astype(np.float64)), torch.from_numpy(x.astype(np.float64)),
+                           False, want_det=True)
+    ref = det.numpy()
+    assert got.shape == ref.shape
+    # fp32 output: differences come only from rare bf16 flips upstream (fp64 vs fp32 intermediate sums)
+    assert np.linalg.norm(got - ref) <= 1e-3 * np.linalg.norm(ref)
+    # the head output is not bf16-rounded: most values carry more than 8 mantissa bits
+    assert (synth.round_bf16(got) != got).mean() > 0.5
+    # a wrong slope (0.01 or 1.0) moves the output by far more than the tolerance
+    neg = (ref < 0).mean()
+    assert 0.05 < neg < 0.95
+
+
+def _labels(n, ncls, seed):
+    return np.random.default_rng(seed).integers(0, ncls, n).astype(np.int32)
+
+
+@pytest.mark.parametrize("which", ["mini", "stem"])
+def test_exact_grad_vs_autograd_and_fd(which):
+    """c.1 steps 10-11: the backward derivation (CE over all exits, head grads, GAP broadcast, ReLU and
+    leaky-ReLU masks, first-max max-pool routing incl. the padded 3x3/2/1 stem pool, residual copy,
+    projection dgrad, conv dgrad/wgrad incl. 7x7/2/3) against torch.autograd (fp64, exact arithmetic)
+    and central finite differences."""
+    spec = SPECS[which]()
     B = 5
     p = synth.init_params(spec, seed=5).astype(np.float64)
-    xb, y = synth.drifted_images(B, 8, 8, 3, num_classes=4, seed=2)
+    xb, _ = synth.drifted_images(B, spec["in_h"], spec["in_w"], 3, num_classes=4, seed=2)
+    y = _labels(B, 4, 2)
     x = synth.bf16_bits_to_f32(xb)
     m = O.Model(spec)
     g = m.grad_exact(p, x, y, n_global=7)
@@ -119,21 +201,56 @@ def test_exact_grad_vs_autograd_and_fd():
         assert abs(fd - g[j]) <= 1e-6 + 1e-4 * abs(g[j]), (j, fd, g[j])
 
 
-def test_bf16_grads_close_to_exact():
-    """The bf16-storage gradient (what the GPU must match) stays within the 2e-2 band of the exact one
-    per parameter tensor on the tiny CNN — guards against a rounding point that destroys the signal."""
-    spec = S.tiny_cnn_ee()
-    B = 8
+@pytest.mark.parametrize("which", ["mini", "tiny", "stem", "resnet32"])
+def test_bf16_storage_grads_vs_torch_emulation(which):
+    """The bf16-storage gradient (what the GPU must match) against
+    torch.autograd over the interpreter with the same rounding points emulated (straight-through bf16 /
+    fp32 rounding forward, bf16 rounding of dZ after the activation mask, of the pooled gradient before
+    the max-pool routing and of the projection dgrad).  Per parameter tensor within 1e-3: a misplaced
+    or missing rounding point (each moves a tensor by ~2^-9 relative per element) fails here."""
+    spec = SPECS[which]()
+    B = 4
     p = synth.init_params(spec, seed=7)
-    xb, y = synth.drifted_images(B, 32, 32, 3, num_classes=10, seed=3)
+    ncls = next(o["num_classes"] for o in spec["ops"] if o["kind"] == "exit")
+    xb, _ = synth.drifted_images(B, spec["in_h"], spec["in_w"], 3, num_classes=ncls, seed=3)
+    y = _labels(B, ncls, 3)
     x = synth.bf16_bits_to_f32(xb)
     m = O.Model(spec)
-    _, _, g16, _ = m.retrain_step(p, np.zeros_like(p), x, y, lr=0.0)
-    ge = m.grad_exact(synth.round_bf16(p).astype(np.float64), x, y)
+    _, _, g16, loss16 = m.retrain_step(p, np.zeros_like(p), x, y, n_global=6, lr=0.0)
+    pt = torch.from_numpy(p.astype(np.float64)).requires_grad_(True)
+    outs = torch_forward(spec, pt, torch.from_numpy(x.astype(np.float64)), False)
+    yt = torch.from_numpy(y.astype(np.int64))
+    loss = sum(F.cross_entropy(lg, yt, reduction="sum") for lg in outs) / 6
+    loss.backward()
+    gt = pt.grad.numpy()
+    assert abs(loss16 - loss.item()) <= 1e-5 * abs(loss.item())
+    ge = m.grad_exact(synth.round_bf16(p).astype(np.float64), x, y, n_global=6)
+    worst = 0.0
     for kind, _i, off, shp in S.param_segments(spec):
         n = int(np.prod(shp))
-        a, b = g16[off:off + n], ge[off:off + n]
-        assert np.linalg.norm(a - b) <= 5e-2 * np.linalg.norm(b) + 1e-9, kind
+        a, b, e = g16[off:off + n], gt[off:off + n], ge[off:off + n]
+        err = np.linalg.norm(a - b) / (np.linalg.norm(b) + 1e-30)
+        worst = max(worst, err)
+        assert err <= 1e-3, (kind, _i, err)
+        # sanity: the storage noise itself does not destroy the signal (0.5-5% per tensor at 32x32; the
+        # 8x8 / 19x21 specs' tiny maps push it above 10%, DESIGN.md §Numerics, so they skip this check)
+        if which == "tiny":
+            assert np.linalg.norm(a - e) <= 5e-2 * np.linalg.norm(e) + 1e-9, kind
+    # the emulation is sensitive: dropping the dZ rounding changes some tensor by well over 1e-3
+    # (checked once on the tiny CNN so the pin cannot pass vacuously)
+    if which == "tiny":
+        pt2 = torch.from_numpy(p.astype(np.float64)).requires_grad_(True)
+        saved = _GradRound.backward
+        try:
+            _GradRound.backward = staticmethod(lambda ctx, g: g)
+            outs2 = torch_forward(spec, pt2, torch.from_numpy(x.astype(np.float64)), False)
+            (sum(F.cross_entropy(lg, yt, reduction="sum") for lg in outs2) / 6).backward()
+        finally:
+            _GradRound.backward = saved
+        g2 = pt2.grad.numpy()
+        diffs = [np.linalg.norm(g16[o:o + int(np.prod(s))] - g2[o:o + int(np.prod(s))]) /
+                 np.linalg.norm(g2[o:o + int(np.prod(s))]) for _k, _i, o, s in S.param_segments(spec)]
+        assert max(diffs) > 3 * max(worst, 1e-4), (max(diffs), worst)
 
 
 def test_sgd_vs_torch_optim():
