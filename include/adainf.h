@@ -21,9 +21,12 @@
  *     memory; the library never reads them back on the hot path.
  *   - Errors: every call returns an adainf_status; 0 = OK.  Argument/shape validation is synchronous.
  *     CUDA errors map to ADAINF_ERR_CUDA with text in adainf_last_error() (thread-local).  No C++
- *     exception crosses the ABI.  A capacity overflow on the device (more routed crops than
- *     max_routed_per_dst) clamps deterministically in index order, reports the required count in
- *     n_routed, and is reported as ADAINF_ERR_CAPACITY by the next call on the app handle.
+ *     exception crosses the ABI.  NCCL errors map to ADAINF_ERR_NCCL.  A capacity overflow on the device
+ *     (more routed crops than max_routed_per_dst) clamps deterministically in index order and reports the
+ *     required count in n_routed (device: n_routed[e] > max_routed_per_dst is the overflow signal, valid
+ *     under CUDA-graph replay too); the library also raises a mapped host flag that makes the next
+ *     adainf_infer_dag or adainf_app_poll on the app return ADAINF_ERR_CAPACITY.  Graph replay does not run
+ *     the host-side check of adainf_infer_dag: callers that replay a captured step poll with adainf_app_poll.
  *   - Thread safety: one handle = one thread + one stream at a time; distinct handles are independent.
  *   - There is no CPU fallback: without an sm_100 device every compute call returns
  *     ADAINF_ERR_UNSUPPORTED.
@@ -137,6 +140,9 @@ typedef struct {
 
 adainf_status adainf_app_create(const adainf_app_spec* spec, adainf_app_t* out);
 adainf_status adainf_app_destroy(adainf_app_t app);
+/* Synchronizes `stream`, then returns ADAINF_ERR_CAPACITY (and clears the flag) if any infer_dag since the last
+ * check routed more crops than max_routed_per_dst; ADAINF_OK otherwise. */
+adainf_status adainf_app_poll(adainf_app_t app, adainf_stream_t stream);
 
 /* Per-model outputs of adainf_infer_dag (all DEVICE pointers, caller-allocated; any may be NULL).
  * Rows refer to the model's input rows in original order (root: the request batch; routed model:
@@ -204,14 +210,37 @@ adainf_status adainf_retrain_step(adainf_model_t m, const void* samples_bf16_nhw
                                   adainf_step_stats* stats_dev, adainf_stream_t stream);
 
 /* The retraining step on rows of a device-resident window pool (samples collected in the previous
- * period), without materialising the batch: sample r of the step is pool row row_idx[r] (device int32[n_local],
- * every entry a valid row, e.g. adainf_select_retrain's out_idx when out_count == k) and its label
- * pool_labels[row_idx[r]].  The rows are read once, straight into the model's packed input layout.
- * Same semantics, results and errors as adainf_retrain_step on the gathered batch; models whose input is used
- * unpacked (in_c a multiple of 8) return ADAINF_ERR_UNSUPPORTED. */
-adainf_status adainf_retrain_step_rows(adainf_model_t m, const void* pool_bf16_nhwc, const int32_t* pool_labels,
-                                       const int32_t* row_idx, int32_t n_local, int64_t n_global, float lr,
+ * period), without materialising the batch.  pool: device bf16 NHWC [pool_rows][in_h][in_w][in_c];
+ * pool_labels: device int32 [pool_rows]; row_idx: device int32 [n_local]; count: device int32 [1] or NULL.
+ * Sample r of the step is pool row row_idx[r] with label pool_labels[row_idx[r]] when r < *count (count == NULL:
+ * every r < n_local) and 0 <= row_idx[r] < pool_rows; any other row contributes nothing (zero input, no loss, no
+ * gradient), so adainf_select_retrain's (out_idx, out_count) can be passed as is even when fewer than k samples
+ * were eligible (exclusions accumulate) — the unwritten tail of out_idx is never read as a row.
+ * A label outside [0, num_classes) likewise contributes nothing (here and in adainf_retrain_step).
+ * The rows are read once, straight into the model's packed input layout.  Same semantics, results and errors
+ * as adainf_retrain_step on the gathered batch; models whose input is used unpacked (in_c a multiple of 8)
+ * return ADAINF_ERR_UNSUPPORTED; pool_rows <= 0 -> ADAINF_ERR_SHAPE. */
+adainf_status adainf_retrain_step_rows(adainf_model_t m, const void* pool_bf16_nhwc, int64_t pool_rows,
+                                       const int32_t* pool_labels, const int32_t* row_idx, const int32_t* count,
+                                       int32_t n_local, int64_t n_global, float lr,
                                        adainf_step_stats* stats_dev, adainf_stream_t stream);
+
+/* The two halves of a retraining step, for callers that reduce gradients themselves (SURVEY §8(c.1) step 13:
+ * each replica's gradient scaled by 1/n_global, summed over replicas):
+ *   adainf_retrain_grad[_rows]: forward + losses + backward only — the replica's gradient is left in the
+ *     model's gradient buffer (adainf_model_grad_ptr), no all-reduce, no update; stats_dev->loss written.
+ *   adainf_model_update: the update of adainf_retrain_step on whatever the gradient buffer holds (all-reduced
+ *     first over an attached communicator), stats_dev->grad_norm written.  ADAINF_ERR_INVALID if no gradient
+ *     was ever computed on the model.
+ * adainf_retrain_step == adainf_retrain_grad + adainf_model_update, bit for bit. */
+adainf_status adainf_retrain_grad(adainf_model_t m, const void* samples_bf16_nhwc, const int32_t* labels,
+                                  int32_t n_local, int64_t n_global, adainf_step_stats* stats_dev,
+                                  adainf_stream_t stream);
+adainf_status adainf_retrain_grad_rows(adainf_model_t m, const void* pool_bf16_nhwc, int64_t pool_rows,
+                                       const int32_t* pool_labels, const int32_t* row_idx, const int32_t* count,
+                                       int32_t n_local, int64_t n_global, adainf_step_stats* stats_dev,
+                                       adainf_stream_t stream);
+adainf_status adainf_model_update(adainf_model_t m, float lr, adainf_step_stats* stats_dev, adainf_stream_t stream);
 
 /* Assemble the retraining batch from the device-resident window pool (samples collected in the
  * previous period): dst[r] = src[idx[r]] for r < min(*count, n) (count device int or NULL -> n);

@@ -55,6 +55,11 @@ adainf_status adainf_dbg_stem_fwd(const void* x, int32_t n, int32_t H, int32_t W
 adainf_status adainf_dbg_stem_wgrad(const void* x, const void* dz, int32_t n, int32_t H, int32_t W, int32_t cin,
                                     float* dw, float* db, adainf_stream_t stream);
 
+/* Device pointer of the routed-crop batch of DET_CROP edge `edge` of `app` (library-owned, valid until the app
+ * is destroyed): [max_routed_per_dst][crop_h][crop_w][dst in_c] bf16, rows in route order, written by the last
+ * adainf_infer_dag (rows past n_routed are stale).  For the stage-isolated crop parity test (reading Q20). */
+adainf_status adainf_dbg_app_crops(adainf_app_t app, int32_t edge, const void** crops);
+
 /* Launch accounting and per-kernel-class timing (CUDA events on the launching stream).
  * adainf_launch_count: total kernels launched by the library since load (host-side counter).
  * adainf_prof_enable(1): bracket every launch class with events; adainf_prof_query (synchronizing)

@@ -47,7 +47,8 @@ adainf_status adainf_retrain_setting(double alloc_ms, const adainf_retrain_profi
 /* Version averaging: dst's fp32 parameters become the unweighted mean of the versions' parameters
  * (reading Q23: summed in the given order in fp32, then divided by n), its momentum is reset to 0 and its bf16
  * GEMM shadows are refreshed.  versions[n] (n >= 1) may include dst; all models must share dst's architecture
- * (same parameter count) and device.  Stream-ordered. */
+ * (same parameter count) and device.  Stream-ordered; with n <= 16 it neither copies from the host nor
+ * synchronizes (CUDA-graph capturable), with n > 16 it synchronizes the stream. */
 adainf_status adainf_model_average(adainf_model_t dst, const adainf_model_t* versions, int32_t n,
                                    adainf_stream_t stream);
 

@@ -98,7 +98,12 @@ def lib():
             "adainf_infer_dag": [vp, vp, i32, C.POINTER(C.c_float), i32, C.POINTER(ModelOut), vp],
             "adainf_select_retrain": [C.POINTER(SelectIn), i32, vp, vp, vp, vp, vp],
             "adainf_retrain_step": [vp, vp, vp, i32, i64, C.c_float, vp, vp],
-            "adainf_retrain_step_rows": [vp, vp, vp, vp, i32, i64, C.c_float, vp, vp],
+            "adainf_retrain_step_rows": [vp, vp, i64, vp, vp, vp, i32, i64, C.c_float, vp, vp],
+            "adainf_retrain_grad": [vp, vp, vp, i32, i64, vp, vp],
+            "adainf_retrain_grad_rows": [vp, vp, i64, vp, vp, vp, i32, i64, vp, vp],
+            "adainf_model_update": [vp, C.c_float, vp, vp],
+            "adainf_app_poll": [vp, vp],
+            "adainf_dbg_app_crops": [vp, i32, C.POINTER(vp)],
             "adainf_dp_attach": [vp, vp, i32, i32],
             "adainf_nccl_unique_id": [vp],
             "adainf_gather_rows": [vp, vp, vp, i32, i64, vp, vp],
@@ -177,6 +182,20 @@ def _exit0_channels(spec):
     return 0
 
 
+class _CudaArray:
+    """__cuda_array_interface__ over a library-owned device buffer (zero-copy torch view)."""
+
+    def __init__(self, p, shape, typestr):
+        self.__cuda_array_interface__ = {"shape": tuple(shape), "typestr": typestr, "data": (int(p), False),
+                                         "version": 2}
+
+
+def _device_view(p, n, dtype, device, shape=None):
+    import torch
+    ts = {torch.float32: "<f4", torch.int16: "<i2", torch.int32: "<i4"}[dtype]
+    return torch.as_tensor(_CudaArray(p, shape or (n,), ts), device=f"cuda:{device}")
+
+
 class Model:
     """Owns an adainf_model_t."""
 
@@ -199,6 +218,7 @@ class Model:
         self.num_exits = e.value
         self.ncls = next((o["num_classes"] for o in spec["ops"] if o["kind"] == "exit"), 0)
         self.max_batch = max_batch
+        self.device = device
         self.exit0_channels = _exit0_channels(spec)
 
     def get_params(self):
@@ -220,11 +240,35 @@ class Model:
                                         int(n_global or samples.shape[0]), float(lr), ptr(stats),
                                         stream_ptr(stream)))
 
-    def retrain_step_rows(self, pool, pool_labels, row_idx, n_global=None, lr=0.01, stats=None, stream=None):
-        """Retraining step on pool rows row_idx (device int32[n]) with labels pool_labels[row_idx]."""
+    def retrain_step_rows(self, pool, pool_labels, row_idx, n_global=None, lr=0.01, stats=None, stream=None,
+                          count=None):
+        """Retraining step on pool rows row_idx (device int32[n]) with labels pool_labels[row_idx]; rows past the
+        device count (int32[1], optional) or outside the pool contribute nothing."""
         n = int(row_idx.shape[0])
-        check(lib().adainf_retrain_step_rows(self.h, ptr(pool), ptr(pool_labels), ptr(row_idx), n,
-                                             int(n_global or n), float(lr), ptr(stats), stream_ptr(stream)))
+        check(lib().adainf_retrain_step_rows(self.h, ptr(pool), int(pool.shape[0]), ptr(pool_labels), ptr(row_idx),
+                                             ptr(count), n, int(n_global or n), float(lr), ptr(stats),
+                                             stream_ptr(stream)))
+
+    def retrain_grad(self, samples, labels, n_global=None, stats=None, stream=None):
+        """Forward + backward only: this replica's 1/n_global-scaled gradient left in the gradient buffer."""
+        check(lib().adainf_retrain_grad(self.h, ptr(samples), ptr(labels), int(samples.shape[0]),
+                                        int(n_global or samples.shape[0]), ptr(stats), stream_ptr(stream)))
+
+    def retrain_grad_rows(self, pool, pool_labels, row_idx, n_global=None, stats=None, stream=None, count=None):
+        n = int(row_idx.shape[0])
+        check(lib().adainf_retrain_grad_rows(self.h, ptr(pool), int(pool.shape[0]), ptr(pool_labels), ptr(row_idx),
+                                             ptr(count), n, int(n_global or n), ptr(stats), stream_ptr(stream)))
+
+    def update(self, lr=0.01, stats=None, stream=None):
+        """SGD / momentum update on the current gradient buffer (all-reduced first over an attached communicator)."""
+        check(lib().adainf_model_update(self.h, float(lr), ptr(stats), stream_ptr(stream)))
+
+    def grad_tensor(self):
+        """The device gradient buffer as a torch float32 tensor view (num_params), for callers reducing it."""
+        import torch
+        p = C.c_void_p()
+        check(lib().adainf_model_grad_ptr(self.h, C.byref(p)))
+        return _device_view(p.value, self.num_params, torch.float32, self.device)
 
     def dp_attach(self, uid: bytes, rank: int, world: int):
         buf = C.create_string_buffer(uid, 128)
@@ -302,6 +346,20 @@ class App:
             mo[i].max_det = int(o["det_table"].shape[0]) if o.get("det_table") is not None else 0
         check(lib().adainf_infer_dag(self.h, ptr(batch), int(batch.shape[0]),
                                      t.ctypes.data_as(C.POINTER(C.c_float)), int(t.size), mo, stream_ptr(stream)))
+
+    def poll(self, stream=None):
+        """Synchronize the stream; raise AdaInfError(ERR_CAPACITY) if a routing overflow happened since the last check."""
+        check(lib().adainf_app_poll(self.h, stream_ptr(stream)))
+
+    def crops(self, edge, rows):
+        """Routed-crop batch of DET_CROP edge `edge` (debug view, bf16 bits as int16 [rows, H, W, C])."""
+        import torch
+        e = self.edges[edge]
+        dst = self.models[e[1]].spec
+        p = C.c_void_p()
+        check(lib().adainf_dbg_app_crops(self.h, edge, C.byref(p)))
+        return _device_view(p.value, 0, torch.int16, self.models[e[1]].device,
+                            shape=(rows, dst["in_h"], dst["in_w"], dst["in_c"]))
 
     def close(self):
         if getattr(self, "h", None):

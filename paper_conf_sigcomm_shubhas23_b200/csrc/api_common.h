@@ -43,6 +43,9 @@ adainf_status guard(F&& f) {
   } catch (const CudaError& e) {
     set_last_error(e.what());
     return ADAINF_ERR_CUDA;
+  } catch (const NcclError& e) {
+    set_last_error(e.what());
+    return ADAINF_ERR_NCCL;
   } catch (const std::bad_alloc& e) {
     set_last_error("out of host memory");
     return ADAINF_ERR_OOM;

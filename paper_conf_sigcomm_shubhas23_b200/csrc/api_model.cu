@@ -334,14 +334,71 @@ extern "C" adainf_status adainf_retrain_step(adainf_model_t m, const void* sampl
   });
 }
 
-extern "C" adainf_status adainf_retrain_step_rows(adainf_model_t m, const void* pool, const int32_t* pool_labels,
-                                                  const int32_t* row_idx, int32_t n_local, int64_t n_global, float lr,
+extern "C" adainf_status adainf_retrain_step_rows(adainf_model_t m, const void* pool, int64_t pool_rows,
+                                                  const int32_t* pool_labels, const int32_t* row_idx,
+                                                  const int32_t* count, int32_t n_local, int64_t n_global, float lr,
                                                   adainf_step_stats* stats, adainf_stream_t stream) {
   return guard([&] {
     if (!m || !pool || !pool_labels || !row_idx) throw InvalidError("retrain_step_rows: null argument");
     if (!(lr == lr)) throw InvalidError("retrain: NaN lr");
     require_device();
-    m->m.train_step_rows((const bf16*)pool, pool_labels, row_idx, n_local, n_global, lr, stats, (cudaStream_t)stream);
+    m->m.train_step_rows((const bf16*)pool, pool_rows, pool_labels, row_idx, count, n_local, n_global, lr, stats,
+                         (cudaStream_t)stream);
+  });
+}
+
+extern "C" adainf_status adainf_retrain_grad(adainf_model_t m, const void* samples, const int32_t* labels,
+                                             int32_t n_local, int64_t n_global, adainf_step_stats* stats,
+                                             adainf_stream_t stream) {
+  return guard([&] {
+    if (!m || !samples || !labels) throw InvalidError("retrain_grad: null argument");
+    require_device();
+    m->m.train_step((const bf16*)samples, labels, n_local, n_global, 0.f, stats, (cudaStream_t)stream, false);
+  });
+}
+
+extern "C" adainf_status adainf_retrain_grad_rows(adainf_model_t m, const void* pool, int64_t pool_rows,
+                                                  const int32_t* pool_labels, const int32_t* row_idx,
+                                                  const int32_t* count, int32_t n_local, int64_t n_global,
+                                                  adainf_step_stats* stats, adainf_stream_t stream) {
+  return guard([&] {
+    if (!m || !pool || !pool_labels || !row_idx) throw InvalidError("retrain_grad_rows: null argument");
+    require_device();
+    m->m.train_step_rows((const bf16*)pool, pool_rows, pool_labels, row_idx, count, n_local, n_global, 0.f, stats,
+                         (cudaStream_t)stream, false);
+  });
+}
+
+extern "C" adainf_status adainf_model_update(adainf_model_t m, float lr, adainf_step_stats* stats,
+                                             adainf_stream_t stream) {
+  return guard([&] {
+    if (!m) throw InvalidError("update: null model");
+    if (!(lr == lr)) throw InvalidError("update: NaN lr");
+    require_device();
+    m->m.update_impl(lr, stats, (cudaStream_t)stream);
+  });
+}
+
+extern "C" adainf_status adainf_app_poll(adainf_app_t app, adainf_stream_t stream) {
+  return guard([&] {
+    if (!app) throw InvalidError("app_poll: null app");
+    require_device();
+    CK(cudaStreamSynchronize((cudaStream_t)stream));
+    AppHolder* H = (AppHolder*)app;
+    if (*H->impl.cap_flag_host) {
+      *H->impl.cap_flag_host = 0;
+      throw CapacityError("infer_dag routed more crops than max_routed_per_dst (clamped in index order)");
+    }
+  });
+}
+
+extern "C" adainf_status adainf_dbg_app_crops(adainf_app_t app, int32_t edge, const void** crops) {
+  return guard([&] {
+    if (!app || !crops) throw InvalidError("dbg_app_crops: null argument");
+    AppHolder* H = (AppHolder*)app;
+    if (edge < 0 || edge >= (int)H->a.edges.size() || H->a.edges[edge].kind != ADAINF_ROUTE_DET_CROP)
+      throw InvalidError("dbg_app_crops: not a DET_CROP edge");
+    *crops = H->impl.routed_in[edge].p;
   });
 }
 
@@ -359,7 +416,7 @@ extern "C" adainf_status adainf_nccl_unique_id(void* out128) {
     if (!out128) throw InvalidError("null argument");
 #ifdef ADAINF_WITH_NCCL
     ncclUniqueId id;
-    if (ncclGetUniqueId(&id) != ncclSuccess) throw std::runtime_error("ncclGetUniqueId failed");
+    if (ncclGetUniqueId(&id) != ncclSuccess) throw NcclError("ncclGetUniqueId failed");
     static_assert(sizeof(id) == 128, "ncclUniqueId is 128 bytes");
     memcpy(out128, &id, 128);
 #else
@@ -385,11 +442,10 @@ extern "C" adainf_status adainf_dp_attach(adainf_model_t m, const void* uid, int
     memcpy(&id, uid, 128);
     CK(cudaSetDevice(m->m.device));
     ncclResult_t r = ncclCommInitRank(&m->m.comm, world, id, rank);
-    if (r != ncclSuccess) throw std::runtime_error(std::string("ncclCommInitRank: ") + ncclGetErrorString(r));
+    if (r != ncclSuccess) throw NcclError(std::string("ncclCommInitRank: ") + ncclGetErrorString(r));
 #else
     if (world > 1) throw UnsupportedError("built without NCCL");
 #endif
   });
-  if (s == ADAINF_ERR_INVALID && std::string(adainf_last_error()).rfind("nccl", 0) == 0) return ADAINF_ERR_NCCL;
   return s;
 }

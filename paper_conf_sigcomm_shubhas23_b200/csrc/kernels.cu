@@ -18,8 +18,13 @@ __global__ void pack_input_kernel(const bf16* __restrict__ x, const int* __restr
   const long long total = (long long)n_rows * HW;
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
     const long long n = i / HW, pix = i - n * HW;
-    const long long src = (map ? map[n] : n) * (long long)HW + pix;
+    const long long row = map ? map[n] : n;
+    const long long src = row * (long long)HW + pix;
     bf16* o = y + i * Cpad;
+    if (row < 0) {  // sanitised row (retrain_step_rows): zero input
+      for (int c = 0; c < Cpad; ++c) o[c] = __float2bfloat16_rn(0.f);
+      continue;
+    }
     if (Cpad == 4) {
       __align__(8) bf16 v[4];
 #pragma unroll
@@ -463,6 +468,11 @@ __global__ void exit_loss_kernel(const float* __restrict__ logits, const int32_t
   float s = 0.f;
   for (int k = 0; k < ncls; ++k) s += expf(l[k] - m);
   const int y = labels[i];
+  if (y < 0 || y >= ncls) {  // ignored row (label outside [0, ncls), e.g. a sanitised pool row): no loss, no gradient
+    for (int k = 0; k < ncls; ++k) dl[(long long)i * ncls + k] = 0.f;
+    if (!accumulate) loss_rows[i] = 0.f;
+    return;
+  }
   for (int k = 0; k < ncls; ++k) {
     const float p = expf(l[k] - m) / s;
     dl[(long long)i * ncls + k] = w * (p - (k == y ? 1.f : 0.f)) * inv_n;
@@ -470,6 +480,26 @@ __global__ void exit_loss_kernel(const float* __restrict__ logits, const int32_t
   const float ce = (logf(s) - (l[y] - m)) * w * inv_n;
   loss_rows[i] = accumulate ? loss_rows[i] + ce : ce;
 }
+// retrain_step_rows: row r reads pool row idx[r] with label pool_labels[idx[r]] when r < *count (count nullable)
+// and 0 <= idx[r] < pool_rows; otherwise map -1 (zero input) and label -1 (ignored by the loss)
+__global__ void sanitize_rows_kernel(const int32_t* __restrict__ pool_labels, const int32_t* __restrict__ idx,
+                                     const int32_t* __restrict__ count, int n, long long pool_rows,
+                                     int32_t* __restrict__ map, int32_t* __restrict__ labels) {
+  const int r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= n) return;
+  const int lim = count ? min(*count, n) : n;
+  const int q = idx[r];
+  const bool ok = r < lim && q >= 0 && (long long)q < pool_rows;
+  map[r] = ok ? q : -1;
+  labels[r] = ok ? pool_labels[q] : -1;
+}
+void launch_sanitize_rows(const int32_t* pool_labels, const int32_t* idx, const int32_t* count, int n,
+                          long long pool_rows, int32_t* map, int32_t* labels, cudaStream_t st) {
+  ProfScope ps(PC_GATHER, st);
+  sanitize_rows_kernel<<<(n + 255) / 256, 256, 0, st>>>(pool_labels, idx, count, n, pool_rows, map, labels);
+  CK(cudaGetLastError());
+}
+
 void launch_exit_loss(const float* logits, const int32_t* labels, int n, int ncls, float w, float inv_n, float* dl,
                       float* loss_rows, int accumulate, cudaStream_t st) {
   ProfScope ps(PC_EXIT_LOSS, st);

@@ -58,6 +58,8 @@ void launch_compact(const uint8_t* alive, const int* count, int n_static, const 
 
 // ---- retraining (K8, K9, K10) ----
 // per exit: dl = w (softmax - onehot) / n_global ; loss_rows[n] += w CE
+void launch_sanitize_rows(const int32_t* pool_labels, const int32_t* idx, const int32_t* count, int n,
+                          long long pool_rows, int32_t* map, int32_t* labels, cudaStream_t st);
 void launch_exit_loss(const float* logits, const int32_t* labels, int n, int ncls, float w, float inv_n, float* dl,
                       float* loss_rows, int accumulate, cudaStream_t st);
 // head grads: dW[c][j] = sum_n pooled[n][c] dl[n][j]; db[j] = sum_n dl[n][j]; bcast[n][c] = (sum_j dl W[c][j]) / HW

@@ -520,22 +520,30 @@ void Model::infer(const bf16* x, const int* in_map, const int* in_count, int n_s
 }
 
 // ------------------------------------------------------------------------------------------------
-void Model::train_step_rows(const bf16* pool, const int32_t* pool_labels, const int32_t* idx, int n,
-                            long long n_global, float lr, adainf_step_stats* stats, cudaStream_t st) {
+void Model::train_step_rows(const bf16* pool, long long pool_rows, const int32_t* pool_labels, const int32_t* idx,
+                            const int32_t* count, int n, long long n_global, float lr, adainf_step_stats* stats,
+                            cudaStream_t st, bool update) {
   if (!pack) throw UnsupportedError("retrain_step_rows: the model reads its input unpacked (in_c % 8 == 0)");
   if (n <= 0 || n > max_batch) throw ShapeError("retrain: n_local must be in 1..max_batch");
-  if (!row_labels.p) row_labels.alloc((size_t)max_batch * 4);
-  launch_gather_rows(pool_labels, idx, nullptr, n, 4, row_labels.p, st);
-  train_step_impl(pool, idx, row_labels.as<int32_t>(), n, n_global, lr, stats, st);
+  if (pool_rows <= 0) throw ShapeError("retrain_step_rows: pool_rows must be positive");
+  if (!row_labels.p) {
+    row_labels.alloc((size_t)max_batch * 4);
+    row_map.alloc((size_t)max_batch * 4);
+  }
+  // rows past the device count / out-of-range indices -> map -1 (zero input) and label -1 (no loss, no gradient)
+  launch_sanitize_rows(pool_labels, idx, count, n, pool_rows, row_map.as<int32_t>(), row_labels.as<int32_t>(), st);
+  train_grad_impl(pool, row_map.as<int32_t>(), row_labels.as<int32_t>(), n, n_global, stats, st);
+  if (update) update_impl(lr, stats, st);
 }
 
 void Model::train_step(const bf16* x, const int32_t* labels, int n, long long n_global, float lr,
-                       adainf_step_stats* stats, cudaStream_t st) {
-  train_step_impl(x, nullptr, labels, n, n_global, lr, stats, st);
+                       adainf_step_stats* stats, cudaStream_t st, bool update) {
+  train_grad_impl(x, nullptr, labels, n, n_global, stats, st);
+  if (update) update_impl(lr, stats, st);
 }
 
-void Model::train_step_impl(const bf16* x, const int32_t* row_map, const int32_t* labels, int n, long long n_global,
-                            float lr, adainf_step_stats* stats, cudaStream_t st) {
+void Model::train_grad_impl(const bf16* x, const int32_t* row_map, const int32_t* labels, int n, long long n_global,
+                            adainf_step_stats* stats, cudaStream_t st) {
   if (n <= 0 || n > max_batch) throw ShapeError("retrain: n_local must be in 1..max_batch");
   if (n_global < n) throw ShapeError("retrain: n_global < n_local");
   ensure_training();
@@ -642,20 +650,23 @@ void Model::train_step_impl(const bf16* x, const int32_t* row_map, const int32_t
       conv_backward(nd, dz);
     }
   }
+  if (stats) launch_sum(loss_rows.as<float>(), n, &stats->loss, 0.f, st);
+}
+
+void Model::update_impl(float lr, adainf_step_stats* stats, cudaStream_t st) {
+  if (!train_ready) throw InvalidError("update: no gradient has been computed on this model");
+  float* G = grads.as<float>();
 #ifdef ADAINF_WITH_NCCL
   if (comm && dp_world > 1) {
     ncclResult_t r = ncclAllReduce(G, G, (size_t)nparams, ncclFloat, ncclSum, comm, st);
-    if (r != ncclSuccess) throw std::runtime_error(std::string("NCCL: ") + ncclGetErrorString(r));
+    if (r != ncclSuccess) throw NcclError(std::string("NCCL all-reduce: ") + ncclGetErrorString(r));
   }
 #endif
   // fused SGD + momentum + shadow refresh (K10)
   launch_sgd(params.as<float>(), mom.as<float>(), G, nparams, lr, momentum, weight_decay, sgd_segs.as<SgdSeg>(),
              sgd_nseg, sgd_block_seg.as<int>(), sgd_block_start.as<long long>(), sgd_nblocks, sq_partial.as<float>(),
              st);
-  if (stats) {
-    launch_sum(loss_rows.as<float>(), n, &stats->loss, 0.f, st);
-    launch_sum(sq_partial.as<float>(), sgd_nblocks, &stats->grad_norm, -1.f, st);
-  }
+  if (stats) launch_sum(sq_partial.as<float>(), sgd_nblocks, &stats->grad_norm, -1.f, st);
 }
 
 }  // namespace adainf

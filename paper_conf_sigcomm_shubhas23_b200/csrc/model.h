@@ -128,13 +128,18 @@ struct Model {
   void infer(const bf16* x, const int* in_map, const int* in_count, int n_static, const float* taus,
              const adainf_model_out& out, cudaStream_t st, bool x_padded = false);
   void train_step(const bf16* x, const int32_t* labels, int n, long long n_global, float lr,
-                  adainf_step_stats* stats, cudaStream_t st);
-  // the same step on pool rows idx[0..n) (packed straight from the pool; labels gathered from pool_labels)
-  void train_step_rows(const bf16* pool, const int32_t* pool_labels, const int32_t* idx, int n, long long n_global,
-                       float lr, adainf_step_stats* stats, cudaStream_t st);
-  DevBuf row_labels;  // labels of the rows of train_step_rows
-  void train_step_impl(const bf16* x, const int32_t* row_map, const int32_t* labels, int n, long long n_global,
-                       float lr, adainf_step_stats* stats, cudaStream_t st);
+                  adainf_step_stats* stats, cudaStream_t st, bool update = true);
+  // the same step on pool rows idx[0..n) (packed straight from the pool; labels gathered from pool_labels);
+  // rows r >= *count (count device, nullable) and indices outside [0, pool_rows) contribute nothing
+  void train_step_rows(const bf16* pool, long long pool_rows, const int32_t* pool_labels, const int32_t* idx,
+                       const int32_t* count, int n, long long n_global, float lr, adainf_step_stats* stats,
+                       cudaStream_t st, bool update = true);
+  DevBuf row_labels, row_map;  // sanitised labels / pool rows of train_step_rows
+  // forward + losses + backward: the gradient of this replica's samples (scaled by 1/n_global) in `grads`
+  void train_grad_impl(const bf16* x, const int32_t* row_map, const int32_t* labels, int n, long long n_global,
+                       adainf_step_stats* stats, cudaStream_t st);
+  // (data-parallel: gradient all-reduce over the attached communicator) + fused SGD / momentum / shadow refresh
+  void update_impl(float lr, adainf_step_stats* stats, cudaStream_t st);
 
  private:
   void forward_nodes(const bf16* x0, const int* map0, const int* count0, int n_static, bool train, const float* taus,

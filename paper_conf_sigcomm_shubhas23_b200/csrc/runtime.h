@@ -16,6 +16,9 @@ struct CudaError : std::runtime_error {
 struct ShapeError : std::runtime_error {
   using std::runtime_error::runtime_error;
 };
+struct NcclError : std::runtime_error {  // -> ADAINF_ERR_NCCL
+  using std::runtime_error::runtime_error;
+};
 
 #define CK(expr)                                                                                         \
   do {                                                                                                   \

@@ -15,8 +15,16 @@ namespace {
 
 bool finite_nonneg(double v) { return std::isfinite(v) && v >= 0.0; }
 
+// up to 16 versions: the pointer table travels as a kernel parameter (no host->device copy, no synchronization:
+// the call can be captured in a CUDA graph)
+struct SrcTable {
+  const float* p[16];
+  __device__ const float* operator[](int v) const { return p[v]; }
+};
+
 // dst = (sum_v src_v in order) / n, fp32; one thread per 4 parameters
-__global__ void average_kernel(float* __restrict__ dst, const float* const* __restrict__ srcs, int n, long long count) {
+template <class Tab>
+__global__ void average_kernel(float* __restrict__ dst, Tab srcs, int n, long long count) {
   const long long i = (blockIdx.x * (long long)blockDim.x + threadIdx.x) * 4;
   if (i >= count) return;
   if (i + 4 <= count) {
@@ -139,20 +147,29 @@ extern "C" adainf_status adainf_model_average(adainf_model_t dst, const adainf_m
     }
     cudaStream_t st = (cudaStream_t)stream;
     CK(cudaSetDevice(d.device));
-    const float** dsrc = nullptr;
-    CK(cudaMallocAsync((void**)&dsrc, sizeof(float*) * n, st));
-    CK(cudaMemcpyAsync(dsrc, srcs.data(), sizeof(float*) * n, cudaMemcpyHostToDevice, st));
     const long long cnt = d.nparams;
     const long long threads = (cnt + 3) / 4;
-    {
+    const unsigned blocks = (unsigned)((threads + 255) / 256);
+    if (n <= 16) {
+      SrcTable t{};
+      for (int v = 0; v < n; ++v) t.p[v] = srcs[v];
       ProfScope ps(PC_SGD, st);
-      average_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(d.params.as<float>(), dsrc, n, cnt);
+      average_kernel<<<blocks, 256, 0, st>>>(d.params.as<float>(), t, n, cnt);
       CK(cudaGetLastError());
+    } else {
+      const float** dsrc = nullptr;
+      CK(cudaMallocAsync((void**)&dsrc, sizeof(float*) * n, st));
+      CK(cudaMemcpyAsync(dsrc, srcs.data(), sizeof(float*) * n, cudaMemcpyHostToDevice, st));
+      {
+        ProfScope ps(PC_SGD, st);
+        average_kernel<<<blocks, 256, 0, st>>>(d.params.as<float>(), (const float* const*)dsrc, n, cnt);
+        CK(cudaGetLastError());
+      }
+      CK(cudaFreeAsync(dsrc, st));
+      CK(cudaStreamSynchronize(st));  // the host pointer table must outlive the copy
     }
-    CK(cudaFreeAsync(dsrc, st));
     CK(cudaMemsetAsync(d.mom.p, 0, d.mom.bytes, st));  // reading Q23: momentum restarts from the averaged version
     d.refresh_shadows(st);
-    CK(cudaStreamSynchronize(st));  // the host pointer table must outlive the copy
   });
 }
 

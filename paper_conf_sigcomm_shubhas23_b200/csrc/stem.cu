@@ -28,6 +28,12 @@ __global__ void pack_s2d_kernel(const bf16* __restrict__ x, const int* __restric
     const int rem = (int)(i - n * Hs * Ws);
     const int si = rem / Ws, sj = rem - si * Ws;
     const long long src = map ? map[n] : n;
+    if (src < 0) {  // sanitised row (retrain_step_rows: past the device count / out of range): zero input
+      uint4* o = (uint4*)(s + i * 16);
+      o[0] = make_uint4(0, 0, 0, 0);
+      o[1] = make_uint4(0, 0, 0, 0);
+      continue;
+    }
     if (cin == 3) {
       // the two pixels of one input row are 12 contiguous, 4-byte aligned bytes (W even): three 32-bit loads
       // per row; channel 3 of each pixel is the zero pad

@@ -76,7 +76,10 @@ def test_video_dag_detector_routing_crops():
     gk = [k for k, r in zip(key(gdet), gdet) if not band[cand_id(r)]]
     ok = [k for k, r in zip(key(odet), odet) if not band[cand_id(r)]]
     assert gk == ok
-    assert n_det == on or band.any()
+    # every candidate detected by one side only is inside the band
+    gset, oset = {cand_id(r) for r in gdet}, {cand_id(r) for r in odet}
+    assert all(band[c] for c in gset ^ oset)
+    assert n_det - on == len(gset - oset) - len(oset - gset)
     # boxes and scores (matched by candidate id)
     omap = {cand_id(r): r for r in odet}
     for r in gdet:
@@ -99,6 +102,9 @@ def test_video_dag_detector_routing_crops():
         if nr == 0:
             continue
         crops = np.stack([O.crop(xf[int(gdet[d][0])], gdet[d][5:9], crop, crop) for d in ridx[e][:nr]])
+        # Q20: crops from the GPU's boxes are bit-exact (the routed batch read back through adainf_dbg_app_crops)
+        gcrops = synth.bf16_bits_to_f32(app.crops(e, nr).cpu().numpy().view(np.uint16))
+        assert np.array_equal(gcrops, crops), np.abs(gcrops - crops).max()
         orc = O.Model(model_spec).forward(params, crops)
         eid, _, _ = O.exit_assign(orc["conf"], taus_cls)
         g_eid = outs[mi]["exit_id"].cpu().numpy()[:nr]
@@ -150,3 +156,70 @@ def test_audio_dag_class_routing():
         lg = outs[mi]["logits"].cpu().numpy()[:len(want)]
         for r in np.nonzero(~b2)[0]:
             assert rel(lg[r], o2["logits"][r, e2[r]]) <= 2e-2
+
+
+def test_video_dag_c3_geometry():
+    """BASELINE config 3 geometry on a few frames: 416x416 frames, TinyYOLOv3-like detector at G = 13 (stride 32),
+    crops resized to 224x224 into two ResNet-18-EE destinations (vehicle 10 classes, person 8 classes), all on
+    the device; detections / routing bit-exact outside the tau_det band, crops bit-exact from the GPU's boxes,
+    downstream exits and logits against the oracle on those crops."""
+    Bn, hw, crop = 3, 416, 224
+    det_spec = S.tiny_yolo_det(in_hw=hw)
+    A, NC = 3, 2
+    p_det = synth.det_head_params(det_spec, synth.init_params(det_spec, seed=51), obj_bias=-1.0)
+    veh, per = S.resnet18_ee(10), S.resnet18_ee(8)
+    p_veh, p_per = synth.init_params(veh, seed=52), synth.init_params(per, seed=53)
+    xb, _ = synth.drifted_images(Bn, hw, hw, 3, seed=51)
+    xf = synth.bf16_bits_to_f32(xb)
+    raw = O.Model(det_spec).forward(p_det, xf, want_det=True)["det"]
+    G = raw.shape[1]
+    assert G == 13
+    sig = lambda v: 1 / (1 + np.exp(-v.astype(np.float64)))
+    r5 = raw.reshape(Bn, G, G, A, 5 + NC)
+    scores = (sig(r5[..., 4]) * sig(r5[..., 5:].max(-1))).reshape(-1)
+    # ~4 detections per frame (SURVEY §8(d) C3), threshold in the widest nearby gap
+    tau_det = _calib_tau(scores, 4.0 * Bn / scores.size)
+    odet, on = O.detect(raw, A, NC, S.YOLO_ANCHORS, 32, hw, hw, tau_det)
+    cap = 48
+    m_det = B.Model(det_spec, Bn, params=p_det)
+    m_veh, m_per = B.Model(veh, cap, params=p_veh), B.Model(per, cap, params=p_per)
+    app = B.App([m_det, m_veh, m_per], edges=[(0, 1, B.ROUTE_DET_CROP, 0, crop, crop),
+                                               (0, 2, B.ROUTE_DET_CROP, 1, crop, crop)], max_routed_per_dst=cap)
+    max_det = Bn * G * G * A
+    outs = [B.alloc_outs(m_det, Bn, max_det=max_det, n_out_edges=2, max_routed=cap), B.alloc_outs(m_veh, cap),
+            B.alloc_outs(m_per, cap)]
+    taus_cls = [0.4, 0.4, 0.4]
+    app.infer(to_cuda_bf16(xb), [tau_det] + taus_cls + taus_cls, outs)
+    app.poll()
+    n_det = int(outs[0]["n_det"].item())
+    gdet = outs[0]["det_table"].cpu().numpy()[:n_det]
+    band = np.abs(scores - tau_det) < BAND
+    cid = lambda r: (int(r[0]) * G * G + int(r[1])) * A + int(r[2])
+    assert [tuple(int(v) for v in r[:4]) for r in gdet if not band[cid(r)]] == \
+        [tuple(int(v) for v in r[:4]) for r in odet if not band[cid(r)]]
+    assert 1 <= n_det <= cap
+    n_routed = outs[0]["n_routed"].cpu().numpy()
+    ridx = outs[0]["route_idx"].cpu().numpy()
+    assert int(n_routed.sum()) == n_det
+    for e, (model_spec, params, mi, taus) in enumerate(((veh, p_veh, 1, taus_cls), (per, p_per, 2, taus_cls))):
+        want = [i for i in range(n_det) if int(gdet[i][3]) == e]
+        assert n_routed[e] == len(want) and ridx[e][:len(want)].tolist() == want
+        nr = len(want)
+        if nr == 0:
+            continue
+        crops = np.stack([O.crop(xf[int(gdet[d][0])], gdet[d][5:9], crop, crop) for d in want])
+        gcrops = synth.bf16_bits_to_f32(app.crops(e, nr).cpu().numpy().view(np.uint16))
+        assert np.array_equal(gcrops, crops)
+        orc = O.Model(model_spec).forward(params, crops)
+        eid, _, counts = O.exit_assign(orc["conf"], taus)
+        from parity import banded_rows
+        cb = banded_rows(orc["conf"], taus, eid)
+        g_eid = outs[mi]["exit_id"].cpu().numpy()[:nr]
+        assert (g_eid[~cb] == eid[~cb]).all()
+        assert outs[mi]["exit_counts"].cpu().numpy().sum() == nr
+        lg = outs[mi]["logits"].cpu().numpy()[:nr]
+        for r in np.nonzero(~cb)[0]:
+            assert rel(lg[r], orc["logits"][r, eid[r]]) <= 2e-2
+    app.close()
+    for m in (m_det, m_veh, m_per):
+        m.close()

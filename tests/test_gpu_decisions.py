@@ -1,0 +1,198 @@
+"""Decision contract under stress (north_star: exit assignments, compaction order, routing and top-k
+indices bit-exact versus the oracle except for items within 1e-3 of a threshold).
+
+Thresholds never come from the batch under test: the base tau vector is calibrated on a SEPARATE batch
+(oracle confidences), and each tau_k is then swept over 20 uniform values in [0.1, 0.95] with the others
+held, so thresholds fall wherever the sweep puts them, not in confidence gaps.  Every GPU decision is
+compared with the oracle's for the same tau; items inside the 1e-3 band (oracle values) are set aside
+and counted.  The per-exit |conf_gpu - conf_oracle| distribution is recorded (gpurun_out/decisions.json
+when that directory exists) because it is what decides whether out-of-band mismatches can occur.
+
+Routing: tau_det swept over 20 values on the detector; top-k: k swept over 20 values on the config-2
+selection pool, band = |d_i - d_(k)| < 1e-3."""
+import json
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+from paper_conf_sigcomm_shubhas23_b200 import binding as B
+from paper_conf_sigcomm_shubhas23_b200 import specs as S
+from paper_conf_sigcomm_shubhas23_b200 import synth
+
+from parity import BAND, banded_rows, to_cuda_bf16
+
+pytestmark = pytest.mark.gpu
+
+SWEEP = np.linspace(0.1, 0.95, 20)
+_RECORD = {}
+
+
+def _record(key, val):
+    _RECORD[key] = val
+    d = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "gpurun_out")
+    if os.path.isdir(d):
+        with open(os.path.join(d, "decisions.json"), "w") as f:
+            json.dump(_RECORD, f, indent=1)
+    print(key, json.dumps(val))
+
+
+def _gpu_conf_all(app, outs, x, E):
+    """GPU confidence of every row at every exit: tau_k = 0 at exit k, later exits disabled."""
+    Bn = x.shape[0]
+    conf = np.zeros((Bn, E), np.float32)
+    for k in range(E):
+        t = [2.0] * (E - 1)
+        if k < E - 1:
+            t[k] = 0.0
+        app.infer(x, t, [outs])
+        torch.cuda.synchronize()
+        conf[:, k] = outs["conf"].cpu().numpy()[:Bn]
+    return conf
+
+
+def _compare(gpu, orc_conf, taus, Bn, E):
+    """(#out-of-band mismatches in exit ids, in survivor lists, in counts (when nothing is banded), #banded)"""
+    eid, surv, counts = O.exit_assign(orc_conf, taus)
+    band = banded_rows(orc_conf, taus, eid)
+    g_eid = gpu["exit_id"][:Bn]
+    mis_eid = int(((g_eid != eid) & ~band).sum())
+    bad = set(np.nonzero(band)[0].tolist())
+    mis_surv = 0
+    for k in range(E - 1):
+        n_alive = Bn - int(gpu["exit_counts"][:k + 1].sum())
+        g = gpu["surv_idx"][k][:n_alive]
+        assert np.all(np.diff(g) > 0), "survivor list not ascending"
+        o = surv[k][surv[k] >= 0]
+        mis_surv += int([i for i in g if i not in bad] != [i for i in o if i not in bad])
+    mis_cnt = int(not band.any() and not np.array_equal(gpu["exit_counts"], counts))
+    assert gpu["exit_counts"].sum() == Bn
+    return mis_eid, mis_surv, mis_cnt, int(band.sum())
+
+
+@pytest.mark.parametrize("hw,Bn", [(224, 128), (64, 512)])
+def test_exit_decisions_tau_sweep(hw, Bn):
+    spec = S.resnet18_ee(in_hw=hw)
+    E = 4
+    p = synth.init_params(spec, seed=1)
+    protos = synth.class_prototypes(10, hw, hw, 3, seed=1244)
+    xb, _ = synth.drifted_images(Bn, hw, hw, 3, seed=211, period=1, protos=protos)
+    cb, _ = synth.drifted_images(32, hw, hw, 3, seed=7, period=1, protos=protos)
+    om = O.Model(spec)
+    base = [float(t) for t in synth.calibrate_thresholds(om.forward(p, synth.bf16_bits_to_f32(cb))["conf"],
+                                                          [0.25, 0.25, 0.25])]
+    orc = om.forward(p, synth.bf16_bits_to_f32(xb))
+    m = B.Model(spec, Bn, params=p)
+    app = B.App([m])
+    outs = B.alloc_outs(m, Bn)
+    x = to_cuda_bf16(xb)
+    gconf = _gpu_conf_all(app, outs, x, E)
+    d = np.abs(gconf - orc["conf"])
+    stats = {"max_dconf_per_exit": d.max(0).tolist(), "p99_dconf_per_exit": np.quantile(d, 0.99, axis=0).tolist(),
+             "frac_dconf_gt_band_per_exit": (d > BAND).mean(0).tolist()}
+    tot = {"mis_exit_id": 0, "mis_surv_lists": 0, "mis_counts": 0, "banded_row_cases": 0, "cases": 0}
+    worst = []
+    for k in range(E - 1):
+        for t in SWEEP:
+            taus = list(base)
+            taus[k] = float(t)
+            app.infer(x, taus, [outs])
+            torch.cuda.synchronize()
+            g = {kk: v.cpu().numpy() for kk, v in outs.items()}
+            me, ms, mc, nb = _compare(g, orc["conf"], taus, Bn, E)
+            tot["mis_exit_id"] += me
+            tot["mis_surv_lists"] += ms
+            tot["mis_counts"] += mc
+            tot["banded_row_cases"] += nb
+            tot["cases"] += 1
+            if me:
+                eid = O.exit_assign(orc["conf"], taus)[0]
+                for r in np.nonzero(g["exit_id"][:Bn] != eid)[0]:
+                    worst.append({"row": int(r), "taus": taus, "gpu_exit": int(g["exit_id"][r]),
+                                  "oracle_exit": int(eid[r]), "oracle_conf": orc["conf"][r].tolist(),
+                                  "gpu_conf": gconf[r].tolist()})
+    _record(f"exit_sweep_{hw}x{Bn}", dict(stats, base_taus=base, **tot, mismatches=worst[:20]))
+    app.close()
+    m.close()
+    assert tot["mis_exit_id"] == 0 and tot["mis_surv_lists"] == 0 and tot["mis_counts"] == 0, tot
+
+
+def test_topk_decisions_k_sweep():
+    """Config-2 selection pool (16,384 x 64 -> P = 16, 10% excluded): the index set outside the
+    |d_i - d_(k)| < 1e-3 band is bit-exact for 20 values of k."""
+    N, D, P = 16384, 64, 16
+    Xb, Wb, ref = synth.embeddings(N, D, P, seed=9)
+    ex = (np.random.default_rng(9).random(N) < 0.1).astype(np.uint8)
+    X = torch.from_numpy(Xb.view(np.int16)).cuda().view(torch.bfloat16).reshape(N, D)
+    W = torch.from_numpy(Wb.view(np.int16)).cuda().view(torch.bfloat16).reshape(D, P)
+    R = torch.from_numpy(ref).cuda()
+    E_ = torch.from_numpy(ex).cuda()
+    Xf = synth.bf16_bits_to_f32(Xb).reshape(N, D)
+    Wf = synth.bf16_bits_to_f32(Wb).reshape(D, P)
+    _, _, _, odist = O.select(Xf, Wf, ref, 1, exclude=ex)
+    el = np.sort(odist[ex == 0])[::-1]
+    mism, banded = 0, 0
+    for k in np.unique(np.linspace(16, 12000, 20).astype(int)):
+        k = int(k)
+        idx, _, cnt = B.select_retrain(X, W, R, k, exclude=E_)
+        torch.cuda.synchronize()
+        cnt = int(cnt.item())
+        assert cnt == k
+        gi = idx.cpu().numpy()[:cnt]
+        assert np.all(np.diff(gi) > 0) and not ex[gi].any()
+        oi = O.select(Xf, Wf, ref, k, exclude=ex)[0]
+        band = np.abs(odist - el[k - 1]) < BAND
+        banded += int(band.sum())
+        mism += len(set(i for i in gi.tolist() if not band[i]) ^ set(i for i in oi.tolist() if not band[i]))
+    _record("topk_sweep", {"mismatched_indices": mism, "banded": banded})
+    assert mism == 0
+
+
+def test_routing_decisions_tau_det_sweep():
+    """Detector decode + routing (Q18/Q20): detection set, class, destination and order bit-exact outside
+    the tau_det band for 20 values of tau_det."""
+    Bn, hw = 4, 416
+    det_spec = S.tiny_yolo_det(in_hw=hw)
+    A, NC = 3, 2
+    p_det = synth.det_head_params(det_spec, synth.init_params(det_spec, seed=21), obj_bias=0.0)
+    xb, _ = synth.drifted_images(Bn, hw, hw, 3, seed=41)
+    xf = synth.bf16_bits_to_f32(xb)
+    raw = O.Model(det_spec).forward(p_det, xf, want_det=True)["det"]
+    G = raw.shape[1]
+    sig = lambda v: 1 / (1 + np.exp(-v.astype(np.float64)))
+    r5 = raw.reshape(Bn, G, G, A, 5 + NC)
+    scores = (sig(r5[..., 4]) * sig(r5[..., 5:].max(-1))).reshape(-1)
+    lo, hi = np.quantile(scores, [0.3, 0.97])
+    m_det = B.Model(det_spec, Bn, params=p_det)
+    max_det = Bn * G * G * A
+    app = B.App([m_det])
+    outs = B.alloc_outs(m_det, Bn, max_det=max_det)
+    x = to_cuda_bf16(xb)
+    mism, banded, detail = 0, 0, []
+    for tau_det in np.linspace(lo, hi, 20):
+        tau_det = float(tau_det)
+        app.infer(x, [tau_det], [outs])
+        torch.cuda.synchronize()
+        n_det = int(outs["n_det"].item())
+        gdet = outs["det_table"].cpu().numpy()[:n_det]
+        odet, on = O.detect(raw, A, NC, S.YOLO_ANCHORS, 32, hw, hw, tau_det)
+        band = np.abs(scores - tau_det) < BAND
+        banded += int(band.sum())
+        cid = lambda r: (int(r[0]) * G * G + int(r[1])) * A + int(r[2])
+        gk = [tuple(int(v) for v in r[:4]) for r in gdet if not band[cid(r)]]
+        ok = [tuple(int(v) for v in r[:4]) for r in odet if not band[cid(r)]]
+        if gk != ok:
+            mism += 1
+            diff = sorted(set(gk) ^ set(ok))[:8]
+            detail.append({"tau_det": tau_det, "diff": [list(d) for d in diff],
+                           "scores": [float(scores[(d[0] * G * G + d[1]) * A + d[2]]) for d in diff],
+                           "cls_margin": [float(np.abs(r5.reshape(-1, 5 + NC)[(d[0] * G * G + d[1]) * A + d[2], 5]
+                                                       - r5.reshape(-1, 5 + NC)[(d[0] * G * G + d[1]) * A + d[2], 6]))
+                                          for d in diff]})
+    _record("tau_det_sweep", {"mismatched_cases": mism, "banded": banded, "candidates": int(scores.size),
+                              "score_quantiles": np.quantile(scores, [0.01, 0.5, 0.99]).tolist(), "detail": detail})
+    app.close()
+    m_det.close()
+    assert mism == 0
