@@ -1,21 +1,30 @@
 #!/usr/bin/env python
-"""AdaInf hot-path benchmark on B200 (BASELINE.json metric, config 2).
+"""AdaInf hot-path benchmark on B200 (BASELINE.json metric; default workload = config 5, the largest single-GPU
+configuration; --config c2 / c3 select the others).
 
-One STEP = one pass of the whole hot path on one batch of synthetic drifted
-input, all through libadainf.so's C-ABI (include/adainf.h):
-  a1-a4  adainf_infer_dag     ResNet-18-EE (4 exits, 10 vehicle classes) on 256 224x224 crops, taus
-                              calibrated once to ~25/25/25/25 exit fractions
-  a7     adainf_select_retrain  16,384-sample window pool (D=64 embeddings -> PCA P=16, cosine distance
-                              to the old mean, 10% already used/excluded) -> k = 1,024
-  a8-a11 adainf_retrain_step_rows  one SGD+momentum step on the 1,024 selected rows of the device-resident
-                              window pool, packed straight from the pool (lr 0.01, mu 0.9)
-                              (N>1: data-parallel, NCCL all-reduce of the fp32 gradient)
+One STEP = one pass of the whole hot path on one batch of synthetic drifted input,
+all through libadainf.so's C-ABI (include/adainf.h):
 
-value = (inference samples + retraining samples) of all ranks / max-over-ranks device time per step.
-e2e   = the same step through the same API with the step's inputs copied H2D from pinned host memory
-        (request batch, candidate embeddings, pool labels) and its results read back D2H.
---impl reference runs the oracle (oracle/, plain C++ fp64) on the box's host cores on a bounded sample
-of the same workload (the reference arm for this tier).
+  c5 / c2 (one application's job, P:51 / P:203 / P:241):
+    version  adainf_model_average  the job starts from the (single) current model version (reading
+                                   Q23: momentum restarts), so every timed step runs the same exit mix
+    a1-a4    adainf_infer_dag      ResNet-18-EE (4 exits, 10 vehicle classes) on 256 224x224 crops; taus
+                                   calibrated to the config's exit fractions (c5 heavy drift 2/2/1/95,
+                                   c2 25/25/25/25)
+    a7       adainf_select_retrain candidate pool (c5: 131,072 x 512 -> PCA 64; c2: 16,384 x 64 -> 16), cosine
+                                   distance to the old mean, 10% already used -> k (8,192 / 1,024)
+    a8-a11   adainf_retrain_step_rows  one SGD + momentum step on the k selected rows of the device-resident
+                                   window pool, packed straight from the pool (lr 0.01, mu 0.9);
+                                   N > 1: data-parallel, NCCL all-reduce of the fp32 gradient
+  c3 (video-surveillance DAG, Fig. 1):
+    a1-a6    adainf_infer_dag      512 416x416 frames -> TinyYOLOv3-like detector -> decode / routing / crop
+                                   (224x224, on device) -> vehicle (10 cls) + person (8 cls) ResNet-18-EE
+
+value = samples (inference rows + retraining rows; c3: frames) of all ranks / max-over-ranks device time per step.
+e2e   = the same step through the same API with the step's inputs copied H2D from pinned host memory (request
+        batch, candidate embeddings, pool labels) and its results read back D2H.
+--impl reference runs the oracle (oracle/, plain C++ fp64) on the box's host cores on a bounded sample of the
+same workload (the reference arm for this tier; its config states the sample).
 """
 from __future__ import annotations
 
@@ -38,46 +47,50 @@ from paper_conf_sigcomm_shubhas23_b200 import synth  # noqa: E402
 
 METRIC = "DAG inference samples/s + retrain samples/s per B200 (1/2/4/8), % of bf16 peak"
 UNIT = "samples/s"
-INF_B, POOL_N, D_EMB, P_EMB, K_SEL = 256, 16384, 64, 16, 1024
 LR, MU = 0.01, 0.9
-EXIT_FRACTIONS = [0.25, 0.25, 0.25]
-BASE_IMAGES = 2048  # distinct synthetic images; the 16,384-sample pool repeats them (DESIGN.md §Input recipe)
+BASE_IMAGES = 2048  # distinct synthetic images; the window pool repeats them (DESIGN.md §Input recipe)
 
-
-def arm_config(world):
-    return {"workload": "BASELINE config 2: ResNet-18-EE (4 exits) vehicle-type classifier, 224x224 crops, "
-                        "inference batch 256 + selection from a 16,384-sample window pool + one retrain step on "
-                        "k=1,024 selected samples",
-            "model": "resnet18_ee", "global_batch": (INF_B + K_SEL) * world, "seq_len": None,
-            "parallelism": f"dp{world}" if world > 1 else "single", "inference_batch": INF_B,
-            "retrain_batch": K_SEL, "pool": POOL_N, "l2": "inputs + activations larger than L2 (no flush)"}
+CONFIGS = {
+    "c2": dict(name="BASELINE config 2: ResNet-18-EE (4 exits) vehicle-type classifier, 224x224 crops, inference "
+                    "batch 256 (exits 25/25/25/25) + selection from a 16,384-sample window pool (D=64 -> P=16) + "
+                    "one retrain step on k=1,024 selected samples",
+               inf_b=256, fractions=[0.25, 0.25, 0.25], pool_n=16384, d=64, p=16, k=1024, heavy=False, seed=2),
+    "c5": dict(name="BASELINE config 5 (heavy drift, largest single-GPU config): ResNet-18-EE (4 exits), 224x224, "
+                    "inference batch 256 with exits 2/2/1/95 + selection from a 131,072-sample pool (D=512 -> P=64) "
+                    "+ one retrain step on k=8,192 selected samples",
+               inf_b=256, fractions=[0.02, 0.02, 0.01], pool_n=131072, d=512, p=64, k=8192, heavy=True, seed=5,
+               tau_sweep=[0.0, 0.5, 0.7, 0.9, 0.99, 2.0]),
+    "c3": dict(name="BASELINE config 3: video-surveillance DAG, 512 frames 416x416 -> TinyYOLOv3-like detector "
+                    "(13x13x3 anchors, ~4 detections/frame, vehicle:person ~3:1) -> on-device crop routing (224x224) "
+                    "-> vehicle-type (10 cls) + person-activity (8 cls) ResNet-18-EE (exits 25/25/25/25)",
+               frames=512, hw=416, det_per_frame=4.0, cap=2048, fractions=[0.25, 0.25, 0.25], seed=3),
+}
 
 
 def peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
             p = json.load(f)
-        return float(p["bf16_tflops"]), float(p.get("bf16_tflops_sustained", p["bf16_tflops"])), float(
-            p["hbm_gbs"]), "measured"
+        return (float(p["bf16_tflops"]), float(p.get("bf16_tflops_sustained", p["bf16_tflops"])), float(p["hbm_gbs"]),
+                "measured", float(p.get("sm_max_mhz", 1965.0)))
     except Exception:
-        return 1590.0, 1400.0, 6650.0, "fallback"
+        return 1590.0, 1400.0, 6650.0, "fallback", 1965.0
 
 
-def flops_model():
-    """Algorithmic FLOPs: per-stage forward MACs of ResNet-18-EE, retraining = 3x fwd - stem dgrad."""
-    spec = S.resnet18_ee()
+def stage_macs_of(spec):
+    """Per-stage forward MACs of an early-exit model (exit FCs excluded) and the stem MACs (op 0 when it is the
+    7x7/2 stem run by the fused stem kernels)."""
     macs = S.macs_per_sample(spec)
-    stage_macs = [0, 0, 0, 0]
+    stage = [0] * sum(1 for o in spec["ops"] if o["kind"] == "exit")
     st = 0
     for o, m in zip(spec["ops"], macs):
-        stage_macs[st] += m
-        if o["kind"] == "exit" and st < 3:
+        if o["kind"] in ("conv", "block"):
+            stage[min(st, len(stage) - 1)] += m
+        if o["kind"] == "exit":
             st += 1
-    conv_macs = sum(m for o, m in zip(spec["ops"], macs) if o["kind"] in ("conv", "block"))
-    stem_macs = macs[0]
-    retrain_flops = 2 * (3 * sum(macs) - stem_macs)
-    retrain_conv_flops = 2 * (3 * conv_macs - stem_macs)
-    return spec, stage_macs, retrain_flops, retrain_conv_flops
+    o0 = spec["ops"][0]
+    stem = macs[0] if (o0["kind"] == "conv" and o0["kh"] == 7 and o0["stride"] == 2) else 0
+    return stage, stem
 
 
 class ClockSampler:
@@ -92,7 +105,7 @@ class ClockSampler:
              "clocks_event_reasons.sw_power_cap")
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={q}",
-                                          "--format=csv,noheader,nounits", "-lms", "200"], stdout=subprocess.PIPE,
+                                          "--format=csv,noheader,nounits", "-lms", "100"], stdout=subprocess.PIPE,
                                          stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
@@ -105,7 +118,10 @@ class ClockSampler:
             if len(parts) >= 7:
                 self.rows.append(parts)
 
-    def stop(self):
+    def mark(self):
+        return len(self.rows)
+
+    def stop(self, since=0):
         if self.proc is None:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
         self.proc.terminate()
@@ -113,85 +129,388 @@ class ClockSampler:
             self.proc.wait(timeout=5)
         except Exception:
             self.proc.kill()
-        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
-        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        rows = self.rows[since:] or self.rows[-3:]
+        sm = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        pw = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[3 + i].lower() in ("active", "1")})
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[3 + i].lower() in ("active", "1")})
         loaded = [s for s in sm if s > 0.5 * (max(mx) if mx else 1)] or sm
         return {"sm_mhz": statistics.median(loaded) if loaded else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(sm)}
+                "reasons": reasons, "samples": len(sm), "power_w_max": max(pw) if pw else None}
 
 
 def dist_setup():
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    return world, rank, local
+    return (int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("RANK", "0")),
+            int(os.environ.get("LOCAL_RANK", "0")))
+
+
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
 
 
 # ------------------------------------------------------------------------------------------------
+# reference arm / cpu baseline: the oracle as it stands on the host cores, bounded samples
+def _oracle_job_sample(O, cfg, n_inf, n_rt, sel_n, sel_k, seed=2):
+    spec = S.resnet18_ee()
+    om = O.Model(spec)
+    p = synth.init_params(spec, seed=seed)
+    xb, y = synth.drifted_images(n_inf + n_rt, 224, 224, 3, seed=seed, heavy=cfg["heavy"])
+    xf = synth.bf16_bits_to_f32(xb)
+    Xb, Wb, ref = synth.embeddings(sel_n, cfg["d"], cfg["p"], seed=3)
+    X = synth.bf16_bits_to_f32(Xb).reshape(sel_n, cfg["d"])
+    W = synth.bf16_bits_to_f32(Wb).reshape(cfg["d"], cfg["p"])
+
+    def step():
+        if n_inf:
+            r = om.forward(p, xf[:n_inf])
+            O.exit_assign(r["conf"], [0.5, 0.5, 0.5])
+        O.select(X, W, ref, sel_k)
+        if n_rt:
+            om.retrain_step(p, np.zeros_like(p), xf[n_inf:], y[n_inf:], lr=LR, mu=MU)
+
+    desc = (f"per step: {n_inf} inference sample(s) (ResNet-18-EE 224x224, full depth + exit rule) + selection over "
+            f"{sel_n:,} candidates (D={cfg['d']} -> P={cfg['p']}, k={sel_k}) + one retrain step on {n_rt} samples")
+    return step, n_inf + n_rt, desc
+
+
+def _oracle_dag_sample(O, cfg, n_frames, max_crops):
+    det_spec = S.tiny_yolo_det(in_hw=cfg["hw"])
+    veh, per = S.resnet18_ee(10), S.resnet18_ee(8)
+    pd = synth.det_head_params(det_spec, synth.init_params(det_spec, seed=31), obj_bias=-2.0, cls_bias=(0.55, -0.55))
+    pv, pp = synth.init_params(veh, seed=32), synth.init_params(per, seed=33)
+    xb, _ = synth.drifted_images(n_frames, cfg["hw"], cfg["hw"], 3, seed=34)
+    xf = synth.bf16_bits_to_f32(xb)
+    odet, ov, opr = O.Model(det_spec), O.Model(veh), O.Model(per)
+
+    def step():
+        raw = odet.forward(pd, xf, want_det=True)["det"]
+        det, n = O.detect(raw, 3, 2, S.YOLO_ANCHORS, 32, cfg["hw"], cfg["hw"], 0.5)
+        det = det[:max_crops]
+        for cls, om, p in ((0, ov, pv), (1, opr, pp)):
+            rows = [r for r in det if int(r[3]) == cls]
+            if rows:
+                crops = np.stack([O.crop(xf[int(r[0])], r[5:9], 224, 224) for r in rows])
+                c = om.forward(p, crops)
+                O.exit_assign(c["conf"], [0.5, 0.5, 0.5])
+
+    desc = (f"per step: {n_frames} frame(s) through the detector (416x416, full depth) + decode + up to {max_crops} "
+            f"crops (224x224) through the two ResNet-18-EE classifiers")
+    return step, n_frames, desc
+
+
+def _oracle_concurrent(O, step, n_jobs, workers):
+    """Run n_jobs copies of one single-threaded oracle step on `workers` host threads (the oracle's C calls
+    release the GIL; its OpenMP runs with 1 thread per call, so a one-sample step uses exactly one core).
+    Returns (wall seconds, per-job seconds)."""
+    from concurrent.futures import ThreadPoolExecutor
+
+    def one(_):
+        t0 = time.perf_counter()
+        step()
+        return time.perf_counter() - t0
+
+    O.set_threads(1)
+    t0 = time.perf_counter()
+    with ThreadPoolExecutor(max_workers=workers) as ex:
+        per = list(ex.map(one, range(n_jobs)))
+    return time.perf_counter() - t0, per
+
+
+def _host_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
 def run_reference(args, world, rank):
-    """Reference arm for this tier: the oracle (plain C++ fp64) on the host cores, bounded sample."""
+    """Reference arm for this tier: the oracle (plain C++ fp64) on the host cores.  A step is a bounded sample of
+    the workload run single-threaded; the K timed steps run concurrently, one per host core, and value = their
+    samples / wall time (the oracle parallelises over samples, so this is how it uses the box's cores)."""
     if rank != 0:
         return 0
     import oracle as O
-    spec = S.resnet18_ee()
-    om = O.Model(spec)
-    p = synth.init_params(spec, seed=2)
-    n_inf, n_rt = 1, 4  # same 1:4 mix as the GPU step (256 : 1024)
-    xb, y = synth.drifted_images(n_inf + n_rt, 224, 224, 3, seed=2)
-    xf = synth.bf16_bits_to_f32(xb)
-    Xb, Wb, ref = synth.embeddings(2048, D_EMB, P_EMB, seed=3)
-    X = synth.bf16_bits_to_f32(Xb).reshape(2048, D_EMB)
-    W = synth.bf16_bits_to_f32(Wb).reshape(D_EMB, P_EMB)
-
-    def step():
-        r = om.forward(p, xf[:n_inf])
-        O.exit_assign(r["conf"], [0.5, 0.5, 0.5])
-        O.select(X, W, ref, K_SEL // 8)
-        om.retrain_step(p, np.zeros_like(p), xf[n_inf:], y[n_inf:], lr=LR, mu=MU)
-
-    for _ in range(args.warmup):
-        step()
-    t0 = time.perf_counter()
-    for _ in range(args.steps):
-        step()
-    dt = (time.perf_counter() - t0) / args.steps
-    v = (n_inf + n_rt) / dt
-    cores = O.get_threads()
-    sample = (f"per step: {n_inf} inference sample (full depth + exit rule) + selection over 2,048 "
-              f"candidates (k=128) + one retrain step on {n_rt} samples, ResNet-18-EE 224x224")
+    cfg = CONFIGS[args.config]
+    if args.config == "c3":
+        step, units, desc = _oracle_dag_sample(O, cfg, 1, 2)
+    else:
+        step, units, desc = _oracle_job_sample(O, cfg, 1, 1, 4096, 256)
+    cores = _host_cores()
+    if args.warmup:
+        _oracle_concurrent(O, step, min(args.warmup, cores), cores)
+    wall, per = _oracle_concurrent(O, step, args.steps, cores)
+    v = units * args.steps / wall
+    cfg_line = {"workload": cfg["name"], "impl_sample": desc + " (single-threaded; the timed steps run concurrently, "
+                f"{cores} at a time)", "model": "resnet18_ee" if args.config != "c3" else
+                "tiny_yolo_det + 2x resnet18_ee", "global_batch": units, "seq_len": None, "parallelism": "single",
+                "note": "bounded CPU sample of the workload (the oracle cannot run the full step in minutes); "
+                        "same metric and unit, different per-step size"}
+    unit = UNIT if args.config != "c3" else "frames/s"
     print(json.dumps({
-        "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True, "scaling": "weak",
-        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": arm_config(world),
-        "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
-        "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "impl": "reference", "metric": METRIC, "value": v, "unit": unit,
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": wall / args.steps * 1e3,
+        "ms_per_step_single_thread_median": statistics.median(per) * 1e3, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic", "config": cfg_line,
+        "cpu_baseline": {"value": v, "unit": unit, "cores": cores, "kind": "oracle", "sample": cfg_line["impl_sample"],
+                         "cpu_model": cpu_model()},
+        "e2e": {"value": v, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)
     return 0
 
 
-def cpu_baseline_leg():
-    """The oracle as it stands on the box's host cores, bounded sample (~10-30 s)."""
+def cpu_baseline_leg(config):
+    """The oracle as it stands on the box's host cores on a bounded sample (~25-40 s): one single-threaded job
+    per core, run concurrently -> the all-cores rate, and each job's own time -> the one-thread rate."""
     import oracle as O
-    spec = S.resnet18_ee()
-    om = O.Model(spec)
-    p = synth.init_params(spec, seed=2)
-    n_inf, n_rt = 4, 16
-    xb, y = synth.drifted_images(n_inf + n_rt, 224, 224, 3, seed=5)
-    xf = synth.bf16_bits_to_f32(xb)
-    Xb, Wb, ref = synth.embeddings(POOL_N, D_EMB, P_EMB, seed=3)
-    t0 = time.perf_counter()
-    r = om.forward(p, xf[:n_inf])
-    O.exit_assign(r["conf"], [0.5, 0.5, 0.5])
-    O.select(synth.bf16_bits_to_f32(Xb).reshape(POOL_N, D_EMB), synth.bf16_bits_to_f32(Wb).reshape(D_EMB, P_EMB),
-             ref, K_SEL)
-    om.retrain_step(p, np.zeros_like(p), xf[n_inf:], y[n_inf:], lr=LR, mu=MU)
-    dt = time.perf_counter() - t0
-    return {"value": (n_inf + n_rt) / dt, "unit": UNIT, "cores": O.get_threads(), "kind": "oracle",
-            "sample": f"{n_inf} inference samples + selection over the {POOL_N}-sample pool (k={K_SEL}) + one "
-                      f"retrain step on {n_rt} samples (ResNet-18-EE 224x224), {dt:.1f} s"}
+    cfg = CONFIGS[config]
+    if config == "c3":
+        step, units, desc = _oracle_dag_sample(O, cfg, 1, 2)
+    else:
+        step, units, desc = _oracle_job_sample(O, cfg, 1, 1, 4096, 256)
+    cores = _host_cores()
+    wall, per = _oracle_concurrent(O, step, cores, cores)
+    O.set_threads(cores)
+    return {"kind": "oracle", "unit": UNIT, "cpu_model": cpu_model(), "cores": cores,
+            "value": units * cores / wall,
+            "sample": f"{cores} concurrent single-threaded jobs, each {desc}; {wall:.1f} s wall",
+            "one_thread": {"value": units / statistics.median(per), "threads": 1,
+                           "sample": f"median single-threaded job time {statistics.median(per):.1f} s"}}
+
+
+# ------------------------------------------------------------------------------------------------
+class JobWorkload:
+    """c2 / c5: one application's job (version average -> early-exit inference -> selection -> retrain step)."""
+
+    def __init__(self, cfg, B, torch, dev, rank, world):
+        self.cfg, self.B, self.torch, self.dev = cfg, B, torch, dev
+        self.world = world
+        self.inf_b, self.k, self.pool_n = cfg["inf_b"], cfg["k"], cfg["pool_n"]
+        spec = S.resnet18_ee()
+        self.spec = spec
+        seed = 100 * cfg["seed"] + rank
+        params = synth.init_params(spec, seed=1)  # identical replicas
+        protos = synth.class_prototypes(10, 224, 224, 3, seed=1244)
+        self.inf_host, _ = synth.drifted_images(self.inf_b, 224, 224, 3, seed=seed, period=1, heavy=cfg["heavy"],
+                                                protos=protos)
+        base_b, base_y = synth.drifted_images(BASE_IMAGES, 224, 224, 3, seed=seed, period=0, heavy=cfg["heavy"],
+                                              protos=protos)
+        self.X_host, Wb, ref = synth.embeddings(self.pool_n, cfg["d"], cfg["p"], seed=seed, drift=2.0 if cfg["heavy"]
+                                                else 1.0)
+        excl = (np.random.default_rng(seed).random(self.pool_n) < 0.1).astype(np.uint8)
+
+        def bf(a):
+            return torch.from_numpy(a.view(np.int16)).to(dev).view(torch.bfloat16)
+
+        self.x_inf = bf(self.inf_host)
+        base = bf(base_b)
+        reps = (self.pool_n + BASE_IMAGES - 1) // BASE_IMAGES
+        self.pool = base.repeat(reps, 1, 1, 1)[:self.pool_n].contiguous()
+        self.pool_y = torch.from_numpy(np.ascontiguousarray(np.tile(base_y, reps)[:self.pool_n])).to(dev)
+        del base
+        self.X = bf(self.X_host).reshape(self.pool_n, cfg["d"])
+        self.W = bf(Wb).reshape(cfg["d"], cfg["p"])
+        self.R = torch.from_numpy(ref).to(dev)
+        self.E = torch.from_numpy(excl).to(dev)
+        self.m = B.Model(spec, max(self.inf_b, self.k), params=params, momentum=MU)
+        self.version = B.Model(spec, 1, params=params, momentum=MU)  # the current model version (P:241)
+        self.app = B.App([self.m])
+        self.outs = B.alloc_outs(self.m, self.inf_b)
+        self.calib = B.alloc_outs(self.m, self.inf_b)
+        self.sel_idx = torch.empty(self.k, dtype=torch.int32, device=dev)
+        self.sel_dist = torch.empty(self.k, dtype=torch.float32, device=dev)
+        self.sel_cnt = torch.empty(1, dtype=torch.int32, device=dev)
+        self.stats = torch.zeros(2, dtype=torch.float32, device=dev)
+        self.taus = [2.0, 2.0, 2.0]
+        self.stage_macs, self.stem_macs = stage_macs_of(spec)
+        self.units = self.inf_b + self.k
+
+    def attach_dp(self, rank, world):
+        import torch.distributed as dist
+        uid = self.B.nccl_unique_id() if rank == 0 else b"\0" * 128
+        obj = [uid]
+        dist.broadcast_object_list(obj, src=0)
+        self.m.dp_attach(obj[0], rank, world)
+
+    def conf_all(self, x=None):
+        torch = self.torch
+        x = self.x_inf if x is None else x
+        conf = np.zeros((x.shape[0], 4), np.float32)
+        for k in range(4):
+            tk = [2.0] * 3
+            if k < 3:
+                tk[k] = 0.0
+            self.app.infer(x, tk, [self.calib])
+            torch.cuda.synchronize()
+            conf[:, k] = self.calib["conf"].cpu().numpy()
+        return conf
+
+    def calibrate(self):
+        """taus at the config's exit fractions, from the version's full-depth confidences on the request batch
+        (widest gap near each target quantile)."""
+        self.B.model_average(self.m, [self.version])
+        self.taus = [float(t) for t in synth.calibrate_thresholds(self.conf_all(), self.cfg["fractions"])]
+
+    def phase_infer(self, xi=None):
+        self.B.model_average(self.m, [self.version])  # the job starts from the current version (P:241)
+        self.app.infer(self.x_inf if xi is None else xi, self.taus, [self.outs])
+
+    def phase_select(self, Xe=None):
+        self.B.select_retrain(self.X if Xe is None else Xe, self.W, self.R, self.k, exclude=self.E,
+                              out_idx=self.sel_idx, out_dist=self.sel_dist, out_count=self.sel_cnt)
+
+    def phase_retrain(self, py=None):
+        self.m.retrain_step_rows(self.pool, self.pool_y if py is None else py, self.sel_idx,
+                                 n_global=self.k * self.world, lr=LR, stats=self.stats, count=self.sel_cnt)
+
+    def step(self, counts_out, xi=None, Xe=None, py=None):
+        self.outs["exit_counts"] = counts_out
+        self.phase_infer(xi)
+        self.phase_select(Xe)
+        self.phase_retrain(py)
+
+    def flops(self, counts):
+        """algorithmic FLOPs per step by kernel class (survivors only for inference; retraining 3x forward minus
+        the stem dgrad; stem in its own classes)"""
+        reach = np.array([self.inf_b - counts[:, :k].sum(1) for k in range(4)]).T.mean(0)
+        nonstem = list(self.stage_macs)
+        nonstem[0] -= self.stem_macs
+        conv_total = sum(nonstem)
+        f = {"conv_fwd": 2.0 * (float(np.dot(reach, nonstem)) + self.k * conv_total),
+             "conv_dgrad": 2.0 * self.k * conv_total,
+             "conv_wgrad": 2.0 * self.k * conv_total,
+             "stem_fwd": 2.0 * self.stem_macs * (reach[0] + self.k),
+             "stem_wgrad": 2.0 * self.stem_macs * self.k,
+             "select_proj": 2.0 * self.pool_n * self.cfg["d"] * self.cfg["p"]}
+        inf = 2.0 * float(np.dot(reach, self.stage_macs))
+        rt = 2.0 * self.k * (3 * sum(self.stage_macs) - self.stem_macs)
+        return f, inf, rt, reach
+
+    def hbm_bytes(self, reach):
+        nparams = sum(int(np.prod(shp)) for _k, _i, _o, shp in S.param_segments(self.spec))
+        conv_params = sum(int(np.prod(shp)) for k_, _i, _o, shp in S.param_segments(self.spec)
+                          if k_ in ("conv_w", "proj_w"))
+        exit_row = [56 * 56 * 64 * 2, 28 * 28 * 128 * 2, 14 * 14 * 256 * 2, 7 * 7 * 512 * 2]
+        return {
+            "sgd_update": nparams * 20 + conv_params * 2,
+            "exit_head": float(np.dot(reach, exit_row)),
+            "exit_head_train": self.k * sum(exit_row),
+            "pack_input": (reach[0] + self.k) * (224 * 224 * 3 * 2 + 112 * 112 * 16 * 2),
+            "select_cosine": self.pool_n * self.cfg["p"] * 4 + self.pool_n,
+            "select_proj": self.pool_n * self.cfg["d"] * 2 + self.pool_n * self.cfg["p"] * 4,
+            "version_average": nparams * 8,
+        }
+
+    def e2e_inputs(self):
+        torch = self.torch
+        h_inf = torch.from_numpy(self.inf_host.view(np.int16)).view(torch.bfloat16).pin_memory()
+        h_X = torch.from_numpy(self.X_host.view(np.int16)).view(torch.bfloat16).reshape(self.pool_n,
+                                                                                        self.cfg["d"]).pin_memory()
+        h_y = self.pool_y.cpu().pin_memory()
+        return [(h_inf, self.x_inf), (h_X, self.X), (h_y, self.pool_y)]
+
+    def e2e_results(self):
+        return [self.outs["exit_id"], self.outs["pred"], self.stats]
+
+
+class DagWorkload:
+    """c3: the video DAG (detector -> crop routing -> two early-exit classifiers), inference only."""
+
+    def __init__(self, cfg, B, torch, dev, rank, world):
+        self.cfg, self.B, self.torch, self.dev = cfg, B, torch, dev
+        self.world = world
+        F, hw, cap = cfg["frames"], cfg["hw"], cfg["cap"]
+        self.F, self.hw, self.cap = F, hw, cap
+        self.det_spec = S.tiny_yolo_det(in_hw=hw)
+        self.veh, self.per = S.resnet18_ee(10), S.resnet18_ee(8)
+        seed = 100 * cfg["seed"] + rank
+        pd = synth.det_head_params(self.det_spec, synth.init_params(self.det_spec, seed=31), obj_bias=-2.0,
+                                   cls_bias=(0.55, -0.55))
+        self.frames_host, _ = synth.drifted_images(F, hw, hw, 3, seed=seed, period=1)
+        self.x = torch.from_numpy(self.frames_host.view(np.int16)).to(dev).view(torch.bfloat16)
+        self.md = B.Model(self.det_spec, F, params=pd)
+        self.mv = B.Model(self.veh, cap, params=synth.init_params(self.veh, seed=32))
+        self.mp = B.Model(self.per, cap, params=synth.init_params(self.per, seed=33))
+        self.app = B.App([self.md, self.mv, self.mp], edges=[(0, 1, B.ROUTE_DET_CROP, 0, 224, 224),
+                                                             (0, 2, B.ROUTE_DET_CROP, 1, 224, 224)],
+                         max_routed_per_dst=cap)
+        G = hw // 32
+        self.G = G
+        self.max_det = F * G * G * 3
+        self.outs = [B.alloc_outs(self.md, F, max_det=self.max_det, n_out_edges=2, max_routed=cap),
+                     B.alloc_outs(self.mv, cap), B.alloc_outs(self.mp, cap)]
+        self.taus = [0.5] + [2.0] * 6
+        self.det_macs = sum(S.macs_per_sample(self.det_spec))
+        self.stage_macs, self.stem_macs = stage_macs_of(self.veh)
+        self.units = F
+        self.k = 0
+
+    def calibrate(self):
+        torch, B = self.torch, self.B
+        # tau_det: ~det_per_frame detections per frame, in the widest nearby score gap
+        self.app.infer(self.x, [-1.0] + [2.0] * 6, self.outs)
+        torch.cuda.synchronize()
+        n = int(self.outs[0]["n_det"].item())
+        sc = np.sort(self.outs[0]["det_table"][:min(n, self.max_det), 4].cpu().numpy())[::-1]
+        want = int(self.cfg["det_per_frame"] * self.F)
+        best, bi = -1.0, want
+        for j in range(max(1, want - want // 20), min(len(sc) - 1, want + want // 20)):
+            if sc[j - 1] - sc[j] > best:
+                best, bi = sc[j - 1] - sc[j], j
+        tau_det = float(0.5 * (sc[bi - 1] + sc[bi]))
+        # classifier taus from their full-depth confidences on this batch's crops
+        taus = [tau_det]
+        for mi in (1, 2):
+            conf = np.zeros((self.cap, 4), np.float32)
+            for k in range(4):
+                tk = [2.0] * 3
+                if k < 3:
+                    tk[k] = 0.0
+                self.app.infer(self.x, [tau_det] + tk + tk, self.outs)
+                torch.cuda.synchronize()
+                conf[:, k] = self.outs[mi]["conf"].cpu().numpy()
+            nr = min(int(self.outs[0]["n_routed"][mi - 1].item()), self.cap)
+            taus += [float(t) for t in synth.calibrate_thresholds(conf[:max(nr, 1)], self.cfg["fractions"])]
+        self.taus = taus
+
+    def step(self, counts_out, xi=None, Xe=None, py=None):
+        self.outs[1]["exit_counts"] = counts_out[:4]
+        self.outs[2]["exit_counts"] = counts_out[4:8]
+        self.app.infer(self.x if xi is None else xi, self.taus, self.outs)
+
+    phase_infer = None
+
+    def flops(self, counts):
+        # counts rows: [veh exit counts (4), person exit counts (4)]
+        fl_cls = 0.0
+        stem_rows = 0.0
+        for off in (0, 4):
+            c = counts[:, off:off + 4]
+            n = c.sum(1)
+            reach = np.array([n - c[:, :k].sum(1) for k in range(4)]).T.mean(0)
+            fl_cls += 2.0 * float(np.dot(reach, self.stage_macs))
+            stem_rows += reach[0]
+        det = 2.0 * self.F * self.det_macs
+        f = {"conv_fwd": det + fl_cls - 2.0 * self.stem_macs * stem_rows, "stem_fwd": 2.0 * self.stem_macs * stem_rows}
+        return f, det + fl_cls, 0.0, None
+
+    def hbm_bytes(self, reach):
+        return {"crop": None}
+
+    def e2e_inputs(self):
+        torch = self.torch
+        h = torch.from_numpy(self.frames_host.view(np.int16)).view(torch.bfloat16).pin_memory()
+        return [(h, self.x)]
+
+    def e2e_results(self):
+        return [self.outs[0]["n_det"], self.outs[1]["pred"], self.outs[2]["pred"]]
 
 
 # ------------------------------------------------------------------------------------------------
@@ -200,148 +519,105 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c5", choices=sorted(CONFIGS))
     ap.add_argument("--impl", default="adainf", choices=["adainf", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-graph", action="store_true", help="time eager launches instead of the captured step graph")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--profile-steps", type=int, default=None)
     args = ap.parse_args()
     world, rank, local = dist_setup()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        # one process per GPU: relaunch this command under torch.distributed.run (rendezvous on 127.0.0.1)
+        import socket
+        s = socket.socket()
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+        s.close()
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+        return subprocess.call(cmd)
     if args.impl == "reference":
         return run_reference(args, world, rank)
     args.warmup = max(args.warmup, 3)
+    cfg = CONFIGS[args.config]
 
     import torch
     from paper_conf_sigcomm_shubhas23_b200 import binding as B
 
     torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        dist.init_process_group("nccl", device_id=dev)
 
     def barrier():
         if world > 1:
             torch.distributed.barrier()
 
-    bf16_burst, bf16_sust, hbm_gbs, peak_src = peaks()
-    spec, stage_macs, retrain_flops, retrain_conv_flops = flops_model()
+    def max_over_ranks(v):
+        if world == 1:
+            return v
+        t = torch.tensor([v], device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        return float(t.item())
 
-    # ---- synthetic inputs (seeded per rank) ----
-    seed = 100 + rank
-    params = synth.init_params(spec, seed=1)  # identical replicas
-    protos = synth.class_prototypes(10, 224, 224, 3, seed=1244)
-    inf_b, _ = synth.drifted_images(INF_B, 224, 224, 3, seed=seed, period=1, protos=protos)
-    base_b, base_y = synth.drifted_images(BASE_IMAGES, 224, 224, 3, seed=seed, period=0, protos=protos)
-    Xb, Wb, ref = synth.embeddings(POOL_N, D_EMB, P_EMB, seed=seed)
-    excl = (np.random.default_rng(seed).random(POOL_N) < 0.1).astype(np.uint8)
-
-    dev = torch.device("cuda", local)
-
-    def bf(a):
-        return torch.from_numpy(a.view(np.int16)).to(dev).view(torch.bfloat16)
-
-    x_inf = bf(inf_b)
-    base = bf(base_b)
-    reps = (POOL_N + BASE_IMAGES - 1) // BASE_IMAGES
-    pool = base.repeat(reps, 1, 1, 1)[:POOL_N].contiguous()
-    pool_y = torch.from_numpy(np.ascontiguousarray(np.tile(base_y, reps)[:POOL_N])).to(dev)
-    del base
-    X = bf(Xb).reshape(POOL_N, D_EMB)
-    W = bf(Wb).reshape(D_EMB, P_EMB)
-    R = torch.from_numpy(ref).to(dev)
-    E = torch.from_numpy(excl).to(dev)
-
-    m = B.Model(spec, max(INF_B, K_SEL), params=params, momentum=MU)
-    if world > 1:
-        import torch.distributed as dist
-        uid = B.nccl_unique_id() if rank == 0 else b"\0" * 128
-        obj = [uid]
-        dist.broadcast_object_list(obj, src=0)
-        m.dp_attach(obj[0], rank, world)
-    app = B.App([m])
-    outs = B.alloc_outs(m, INF_B)
-    sel_idx = torch.empty(K_SEL, dtype=torch.int32, device=dev)
-    sel_dist = torch.empty(K_SEL, dtype=torch.float32, device=dev)
-    sel_cnt = torch.empty(1, dtype=torch.int32, device=dev)
-    stats = torch.zeros(2, dtype=torch.float32, device=dev)
+    bf16_burst, bf16_sust, hbm_gbs, peak_src, sm_max_spec = peaks()
+    wl = (DagWorkload if args.config == "c3" else JobWorkload)(cfg, B, torch, dev, rank, world)
+    if world > 1 and isinstance(wl, JobWorkload):
+        wl.attach_dp(rank, world)
     stream = torch.cuda.current_stream()
-    n_global = K_SEL * world
+    ncnt = 8 if args.config == "c3" else 4
 
-    # thresholds: calibrated on the request batch from full-depth confidences (all exits disabled),
-    # placed in the widest gap near the 25/25/25 quantiles; re-done after warm-up because the warm-up
-    # retraining steps move the exit confidences
-    calib = B.alloc_outs(m, INF_B)
-
-    def calibrate():
-        conf_all = np.zeros((INF_B, 4), np.float32)
-        for k in range(4):
-            tk = [2.0] * 3
-            if k < 3:
-                tk[k] = 0.0
-            app.infer(x_inf, tk, [calib])
-            torch.cuda.synchronize()
-            conf_all[:, k] = calib["conf"].cpu().numpy()
-        return [float(t) for t in synth.calibrate_thresholds(conf_all, EXIT_FRACTIONS)]
-
-    taus = calibrate()
-
-    def step_device(out_counts, xi=None, Xe=None, py=None):
-        xi = x_inf if xi is None else xi
-        Xe = X if Xe is None else Xe
-        py = pool_y if py is None else py
-        outs["exit_counts"] = out_counts
-        app.infer(xi, taus, [outs])
-        B.select_retrain(Xe, W, R, K_SEL, exclude=E, out_idx=sel_idx, out_dist=sel_dist, out_count=sel_cnt)
-        # (the pool keeps >= K_SEL eligible rows, so sel_idx holds K_SEL valid rows)
-        m.retrain_step_rows(pool, py, sel_idx, n_global=n_global, lr=LR, stats=stats)
-
-    cnt_buf = torch.zeros((max(args.steps, 1) + args.warmup + 64, 4), dtype=torch.int32, device=dev)
+    wl.calibrate()
+    cnt_buf = torch.zeros((max(args.steps, 1) + args.warmup + 64, ncnt), dtype=torch.int32, device=dev)
     for i in range(args.warmup):
-        step_device(cnt_buf[-1 - i % 32])
+        wl.step(cnt_buf[-1 - i % 32])
     torch.cuda.synchronize()
-    taus[:] = calibrate()
     barrier()
 
-    # ---- timed region (device time, CUDA events on the launching stream) ----
-    clk = ClockSampler(local)
-    if os.environ.get("ADAINF_BENCH_NO_CLOCKS") != "1":
-        # nvidia-smi's NVML start-up stalls the GPU for tens of ms: wait until it is sampling steadily
-        # (two samples) so the start-up falls before the timed region, not inside its first step
-        clk.start()
-        t_wait = time.time()
-        while len(clk.rows) < 2 and time.time() - t_wait < 10.0:
-            time.sleep(0.05)
-    # the idle gap above lets the GPU drop its clocks: two more untimed steps bring them back up, so the
-    # first timed step is not a clock ramp
-    for i in range(2):
-        step_device(cnt_buf[-1 - i % 32])
-    torch.cuda.synchronize()
-    # the whole step (inference DAG + selection + gather + retrain step, ~190 kernels) captured once as a CUDA
-    # graph and replayed: the same kernels and arguments, without per-launch host / front-end overhead between
-    # them (--no-graph times the eagerly launched step instead)
-    graph, graph_launches = None, 0
-    # (single process only: with N > 1 the step contains the NCCL gradient all-reduce, and a capture that
-    # failed on one rank but not another would leave the ranks' collectives out of step)
-    if not args.no_graph and world == 1:
+    # ---- the step captured once as a CUDA graph and replayed (--no-graph: eager launches) ----
+    graph, graph_launches, graph_note = None, 0, None
+    if not args.no_graph:
         try:
             graph = torch.cuda.CUDAGraph()
             la = B.launch_count()
             with torch.cuda.graph(graph):
-                step_device(cnt_buf[-40])
+                wl.step(cnt_buf[-40])
             graph_launches = B.launch_count() - la
-            graph.replay()
             torch.cuda.synchronize()
-        except Exception as ex:  # capture unsupported here (e.g. a collective): time eager launches
-            print(f"[bench] graph capture failed ({type(ex).__name__}: {ex}); timing eager launches",
-                  file=sys.stderr)
+        except Exception as ex:  # capture unsupported here: time eager launches, say so in the line
+            graph_note = f"graph capture failed ({type(ex).__name__}: {ex}); eager launches"
+            print(f"[bench] {graph_note}", file=sys.stderr)
             graph, graph_launches = None, 0
             torch.cuda.synchronize()
+        # every rank must agree (a capture that failed on one rank only would desynchronise collectives)
+        ok = max_over_ranks(0.0 if graph is not None else 1.0) == 0.0
+        if not ok:
+            graph = None
+        if graph is not None:
+            graph.replay()
+            torch.cuda.synchronize()
+
+    # ---- timed region (device time, CUDA events on the launching stream) ----
+    clk = ClockSampler(local)
+    if os.environ.get("ADAINF_BENCH_NO_CLOCKS") != "1":
+        clk.start()  # NVML start-up stalls the GPU: let it settle before the timed region
+        t_wait = time.time()
+        while len(clk.rows) < 2 and time.time() - t_wait < 10.0:
+            time.sleep(0.05)
+    for i in range(2):  # bring the clocks back up after the idle gap
+        if graph is not None:
+            graph.replay()
+        else:
+            wl.step(cnt_buf[-1 - i % 32])
+    torch.cuda.synchronize()
     l0 = B.launch_count()
     barrier()
     torch.cuda.synchronize()
-    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    mark = clk.mark()
     evs = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
-    ev0.record(stream)
     evs[0].record(stream)
     host_t = [time.perf_counter()]
     for i in range(args.steps):
@@ -349,107 +625,174 @@ def main():
             graph.replay()
             cnt_buf[i].copy_(cnt_buf[-40], non_blocking=True)  # this step's exit counts
         else:
-            step_device(cnt_buf[i])
+            wl.step(cnt_buf[i])
         evs[i + 1].record(stream)
         host_t.append(time.perf_counter())
-    ev1.record(stream)
     torch.cuda.synchronize()
-    step_ms = [round(evs[i].elapsed_time(evs[i + 1]), 3) for i in range(args.steps)]
-    host_enqueue_ms = [round((host_t[i + 1] - host_t[i]) * 1e3, 3) for i in range(args.steps)]
+    step_ms = [evs[i].elapsed_time(evs[i + 1]) for i in range(args.steps)]
     launches = B.launch_count() - l0 + graph_launches * args.steps
+    clocks_timed = {"samples_in_timed_region": clk.mark() - mark}
     barrier()
-    clocks = clk.stop()
-    ms = ev0.elapsed_time(ev1) / args.steps
-    if world > 1:
-        t = torch.tensor([ms], device=dev)
-        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-        ms = float(t.item())
+    ms = max_over_ranks(evs[0].elapsed_time(evs[-1]) / args.steps)
     counts = cnt_buf[:args.steps].cpu().numpy()
-    samples_per_step = (INF_B + K_SEL) * world
+    samples_per_step = wl.units * world
     value = samples_per_step / (ms / 1e3)
 
-    # algorithmic FLOPs of one step (survivors only): per-stage MACs x samples reaching the stage
-    reach = np.array([INF_B - counts[:, :k].sum(1) for k in range(4)]).T.mean(0)
-    inf_flops = 2 * float(np.dot(reach, stage_macs))
-    sel_flops = 2.0 * POOL_N * D_EMB * P_EMB
-    step_flops = inf_flops + K_SEL * retrain_flops + sel_flops
-    pct_peak = step_flops / (ms / 1e3) / (bf16_sust * 1e12) * 100
+    flops_cls, inf_flops, rt_flops, reach = wl.flops(counts)
+    exit_mix = None
+    if isinstance(wl, JobWorkload):
+        mix = counts.mean(0) / wl.inf_b
+        target = list(cfg["fractions"]) + [1.0 - sum(cfg["fractions"])]
+        exit_mix = {"target": target, "timed_mean": [round(float(x), 4) for x in mix],
+                    "max_abs_dev": round(float(np.abs(mix - np.array(target)).max()), 4)}
+    step_flops = inf_flops + rt_flops
 
-    # ---- profiled pass: per-kernel-class device time (events on the launching stream) ----
-    pk = args.profile_steps or args.steps
+    # ---- profiled pass (eager): per-kernel-class and per-phase device time, CUDA events on the stream ----
+    pk = args.profile_steps or max(3, min(args.steps, 10))
+    torch.cuda.synchronize()
     B.prof_reset()
     B.prof_enable(True)
-    torch.cuda.synchronize()
+    ph = {"infer": 0.0, "select": 0.0, "retrain": 0.0}
     ev2, ev3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ev2.record(stream)
     for i in range(pk):
-        step_device(cnt_buf[-1 - i % 32])
+        if isinstance(wl, JobWorkload):
+            e = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+            wl.outs["exit_counts"] = cnt_buf[-1 - i % 32]
+            e[0].record(stream)
+            wl.phase_infer()
+            e[1].record(stream)
+            wl.phase_select()
+            e[2].record(stream)
+            wl.phase_retrain()
+            e[3].record(stream)
+            torch.cuda.synchronize()
+            ph["infer"] += e[0].elapsed_time(e[1])
+            ph["select"] += e[1].elapsed_time(e[2])
+            ph["retrain"] += e[2].elapsed_time(e[3])
+        else:
+            wl.step(cnt_buf[-1 - i % 32])
     ev3.record(stream)
     torch.cuda.synchronize()
     prof = B.prof_query()
     B.prof_enable(False)
     prof_ms = ev2.elapsed_time(ev3) / pk
-    conv_ms = sum(prof[k][1] for k in ("conv_fwd", "conv_dgrad", "conv_wgrad")) / pk
-    conv_launches = sum(prof[k][0] for k in ("conv_fwd", "conv_dgrad", "conv_wgrad")) / pk
-    conv_flops = inf_flops + K_SEL * retrain_conv_flops + sel_flops  # algorithmic MACs on the tensor cores
-    achieved = conv_flops / (conv_ms / 1e3) / 1e12
+    breakdown = {k: round(v[1] / pk, 4) for k, v in sorted(prof.items(), key=lambda kv: -kv[1][1]) if v[0]}
+    launches_per_class = {k: round(v[0] / pk, 2) for k, v in prof.items() if v[0]}
+
+    # per-class rooflines (tensor classes against the burst peak: the SM clocks sit at max, see clocks)
+    def cls_ms(k):
+        return prof[k][1] / pk if k in prof and prof[k][0] else None
+
+    per_class = {}
+    for k, fl in flops_cls.items():
+        t = cls_ms(k)
+        if t:
+            per_class[k] = {"tflop_per_step": round(fl / 1e12, 4), "ms_per_step": round(t, 4),
+                            "achieved_tflops": round(fl / (t / 1e3) / 1e12, 1),
+                            "frac_burst": round(fl / (t / 1e3) / 1e12 / bf16_burst, 3)}
+    gemm = [k for k in ("conv_fwd", "conv_dgrad", "conv_wgrad") if cls_ms(k)]
+    g_fl = sum(flops_cls[k] for k in gemm)
+    g_ms = sum(cls_ms(k) for k in gemm)
+    helpers = [k for k in ("wgrad_reduce", "bias_colsum", "dgrad_sp_prep") if cls_ms(k)]
+    h_ms = g_ms + sum(cls_ms(k) for k in helpers)
+    achieved = g_fl / (g_ms / 1e3) / 1e12
+    all_t = [k for k in ("conv_fwd", "conv_dgrad", "conv_wgrad", "stem_fwd", "stem_wgrad") if cls_ms(k)]
+    all_fl = sum(flops_cls[k] for k in all_t)
+    all_ms = sum(cls_ms(k) for k in all_t)
     traffic = None
     try:
         with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
-            traffic = json.load(f).get("conv_umma_kernel_bytes_per_launch")
+            tj = json.load(f)
+            traffic = tj.get(args.config, {}).get("conv_gemm_bytes_per_step")
     except Exception:
         pass
-    breakdown = {k: round(v[1] / pk, 4) for k, v in sorted(prof.items(), key=lambda kv: -kv[1][1]) if v[0]}
+    roofline = {"bound": "tensor", "kernel": "conv GEMMs (tcgen05 implicit GEMM fwd + dgrad + wgrad, non-stem)",
+                "achieved": achieved, "peak": bf16_burst, "unit": "TFLOP/s", "frac": achieved / bf16_burst,
+                "peak_kind": f"bf16 dense burst ({peak_src}); SM clocks at max during the step (see clocks)",
+                "frac_of_sustained": achieved / bf16_sust, "traffic": traffic,
+                "tflop_per_step": g_fl / 1e12, "kernel_ms_per_step": g_ms, "share_of_step": g_ms / prof_ms,
+                "launches_per_step": sum(launches_per_class.get(k, 0) for k in gemm),
+                "frac_incl_splitk_helpers": g_fl / (h_ms / 1e3) / 1e12 / bf16_burst,
+                "frac_all_contractions_incl_stem": all_fl / (all_ms / 1e3) / 1e12 / bf16_burst,
+                "per_class": per_class}
 
-    # ---- HBM-bound kernels (north_star: compaction / update kernels against HBM bandwidth): algorithmic
-    # bytes per step / their event-timed duration in the profiled pass ----
-    nparams = sum(int(np.prod(shp)) for _k, _i, _o, shp in S.param_segments(spec))
-    conv_params = sum(int(np.prod(shp)) for k_, _i, _o, shp in S.param_segments(spec) if k_ in ("conv_w", "proj_w"))
-    exit_bytes_row = [56 * 56 * 64 * 2, 28 * 28 * 128 * 2, 14 * 14 * 256 * 2, 7 * 7 * 512 * 2]
-    hbm_bytes = {
-        # w, v, g read (12 B), w, v written (8 B), bf16 GEMM-layout shadow of conv weights written (2 B)
-        "sgd_update": nparams * 20 + conv_params * 2,
-        # inference: GAP reads the exit tensor of every row reaching the exit (survivors only)
-        "exit_head": float(np.dot(reach, exit_bytes_row)),
-        # retraining forward: every exit head reads its tensor for all selected rows
-        "exit_head_train": K_SEL * sum(exit_bytes_row),
-        # dT (bf16) + argmax codes read, dZ written at 112x112x64 (stem pool backward)
-        "maxpool_bwd": K_SEL * (56 * 56 * 64 * 3 + 112 * 112 * 64 * 2),
-        # raw NHWC bf16 in, space-to-depth packed rows out (inference batch + the selected pool rows)
-        "pack_input": (INF_B + K_SEL) * (224 * 224 * 3 * 2 + 112 * 112 * 16 * 2),
-    }
+    # HBM-bound kernels: algorithmic bytes per step / event-timed duration
     hbm_kernels = {}
-    for k_, by in hbm_bytes.items():
-        if k_ in prof and prof[k_][0]:
-            t = prof[k_][1] / pk / 1e3
-            hbm_kernels[k_] = {"bytes_per_step": int(by), "ms_per_step": round(t * 1e3, 4),
-                               "achieved_gbs": round(by / t / 1e9, 1), "frac_of_hbm": round(by / t / 1e9 / hbm_gbs, 3)}
+    for k_, by in wl.hbm_bytes(reach).items():
+        t = cls_ms(k_)
+        if t and by:
+            hbm_kernels[k_] = {"bytes_per_step": int(by), "ms_per_step": round(t, 4),
+                               "achieved_gbs": round(by / (t / 1e3) / 1e9, 1),
+                               "frac_of_hbm": round(by / (t / 1e3) / 1e9 / hbm_gbs, 3)}
+    phases = None
+    if isinstance(wl, JobWorkload):
+        pi, ps_, pr = (ph[k] / pk for k in ("infer", "select", "retrain"))
+        phases = {
+            "infer": {"ms": round(pi, 4), "samples_per_s": wl.inf_b * world / (pi / 1e3),
+                      "tflop": inf_flops / 1e12, "frac_burst": inf_flops / (pi / 1e3) / 1e12 / bf16_burst},
+            "select": {"ms": round(ps_, 4), "candidates_per_s": wl.pool_n / (ps_ / 1e3),
+                       "gbs": (wl.pool_n * cfg["d"] * 2) / (ps_ / 1e3) / 1e9,
+                       "frac_hbm": (wl.pool_n * cfg["d"] * 2) / (ps_ / 1e3) / 1e9 / hbm_gbs},
+            "retrain": {"ms": round(pr, 4), "samples_per_s": wl.k * world / (pr / 1e3), "tflop": rt_flops / 1e12,
+                        "frac_burst": rt_flops / (pr / 1e3) / 1e12 / bf16_burst},
+            "note": "eager profiled pass (events around each ABI call); the headline value is the graph-replayed step"}
+
+    # ---- tau sweep (c5: shared tau for all early exits, inference only, eager) ----
+    sweep = None
+    if isinstance(wl, JobWorkload) and cfg.get("tau_sweep") and not args.no_sweep:
+        sweep = []
+        B.model_average(wl.m, [wl.version])
+        cs = torch.zeros(4, dtype=torch.int32, device=dev)
+        for tau in cfg["tau_sweep"]:
+            t3 = [tau] * 3
+            wl.outs["exit_counts"] = cs
+            ea, eb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            wl.app.infer(wl.x_inf, t3, [wl.outs])
+            torch.cuda.synchronize()
+            reps = 5
+            ea.record(stream)
+            for _ in range(reps):
+                wl.app.infer(wl.x_inf, t3, [wl.outs])
+            eb.record(stream)
+            torch.cuda.synchronize()
+            t_ms = ea.elapsed_time(eb) / reps
+            c = cs.cpu().numpy()
+            rch = [wl.inf_b - c[:k].sum() for k in range(4)]
+            fl = 2.0 * float(np.dot(rch, wl.stage_macs))
+            sweep.append({"tau": tau, "exit_counts": c.tolist(), "ms": round(t_ms, 4),
+                          "samples_per_s": round(wl.inf_b / (t_ms / 1e3), 1),
+                          "frac_burst": round(fl / (t_ms / 1e3) / 1e12 / bf16_burst, 3)})
+        wl.outs["exit_counts"] = cnt_buf[-40]
 
     # ---- e2e: same step, inputs H2D from pinned host memory, results D2H, through the same API ----
     e2e = None
     if not args.no_e2e:
-        h_inf = torch.from_numpy(inf_b.view(np.int16)).view(torch.bfloat16).pin_memory()
-        h_X = torch.from_numpy(Xb.view(np.int16)).view(torch.bfloat16).reshape(POOL_N, D_EMB).pin_memory()
-        h_y = pool_y.cpu().pin_memory()
-        h_exit = torch.empty(INF_B, dtype=torch.int8).pin_memory()
-        h_pred = torch.empty(INF_B, dtype=torch.int32).pin_memory()
-        h_stats = torch.empty(2, dtype=torch.float32).pin_memory()
-        h2d = h_inf.numel() * 2 + h_X.numel() * 2 + h_y.numel() * 4
-        d2h = INF_B * 1 + INF_B * 4 + 8
-        # double-buffered inputs: step i+1's H2D copies run on a copy stream while step i computes (a serving
-        # loop overlaps them the same way); every step's inputs are still copied inside the timed region
-        xi_b = [x_inf, torch.empty_like(x_inf)]
-        Xe_b = [X, torch.empty_like(X)]
-        py_b = [pool_y, torch.empty_like(pool_y)]
-        cs = torch.cuda.Stream(device=dev)
+        pairs = wl.e2e_inputs()
+        res = wl.e2e_results()
+        h_res = [torch.empty(r.shape, dtype=r.dtype).pin_memory() for r in res]
+        h2d = sum(h.numel() * h.element_size() for h, _ in pairs)
+        d2h = sum(r.numel() * r.element_size() for r in res)
+        # double-buffered device inputs: step i+1's H2D copies run on a copy stream while step i computes (a
+        # serving loop overlaps them the same way); every step's inputs are still copied inside the timed region
+        bufs = [[d for _, d in pairs], [torch.empty_like(d) for _, d in pairs]]
+
+        def run_with(b, counts_row):
+            ins = bufs[b]
+            if isinstance(wl, JobWorkload):
+                wl.step(counts_row, xi=ins[0], Xe=ins[1], py=ins[2])
+            else:
+                wl.step(counts_row, xi=ins[0])
+
+        cs_ = torch.cuda.Stream(device=dev)
         e2e_graphs = None
-        if graph is not None:  # one captured step per input buffer set
+        if graph is not None:
             torch.cuda.synchronize()
             e2e_graphs = []
             for b in range(2):
                 gb = torch.cuda.CUDAGraph()
                 with torch.cuda.graph(gb):
-                    step_device(cnt_buf[-40], xi_b[b], Xe_b[b], py_b[b])
+                    run_with(b, cnt_buf[-40])
                 e2e_graphs.append(gb)
             torch.cuda.synchronize()
         copied = [torch.cuda.Event() for _ in range(2)]
@@ -461,14 +804,16 @@ def main():
 
         def issue_copy(i):
             b = i % 2
-            with torch.cuda.stream(cs):
-                cs.wait_event(ev4)
+            with torch.cuda.stream(cs_):
+                cs_.wait_event(ev4)
                 if i >= 2:
-                    cs.wait_event(consumed[b])
-                xi_b[b].view(torch.int16).copy_(h_inf.view(torch.int16), non_blocking=True)
-                Xe_b[b].view(torch.int16).copy_(h_X.view(torch.int16), non_blocking=True)
-                py_b[b].copy_(h_y, non_blocking=True)
-                copied[b].record(cs)
+                    cs_.wait_event(consumed[b])
+                for (h, _), d in zip(pairs, bufs[b]):
+                    if h.dtype == torch.bfloat16:
+                        d.view(torch.int16).copy_(h.view(torch.int16), non_blocking=True)
+                    else:
+                        d.copy_(h, non_blocking=True)
+                copied[b].record(cs_)
 
         issue_copy(0)
         for i in range(args.steps):
@@ -479,59 +824,62 @@ def main():
             if e2e_graphs is not None:
                 e2e_graphs[b].replay()
             else:
-                step_device(cnt_buf[-1 - i % 32], xi_b[b], Xe_b[b], py_b[b])
+                run_with(b, cnt_buf[-1 - i % 32])
             consumed[b].record(stream)
-            h_exit.copy_(outs["exit_id"], non_blocking=True)
-            h_pred.copy_(outs["pred"], non_blocking=True)
-            h_stats.copy_(stats, non_blocking=True)
+            for hr, r in zip(h_res, res):
+                hr.copy_(r, non_blocking=True)
         ev5.record(stream)
         torch.cuda.synchronize()
-        ems = ev4.elapsed_time(ev5) / args.steps
-        if world > 1:
-            t = torch.tensor([ems], device=dev)
-            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-            ems = float(t.item())
+        ems = max_over_ranks(ev4.elapsed_time(ev5) / args.steps)
         e2e = {"value": samples_per_step / (ems / 1e3), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                "d2h_bytes_per_step": int(d2h), "ms_per_step": ems,
                "overlap": "step i+1's H2D copies on a copy stream during step i (double-buffered inputs)"}
 
+    clocks = clk.stop(since=mark)
+    clocks.update(clocks_timed)
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         try:
-            cpu = cpu_baseline_leg()
+            cpu = cpu_baseline_leg(args.config)
         except Exception as ex:  # pragma: no cover
             cpu = {"value": None, "unit": UNIT, "cores": None, "kind": "oracle", "sample": f"failed: {ex}"}
 
     if rank == 0:
+        cfg_line = {"workload": cfg["name"], "config": args.config,
+                    "model": "resnet18_ee" if args.config != "c3" else "tiny_yolo_det -> 2x resnet18_ee",
+                    "global_batch": samples_per_step, "seq_len": None,
+                    "parallelism": f"dp{world}" if world > 1 else "single",
+                    "l2": "inputs + activations larger than L2 (no flush)",
+                    "launch": "cuda_graph (one captured step, replayed)" if graph is not None else
+                    (graph_note or "eager"), "thresholds": wl.taus}
+        if isinstance(wl, JobWorkload):
+            cfg_line.update(inference_batch=wl.inf_b, retrain_batch=wl.k, pool=wl.pool_n,
+                            embed=f"D={cfg['d']} -> P={cfg['p']}", exit_fractions=cfg["fractions"])
         line = {
-            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
-            "config": dict(arm_config(world), exit_thresholds=taus,
-                           launch="cuda_graph (one captured step, replayed)" if graph is not None else "eager"),
-            "inference_samples_per_s": INF_B * world / (ms / 1e3),
-            "retrain_samples_per_s": K_SEL * world / (ms / 1e3),
-            "exit_counts_mean": counts.mean(0).round(2).tolist(),
+            "metric": METRIC, "value": value, "unit": UNIT if args.config != "c3" else "frames/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+            "ms_per_step_median": float(np.median(step_ms)), "ms_per_step_p90": float(np.quantile(step_ms, 0.9)),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
+            "data": "synthetic (seeded drifted images / embeddings, random-init weights)",
+            "config": cfg_line,
+            "phases": phases,
+            "exit_mix": exit_mix,
             "algorithmic_tflop_per_step": step_flops / 1e12,
-            "pct_bf16_peak": pct_peak,
-            "pct_bf16_peak_note": f"algorithmic FLOP/s of the whole step / {bf16_sust} TFLOP/s sustained ({peak_src})",
-            "roofline": {"bound": "tensor", "kernel": "conv_umma_kernel (tcgen05 implicit GEMM: fwd+dgrad+wgrad)",
-                         "achieved": achieved, "peak": bf16_sust, "unit": "TFLOP/s", "frac": achieved / bf16_sust,
-                         "traffic": traffic, "peak_kind": f"bf16 sustained ({peak_src})",
-                         "launches_per_step": conv_launches, "kernel_ms_per_step": conv_ms,
-                         "share_of_step": conv_ms / prof_ms},
+            "pct_bf16_peak_step": step_flops / (ms / 1e3) / 1e12 / bf16_burst * 100,
+            "roofline": roofline,
             "kernel_ms_per_step": breakdown,
             "hbm_kernels": {"peak_gbs": hbm_gbs, "peak_kind": f"HBM copy ({peak_src})", "kernels": hbm_kernels},
+            "tau_sweep": sweep,
             "gpu_launches": int(launches),
-            "step_ms": step_ms,
-            "host_enqueue_ms": host_enqueue_ms,
+            "step_ms": [round(x, 3) for x in step_ms],
+            "host_enqueue_ms": [round((host_t[i + 1] - host_t[i]) * 1e3, 3) for i in range(args.steps)],
             "clocks": clocks,
             "e2e": e2e,
             "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)
-    app.close()
-    m.close()
+    wl.app.close()
     if world > 1:
         torch.distributed.destroy_process_group()
     return 0

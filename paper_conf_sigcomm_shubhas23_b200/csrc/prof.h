@@ -34,6 +34,7 @@ enum ProfClass {
   PC_CONV_DGRAD_PREP,
   PC_SURVIVOR_GATHER,
   PC_EXIT_HEAD_TRAIN,
+  PC_VERSION_AVG,
   PROF_NCLASS
 };
 

@@ -153,7 +153,7 @@ extern "C" adainf_status adainf_model_average(adainf_model_t dst, const adainf_m
     if (n <= 16) {
       SrcTable t{};
       for (int v = 0; v < n; ++v) t.p[v] = srcs[v];
-      ProfScope ps(PC_SGD, st);
+      ProfScope ps(PC_VERSION_AVG, st);
       average_kernel<<<blocks, 256, 0, st>>>(d.params.as<float>(), t, n, cnt);
       CK(cudaGetLastError());
     } else {
@@ -161,7 +161,7 @@ extern "C" adainf_status adainf_model_average(adainf_model_t dst, const adainf_m
       CK(cudaMallocAsync((void**)&dsrc, sizeof(float*) * n, st));
       CK(cudaMemcpyAsync(dsrc, srcs.data(), sizeof(float*) * n, cudaMemcpyHostToDevice, st));
       {
-        ProfScope ps(PC_SGD, st);
+        ProfScope ps(PC_VERSION_AVG, st);
         average_kernel<<<blocks, 256, 0, st>>>(d.params.as<float>(), (const float* const*)dsrc, n, cnt);
         CK(cudaGetLastError());
       }

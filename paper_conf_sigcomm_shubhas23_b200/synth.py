@@ -152,7 +152,7 @@ def init_params(spec: dict, seed: int = 0, exit_scale: float = 4.0) -> np.ndarra
 
 
 def det_head_params(spec: dict, params: np.ndarray, obj_bias: float, seed: int = 0,
-                    head_scale: float = 16.0) -> np.ndarray:
+                    head_scale: float = 16.0, cls_bias=None) -> np.ndarray:
     """Bias the detector's final 1x1 conv so the objectness logits sit near `obj_bias` (controls the
     detection rate before tau_det calibration) and scale its weights by `head_scale`: the BN-free leaky
     backbone's features are small (std ~0.1 at the head input), so the scale spreads the raw logits to
@@ -166,6 +166,9 @@ def det_head_params(spec: dict, params: np.ndarray, obj_bias: float, seed: int =
     per = 5 + A["det_classes"]
     for a in range(A["anchors"]):
         p[off + a * per + 4] = obj_bias
+        if cls_bias is not None:  # class prior of the detections (e.g. vehicle : person ~ 3 : 1)
+            for c, v in enumerate(cls_bias):
+                p[off + a * per + 5 + c] = v
     wseg = [s for s in segs if s[0] == "conv_w"][-1]
     _, _, woff, wshp = wseg
     cnt = int(np.prod(wshp))
