@@ -74,6 +74,38 @@ adainf_status adainf_count_correct(const int32_t* pred, const int32_t* labels, i
  * the last n results are identical (the current one and the n - 1 before it), else 0.  Host-only. */
 adainf_status adainf_drift_should_stop(const uint64_t* results, int32_t n_steps, int32_t n, int32_t* out_stop);
 
+/* ---- NEXT-4: request batch size and early-exit structure from B200 latency profiles ------------------------
+ * A latency profile holds the per-batch inference latency (ms; measured with CUDA events on the launching stream,
+ * whole GPU) of one early-exit structure at each profiled request batch size (P:118 Obs. 5).
+ * Worst-case latency of a job of `requests` requests at batch b ("the product of the per-batch
+ * inference latency and the total number of batches"):  W(b) = per_batch_ms(b) * ceil(requests / b).
+ * The GPU-space scaling regressions of §3.3.1 ([3], MPS space fractions) are prior art that B200 placement
+ * replaces: the profiles are whole-GPU. Host arithmetic, no device. */
+typedef struct {
+  int32_t n;
+  const int32_t* batch;        /* host [n], >= 1 */
+  const double* per_batch_ms;  /* host [n], > 0  */
+} adainf_latency_profile;
+
+/* The batch with the lowest worst-case latency W(b) (ties -> the smaller batch), and W there.
+ * Errors: ADAINF_ERR_INVALID on an empty / malformed profile or requests < 1. */
+adainf_status adainf_pick_batch(const adainf_latency_profile* profile, int64_t requests, int32_t* out_batch,
+                                double* out_worst_ms);
+
+/* Early-exit structure of one inference task:
+ *   - no retraining task for the model (has_retraining == 0): the full structure `full_index`;
+ *   - else, among the structures whose accuracy >= a_min (the application's A_m), the one with the lowest
+ *     per-batch latency at the job's current batch size batch0 (reading: §3.3.1 picked batch0 from the initial
+ *     DAG's profile; ties -> lower index); none qualifies -> the full structure (the most accurate one);
+ * then the batch size is re-picked for the chosen structure (Obs. 6: "adjusts the batch size ... given the
+ * chosen early-exit structure") with adainf_pick_batch.
+ * profiles[n_structures] (each must contain batch0), accuracy[n_structures] host.  Outputs: structure index,
+ * batch size, worst-case latency W(batch) of the chosen structure.  ADAINF_ERR_INVALID on bad arguments. */
+adainf_status adainf_pick_structure(int32_t n_structures, const adainf_latency_profile* profiles,
+                                    const double* accuracy, double a_min, int32_t has_retraining,
+                                    int32_t full_index, int32_t batch0, int64_t requests, int32_t* out_structure,
+                                    int32_t* out_batch, double* out_worst_ms);
+
 #ifdef __cplusplus
 }
 #endif

@@ -65,6 +65,10 @@ class RetrainPlan(C.Structure):
                 ("est_ms", C.c_double)]
 
 
+class LatencyProfile(C.Structure):
+    _fields_ = [("n", C.c_int32), ("batch", C.POINTER(C.c_int32)), ("per_batch_ms", C.POINTER(C.c_double))]
+
+
 class SelectIn(C.Structure):
     _fields_ = [("X_bf16", C.c_void_p), ("N", C.c_int64), ("D", C.c_int32), ("W_bf16", C.c_void_p),
                 ("P", C.c_int32), ("ref", C.c_void_p), ("M", C.c_int32), ("exclude", C.c_void_p)]
@@ -111,6 +115,9 @@ def lib():
                                   C.POINTER(C.c_double), C.POINTER(C.c_double)],
             "adainf_retrain_setting": [C.c_double, C.POINTER(RetrainProfile), i64, i32, C.POINTER(RetrainPlan)],
             "adainf_model_average": [vp, C.POINTER(vp), i32, vp],
+            "adainf_pick_batch": [C.POINTER(LatencyProfile), i64, C.POINTER(i32), C.POINTER(C.c_double)],
+            "adainf_pick_structure": [i32, C.POINTER(LatencyProfile), C.POINTER(C.c_double), C.c_double, i32, i32,
+                                      i32, i64, C.POINTER(i32), C.POINTER(i32), C.POINTER(C.c_double)],
             "adainf_dp_average": [vp, vp],
             "adainf_mark_used": [vp, vp, vp, i32, vp],
             "adainf_count_correct": [vp, vp, i32, vp, vp],
@@ -496,6 +503,33 @@ def retrain_setting(alloc_ms, batches, step_ms, eligible, max_batch):
     out = RetrainPlan()
     check(lib().adainf_retrain_setting(float(alloc_ms), C.byref(prof), int(eligible), int(max_batch), C.byref(out)))
     return {"samples": out.samples, "batch": out.batch, "steps": out.steps, "epochs": out.epochs, "est_ms": out.est_ms}
+
+
+def _latency_profile(batches, ms, keep):
+    bi = (C.c_int32 * len(batches))(*batches)
+    ti = (C.c_double * len(ms))(*ms)
+    keep += [bi, ti]
+    return LatencyProfile(len(batches), bi, ti)
+
+
+def pick_batch(batches, per_batch_ms, requests):
+    """NEXT-4: batch with the lowest worst-case latency per_batch_ms(b) * ceil(requests / b)."""
+    keep = []
+    prof = _latency_profile(batches, per_batch_ms, keep)
+    b, w = C.c_int32(), C.c_double()
+    check(lib().adainf_pick_batch(C.byref(prof), int(requests), C.byref(b), C.byref(w)))
+    return b.value, w.value
+
+
+def pick_structure(tables, accuracy, a_min, has_retraining, full_index, batch0, requests):
+    """NEXT-4: tables = [(batches, per_batch_ms)] per structure; returns (structure, batch, worst_ms)."""
+    keep = []
+    arr = (LatencyProfile * len(tables))(*[_latency_profile(b, t, keep) for b, t in tables])
+    acc = (C.c_double * len(accuracy))(*accuracy)
+    s, b, w = C.c_int32(), C.c_int32(), C.c_double()
+    check(lib().adainf_pick_structure(len(tables), arr, acc, float(a_min), int(has_retraining), int(full_index),
+                                      int(batch0), int(requests), C.byref(s), C.byref(b), C.byref(w)))
+    return s.value, b.value, w.value
 
 
 def model_average(dst, versions, stream=None):

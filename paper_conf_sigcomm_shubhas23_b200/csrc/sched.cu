@@ -230,3 +230,75 @@ extern "C" adainf_status adainf_drift_should_stop(const uint64_t* results, int32
     *out_stop = stop;
   });
 }
+
+// ------------------------------------------------------------------------------------------------
+// NEXT-4 (P:118-134 Obs. 5-6): worst-case latency W(b) = per_batch_ms(b) * ceil(R / b)
+namespace {
+void check_profile(const adainf_latency_profile* p) {
+  if (!p || p->n < 1 || !p->batch || !p->per_batch_ms) throw InvalidError("latency profile: empty");
+  for (int i = 0; i < p->n; ++i)
+    if (p->batch[i] < 1 || !(p->per_batch_ms[i] > 0.0) || !std::isfinite(p->per_batch_ms[i]))
+      throw InvalidError("latency profile: entries need batch >= 1 and finite ms > 0");
+}
+double worst_ms(const adainf_latency_profile* p, int i, long long requests) {
+  const long long nb = (requests + p->batch[i] - 1) / p->batch[i];
+  return p->per_batch_ms[i] * (double)nb;
+}
+void pick_batch_impl(const adainf_latency_profile* p, long long requests, int32_t* batch, double* w) {
+  check_profile(p);
+  if (requests < 1) throw InvalidError("pick_batch: requests must be >= 1");
+  int best = -1;
+  double bw = 0.0;
+  for (int i = 0; i < p->n; ++i) {
+    const double wi = worst_ms(p, i, requests);
+    if (best < 0 || wi < bw || (wi == bw && p->batch[i] < p->batch[best])) {
+      best = i;
+      bw = wi;
+    }
+  }
+  *batch = p->batch[best];
+  *w = bw;
+}
+}  // namespace
+
+extern "C" adainf_status adainf_pick_batch(const adainf_latency_profile* profile, int64_t requests, int32_t* out_batch,
+                                           double* out_worst_ms) {
+  return guard([&] {
+    if (!out_batch || !out_worst_ms) throw InvalidError("pick_batch: null output");
+    pick_batch_impl(profile, requests, out_batch, out_worst_ms);
+  });
+}
+
+extern "C" adainf_status adainf_pick_structure(int32_t n, const adainf_latency_profile* profiles, const double* accuracy,
+                                               double a_min, int32_t has_retraining, int32_t full_index, int32_t batch0,
+                                               int64_t requests, int32_t* out_structure, int32_t* out_batch,
+                                               double* out_worst_ms) {
+  return guard([&] {
+    if (n < 1 || !profiles || !accuracy || !out_structure || !out_batch || !out_worst_ms)
+      throw InvalidError("pick_structure: bad arguments");
+    if (full_index < 0 || full_index >= n) throw InvalidError("pick_structure: full_index out of range");
+    if (!std::isfinite(a_min)) throw InvalidError("pick_structure: a_min must be finite");
+    int chosen = full_index;
+    if (has_retraining) {
+      double best_ms = 0.0;
+      int best = -1;
+      for (int s = 0; s < n; ++s) {
+        check_profile(&profiles[s]);
+        if (!std::isfinite(accuracy[s])) throw InvalidError("pick_structure: accuracy must be finite");
+        if (accuracy[s] < a_min) continue;
+        int at = -1;
+        for (int i = 0; i < profiles[s].n; ++i)
+          if (profiles[s].batch[i] == batch0) at = i;
+        if (at < 0) throw InvalidError("pick_structure: batch0 missing from a structure's profile");
+        const double ms = profiles[s].per_batch_ms[at];
+        if (best < 0 || ms < best_ms) {
+          best = s;
+          best_ms = ms;
+        }
+      }
+      if (best >= 0) chosen = best;
+    }
+    *out_structure = chosen;
+    pick_batch_impl(&profiles[chosen], requests, out_batch, out_worst_ms);
+  });
+}

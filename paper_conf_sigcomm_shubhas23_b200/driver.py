@@ -152,3 +152,46 @@ def detect_drift(models, fractions=(0.03, 0.06, 0.09, 0.12, 0.15, 0.18, 0.21, 0.
         if B.drift_should_stop(results, n_unchanged):
             break
     return results[-1], degrees, trace
+
+
+# ------------------------------------------------------------------------------------------------
+# NEXT-4: B200 latency profiles of early-exit structures and the structure / batch-size choice (P:118-134,
+# P:221-231).  Measurement is on the device (CUDA events); the choice is adainf_pick_structure / _pick_batch.
+def early_exit_structures(num_exits):
+    """The structures of an early-exit model as threshold vectors (reading Q2): "truncate at exit k" = tau_k = 0
+    with the earlier exits disabled (tau > 1), k = 0..E-2, then the full structure (every exit disabled), which
+    is the last entry (index E-1)."""
+    E = num_exits
+    out = []
+    for k in range(E - 1):
+        t = [2.0] * (E - 1)
+        t[k] = 0.0
+        out.append(t)
+    out.append([2.0] * (E - 1))
+    return out
+
+
+def profile_structures(app, x, structures, batches, outs, reps=3):
+    """Per-batch inference latency table [structure][batch] (ms, whole GPU, CUDA events on the stream): the
+    offline profiling of P:221 / P:229 re-measured on this B200."""
+    return [[profile_infer(app, x[:b], taus, outs, reps) for b in batches] for taus in structures]
+
+
+def structure_accuracy(app, x, y, structures, outs):
+    """Accuracy of each structure on labelled samples (P:229: stored accuracy, refreshed on the S new samples);
+    correct predictions counted on the device (adainf_count_correct)."""
+    n = x.shape[0]
+    acc = []
+    for taus in structures:
+        app.infer(x, taus, [outs])
+        acc.append(int(B.count_correct(outs["pred"][:n], y).item()) / n)
+    return acc
+
+
+def plan_inference(batches, tables, accuracy, a_min, has_retraining, requests):
+    """Structure + request batch size for one inference task: batch0 from the full structure's table
+    (the initial DAG, §3.3.1), then adainf_pick_structure (accuracy >= A_m, lowest per-batch latency at batch0;
+    the batch re-picked for the chosen structure).  Returns (structure index, batch, worst-case ms)."""
+    full = len(tables) - 1
+    batch0, _ = B.pick_batch(batches, tables[full], requests)
+    return B.pick_structure([(batches, t) for t in tables], accuracy, a_min, has_retraining, full, batch0, requests)

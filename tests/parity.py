@@ -53,8 +53,10 @@ def banded_rows(conf_all, taus, exit_oracle):
     return band
 
 
-def check_infer_parity(orc, gpu, taus):
-    """exit ids, survivor lists, counts bit-exact outside the band; logits rel 2e-2; conf within 1e-3."""
+def check_infer_parity(orc, gpu, taus, conf_atol=2e-3):
+    """exit ids, survivor lists, counts bit-exact outside the band; logits rel 2e-2; confidences within conf_atol
+    (what the kernels achieve: max |dconf| 6e-4 at the decision exits and 1.3e-3 at the final exit of 224x224
+    ResNet-18-EE; reduced geometries drift more, up to ~6e-3 at 64x64, tests/test_gpu_decisions.py)."""
     conf_all = orc["conf"]
     E = conf_all.shape[1]
     eid, surv, counts = O.exit_assign(conf_all, taus)
@@ -76,9 +78,7 @@ def check_infer_parity(orc, gpu, taus):
     ref_logits = orc["logits"][rows, ex, :]
     for i, r in enumerate(rows):
         assert rel(gpu["logits"][r], ref_logits[i]) <= 2e-2, (r, gpu["logits"][r], ref_logits[i])
-    # confidences follow from the logits (rel 2e-2); deep random nets amplify bf16 rounding flips, so
-    # the observed |dconf| is reported by the caller rather than held to the decision band
-    np.testing.assert_allclose(gpu["conf"][rows], conf_all[rows, ex], atol=1e-2)
+    np.testing.assert_allclose(gpu["conf"][rows], conf_all[rows, ex], atol=conf_atol)
     # argmax equal where the top-2 oracle logits are separated
     srt = np.sort(ref_logits, axis=1)
     sep = (srt[:, -1] - srt[:, -2]) > 1e-2 * np.maximum(1, np.abs(srt[:, -1]))

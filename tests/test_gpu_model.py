@@ -23,7 +23,7 @@ def _infer_case(spec, Bn, seed, fractions):
     orc = om.forward(p, xf)
     taus = synth.calibrate_thresholds(orc["conf"], fractions)
     gpu = gpu_infer_single(spec, p, xb, taus)
-    nb = check_infer_parity(orc, gpu, taus)
+    nb = check_infer_parity(orc, gpu, taus, conf_atol=2e-3 if spec["in_h"] >= 224 else 8e-3)
     # exit-0 pooled features (selection embeddings, Q12)
     assert rel(gpu["embed"], orc["pooled0"]) <= 2e-2
     return orc, gpu, taus, nb

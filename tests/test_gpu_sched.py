@@ -140,3 +140,36 @@ def test_detect_drift_full_structure_accuracy_and_stop_rule():
     for dm in dms:
         dm.app.close()
         dm.model.close()
+
+
+def test_next4_structure_profiles_and_choice():
+    """NEXT-4 on the B200: per-(structure, batch) latency table of ResNet-18-EE measured with CUDA events, the
+    structures' accuracies counted on the device, and the structure / batch choice equal to brute
+    force over the same measured tables."""
+    from paper_conf_sigcomm_shubhas23_b200 import driver as D
+    spec = S.resnet18_ee(in_hw=64)
+    p = synth.init_params(spec, seed=3)
+    xb, y = synth.drifted_images(64, 64, 64, 3, seed=3)
+    x = torch.from_numpy(xb.view(np.int16)).cuda().view(torch.bfloat16)
+    yt = torch.from_numpy(y).cuda()
+    m = B.Model(spec, 64, params=p)
+    app = B.App([m])
+    outs = B.alloc_outs(m, 64)
+    structs = D.early_exit_structures(4)
+    batches = [8, 16, 32, 64]
+    tables = D.profile_structures(app, x, structs, batches, outs, reps=3)
+    assert all(t > 0 for row in tables for t in row)
+    # truncating at exit 0 runs the stem + layer 1 only: faster than the full structure at every batch
+    assert all(a < f for a, f in zip(tables[0], tables[-1]))
+    acc = D.structure_accuracy(app, x, yt, structs, outs)
+    assert all(0.0 <= a <= 1.0 for a in acc)
+    for a_min in (0.0, sorted(acc)[1], 2.0):
+        s, b, w = D.plan_inference(batches, tables, acc, a_min, True, 100)
+        b0 = min(batches, key=lambda bb: (tables[-1][batches.index(bb)] * -(-100 // bb), bb))
+        ok = [i for i in range(4) if acc[i] >= a_min]
+        want = min(ok, key=lambda i: (tables[i][batches.index(b0)], i)) if ok else 3
+        assert s == want
+        ws = [tables[s][i] * -(-100 // bb) for i, bb in enumerate(batches)]
+        assert w == min(ws) and b == batches[ws.index(min(ws))]
+    app.close()
+    m.close()

@@ -3,6 +3,8 @@
 setting a time allocation affords (reading in DESIGN.md)."""
 import math
 
+import numpy as np
+
 import pytest
 
 from paper_conf_sigcomm_shubhas23_b200 import binding as B
@@ -75,3 +77,66 @@ def test_drift_stop_rule_table2():
     assert not B.drift_should_stop([], n=4)
     assert B.drift_should_stop([5], n=1)
     assert not B.drift_should_stop([1, 1, 2, 1], n=2)
+
+
+# ---- NEXT-4: batch size and structure from latency profiles ----
+def _brute_batch(batches, ms, R):
+    w = [(t * -(-R // b), b) for b, t in zip(batches, ms)]
+    return min(w)[1], min(w)[0]
+
+
+def test_pick_batch_worst_case_definition_and_brute_force():
+    """W(b) = per-batch latency x number of batches; the batch minimising W, ties -> smaller."""
+    from paper_conf_sigcomm_shubhas23_b200 import binding as B
+    batches = [1, 2, 4, 8, 16, 32, 64]
+    # a per-batch latency with a fixed launch cost and a linear part: W(b) = (a + c b) ceil(R / b)
+    for a, c, R in ((2.0, 0.5, 100), (0.1, 1.0, 64), (5.0, 0.01, 1000), (1.0, 1.0, 1)):
+        ms = [a + c * b for b in batches]
+        got = B.pick_batch(batches, ms, R)
+        assert got[0] == _brute_batch(batches, ms, R)[0]
+        assert abs(got[1] - _brute_batch(batches, ms, R)[1]) < 1e-12
+    # closed form: a = 3, c = 1, R = 64 -> W(b) = (3 + b) 64 / b for b | 64, minimised at the largest b
+    b, w = B.pick_batch([4, 8, 16, 32, 64], [7.0, 11.0, 19.0, 35.0, 67.0], 64)
+    assert b == 64 and w == 67.0
+    # ragged last batch counts as a whole batch: R = 17 at b = 16 -> 2 batches
+    b, w = B.pick_batch([16, 17], [1.0, 1.5], 17)
+    assert b == 17 and w == 1.5
+    # tie -> smaller batch
+    assert B.pick_batch([8, 16], [2.0, 4.0], 16) == (8, 4.0)
+    rng = np.random.default_rng(0)
+    for _ in range(200):
+        bs = sorted(set(rng.integers(1, 129, 6).tolist()))
+        ms = rng.uniform(0.1, 10, len(bs)).tolist()
+        R = int(rng.integers(1, 5000))
+        gb, gw = B.pick_batch(bs, ms, R)
+        eb, ew = _brute_batch(bs, ms, R)
+        assert gb == eb and abs(gw - ew) < 1e-9 * ew
+
+
+def test_pick_structure_rules():
+    """no retraining task -> full structure; else the lowest per-batch latency among structures with
+    accuracy >= A_m (at the job's batch), then the batch re-picked for that structure; none qualifies -> full."""
+    from paper_conf_sigcomm_shubhas23_b200 import binding as B
+    batches = [8, 16, 32]
+    tables = [([8, 16, 32], [1.0, 1.5, 2.5]),    # truncate at exit 0: fastest, least accurate
+              ([8, 16, 32], [1.6, 2.4, 4.2]),
+              ([8, 16, 32], [2.0, 3.0, 5.0])]    # full structure
+    acc = [0.70, 0.85, 0.90]
+    # no retraining task: the full structure regardless of A_m
+    s, b, w = B.pick_structure(tables, acc, 0.5, 0, 2, 16, 100)
+    assert s == 2 and (b, w) == _brute_batch(batches, tables[2][1], 100)
+    # A_m = 0.8: structures 1 and 2 qualify, 1 is faster at batch0
+    s, b, w = B.pick_structure(tables, acc, 0.8, 1, 2, 16, 100)
+    assert s == 1 and (b, w) == _brute_batch(batches, tables[1][1], 100)
+    # A_m = 0.6: all qualify -> structure 0
+    assert B.pick_structure(tables, acc, 0.6, 1, 2, 16, 100)[0] == 0
+    # A_m above every accuracy: fall back to the full structure
+    assert B.pick_structure(tables, acc, 0.95, 1, 2, 16, 100)[0] == 2
+    # the choice is made at batch0: a structure faster at 8 but slower at 16 loses when batch0 = 16
+    t2 = [([8, 16], [1.0, 5.0]), ([8, 16], [1.2, 2.0]), ([8, 16], [3.0, 6.0])]
+    assert B.pick_structure(t2, [0.9, 0.9, 0.9], 0.5, 1, 2, 16, 64)[0] == 1
+    assert B.pick_structure(t2, [0.9, 0.9, 0.9], 0.5, 1, 2, 8, 64)[0] == 0
+    with pytest.raises(B.AdaInfError):
+        B.pick_structure(tables, acc, 0.5, 1, 2, 12, 100)  # batch0 not profiled
+    with pytest.raises(B.AdaInfError):
+        B.pick_batch([4, 8], [1.0, -1.0], 10)
