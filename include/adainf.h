@@ -194,6 +194,18 @@ adainf_status adainf_select_retrain(const adainf_select_in* in, int32_t k, int32
                                     adainf_stream_t stream);
 /* out_idx, out_dist: device [k]; out_count: device [1]; dist_all: device [N] or NULL (excluded -> -1) */
 
+/* Sharded selection: each of G shards of the candidate pool runs adainf_select_retrain on its
+ * own rows with the same k; the G (out_dist, out_idx, out_count) lists are gathered (e.g. an NCCL all-gather) into
+ * dist / idx [n_blocks * block_len] and block_count [n_blocks] (device; NULL -> every block full), and this call
+ * returns the global top-k exactly as adainf_select_retrain on the whole pool would (ties -> lower GLOBAL index,
+ * ascending output, count = min(k, #eligible)): local index i of block b is global index i * idx_mul + b * block_off
+ * (contiguous shards: idx_mul = 1, block_off = rows per shard; index-mod-G shards: idx_mul = G,
+ * block_off = 1), n_total = the global pool size.  Entries with dist < 0 or a global index outside [0, n_total) are
+ * ignored.  Workspace n_total * 4 bytes, stream-ordered.  Errors: ADAINF_ERR_SHAPE on bad sizes. */
+adainf_status adainf_select_merge(const float* dist, const int32_t* idx, const int32_t* block_count, int32_t n_blocks,
+                                  int32_t block_len, int64_t idx_mul, int64_t block_off, int64_t n_total, int32_t k,
+                                  int32_t* out_idx, float* out_dist, int32_t* out_count, adainf_stream_t stream);
+
 /* ---- Incremental-retraining SGD step (readings Q8, Q9, Q22) -----------------------
  * One SGD-with-momentum step on n_local samples (device bf16 NHWC, labels device int32):
  * forward at full depth (all exits), loss L = (1/n_global) sum_n sum_k w_k CE(softmax(l_k(n)), y_n),

@@ -109,6 +109,7 @@ def lib():
             "adainf_app_poll": [vp, vp],
             "adainf_dbg_app_crops": [vp, i32, C.POINTER(vp)],
             "adainf_dp_attach": [vp, vp, i32, i32],
+            "adainf_select_merge": [vp, vp, vp, i32, i32, i64, i64, i64, i32, vp, vp, vp, vp],
             "adainf_nccl_unique_id": [vp],
             "adainf_gather_rows": [vp, vp, vp, i32, i64, vp, vp],
             "adainf_time_split": [C.c_double, C.POINTER(C.c_double), i32, C.POINTER(C.c_double), i32,
@@ -395,6 +396,46 @@ def select_retrain(X, W, ref, k, exclude=None, out_idx=None, out_dist=None, out_
     check(lib().adainf_select_retrain(C.byref(si), int(k), ptr(out_idx), ptr(out_dist), ptr(out_count),
                                       ptr(dist_all), stream_ptr(stream)))
     return out_idx, out_dist, out_count
+
+
+def select_merge(dist, idx, block_count, n_blocks, block_len, idx_mul, block_off, n_total, k, stream=None):
+    """K12: global top-k from gathered per-shard top-k lists (device tensors [n_blocks * block_len])."""
+    import torch
+    dev = dist.device
+    out_idx = torch.empty(k, dtype=torch.int32, device=dev)
+    out_dist = torch.empty(k, dtype=torch.float32, device=dev)
+    out_count = torch.empty(1, dtype=torch.int32, device=dev)
+    check(lib().adainf_select_merge(ptr(dist), ptr(idx), ptr(block_count), int(n_blocks), int(block_len),
+                                    int(idx_mul), int(block_off), int(n_total), int(k), ptr(out_idx), ptr(out_dist),
+                                    ptr(out_count), stream_ptr(stream)))
+    return out_idx, out_dist, out_count
+
+
+def select_retrain_sharded(X_local, W, ref, k, group, exclude=None, mode="contiguous", n_total=None):
+    """Selection over a pool sharded across the ranks of `group`: local exact top-k on this rank's
+    rows (adainf_select_retrain), all-gather of (distance, local index, count) over the process group (NCCL on
+    GPUs), exact merge on the device (adainf_select_merge).  mode "contiguous": rank r holds global rows
+    [r * N_local, (r + 1) * N_local); "mod": rank r holds rows r, r + G, r + 2G, ... (P:243 disjoint shards)."""
+    import torch
+    import torch.distributed as dist
+    G = dist.get_world_size(group)
+    n_local = X_local.shape[0]
+    idx, dd, cnt = select_retrain(X_local, W, ref, k, exclude=exclude)
+    cat = torch.cat([dd.view(torch.int32), idx, cnt]).contiguous()
+    gathered = [torch.empty_like(cat) for _ in range(G)]
+    if dist.get_backend(group) == "gloo":
+        g_cpu = [torch.empty_like(cat, device="cpu") for _ in range(G)]
+        dist.all_gather(g_cpu, cat.cpu(), group=group)
+        gathered = [t.to(X_local.device) for t in g_cpu]
+    else:
+        dist.all_gather(gathered, cat, group=group)
+    st = torch.stack(gathered)  # [G][2k + 1]
+    dists = st[:, :k].contiguous().view(torch.float32).reshape(-1)
+    idxs = st[:, k:2 * k].contiguous().reshape(-1)
+    cnts = st[:, 2 * k].contiguous()
+    total = n_total or n_local * G
+    mul, off = (1, n_local) if mode == "contiguous" else (G, 1)
+    return select_merge(dists, idxs, cnts, G, k, mul, off, total, k)
 
 
 def gather_rows(src, idx, count, n, dst, stream=None):

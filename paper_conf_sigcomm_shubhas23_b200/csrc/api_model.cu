@@ -7,6 +7,9 @@
 #include "model.h"
 
 namespace adainf {
+void select_merge(const float* dist, const int32_t* idx, const int32_t* block_count, int n_blocks, int block_len,
+                  long long idx_mul, long long block_off, long long n_total, int k, int32_t* out_idx, float* out_dist,
+                  int32_t* out_count, cudaStream_t st);
 void select_retrain(const adainf_select_in& in, int k, int32_t* out_idx, float* out_dist, int32_t* out_count,
                     float* dist_all, cudaStream_t st);
 }
@@ -320,6 +323,18 @@ extern "C" adainf_status adainf_select_retrain(const adainf_select_in* in, int32
     if (!in || !out_idx || !out_count) throw InvalidError("select: null argument");
     require_device();
     select_retrain(*in, k, out_idx, out_dist, out_count, dist_all, (cudaStream_t)stream);
+  });
+}
+
+extern "C" adainf_status adainf_select_merge(const float* dist, const int32_t* idx, const int32_t* block_count,
+                                             int32_t n_blocks, int32_t block_len, int64_t idx_mul, int64_t block_off,
+                                             int64_t n_total, int32_t k, int32_t* out_idx, float* out_dist,
+                                             int32_t* out_count, adainf_stream_t stream) {
+  return guard([&] {
+    if (!out_idx || !out_count) throw InvalidError("select_merge: null output");
+    require_device();
+    select_merge(dist, idx, block_count, n_blocks, block_len, idx_mul, block_off, n_total, k, out_idx, out_dist,
+                 out_count, (cudaStream_t)stream);
   });
 }
 

@@ -277,6 +277,26 @@ __global__ void emit_write_kernel(const uint32_t* __restrict__ keys, long long N
   }
 }
 
+// exact top-k of 32-bit keys (0 = not eligible), ties -> lower position, emitted in ascending position order
+static void topk_emit(const uint32_t* keys, long long N, int k, RadixState* rs, int* blk, int* offs, int32_t* out_idx,
+                      float* out_dist, int32_t* out_count, cudaStream_t st) {
+  const long long nb = (N + EMIT_THREADS - 1) / EMIT_THREADS;
+  const int k_eff = (int)std::min<long long>(k, N);  // the k-th largest must exist
+  ProfScope ps_topk(PC_SELECT_TOPK, st, 12);
+  radix_init_kernel<<<1, 256, 0, st>>>(rs, k_eff);
+  const int hb = (int)std::min<long long>((N + 1023) / 1024, 4LL * num_sms());
+  for (int pass = 0; pass < 4; ++pass) {
+    const int shift = 24 - 8 * pass;
+    const uint32_t mask_hi = pass == 0 ? 0u : (0xFFFFFFFFu << (32 - 8 * pass));
+    radix_hist_kernel<<<hb, 256, 0, st>>>(keys, N, rs, shift, mask_hi, pass == 0);
+    radix_pick_kernel<<<1, 32, 0, st>>>(rs, shift, pass == 3);
+  }
+  emit_count_kernel<<<(unsigned)nb, EMIT_THREADS, 0, st>>>(keys, N, rs, blk);
+  emit_scan_kernel<<<1, 32, 0, st>>>((int)nb, rs, blk, offs, out_count, k);
+  emit_write_kernel<<<(unsigned)nb, EMIT_THREADS, 0, st>>>(keys, N, rs, offs, out_idx, out_dist, k);
+  CK(cudaGetLastError());
+}
+
 struct SelectWs {
   size_t bytes(long long N, int P, int M) const {
     const long long nb = (N + EMIT_THREADS - 1) / EMIT_THREADS;
@@ -344,20 +364,60 @@ void select_retrain(const adainf_select_in& in, int k, int32_t* out_idx, float* 
       cosine_key_kernel<true><<<(unsigned)((N * 32 + 255) / 256), 256, 0, st>>>(in.X_bf16, N, P, mu, mun, M,
                                                                                in.exclude, keys, dist_all);
   }
-  const int k_eff = (int)std::min<long long>(k, N);  // the k-th largest must exist
-  ProfScope ps_topk(PC_SELECT_TOPK, st, 12);
-  radix_init_kernel<<<1, 256, 0, st>>>(rs, k_eff);
-  const int hb = (int)std::min<long long>((N + 1023) / 1024, 4LL * num_sms());
-  for (int pass = 0; pass < 4; ++pass) {
-    const int shift = 24 - 8 * pass;
-    const uint32_t mask_hi = pass == 0 ? 0u : (0xFFFFFFFFu << (32 - 8 * pass));
-    radix_hist_kernel<<<hb, 256, 0, st>>>(keys, N, rs, shift, mask_hi, pass == 0);
-    radix_pick_kernel<<<1, 32, 0, st>>>(rs, shift, pass == 3);
+  topk_emit(keys, N, k, rs, blk, offs, out_idx, out_dist, out_count, st);
+  CK(cudaFreeAsync(wsp, st));
+}
+
+// K12: merge of per-shard top-k lists into the global top-k.  Candidate block b (one per shard,
+// block_len entries, the first block_count[b] valid) holds local indices i -> global index i * idx_mul + b *
+// block_off, with their distances; the keys are scattered into a dense key array over the global index space so
+// the same radix select + ascending emit applies (ties -> lower GLOBAL index, reading Q15).
+__global__ void merge_scatter_kernel(const float* __restrict__ dist, const int32_t* __restrict__ idx,
+                                     const int32_t* __restrict__ block_count, int n_blocks, int block_len,
+                                     long long idx_mul, long long block_off, long long n_total,
+                                     uint32_t* __restrict__ keys) {
+  const long long t = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+  if (t >= (long long)n_blocks * block_len) return;
+  const int b = (int)(t / block_len), j = (int)(t - (long long)b * block_len);
+  const int cnt = block_count ? min(block_count[b], block_len) : block_len;
+  if (j >= cnt) return;
+  const float d = dist[t];
+  const long long g = (long long)idx[t] * idx_mul + b * block_off;
+  if (g < 0 || g >= n_total || !(d >= 0.f)) return;
+  keys[g] = __float_as_uint(d) + 1u;
+}
+
+void select_merge(const float* dist, const int32_t* idx, const int32_t* block_count, int n_blocks, int block_len,
+                  long long idx_mul, long long block_off, long long n_total, int k, int32_t* out_idx, float* out_dist,
+                  int32_t* out_count, cudaStream_t st) {
+  if (n_blocks <= 0 || block_len <= 0 || n_total <= 0 || n_total > (1LL << 31) - 1 || k <= 0 || idx_mul <= 0 ||
+      block_off < 0)
+    throw ShapeError("select_merge: bad sizes");
+  if (!dist || !idx) throw InvalidError("select_merge: dist and idx are required");
+  const long long nb = (n_total + EMIT_THREADS - 1) / EMIT_THREADS;
+  const size_t bytes = (size_t)n_total * 4 + 256 + sizeof(RadixState) + 256 + (size_t)nb * 16 + 512;
+  void* wsp = nullptr;
+  CK(cudaMallocAsync(&wsp, bytes, st));
+  char* w = (char*)wsp;
+  auto take = [&](size_t b) {
+    char* p = w;
+    w += (b + 255) / 256 * 256;
+    return p;
+  };
+  uint32_t* keys = (uint32_t*)take((size_t)n_total * 4);
+  RadixState* rs = (RadixState*)take(sizeof(RadixState));
+  int* blk = (int*)take((size_t)nb * 8);
+  int* offs = (int*)take((size_t)nb * 8);
+  CK(cudaMemsetAsync(keys, 0, (size_t)n_total * 4, st));
+  {
+    ProfScope ps(PC_SELECT_COSINE, st);
+    const long long n = (long long)n_blocks * block_len;
+    merge_scatter_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(dist, idx, block_count, n_blocks, block_len,
+                                                                     idx_mul, block_off, n_total, keys);
   }
-  emit_count_kernel<<<(unsigned)nb, EMIT_THREADS, 0, st>>>(keys, N, rs, blk);
-  emit_scan_kernel<<<1, 32, 0, st>>>((int)nb, rs, blk, offs, out_count, k);
-  emit_write_kernel<<<(unsigned)nb, EMIT_THREADS, 0, st>>>(keys, N, rs, offs, out_idx, out_dist, k);
-  CK(cudaGetLastError());
+  RadixState* unused = nullptr;
+  (void)unused;
+  topk_emit(keys, n_total, k, rs, blk, offs, out_idx, out_dist, out_count, st);
   CK(cudaFreeAsync(wsp, st));
 }
 

@@ -158,3 +158,52 @@ def test_retrain_rows_count_and_out_of_range_rows_contribute_nothing():
     g2 = m.get_grads()
     m.close()
     assert rel(g2, g_ref) <= 1e-5
+
+
+def _sel_worker(rank, world, port, mode, q):
+    try:
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        torch.cuda.set_device(0)
+        N, D, P, k = 8192, 64, 16, 700
+        Xb, Wb, ref = synth.embeddings(N, D, P, seed=17)
+        ex = (np.random.default_rng(17).random(N) < 0.1).astype(np.uint8)
+        rows = np.arange(N)[rank::world] if mode == "mod" else np.arange(N).reshape(world, -1)[rank]
+        X = torch.from_numpy(Xb.reshape(N, D)[rows].view(np.int16)).cuda().view(torch.bfloat16)
+        W = torch.from_numpy(Wb.view(np.int16)).cuda().view(torch.bfloat16).reshape(D, P)
+        e = torch.from_numpy(ex[rows]).cuda()
+        idx, dd, cnt = B.select_retrain_sharded(X, W, torch.from_numpy(ref).cuda(), k, dist.group.WORLD, exclude=e,
+                                                mode=mode, n_total=N)
+        torch.cuda.synchronize()
+        c = int(cnt.item())
+        q.put((rank, (idx.cpu().numpy()[:c].copy(), dd.cpu().numpy()[:c].copy())))
+        dist.destroy_process_group()
+    except Exception as ex_:  # pragma: no cover
+        q.put((rank, repr(ex_)))
+
+
+@pytest.mark.parametrize("mode", ["contiguous", "mod"])
+def test_sharded_selection_k12_equals_single_gpu(mode):
+    """K12: per-shard exact top-k + all-gather + adainf_select_merge == adainf_select_retrain on the
+    whole pool, bit for bit (index set, order, distances), for contiguous and index-mod-G shards."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_sel_worker, args=(r, 2, port, mode, q)) for r in range(2)]
+    for pr in procs:
+        pr.start()
+    res = dict(q.get(timeout=600) for _ in range(2))
+    for pr in procs:
+        pr.join(timeout=60)
+    assert all(isinstance(v, tuple) for v in res.values()), res
+    N, D, P, k = 8192, 64, 16, 700
+    Xb, Wb, ref = synth.embeddings(N, D, P, seed=17)
+    ex = (np.random.default_rng(17).random(N) < 0.1).astype(np.uint8)
+    X = torch.from_numpy(Xb.view(np.int16)).cuda().view(torch.bfloat16).reshape(N, D)
+    W = torch.from_numpy(Wb.view(np.int16)).cuda().view(torch.bfloat16).reshape(D, P)
+    idx, dd, cnt = B.select_retrain(X, W, torch.from_numpy(ref).cuda(), k, exclude=torch.from_numpy(ex).cuda())
+    torch.cuda.synchronize()
+    c = int(cnt.item())
+    for r in range(2):
+        assert np.array_equal(res[r][0], idx.cpu().numpy()[:c])
+        assert np.array_equal(res[r][1], dd.cpu().numpy()[:c])
