@@ -400,7 +400,9 @@ class JobWorkload:
         exit_row = [56 * 56 * 64 * 2, 28 * 28 * 128 * 2, 14 * 14 * 256 * 2, 7 * 7 * 512 * 2]
         return {
             "sgd_update": nparams * 20 + conv_params * 2,
-            "exit_head": float(np.dot(reach, exit_row)),
+            # fused K4 + K5: GAP read of every row reaching the exit + the survivors' row copy (read + write) into
+            # the next stage's dense input
+            "exit_head": float(np.dot(reach, exit_row)) + 2.0 * sum(reach[k + 1] * exit_row[k] for k in range(3)),
             "exit_head_train": self.k * sum(exit_row),
             "pack_input": (reach[0] + self.k) * (224 * 224 * 3 * 2 + 112 * 112 * 16 * 2),
             "select_cosine": self.pool_n * self.cfg["p"] * 4 + self.pool_n,

@@ -397,6 +397,220 @@ void launch_exit_head(const ExitHeadArgs& a, cudaStream_t st, int prof_class) {
 }
 
 // ------------------------------------------------------------------------------------------------
+// K4 + K5 in one kernel (north_star "exit heads"): per row the exit head (GAP -> FC -> softmax confidence /
+// entropy / argmax), the threshold decision, and the stable compaction of the survivors by a single-pass
+// decoupled look-back scan over the rows (row order = ticket order, so every predecessor is resident or done:
+// no deadlock), then each surviving CTA copies its own row of the stage tensor to its compacted slot of the next
+// stage's dense input (the row was just streamed for the GAP, so the copy reads it back from L2).
+// Status words: bits 31..30 = 1 (aggregate of this row) / 2 (inclusive prefix), bits 29..0 = value; the workspace
+// ([0] ticket, [1..] status per row) is zeroed by a memset node before the kernel.
+struct ExitFusedArgs {
+  ExitHeadArgs h;
+  unsigned* ws;
+  int* pos_next;
+  int* orig_next;
+  int* count_next;
+  int32_t* counts_out;
+  int32_t* surv_out;
+  int32_t* last_count_out;
+  int last_index;
+  const bf16* src;   // stage tensor rows [n][row_elems] (nullptr: no survivor copy)
+  bf16* dense_next;  // [n][row_elems]
+  long long row_elems;
+};
+
+__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_u32(unsigned* p, unsigned v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+template <int EH_THREADS>
+__global__ void __launch_bounds__(EH_THREADS) exit_fused_kernel(const ExitFusedArgs F) {
+  const ExitHeadArgs& a = F.h;
+  __shared__ int s_row, s_exit, s_am, s_excl;
+  __shared__ float s_conf, s_ent;
+  const int t = threadIdx.x;
+  if (t == 0) s_row = (int)atomicAdd(F.ws, 1u);
+  __syncthreads();
+  const int j = s_row;
+  const int n_rows = a.count ? *a.count : a.n_static;
+  if (j >= n_rows) {
+    if (n_rows == 0 && j == 0 && t == 0 && !a.is_final) {  // empty stage: the counts still have to be written
+      *F.count_next = 0;
+      if (F.counts_out) {
+        F.counts_out[a.exit_index] = 0;
+        if (F.last_count_out) F.counts_out[F.last_index] = 0;
+      }
+    }
+    return;
+  }
+  extern __shared__ float sh[];
+  const int C = a.C, CV = C / 8;
+  const int groups = EH_THREADS / CV;
+  float acc[8];
+#pragma unroll
+  for (int q = 0; q < 8; ++q) acc[q] = 0.f;
+  const int v = t % CV, g0 = t / CV;
+  if (g0 < groups) {
+    const bf16* base = a.fmap + (long long)j * a.HW * C + v * 8;
+    int pix = g0;
+    for (; pix + 7 * groups < a.HW; pix += 8 * groups) {
+      uint4 raw[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) raw[u] = __ldg((const uint4*)(base + (long long)(pix + u * groups) * C));
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const bf16* hh = (const bf16*)&raw[u];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) acc[q] += __bfloat162float(hh[q]);
+      }
+    }
+    for (; pix < a.HW; pix += groups) {
+      const uint4 raw = __ldg((const uint4*)(base + (long long)pix * C));
+      const bf16* hh = (const bf16*)&raw;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) acc[q] += __bfloat162float(hh[q]);
+    }
+#pragma unroll
+    for (int q = 0; q < 8; ++q) sh[g0 * C + v * 8 + q] = acc[q];
+  }
+  __syncthreads();
+  float* pooled = sh + groups * C;
+  float* logits = pooled + C;
+  const float inv_hw = 1.0f / (float)a.HW;
+  for (int c = t; c < C; c += EH_THREADS) {
+    float s = 0.f;
+    for (int g = 0; g < groups; ++g) s += sh[g * C + c];
+    pooled[c] = s * inv_hw;
+  }
+  __syncthreads();
+  {
+    const int wp = t >> 5, ln = t & 31;
+    for (int k = wp; k < a.ncls; k += EH_THREADS / 32) {
+      float l = 0.f;
+      for (int c = ln; c < C; c += 32) l = fmaf(pooled[c], __ldg(a.Wk + c * a.ncls + k), l);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) l += __shfl_xor_sync(0xffffffffu, l, o);
+      if (ln == 0) logits[k] = __fadd_rn(l, a.bk[k]);
+    }
+  }
+  __syncthreads();
+  const int orig = a.orig ? a.orig[j] : j;
+  if (a.embed)
+    for (int c = t; c < C; c += EH_THREADS) a.embed[(long long)orig * C + c] = pooled[c];
+  if (t == 0) {
+    int am = 0;
+    for (int k = 1; k < a.ncls; ++k)
+      if (logits[k] > logits[am]) am = k;
+    const float m = logits[am];
+    float s = 0.f, tt = 0.f;
+    for (int k = 0; k < a.ncls; ++k) {
+      const float e = expf(logits[k] - m);
+      s += e;
+      tt += e * (logits[k] - m);
+    }
+    const float conf = 1.0f / s;
+    s_conf = conf;
+    s_ent = logf(s) - tt / s;
+    s_am = am;
+    s_exit = a.is_final || conf >= a.tau;
+  }
+  __syncthreads();
+  const int ex = s_exit;
+  if (ex) {
+    if (t == 0) {
+      if (a.exit_id) a.exit_id[orig] = (int8_t)a.exit_index;
+      if (a.pred) a.pred[orig] = s_am;
+      if (a.conf) a.conf[orig] = s_conf;
+      if (a.entropy) a.entropy[orig] = s_ent;
+    }
+    if (a.logits)
+      for (int k = t; k < a.ncls; k += EH_THREADS) a.logits[(long long)orig * a.ncls + k] = logits[k];
+  }
+  if (a.is_final) return;
+  // ---- decoupled look-back: exclusive count of surviving rows before j ----
+  unsigned* status = F.ws + 1;
+  const unsigned mine = ex ? 0u : 1u;
+  if (t < 32) {
+    if (t == 0) st_release_u32(status + j, (1u << 30) | mine);
+    int excl = 0;
+    int k = j - 1;
+    while (k >= 0) {
+      const int idx = k - t;  // lane t looks at row k - t
+      unsigned sv = 0;
+      bool ready;
+      do {
+        sv = idx >= 0 ? ld_acquire_u32(status + idx) : (2u << 30);
+        ready = (sv >> 30) != 0;
+      } while (!__all_sync(0xffffffffu, ready));
+      const unsigned incl_mask = __ballot_sync(0xffffffffu, idx >= 0 && (sv >> 30) == 2u);
+      // lanes up to (and including) the first inclusive prefix contribute
+      const int stop = incl_mask ? __ffs(incl_mask) - 1 : 31;
+      int val = (t <= stop && idx >= 0) ? (int)(sv & 0x3FFFFFFFu) : 0;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) val += __shfl_xor_sync(0xffffffffu, val, o);
+      excl += val;
+      if (incl_mask) break;
+      k -= 32;
+    }
+    if (t == 0) {
+      st_release_u32(status + j, (2u << 30) | (unsigned)(excl + (int)mine));
+      s_excl = excl;
+      if (j == n_rows - 1) {
+        const int nn = excl + (int)mine;
+        *F.count_next = nn;
+        if (F.counts_out) {
+          F.counts_out[a.exit_index] = n_rows - nn;
+          if (F.last_count_out) F.counts_out[F.last_index] = nn;
+        }
+      }
+    }
+  }
+  __syncthreads();
+  if (ex) return;
+  const int o = s_excl;
+  if (t == 0) {
+    F.pos_next[o] = j;
+    F.orig_next[o] = orig;
+    if (F.surv_out) F.surv_out[o] = orig;
+  }
+  if (F.src) {
+    const uint4* sp = (const uint4*)(F.src + (long long)j * F.row_elems);
+    uint4* dp = (uint4*)(F.dense_next + (long long)o * F.row_elems);
+    const long long nv = F.row_elems / 8;
+    for (long long i = t; i < nv; i += EH_THREADS) dp[i] = sp[i];
+  }
+}
+
+size_t exit_fused_ws_bytes(int max_batch) { return (size_t)(max_batch + 1) * 4; }
+
+void launch_exit_fused(const ExitHeadArgs& h, unsigned* ws, int* pos_next, int* orig_next, int* count_next,
+                       int32_t* counts_out, int32_t* surv_out, int32_t* last_count_out, int last_index,
+                       const bf16* src, bf16* dense_next, long long row_elems, cudaStream_t st) {
+  if (h.n_static <= 0) return;
+  const bool wide = h.n_static < 4 * num_sms();
+  const bool widest = h.n_static <= 2 * num_sms();
+  const int T = widest ? 1024 : (wide ? 512 : 128);
+  if (h.C % 8 || (T % (h.C / 8)) != 0 || h.C / 8 > 128)
+    throw ShapeError("exit head: C must be 8 * a power of two <= 1024");
+  if (src && (row_elems % 8)) throw ShapeError("exit_fused: row must be a multiple of 16 bytes");
+  const int groups = T / (h.C / 8);
+  const size_t smem = (size_t)(groups * h.C + h.C + h.ncls) * sizeof(float);
+  ExitFusedArgs F{h, ws, pos_next, orig_next, count_next, counts_out, surv_out, last_count_out, last_index, src,
+                  dense_next, row_elems};
+  CK(cudaMemsetAsync(ws, 0, (size_t)(h.n_static + 1) * 4, st));
+  ProfScope ps(PC_EXIT_HEAD, st);
+  if (widest) exit_fused_kernel<1024><<<h.n_static, 1024, smem, st>>>(F);
+  else if (wide) exit_fused_kernel<512><<<h.n_static, 512, smem, st>>>(F);
+  else exit_fused_kernel<128><<<h.n_static, 128, smem, st>>>(F);
+  CK(cudaGetLastError());
+}
+
+// ------------------------------------------------------------------------------------------------
 // Stable compaction of alive rows (warp ballot + popc, block scan), single CTA, rows in chunks of 1024.
 __global__ void __launch_bounds__(1024) compact_kernel(const uint8_t* __restrict__ alive, const int* count,
                                                        int n_static, const int* __restrict__ orig,

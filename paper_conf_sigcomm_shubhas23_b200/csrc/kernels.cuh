@@ -50,6 +50,13 @@ struct ExitHeadArgs {
 };
 void launch_exit_head(const ExitHeadArgs& a, cudaStream_t st, int prof_class = PC_EXIT_HEAD);
 
+// K4 + K5 fused: exit head + decision + decoupled look-back compaction (+ survivor row copy when src != nullptr);
+// ws: exit_fused_ws_bytes(max_batch) of device scratch (zeroed by the launcher)
+size_t exit_fused_ws_bytes(int max_batch);
+void launch_exit_fused(const ExitHeadArgs& h, unsigned* ws, int* pos_next, int* orig_next, int* count_next,
+                       int32_t* counts_out, int32_t* surv_out, int32_t* last_count_out, int last_index,
+                       const bf16* src, bf16* dense_next, long long row_elems, cudaStream_t st);
+
 // stable compaction of alive rows: pos_next[j'] = j, orig_next[j'] = orig[j]; count_next; counts[k] += exited;
 // surv_out (optional, user): ascending original rows
 void launch_compact(const uint8_t* alive, const int* count, int n_static, const int* orig, int* pos_next,

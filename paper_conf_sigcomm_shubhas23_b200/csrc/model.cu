@@ -260,6 +260,7 @@ void Model::build(const adainf_model_spec& s) {
   orig.alloc((size_t)nstages * max_batch * 4);
   counts.alloc((size_t)nstages * 4 + 16);
   alive.alloc((size_t)max_batch);
+  exit_ws.alloc(exit_fused_ws_bytes(max_batch));
 
   // SGD segment tables (shadow layout per conv weight)
   std::vector<SgdSeg> segs;
@@ -482,6 +483,23 @@ void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, in
     a.embed = k == 0 ? out->embed : nullptr;
     a.alive = a.is_final ? nullptr : alive.as<uint8_t>();
     if (e.tensor == 0 && map0) throw InvalidError("exit directly on a mapped input is not supported");
+    static int fused_env = -1;
+    if (fused_env < 0) {
+      const char* ev = getenv("ADAINF_EXIT_FUSED");
+      fused_env = ev ? atoi(ev) : 1;
+    }
+    if (fused_env) {
+      // K4 + K5: head, decision, look-back compaction and the survivors' dense copy in one kernel
+      a.alive = nullptr;
+      const bool copy = !a.is_final && e.dense_next.p;
+      launch_exit_fused(a, exit_ws.as<unsigned>(), posb + (size_t)(s + 1) * max_batch,
+                        origb + (size_t)(s + 1) * max_batch, cnt + s + 1, out->exit_counts,
+                        (!a.is_final && out->surv_idx) ? out->surv_idx + (size_t)k * n_static : nullptr,
+                        (k == E - 2) ? out->exit_counts : nullptr, E - 1, copy ? T[e.tensor].buf : nullptr,
+                        copy ? e.dense_next.as<bf16>() : nullptr, (long long)X.row_elems(), st);
+      if (copy) dense_t[e.tensor] = e.dense_next.as<bf16>();
+      continue;
+    }
     launch_exit_head(a, st);
     if (!a.is_final) {
       // survivors of exit k -> stage s+1 (stable, ascending original rows)

@@ -108,6 +108,7 @@ struct Model {
   DevBuf stem_wprep;          // per-tap bf16 weights [16][2][64][8], rebuilt from the shadow every forward
   // inference stage bookkeeping
   DevBuf pos, orig, counts, alive;  // pos/orig: [nstages][max_batch] int; counts [nstages] int
+  DevBuf exit_ws;                   // fused exit kernel: ticket + look-back status words
   // training
   bool train_ready = false;
   DevBuf wgrad_ws, loss_rows, stats_tmp, sq_partial;

@@ -13,6 +13,7 @@
 #include "common.cuh"
 #include "model.h"
 #include "prof.h"
+#include "tma.cuh"
 
 namespace adainf {
 
@@ -23,28 +24,33 @@ __global__ void transpose_w_kernel(const bf16* __restrict__ W, int D, int P, bf1
   Wt[(long long)p * D + d] = W[i];
 }
 
-// mu[r][p] = sum_d ref[r][d] * W[d][p]  (fp32); mun[r] = ||mu_r||
-__global__ void project_ref_kernel(const float* __restrict__ ref, const bf16* __restrict__ W, int D, int P, int M,
-                                   float* __restrict__ mu, float* __restrict__ mun) {
-  const int r = blockIdx.x;
-  __shared__ float red[256];
-  float sq = 0.f;
-  for (int p = threadIdx.x; p < P; p += blockDim.x) {
-    float a = 0.f;
-    if (W)
-      for (int d = 0; d < D; ++d) a = fmaf(ref[(long long)r * D + d], __bfloat162float(W[(long long)d * P + p]), a);
-    else
-      a = ref[(long long)r * D + p];
-    mu[(long long)r * P + p] = a;
-    sq = fmaf(a, a, sq);
+// mu[r][p] = sum_d ref[r][d] * W[d][p]  (fp32): one warp per (r, p), lanes stride d (independent loads in flight),
+// fixed xor-tree combine
+__global__ void __launch_bounds__(256) project_ref_kernel(const float* __restrict__ ref, const bf16* __restrict__ W, int D,
+                                                          int P, int M, float* __restrict__ mu) {
+  const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (gw >= M * P) return;
+  const int r = gw / P, p = gw - r * P;
+  float a = 0.f;
+  if (W) {
+#pragma unroll 4
+    for (int d = lane; d < D; d += 32) a = fmaf(ref[(long long)r * D + d], __bfloat162float(W[(long long)d * P + p]), a);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
+  } else {
+    a = ref[(long long)r * D + p];
   }
-  red[threadIdx.x] = sq;
-  __syncthreads();
-  for (int o = blockDim.x / 2; o > 0; o >>= 1) {
-    if (threadIdx.x < o) red[threadIdx.x] += red[threadIdx.x + o];
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) mun[r] = sqrtf(red[0]);
+  if (lane == 0) mu[(long long)r * P + p] = a;
+}
+// mun[r] = ||mu_r||: one warp per reference row, lanes stride p, fixed xor-tree combine
+__global__ void ref_norm_kernel(const float* __restrict__ mu, int P, int M, float* __restrict__ mun) {
+  const int r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (r >= M) return;
+  float s = 0.f;
+  for (int p = lane; p < P; p += 32) s = fmaf(mu[(long long)r * P + p], mu[(long long)r * P + p], s);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if (lane == 0) mun[r] = sqrtf(s);
 }
 
 // one warp per row: cosine distance to every reference row, min; key
@@ -127,6 +133,216 @@ __global__ void __launch_bounds__(256) cosine_key_multi_kernel(const void* __res
   }
 }
 
+// ---- fused projection + cosine key (one pass over X, no fp32 Y round trip) ---------------------------------
+// Persistent, one CTA per SM: W^T [P][D] resident in shared memory (TMA, 128B swizzle, 64-column chunks), X streamed
+// in 128-row x 64-column TMA boxes through a stage ring, Y tile = X W on the tensor cores (tcgen05.mma M=128,
+// N=P, K=16; fp32 accumulators in TMEM, double-buffered), epilogue: one thread per row reads its P values from TMEM
+// and computes ||y||, y.mu_r, d = max(0, min_r 1 - cos) and the key, in the row's own fixed order.
+constexpr int SELF_THREADS = 192;  // warp 0 TMA, warp 1 MMA, warps 2-5 epilogue (TMEM lane quadrants 2,3,0,1)
+constexpr int SELF_STAGES = 6;
+constexpr int SELF_STAGE_BYTES = 128 * 128;  // 128 rows x 64 bf16 columns
+
+struct SelFusedArgs {
+  CUtensorMap x_map;  // X [N][D] bf16, box {64, 128}
+  CUtensorMap w_map;  // W^T [P][D] bf16, box {64, P}
+  long long N;
+  int D, M;
+  const float* mu;   // [M][P]
+  const float* mun;  // [M]
+  const uint8_t* exclude;
+  uint32_t* keys;
+  float* dist_all;
+};
+
+template <int NC>
+__device__ __forceinline__ void tmem_ld_cols(uint32_t taddr, float* v) {
+  if constexpr (NC == 16) {
+    uint32_t r[16];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+        : "r"(taddr));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+    for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+  } else {
+    tmem_ld32(taddr, v);
+  }
+}
+
+template <int P>
+__global__ void __launch_bounds__(SELF_THREADS, 1) select_fused_kernel(const __grid_constant__ SelFusedArgs a) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  const int nkb = a.D / 64;
+  uint8_t* wsm = smem;                                  // nkb chunks of [P][64] bf16 (P * 128 bytes each)
+  uint8_t* xst = wsm + (size_t)nkb * P * 128;           // stage ring
+  float* mus = (float*)(xst + SELF_STAGES * SELF_STAGE_BYTES);  // [M][P] then mun[M]
+  uint64_t* full = (uint64_t*)(mus + 4 * P + 4);
+  uint64_t* empty = full + SELF_STAGES;
+  uint64_t* wbar = empty + SELF_STAGES;
+  uint64_t* tfull = wbar + 1;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+  constexpr int ACC = P;
+  constexpr int TCOLS = 2 * P < 32 ? 32 : 2 * P;
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const long long ntiles = (a.N + 127) / 128;
+  for (int i = threadIdx.x; i < a.M * P; i += blockDim.x) mus[i] = a.mu[i];
+  if (threadIdx.x < a.M) mus[4 * P + threadIdx.x] = a.mun[threadIdx.x];
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < SELF_STAGES; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    mbar_init(wbar, 1);
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 128);
+    }
+    fence_mbar_init();
+    tma_prefetch_desc(&a.x_map);
+    tma_prefetch_desc(&a.w_map);
+  }
+  if (warp == 1) tmem_alloc<TCOLS>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      mbar_expect_tx(wbar, (uint32_t)(nkb * P * 128));
+      for (int kb = 0; kb < nkb; ++kb) tma_load_2d(smem_u32(wsm + (size_t)kb * P * 128), &a.w_map, wbar, kb * 64, 0);
+      int it = 0;
+      for (long long t = blockIdx.x; t < ntiles; t += gridDim.x)
+        for (int kb = 0; kb < nkb; ++kb, ++it) {
+          const int s = it % SELF_STAGES, ph = it / SELF_STAGES;
+          if (ph > 0) mbar_wait(&empty[s], (ph - 1) & 1);
+          mbar_expect_tx(&full[s], SELF_STAGE_BYTES);
+          tma_load_2d(smem_u32(xst + s * SELF_STAGE_BYTES), &a.x_map, &full[s], kb * 64, (int)(t * 128));
+        }
+    }
+  } else if (warp == 1) {
+    constexpr uint32_t IDESC = make_idesc(128, P, 0, 0);
+    mbar_wait(wbar, 0);
+    int it = 0, lt = 0;
+    for (long long t = blockIdx.x; t < ntiles; t += gridDim.x, ++lt) {
+      const int b = lt & 1, ub = lt >> 1;
+      if (ub > 0) mbar_wait(&tempty[b], (ub - 1) & 1);
+      tc_fence_after();
+      for (int kb = 0; kb < nkb; ++kb, ++it) {
+        const int s = it % SELF_STAGES, u = it / SELF_STAGES;
+        mbar_wait(&full[s], u & 1);
+        tc_fence_after();
+        if (elect_one()) {
+          const uint64_t ad0 = make_sdesc(smem_u32(xst + s * SELF_STAGE_BYTES), 16, 1024);
+          const uint64_t bd0 = make_sdesc(smem_u32(wsm + (size_t)kb * P * 128), 16, 1024);
+#pragma unroll
+          for (int kk = 0; kk < 4; ++kk)
+            umma_bf16(tmem + (uint32_t)(b * ACC), ad0 + kk * 2, bd0 + kk * 2, IDESC, (kb | kk) != 0);
+          umma_commit(&empty[s]);
+          if (kb == nkb - 1) umma_commit(&tfull[b]);
+        }
+        __syncwarp();
+      }
+    }
+  } else {
+    const int q = warp & 3;
+    const float* mun = mus + 4 * P;
+    int lt = 0;
+    for (long long t = blockIdx.x; t < ntiles; t += gridDim.x, ++lt) {
+      const int b = lt & 1, ub = lt >> 1;
+      mbar_wait(&tfull[b], ub & 1);
+      tc_fence_after();
+      const uint32_t trow = tmem + (uint32_t)(b * ACC) + ((uint32_t)(q * 32) << 16);
+      float nn = 0.f, dot[4] = {0.f, 0.f, 0.f, 0.f};
+      constexpr int CH = P < 32 ? P : 32;
+#pragma unroll 1
+      for (int c0 = 0; c0 < P; c0 += CH) {
+        float v[CH];
+        tmem_ld_cols<CH>(trow + (uint32_t)c0, v);
+#pragma unroll
+        for (int i = 0; i < CH; ++i) {
+          nn = fmaf(v[i], v[i], nn);
+#pragma unroll
+          for (int r = 0; r < 4; ++r)
+            if (r < a.M) dot[r] = fmaf(v[i], mus[r * P + c0 + i], dot[r]);
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(&tempty[b]);
+      const long long row = t * 128 + q * 32 + lane;
+      if (row < a.N) {
+        const float yn = sqrtf(nn);
+        float best = FLT_MAX;
+#pragma unroll
+        for (int r = 0; r < 4; ++r)
+          if (r < a.M) best = fminf(best, 1.0f - dot[r] / fmaxf(yn * mun[r], 1e-12f));
+        const bool ex = a.exclude && a.exclude[row];
+        const float d = fmaxf(best, 0.f);
+        a.keys[row] = ex ? 0u : (__float_as_uint(d) + 1u);
+        if (a.dist_all) a.dist_all[row] = ex ? -1.f : d;
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<TCOLS>(tmem);
+  }
+}
+
+static bool select_fused_ok(int D, int P, int M) {
+  return D % 64 == 0 && (P == 16 || P == 32 || P == 64 || P == 128 || P == 256) && M <= 4 && (long long)D * P * 2 <= 98304;
+}
+
+static size_t select_fused_smem(int D, int P) {
+  return 1024 + (size_t)D * P * 2 + SELF_STAGES * SELF_STAGE_BYTES + (4 * P + 4) * 4 + 256;
+}
+
+template <int P>
+static void launch_select_fused_p(const SelFusedArgs& a, int D, cudaStream_t st) {
+  const size_t sm = select_fused_smem(D, P);
+  static bool attr = false;
+  if (!attr) {
+    CK(cudaFuncSetAttribute(select_fused_kernel<P>, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448));
+    attr = true;
+  }
+  const long long ntiles = (a.N + 127) / 128;
+  const int grid = (int)std::min<long long>(ntiles, num_sms());
+  select_fused_kernel<P><<<grid, SELF_THREADS, sm, st>>>(a);
+  CK(cudaGetLastError());
+}
+
+static void launch_select_fused(const bf16* X, const bf16* Wt, long long N, int D, int P, int M, const float* mu,
+                                const float* mun, const uint8_t* exclude, uint32_t* keys, float* dist_all,
+                                cudaStream_t st) {
+  thread_local SelFusedArgs a;
+  a = SelFusedArgs{};
+  a.x_map = make_tmap_2d(X, N, D, D, 64, 128);
+  a.w_map = make_tmap_2d(Wt, P, D, D, 64, P);
+  a.N = N;
+  a.D = D;
+  a.M = M;
+  a.mu = mu;
+  a.mun = mun;
+  a.exclude = exclude;
+  a.keys = keys;
+  a.dist_all = dist_all;
+  ProfScope ps(PC_SELECT_PROJ, st);
+  switch (P) {
+    case 16: launch_select_fused_p<16>(a, D, st); break;
+    case 32: launch_select_fused_p<32>(a, D, st); break;
+    case 64: launch_select_fused_p<64>(a, D, st); break;
+    case 128: launch_select_fused_p<128>(a, D, st); break;
+    default: launch_select_fused_p<256>(a, D, st); break;
+  }
+}
+
 // ---- radix select state: [0] prefix, [1] k remaining, [2] pass, hist[256] ----
 struct RadixState {
   uint32_t prefix;
@@ -166,25 +382,41 @@ __global__ void radix_hist_kernel(const uint32_t* __restrict__ keys, long long N
   if (count_eligible && threadIdx.x == 0) atomicAdd(&s->n_eligible, elig);
 }
 
-__global__ void radix_pick_kernel(RadixState* s, int shift, int last) {
-  // single warp: find the digit d (from 255 down) where the cumulative count reaches krem
-  if (threadIdx.x != 0) return;
-  uint32_t krem = s->krem;
-  uint32_t cum = 0;
-  int d = 255;
-  for (; d >= 0; --d) {
-    const uint32_t c = s->hist[d];
-    if (cum + c >= krem) break;
-    cum += c;
+// 256 threads: suffix counts of the histogram (digit 255 down), the digit d where the running count reaches krem
+__global__ void __launch_bounds__(256) radix_pick_kernel(RadixState* s, int shift, int last) {
+  __shared__ uint32_t suf[256];  // suf[d] = count of digits > d
+  __shared__ int s_d;
+  const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+  const int d = 255 - t;  // thread t handles digit 255 - t (descending)
+  const uint32_t c = s->hist[d];
+  uint32_t x = c;  // inclusive scan over t (i.e. over descending digits)
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
   }
-  if (d < 0) d = 0;  // fewer keys than k with this prefix (only when k > #keys): take everything
-  s->prefix |= ((uint32_t)d << shift);
-  s->krem = krem - cum;
-  for (int q = 0; q < 256; ++q) s->hist[q] = 0;
-  if (last) {
-    s->T = s->prefix;
-    s->need_eq = s->krem;
+  __shared__ uint32_t wsum[8];
+  if (lane == 31) wsum[w] = x;
+  __syncthreads();
+  uint32_t off = 0;
+  for (int q = 0; q < w; ++q) off += wsum[q];
+  const uint32_t incl = off + x, excl = incl - c;
+  suf[d] = excl;
+  if (t == 0) s_d = 0;  // fewer keys than k with this prefix (only when k > #keys): take everything
+  __syncthreads();
+  const uint32_t krem = s->krem;
+  if (excl < krem && incl >= krem) s_d = d;  // exactly one digit satisfies this (counts are non-negative)
+  __syncthreads();
+  if (t == 0) {
+    const int dd = s_d;
+    s->prefix |= ((uint32_t)dd << shift);
+    s->krem = krem - suf[dd];
+    if (last) {
+      s->T = s->prefix;
+      s->need_eq = s->krem;
+    }
   }
+  s->hist[t] = 0;
 }
 
 constexpr int EMIT_THREADS = 1024;
@@ -277,11 +509,109 @@ __global__ void emit_write_kernel(const uint32_t* __restrict__ keys, long long N
   }
 }
 
+// Single-CTA exact top-k for pools up to ~1M keys: the four 8-bit MSB radix passes (warp-aggregated shared-memory
+// histograms: the distance keys share few top bytes) and the ascending stable emit (block ballot scan per 1,024-key
+// chunk, ties -> lower position) in one launch, instead of 12 launches of the multi-CTA path.
+constexpr int TOPK1_THREADS = 1024;
+__global__ void __launch_bounds__(TOPK1_THREADS) topk_single_kernel(const uint32_t* __restrict__ keys, int N, int k,
+                                                                    int32_t* __restrict__ out_idx,
+                                                                    float* __restrict__ out_dist,
+                                                                    int32_t* __restrict__ out_count) {
+  __shared__ uint32_t hist[256];
+  __shared__ uint32_t s_prefix, s_krem;
+  __shared__ int warp_g[32], warp_e[32];
+  __shared__ int s_run_take, s_run_eq;
+  const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+  const int k_eff = min(k, N);
+  if (t == 0) {
+    s_prefix = 0;
+    s_krem = (uint32_t)k_eff;
+  }
+  for (int pass = 0; pass < 4; ++pass) {
+    const int shift = 24 - 8 * pass;
+    const uint32_t mask_hi = pass == 0 ? 0u : (0xFFFFFFFFu << (32 - 8 * pass));
+    if (t < 256) hist[t] = 0;
+    __syncthreads();
+    const uint32_t prefix = s_prefix;
+    for (int i0 = 0; i0 < N; i0 += TOPK1_THREADS) {
+      const int i = i0 + t;
+      const uint32_t key = i < N ? keys[i] : 0u;
+      const bool in = i < N && (key & mask_hi) == prefix;
+      const uint32_t dig = (key >> shift) & 255u;
+      const unsigned act = __ballot_sync(0xffffffffu, in);
+      if (in) {
+        const unsigned peers = __match_any_sync(act, dig);
+        if ((int)(__ffs(peers) - 1) == lane) atomicAdd(&hist[dig], (uint32_t)__popc(peers));
+      }
+    }
+    __syncthreads();
+    if (t == 0) {
+      uint32_t krem = s_krem, cum = 0;
+      int d = 255;
+      for (; d >= 0; --d) {
+        const uint32_t c = hist[d];
+        if (cum + c >= krem) break;
+        cum += c;
+      }
+      if (d < 0) d = 0;
+      s_prefix = prefix | ((uint32_t)d << shift);
+      s_krem = krem - cum;
+    }
+    __syncthreads();
+  }
+  const uint32_t T = s_prefix;
+  const int need = (int)s_krem;
+  if (t == 0) {
+    s_run_take = 0;
+    s_run_eq = 0;
+  }
+  __syncthreads();
+  for (int i0 = 0; i0 < N; i0 += TOPK1_THREADS) {
+    const int i = i0 + t;
+    const uint32_t key = i < N ? keys[i] : 0u;
+    const bool g = (T == 0) ? key > 0 : key > T;
+    const bool e = (T != 0) && key == T;
+    const unsigned be = __ballot_sync(0xffffffffu, e);
+    if (lane == 0) warp_e[w] = __popc(be);
+    __syncthreads();
+    int eqrank = s_run_eq + __popc(be & ((1u << lane) - 1u));
+    for (int q = 0; q < w; ++q) eqrank += warp_e[q];
+    const bool take = g || (e && eqrank < need);
+    const unsigned bt = __ballot_sync(0xffffffffu, take);
+    if (lane == 0) warp_g[w] = __popc(bt);
+    __syncthreads();
+    int o = s_run_take + __popc(bt & ((1u << lane) - 1u));
+    for (int q = 0; q < w; ++q) o += warp_g[q];
+    if (take && o < k) {
+      out_idx[o] = i;
+      if (out_dist) out_dist[o] = __uint_as_float(key - 1u);
+    }
+    __syncthreads();
+    if (t == 0) {
+      int tt = 0, te = 0;
+      for (int q = 0; q < 32; ++q) {
+        tt += warp_g[q];
+        te += warp_e[q];
+      }
+      s_run_take += tt;
+      s_run_eq += te;
+    }
+    __syncthreads();
+  }
+  if (t == 0) *out_count = min(s_run_take, k);
+}
+
 // exact top-k of 32-bit keys (0 = not eligible), ties -> lower position, emitted in ascending position order
 static void topk_emit(const uint32_t* keys, long long N, int k, RadixState* rs, int* blk, int* offs, int32_t* out_idx,
                       float* out_dist, int32_t* out_count, cudaStream_t st) {
   const long long nb = (N + EMIT_THREADS - 1) / EMIT_THREADS;
   const int k_eff = (int)std::min<long long>(k, N);  // the k-th largest must exist
+  if (N <= 24576 && !getenv("ADAINF_TOPK_MULTI")) {  // single CTA wins below ~24k keys (measured)
+    ProfScope ps_topk(PC_SELECT_TOPK, st, 1);
+    topk_single_kernel<<<1, TOPK1_THREADS, 0, st>>>(keys, (int)N, k, out_idx, out_dist, out_count);
+    CK(cudaGetLastError());
+    return;
+  }
   ProfScope ps_topk(PC_SELECT_TOPK, st, 12);
   radix_init_kernel<<<1, 256, 0, st>>>(rs, k_eff);
   const int hb = (int)std::min<long long>((N + 1023) / 1024, 4LL * num_sms());
@@ -289,7 +619,7 @@ static void topk_emit(const uint32_t* keys, long long N, int k, RadixState* rs, 
     const int shift = 24 - 8 * pass;
     const uint32_t mask_hi = pass == 0 ? 0u : (0xFFFFFFFFu << (32 - 8 * pass));
     radix_hist_kernel<<<hb, 256, 0, st>>>(keys, N, rs, shift, mask_hi, pass == 0);
-    radix_pick_kernel<<<1, 32, 0, st>>>(rs, shift, pass == 3);
+    radix_pick_kernel<<<1, 256, 0, st>>>(rs, shift, pass == 3);
   }
   emit_count_kernel<<<(unsigned)nb, EMIT_THREADS, 0, st>>>(keys, N, rs, blk);
   emit_scan_kernel<<<1, 32, 0, st>>>((int)nb, rs, blk, offs, out_count, k);
@@ -323,7 +653,13 @@ void select_retrain(const adainf_select_in& in, int k, int32_t* out_idx, float* 
     w += (b + 255) / 256 * 256;
     return p;
   };
-  float* Y = in.W_bf16 ? (float*)take((size_t)N * P * 4) : nullptr;
+  static int fused_env = -1;
+  if (fused_env < 0) {
+    const char* e = getenv("ADAINF_SELECT_FUSED");
+    fused_env = e ? atoi(e) : 1;
+  }
+  const bool fused = in.W_bf16 && fused_env && select_fused_ok(D, P, M);
+  float* Y = (in.W_bf16 && !fused) ? (float*)take((size_t)N * P * 4) : nullptr;
   bf16* Wt = in.W_bf16 ? (bf16*)take((size_t)P * D * 2) : nullptr;
   float* mu = (float*)take((size_t)M * P * 4);
   float* mun = (float*)take((size_t)M * 4);
@@ -334,8 +670,13 @@ void select_retrain(const adainf_select_in& in, int k, int32_t* out_idx, float* 
   int* blk = (int*)take((size_t)nb * 8);
   int* offs = (int*)take((size_t)nb * 8);
   { ProfScope ps(PC_SELECT_PROJ, st);
-  project_ref_kernel<<<M, 256, 0, st>>>(in.ref, (const bf16*)in.W_bf16, D, P, M, mu, mun); }
-  if (in.W_bf16) {
+  project_ref_kernel<<<(M * P * 32 + 255) / 256, 256, 0, st>>>(in.ref, (const bf16*)in.W_bf16, D, P, M, mu);
+  ref_norm_kernel<<<(M * 32 + 255) / 256, 256, 0, st>>>(mu, P, M, mun); }
+  if (fused) {
+    { ProfScope ps(PC_SELECT_PROJ, st);
+    transpose_w_kernel<<<(D * P + 255) / 256, 256, 0, st>>>((const bf16*)in.W_bf16, D, P, Wt); }
+    launch_select_fused((const bf16*)in.X_bf16, Wt, N, D, P, M, mu, mun, in.exclude, keys, dist_all, st);
+  } else if (in.W_bf16) {
     { ProfScope ps(PC_SELECT_PROJ, st);
     transpose_w_kernel<<<(D * P + 255) / 256, 256, 0, st>>>((const bf16*)in.W_bf16, D, P, Wt); }
     CK(cudaMemsetAsync(zb, 0, (size_t)P * 4, st));
@@ -415,8 +756,6 @@ void select_merge(const float* dist, const int32_t* idx, const int32_t* block_co
     merge_scatter_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(dist, idx, block_count, n_blocks, block_len,
                                                                      idx_mul, block_off, n_total, keys);
   }
-  RadixState* unused = nullptr;
-  (void)unused;
   topk_emit(keys, n_total, k, rs, blk, offs, out_idx, out_dist, out_count, st);
   CK(cudaFreeAsync(wsp, st));
 }
