@@ -81,6 +81,10 @@ def lib():
         L.or_detect.restype = C.c_int32
         L.or_detect.argtypes = [f32p, C.c_int, C.c_int, C.c_int, C.c_int, f32p, C.c_int, C.c_int, C.c_int,
                                 C.c_float, f32p, C.c_int32]
+        L.or_nms.restype = C.c_int32
+        L.or_nms.argtypes = [f32p, C.c_int32, C.c_float, u8p]
+        L.or_iou.restype = C.c_float
+        L.or_iou.argtypes = [f32p, f32p]
         L.or_crop.argtypes = [f32p, C.c_int, C.c_int, C.c_int, C.c_float, C.c_float, C.c_float, C.c_float,
                               C.c_int, C.c_int, f32p]
         L.or_select.restype = C.c_int32
@@ -268,6 +272,19 @@ def detect(raw, anchors, nc, anchor_wh, stride, img_w, img_h, tau_det, max_det=1
     n = lib().or_detect(_p(raw, C.c_float), B, G, anchors, nc, _p(aw, C.c_float), stride, img_w, img_h,
                         tau_det, _p(det, C.c_float), max_det)
     return det[:min(n, max_det)].copy(), int(n)
+
+
+def nms(det, iou_thr):
+    """Greedy per-(frame, class) NMS over or_detect rows; returns keep[n] (uint8) and the kept count."""
+    det = _f32(det).reshape(-1, 9)
+    keep = np.zeros(det.shape[0], np.uint8)
+    k = lib().or_nms(_p(det, C.c_float), det.shape[0], float(iou_thr), _p(keep, C.c_uint8))
+    return keep, int(k)
+
+
+def iou(a, b):
+    a, b = _f32(a), _f32(b)
+    return float(lib().or_iou(_p(a, C.c_float), _p(b, C.c_float)))
 
 
 def crop(frame, box, crop_h, crop_w):

@@ -632,6 +632,52 @@ extern "C" int32_t or_detect(const float* raw, int B, int G, int A, int NC, cons
   return n;
 }
 
+// Non-maximum suppression (NEXT-3 of SURVEY §8(f): TinyYOLOv3 post-processing; the paper gives no
+// parameters: reading Q18b in DESIGN.md).  Plain greedy definition, per (frame, class).
+extern "C" float or_iou(const float* a, const float* b) {
+  const float iw = std::max(0.0f, std::min(a[2], b[2]) - std::max(a[0], b[0]));
+  const float ih = std::max(0.0f, std::min(a[3], b[3]) - std::max(a[1], b[1]));
+  const float inter = iw * ih;
+  const float area_a = (a[2] - a[0]) * (a[3] - a[1]);
+  const float area_b = (b[2] - b[0]) * (b[3] - b[1]);
+  const float uni = (area_a + area_b) - inter;
+  return uni > 0.0f ? inter / uni : 0.0f;
+}
+
+extern "C" int32_t or_nms(const float* det, int32_t n, float iou_thr, uint8_t* keep) {
+  vector<int> order(n);
+  for (int i = 0; i < n; ++i) order[i] = i;
+  // visit order: frame, class, score descending, row ascending
+  std::stable_sort(order.begin(), order.end(), [&](int x, int y) {
+    const float* a = det + (int64_t)x * 9;
+    const float* b = det + (int64_t)y * 9;
+    if (a[0] != b[0]) return a[0] < b[0];
+    if (a[3] != b[3]) return a[3] < b[3];
+    return a[4] > b[4];
+  });
+  int32_t kept = 0;
+  vector<int> kept_rows;
+  for (int i = 0; i < n; ++i) keep[i] = 0;
+  for (int q = 0; q < n; ++q) {
+    const int i = order[q];
+    const float* a = det + (int64_t)i * 9;
+    bool ok = true;
+    for (int k : kept_rows) {
+      const float* b = det + (int64_t)k * 9;
+      if (b[0] == a[0] && b[3] == a[3] && or_iou(a + 5, b + 5) > iou_thr) {
+        ok = false;
+        break;
+      }
+    }
+    if (ok) {
+      keep[i] = 1;
+      kept_rows.push_back(i);
+      kept++;
+    }
+  }
+  return kept;
+}
+
 // Crop-resize (reading Q19): half-pixel centres, clamped edges, every fp32 op rounded separately (no
 // FMA contraction: compiled with -ffp-contract=off), result rounded to bf16.
 extern "C" void or_crop(const float* fr, int H, int W, int C, float x0, float y0, float x1, float y1, int ch,

@@ -82,6 +82,16 @@ void or_exit_assign(const float* conf, int B, int E, const float* tau, int8_t* e
  * in ascending linear index; returns the true number of detections. */
 int32_t or_detect(const float* det_raw, int B, int G, int A, int NC, const float* anchor_wh, int stride,
                   int img_w, int img_h, float tau_det, float* det_table, int32_t max_det);
+/* Greedy non-maximum suppression (NEXT-3; reading Q18b): det rows as written by or_detect (ascending
+ * candidate index).  Within each (frame, class), detections are visited by score descending (ties -> lower row);
+ * a detection is kept unless its IoU with an already kept one exceeds iou_thr.  IoU in fp32, every op rounded:
+ *   iw = max(0, min(x1a, x1b) - max(x0a, x0b)), ih likewise, inter = iw * ih,
+ *   union = (x1a - x0a) * (y1a - y0a) + (x1b - x0b) * (y1b - y0b) - inter   (area_a + area_b, then - inter),
+ *   iou = union > 0 ? inter / union : 0.
+ * keep[n] out (0/1); returns the number kept. */
+int32_t or_nms(const float* det, int32_t n, float iou_thr, uint8_t* keep);
+float or_iou(const float* a, const float* b); /* boxes x0, y0, x1, y1 */
+
 /* Bilinear crop-resize of one box from a bf16 (as float) NHWC frame -> crop_h*crop_w*C, bf16-rounded
  * (SURVEY c.1 step 7 / Q19). */
 void or_crop(const float* frame, int H, int W, int C, float x0, float y0, float x1, float y1, int crop_h,

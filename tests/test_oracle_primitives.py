@@ -219,3 +219,85 @@ def test_select_closed_forms_and_bruteforce():
     np.testing.assert_allclose(dist, d, rtol=1e-5, atol=1e-6)
     order = sorted(range(N), key=lambda i: (-np.float32(d[i]), i))[:37]
     assert list(idx) == sorted(order)
+
+
+def test_iou_closed_forms():
+    """NEXT-3 NMS (reading Q18b): IoU = inter / (area_a + area_b - inter) in fp32."""
+    assert abs(O.iou([0, 0, 2, 2], [1, 1, 3, 3]) - 1.0 / 7.0) < 1e-7
+    assert O.iou([1, 2, 5, 7], [1, 2, 5, 7]) == 1.0
+    assert O.iou([0, 0, 1, 1], [2, 2, 3, 3]) == 0.0
+    assert O.iou([0, 0, 1, 1], [1, 0, 2, 1]) == 0.0  # touching edges: zero intersection
+    assert abs(O.iou([0, 0, 4, 4], [1, 1, 3, 3]) - 0.25) < 1e-7  # contained
+    assert O.iou([0, 0, 0, 0], [0, 0, 0, 0]) == 0.0  # zero-area union
+
+
+def _det_rows(rows):
+    return np.array([[f, i, 0, c, s, x0, y0, x1, y1] for i, (f, c, s, x0, y0, x1, y1) in enumerate(rows)],
+                    np.float32)
+
+
+def test_nms_closed_forms_and_greedy_chain():
+    thr = 0.45
+    # identical boxes, same frame and class: the higher score survives; equal scores -> the lower row survives
+    k, n = O.nms(_det_rows([(0, 0, 0.9, 0, 0, 10, 10), (0, 0, 0.8, 0, 0, 10, 10)]), thr)
+    assert k.tolist() == [1, 0] and n == 1
+    k, _ = O.nms(_det_rows([(0, 0, 0.8, 0, 0, 10, 10), (0, 0, 0.9, 0, 0, 10, 10)]), thr)
+    assert k.tolist() == [0, 1]
+    k, _ = O.nms(_det_rows([(0, 0, 0.7, 0, 0, 10, 10), (0, 0, 0.7, 0, 0, 10, 10)]), thr)
+    assert k.tolist() == [1, 0]
+    # other class or other frame never suppresses
+    assert O.nms(_det_rows([(0, 0, 0.9, 0, 0, 10, 10), (0, 1, 0.8, 0, 0, 10, 10)]), thr)[0].tolist() == [1, 1]
+    assert O.nms(_det_rows([(0, 0, 0.9, 0, 0, 10, 10), (1, 0, 0.8, 0, 0, 10, 10)]), thr)[0].tolist() == [1, 1]
+    # IoU exactly at the threshold is kept (suppression is strict >): [0,0,2,2] vs [1,1,3,3] -> 1/7
+    t7 = np.float32(1.0) / np.float32(7.0)
+    assert O.nms(_det_rows([(0, 0, 0.9, 0, 0, 2, 2), (0, 0, 0.8, 1, 1, 3, 3)]), float(t7))[0].tolist() == [1, 1]
+    assert O.nms(_det_rows([(0, 0, 0.9, 0, 0, 2, 2), (0, 0, 0.8, 1, 1, 3, 3)]), float(t7) * 0.99)[0].tolist() == [1, 0]
+    # greedy chain: A suppresses B, B (not kept) cannot suppress C although IoU(B, C) > thr
+    rows = [(0, 0, 0.9, 0, 0, 10, 10), (0, 0, 0.8, 3, 0, 13, 10), (0, 0, 0.7, 6, 0, 16, 10)]
+    d = _det_rows(rows)
+    assert O.iou(d[0, 5:], d[1, 5:]) > thr and O.iou(d[1, 5:], d[2, 5:]) > thr and O.iou(d[0, 5:], d[2, 5:]) < thr
+    assert O.nms(d, thr)[0].tolist() == [1, 0, 1]
+
+
+def _iou_np(a, b):
+    f = np.float32
+    iw = max(f(0), min(a[2], b[2]) - max(a[0], b[0]))
+    ih = max(f(0), min(a[3], b[3]) - max(a[1], b[1]))
+    inter = f(iw * ih)
+    uni = f(f(f((a[2] - a[0]) * (a[3] - a[1])) + f((b[2] - b[0]) * (b[3] - b[1]))) - inter)
+    return f(inter / uni) if uni > 0 else f(0)
+
+
+def test_nms_textbook_loop_and_invariants():
+    """Against the textbook loop (repeatedly take the best remaining box of a (frame, class) group, drop every
+    box overlapping it by more than the threshold) and the two invariants of greedy NMS: kept boxes of a group
+    overlap pairwise by <= thr, and every dropped box overlaps a kept box that precedes it in score order."""
+    rng = np.random.default_rng(3)
+    thr = 0.45
+    for trial in range(20):
+        n = int(rng.integers(1, 60))
+        x0 = rng.uniform(0, 80, n)
+        y0 = rng.uniform(0, 80, n)
+        w = rng.uniform(2, 30, n)
+        h = rng.uniform(2, 30, n)
+        sc = np.round(rng.uniform(0.1, 1.0, n), 2)  # rounded: ties occur
+        rows = [(int(rng.integers(0, 2)), int(rng.integers(0, 3)), sc[i], x0[i], y0[i], x0[i] + w[i], y0[i] + h[i])
+                for i in range(n)]
+        d = _det_rows(rows)
+        keep, _ = O.nms(d, thr)
+        ref = np.zeros(n, np.uint8)
+        for f_ in (0, 1):
+            for c_ in range(3):
+                rem = [i for i in range(n) if d[i, 0] == f_ and d[i, 3] == c_]
+                while rem:
+                    best = min(rem, key=lambda i: (-d[i, 4], i))
+                    ref[best] = 1
+                    rem = [i for i in rem if i != best and not _iou_np(d[best, 5:], d[i, 5:]) > np.float32(thr)]
+        assert keep.tolist() == ref.tolist(), trial
+        for i in range(n):
+            same = [j for j in range(n) if j != i and d[j, 0] == d[i, 0] and d[j, 3] == d[i, 3]]
+            if keep[i]:
+                assert all(not (keep[j] and _iou_np(d[i, 5:], d[j, 5:]) > np.float32(thr)) for j in same)
+            else:
+                assert any(keep[j] and (d[j, 4], -j) > (d[i, 4], -i) and _iou_np(d[i, 5:], d[j, 5:]) > np.float32(thr)
+                           for j in same)
