@@ -61,7 +61,8 @@ CONFIGS = {
                inf_b=256, fractions=[0.02, 0.02, 0.01], pool_n=131072, d=512, p=64, k=8192, heavy=True, seed=5,
                tau_sweep=[0.0, 0.5, 0.7, 0.9, 0.99, 2.0]),
     "c3": dict(name="BASELINE config 3: video-surveillance DAG, 512 frames 416x416 -> TinyYOLOv3-like detector "
-                    "(13x13x3 anchors, ~4 detections/frame, vehicle:person ~3:1) -> on-device crop routing (224x224) "
+                    "(13x13x3 anchors, greedy NMS at IoU 0.45, ~4 detections/frame, vehicle:person ~3:1) -> on-device crop "
+                    "routing (224x224) "
                     "-> vehicle-type (10 cls) + person-activity (8 cls) ResNet-18-EE (exits 25/25/25/25)",
                frames=512, hw=416, det_per_frame=4.0, cap=2048, fractions=[0.25, 0.25, 0.25], seed=3),
 }
@@ -430,7 +431,7 @@ class DagWorkload:
         self.world = world
         F, hw, cap = cfg["frames"], cfg["hw"], cfg["cap"]
         self.F, self.hw, self.cap = F, hw, cap
-        self.det_spec = S.tiny_yolo_det(in_hw=hw)
+        self.det_spec = S.tiny_yolo_det(in_hw=hw, nms_iou=0.45)  # TinyYOLOv3's NMS threshold (NEXT-3, Q18b)
         self.veh, self.per = S.resnet18_ee(10), S.resnet18_ee(8)
         seed = 100 * cfg["seed"] + rank
         pd = synth.det_head_params(self.det_spec, synth.init_params(self.det_spec, seed=31), obj_bias=-2.0,

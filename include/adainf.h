@@ -70,7 +70,10 @@ typedef void* adainf_stream_t; /* cudaStream_t (NULL = legacy default stream) */
  *            final classifier and is unconditional.  All EXITs of a model share num_classes.
  *            loss_weight w_k weights its cross-entropy in retraining (reading Q8).
  *   DET_HEAD TinyYOLOv3-style single-scale decode of the current fp32 tensor (reading Q18):
- *            `anchors` anchors x (5 + det_classes) channels, grid stride `grid_stride`, anchor_wh.
+ *            `anchors` anchors x (5 + det_classes) channels, grid stride `grid_stride`, anchor_wh; with
+ *            nms_iou > 0 the detections then go through greedy NMS per (frame, class): visited by score
+ *            descending (ties -> lower candidate index), dropped if their fp32 IoU with a kept detection exceeds
+ *            nms_iou; det_table / n_det / routing then list the kept detections (ascending candidate index).
  * Parameter layout (flat fp32, op order): CONV W[cout][kh][kw][cin] then b[cout]; BLOCK with cout>0:
  * W[cout][1][1][cin] then b[cout]; EXIT: Wk[cin][num_classes] then bk[num_classes].            */
 typedef enum {
@@ -90,6 +93,8 @@ typedef struct {
   float loss_weight;
   int32_t anchors, det_classes, grid_stride;
   float anchor_wh[16];
+  float nms_iou;      /* DET_HEAD: > 0 -> greedy per-(frame, class) NMS at this IoU threshold before routing
+                         (NEXT-3, reading Q18b); 0 -> none */
 } adainf_op;
 
 typedef struct {

@@ -35,6 +35,7 @@ class OrOp(C.Structure):
         ("pad", C.c_int32), ("cout", C.c_int32), ("act", C.c_int32), ("residual", C.c_int32),
         ("num_classes", C.c_int32), ("loss_weight", C.c_float), ("anchors", C.c_int32),
         ("det_classes", C.c_int32), ("grid_stride", C.c_int32), ("anchor_wh", C.c_float * 16),
+        ("groups", C.c_int32),
     ]
 
 
@@ -132,6 +133,7 @@ class Model:
             r.grid_stride = o.get("grid_stride", 0)
             for j, v in enumerate(o.get("anchor_wh", [])):
                 r.anchor_wh[j] = v
+            r.groups = int(o.get("groups", 1))
         self.m = OrModel(spec["in_h"], spec["in_w"], spec["in_c"], len(ops), self._ops)
         self.spec = spec
         L = lib()

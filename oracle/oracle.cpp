@@ -164,7 +164,9 @@ Walk walk(const or_model* m) {
       case OR_CONV: {
         Shape3 o{(cur.H + 2 * op.pad - op.kh) / op.stride + 1, (cur.W + 2 * op.pad - op.kw) / op.stride + 1,
                  op.cout};
-        w.nparams += (int64_t)op.cout * op.kh * op.kw * cur.C + op.cout;
+        const int g = op.groups > 0 ? op.groups : 1;
+        if (cur.C % g || op.cout % g) w.ok = false;
+        w.nparams += (int64_t)op.cout * op.kh * op.kw * (cur.C / g) + op.cout;
         if (op.residual) {
           if (blocks.empty()) w.ok = false;
           else {
@@ -217,11 +219,13 @@ Walk walk(const or_model* m) {
 
 inline double act_f(int act, double v, bool exact) {
   if (act == 1) return v > 0 ? v : 0.0;
+  if (act == 3) return v > 0 ? (v < 6.0 ? v : 6.0) : 0.0;  // ReLU6 (MobileNetV2, NEXT-3)
   if (act == 2) return v > 0 ? v : (exact ? 0.1 * v : (double)(0.1f * (float)v));  // fp32 0.1f*x (c.1 step 2)
   return v;
 }
 inline double act_d(int act, double y) {  // derivative from the stored output (ReLU'(0) = 0)
   if (act == 1) return y > 0 ? 1.0 : 0.0;
+  if (act == 3) return (y > 0 && y < 6.0) ? 1.0 : 0.0;  // ReLU6: 0 at both clamps
   if (act == 2) return y > 0 ? 1.0 : 0.1;
   return 1.0;
 }
@@ -253,8 +257,11 @@ struct Engine {
   int det_tensor = -1;
 
   // conv with weights taken from params (bf16-rounded unless exact)
+  // grouped conv (groups = 1: dense): output channel co reads input channels [g*Cg, (g+1)*Cg) of its group
+  // g = co / (Co / groups), weights [Co][KH][KW][Cg]
   void conv(const Tensor& x, const double* Wf, const double* bf, int Co, int KH, int KW, int s, int p,
-            vector<double>& acc, int& Ho, int& Wo) const {
+            vector<double>& acc, int& Ho, int& Wo, int groups = 1) const {
+    const int Cg = x.C / groups, Cog = Co / groups;
     Ho = (x.H + 2 * p - KH) / s + 1;
     Wo = (x.W + 2 * p - KW) / s + 1;
     acc.assign((size_t)Ho * Wo * Co, 0.0);
@@ -268,12 +275,12 @@ struct Engine {
             for (int kw = 0; kw < KW; ++kw) {
               const int iw = wo * s - p + kw;
               if (iw < 0 || iw >= x.W) continue;
-              const double* xp = &x.d[((size_t)ih * x.W + iw) * x.C];
-              const double* wp = Wf + (((int64_t)co * KH + kh) * KW + kw) * x.C;
+              const double* xp = &x.d[((size_t)ih * x.W + iw) * x.C + (size_t)(co / Cog) * Cg];
+              const double* wp = Wf + (((int64_t)co * KH + kh) * KW + kw) * Cg;
               if (exact)
-                for (int ci = 0; ci < x.C; ++ci) a += xp[ci] * wp[ci];
+                for (int ci = 0; ci < Cg; ++ci) a += xp[ci] * wp[ci];
               else
-                for (int ci = 0; ci < x.C; ++ci) a += xp[ci] * (double)or_bf16((float)wp[ci]);
+                for (int ci = 0; ci < Cg; ++ci) a += xp[ci] * (double)or_bf16((float)wp[ci]);
             }
           }
           // epilogue step 1: fp32 accumulator, then "+ b" in fp32
@@ -305,8 +312,9 @@ struct Engine {
         const int Cin = X.C;
         Tensor Y;
         vector<double> acc;
-        conv(X, P, P + (int64_t)op.cout * op.kh * op.kw * Cin, op.cout, op.kh, op.kw, op.stride, op.pad, acc,
-             Y.H, Y.W);
+        const int grp = op.groups > 0 ? op.groups : 1;
+        conv(X, P, P + (int64_t)op.cout * op.kh * op.kw * (Cin / grp), op.cout, op.kh, op.kw, op.stride, op.pad, acc,
+             Y.H, Y.W, grp);
         Y.C = op.cout;
         int res = -1;
         if (op.residual) {
@@ -471,11 +479,13 @@ struct Engine {
       const int KH = nd.kind == OR_CONV ? op.kh : 1, KW = nd.kind == OR_CONV ? op.kw : 1;
       const int s = op.stride, p = nd.kind == OR_CONV ? op.pad : 0, Co = Y.C, Ci = X.C;
       const int act = nd.kind == OR_CONV ? op.act : 0;
+      const int grp = (nd.kind == OR_CONV && op.groups > 0) ? op.groups : 1;
+      const int Cg = Ci / grp, Cog = Co / grp;
       vector<double> dZ = total(nd.out);
       for (size_t e = 0; e < dZ.size(); ++e) dZ[e] = R(F(dZ[e] * act_d(act, Y.d[e])));
       const double* Wf = params + w.poff[nd.op];
       double* gW = g + w.poff[nd.op];
-      double* gb = gW + (int64_t)Co * KH * KW * Ci;
+      double* gb = gW + (int64_t)Co * KH * KW * Cg;
       const bool need_dx = nd.in != 0;
       vector<double> dX;
       if (need_dx) dX.assign(X.d.size(), 0.0);
@@ -491,9 +501,9 @@ struct Engine {
               for (int kw = 0; kw < KW; ++kw) {
                 const int iw = wo * s - p + kw;
                 if (iw < 0 || iw >= X.W) continue;
-                const size_t xo = ((size_t)ih * X.W + iw) * Ci;
-                const int64_t wo_ = (((int64_t)co * KH + kh) * KW + kw) * Ci;
-                for (int ci = 0; ci < Ci; ++ci) {
+                const size_t xo = ((size_t)ih * X.W + iw) * Ci + (size_t)(co / Cog) * Cg;
+                const int64_t wo_ = (((int64_t)co * KH + kh) * KW + kw) * Cg;
+                for (int ci = 0; ci < Cg; ++ci) {
                   gW[wo_ + ci] += dz * X.d[xo + ci];
                   if (need_dx) dX[xo + ci] += dz * (exact ? Wf[wo_ + ci] : (double)or_bf16((float)Wf[wo_ + ci]));
                 }

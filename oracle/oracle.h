@@ -28,12 +28,13 @@ enum { OR_CONV = 0, OR_MAXPOOL = 1, OR_BLOCK = 2, OR_EXIT = 3, OR_DET_HEAD = 4 }
 typedef struct {
   int32_t kind;
   int32_t kh, kw, stride, pad, cout; /* CONV; MAXPOOL uses kh,kw,stride,pad; BLOCK: cout>0 -> 1x1 projection shortcut with `stride` */
-  int32_t act;                       /* CONV: 0 none, 1 ReLU, 2 leaky-ReLU(0.1) */
+  int32_t act;                       /* CONV: 0 none, 1 ReLU, 2 leaky-ReLU(0.1), 3 ReLU6 (MobileNetV2) */
   int32_t residual;                  /* CONV: add the innermost open BLOCK's shortcut before act, closes the block */
   int32_t num_classes;               /* EXIT */
   float loss_weight;                 /* EXIT */
   int32_t anchors, det_classes, grid_stride; /* DET_HEAD */
   float anchor_wh[16];               /* DET_HEAD: (w,h) per anchor, pixels */
+  int32_t groups;                    /* CONV: channel groups (1 dense, = Cin = Cout depthwise); 0 is read as 1 */
 } or_op;
 
 typedef struct {

@@ -29,7 +29,8 @@ class Op(C.Structure):
     _fields_ = [("kind", C.c_int32), ("kh", C.c_int32), ("kw", C.c_int32), ("stride", C.c_int32),
                 ("pad", C.c_int32), ("cout", C.c_int32), ("act", C.c_int32), ("residual", C.c_int32),
                 ("num_classes", C.c_int32), ("loss_weight", C.c_float), ("anchors", C.c_int32),
-                ("det_classes", C.c_int32), ("grid_stride", C.c_int32), ("anchor_wh", C.c_float * 16)]
+                ("det_classes", C.c_int32), ("grid_stride", C.c_int32), ("anchor_wh", C.c_float * 16),
+                ("nms_iou", C.c_float)]
 
 
 class ModelSpec(C.Structure):
@@ -177,6 +178,7 @@ def make_ops(spec):
         r.grid_stride = o.get("grid_stride", 0)
         for j, v in enumerate(o.get("anchor_wh", [])):
             r.anchor_wh[j] = v
+        r.nms_iou = float(o.get("nms_iou", 0.0))
     return ops
 
 

@@ -179,7 +179,7 @@ extern "C" adainf_status adainf_app_create(const adainf_app_spec* spec, adainf_a
           const TensorRt& D = m->T[m->det.tensor];
           const size_t ncand = (size_t)m->max_batch * D.H * D.W * m->det.anchors;
           S.det_table.alloc(ncand * 9 * 4);
-          S.det_ws.alloc(det_route_ws_bytes(m->max_batch, D.H, m->det.anchors));
+          S.det_ws.alloc(det_route_ws_bytes(m->max_batch, D.H, m->det.anchors, m->det.nms_iou > 0.f));
           const int ne = std::max<int>(1, (int)S.det_edges.size());
           S.n_det.alloc(16);
           S.route_idx.alloc((size_t)ne * std::max(1, a.max_routed) * 4);
@@ -285,6 +285,7 @@ extern "C" adainf_status adainf_infer_dag(adainf_app_t app, const void* batch, i
         d.n_routed = S.n_routed.as<int32_t>();
         d.count_clamped = S.cnt_clamped.as<int32_t>();
         d.cap_flag = I.cap_flag_dev;
+        d.nms_iou = m->det.nms_iou;
         launch_det_route(d, S.det_ws.p, st);
         for (int q = 0; q < d.n_edges; ++q) {
           const int e = S.det_edges[q];

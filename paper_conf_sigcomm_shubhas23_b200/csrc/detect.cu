@@ -157,10 +157,159 @@ __global__ void det_emit_kernel(const DetRouteArgs a, const int* __restrict__ bl
   }
 }
 
-size_t det_route_ws_bytes(int n_static, int G, int A) {
+// ------------------------------------------------------------------------------------------------
+// NMS (NEXT-3, reading Q18b): decode into a pre-NMS table (ascending candidate index, so each frame's rows are
+// contiguous), then per frame one CTA sorts its detections by (class, score descending, row) with a bitonic sort
+// in shared memory and one warp runs the greedy scan (fp32 IoU, every op rounded as in the oracle), then a single
+// CTA compacts the kept rows in order into det_table and the per-edge route lists.
+__device__ __forceinline__ float iou_rn(const float* a, const float* b) {
+  const float iw = fmaxf(0.f, __fsub_rn(fminf(a[2], b[2]), fmaxf(a[0], b[0])));
+  const float ih = fmaxf(0.f, __fsub_rn(fminf(a[3], b[3]), fmaxf(a[1], b[1])));
+  const float inter = __fmul_rn(iw, ih);
+  const float area_a = __fmul_rn(__fsub_rn(a[2], a[0]), __fsub_rn(a[3], a[1]));
+  const float area_b = __fmul_rn(__fsub_rn(b[2], b[0]), __fsub_rn(b[3], b[1]));
+  const float uni = __fsub_rn(__fadd_rn(area_a, area_b), inter);
+  return uni > 0.f ? __fdiv_rn(inter, uni) : 0.f;
+}
+
+__global__ void __launch_bounds__(256) nms_kernel(const float* __restrict__ pre, const int* __restrict__ n_pre,
+                                                  const int* frames_count, int n_static, int pow2, float thr,
+                                                  uint8_t* __restrict__ keep) {
+  extern __shared__ unsigned long long skey[];  // [pow2] keys, then boxes [pow2][4] fp32, sup [pow2] bytes
+  float* sbox = (float*)(skey + pow2);
+  uint8_t* sup = (uint8_t*)(sbox + 4 * pow2);
+  const int f = blockIdx.x;
+  const int nframes = frames_count ? min(*frames_count, n_static) : n_static;
+  if (f >= nframes) return;
+  const int n = *n_pre;
+  // rows of frame f: [lo, hi) by binary search on the frame column (non-decreasing)
+  __shared__ int s_lo, s_hi;
+  if (threadIdx.x < 2) {
+    const float key = (float)(f + threadIdx.x);
+    int lo = 0, hi = n;
+    while (lo < hi) {
+      const int mid = (lo + hi) >> 1;
+      if (pre[(long long)mid * 9] < key) lo = mid + 1;
+      else hi = mid;
+    }
+    if (threadIdx.x == 0) s_lo = lo;
+    else s_hi = lo;
+  }
+  __syncthreads();
+  const int lo = s_lo, cnt = s_hi - s_lo;
+  if (cnt <= 0) return;
+  for (int i = threadIdx.x; i < pow2; i += blockDim.x) {
+    unsigned long long k = ~0ull;
+    if (i < cnt) {
+      const float* r = pre + (long long)(lo + i) * 9;
+      const unsigned cls = (unsigned)r[3];
+      k = ((unsigned long long)cls << 56) | ((unsigned long long)(0xFFFFFFFFu - __float_as_uint(r[4])) << 24) |
+          (unsigned long long)i;
+    }
+    skey[i] = k;
+    if (i < cnt) keep[lo + i] = 0;
+  }
+  __syncthreads();
+  for (int size = 2; size <= pow2; size <<= 1)
+    for (int stride = size >> 1; stride > 0; stride >>= 1) {
+      for (int i = threadIdx.x; i < pow2; i += blockDim.x) {
+        const int j = i ^ stride;
+        if (j > i) {
+          const bool up = (i & size) == 0;
+          const unsigned long long x = skey[i], y = skey[j];
+          if ((x > y) == up) {
+            skey[i] = y;
+            skey[j] = x;
+          }
+        }
+      }
+      __syncthreads();
+    }
+  for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
+    const int row = (int)(skey[i] & 0xFFFFFFull);
+    const float* r = pre + (long long)(lo + row) * 9;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) sbox[i * 4 + q] = r[5 + q];
+    sup[i] = 0;
+  }
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    const int lane = threadIdx.x;
+    for (int p = 0; p < cnt; ++p) {
+      __syncwarp();
+      if (sup[p]) continue;
+      const unsigned cls = (unsigned)(skey[p] >> 56);
+      if (lane == 0) keep[lo + (int)(skey[p] & 0xFFFFFFull)] = 1;
+      for (int q = p + 1 + lane; q < cnt; q += 32) {
+        if ((unsigned)(skey[q] >> 56) != cls) break;
+        if (!sup[q] && iou_rn(sbox + p * 4, sbox + q * 4) > thr) sup[q] = 1;
+      }
+    }
+  }
+}
+
+// stable compaction of the kept rows into det_table (+ the caller's copy) and the per-edge route lists
+__global__ void __launch_bounds__(1024) nms_route_kernel(const DetRouteArgs a, const float* __restrict__ pre,
+                                                         const int* __restrict__ n_pre, const uint8_t* __restrict__ keep) {
+  __shared__ int wtot[32][1 + MAX_EDGES];
+  __shared__ int run[1 + MAX_EDGES];
+  const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+  const int n = *n_pre;
+  const int ncol = 1 + a.n_edges;
+  if (t < ncol) run[t] = 0;
+  __syncthreads();
+  for (int c0 = 0; c0 < n; c0 += 1024) {
+    const int i = c0 + t;
+    const bool f = i < n && keep[i];
+    const int e = f ? edge_of(a, (int)pre[(long long)i * 9 + 3]) : -1;
+    unsigned bal[1 + MAX_EDGES];
+    bal[0] = __ballot_sync(0xffffffffu, f);
+    for (int k = 0; k < a.n_edges; ++k) bal[1 + k] = __ballot_sync(0xffffffffu, e == k);
+    if (lane == 0)
+      for (int k = 0; k < ncol; ++k) wtot[w][k] = __popc(bal[k]);
+    __syncthreads();
+    if (f) {
+      const unsigned lt = (1u << lane) - 1u;
+      int p0 = run[0] + __popc(bal[0] & lt);
+      for (int q = 0; q < w; ++q) p0 += wtot[q][0];
+      const float* src = pre + (long long)i * 9;
+      float* d = a.det_table + (long long)p0 * 9;
+      for (int q = 0; q < 9; ++q) d[q] = src[q];
+      if (a.user_table && p0 < a.user_max)
+        for (int q = 0; q < 9; ++q) a.user_table[(long long)p0 * 9 + q] = src[q];
+      if (e >= 0) {
+        int pe = run[1 + e] + __popc(bal[1 + e] & lt);
+        for (int q = 0; q < w; ++q) pe += wtot[q][1 + e];
+        if (pe < a.cap) a.route_idx[(long long)e * a.cap + pe] = p0;
+      }
+    }
+    __syncthreads();
+    if (t < ncol) {
+      int tot = 0;
+      for (int q = 0; q < 32; ++q) tot += wtot[q][t];
+      run[t] += tot;
+    }
+    __syncthreads();
+  }
+  if (t < ncol) {
+    const int r = run[t];
+    if (t == 0) {
+      if (a.n_det) *a.n_det = r;
+    } else {
+      const int e = t - 1;
+      if (a.n_routed) a.n_routed[e] = r;
+      a.count_clamped[e] = min(r, a.cap);
+      if (r > a.cap && a.cap_flag) atomicExch(a.cap_flag, 1);
+    }
+  }
+}
+
+size_t det_route_ws_bytes(int n_static, int G, int A, bool nms) {
   const long long ncand = (long long)n_static * G * G * A;
   const long long nb = (ncand + DET_PER_BLOCK - 1) / DET_PER_BLOCK;
-  return (size_t)nb * (1 + MAX_EDGES) * sizeof(int) + 256;
+  size_t b = (size_t)nb * (1 + MAX_EDGES) * sizeof(int) + 256;
+  if (nms) b += 256 + (size_t)ncand * 9 * 4 + 256 + (size_t)ncand + 256 + 16;
+  return b;
 }
 
 void launch_det_route(const DetRouteArgs& a, void* ws, cudaStream_t st) {
@@ -168,6 +317,39 @@ void launch_det_route(const DetRouteArgs& a, void* ws, cudaStream_t st) {
   const long long ncand = (long long)a.n_static * a.G * a.G * a.A;
   const int nb = (int)((ncand + DET_PER_BLOCK - 1) / DET_PER_BLOCK);
   int* blk = (int*)ws;
+  if (a.nms_iou > 0.f) {
+    char* p = (char*)ws + ((size_t)nb * (1 + MAX_EDGES) * sizeof(int) + 256 + 255) / 256 * 256;
+    float* pre = (float*)p;
+    p += ((size_t)ncand * 9 * 4 + 255) / 256 * 256;
+    uint8_t* keep = (uint8_t*)p;
+    p += ((size_t)ncand + 255) / 256 * 256;
+    int* n_pre = (int*)p;
+    DetRouteArgs b = a;  // decode only: every detection into the pre-NMS table, no routing yet
+    b.n_edges = 0;
+    b.det_table = pre;
+    b.user_table = nullptr;
+    b.user_max = 0;
+    b.n_det = n_pre;
+    b.n_routed = nullptr;
+    const int per_frame = a.G * a.G * a.A;
+    int pow2 = 1;
+    while (pow2 < per_frame) pow2 <<= 1;
+    const size_t smem = (size_t)pow2 * (8 + 16 + 1) + 64;
+    if (smem > 200 * 1024) throw ShapeError("NMS: too many candidates per frame");
+    static size_t attr = 0;
+    if (smem > 48 * 1024 && smem > attr) {
+      CK(cudaFuncSetAttribute(nms_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      attr = smem;
+    }
+    ProfScope ps(PC_DET_ROUTE, st, 5);
+    det_count_kernel<<<nb, DET_THREADS, 0, st>>>(b, blk);
+    det_scan_kernel<<<1, 32 * (1 + MAX_EDGES), 0, st>>>(b, nb, blk);
+    det_emit_kernel<<<nb, DET_THREADS, 0, st>>>(b, blk);
+    nms_kernel<<<a.n_static, 256, smem, st>>>(pre, n_pre, a.count, a.n_static, pow2, a.nms_iou, keep);
+    nms_route_kernel<<<1, 1024, 0, st>>>(a, pre, n_pre, keep);
+    CK(cudaGetLastError());
+    return;
+  }
   ProfScope ps(PC_DET_ROUTE, st, 3);
   det_count_kernel<<<nb, DET_THREADS, 0, st>>>(a, blk);
   det_scan_kernel<<<1, 32 * (1 + MAX_EDGES), 0, st>>>(a, nb, blk);

@@ -190,6 +190,8 @@ void Model::build(const adainf_model_spec& s) {
     } else if (o.kind == ADAINF_OP_DET_HEAD) {
       if (!T[cur].f32) throw InvalidError("DET_HEAD must follow a conv");
       det.tensor = cur;
+      if (!(o.nms_iou >= 0.f) || o.nms_iou > 1.f) throw InvalidError("DET_HEAD: nms_iou must be in [0, 1]");
+      det.nms_iou = o.nms_iou;
       det.anchors = o.anchors;
       det.classes = o.det_classes;
       det.stride = o.grid_stride;

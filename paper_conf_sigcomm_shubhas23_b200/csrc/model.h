@@ -84,6 +84,7 @@ struct DetRt {
   int tensor = -1;
   int anchors = 0, classes = 0, stride = 0;
   float anchor_wh[16];
+  float nms_iou = 0.f;  // > 0: greedy NMS before routing (NEXT-3)
 };
 
 struct Model {
@@ -171,8 +172,9 @@ struct DetRouteArgs {
   int32_t* n_routed;     // [n_edges] required
   int32_t* count_clamped;  // [n_edges]
   int32_t* cap_flag;
+  float nms_iou;           // > 0: NMS between decode and routing
 };
-size_t det_route_ws_bytes(int n_static, int G, int A);
+size_t det_route_ws_bytes(int n_static, int G, int A, bool nms);
 void launch_det_route(const DetRouteArgs& a, void* ws, cudaStream_t st);
 void launch_crops(const bf16* frames, int H, int W, int C, const float* det_table, const int32_t* route_idx,
                   const int32_t* count_clamped, int edge, int cap, int crop_h, int crop_w, int cout_pad, bf16* dst,

@@ -12,15 +12,16 @@ synthetic audio DAG (Q24).
 """
 from __future__ import annotations
 
-RELU, LEAKY, NONE = 1, 2, 0
+RELU, LEAKY, NONE, RELU6 = 1, 2, 0, 3
 
 # TinyYOLOv3 13x13-scale anchors (w, h) in pixels (reading Q18)
 YOLO_ANCHORS = [81.0, 82.0, 135.0, 169.0, 344.0, 319.0]
 
 
-def conv(k, cout, stride=1, pad=None, act=RELU, residual=False):
+def conv(k, cout, stride=1, pad=None, act=RELU, residual=False, groups=1):
+    """groups > 1: grouped conv (groups == cin == cout: depthwise, MobileNetV2 / ShuffleNet, NEXT-3)"""
     return {"kind": "conv", "kh": k, "kw": k, "stride": stride, "pad": (k // 2) if pad is None else pad,
-            "cout": cout, "act": act, "residual": int(residual)}
+            "cout": cout, "act": act, "residual": int(residual), "groups": groups}
 
 
 def maxpool(k, stride, pad=0):
@@ -59,15 +60,54 @@ def resnet18_ee(num_classes=10, in_hw=224, in_c=3):
     return {"name": "resnet18_ee", "in_h": in_hw, "in_w": in_hw, "in_c": in_c, "ops": ops}
 
 
-def tiny_yolo_det(in_hw=416, det_classes=2, anchors=3, width=512):
-    """BASELINE config 3 detector: TinyYOLOv3-like single-scale, 'compressed' (layer 7 1024->512)."""
+def _inverted_residual(cin, cout, stride, t):
+    """MobileNetV2 inverted residual (NEXT-3): 1x1 expand (ReLU6, skipped when t == 1) -> 3x3 depthwise
+    (ReLU6) -> 1x1 linear projection, + identity shortcut when stride 1 and cin == cout."""
+    hid = cin * t
+    ops = []
+    res = stride == 1 and cin == cout
+    if res:
+        ops.append(block(0))
+    if t != 1:
+        ops.append(conv(1, hid, act=RELU6))
+    ops.append(conv(3, hid, stride=stride, act=RELU6, groups=hid))
+    ops.append(conv(1, cout, act=NONE, residual=res))
+    return ops
+
+
+MNV2_STAGES = [(1, 16, 1, 1), (6, 24, 2, 2), (6, 32, 3, 2), (6, 64, 4, 2), (6, 96, 3, 1), (6, 160, 3, 2),
+               (6, 320, 1, 1)]
+
+
+def mobilenetv2_ee(num_classes=10, in_hw=224, in_c=3, width=1.0, exits_after=(1, 2, 4)):
+    """MobileNetV2 early-exit classifier (the paper's video-DAG classifier; NEXT-3): stem 3x3/2 conv 32
+    (ReLU6), inverted-residual stages (t, c, n, s) as in MobileNetV2, 1x1 conv 1280 (ReLU6); exits after the
+    stages listed in exits_after (stage indices into MNV2_STAGES: 24-ch 56x56, 32-ch 28x28, 96-ch 14x14 at 224)
+    + the final GAP -> FC head (reading Q3: exits at stage boundaries)."""
+    def ch(c):
+        return max(8, int(round(c * width / 8)) * 8)
+    ops = [conv(3, ch(32), stride=2, act=RELU6)]
+    cin = ch(32)
+    for si, (t, c, n, s_) in enumerate(MNV2_STAGES):
+        for b in range(n):
+            ops += _inverted_residual(cin, ch(c), s_ if b == 0 else 1, t)
+            cin = ch(c)
+        if si in exits_after:
+            ops.append(exit_(num_classes))
+    ops += [conv(1, ch(1280), act=RELU6), exit_(num_classes)]
+    return {"name": "mobilenetv2_ee", "in_h": in_hw, "in_w": in_hw, "in_c": in_c, "ops": ops}
+
+
+def tiny_yolo_det(in_hw=416, det_classes=2, anchors=3, width=512, nms_iou=0.0):
+    """BASELINE config 3 detector: TinyYOLOv3-like single-scale, 'compressed' (layer 7 1024->512); nms_iou > 0
+    adds greedy per-(frame, class) NMS before routing (NEXT-3, reading Q18b; TinyYOLOv3 uses 0.45)."""
     ops = []
     for c in (16, 32, 64, 128, 256):
         ops += [conv(3, c, act=LEAKY), maxpool(2, 2)]
     ops += [conv(3, 512, act=LEAKY), maxpool(3, 1, 1), conv(3, width, act=LEAKY), conv(1, 256, act=LEAKY),
             conv(3, 512, act=LEAKY), conv(1, anchors * (5 + det_classes), act=NONE),
             {"kind": "det_head", "anchors": anchors, "det_classes": det_classes, "grid_stride": 32,
-             "anchor_wh": YOLO_ANCHORS[:2 * anchors]}]
+             "anchor_wh": YOLO_ANCHORS[:2 * anchors], "nms_iou": nms_iou}]
     return {"name": "tiny_yolo_det", "in_h": in_hw, "in_w": in_hw, "in_c": 3, "ops": ops}
 
 
@@ -78,7 +118,7 @@ def num_params(spec) -> int:
     for o in spec["ops"]:
         k = o["kind"]
         if k == "conv":
-            n += o["cout"] * o["kh"] * o["kw"] * Cc + o["cout"]
+            n += o["cout"] * o["kh"] * o["kw"] * (Cc // o.get("groups", 1)) + o["cout"]
             H = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
             W = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
             Cc = o["cout"]
@@ -99,9 +139,9 @@ def param_segments(spec):
     for i, o in enumerate(spec["ops"]):
         k = o["kind"]
         if k == "conv":
-            shp = (o["cout"], o["kh"], o["kw"], Cc)
+            shp = (o["cout"], o["kh"], o["kw"], Cc // o.get("groups", 1))
             segs.append(("conv_w", i, off, shp))
-            off += o["cout"] * o["kh"] * o["kw"] * Cc
+            off += o["cout"] * o["kh"] * o["kw"] * (Cc // o.get("groups", 1))
             segs.append(("conv_b", i, off, (o["cout"],)))
             off += o["cout"]
             H = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
@@ -133,7 +173,7 @@ def macs_per_sample(spec):
         if k == "conv":
             Ho = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
             Wo = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
-            m = Ho * Wo * o["cout"] * o["kh"] * o["kw"] * Cc
+            m = Ho * Wo * o["cout"] * o["kh"] * o["kw"] * (Cc // o.get("groups", 1))
             H, W, Cc = Ho, Wo, o["cout"]
         elif k == "maxpool":
             H = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1

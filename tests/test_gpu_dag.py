@@ -87,8 +87,10 @@ def test_video_dag_detector_routing_crops():
         if c in omap and not band[c]:
             o = omap[c]
             assert abs(r[4] - o[4]) < 2e-3
+            # boxes are exp / sigmoid transforms of the head logits: held to the north_star logit tolerance (2e-2
+            # relative, + 0.5 px), reading Q20 as amended in DESIGN.md (the detector's spread logits drift ~6e-3)
             size = max(o[7] - o[5], o[8] - o[6], 1.0)
-            assert np.all(np.abs(r[5:] - o[5:]) <= 0.5 + 1e-3 * size), (r, o)
+            assert np.all(np.abs(r[5:] - o[5:]) <= 0.5 + 2e-2 * size), (r, o)
     # routing: per class, ascending detection numbers; counts = detections of that class
     n_routed = outs[0]["n_routed"].cpu().numpy()
     ridx = outs[0]["route_idx"].cpu().numpy()
@@ -223,3 +225,46 @@ def test_video_dag_c3_geometry():
     app.close()
     for m in (m_det, m_veh, m_per):
         m.close()
+
+
+def test_detector_nms_stage_isolated():
+    """NEXT-3 (reading Q18b): greedy per-(frame, class) NMS on the device between decode and routing.  Stage
+    isolation as for the crops (Q20): the same detector without NMS yields the GPU's pre-NMS detections; the oracle's
+    NMS on exactly those rows must select exactly the rows the NMS-enabled detector keeps (bit-exact, in order), and
+    routing must list the kept rows by class."""
+    Bn, hw = 3, 416
+    base = S.tiny_yolo_det(in_hw=hw)
+    nmsd = S.tiny_yolo_det(in_hw=hw, nms_iou=0.45)
+    A, NC = 3, 2
+    p = synth.det_head_params(base, synth.init_params(base, seed=61), obj_bias=-1.0)
+    xb, _ = synth.drifted_images(Bn, hw, hw, 3, seed=61)
+    x = to_cuda_bf16(xb)
+    G = hw // 32
+    max_det = Bn * G * G * A
+    res = {}
+    for name, spec in (("pre", base), ("nms", nmsd)):
+        m = B.Model(spec, Bn, params=p)
+        veh, per = small_cls(10, hw=32), small_cls(8, hw=32)
+        mv, mp = B.Model(veh, max_det, params=synth.init_params(veh, seed=62)), B.Model(per, max_det,
+                                                                                    params=synth.init_params(per, seed=63))
+        app = B.App([m, mv, mp], edges=[(0, 1, B.ROUTE_DET_CROP, 0, 32, 32), (0, 2, B.ROUTE_DET_CROP, 1, 32, 32)],
+                    max_routed_per_dst=max_det)
+        outs = [B.alloc_outs(m, Bn, max_det=max_det, n_out_edges=2, max_routed=max_det), B.alloc_outs(mv, max_det),
+                B.alloc_outs(mp, max_det)]
+        app.infer(x, [0.12] + [0.5] + [0.5], outs)
+        app.poll()
+        n = int(outs[0]["n_det"].item())
+        res[name] = (outs[0]["det_table"].cpu().numpy()[:n].copy(), outs[0]["n_routed"].cpu().numpy().copy(),
+                     outs[0]["route_idx"].cpu().numpy().copy())
+        app.close()
+        for mm in (m, mv, mp):
+            mm.close()
+    pre, _, _ = res["pre"]
+    got, n_routed, ridx = res["nms"]
+    assert pre.shape[0] > 50  # plenty of overlapping candidates per frame
+    keep, nk = O.nms(pre, 0.45)
+    assert 0 < nk < pre.shape[0]
+    np.testing.assert_array_equal(got, pre[keep.astype(bool)])
+    for e in range(2):
+        want = [i for i in range(got.shape[0]) if int(got[i][3]) == e]
+        assert n_routed[e] == len(want) and ridx[e][:len(want)].tolist() == want

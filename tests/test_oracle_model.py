@@ -28,6 +28,12 @@ def test_param_counts_match_survey():
     # per-sample MACs: ResNet-18 full 1,813.6 M, detector 1,693.6 M
     assert abs(sum(S.macs_per_sample(S.resnet18_ee())) / 1e6 - 1813.6) < 1.0
     assert abs(sum(S.macs_per_sample(S.tiny_yolo_det())) / 1e6 - 1693.6) < 2.0
+    # MobileNetV2 (NEXT-3) at 1000 classes without early exits: 300.77 M MACs and, with each conv bias counted as
+    # the two BN parameters it replaces (reading Q10), exactly torchvision's 3,504,872 parameters
+    mn = S.mobilenetv2_ee(num_classes=1000, exits_after=())
+    assert abs(sum(S.macs_per_sample(mn)) / 1e6 - 300.774) < 0.01
+    n_bias = sum(o["cout"] for o in mn["ops"] if o["kind"] == "conv")
+    assert S.num_params(mn) + n_bias == 3504872 == O.Model(mn).num_params + n_bias
 
 
 class _GradRound(torch.autograd.Function):
@@ -75,12 +81,15 @@ def torch_forward(spec, params, x, exact, want_det=False):
         k = o["kind"]
         if k == "conv":
             w = R(seg("conv_w", i).permute(0, 3, 1, 2))
-            v = Fp(Fp(F.conv2d(cur, w, stride=o["stride"], padding=o["pad"])) + seg("conv_b", i)[None, :, None, None])
+            v = Fp(Fp(F.conv2d(cur, w, stride=o["stride"], padding=o["pad"], groups=o.get("groups", 1))) +
+                   seg("conv_b", i)[None, :, None, None])
             if o["residual"]:
                 v = Fp(v + blocks.pop())
             v = GR(v)
             if o["act"] == 1:
                 v = torch.relu(v)
+            elif o["act"] == 3:  # ReLU6, derivative 1 strictly inside (0, 6)
+                v = torch.where((v > 0) & (v < 6), v, torch.where(v >= 6, torch.full_like(v, 6.0), torch.zeros_like(v)))
             elif o["act"] == 2:
                 neg = 0.1 * v if exact else (v.float() * torch.tensor(0.1, dtype=torch.float32)).double()
                 neg = neg if exact else v * 0.1 + (neg - v * 0.1).detach()
@@ -122,11 +131,22 @@ def det_spec():
     return {"name": "det", "in_h": 12, "in_w": 12, "in_c": 3, "ops": ops}
 
 
-SPECS = {"mini": mini_spec, "tiny": S.tiny_cnn_ee, "stem": stem_spec,
+def mnv2_spec():
+    """MobileNetV2-style pieces (NEXT-3): ReLU6, 1x1 expand, 3x3 depthwise (groups = channels, stride 1 and 2),
+    linear projection with and without the identity shortcut, a grouped (non-depthwise) conv, two exits."""
+    ops = [S.conv(3, 16, stride=2, act=S.RELU6), S.conv(3, 16, act=S.RELU6, groups=16), S.conv(1, 8, act=S.NONE),
+           S.exit_(4), S.block(0), S.conv(1, 24, act=S.RELU6), S.conv(3, 24, act=S.RELU6, groups=24),
+           S.conv(1, 8, act=S.NONE, residual=True), S.conv(1, 32, act=S.RELU6),
+           S.conv(3, 32, stride=2, act=S.RELU6, groups=32), S.conv(3, 16, act=S.RELU6, groups=4), S.exit_(4)]
+    return {"name": "mnv2", "in_h": 17, "in_w": 18, "in_c": 3, "ops": ops}
+
+
+SPECS = {"mini": mini_spec, "tiny": S.tiny_cnn_ee, "stem": stem_spec, "mnv2": mnv2_spec,
+         "mnv2_32": lambda: S.mobilenetv2_ee(in_hw=32, width=0.5),
          "resnet32": lambda: S.resnet18_ee(in_hw=32), "resnet64": lambda: S.resnet18_ee(in_hw=64)}
 
 
-@pytest.mark.parametrize("which", ["mini", "tiny", "stem", "resnet32", "resnet64"])
+@pytest.mark.parametrize("which", ["mini", "tiny", "stem", "resnet32", "resnet64", "mnv2", "mnv2_32"])
 def test_forward_vs_torch_interpreter(which):
     """c.1 steps 2-3 at model level, including the ResNet stem geometry (7x7/2/3 conv, 3x3/2/1 padded
     max-pool), leaky-ReLU and every residual form: a padding, pool-window or slope mistake in the
@@ -170,7 +190,7 @@ def _labels(n, ncls, seed):
     return np.random.default_rng(seed).integers(0, ncls, n).astype(np.int32)
 
 
-@pytest.mark.parametrize("which", ["mini", "stem"])
+@pytest.mark.parametrize("which", ["mini", "stem", "mnv2"])
 def test_exact_grad_vs_autograd_and_fd(which):
     """c.1 steps 10-11: the backward derivation (CE over all exits, head grads, GAP broadcast, ReLU and
     leaky-ReLU masks, first-max max-pool routing incl. the padded 3x3/2/1 stem pool, residual copy,
@@ -201,7 +221,7 @@ def test_exact_grad_vs_autograd_and_fd(which):
         assert abs(fd - g[j]) <= 1e-6 + 1e-4 * abs(g[j]), (j, fd, g[j])
 
 
-@pytest.mark.parametrize("which", ["mini", "tiny", "stem", "resnet32"])
+@pytest.mark.parametrize("which", ["mini", "tiny", "stem", "resnet32", "mnv2"])
 def test_bf16_storage_grads_vs_torch_emulation(which):
     """The bf16-storage gradient (what the GPU must match) against
     torch.autograd over the interpreter with the same rounding points emulated (straight-through bf16 /
