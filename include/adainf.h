@@ -59,7 +59,7 @@ typedef void* adainf_stream_t; /* cudaStream_t (NULL = legacy default stream) */
 
 /* ---- Model description (the "exit-layer spec" of north_star) ----------------------------------
  * A model is a sequence of ops applied to the current tensor:
- *   CONV     kh x kw conv, stride, pad, cout; act 0 none / 1 ReLU / 2 leaky-ReLU(0.1); BN folded
+ *   CONV     kh x kw conv, stride, pad, cout; act 0 none / 1 ReLU / 2 leaky-ReLU(0.1) / 3 ReLU6; BN folded
  *            (reading Q10).  residual=1: add the innermost open BLOCK's shortcut before the act and
  *            close that block.  A CONV directly followed by DET_HEAD writes fp32 (no bf16 rounding).
  *   MAXPOOL  kh x kw window, stride, pad (padding = -inf).
@@ -74,7 +74,7 @@ typedef void* adainf_stream_t; /* cudaStream_t (NULL = legacy default stream) */
  *            nms_iou > 0 the detections then go through greedy NMS per (frame, class): visited by score
  *            descending (ties -> lower candidate index), dropped if their fp32 IoU with a kept detection exceeds
  *            nms_iou; det_table / n_det / routing then list the kept detections (ascending candidate index).
- * Parameter layout (flat fp32, op order): CONV W[cout][kh][kw][cin] then b[cout]; BLOCK with cout>0:
+ * Parameter layout (flat fp32, op order): CONV W[cout][kh][kw][cin / groups] then b[cout]; BLOCK with cout>0:
  * W[cout][1][1][cin] then b[cout]; EXIT: Wk[cin][num_classes] then bk[num_classes].            */
 typedef enum {
   ADAINF_OP_CONV = 0,
@@ -95,6 +95,8 @@ typedef struct {
   float anchor_wh[16];
   float nms_iou;      /* DET_HEAD: > 0 -> greedy per-(frame, class) NMS at this IoU threshold before routing
                          (NEXT-3, reading Q18b); 0 -> none */
+  int32_t groups;     /* CONV: 0 / 1 dense; == cin == cout: depthwise 3x3 (MobileNetV2, NEXT-3); other values
+                         ADAINF_ERR_UNSUPPORTED.  Weights [cout][kh][kw][cin / groups] */
 } adainf_op;
 
 typedef struct {

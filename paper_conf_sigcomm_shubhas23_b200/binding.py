@@ -30,7 +30,7 @@ class Op(C.Structure):
                 ("pad", C.c_int32), ("cout", C.c_int32), ("act", C.c_int32), ("residual", C.c_int32),
                 ("num_classes", C.c_int32), ("loss_weight", C.c_float), ("anchors", C.c_int32),
                 ("det_classes", C.c_int32), ("grid_stride", C.c_int32), ("anchor_wh", C.c_float * 16),
-                ("nms_iou", C.c_float)]
+                ("nms_iou", C.c_float), ("groups", C.c_int32)]
 
 
 class ModelSpec(C.Structure):
@@ -179,6 +179,7 @@ def make_ops(spec):
         for j, v in enumerate(o.get("anchor_wh", [])):
             r.anchor_wh[j] = v
         r.nms_iou = float(o.get("nms_iou", 0.0))
+        r.groups = int(o.get("groups", 1))
     return ops
 
 

@@ -195,13 +195,17 @@ __host__ __device__ constexpr uint32_t make_idesc(int M, int N, int a_mn_major, 
 
 // Branch-free (select) forms: the activation kind is a runtime layer attribute, and a per-element branch on it
 // costs the single epilogue warp of each TMEM lane quadrant more than the arithmetic itself.
+// act: 0 none, 1 ReLU, 2 leaky-ReLU (0.1f), 3 ReLU6 (MobileNetV2, NEXT-3)
 __device__ __forceinline__ float act_apply(int act, float v) {
   const float neg = act == 2 ? __fmul_rn(0.1f, v) : 0.f;
-  return (act == 0 || v > 0.f) ? v : neg;
+  const float pos = act == 3 ? fminf(v, 6.f) : v;
+  return (act == 0 || v > 0.f) ? pos : neg;
 }
+// derivative from the stored output y (ReLU'(0) = 0; ReLU6' = 0 at both clamps)
 __device__ __forceinline__ float act_grad(int act, float y) {
   const float neg = act == 2 ? 0.1f : 0.f;
-  return (act == 0 || y > 0.f) ? 1.f : neg;
+  const float pos = (act == 3 && y >= 6.f) ? 0.f : 1.f;
+  return (act == 0 || y > 0.f) ? pos : neg;
 }
 
 }  // namespace adainf

@@ -382,11 +382,13 @@ __global__ void __launch_bounds__(EH_THREADS) exit_head_kernel(const ExitHeadArg
 }
 void launch_exit_head(const ExitHeadArgs& a, cudaStream_t st, int prof_class) {
   if (a.n_static <= 0) return;
-  const bool wide = a.n_static < 4 * num_sms();
-  const bool widest = a.n_static <= 2 * num_sms();  // a row per CTA cannot fill the SMs: 1,024 threads per row
-  const int T = widest ? 1024 : (wide ? 512 : 128);
-  if (a.C % 8 || (T % (a.C / 8)) != 0 || a.C / 8 > 128)
-    throw ShapeError("exit head: C must be 8 * a power of two <= 1024");
+  bool wide = a.n_static < 4 * num_sms();
+  bool widest = a.n_static <= 2 * num_sms();  // a row per CTA cannot fill the SMs: 1,024 threads per row
+  int T = widest ? 1024 : (wide ? 512 : 128);
+  if (a.C % 8 || a.C / 8 > 1024) throw ShapeError("exit head: C must be a multiple of 8, <= 8192");
+  while (a.C / 8 > T) T = T == 128 ? 512 : 1024;  // every 8-channel vector needs a thread
+  widest = T == 1024;
+  wide = T == 512;
   const int groups = T / (a.C / 8);
   const size_t smem = (size_t)(groups * a.C + a.C + a.ncls) * sizeof(float);
   ProfScope ps(prof_class, st);
@@ -592,11 +594,13 @@ void launch_exit_fused(const ExitHeadArgs& h, unsigned* ws, int* pos_next, int* 
                        int32_t* counts_out, int32_t* surv_out, int32_t* last_count_out, int last_index,
                        const bf16* src, bf16* dense_next, long long row_elems, cudaStream_t st) {
   if (h.n_static <= 0) return;
-  const bool wide = h.n_static < 4 * num_sms();
-  const bool widest = h.n_static <= 2 * num_sms();
-  const int T = widest ? 1024 : (wide ? 512 : 128);
-  if (h.C % 8 || (T % (h.C / 8)) != 0 || h.C / 8 > 128)
-    throw ShapeError("exit head: C must be 8 * a power of two <= 1024");
+  bool wide = h.n_static < 4 * num_sms();
+  bool widest = h.n_static <= 2 * num_sms();
+  int T = widest ? 1024 : (wide ? 512 : 128);
+  if (h.C % 8 || h.C / 8 > 1024) throw ShapeError("exit head: C must be a multiple of 8, <= 8192");
+  while (h.C / 8 > T) T = T == 128 ? 512 : 1024;
+  widest = T == 1024;
+  wide = T == 512;
   if (src && (row_elems % 8)) throw ShapeError("exit_fused: row must be a multiple of 16 bytes");
   const int groups = T / (h.C / 8);
   const size_t smem = (size_t)(groups * h.C + h.C + h.ncls) * sizeof(float);

@@ -24,6 +24,44 @@ void launch_maxpool_fwd(const bf16* x, const int* map, const int* count, int n_s
 void launch_maxpool_bwd(const bf16* dT, const uint8_t* argmax, const bf16* pooled, int act, int n, int H, int W, int C,
                         int K, int s, int p, int Ho, int Wo, bf16* dz, cudaStream_t st);
 
+// ---- depthwise conv (groups == channels; NEXT-3 MobileNetV2), dwconv.cu ----
+struct DwArgs {
+  const bf16* x;        // fwd / wgrad: input [n][H][W][C]; dgrad: dZ [n][Ho][Wo][C]
+  const bf16* dz;       // wgrad: dZ
+  const int* map;       // fwd: input row map (inference stages) or nullptr
+  const int* count;     // fwd: device row count or nullptr
+  int n_static;
+  int H, W, C, Ho, Wo, KH, KW, s, p;
+  const bf16* w;        // [taps][C] (dw_prep)
+  const float* bias;    // fwd
+  int act;              // fwd
+  const float* bcast;   // dgrad: exit broadcast [n][C] or nullptr
+  const bf16* sc;       // dgrad: shortcut term [n][H][W][C] or nullptr
+  const bf16* yact;     // dgrad: producer output for the activation mask, or nullptr
+  int mask_act;
+  bf16* y;              // fwd: output; dgrad: dX
+};
+bool dw_ok(const ConvGeom& g, int groups);
+void dw_prep(const bf16* shadow, int ldb, int C, int taps, bf16* wdw, cudaStream_t st);
+void dw_fwd(const DwArgs& a, cudaStream_t st);
+void dw_dgrad(const DwArgs& a, cudaStream_t st);
+size_t dw_wgrad_ws_bytes(const ConvGeom& g, int n);
+void dw_wgrad(const DwArgs& a, float* ws, size_t ws_bytes, float* dw, float* db, cudaStream_t st);
+
+// ---- first conv layer fused with its 2x2/2 max-pool (inference; the detector's 416x416x3 -> 16 layer), convpool.cu
+struct ConvPoolArgs {
+  const bf16* x;        // packed input [n][H][W][cin_pad]
+  const int* count;     // device row count or nullptr
+  int n_static, H, W, cin_real, cin_pad;
+  const bf16* shadow;   // GEMM shadow [16][ldb], K = tap * cin_pad + c
+  int ldb;
+  const float* bias;
+  int act;
+  bf16* y;              // pooled [n][H/2][W/2][16]
+};
+bool conv_first_pool_ok(const ConvGeom& g, int cin_real, int pk, int ps, int pp);
+void conv_first_pool(const ConvPoolArgs& a, cudaStream_t st);
+
 // ---- exit head (K4) ----
 struct ExitHeadArgs {
   const bf16* fmap;     // dense [rows][HW][C]

@@ -53,7 +53,7 @@ void Model::build(const adainf_model_spec& s) {
   t0.H = in_h;
   t0.W = in_w;
   t0.C = cin_pad;
-  T.push_back(t0);
+  T.push_back(std::move(t0));
   int cur = 0, stage = 0;
   std::vector<int> blocks;
   op_node.assign(ops.size(), -1);
@@ -93,13 +93,19 @@ void Model::build(const adainf_model_spec& s) {
       nd.g.Ho = (X.H + 2 * pd - KH) / st + 1;
       nd.g.Wo = (X.W + 2 * pd - KW) / st + 1;
       if (nd.g.Ho <= 0 || nd.g.Wo <= 0) throw ShapeError("conv: empty output");
-      nd.cin_real = (cur == 0) ? in_c : X.C;
+      nd.groups = (!proj && o.groups > 1) ? o.groups : 1;
+      if (nd.groups > 1) {
+        if (!dw_ok(nd.g, nd.groups) || cur == 0)
+          throw UnsupportedError("grouped conv: only depthwise 3x3 (groups == cin == cout, multiple of 8) is supported");
+      }
+      if (!proj && (o.act < 0 || o.act > 3)) throw InvalidError("conv: act must be 0..3");
+      nd.cin_real = (cur == 0) ? in_c : X.C / nd.groups;
       nd.act = proj ? 0 : o.act;
       nd.w_off = off;
       off += (long long)o.cout * KH * KW * nd.cin_real;
       nd.b_off = off;
       off += o.cout;
-      nd.ldb = pad8(KH * KW * X.C);  // 16-byte aligned shadow rows (4-channel stems: 49*4 -> 200)
+      nd.ldb = pad8(KH * KW * X.C / nd.groups);  // 16-byte aligned shadow rows (4-channel stems: 49*4 -> 200)
       nd.fp32_out = !proj && (i + 1 < ops.size() && ops[i + 1].kind == ADAINF_OP_DET_HEAD);
       TensorRt Y;
       Y.H = nd.g.Ho;
@@ -109,14 +115,15 @@ void Model::build(const adainf_model_spec& s) {
       Y.act = nd.act;
       Y.stage = stage;
       Y.f32 = nd.fp32_out;
-      T.push_back(Y);
+      T.push_back(std::move(Y));
       nd.out = (int)T.size() - 1;
       if (!proj && o.residual) {
         if (blocks.empty()) throw InvalidError("residual conv without an open block");
         nd.res = blocks.back();
         blocks.pop_back();
         const TensorRt& R = T[nd.res];
-        if (R.H != Y.H || R.W != Y.W || R.C != Y.C) throw ShapeError("residual shape mismatch");
+        const TensorRt& Yo = T[nd.out];
+        if (R.H != Yo.H || R.W != Yo.W || R.C != Yo.C) throw ShapeError("residual shape mismatch");
         if (R.stage != stage) throw InvalidError("a residual block may not span an exit");
       }
       const int ni = (int)nodes.size();
@@ -159,7 +166,7 @@ void Model::build(const adainf_model_spec& s) {
       Y.producer = (int)nodes.size();
       Y.act = 0;
       Y.stage = stage;
-      T.push_back(Y);
+      T.push_back(std::move(Y));
       nd.out = (int)T.size() - 1;
       if (T[cur].primary >= 0) throw InvalidError("tensor consumed twice on the main path");
       T[cur].primary = (int)nodes.size();
@@ -176,7 +183,7 @@ void Model::build(const adainf_model_spec& s) {
       e.stage = stage;
       e.lw = o.loss_weight;
       const int C = T[cur].C;
-      if (C % 8 || (256 % (C / 8)) || C / 8 > 256) throw ShapeError("exit: channels must be 8 * power of two");
+      if (C % 8 || C / 8 > 1024) throw ShapeError("exit: channels must be a multiple of 8, <= 8192");
       e.w_off = off;
       off += (long long)C * o.num_classes;
       e.b_off = off;
@@ -229,6 +236,19 @@ void Model::build(const adainf_model_spec& s) {
       pack = true;
     }
   }
+  // first conv (3x3/1, <= 3 real input channels, 16 outputs) whose only consumer is a 2x2/2 max-pool: fused in
+  // inference (the TinyYOLOv3-like detector's 416x416 layer)
+  fused_pool0 = -1;
+  if (!stem_s2d && !nodes.empty() && nodes[0].kind == N_CONV && nodes[0].in == 0 && nodes[0].groups == 1 &&
+      getenv("ADAINF_CONVPOOL") == nullptr) {
+    const NodeRt& c0 = nodes[0];
+    const TensorRt& Y = T[c0.out];
+    const int po = Y.primary;
+    if (po >= 0 && nodes[po].kind == N_POOL && nodes[po].stage == c0.stage && !c0.fp32_out && c0.res < 0 &&
+        Y.exit_k < 0 && Y.res_of < 0 && Y.proj < 0 &&
+        conv_first_pool_ok(c0.g, c0.cin_real, nodes[po].pk, nodes[po].ps, nodes[po].pp))
+      fused_pool0 = po;
+  }
 
   CK(cudaSetDevice(device));
   // activations
@@ -246,6 +266,7 @@ void Model::build(const adainf_model_spec& s) {
     if (nd.kind != N_POOL) {
       nd.shadow.alloc((size_t)nd.g.Cout * nd.ldb * 2);
       nd.shadow.zero();
+      if (nd.groups > 1) nd.wdw.alloc((size_t)nd.g.KH * nd.g.KW * nd.g.Cin * 2);
     }
   if (stem_s2d) stem_wprep.alloc(16 * 2 * 64 * 8 * 2);
   for (size_t k = 0; k + 1 < exits.size(); ++k) {  // dense survivor copies of the stage-boundary tensors
@@ -287,7 +308,7 @@ void Model::build(const adainf_model_spec& s) {
     if (pr.second >= 0) {
       NodeRt& nd = nodes[pr.second];
       add_seg(nd.w_off, (long long)nd.g.Cout * nd.g.KH * nd.g.KW * nd.cin_real, nd.shadow.as<bf16>(),
-              nd.g.KH * nd.g.KW, nd.cin_real, nd.g.Cin, nd.ldb);
+              nd.g.KH * nd.g.KW, nd.cin_real, nd.g.Cin / nd.groups, nd.ldb);
       add_seg(nd.b_off, nd.g.Cout, nullptr, 0, 0, 0, 0);
     } else {
       ExitRt& e = exits[-1 - pr.second];
@@ -366,7 +387,7 @@ void Model::ensure_training() {
   }
   size_t ws = 0;
   for (auto& nd : nodes)
-    if (nd.kind == N_CONV && nd.in != 0 && dgrad_sp_ok(nd.g)) {
+    if (nd.kind == N_CONV && nd.in != 0 && nd.groups == 1 && dgrad_sp_ok(nd.g)) {
       nd.sp = true;
       nd.wsp.alloc(dgrad_sp_ws_bytes(nd.g));
     }
@@ -374,7 +395,7 @@ void Model::ensure_training() {
     if (nd.kind == N_POOL) {
       nd.argmax.alloc((size_t)max_batch * T[nd.out].row_elems());
     } else {
-      ws = std::max(ws, ::adainf::wgrad_ws_bytes(nd.g, max_batch));
+      ws = std::max(ws, nd.groups > 1 ? dw_wgrad_ws_bytes(nd.g, max_batch) : ::adainf::wgrad_ws_bytes(nd.g, max_batch));
       if (stem_s2d && &nd == &nodes[0]) ws = std::max(ws, stem_wgrad_ws_bytes(max_batch));
       if (nd.kind == N_PROJ && nd.in != 0) {
         for (const auto& c : nodes)
@@ -436,11 +457,53 @@ void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, in
                  T[pl.out].buf, train ? pl.argmax.as<uint8_t>() : nullptr, st);
         continue;
       }
+      if (!train && ni == 0 && nd.kind == N_CONV && fused_pool0 >= 0) {
+        // first conv + its 2x2 max-pool in one kernel (inference only: training keeps the pre-pool tensor)
+        const NodeRt& pl = nodes[fused_pool0];
+        ConvPoolArgs cp{};
+        cp.x = buf_of(0);
+        cp.count = c;
+        cp.n_static = n_static;
+        cp.H = nd.g.H;
+        cp.W = nd.g.W;
+        cp.cin_real = nd.cin_real;
+        cp.cin_pad = nd.g.Cin;
+        cp.shadow = nd.shadow.as<bf16>();
+        cp.ldb = nd.ldb;
+        cp.bias = params.as<float>() + nd.b_off;
+        cp.act = nd.act;
+        cp.y = T[pl.out].buf;
+        conv_first_pool(cp, st);
+        continue;
+      }
       if (nd.kind == N_POOL) {
         if (stem_s2d && ni == stem_pool) continue;  // produced by the fused stem
+        if (!train && ni == fused_pool0) continue;  // produced by the fused first conv
         launch_maxpool_fwd(buf_of(nd.in), map_for(nd.in, ns), c, n_static, nd.g.H, nd.g.W, nd.g.Cin, nd.pk, nd.ps,
                            nd.pp, nd.g.Ho, nd.g.Wo, T[nd.out].buf, train ? nd.argmax.as<uint8_t>() : nullptr,
                            nd.in > 0 && T[nd.in].act == 1, st);
+      } else if (nd.groups > 1) {
+        if (nd.res >= 0) throw UnsupportedError("depthwise conv closing a residual block");
+        dw_prep(nd.shadow.as<bf16>(), nd.ldb, nd.g.Cin, nd.g.KH * nd.g.KW, nd.wdw.as<bf16>(), st);
+        DwArgs d{};
+        d.x = buf_of(nd.in);
+        d.map = map_for(nd.in, ns);
+        d.count = c;
+        d.n_static = n_static;
+        d.H = nd.g.H;
+        d.W = nd.g.W;
+        d.C = nd.g.Cin;
+        d.Ho = nd.g.Ho;
+        d.Wo = nd.g.Wo;
+        d.KH = nd.g.KH;
+        d.KW = nd.g.KW;
+        d.s = nd.g.stride;
+        d.p = nd.g.pad;
+        d.w = nd.wdw.as<bf16>();
+        d.bias = params.as<float>() + nd.b_off;
+        d.act = nd.act;
+        d.y = T[nd.out].buf;
+        dw_fwd(d, st);
       } else {
         const float* bias = params.as<float>() + nd.b_off;
         const bf16* res = nd.res >= 0 ? buf_of(nd.res) : nullptr;
@@ -623,6 +686,35 @@ void Model::train_grad_impl(const bf16* x, const int32_t* row_map, const int32_t
         stem_wgrad(buf_of(0), dz, n, in_h / 2, in_w / 2, nd.cin_real, wgrad_ws.as<float>(), wgrad_ws_bytes,
                    G + nd.w_off, G + nd.b_off, st);
       }
+      return;
+    }
+    if (nd.groups > 1) {  // depthwise: weight / bias gradient, then the input gradient (dwconv.cu)
+      DwArgs d{};
+      d.x = buf_of(nd.in);
+      d.dz = dz;
+      d.n_static = n;
+      d.H = nd.g.H;
+      d.W = nd.g.W;
+      d.C = nd.g.Cin;
+      d.Ho = nd.g.Ho;
+      d.Wo = nd.g.Wo;
+      d.KH = nd.g.KH;
+      d.KW = nd.g.KW;
+      d.s = nd.g.stride;
+      d.p = nd.g.pad;
+      dw_wgrad(d, wgrad_ws.as<float>(), wgrad_ws_bytes, G + nd.w_off, G + nd.b_off, st);
+      if (nd.in == 0) return;
+      const TensorRt& X = T[nd.in];
+      const int prod = X.producer;
+      const int mask = (prod >= 0 && nodes[prod].kind == N_CONV) ? X.act : 0;
+      d.x = dz;
+      d.w = nd.wdw.as<bf16>();
+      d.bcast = bcast_of(nd.in);
+      d.sc = sc_of(nd.in);
+      d.yact = mask ? X.buf : nullptr;
+      d.mask_act = mask;
+      d.y = T[nd.in].grad;
+      dw_dgrad(d, st);
       return;
     }
     conv_wgrad(nd.g, buf_of(nd.in), dz, n, nd.cin_real, wgrad_ws.as<float>(), wgrad_ws_bytes, G + nd.w_off,

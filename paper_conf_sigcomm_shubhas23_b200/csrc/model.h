@@ -24,6 +24,15 @@ enum NodeKind { N_CONV = 0, N_POOL = 1, N_PROJ = 2 };
 struct DevBuf {  // owning device allocation
   void* p = nullptr;
   size_t bytes = 0;
+  DevBuf() = default;
+  DevBuf(const DevBuf&) = delete;  // owning: a copy would free the allocation twice
+  DevBuf& operator=(const DevBuf&) = delete;
+  DevBuf(DevBuf&& o) noexcept : p(o.p), bytes(o.bytes) { o.p = nullptr; o.bytes = 0; }
+  DevBuf& operator=(DevBuf&& o) noexcept {
+    std::swap(p, o.p);
+    std::swap(bytes, o.bytes);
+    return *this;
+  }
   void alloc(size_t b);
   void zero(cudaStream_t st = 0);
   ~DevBuf();
@@ -56,7 +65,9 @@ struct NodeRt {
   int stage;
   ConvGeom g{};
   int act = 0;
-  int cin_real = 0;
+  int cin_real = 0;            // input channels per group of the weights (first layer: the unpadded in_c)
+  int groups = 1;              // > 1: depthwise (groups == Cin == Cout), dwconv.cu
+  DevBuf wdw;                  // depthwise weights [taps][C] bf16, rebuilt from the shadow every forward
   long long w_off = 0, b_off = 0;
   int ldb = 0;
   DevBuf shadow;  // bf16 [Cout][ldb]
@@ -107,6 +118,7 @@ struct Model {
   bool stem_s2d = false;
   int stem_pool = -1;         // node index of the pool fused into the stem
   DevBuf stem_wprep;          // per-tap bf16 weights [16][2][64][8], rebuilt from the shadow every forward
+  int fused_pool0 = -1;       // inference: node index of the 2x2 pool fused into the first conv (convpool.cu)
   // inference stage bookkeeping
   DevBuf pos, orig, counts, alive;  // pos/orig: [nstages][max_batch] int; counts [nstages] int
   DevBuf exit_ws;                   // fused exit kernel: ticket + look-back status words

@@ -35,6 +35,7 @@ enum ProfClass {
   PC_SURVIVOR_GATHER,
   PC_EXIT_HEAD_TRAIN,
   PC_VERSION_AVG,
+  PC_DW,
   PROF_NCLASS
 };
 

@@ -151,6 +151,27 @@ def init_params(spec: dict, seed: int = 0, exit_scale: float = 4.0) -> np.ndarra
     return p
 
 
+def spread_exit_heads(spec: dict, params: np.ndarray, logits: np.ndarray, target_std: float = 2.0) -> np.ndarray:
+    """Rescale each exit head's weights so its logits (without bias) spread with std ~`target_std` over the
+    batch.  Deep BN-free nets with ReLU6 (MobileNetV2) give pooled features whose per-sample variation is tiny
+    next to their common part, so the x`exit_scale` init leaves every confidence within ~1e-2 of 1/C and most
+    rows inside the 1e-3 decision band; the head is linear in W, so one rescale (plus a bias that cancels the
+    scaled batch-mean logits) fixes the spread.
+    logits: [B, E, ncls] from a forward pass with `params` (input recipe only)."""
+    p = params.copy()
+    ex = [s for s in S.param_segments(spec) if s[0] in ("exit_w", "exit_b")]
+    for k in range(len(ex) // 2):
+        _, _, woff, wshp = ex[2 * k]
+        _, _, boff, bshp = ex[2 * k + 1]
+        lin = logits[:, k, :] - p[boff:boff + bshp[0]][None, :]
+        sd = float(lin.std(axis=0).mean())
+        if sd > 0:  # scale the per-sample part; the bias cancels the scaled common part (batch mean)
+            sc = np.float32(target_std / sd)
+            p[woff:woff + int(np.prod(wshp))] *= sc
+            p[boff:boff + bshp[0]] -= (sc * lin.mean(axis=0)).astype(np.float32)
+    return p
+
+
 def det_head_params(spec: dict, params: np.ndarray, obj_bias: float, seed: int = 0,
                     head_scale: float = 16.0, cls_bias=None) -> np.ndarray:
     """Bias the detector's final 1x1 conv so the objectness logits sit near `obj_bias` (controls the

@@ -44,23 +44,43 @@ def gpu_infer_single(spec, params, xb, taus, max_batch=None):
     return res
 
 
-def banded_rows(conf_all, taus, exit_oracle):
-    """rows whose confidence at any exit k <= e_oracle (k < E-1) lies within BAND of tau_k"""
+def banded_rows(conf_all, taus, exit_oracle, band_width=BAND):
+    """rows whose confidence at any exit k <= e_oracle (k < E-1) lies within the band (BAND, or a per-exit
+    array) of tau_k"""
     Bn, E = conf_all.shape
+    bw = np.broadcast_to(np.asarray(band_width, np.float64), (E - 1,)) if E > 1 else []
     band = np.zeros(Bn, bool)
     for k in range(E - 1):
-        band |= (np.abs(conf_all[:, k] - taus[k]) < BAND) & (exit_oracle >= k)
+        band |= (np.abs(conf_all[:, k] - taus[k]) < bw[k]) & (exit_oracle >= k)
     return band
 
 
-def check_infer_parity(orc, gpu, taus, conf_atol=2e-3):
+def oracle_sensitivity(spec, params, xb, n_flips=20, seed=0):
+    """How far the ORACLE moves when n_flips random input elements change by one bf16 ulp: per exit, the max
+    |dconf| and the max per-row relative logit change.  Deep BN-folded bf16 nets (MobileNetV2-EE) amplify a single
+    rounding flip to ~1e-2 of the deep exits' logits (reading Q28), so there the GPU (whose fp32
+    accumulation order flips a few bf16 roundings) is held to the oracle's own conditioning instead of 1e-3 / 2e-2."""
+    rng = np.random.default_rng(seed)
+    x2 = xb.copy().view(np.uint16)
+    idx = rng.choice(x2.size, n_flips, replace=False)
+    x2.reshape(-1)[idx] ^= 1
+    m = O.Model(spec)
+    a = m.forward(params, synth.bf16_bits_to_f32(xb))
+    b = m.forward(params, synth.bf16_bits_to_f32(x2.view(xb.dtype)))
+    E = a["conf"].shape[1]
+    dconf = np.abs(a["conf"] - b["conf"]).max(axis=0)
+    dlog = np.array([max(rel(b["logits"][n, k], a["logits"][n, k]) for n in range(xb.shape[0])) for k in range(E)])
+    return dconf, dlog
+
+
+def check_infer_parity(orc, gpu, taus, conf_atol=2e-3, band_width=BAND, logit_tol=2e-2):
     """exit ids, survivor lists, counts bit-exact outside the band; logits rel 2e-2; confidences within conf_atol
     (what the kernels achieve: max |dconf| 6e-4 at the decision exits and 1.3e-3 at the final exit of 224x224
     ResNet-18-EE; reduced geometries drift more, up to ~6e-3 at 64x64, tests/test_gpu_decisions.py)."""
     conf_all = orc["conf"]
     E = conf_all.shape[1]
     eid, surv, counts = O.exit_assign(conf_all, taus)
-    band = banded_rows(conf_all, taus, eid)
+    band = banded_rows(conf_all, taus, eid, band_width)
     ok = ~band
     assert (gpu["exit_id"][ok] == eid[ok]).all(), np.nonzero((gpu["exit_id"] != eid) & ok)
     if not band.any():
@@ -76,8 +96,9 @@ def check_infer_parity(orc, gpu, taus, conf_atol=2e-3):
     rows = np.nonzero(ok)[0]
     ex = eid[rows]
     ref_logits = orc["logits"][rows, ex, :]
+    ltol = np.broadcast_to(np.asarray(logit_tol, np.float64), (E,))
     for i, r in enumerate(rows):
-        assert rel(gpu["logits"][r], ref_logits[i]) <= 2e-2, (r, gpu["logits"][r], ref_logits[i])
+        assert rel(gpu["logits"][r], ref_logits[i]) <= ltol[ex[i]], (r, gpu["logits"][r], ref_logits[i])
     np.testing.assert_allclose(gpu["conf"][rows], conf_all[rows, ex], atol=conf_atol)
     # argmax equal where the top-2 oracle logits are separated
     srt = np.sort(ref_logits, axis=1)
@@ -95,3 +116,61 @@ def check_grads(spec, g_gpu, g_orc, tol=2e-2):
         worst = max(worst, r)
         assert r <= tol, (kind, i, r)
     return worst
+
+
+def bn_folded_params(spec, params, xf, gamma_act=1.0, beta_act=1.0, gamma_lin=0.7):
+    """Input recipe for deep BN-free nets (MobileNetV2-EE): the paper's models carry BatchNorm,
+    folded into each conv at create time (reading Q10).  Emulate a BN-folded network by choosing every conv's
+    scale and bias so its pre-activation output has per-channel mean beta / std gamma over this batch (batch
+    statistics, computed once in plain fp32 torch here, test side): W <- W * gamma / sd, b <- beta - mean * gamma / sd.
+    Without it the random ReLU6 stack collapses every sample onto nearly the same pooled features and the
+    exits' confidences bunch within 1e-2 of 1/C.  Linear (act 0) convs get beta 0, gamma `gamma_lin`.
+    xf: [B, H, W, C] float images.  Returns a new flat parameter vector (an input to both sides)."""
+    import torch
+    import torch.nn.functional as F
+    from paper_conf_sigcomm_shubhas23_b200 import specs as S
+    p = params.copy()
+    segs = {(k, i): (off, shp) for k, i, off, shp in S.param_segments(spec)}
+
+    def view(kind, i):
+        off, shp = segs[(kind, i)]
+        return off, shp
+
+    cur = torch.from_numpy(np.ascontiguousarray(xf)).float().permute(0, 3, 1, 2)
+    blocks = []
+    for i, o in enumerate(spec["ops"]):
+        k = o["kind"]
+        if k == "conv":
+            woff, wshp = view("conv_w", i)
+            boff, _ = view("conv_b", i)
+            cnt = int(np.prod(wshp))
+            w = torch.from_numpy(p[woff:woff + cnt].reshape(wshp)).permute(0, 3, 1, 2)
+            z = F.conv2d(cur, w, stride=o["stride"], padding=o["pad"], groups=o.get("groups", 1))
+            mean = z.mean(dim=(0, 2, 3))
+            sd = z.std(dim=(0, 2, 3)).clamp_min(1e-6)
+            act = o["act"] != 0
+            g, b = (gamma_act, beta_act) if act else (gamma_lin, 0.0)
+            scale = (g / sd).numpy().astype(np.float32)
+            p[woff:woff + cnt] = (p[woff:woff + cnt].reshape(wshp) * scale[:, None, None, None]).reshape(-1)
+            p[boff:boff + wshp[0]] = (b - mean.numpy() * scale).astype(np.float32)
+            v = (z - mean[None, :, None, None]) * torch.from_numpy(scale)[None, :, None, None] + b
+            if o["residual"]:
+                v = v + blocks.pop()
+            if o["act"] == 1:
+                v = torch.relu(v)
+            elif o["act"] == 3:
+                v = v.clamp(0.0, 6.0)
+            elif o["act"] == 2:
+                v = torch.where(v > 0, v, 0.1 * v)
+            cur = v
+        elif k == "maxpool":
+            cur = F.max_pool2d(cur, o["kh"], o["stride"], o["pad"])
+        elif k == "block":
+            if o["cout"] > 0:
+                woff, wshp = view("proj_w", i)
+                w = torch.from_numpy(p[woff:woff + int(np.prod(wshp))].reshape(wshp)).permute(0, 3, 1, 2)
+                blocks.append(F.conv2d(cur, w, stride=o["stride"]) + torch.from_numpy(
+                    p[view("proj_b", i)[0]:view("proj_b", i)[0] + wshp[0]])[None, :, None, None])
+            else:
+                blocks.append(cur)
+    return p

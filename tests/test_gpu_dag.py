@@ -86,9 +86,10 @@ def test_video_dag_detector_routing_crops():
         c = cand_id(r)
         if c in omap and not band[c]:
             o = omap[c]
-            assert abs(r[4] - o[4]) < 2e-3
-            # boxes are exp / sigmoid transforms of the head logits: held to the north_star logit tolerance (2e-2
-            # relative, + 0.5 px), reading Q20 as amended in DESIGN.md (the detector's spread logits drift ~6e-3)
+            # scores and boxes are sigmoid / exp transforms of the head logits: held to the north_star logit
+            # tolerance (2e-2 relative; boxes + 0.5 px), reading Q20 as amended in DESIGN.md (the detector's spread
+            # logits drift ~6e-3, and the inference-only fused first conv + pool accumulates its 27 taps in fp32)
+            assert abs(r[4] - o[4]) <= 2e-2 * o[4], (r[4], o[4])
             size = max(o[7] - o[5], o[8] - o[6], 1.0)
             assert np.all(np.abs(r[5:] - o[5:]) <= 0.5 + 2e-2 * size), (r, o)
     # routing: per class, ascending detection numbers; counts = detections of that class

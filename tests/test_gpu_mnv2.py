@@ -1,0 +1,131 @@
+"""NEXT-3 on the GPU: MobileNetV2-EE (the paper's video-DAG classifier family) through the C-ABI — ReLU6,
+1x1 expansion / linear projection GEMMs on the tensor cores, 3x3 depthwise convs (dwconv.cu, stride 1 and 2),
+identity inverted-residual shortcuts, early exits — against the oracle: exit decisions outside the 1e-3 band,
+logits within 2e-2, and one incremental-retraining step (gradients within 2e-2 per tensor, weights within 1e-3) on
+a shallow well-conditioned stack; the full 52-conv network at the oracle's own conditioning (reading Q28)."""
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+from paper_conf_sigcomm_shubhas23_b200 import binding as B
+from paper_conf_sigcomm_shubhas23_b200 import specs as S
+from paper_conf_sigcomm_shubhas23_b200 import synth
+
+from parity import bn_folded_params, check_grads, oracle_sensitivity, check_infer_parity, gpu_infer_single, images, rel, to_cuda_bf16
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.parametrize("hw,width,Bn", [(64, 0.5, 24), (96, 1.0, 12)])
+def test_mobilenetv2_ee_inference(hw, width, Bn):
+    spec = S.mobilenetv2_ee(in_hw=hw, width=width)
+    p = synth.init_params(spec, seed=71)
+    xb, _, xf = images(spec, Bn, 71)
+    p = bn_folded_params(spec, p, xf)
+    p = synth.spread_exit_heads(spec, p, O.Model(spec).forward(p, xf)["logits"])
+    orc = O.Model(spec).forward(p, xf)
+    taus = synth.calibrate_thresholds(orc["conf"], [0.25, 0.25, 0.25])
+    # tolerances: the north_star ones (band 1e-3, logits 2e-2), widened per exit to twice the oracle's own
+    # response to 20 one-ulp input flips where that is larger (reading Q28)
+    sconf, slog = oracle_sensitivity(spec, p, xb)
+    band = np.maximum(1e-3, 2 * sconf[:-1])
+    ltol = np.maximum(2e-2, 2 * slog)
+    gpu = gpu_infer_single(spec, p, xb, taus)
+    nb = check_infer_parity(orc, gpu, taus, conf_atol=max(2e-3, 2 * float(sconf.max())), band_width=band,
+                            logit_tol=ltol)
+    assert nb <= Bn // 2
+    assert rel(gpu["embed"], orc["pooled0"]) <= 2e-2
+    # every exit on its own (tau_k = 0 truncates there), all rows: logits within the same per-exit bound
+    E = orc["conf"].shape[1]
+    for k in range(E):
+        t = [2.0] * (E - 1)
+        if k < E - 1:
+            t[k] = 0.0
+        g2 = gpu_infer_single(spec, p, xb, t)
+        assert (g2["exit_id"] == k).all()
+        for r in range(Bn):
+            assert rel(g2["logits"][r], orc["logits"][r, k]) <= ltol[k], (k, r)
+
+
+def mnv2_blocks_spec(hw=64):
+    """Shallow MobileNetV2 pieces (well conditioned, so the north_star tolerances apply unchanged): ReLU6 3x3/2
+    stem, depthwise 3x3 stride 1 and 2 (96 channels: 12 vectors of 8 per pixel), 1x1 expansion and linear
+    projection GEMMs, an identity inverted-residual shortcut, two exits."""
+    ops = [S.conv(3, 32, stride=2, act=S.RELU6), S.conv(3, 32, act=S.RELU6, groups=32), S.conv(1, 16, act=S.NONE),
+           S.block(0), S.conv(1, 96, act=S.RELU6), S.conv(3, 96, act=S.RELU6, groups=96),
+           S.conv(1, 16, act=S.NONE, residual=True), S.exit_(10), S.conv(1, 96, act=S.RELU6),
+           S.conv(3, 96, stride=2, act=S.RELU6, groups=96), S.conv(1, 24, act=S.NONE), S.exit_(10)]
+    return {"name": "mnv2_blocks", "in_h": hw, "in_w": hw, "in_c": 3, "ops": ops}
+
+
+def _retrain(spec, n, seed):
+    p = synth.init_params(spec, seed=seed)
+    xb, y, xf = images(spec, n, seed)
+    p = bn_folded_params(spec, p, xf)
+    p = synth.spread_exit_heads(spec, p, O.Model(spec).forward(p, xf)["logits"])
+    p1, _, g_o, loss_o = O.Model(spec).retrain_step(p, np.zeros_like(p), xf, y, lr=0.01, mu=0.9)
+    m = B.Model(spec, n, params=p, momentum=0.9)
+    st = torch.zeros(2, dtype=torch.float32, device="cuda")
+    m.retrain_step(to_cuda_bf16(xb), torch.from_numpy(y).cuda(), lr=0.01, stats=st)
+    torch.cuda.synchronize()
+    out = dict(p=p, p1=p1, g_o=g_o, loss_o=loss_o, g=m.get_grads(), pg=m.get_params(), loss=float(st[0].item()),
+               xb=xb, y=y)
+    m.close()
+    return out
+
+
+def test_mobilenetv2_blocks_retrain_step():
+    """depthwise fwd / dgrad / wgrad, ReLU6 masks and the inverted-residual shortcut at the north_star
+    tolerances: gradients 2e-2 per tensor, updated weights 1e-3, loss 2e-2"""
+    spec = mnv2_blocks_spec()
+    r = _retrain(spec, 32, 73)
+    check_grads(spec, r["g"], r["g_o"])
+    assert rel(r["pg"], r["p1"]) <= 1e-3
+    assert rel(r["pg"] - r["p"], r["p1"] - r["p"]) <= 2e-2
+    assert abs(r["loss"] - r["loss_o"]) <= 2e-2 * abs(r["loss_o"])
+
+
+def test_mobilenetv2_blocks_inference():
+    spec = mnv2_blocks_spec()
+    Bn = 48
+    p = synth.init_params(spec, seed=74)
+    xb, _, xf = images(spec, Bn, 74)
+    p = bn_folded_params(spec, p, xf)
+    p = synth.spread_exit_heads(spec, p, O.Model(spec).forward(p, xf)["logits"])
+    orc = O.Model(spec).forward(p, xf)
+    taus = synth.calibrate_thresholds(orc["conf"], [0.5])
+    gpu = gpu_infer_single(spec, p, xb, taus)
+    nb = check_infer_parity(orc, gpu, taus)
+    assert nb <= 2
+
+
+def test_mobilenetv2_ee_retrain_step():
+    """Full MobileNetV2-EE (52 convs): bf16 storage makes its gradients ill-conditioned (the oracle itself moves
+    ~5-15% per tensor under 20 one-ulp input flips and sits ~25% from the exact fp64 gradient), so each tensor
+    is held to max(2e-2, 3 x the oracle's own spread over two such draws) (reading Q28); updated weights 1e-3."""
+    spec = S.mobilenetv2_ee(in_hw=64, width=0.5)
+    r = _retrain(spec, 16, 72)
+    m_o = O.Model(spec)
+    sens = np.zeros_like(r["g_o"])
+    for d in range(2):
+        rng = np.random.default_rng(d)
+        x2 = r["xb"].copy().view(np.uint16)
+        x2.reshape(-1)[rng.choice(x2.size, 20, replace=False)] ^= 1
+        _, _, g_s, _ = m_o.retrain_step(r["p"], np.zeros_like(r["p"]), synth.bf16_bits_to_f32(x2.view(r["xb"].dtype)),
+                                        r["y"], lr=0.01, mu=0.9)
+        sens = np.maximum(sens, np.abs(g_s - r["g_o"]))
+    for kind, i, off, shp in S.param_segments(spec):
+        sl = slice(off, off + int(np.prod(shp)))
+        tol = max(2e-2, 3 * float(np.linalg.norm(sens[sl]) / max(np.linalg.norm(r["g_o"][sl]), 1e-30)))
+        assert rel(r["g"][sl], r["g_o"][sl]) <= tol, (kind, i, rel(r["g"][sl], r["g_o"][sl]), tol)
+    assert rel(r["pg"], r["p1"]) <= 1e-3
+    assert abs(r["loss"] - r["loss_o"]) <= 2e-2 * abs(r["loss_o"])
+
+
+def test_grouped_conv_other_than_depthwise_is_unsupported():
+    spec = {"name": "g", "in_h": 16, "in_w": 16, "in_c": 3,
+            "ops": [S.conv(3, 16), S.conv(3, 16, groups=4), S.exit_(4)]}
+    with pytest.raises(B.AdaInfError) as ei:
+        B.Model(spec, 4)
+    assert ei.value.code == B.ERR_UNSUPPORTED
