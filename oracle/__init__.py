@@ -25,8 +25,9 @@ _SRC = os.path.join(_HERE, "oracle.cpp")
 _lock = threading.Lock()
 _lib = None
 
-OR_CONV, OR_MAXPOOL, OR_BLOCK, OR_EXIT, OR_DET_HEAD = 0, 1, 2, 3, 4
-_KIND = {"conv": OR_CONV, "maxpool": OR_MAXPOOL, "block": OR_BLOCK, "exit": OR_EXIT, "det_head": OR_DET_HEAD}
+OR_CONV, OR_MAXPOOL, OR_BLOCK, OR_EXIT, OR_DET_HEAD, OR_SHUFFLE = 0, 1, 2, 3, 4, 5
+_KIND = {"conv": OR_CONV, "maxpool": OR_MAXPOOL, "block": OR_BLOCK, "exit": OR_EXIT, "det_head": OR_DET_HEAD,
+         "shuffle": OR_SHUFFLE}
 
 
 class OrOp(C.Structure):
@@ -35,7 +36,7 @@ class OrOp(C.Structure):
         ("pad", C.c_int32), ("cout", C.c_int32), ("act", C.c_int32), ("residual", C.c_int32),
         ("num_classes", C.c_int32), ("loss_weight", C.c_float), ("anchors", C.c_int32),
         ("det_classes", C.c_int32), ("grid_stride", C.c_int32), ("anchor_wh", C.c_float * 16),
-        ("groups", C.c_int32),
+        ("groups", C.c_int32), ("pool", C.c_int32),
     ]
 
 
@@ -134,6 +135,7 @@ class Model:
             for j, v in enumerate(o.get("anchor_wh", [])):
                 r.anchor_wh[j] = v
             r.groups = int(o.get("groups", 1))
+            r.pool = int(o.get("pool", 0))
         self.m = OrModel(spec["in_h"], spec["in_w"], spec["in_c"], len(ops), self._ops)
         self.spec = spec
         L = lib()

@@ -171,7 +171,12 @@ Walk walk(const or_model* m) {
           if (blocks.empty()) w.ok = false;
           else {
             const Shape3 b = blocks.back();
-            if (b.H != o.H || b.W != o.W || b.C != o.C) w.ok = false;
+            if (op.residual == 2) {  // concat [shortcut, conv] (ShuffleNet stride-2 unit)
+              if (b.H != o.H || b.W != o.W) w.ok = false;
+              o.C = b.C + op.cout;
+            } else if (b.H != o.H || b.W != o.W || b.C != o.C) {
+              w.ok = false;
+            }
             blocks.pop_back();
           }
         }
@@ -192,10 +197,19 @@ Walk walk(const or_model* m) {
           w.nparams += (int64_t)op.cout * cur.C + op.cout;
           blocks.push_back(o);
           w.out_shape.push_back(o);
+        } else if (op.pool) {  // average-pool shortcut (ShuffleNet)
+          Shape3 o{(cur.H + 2 * op.pad - op.kh) / op.stride + 1, (cur.W + 2 * op.pad - op.kw) / op.stride + 1, cur.C};
+          blocks.push_back(o);
+          w.out_shape.push_back(o);
         } else {
           blocks.push_back(cur);
           w.out_shape.push_back(cur);
         }
+        break;
+      }
+      case OR_SHUFFLE: {
+        if (op.groups <= 0 || cur.C % op.groups) w.ok = false;
+        w.out_shape.push_back(cur);
         break;
       }
       case OR_EXIT: {
@@ -321,14 +335,28 @@ struct Engine {
           res = blocks.back();
           blocks.pop_back();
           const Tensor& S = T[res];
-          for (size_t e = 0; e < acc.size(); ++e) acc[e] = F(acc[e] + S.d[e]);  // "+ float(residual)"
+          if (op.residual == 1)
+            for (size_t e = 0; e < acc.size(); ++e) acc[e] = F(acc[e] + S.d[e]);  // "+ float(residual)"
         }
         // det-head input (act none, followed by DET_HEAD) stays fp32; everything else bf16
         const bool fp32_out = (i + 1 < m->n_ops && m->ops[i + 1].kind == OR_DET_HEAD);
-        Y.d.resize(acc.size());
-        for (size_t e = 0; e < acc.size(); ++e) {
-          const double v = F(act_f(op.act, acc[e], exact));
-          Y.d[e] = fp32_out ? v : R(v);
+        if (op.residual == 2) {
+          // concat along channels: [act(shortcut), act(conv)] (ShuffleNet: ReLU after the concat), bf16
+          const Tensor& S = T[res];
+          const int Cs = S.C, Co = op.cout;
+          Y.C = Cs + Co;
+          Y.d.resize((size_t)Y.H * Y.W * Y.C);
+          for (int e = 0; e < Y.H * Y.W; ++e) {
+            for (int c = 0; c < Cs; ++c) Y.d[(size_t)e * Y.C + c] = R(F(act_f(op.act, S.d[(size_t)e * Cs + c], exact)));
+            for (int c = 0; c < Co; ++c)
+              Y.d[(size_t)e * Y.C + Cs + c] = R(F(act_f(op.act, acc[(size_t)e * Co + c], exact)));
+          }
+        } else {
+          Y.d.resize(acc.size());
+          for (size_t e = 0; e < acc.size(); ++e) {
+            const double v = F(act_f(op.act, acc[e], exact));
+            Y.d[e] = fp32_out ? v : R(v);
+          }
         }
         T.push_back(std::move(Y));
         nodes.push_back({OR_CONV, i, cur, (int)T.size() - 1, res});
@@ -367,9 +395,48 @@ struct Engine {
           T.push_back(std::move(Y));
           nodes.push_back({OR_BLOCK, i, cur, (int)T.size() - 1, -1});
           blocks.push_back((int)T.size() - 1);
+        } else if (op.pool) {
+          // average-pool shortcut: fp64 sum of the window (zero padding), fp32, / (kh*kw) in fp32, bf16
+          const Tensor& X = T[cur];
+          Tensor Y;
+          Y.H = (X.H + 2 * op.pad - op.kh) / op.stride + 1;
+          Y.W = (X.W + 2 * op.pad - op.kw) / op.stride + 1;
+          Y.C = X.C;
+          Y.d.assign((size_t)Y.H * Y.W * Y.C, 0.0);
+          for (int ho = 0; ho < Y.H; ++ho)
+            for (int wo = 0; wo < Y.W; ++wo)
+              for (int c = 0; c < Y.C; ++c) {
+                double a = 0.0;
+                for (int kh = 0; kh < op.kh; ++kh)
+                  for (int kw = 0; kw < op.kw; ++kw) {
+                    const int ih = ho * op.stride - op.pad + kh, iw = wo * op.stride - op.pad + kw;
+                    if (ih < 0 || ih >= X.H || iw < 0 || iw >= X.W) continue;
+                    a += X.d[((size_t)ih * X.W + iw) * X.C + c];
+                  }
+                Y.d[((size_t)ho * Y.W + wo) * Y.C + c] = R(F(F(a) / (double)(op.kh * op.kw)));
+              }
+          T.push_back(std::move(Y));
+          nodes.push_back({OR_BLOCK, i, cur, (int)T.size() - 1, -1});
+          blocks.push_back((int)T.size() - 1);
         } else {
           blocks.push_back(cur);
         }
+      } else if (op.kind == OR_SHUFFLE) {
+        // channel shuffle: channel c = gi*(C/g) + j of the input moves to position j*g + gi (view (g, C/g),
+        // transpose, flatten); values unchanged
+        const Tensor& X = T[cur];
+        Tensor Y;
+        Y.H = X.H;
+        Y.W = X.W;
+        Y.C = X.C;
+        Y.d.assign(X.d.size(), 0.0);
+        const int g = op.groups, Cg = X.C / g;
+        for (int e = 0; e < X.H * X.W; ++e)
+          for (int gi = 0; gi < g; ++gi)
+            for (int j = 0; j < Cg; ++j) Y.d[(size_t)e * X.C + j * g + gi] = X.d[(size_t)e * X.C + gi * Cg + j];
+        T.push_back(std::move(Y));
+        nodes.push_back({OR_SHUFFLE, i, cur, (int)T.size() - 1, -1});
+        cur = (int)T.size() - 1;
       } else if (op.kind == OR_EXIT) {
         const Tensor& X = T[cur];
         const int ncls = op.num_classes;
@@ -475,14 +542,59 @@ struct Engine {
             }
         continue;
       }
+      if (nd.kind == OR_SHUFFLE) {  // a permutation: the gradient moves back unchanged
+        const vector<double> dT = total(nd.out);
+        ensure(prim[nd.in], nd.in);
+        const int g = op.groups, Cg = X.C / g;
+        for (int e = 0; e < X.H * X.W; ++e)
+          for (int gi = 0; gi < g; ++gi)
+            for (int j = 0; j < Cg; ++j) prim[nd.in][(size_t)e * X.C + gi * Cg + j] += dT[(size_t)e * X.C + j * g + gi];
+        continue;
+      }
+      if (nd.kind == OR_BLOCK && op.pool) {
+        // average-pool shortcut backward: each window's gradient / (kh*kw) to its in-range taps, summed in fp64,
+        // divided in fp32 and stored bf16, then added as the block input's shortcut term (like a projection's dgrad)
+        const vector<double> dS = total(nd.out);
+        vector<double> a(X.d.size(), 0.0);
+        for (int ho = 0; ho < Y.H; ++ho)
+          for (int wo = 0; wo < Y.W; ++wo)
+            for (int c = 0; c < Y.C; ++c)
+              for (int kh = 0; kh < op.kh; ++kh)
+                for (int kw = 0; kw < op.kw; ++kw) {
+                  const int ih = ho * op.stride - op.pad + kh, iw = wo * op.stride - op.pad + kw;
+                  if (ih < 0 || ih >= X.H || iw < 0 || iw >= X.W) continue;
+                  a[((size_t)ih * X.W + iw) * X.C + c] += dS[((size_t)ho * Y.W + wo) * Y.C + c];
+                }
+        if (nd.in != 0) {
+          ensure(sc[nd.in], nd.in);
+          for (size_t e = 0; e < a.size(); ++e)
+            sc[nd.in][e] = F(sc[nd.in][e] + R(F(F(a[e]) / (double)(op.kh * op.kw))));
+        }
+        continue;
+      }
       // CONV or BLOCK projection
       const int KH = nd.kind == OR_CONV ? op.kh : 1, KW = nd.kind == OR_CONV ? op.kw : 1;
-      const int s = op.stride, p = nd.kind == OR_CONV ? op.pad : 0, Co = Y.C, Ci = X.C;
+      const bool concat = nd.kind == OR_CONV && op.residual == 2;
+      const int Cs = concat ? T[nd.res].C : 0;  // concat: the conv's channels sit after the shortcut's
+      const int s = op.stride, p = nd.kind == OR_CONV ? op.pad : 0, Co = Y.C - Cs, Ci = X.C;
       const int act = nd.kind == OR_CONV ? op.act : 0;
       const int grp = (nd.kind == OR_CONV && op.groups > 0) ? op.groups : 1;
       const int Cg = Ci / grp, Cog = Co / grp;
-      vector<double> dZ = total(nd.out);
-      for (size_t e = 0; e < dZ.size(); ++e) dZ[e] = R(F(dZ[e] * act_d(act, Y.d[e])));
+      const vector<double> dY = total(nd.out);
+      vector<double> dZ((size_t)Y.H * Y.W * Co);
+      for (int e = 0; e < Y.H * Y.W; ++e)
+        for (int c = 0; c < Co; ++c) {
+          const size_t yi = (size_t)e * Y.C + Cs + c;
+          dZ[(size_t)e * Co + c] = R(F(dY[yi] * act_d(act, Y.d[yi])));
+        }
+      if (concat) {  // shortcut part: masked by the act of the stored concat output, bf16, into the shortcut tensor
+        ensure(sc[nd.res], nd.res);
+        for (int e = 0; e < Y.H * Y.W; ++e)
+          for (int c = 0; c < Cs; ++c) {
+            const size_t yi = (size_t)e * Y.C + c;
+            sc[nd.res][(size_t)e * Cs + c] = F(sc[nd.res][(size_t)e * Cs + c] + R(F(dY[yi] * act_d(act, Y.d[yi]))));
+          }
+      }
       const double* Wf = params + w.poff[nd.op];
       double* gW = g + w.poff[nd.op];
       double* gb = gW + (int64_t)Co * KH * KW * Cg;
@@ -519,7 +631,7 @@ struct Engine {
           for (size_t e = 0; e < dX.size(); ++e) prim[nd.in][e] += dX[e];
         }
       }
-      if (nd.kind == OR_CONV && nd.res >= 0) {  // residual add: dZ flows unchanged into the shortcut
+      if (nd.kind == OR_CONV && nd.res >= 0 && !concat) {  // residual add: dZ flows unchanged into the shortcut
         ensure(sc[nd.res], nd.res);
         for (size_t e = 0; e < dZ.size(); ++e) sc[nd.res][e] = F(sc[nd.res][e] + dZ[e]);
       }

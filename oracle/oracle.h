@@ -23,18 +23,23 @@ extern "C" {
 #endif
 
 /* Op kinds of the oracle's own model description (same meaning as the ABI's, declared separately). */
-enum { OR_CONV = 0, OR_MAXPOOL = 1, OR_BLOCK = 2, OR_EXIT = 3, OR_DET_HEAD = 4 };
+enum { OR_CONV = 0, OR_MAXPOOL = 1, OR_BLOCK = 2, OR_EXIT = 3, OR_DET_HEAD = 4, OR_SHUFFLE = 5 };
 
 typedef struct {
   int32_t kind;
   int32_t kh, kw, stride, pad, cout; /* CONV; MAXPOOL uses kh,kw,stride,pad; BLOCK: cout>0 -> 1x1 projection shortcut with `stride` */
   int32_t act;                       /* CONV: 0 none, 1 ReLU, 2 leaky-ReLU(0.1), 3 ReLU6 (MobileNetV2) */
-  int32_t residual;                  /* CONV: add the innermost open BLOCK's shortcut before act, closes the block */
+  int32_t residual;                  /* CONV: 1 = add the innermost open BLOCK's shortcut before act; 2 = concat
+                                        [shortcut, conv] along channels, act applied to both parts (ShuffleNet
+                                        stride-2 unit); either closes the block */
   int32_t num_classes;               /* EXIT */
   float loss_weight;                 /* EXIT */
   int32_t anchors, det_classes, grid_stride; /* DET_HEAD */
   float anchor_wh[16];               /* DET_HEAD: (w,h) per anchor, pixels */
-  int32_t groups;                    /* CONV: channel groups (1 dense, = Cin = Cout depthwise); 0 is read as 1 */
+  int32_t groups;                    /* CONV: channel groups (1 dense, = Cin = Cout depthwise); 0 is read as 1;
+                                        SHUFFLE: g of the channel shuffle (ShuffleNet: view (g, C/g) -> transpose) */
+  int32_t pool;                      /* BLOCK with cout == 0: 1 = shortcut is an average pool kh x kw / stride / pad
+                                        of the block input, zero padding counted in the divisor (ShuffleNet) */
 } or_op;
 
 typedef struct {

@@ -19,17 +19,60 @@ YOLO_ANCHORS = [81.0, 82.0, 135.0, 169.0, 344.0, 319.0]
 
 
 def conv(k, cout, stride=1, pad=None, act=RELU, residual=False, groups=1):
-    """groups > 1: grouped conv (groups == cin == cout: depthwise, MobileNetV2 / ShuffleNet, NEXT-3)"""
+    """groups > 1: grouped conv (groups == cin == cout: depthwise, MobileNetV2 / ShuffleNet, NEXT-3);
+    residual: True / 1 add the open block's shortcut, 2 concatenate it in front of this conv's channels"""
     return {"kind": "conv", "kh": k, "kw": k, "stride": stride, "pad": (k // 2) if pad is None else pad,
             "cout": cout, "act": act, "residual": int(residual), "groups": groups}
+
+
+SHUFFLE_G8_STAGES = [(384, 4), (768, 8), (1536, 4)]  # ShuffleNet 1x, g = 8: (output channels, units) per stage
+
+
+def shufflenet_ee(num_classes=10, in_hw=224, in_c=3, groups=8, width=1.0, exits_after=(0, 1)):
+    """ShuffleNet (v1) early-exit classifier (the paper's video-DAG classifier family; NEXT-3): 3x3/2 conv 24
+    + 3x3/2 max-pool, then per stage one stride-2 unit (3x3/2 average-pool shortcut concatenated with the branch)
+    and stride-1 units (identity shortcut added); a unit = grouped 1x1 conv (bottleneck = out/4, ReLU; the first
+    one of stage 2 dense) -> channel shuffle (g) -> 3x3 depthwise (stride, no act) -> grouped 1x1 conv (no act
+    before the join) -> ReLU after the add / concat.  Exits after the stages in exits_after + the final exit
+    (reading Q3)."""
+    def ch(c):
+        return max(8 * groups, int(round(c * width / (8 * groups))) * 8 * groups)
+    ops = [conv(3, 24, stride=2), maxpool(3, 2, 1)]
+    cin = 24
+    for si, (cout, n) in enumerate(SHUFFLE_G8_STAGES):
+        cout = ch(cout)
+        for u in range(n):
+            mid = cout // 4
+            g1 = 1 if (si == 0 and u == 0) else groups
+            if u == 0:
+                ops += [block(stride=2, pool=1), conv(1, mid, groups=g1), shuffle(groups),
+                        conv(3, mid, stride=2, act=NONE, groups=mid), conv(1, cout - cin, act=RELU, groups=groups,
+                                                                       residual=2)]
+            else:
+                ops += [block(0), conv(1, mid, groups=groups), shuffle(groups), conv(3, mid, act=NONE, groups=mid),
+                        conv(1, cout, act=RELU, groups=groups, residual=True)]
+            cin = cout
+        if si in exits_after:
+            ops.append(exit_(num_classes))
+    ops.append(exit_(num_classes))
+    return {"name": "shufflenet_ee", "in_h": in_hw, "in_w": in_hw, "in_c": in_c, "ops": ops}
 
 
 def maxpool(k, stride, pad=0):
     return {"kind": "maxpool", "kh": k, "kw": k, "stride": stride, "pad": pad}
 
 
-def block(cout=0, stride=1):
+def block(cout=0, stride=1, pool=0, k=3, pad=1):
+    """cout > 0: 1x1 projection shortcut; pool = 1: k x k average-pool shortcut (stride, pad; zero padding counted,
+    ShuffleNet stride-2 unit); else identity"""
+    if pool:
+        return {"kind": "block", "cout": 0, "stride": stride, "pool": 1, "kh": k, "kw": k, "pad": pad}
     return {"kind": "block", "cout": cout, "stride": stride}
+
+
+def shuffle(groups):
+    """ShuffleNet channel shuffle (view (g, C/g) -> transpose -> flatten)"""
+    return {"kind": "shuffle", "groups": groups}
 
 
 def exit_(num_classes, loss_weight=1.0):
@@ -111,32 +154,52 @@ def tiny_yolo_det(in_hw=416, det_classes=2, anchors=3, width=512, nms_iou=0.0):
     return {"name": "tiny_yolo_det", "in_h": in_hw, "in_w": in_hw, "in_c": 3, "ops": ops}
 
 
-def num_params(spec) -> int:
-    """Parameter count from the documented flat layout (include/adainf.h)."""
+def _walk(spec):
+    """(op index, op, H, W, C of the tensor entering the op, H, W, C after it) along the op list; BLOCK reports its
+    shortcut's shape as the output.  A CONV with residual 2 concatenates the open block's shortcut channels."""
     H, W, Cc = spec["in_h"], spec["in_w"], spec["in_c"]
-    n = 0
-    for o in spec["ops"]:
+    blocks = []
+    for i, o in enumerate(spec["ops"]):
         k = o["kind"]
         if k == "conv":
-            n += o["cout"] * o["kh"] * o["kw"] * (Cc // o.get("groups", 1)) + o["cout"]
-            H = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
-            W = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
-            Cc = o["cout"]
+            Ho = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
+            Wo = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
+            Co = o["cout"]
+            if o.get("residual", 0):
+                sc = blocks.pop()
+                if o["residual"] == 2:
+                    Co += sc
+            yield i, o, H, W, Cc, Ho, Wo, Co
+            H, W, Cc = Ho, Wo, Co
         elif k == "maxpool":
-            H = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
-            W = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
-        elif k == "block" and o["cout"] > 0:
-            n += o["cout"] * Cc + o["cout"]
-        elif k == "exit":
-            n += Cc * o["num_classes"] + o["num_classes"]
-    return n
+            Ho = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
+            Wo = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
+            yield i, o, H, W, Cc, Ho, Wo, Cc
+            H, W = Ho, Wo
+        elif k == "block":
+            if o["cout"] > 0:
+                Ho, Wo, Co = (H - 1) // o["stride"] + 1, (W - 1) // o["stride"] + 1, o["cout"]
+            elif o.get("pool", 0):
+                Ho = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
+                Wo = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
+                Co = Cc
+            else:
+                Ho, Wo, Co = H, W, Cc
+            blocks.append(Co)
+            yield i, o, H, W, Cc, Ho, Wo, Co
+        else:
+            yield i, o, H, W, Cc, H, W, Cc
+
+
+def num_params(spec) -> int:
+    """Parameter count from the documented flat layout (include/adainf.h)."""
+    return sum(int(__import__("math").prod(shp)) for _k, _i, _o, shp in param_segments(spec))
 
 
 def param_segments(spec):
     """[(kind, op_index, offset, shape)] of the flat fp32 parameter vector, in layout order."""
-    H, W, Cc = spec["in_h"], spec["in_w"], spec["in_c"]
     segs, off = [], 0
-    for i, o in enumerate(spec["ops"]):
+    for i, o, _H, _W, Cc, _Ho, _Wo, _Co in _walk(spec):
         k = o["kind"]
         if k == "conv":
             shp = (o["cout"], o["kh"], o["kw"], Cc // o.get("groups", 1))
@@ -144,12 +207,6 @@ def param_segments(spec):
             off += o["cout"] * o["kh"] * o["kw"] * (Cc // o.get("groups", 1))
             segs.append(("conv_b", i, off, (o["cout"],)))
             off += o["cout"]
-            H = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
-            W = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
-            Cc = o["cout"]
-        elif k == "maxpool":
-            H = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
-            W = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
         elif k == "block" and o["cout"] > 0:
             segs.append(("proj_w", i, off, (o["cout"], 1, 1, Cc)))
             off += o["cout"] * Cc
@@ -165,21 +222,13 @@ def param_segments(spec):
 
 def macs_per_sample(spec):
     """Per-op forward MACs of one sample (conv + projection + exit FC), list aligned with ops."""
-    H, W, Cc = spec["in_h"], spec["in_w"], spec["in_c"]
     out = []
-    for o in spec["ops"]:
+    for _i, o, _H, _W, Cc, Ho, Wo, _Co in _walk(spec):
         k = o["kind"]
         m = 0
         if k == "conv":
-            Ho = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
-            Wo = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
             m = Ho * Wo * o["cout"] * o["kh"] * o["kw"] * (Cc // o.get("groups", 1))
-            H, W, Cc = Ho, Wo, o["cout"]
-        elif k == "maxpool":
-            H = (H + 2 * o["pad"] - o["kh"]) // o["stride"] + 1
-            W = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
         elif k == "block" and o["cout"] > 0:
-            Ho, Wo = (H - 1) // o["stride"] + 1, (W - 1) // o["stride"] + 1
             m = Ho * Wo * o["cout"] * Cc
         elif k == "exit":
             m = Cc * o["num_classes"]

@@ -83,7 +83,9 @@ def torch_forward(spec, params, x, exact, want_det=False):
             w = R(seg("conv_w", i).permute(0, 3, 1, 2))
             v = Fp(Fp(F.conv2d(cur, w, stride=o["stride"], padding=o["pad"], groups=o.get("groups", 1))) +
                    seg("conv_b", i)[None, :, None, None])
-            if o["residual"]:
+            if o["residual"] == 2:  # concat [shortcut, conv] (ShuffleNet stride-2 unit)
+                v = torch.cat([blocks.pop(), v], dim=1)
+            elif o["residual"]:
                 v = Fp(v + blocks.pop())
             v = GR(v)
             if o["act"] == 1:
@@ -98,8 +100,15 @@ def torch_forward(spec, params, x, exact, want_det=False):
             cur = Fp(v) if fp32_out else R(v)
         elif k == "maxpool":
             cur = GR(F.max_pool2d(cur, o["kh"], o["stride"], o["pad"]))
+        elif k == "shuffle":
+            n_, c_, h_, w_ = cur.shape
+            cur = cur.reshape(n_, o["groups"], c_ // o["groups"], h_, w_).transpose(1, 2).reshape(n_, c_, h_, w_)
         elif k == "block":
-            if o["cout"] > 0:
+            if o.get("pool", 0):  # average-pool shortcut: fp32 window sum, / (k*k) in fp32, bf16
+                kk = o["kh"] * o["kw"]
+                sm = Fp(F.avg_pool2d(GR(cur), o["kh"], o["stride"], o["pad"], count_include_pad=True) * kk)
+                blocks.append(R(Fp(sm / kk)))
+            elif o["cout"] > 0:
                 w = R(seg("proj_w", i).permute(0, 3, 1, 2))
                 blocks.append(R(Fp(Fp(F.conv2d(GR(cur), w, stride=o["stride"])) +
                                    seg("proj_b", i)[None, :, None, None])))
@@ -141,12 +150,24 @@ def mnv2_spec():
     return {"name": "mnv2", "in_h": 17, "in_w": 18, "in_c": 3, "ops": ops}
 
 
-SPECS = {"mini": mini_spec, "tiny": S.tiny_cnn_ee, "stem": stem_spec, "mnv2": mnv2_spec,
+def shuffle_spec():
+    """ShuffleNet pieces (NEXT-3): grouped 1x1 convs, channel shuffle, depthwise 3x3 without activation, the
+    stride-2 unit (3x3/2 average-pool shortcut concatenated in front of the branch, ReLU after the concat) and
+    the stride-1 unit (identity shortcut added), two exits."""
+    ops = [S.conv(3, 16, stride=2), S.maxpool(3, 2, 1), S.block(stride=2, pool=1), S.conv(1, 8, groups=1),
+           S.shuffle(4), S.conv(3, 8, stride=2, act=S.NONE, groups=8), S.conv(1, 16, groups=4, residual=2),
+           S.exit_(4), S.block(0), S.conv(1, 8, groups=4), S.shuffle(4), S.conv(3, 8, act=S.NONE, groups=8),
+           S.conv(1, 32, groups=4, residual=True), S.exit_(4)]
+    return {"name": "shuffle", "in_h": 24, "in_w": 26, "in_c": 3, "ops": ops}
+
+
+SPECS = {"mini": mini_spec, "shuffle": shuffle_spec, "shuffle_32": lambda: S.shufflenet_ee(in_hw=32), "tiny": S.tiny_cnn_ee, "stem": stem_spec, "mnv2": mnv2_spec,
          "mnv2_32": lambda: S.mobilenetv2_ee(in_hw=32, width=0.5),
          "resnet32": lambda: S.resnet18_ee(in_hw=32), "resnet64": lambda: S.resnet18_ee(in_hw=64)}
 
 
-@pytest.mark.parametrize("which", ["mini", "tiny", "stem", "resnet32", "resnet64", "mnv2", "mnv2_32"])
+@pytest.mark.parametrize("which", ["mini", "tiny", "stem", "resnet32", "resnet64", "mnv2", "mnv2_32", "shuffle",
+                                   "shuffle_32"])
 def test_forward_vs_torch_interpreter(which):
     """c.1 steps 2-3 at model level, including the ResNet stem geometry (7x7/2/3 conv, 3x3/2/1 padded
     max-pool), leaky-ReLU and every residual form: a padding, pool-window or slope mistake in the
@@ -190,7 +211,7 @@ def _labels(n, ncls, seed):
     return np.random.default_rng(seed).integers(0, ncls, n).astype(np.int32)
 
 
-@pytest.mark.parametrize("which", ["mini", "stem", "mnv2"])
+@pytest.mark.parametrize("which", ["mini", "stem", "mnv2", "shuffle"])
 def test_exact_grad_vs_autograd_and_fd(which):
     """c.1 steps 10-11: the backward derivation (CE over all exits, head grads, GAP broadcast, ReLU and
     leaky-ReLU masks, first-max max-pool routing incl. the padded 3x3/2/1 stem pool, residual copy,
@@ -221,7 +242,7 @@ def test_exact_grad_vs_autograd_and_fd(which):
         assert abs(fd - g[j]) <= 1e-6 + 1e-4 * abs(g[j]), (j, fd, g[j])
 
 
-@pytest.mark.parametrize("which", ["mini", "tiny", "stem", "resnet32", "mnv2"])
+@pytest.mark.parametrize("which", ["mini", "tiny", "stem", "resnet32", "mnv2", "shuffle"])
 def test_bf16_storage_grads_vs_torch_emulation(which):
     """The bf16-storage gradient (what the GPU must match) against
     torch.autograd over the interpreter with the same rounding points emulated (straight-through bf16 /
