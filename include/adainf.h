@@ -61,10 +61,17 @@ typedef void* adainf_stream_t; /* cudaStream_t (NULL = legacy default stream) */
  * A model is a sequence of ops applied to the current tensor:
  *   CONV     kh x kw conv, stride, pad, cout; act 0 none / 1 ReLU / 2 leaky-ReLU(0.1) / 3 ReLU6; BN folded
  *            (reading Q10).  residual=1: add the innermost open BLOCK's shortcut before the act and
- *            close that block.  A CONV directly followed by DET_HEAD writes fp32 (no bf16 rounding).
+ *            close that block; residual=2: close it by concatenating [shortcut, conv] along channels, act
+ *            applied to both parts (ShuffleNet stride-2 unit; output channels = shortcut's + cout).
+ *            A CONV directly followed by DET_HEAD writes fp32 (no bf16 rounding).
+ *   SHUFFLE  ShuffleNet channel shuffle of the current tensor with `groups` g (view (g, C/g), transpose,
+ *            flatten; NEXT-3).  It must directly follow a non-depthwise CONV whose output has no other
+ *            reader yet: the permutation is folded into that conv's output channel order (weights and bias),
+ *            so no data moves (ADAINF_ERR_UNSUPPORTED otherwise).
  *   MAXPOOL  kh x kw window, stride, pad (padding = -inf).
  *   BLOCK    opens a residual block on the current tensor; cout > 0 -> 1x1 projection shortcut with
- *            `stride` (no activation), else identity.
+ *            `stride` (no activation); pool = 1 -> kh x kw average-pool shortcut (stride, pad; zero padding
+ *            counted in the divisor, ShuffleNet); else identity.
  *   EXIT     early-exit head on the current tensor: GAP -> FC (num_classes) -> softmax (reading Q4);
  *            exit criterion max-softmax confidence >= tau (readings Q1/Q5); the last EXIT is the
  *            final classifier and is unconditional.  All EXITs of a model share num_classes.
@@ -81,7 +88,8 @@ typedef enum {
   ADAINF_OP_MAXPOOL = 1,
   ADAINF_OP_BLOCK = 2,
   ADAINF_OP_EXIT = 3,
-  ADAINF_OP_DET_HEAD = 4
+  ADAINF_OP_DET_HEAD = 4,
+  ADAINF_OP_SHUFFLE = 5
 } adainf_op_kind;
 
 typedef struct {
@@ -95,8 +103,10 @@ typedef struct {
   float anchor_wh[16];
   float nms_iou;      /* DET_HEAD: > 0 -> greedy per-(frame, class) NMS at this IoU threshold before routing
                          (NEXT-3, reading Q18b); 0 -> none */
-  int32_t groups;     /* CONV: 0 / 1 dense; == cin == cout: depthwise 3x3 (MobileNetV2, NEXT-3); other values
-                         ADAINF_ERR_UNSUPPORTED.  Weights [cout][kh][kw][cin / groups] */
+  int32_t groups;     /* CONV: 0 / 1 dense; == cin == cout: depthwise 3x3 (MobileNetV2, NEXT-3); 1 < groups < cin:
+                         grouped conv (ShuffleNet, NEXT-3; cin, cout multiples of groups), run as one tensor-core GEMM
+                         over a block-diagonal weight.  Weights [cout][kh][kw][cin / groups].  SHUFFLE: g */
+  int32_t pool;       /* BLOCK: 1 -> average-pool shortcut (kh, kw, stride, pad) */
 } adainf_op;
 
 typedef struct {

@@ -15,7 +15,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libadainf.so")
 
 OK, ERR_INVALID, ERR_SHAPE, ERR_CAPACITY, ERR_OOM, ERR_CUDA, ERR_NCCL, ERR_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6, -7
-_OPKIND = {"conv": 0, "maxpool": 1, "block": 2, "exit": 3, "det_head": 4}
+_OPKIND = {"conv": 0, "maxpool": 1, "block": 2, "exit": 3, "det_head": 4, "shuffle": 5}
 ROUTE_DET_CROP, ROUTE_CLASS_WHOLE = 0, 1
 
 
@@ -30,7 +30,7 @@ class Op(C.Structure):
                 ("pad", C.c_int32), ("cout", C.c_int32), ("act", C.c_int32), ("residual", C.c_int32),
                 ("num_classes", C.c_int32), ("loss_weight", C.c_float), ("anchors", C.c_int32),
                 ("det_classes", C.c_int32), ("grid_stride", C.c_int32), ("anchor_wh", C.c_float * 16),
-                ("nms_iou", C.c_float), ("groups", C.c_int32)]
+                ("nms_iou", C.c_float), ("groups", C.c_int32), ("pool", C.c_int32)]
 
 
 class ModelSpec(C.Structure):
@@ -180,6 +180,7 @@ def make_ops(spec):
             r.anchor_wh[j] = v
         r.nms_iou = float(o.get("nms_iou", 0.0))
         r.groups = int(o.get("groups", 1))
+        r.pool = int(o.get("pool", 0))
     return ops
 
 

@@ -894,7 +894,14 @@ __device__ __forceinline__ void shadow_store(const SgdSeg& sg, long long local, 
     const unsigned co = l / (unsigned)K;
     const int rem = (int)(l - co * (unsigned)K);
     const int tap = rem / sg.cin, ci = rem - tap * sg.cin;
-    sg.shadow[(long long)co * sg.ldb + tap * sg.cin_pad + ci] = __float2bfloat16_rn(w4[q]);
+    int col = tap * sg.cin_pad + ci;
+    if (sg.cog) col += (int)(co / (unsigned)sg.cog) * sg.cin;  // block-diagonal (grouped conv)
+    unsigned row = co;
+    if (sg.shuf_g) {  // folded channel shuffle
+      const unsigned Cs = (unsigned)(sg.cout / sg.shuf_g);
+      row = (co % Cs) * (unsigned)sg.shuf_g + co / Cs;
+    }
+    sg.shadow[(long long)row * sg.ldb + col] = __float2bfloat16_rn(w4[q]);
   }
 }
 
@@ -958,7 +965,7 @@ __global__ void __launch_bounds__(SGD_THREADS) sgd_kernel(float* __restrict__ w,
     }
     if (sg.shadow) {
       const long long local = i - sg.off;
-      if (sg.cin == sg.cin_pad && (sg.cin & 3) == 0 && cnt == 4 && (local & 3) == 0) {
+      if (sg.cin == sg.cin_pad && !sg.shuf_g && (sg.cin & 3) == 0 && cnt == 4 && (local & 3) == 0) {
         const unsigned K = (unsigned)(sg.taps * sg.cin);  // segment-local offsets < 2^31: 32-bit division
         const unsigned co = (unsigned)local / K;
         const int rem = (int)((unsigned)local - co * K);

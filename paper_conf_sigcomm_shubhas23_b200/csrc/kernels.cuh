@@ -48,6 +48,24 @@ void dw_dgrad(const DwArgs& a, cudaStream_t st);
 size_t dw_wgrad_ws_bytes(const ConvGeom& g, int n);
 void dw_wgrad(const DwArgs& a, float* ws, size_t ws_bytes, float* dw, float* db, cudaStream_t st);
 
+// ---- ShuffleNet pieces (NEXT-3), shuffle.cu: channel-shuffle fold (permuted bias), grouped weight-gradient gather,
+// stride-2 unit's average-pool shortcut + concat
+struct AvgPoolArgs {
+  const bf16* x;       // [n][H][W][C] (rows through map)
+  const int* map;
+  const int* count;
+  int n_static, H, W, C, K, s, p, Ho, Wo;
+  bf16* y;             // [n][Ho][Wo][C]
+};
+void permute_bias(const float* b, int Cout, int g, float* out, cudaStream_t st);
+void grouped_wgrad_gather(const float* dense, const float* dbs, int Cout, int taps, int Cin, int groups, int shuf_g,
+                          float* dw, float* db, cudaStream_t st);
+void avgpool_fwd(const AvgPoolArgs& a, cudaStream_t st);
+void concat_fwd(const bf16* S, const bf16* Y, const int* count, int n_static, int HW, int Cs, int Co, int act, bf16* Z,
+                cudaStream_t st);
+void concat_bwd(const bf16* dZ, int n, int H, int W, int Cs, int Co, int K, int s, int p, int Ho, int Wo, bf16* dY,
+                bf16* sc, cudaStream_t st);
+
 // ---- first conv layer fused with its 2x2/2 max-pool (inference; the detector's 416x416x3 -> 16 layer), convpool.cu
 struct ConvPoolArgs {
   const bf16* x;        // packed input [n][H][W][cin_pad]
@@ -126,6 +144,9 @@ struct SgdSeg {
   long long count;
   bf16* shadow;        // conv weight shadow [Cout][ldb] or nullptr
   int taps, cin, cin_pad, ldb;
+  int cog;             // grouped conv: output channels per group (weight (co, tap, ci) -> column tap*cin_pad +
+                       // (co / cog) * cin + ci of the block-diagonal shadow); 0 = dense
+  int shuf_g, cout;    // folded channel shuffle: master row co -> shadow row (co % (cout/shuf_g)) * shuf_g + co / ...
 };
 // elements per sgd_kernel block (the host partitions the parameter segments into units of this size)
 constexpr int SGD_BLOCK_ELEMS = 256 * 4 * 2;

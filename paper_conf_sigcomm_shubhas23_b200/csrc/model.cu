@@ -64,6 +64,53 @@ void Model::build(const adainf_model_spec& s) {
   long long off = 0;
   for (size_t i = 0; i < ops.size(); ++i) {
     const adainf_op& o = ops[i];
+    if (o.kind == ADAINF_OP_BLOCK && o.cout <= 0 && o.pool) {
+      // average-pool shortcut (ShuffleNet stride-2 unit): its own node and tensor, closed by a concat
+      NodeRt nd;
+      nd.kind = N_AVGPOOL;
+      nd.op = (int)i;
+      nd.in = cur;
+      nd.stage = stage;
+      const TensorRt& X = T[cur];
+      if (X.f32 || X.C % 8) throw ShapeError("pool shortcut: bf16 input with a multiple of 8 channels");
+      if (o.kh <= 0 || o.kh != o.kw || o.stride <= 0 || o.pad < 0 || o.pad >= o.kh)
+        throw ShapeError("pool shortcut: bad window");
+      nd.pk = o.kh;
+      nd.ps = o.stride;
+      nd.pp = o.pad;
+      nd.g.H = X.H;
+      nd.g.W = X.W;
+      nd.g.Cin = nd.g.Cout = X.C;
+      nd.g.Ho = (X.H + 2 * o.pad - o.kh) / o.stride + 1;
+      nd.g.Wo = (X.W + 2 * o.pad - o.kw) / o.stride + 1;
+      if (T[cur].avgpool >= 0) throw InvalidError("tensor used by two pool shortcuts");
+      TensorRt Y;
+      Y.H = nd.g.Ho;
+      Y.W = nd.g.Wo;
+      Y.C = X.C;
+      Y.producer = (int)nodes.size();
+      Y.stage = stage;
+      T[cur].avgpool = (int)nodes.size();
+      T.push_back(std::move(Y));
+      nd.out = (int)T.size() - 1;
+      blocks.push_back(nd.out);
+      op_node[i] = (int)nodes.size();
+      nodes.push_back(std::move(nd));
+      continue;
+    }
+    if (o.kind == ADAINF_OP_SHUFFLE) {
+      // channel shuffle folded into the producing conv's output order (shadow rows + bias): no data moves
+      const int pr = T[cur].producer;
+      bool ok = pr >= 0 && nodes[pr].kind == N_CONV && nodes[pr].out == cur && nodes[pr].in != 0 &&
+                !nodes[pr].fp32_out && nodes[pr].shuf_g == 0 && nodes[pr].res < 0 &&
+                (nodes[pr].groups == 1 || nodes[pr].gdense) && T[cur].primary < 0 && T[cur].exit_k < 0 &&
+                T[cur].res_of < 0 && T[cur].proj < 0 && T[cur].avgpool < 0;
+      for (int b : blocks) ok = ok && b != cur;
+      if (!ok) throw UnsupportedError("SHUFFLE must directly follow a dense / grouped conv whose output has no other reader");
+      if (o.groups <= 1 || T[cur].C % o.groups) throw ShapeError("shuffle: groups must divide the channels");
+      nodes[pr].shuf_g = o.groups;
+      continue;
+    }
     if (o.kind == ADAINF_OP_CONV || o.kind == ADAINF_OP_BLOCK) {
       const bool proj = o.kind == ADAINF_OP_BLOCK;
       if (proj && o.cout <= 0) {
@@ -95,8 +142,13 @@ void Model::build(const adainf_model_spec& s) {
       if (nd.g.Ho <= 0 || nd.g.Wo <= 0) throw ShapeError("conv: empty output");
       nd.groups = (!proj && o.groups > 1) ? o.groups : 1;
       if (nd.groups > 1) {
-        if (!dw_ok(nd.g, nd.groups) || cur == 0)
-          throw UnsupportedError("grouped conv: only depthwise 3x3 (groups == cin == cout, multiple of 8) is supported");
+        if (cur == 0) throw UnsupportedError("grouped conv on the model input");
+        if (!dw_ok(nd.g, nd.groups)) {
+          // grouped (ShuffleNet): one dense GEMM over a block-diagonal weight
+          if (X.C % nd.groups || o.cout % nd.groups || nd.groups >= X.C)
+            throw UnsupportedError("grouped conv: groups must divide cin and cout (depthwise: 3x3, groups == cin == cout)");
+          nd.gdense = true;
+        }
       }
       if (!proj && (o.act < 0 || o.act > 3)) throw InvalidError("conv: act must be 0..3");
       nd.cin_real = (cur == 0) ? in_c : X.C / nd.groups;
@@ -105,7 +157,8 @@ void Model::build(const adainf_model_spec& s) {
       off += (long long)o.cout * KH * KW * nd.cin_real;
       nd.b_off = off;
       off += o.cout;
-      nd.ldb = pad8(KH * KW * X.C / nd.groups);  // 16-byte aligned shadow rows (4-channel stems: 49*4 -> 200)
+      // 16-byte aligned shadow rows (4-channel stems: 49*4 -> 200); grouped-dense rows span all input channels
+      nd.ldb = pad8(KH * KW * X.C / (nd.gdense ? 1 : nd.groups));
       nd.fp32_out = !proj && (i + 1 < ops.size() && ops[i + 1].kind == ADAINF_OP_DET_HEAD);
       TensorRt Y;
       Y.H = nd.g.Ho;
@@ -117,7 +170,17 @@ void Model::build(const adainf_model_spec& s) {
       Y.f32 = nd.fp32_out;
       T.push_back(std::move(Y));
       nd.out = (int)T.size() - 1;
-      if (!proj && o.residual) {
+      int concat_src = -1;
+      if (!proj && o.residual == 2) {  // concat join: [shortcut, this conv] (ShuffleNet stride-2 unit)
+        if (blocks.empty()) throw InvalidError("concat conv without an open block");
+        concat_src = blocks.back();
+        blocks.pop_back();
+        const TensorRt& R = T[concat_src];
+        const TensorRt& Yo = T[nd.out];
+        if (R.H != Yo.H || R.W != Yo.W || R.f32) throw ShapeError("concat shape mismatch");
+        if (R.stage != stage) throw InvalidError("a residual block may not span an exit");
+        if (nd.fp32_out) throw UnsupportedError("concat into a detector head");
+      } else if (!proj && o.residual) {
         if (blocks.empty()) throw InvalidError("residual conv without an open block");
         nd.res = blocks.back();
         blocks.pop_back();
@@ -143,6 +206,29 @@ void Model::build(const adainf_model_spec& s) {
       }
       op_node[i] = ni;
       nodes.push_back(std::move(nd));
+      if (concat_src >= 0) {
+        const int yi = cur;
+        NodeRt cn;
+        cn.kind = N_CONCAT;
+        cn.op = (int)i;
+        cn.in = yi;
+        cn.res = concat_src;
+        cn.stage = stage;
+        cn.act = o.act;
+        TensorRt Z;
+        Z.H = T[yi].H;
+        Z.W = T[yi].W;
+        Z.C = T[concat_src].C + T[yi].C;
+        Z.producer = (int)nodes.size();
+        Z.act = o.act;
+        Z.stage = stage;
+        T[yi].primary = (int)nodes.size();
+        T[concat_src].primary = (int)nodes.size();
+        T.push_back(std::move(Z));
+        cn.out = (int)T.size() - 1;
+        cur = cn.out;
+        nodes.push_back(std::move(cn));
+      }
     } else if (o.kind == ADAINF_OP_MAXPOOL) {
       NodeRt nd;
       nd.kind = N_POOL;
@@ -263,10 +349,11 @@ void Model::build(const adainf_model_spec& s) {
     T[0].buf = packed_in.as<bf16>();
   }
   for (auto& nd : nodes)
-    if (nd.kind != N_POOL) {
+    if (nd.kind == N_CONV || nd.kind == N_PROJ) {
       nd.shadow.alloc((size_t)nd.g.Cout * nd.ldb * 2);
-      nd.shadow.zero();
-      if (nd.groups > 1) nd.wdw.alloc((size_t)nd.g.KH * nd.g.KW * nd.g.Cin * 2);
+      nd.shadow.zero();  // grouped-dense: the off-diagonal blocks stay zero
+      if (nd.groups > 1 && !nd.gdense) nd.wdw.alloc((size_t)nd.g.KH * nd.g.KW * nd.g.Cin * 2);
+      if (nd.shuf_g) nd.bias_perm.alloc((size_t)nd.g.Cout * 4);
     }
   if (stem_s2d) stem_wprep.alloc(16 * 2 * 64 * 8 * 2);
   for (size_t k = 0; k + 1 < exits.size(); ++k) {  // dense survivor copies of the stage-boundary tensors
@@ -301,14 +388,17 @@ void Model::build(const adainf_model_spec& s) {
   // segments in flat order
   std::vector<std::pair<long long, int>> order;  // (offset, kind/index)
   for (size_t i = 0; i < nodes.size(); ++i)
-    if (nodes[i].kind != N_POOL) order.push_back({nodes[i].w_off, (int)i});
+    if (nodes[i].kind == N_CONV || nodes[i].kind == N_PROJ) order.push_back({nodes[i].w_off, (int)i});
   for (size_t k = 0; k < exits.size(); ++k) order.push_back({exits[k].w_off, -1 - (int)k});
   std::sort(order.begin(), order.end());
   for (auto& pr : order) {
     if (pr.second >= 0) {
       NodeRt& nd = nodes[pr.second];
       add_seg(nd.w_off, (long long)nd.g.Cout * nd.g.KH * nd.g.KW * nd.cin_real, nd.shadow.as<bf16>(),
-              nd.g.KH * nd.g.KW, nd.cin_real, nd.g.Cin / nd.groups, nd.ldb);
+              nd.g.KH * nd.g.KW, nd.cin_real, nd.gdense ? nd.g.Cin : nd.g.Cin / nd.groups, nd.ldb);
+      segs.back().cog = nd.gdense ? nd.g.Cout / nd.groups : 0;
+      segs.back().shuf_g = nd.shuf_g;
+      segs.back().cout = nd.g.Cout;
       add_seg(nd.b_off, nd.g.Cout, nullptr, 0, 0, 0, 0);
     } else {
       ExitRt& e = exits[-1 - pr.second];
@@ -341,7 +431,7 @@ void Model::build(const adainf_model_spec& s) {
     std::mt19937_64 rng(s.seed);
     std::normal_distribution<float> nd01(0.f, 1.f);
     for (auto& nd : nodes) {
-      if (nd.kind == N_POOL) continue;
+      if (nd.kind != N_CONV && nd.kind != N_PROJ) continue;
       const float sd = std::sqrt(1.0f / (float)(nd.g.KH * nd.g.KW * nd.cin_real));
       for (long long j = nd.w_off; j < nd.b_off; ++j) host[j] = nd01(rng) * sd;
       for (int j = 0; j < nd.g.Cout; ++j) host[nd.b_off + j] = 0.01f * nd01(rng);
@@ -391,11 +481,19 @@ void Model::ensure_training() {
       nd.sp = true;
       nd.wsp.alloc(dgrad_sp_ws_bytes(nd.g));
     }
+  size_t gd = 0;  // dense weight-gradient scratch of grouped / shuffled convs (gathered into the master layout)
   for (auto& nd : nodes) {
+    if (nd.kind == N_CONCAT) continue;
+    if (nd.kind == N_AVGPOOL) {
+      if (nd.in != 0) nd.pool_sc.alloc((size_t)max_batch * T[nd.in].row_elems() * 2);
+      continue;
+    }
+    if (nd.gdense || nd.shuf_g)
+      gd = std::max(gd, ((size_t)nd.g.Cout * nd.g.KH * nd.g.KW * nd.g.Cin + nd.g.Cout) * 4);
     if (nd.kind == N_POOL) {
       nd.argmax.alloc((size_t)max_batch * T[nd.out].row_elems());
     } else {
-      ws = std::max(ws, nd.groups > 1 ? dw_wgrad_ws_bytes(nd.g, max_batch) : ::adainf::wgrad_ws_bytes(nd.g, max_batch));
+      ws = std::max(ws, (nd.groups > 1 && !nd.gdense) ? dw_wgrad_ws_bytes(nd.g, max_batch) : ::adainf::wgrad_ws_bytes(nd.g, max_batch));
       if (stem_s2d && &nd == &nodes[0]) ws = std::max(ws, stem_wgrad_ws_bytes(max_batch));
       if (nd.kind == N_PROJ && nd.in != 0) {
         for (const auto& c : nodes)
@@ -408,6 +506,7 @@ void Model::ensure_training() {
   for (auto& e : exits) ws = std::max(ws, head_grads_ws_bytes(max_batch, T[e.tensor].C, e.ncls));
   wgrad_ws.alloc(ws);
   wgrad_ws_bytes = ws;
+  gw_dense.alloc(gd);
   for (auto& e : exits) {
     const int C = T[e.tensor].C;
     e.pooled.alloc((size_t)max_batch * C * 4);
@@ -476,13 +575,31 @@ void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, in
         conv_first_pool(cp, st);
         continue;
       }
+      if (nd.kind == N_AVGPOOL) {
+        AvgPoolArgs ap{};
+        ap.x = buf_of(nd.in);
+        ap.map = map_for(nd.in, ns);
+        ap.count = c;
+        ap.n_static = n_static;
+        ap.H = nd.g.H;
+        ap.W = nd.g.W;
+        ap.C = nd.g.Cin;
+        ap.K = nd.pk;
+        ap.s = nd.ps;
+        ap.p = nd.pp;
+        ap.Ho = nd.g.Ho;
+        ap.Wo = nd.g.Wo;
+        ap.y = T[nd.out].buf;
+        avgpool_fwd(ap, st);
+        continue;
+      }
       if (nd.kind == N_POOL) {
         if (stem_s2d && ni == stem_pool) continue;  // produced by the fused stem
         if (!train && ni == fused_pool0) continue;  // produced by the fused first conv
         launch_maxpool_fwd(buf_of(nd.in), map_for(nd.in, ns), c, n_static, nd.g.H, nd.g.W, nd.g.Cin, nd.pk, nd.ps,
                            nd.pp, nd.g.Ho, nd.g.Wo, T[nd.out].buf, train ? nd.argmax.as<uint8_t>() : nullptr,
                            nd.in > 0 && T[nd.in].act == 1, st);
-      } else if (nd.groups > 1) {
+      } else if (nd.groups > 1 && !nd.gdense) {
         if (nd.res >= 0) throw UnsupportedError("depthwise conv closing a residual block");
         dw_prep(nd.shadow.as<bf16>(), nd.ldb, nd.g.Cin, nd.g.KH * nd.g.KW, nd.wdw.as<bf16>(), st);
         DwArgs d{};
@@ -506,10 +623,19 @@ void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, in
         dw_fwd(d, st);
       } else {
         const float* bias = params.as<float>() + nd.b_off;
+        if (nd.shuf_g) {  // folded channel shuffle: bias in the physical output order
+          permute_bias(bias, nd.g.Cout, nd.shuf_g, nd.bias_perm.as<float>(), st);
+          bias = nd.bias_perm.as<float>();
+        }
         const bf16* res = nd.res >= 0 ? buf_of(nd.res) : nullptr;
         const int* rmap = nd.res >= 0 ? map_for(nd.res, ns) : nullptr;
         conv_fwd(nd.g, buf_of(nd.in), map_for(nd.in, ns), c, n_static, nd.shadow.as<bf16>(), nd.ldb, bias, res, rmap,
                  nd.act, T[nd.out].buf, nd.fp32_out, st);
+        if (ni + 1 < (int)nodes.size() && nodes[ni + 1].kind == N_CONCAT && nodes[ni + 1].in == nd.out) {
+          const NodeRt& cn = nodes[ni + 1];  // [shortcut, conv] join right after its conv (same stage rows)
+          const TensorRt& Z = T[cn.out];
+          concat_fwd(T[cn.res].buf, T[nd.out].buf, c, n_static, Z.H * Z.W, T[cn.res].C, nd.g.Cout, cn.act, Z.buf, st);
+        }
       }
       continue;
     }
@@ -655,11 +781,13 @@ void Model::train_grad_impl(const bf16* x, const int32_t* row_map, const int32_t
   auto sc_of = [&](int t) -> const bf16* {
     if (T[t].res_of >= 0) return T[nodes[T[t].res_of].out].grad;  // identity shortcut: dZ of the residual conv
     if (T[t].proj >= 0) return nodes[T[t].proj].proj_dx.as<bf16>();
+    if (T[t].avgpool >= 0) return nodes[T[t].avgpool].pool_sc.as<bf16>();  // average-pool shortcut's backward
     return nullptr;
   };
   // tensors with no main-path consumer (the final exit's input): gradient = broadcast (+ shortcut)
   for (size_t t = 1; t < T.size(); ++t)
-    if (T[t].primary < 0 && !T[t].f32 && T[t].producer >= 0 && nodes[T[t].producer].kind != N_PROJ)
+    if (T[t].primary < 0 && !T[t].f32 && T[t].producer >= 0 && nodes[T[t].producer].kind != N_PROJ &&
+        nodes[T[t].producer].kind != N_AVGPOOL)
       launch_grad_finalize(bcast_of((int)t), sc_of((int)t), T[t].buf, T[t].act, n, T[t].H * T[t].W, T[t].C,
                            T[t].grad, st);
   // reverse walk (K2, K3, K9)
@@ -688,7 +816,7 @@ void Model::train_grad_impl(const bf16* x, const int32_t* row_map, const int32_t
       }
       return;
     }
-    if (nd.groups > 1) {  // depthwise: weight / bias gradient, then the input gradient (dwconv.cu)
+    if (nd.groups > 1 && !nd.gdense) {  // depthwise: weight / bias gradient, then the input gradient (dwconv.cu)
       DwArgs d{};
       d.x = buf_of(nd.in);
       d.dz = dz;
@@ -706,7 +834,7 @@ void Model::train_grad_impl(const bf16* x, const int32_t* row_map, const int32_t
       if (nd.in == 0) return;
       const TensorRt& X = T[nd.in];
       const int prod = X.producer;
-      const int mask = (prod >= 0 && nodes[prod].kind == N_CONV) ? X.act : 0;
+      const int mask = (prod >= 0 && (nodes[prod].kind == N_CONV || nodes[prod].kind == N_CONCAT)) ? X.act : 0;
       d.x = dz;
       d.w = nd.wdw.as<bf16>();
       d.bcast = bcast_of(nd.in);
@@ -717,8 +845,18 @@ void Model::train_grad_impl(const bf16* x, const int32_t* row_map, const int32_t
       dw_dgrad(d, st);
       return;
     }
-    conv_wgrad(nd.g, buf_of(nd.in), dz, n, nd.cin_real, wgrad_ws.as<float>(), wgrad_ws_bytes, G + nd.w_off,
-               G + nd.b_off, st);
+    if (nd.gdense || nd.shuf_g) {
+      // dense weight gradient over the block-diagonal / row-permuted shadow, then its diagonal blocks gathered
+      // back into the master layout (shuffle.cu)
+      float* dense = gw_dense.as<float>();
+      float* dbs = dense + (size_t)nd.g.Cout * nd.g.KH * nd.g.KW * nd.g.Cin;
+      conv_wgrad(nd.g, buf_of(nd.in), dz, n, nd.g.Cin, wgrad_ws.as<float>(), wgrad_ws_bytes, dense, dbs, st);
+      grouped_wgrad_gather(dense, dbs, nd.g.Cout, nd.g.KH * nd.g.KW, nd.g.Cin, nd.gdense ? nd.groups : 1, nd.shuf_g,
+                           G + nd.w_off, G + nd.b_off, st);
+    } else {
+      conv_wgrad(nd.g, buf_of(nd.in), dz, n, nd.cin_real, wgrad_ws.as<float>(), wgrad_ws_bytes, G + nd.w_off,
+                 G + nd.b_off, st);
+    }
     if (nd.in == 0) return;  // no input gradient for the first layer
     const TensorRt& X = T[nd.in];
     if (nd.kind == N_PROJ) {
@@ -731,7 +869,7 @@ void Model::train_grad_impl(const bf16* x, const int32_t* row_map, const int32_t
       conv_dgrad(g, dz, nd.shadow.as<bf16>(), nd.ldb, n, nullptr, nullptr, nullptr, 0, nd.proj_dx.as<bf16>(), st);
     } else {
       const int prod = X.producer;
-      const int mask = (prod >= 0 && nodes[prod].kind == N_CONV) ? X.act : 0;
+      const int mask = (prod >= 0 && (nodes[prod].kind == N_CONV || nodes[prod].kind == N_CONCAT)) ? X.act : 0;
       if (nd.sp) {
         const bool sc_compact = X.res_of < 0 && X.proj >= 0 && nodes[X.proj].proj_compact;
         conv_dgrad_sp(nd.g, dz, nd.shadow.as<bf16>(), nd.ldb, nd.wsp.as<bf16>(), n, bcast_of(nd.in), sc_of(nd.in),
@@ -744,7 +882,20 @@ void Model::train_grad_impl(const bf16* x, const int32_t* row_map, const int32_t
   };
   for (int ni = (int)nodes.size() - 1; ni >= 0; --ni) {
     NodeRt& nd = nodes[ni];
-    if (nd.kind == N_PROJ) continue;  // handled right after its residual conv
+    if (nd.kind == N_PROJ || nd.kind == N_AVGPOOL) continue;  // projection: right after its residual conv;
+                                                              // avg-pool shortcut: inside its concat's backward
+    if (nd.kind == N_CONCAT) {
+      // T[out].grad = the consumer's gradient of [shortcut, conv], already masked by act'(Z) and bf16: its conv
+      // part is the conv's dZ, its shortcut part goes through the average-pool backward into the block input's
+      // shortcut term
+      const NodeRt& ap = nodes[T[nd.res].producer];
+      const TensorRt& Z = T[nd.out];
+      bf16* sc = ap.in != 0 ? nodes[T[nd.res].producer].pool_sc.as<bf16>() : nullptr;
+      if (!sc) throw UnsupportedError("pool shortcut on the model input");
+      concat_bwd(Z.grad, n, ap.g.H, ap.g.W, T[nd.res].C, T[nd.in].C, ap.pk, ap.ps, ap.pp, Z.H, Z.W, T[nd.in].grad, sc,
+                 st);
+      continue;
+    }
     if (nd.kind == N_POOL) {
       const TensorRt& X = T[nd.in];
       if (nd.in == 0) continue;

@@ -19,7 +19,8 @@
 
 namespace adainf {
 
-enum NodeKind { N_CONV = 0, N_POOL = 1, N_PROJ = 2 };
+// N_AVGPOOL: a BLOCK's average-pool shortcut; N_CONCAT: [shortcut, conv] join closing such a block (ShuffleNet)
+enum NodeKind { N_CONV = 0, N_POOL = 1, N_PROJ = 2, N_AVGPOOL = 3, N_CONCAT = 4 };
 
 struct DevBuf {  // owning device allocation
   void* p = nullptr;
@@ -55,6 +56,7 @@ struct TensorRt {
   int proj = -1;         // projection node reading it
   int res_of = -1;       // conv node adding it as identity shortcut
   int exit_k = -1;       // exit attached
+  int avgpool = -1;      // N_AVGPOOL node reading it as a block input (its shortcut term comes from there)
   size_t row_elems() const { return (size_t)H * W * C; }
 };
 
@@ -66,7 +68,11 @@ struct NodeRt {
   ConvGeom g{};
   int act = 0;
   int cin_real = 0;            // input channels per group of the weights (first layer: the unpadded in_c)
-  int groups = 1;              // > 1: depthwise (groups == Cin == Cout), dwconv.cu
+  int groups = 1;              // > 1: depthwise (groups == Cin == Cout, dwconv.cu) or, with gdense, grouped
+  bool gdense = false;         // grouped conv as one dense GEMM over a block-diagonal shadow (shuffle.cu)
+  int shuf_g = 0;              // > 1: channel shuffle folded into the output channel order (shadow rows, bias)
+  DevBuf bias_perm;            // shuf_g: bias in the physical (shuffled) order, rebuilt every forward
+  DevBuf pool_sc;              // N_AVGPOOL (training): shortcut term of the block input, bf16 [max_batch][H][W][C]
   DevBuf wdw;                  // depthwise weights [taps][C] bf16, rebuilt from the shadow every forward
   long long w_off = 0, b_off = 0;
   int ldb = 0;
@@ -125,6 +131,7 @@ struct Model {
   // training
   bool train_ready = false;
   DevBuf wgrad_ws, loss_rows, stats_tmp, sq_partial;
+  DevBuf gw_dense;  // grouped / shuffled convs: dense weight-gradient scratch [Cout][taps][Cin] + [Cout]
   size_t wgrad_ws_bytes = 0;
   DevBuf sgd_segs, sgd_block_seg, sgd_block_start;
   int sgd_nblocks = 0, sgd_nseg = 0;

@@ -15,7 +15,7 @@ static const char* kNames[PROF_NCLASS] = {"conv_fwd",     "conv_dgrad", "conv_wg
                                           "shadow_pack",  "select_proj", "select_cosine", "select_topk", "det_route",
                                           "crop",         "route_class", "gather_rows", "stem_fwd",   "stem_wgrad",
                                           "stem_aux",     "dgrad_sp_prep", "survivor_gather", "exit_head_train",
-                                          "version_average", "depthwise"};
+                                          "version_average", "depthwise", "shufflenet_aux"};
 
 struct Prof {
   std::mutex mu;

@@ -36,6 +36,7 @@ enum ProfClass {
   PC_EXIT_HEAD_TRAIN,
   PC_VERSION_AVG,
   PC_DW,
+  PC_SHUFFLE,
   PROF_NCLASS
 };
 

@@ -123,9 +123,11 @@ def test_mobilenetv2_ee_retrain_step():
     assert abs(r["loss"] - r["loss_o"]) <= 2e-2 * abs(r["loss_o"])
 
 
-def test_grouped_conv_other_than_depthwise_is_unsupported():
-    spec = {"name": "g", "in_h": 16, "in_w": 16, "in_c": 3,
-            "ops": [S.conv(3, 16), S.conv(3, 16, groups=4), S.exit_(4)]}
-    with pytest.raises(B.AdaInfError) as ei:
-        B.Model(spec, 4)
-    assert ei.value.code == B.ERR_UNSUPPORTED
+def test_grouped_conv_not_dividing_channels_is_unsupported():
+    """grouped convs run as one block-diagonal GEMM (ShuffleNet, tests/test_gpu_shufflenet.py); groups must divide
+    cin and cout, and groups == cin needs the depthwise geometry (3x3, cout == cin)"""
+    for bad in (S.conv(3, 24, groups=16), S.conv(1, 32, groups=16)):
+        spec = {"name": "g", "in_h": 16, "in_w": 16, "in_c": 3, "ops": [S.conv(3, 16), bad, S.exit_(4)]}
+        with pytest.raises(B.AdaInfError) as ei:
+            B.Model(spec, 4)
+        assert ei.value.code == B.ERR_UNSUPPORTED
