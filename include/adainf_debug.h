@@ -43,6 +43,15 @@ adainf_status adainf_dbg_conv_wgrad(const void* x, const void* dz, int32_t n, in
  *       separate max-pool) instead of the space-to-depth stem kernels */
 adainf_status adainf_dbg_set_win_mode(int32_t mode);
 
+/* 3x3/1 pad-1 conv + bias + act + 2x2/2 max-pool in one tensor-core kernel (conv3pool.cu, the detector's few-channel
+ * layers; C3, reading Q18):  x [n][H][W][C] bf16 (H, W even), w [Co][3][3][C] bf16, b [Co] fp32 ->
+ * y [n][H/2][W/2][Co] bf16 = maxpool2x2(bf16(act(conv + b))).  first = 0: C in {16, 32}, Co in {32, 64, 96, 128};
+ * first = 1: C <= 4 real channels given as 4 (space-to-depth packed internally), Co in {16, 32}.
+ * ADAINF_ERR_SHAPE outside those. */
+adainf_status adainf_dbg_conv3_pool(const void* x, int32_t n, int32_t H, int32_t W, int32_t C, int32_t cin_real,
+                                    const void* w, const float* b, int32_t Co, int32_t act, int32_t first, void* y,
+                                    adainf_stream_t stream);
+
 /* ResNet stem (7x7/2 pad 3 conv, <= 4 input channels, 64 outputs, ReLU, then 3x3/2 pad 1 max-pool) through
  * the space-to-depth kernels (stem.cuh):
  *   stem_fwd  : x [n][H][W][cin] bf16 (H, W even, W/2 <= 125), w [64][7][7][cin] bf16, b [64] fp32 ->

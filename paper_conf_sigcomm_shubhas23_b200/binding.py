@@ -129,6 +129,7 @@ def lib():
             "adainf_prof_reset": [],
             "adainf_prof_query": [vp, i32, C.POINTER(i32)],
             "adainf_dbg_conv_fwd": [vp, i32, i32, i32, i32, vp, vp, i32, i32, i32, i32, i32, i32, vp, vp, i32, vp],
+            "adainf_dbg_conv3_pool": [vp, i32, i32, i32, i32, i32, vp, vp, i32, i32, i32, vp, vp],
             "adainf_dbg_conv_dgrad": [vp, i32, i32, i32, i32, vp, i32, i32, i32, i32, i32, vp, vp, vp, i32, vp,
                                       vp],
             "adainf_dbg_conv_wgrad": [vp, vp, i32, i32, i32, i32, i32, i32, i32, i32, i32, vp, vp, vp],
@@ -486,6 +487,17 @@ def dbg_conv_fwd(x, w, b, stride, pad, act=0, res=None, out_f32=False, stream=No
     check(lib().adainf_dbg_conv_fwd(ptr(x), n, H, W_, Cc, ptr(w), ptr(b), Co, KH, KW, stride, pad, act, ptr(res),
                                     ptr(out), int(out_f32), stream_ptr(stream)))
     return out
+
+
+def dbg_conv3_pool(x, w, b, act=0, first=False, cin_real=None, stream=None):
+    """3x3/1 conv + bias + act + 2x2/2 max-pool in one kernel (include/adainf_debug.h)."""
+    import torch
+    n, H, W_, Cc = x.shape
+    Co = w.shape[0]
+    y = torch.empty((n, H // 2, W_ // 2, Co), dtype=torch.bfloat16, device=x.device)
+    check(lib().adainf_dbg_conv3_pool(ptr(x), n, H, W_, Cc, Cc if cin_real is None else cin_real, ptr(w), ptr(b), Co,
+                                      act, int(first), ptr(y), stream_ptr(stream)))
+    return y
 
 
 def dbg_conv_dgrad(dz, w, H, W_, stride, pad, bcast=None, sc=None, yact=None, mask_act=0, stream=None):

@@ -4,6 +4,7 @@
 #include "../../include/adainf_debug.h"
 #include "api_common.h"
 #include "runtime.h"
+#include "kernels.cuh"
 #include "stem.cuh"
 
 using namespace adainf;
@@ -43,6 +44,36 @@ extern "C" adainf_status adainf_dbg_conv_fwd(const void* x, int32_t n, int32_t H
     }
     conv_fwd(g, (const bf16*)x, nullptr, nullptr, n, wp, ldb, b, (const bf16*)res, nullptr, act, out, out_f32 != 0, st);
     if (tmp) CK(cudaFreeAsync(tmp, st));
+  });
+}
+
+extern "C" adainf_status adainf_dbg_conv3_pool(const void* x, int32_t n, int32_t H, int32_t W, int32_t C,
+                                               int32_t cin_real, const void* w, const float* b, int32_t Co,
+                                               int32_t act, int32_t first, void* y, adainf_stream_t stream) {
+  return guard([&] {
+    if (n <= 0) throw ShapeError("conv3_pool: n must be positive");
+    require_device();
+    ConvGeom g = geom(H, W, C, Co, 3, 3, 1, 1);
+    if (!conv3_pool_ok(g, first != 0, cin_real, 2, 2, 0)) throw ShapeError("conv3_pool: unsupported geometry");
+    cudaStream_t st = (cudaStream_t)stream;
+    const int K = 9 * C, ldb = (K + 7) / 8 * 8;
+    bf16* tmp = nullptr;  // GEMM-ready shadow rows (16-byte aligned) and the expanded weights
+    bf16* wexp = nullptr;
+    bf16* xs = nullptr;
+    CK(cudaMallocAsync((void**)&tmp, (size_t)Co * ldb * 2, st));
+    CK(cudaMemsetAsync(tmp, 0, (size_t)Co * ldb * 2, st));
+    CK(cudaMemcpy2DAsync(tmp, ldb * 2, w, K * 2, K * 2, Co, cudaMemcpyDeviceToDevice, st));
+    CK(cudaMallocAsync((void**)&wexp, conv3_pool_wexp_bytes(g, first != 0), st));
+    const bf16* src = (const bf16*)x;
+    if (first) {  // space-to-depth pack of the 4-channel input, as the model's ingest does
+      CK(cudaMallocAsync((void**)&xs, (size_t)n * H * W * 4 * 2, st));
+      launch_pack_s2d((const bf16*)x, nullptr, nullptr, n, H, W, 4, xs, st);
+      src = xs;
+    }
+    conv3_pool(g, first != 0, src, nullptr, n, tmp, ldb, cin_real, b, act, wexp, (bf16*)y, st);
+    CK(cudaFreeAsync(tmp, st));
+    CK(cudaFreeAsync(wexp, st));
+    if (xs) CK(cudaFreeAsync(xs, st));
   });
 }
 

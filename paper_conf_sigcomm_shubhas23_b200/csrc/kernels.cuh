@@ -66,19 +66,12 @@ void concat_fwd(const bf16* S, const bf16* Y, const int* count, int n_static, in
 void concat_bwd(const bf16* dZ, int n, int H, int W, int Cs, int Co, int K, int s, int p, int Ho, int Wo, bf16* dY,
                 bf16* sc, cudaStream_t st);
 
-// ---- first conv layer fused with its 2x2/2 max-pool (inference; the detector's 416x416x3 -> 16 layer), convpool.cu
-struct ConvPoolArgs {
-  const bf16* x;        // packed input [n][H][W][cin_pad]
-  const int* count;     // device row count or nullptr
-  int n_static, H, W, cin_real, cin_pad;
-  const bf16* shadow;   // GEMM shadow [16][ldb], K = tap * cin_pad + c
-  int ldb;
-  const float* bias;
-  int act;
-  bf16* y;              // pooled [n][H/2][W/2][16]
-};
-bool conv_first_pool_ok(const ConvGeom& g, int cin_real, int pk, int ps, int pp);
-void conv_first_pool(const ConvPoolArgs& a, cudaStream_t st);
+// ---- 3x3/1 conv + bias + act + 2x2/2 max-pool in one tensor-core kernel (inference), conv3pool.cu: the detector's
+// few-channel early layers; first = the model's first layer on the space-to-depth packed input (<= 4 channels)
+bool conv3_pool_ok(const ConvGeom& g, bool first, int cin_real, int pk, int ps, int pp);
+size_t conv3_pool_wexp_bytes(const ConvGeom& g, bool first);
+void conv3_pool(const ConvGeom& g, bool first, const bf16* x, const int* count, int n_static, const bf16* shadow,
+                int ldb, int cin_real, const float* bias, int act, bf16* wexp, bf16* y, cudaStream_t st);
 
 // ---- exit head (K4) ----
 struct ExitHeadArgs {

@@ -322,18 +322,26 @@ void Model::build(const adainf_model_spec& s) {
       pack = true;
     }
   }
-  // first conv (3x3/1, <= 3 real input channels, 16 outputs) whose only consumer is a 2x2/2 max-pool: fused in
-  // inference (the TinyYOLOv3-like detector's 416x416 layer)
-  fused_pool0 = -1;
-  if (!stem_s2d && !nodes.empty() && nodes[0].kind == N_CONV && nodes[0].in == 0 && nodes[0].groups == 1 &&
-      getenv("ADAINF_CONVPOOL") == nullptr) {
-    const NodeRt& c0 = nodes[0];
-    const TensorRt& Y = T[c0.out];
-    const int po = Y.primary;
-    if (po >= 0 && nodes[po].kind == N_POOL && nodes[po].stage == c0.stage && !c0.fp32_out && c0.res < 0 &&
-        Y.exit_k < 0 && Y.res_of < 0 && Y.proj < 0 &&
-        conv_first_pool_ok(c0.g, c0.cin_real, nodes[po].pk, nodes[po].ps, nodes[po].pp))
-      fused_pool0 = po;
+  // 3x3/1 convs whose only reader is a 2x2/2 max-pool (the TinyYOLOv3-like detector's few-channel layers): conv +
+  // pool in one tensor-core kernel in inference (conv3pool.cu); the first layer on the space-to-depth packed input
+  first_s2d = false;
+  const char* c3p_env = getenv("ADAINF_CONV3POOL");
+  if (!c3p_env || atoi(c3p_env) != 0) {
+    for (size_t ni = 0; ni < nodes.size(); ++ni) {
+      NodeRt& nd = nodes[ni];
+      if (nd.kind != N_CONV || nd.groups != 1 || nd.shuf_g || nd.res >= 0 || nd.fp32_out) continue;
+      if (stem_s2d && ni == 0) continue;
+      const TensorRt& Y = T[nd.out];
+      const int po = Y.primary;
+      if (po < 0 || nodes[po].kind != N_POOL || nodes[po].stage != nd.stage || Y.exit_k >= 0 || Y.res_of >= 0 ||
+          Y.proj >= 0 || Y.avgpool >= 0)
+        continue;
+      const bool first = nd.in == 0;
+      if (first && cin_pad != 4) continue;
+      if (!conv3_pool_ok(nd.g, first, nd.cin_real, nodes[po].pk, nodes[po].ps, nodes[po].pp)) continue;
+      nd.fuse_pool = po;
+      if (first) first_s2d = true;
+    }
   }
 
   CK(cudaSetDevice(device));
@@ -354,6 +362,7 @@ void Model::build(const adainf_model_spec& s) {
       nd.shadow.zero();  // grouped-dense: the off-diagonal blocks stay zero
       if (nd.groups > 1 && !nd.gdense) nd.wdw.alloc((size_t)nd.g.KH * nd.g.KW * nd.g.Cin * 2);
       if (nd.shuf_g) nd.bias_perm.alloc((size_t)nd.g.Cout * 4);
+      if (nd.fuse_pool >= 0) nd.wexp.alloc(conv3_pool_wexp_bytes(nd.g, nd.in == 0));
     }
   if (stem_s2d) stem_wprep.alloc(16 * 2 * 64 * 8 * 2);
   for (size_t k = 0; k + 1 < exits.size(); ++k) {  // dense survivor copies of the stage-boundary tensors
@@ -455,8 +464,8 @@ void Model::build(const adainf_model_spec& s) {
 }
 
 // a1 ingest: channel padding (to 4 for few-channel inputs, else to a multiple of 8)
-void Model::ingest(const bf16* x, const int* map, const int* count, int n_static, cudaStream_t st) {
-  if (stem_s2d) {
+void Model::ingest(const bf16* x, const int* map, const int* count, int n_static, cudaStream_t st, bool s2d) {
+  if (stem_s2d || s2d) {
     launch_pack_s2d(x, map, count, n_static, in_h, in_w, in_c, packed_in.as<bf16>(), st);
     return;
   }
@@ -524,7 +533,8 @@ void Model::ensure_training() {
 // positions) and works on count[s] rows (device-side), outputs are scattered through orig[s].
 // Training: all rows, no exits taken, heads evaluated for every row (SURVEY c.1 step 9).
 void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, int n_static, bool train,
-                          const float* taus, const adainf_model_out* out, cudaStream_t st) {
+                          const float* taus, const adainf_model_out* out, cudaStream_t st, bool in_s2d) {
+  std::vector<char> pool_done(nodes.size(), 0);  // max-pools already produced by their conv (conv3_pool)
   int* posb = pos.as<int>();
   int* origb = orig.as<int>();
   int* cnt = counts.as<int>();
@@ -556,23 +566,12 @@ void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, in
                  T[pl.out].buf, train ? pl.argmax.as<uint8_t>() : nullptr, st);
         continue;
       }
-      if (!train && ni == 0 && nd.kind == N_CONV && fused_pool0 >= 0) {
-        // first conv + its 2x2 max-pool in one kernel (inference only: training keeps the pre-pool tensor)
-        const NodeRt& pl = nodes[fused_pool0];
-        ConvPoolArgs cp{};
-        cp.x = buf_of(0);
-        cp.count = c;
-        cp.n_static = n_static;
-        cp.H = nd.g.H;
-        cp.W = nd.g.W;
-        cp.cin_real = nd.cin_real;
-        cp.cin_pad = nd.g.Cin;
-        cp.shadow = nd.shadow.as<bf16>();
-        cp.ldb = nd.ldb;
-        cp.bias = params.as<float>() + nd.b_off;
-        cp.act = nd.act;
-        cp.y = T[pl.out].buf;
-        conv_first_pool(cp, st);
+      if (!train && nd.kind == N_CONV && nd.fuse_pool >= 0 && !map_for(nd.in, ns) && (nd.in != 0 || in_s2d)) {
+        // conv + its 2x2 max-pool in one kernel (inference only: training keeps the pre-pool tensor)
+        const NodeRt& pl = nodes[nd.fuse_pool];
+        conv3_pool(nd.g, nd.in == 0, buf_of(nd.in), c, n_static, nd.shadow.as<bf16>(), nd.ldb, nd.cin_real,
+                   params.as<float>() + nd.b_off, nd.act, nd.wexp.as<bf16>(), T[pl.out].buf, st);
+        pool_done[nd.fuse_pool] = 1;
         continue;
       }
       if (nd.kind == N_AVGPOOL) {
@@ -595,7 +594,7 @@ void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, in
       }
       if (nd.kind == N_POOL) {
         if (stem_s2d && ni == stem_pool) continue;  // produced by the fused stem
-        if (!train && ni == fused_pool0) continue;  // produced by the fused first conv
+        if (pool_done[ni]) continue;  // produced by its conv (conv3_pool)
         launch_maxpool_fwd(buf_of(nd.in), map_for(nd.in, ns), c, n_static, nd.g.H, nd.g.W, nd.g.Cin, nd.pk, nd.ps,
                            nd.pp, nd.g.Ho, nd.g.Wo, T[nd.out].buf, train ? nd.argmax.as<uint8_t>() : nullptr,
                            nd.in > 0 && T[nd.in].act == 1, st);
@@ -712,9 +711,11 @@ void Model::infer(const bf16* x, const int* in_map, const int* in_count, int n_s
   if (n_static <= 0) return;
   if (n_static > max_batch) throw ShapeError("batch exceeds max_batch");
   const bf16* x0 = x;
+  bool in_s2d = false;
   const int* map0 = in_map;
   if (pack && !x_padded) {
-    ingest(x, in_map, in_count, n_static, st);
+    ingest(x, in_map, in_count, n_static, st, first_s2d);
+    in_s2d = first_s2d;
     x0 = packed_in.as<bf16>();
     map0 = nullptr;
   }
@@ -725,7 +726,7 @@ void Model::infer(const bf16* x, const int* in_map, const int* in_count, int n_s
     else
       launch_fill_i32(out.exit_counts, n_static, st);
   }
-  forward_nodes(x0, map0, in_count, n_static, false, taus, &out, st);
+  forward_nodes(x0, map0, in_count, n_static, false, taus, &out, st, in_s2d);
 }
 
 // ------------------------------------------------------------------------------------------------

@@ -72,6 +72,8 @@ struct NodeRt {
   bool gdense = false;         // grouped conv as one dense GEMM over a block-diagonal shadow (shuffle.cu)
   int shuf_g = 0;              // > 1: channel shuffle folded into the output channel order (shadow rows, bias)
   DevBuf bias_perm;            // shuf_g: bias in the physical (shuffled) order, rebuilt every forward
+  int fuse_pool = -1;          // inference: the 2x2/2 max-pool node computed by this conv's conv3_pool kernel
+  DevBuf wexp;                 // its expanded weights (conv3pool.cu), rebuilt from the shadow every forward
   DevBuf pool_sc;              // N_AVGPOOL (training): shortcut term of the block input, bf16 [max_batch][H][W][C]
   DevBuf wdw;                  // depthwise weights [taps][C] bf16, rebuilt from the shadow every forward
   long long w_off = 0, b_off = 0;
@@ -124,7 +126,7 @@ struct Model {
   bool stem_s2d = false;
   int stem_pool = -1;         // node index of the pool fused into the stem
   DevBuf stem_wprep;          // per-tap bf16 weights [16][2][64][8], rebuilt from the shadow every forward
-  int fused_pool0 = -1;       // inference: node index of the 2x2 pool fused into the first conv (convpool.cu)
+  bool first_s2d = false;     // inference: the first conv runs fused with its pool on the s2d-packed input (conv3pool.cu)
   // inference stage bookkeeping
   DevBuf pos, orig, counts, alive;  // pos/orig: [nstages][max_batch] int; counts [nstages] int
   DevBuf exit_ws;                   // fused exit kernel: ticket + look-back status words
@@ -143,7 +145,7 @@ struct Model {
 
   void build(const adainf_model_spec& s);
   void refresh_shadows(cudaStream_t st);
-  void ingest(const bf16* x, const int* map, const int* count, int n_static, cudaStream_t st);
+  void ingest(const bf16* x, const int* map, const int* count, int n_static, cudaStream_t st, bool s2d = false);
   void ensure_training();
   // inference of one (possibly routed / device-counted) batch
   void infer(const bf16* x, const int* in_map, const int* in_count, int n_static, const float* taus,
@@ -164,7 +166,7 @@ struct Model {
 
  private:
   void forward_nodes(const bf16* x0, const int* map0, const int* count0, int n_static, bool train, const float* taus,
-                     const adainf_model_out* out, cudaStream_t st);
+                     const adainf_model_out* out, cudaStream_t st, bool in_s2d = false);
 };
 
 struct App {
