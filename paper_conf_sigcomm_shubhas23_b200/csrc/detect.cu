@@ -359,44 +359,77 @@ void launch_det_route(const DetRouteArgs& a, void* ws, cudaStream_t st) {
 
 // ------------------------------------------------------------------------------------------------
 // crop-resize: dst[r][v][u][c] for routed detection r of edge e (c >= C zero-padded to cout_pad)
-__global__ void crop_kernel(const bf16* __restrict__ frames, int H, int W, int C, const float* __restrict__ det,
-                            const int32_t* __restrict__ route_idx, const int32_t* __restrict__ cnt, int edge, int cap,
-                            int ch, int cw, int cpad, bf16* __restrict__ dst) {
+// One crop per CTA row-band (grid.y = routed detection r, grid.x = band of output rows): the per-column
+// source coordinates (xl, xh, fx) of the crop are computed once into shared memory, each thread then emits two
+// horizontally adjacent output pixels per row (3-channel crops: 12 contiguous bytes = three 32-bit stores instead
+// of six 16-bit ones).  The per-pixel arithmetic is the oracle's, op for op (reading Q19): every value is bit-exact.
+constexpr int CROP_BANDS = 8, CROP_MAXW = 512;
+__global__ void __launch_bounds__(256) crop_kernel(const bf16* __restrict__ frames, int H, int W, int C,
+                                                   const float* __restrict__ det, const int32_t* __restrict__ route_idx,
+                                                   const int32_t* __restrict__ cnt, int edge, int cap, int ch, int cw,
+                                                   int cpad, bf16* __restrict__ dst) {
   const int r = blockIdx.y;
   if (r >= cnt[edge]) return;
+  __shared__ int s_xl[CROP_MAXW], s_xh[CROP_MAXW];
+  __shared__ float s_fx[CROP_MAXW];
   const int di = route_idx[(long long)edge * cap + r];
   const float* d = det + (long long)di * 9;
   const int f = (int)d[0];
   const float x0 = d[5], y0 = d[6], x1 = d[7], y1 = d[8];
   const float sxs = __fdiv_rn(__fsub_rn(x1, x0), (float)cw);
   const float sys = __fdiv_rn(__fsub_rn(y1, y0), (float)ch);
+  for (int u = threadIdx.x; u < cw; u += blockDim.x) {
+    float sx = __fsub_rn(__fadd_rn(x0, __fmul_rn(__fadd_rn((float)u, 0.5f), sxs)), 0.5f);
+    sx = fminf(fmaxf(sx, 0.f), (float)(W - 1));
+    const int xl = (int)floorf(sx);
+    s_xl[u] = xl;
+    s_xh[u] = min(xl + 1, W - 1);
+    s_fx[u] = __fsub_rn(sx, (float)xl);
+  }
+  __syncthreads();
   const bf16* fr = frames + (long long)f * H * W * C;
-  for (int pix = blockIdx.x * blockDim.x + threadIdx.x; pix < ch * cw; pix += gridDim.x * blockDim.x) {
-    const int v = pix / cw, u = pix - v * cw;
+  const int rows_per = (ch + CROP_BANDS - 1) / CROP_BANDS;
+  const int v0 = blockIdx.x * rows_per, v1 = min(ch, v0 + rows_per);
+  const int pairs = (cw + 1) / 2;
+  for (int idx = threadIdx.x; idx < (v1 - v0) * pairs; idx += blockDim.x) {
+    const int v = v0 + idx / pairs, u0 = 2 * (idx % pairs);
     float sy = __fsub_rn(__fadd_rn(y0, __fmul_rn(__fadd_rn((float)v, 0.5f), sys)), 0.5f);
     sy = fminf(fmaxf(sy, 0.f), (float)(H - 1));
     const int yl = (int)floorf(sy);
     const int yh = min(yl + 1, H - 1);
     const float fy = __fsub_rn(sy, (float)yl);
-    float sx = __fsub_rn(__fadd_rn(x0, __fmul_rn(__fadd_rn((float)u, 0.5f), sxs)), 0.5f);
-    sx = fminf(fmaxf(sx, 0.f), (float)(W - 1));
-    const int xl = (int)floorf(sx);
-    const int xh = min(xl + 1, W - 1);
-    const float fx = __fsub_rn(sx, (float)xl);
-    const float wx0 = __fsub_rn(1.0f, fx), wy0 = __fsub_rn(1.0f, fy);
-    bf16* o = dst + ((long long)r * ch * cw + pix) * cpad;
-    for (int c = 0; c < cpad; ++c) {
-      float val = 0.f;
-      if (c < C) {
-        const float p00 = __bfloat162float(fr[((long long)yl * W + xl) * C + c]);
-        const float p01 = __bfloat162float(fr[((long long)yl * W + xh) * C + c]);
-        const float p10 = __bfloat162float(fr[((long long)yh * W + xl) * C + c]);
-        const float p11 = __bfloat162float(fr[((long long)yh * W + xh) * C + c]);
-        const float top = __fadd_rn(__fmul_rn(wx0, p00), __fmul_rn(fx, p01));
-        const float bot = __fadd_rn(__fmul_rn(wx0, p10), __fmul_rn(fx, p11));
-        val = __fadd_rn(__fmul_rn(wy0, top), __fmul_rn(fy, bot));
+    const float wy0 = __fsub_rn(1.0f, fy);
+    const bf16* rl = fr + (long long)yl * W * C;
+    const bf16* rh = fr + (long long)yh * W * C;
+    __align__(4) bf16 out[2 * 4];
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+      const int u = min(u0 + k, cw - 1);
+      const int xl = s_xl[u], xh = s_xh[u];
+      const float fx = s_fx[u];
+      const float wx0 = __fsub_rn(1.0f, fx);
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        if (c >= cpad) break;
+        float val = 0.f;
+        if (c < C) {
+          const float p00 = __bfloat162float(rl[xl * C + c]);
+          const float p01 = __bfloat162float(rl[xh * C + c]);
+          const float p10 = __bfloat162float(rh[xl * C + c]);
+          const float p11 = __bfloat162float(rh[xh * C + c]);
+          const float top = __fadd_rn(__fmul_rn(wx0, p00), __fmul_rn(fx, p01));
+          const float bot = __fadd_rn(__fmul_rn(wx0, p10), __fmul_rn(fx, p11));
+          val = __fadd_rn(__fmul_rn(wy0, top), __fmul_rn(fy, bot));
+        }
+        out[k * cpad + c] = __float2bfloat16_rn(val);
       }
-      o[c] = __float2bfloat16_rn(val);
+    }
+    bf16* o = dst + ((long long)r * ch * cw + (long long)v * cw + u0) * cpad;
+    const int nv = min(2, cw - u0) * cpad;  // values of this pixel pair
+    if (nv % 2 == 0 && (((uintptr_t)o) & 3) == 0) {
+      for (int q = 0; q < nv / 2; ++q) ((uint32_t*)o)[q] = ((const uint32_t*)out)[q];
+    } else {
+      for (int q = 0; q < nv; ++q) o[q] = out[q];
     }
   }
 }
@@ -404,7 +437,8 @@ __global__ void crop_kernel(const bf16* __restrict__ frames, int H, int W, int C
 void launch_crops(const bf16* frames, int H, int W, int C, const float* det_table, const int32_t* route_idx,
                   const int32_t* count_clamped, int edge, int cap, int crop_h, int crop_w, int cout_pad, bf16* dst,
                   cudaStream_t st) {
-  dim3 grid((crop_h * crop_w + 255) / 256, cap);
+  if (crop_w > CROP_MAXW || cout_pad > 4) throw ShapeError("crop: width <= 512 and <= 4 channels");
+  dim3 grid(CROP_BANDS, cap);
   ProfScope ps(PC_CROP, st);
   crop_kernel<<<grid, 256, 0, st>>>(frames, H, W, C, det_table, route_idx, count_clamped, edge, cap, crop_h, crop_w,
                                      cout_pad, dst);
