@@ -25,9 +25,9 @@ _SRC = os.path.join(_HERE, "oracle.cpp")
 _lock = threading.Lock()
 _lib = None
 
-OR_CONV, OR_MAXPOOL, OR_BLOCK, OR_EXIT, OR_DET_HEAD, OR_SHUFFLE = 0, 1, 2, 3, 4, 5
+OR_CONV, OR_MAXPOOL, OR_BLOCK, OR_EXIT, OR_DET_HEAD, OR_SHUFFLE, OR_UPSAMPLE, OR_ROUTE = 0, 1, 2, 3, 4, 5, 6, 7
 _KIND = {"conv": OR_CONV, "maxpool": OR_MAXPOOL, "block": OR_BLOCK, "exit": OR_EXIT, "det_head": OR_DET_HEAD,
-         "shuffle": OR_SHUFFLE}
+         "shuffle": OR_SHUFFLE, "upsample": OR_UPSAMPLE, "route": OR_ROUTE}
 
 
 class OrOp(C.Structure):
@@ -165,14 +165,20 @@ class Model:
                 break
         pooled0 = np.zeros((B, max(c0, 1)), np.float32)
         det = None
+        heads = []
         if want_det:
-            di = [i for i, o in enumerate(self.spec["ops"]) if o["kind"] == "det_head"][0]
-            G, _, CH = self.tensor_shape(di)
-            det = np.zeros((B, G, G, CH), np.float32)
+            heads = [self.tensor_shape(i) for i, o in enumerate(self.spec["ops"]) if o["kind"] == "det_head"]
+            det = np.zeros((B, sum(G * G2 * CH for G, G2, CH in heads)), np.float32)
         rc = lib().or_forward(C.byref(self.m), _p(params, C.c_float), _p(x, C.c_float), B,
                               _p(conf, C.c_float), _p(ent, C.c_float), _p(pred, C.c_int32),
                               _p(logits, C.c_float), _p(pooled0, C.c_float), _p(det, C.c_float))
         assert rc == 0, rc
+        if want_det:  # per head [B, G, G, A*(5+nc)], op order; a single head is returned as the array itself
+            outs, o = [], 0
+            for G, G2, CH in heads:
+                outs.append(det[:, o:o + G * G2 * CH].reshape(B, G, G2, CH).copy())
+                o += G * G2 * CH
+            det = outs[0] if len(outs) == 1 else outs
         return dict(conf=conf, ent=ent, pred=pred, logits=logits, pooled0=pooled0, det=det)
 
     def retrain_step(self, params, mom, x, labels, n_global=None, lr=0.01, mu=0.9, wd=0.0):
@@ -276,6 +282,26 @@ def detect(raw, anchors, nc, anchor_wh, stride, img_w, img_h, tau_det, max_det=1
     n = lib().or_detect(_p(raw, C.c_float), B, G, anchors, nc, _p(aw, C.c_float), stride, img_w, img_h,
                         tau_det, _p(det, C.c_float), max_det)
     return det[:min(n, max_det)].copy(), int(n)
+
+
+def detect_multi(raws, anchors, nc, anchor_whs, strides, img_w, img_h, tau_det, max_det=1 << 20):
+    """Two-scale TinyYOLOv3 decode (NEXT-3, reading Q18c): each head decoded by or_detect on its own grid, the cell
+    column re-based to the frame's concatenated cell space (head h's cells follow the G_i^2 cells of heads i < h),
+    rows merged in ascending candidate index ((frame * sum_h G_h^2 + cell) * A + anchor): a stable sort as a step."""
+    rows, off = [], 0
+    cpf = sum(int(r.shape[1]) * int(r.shape[2]) for r in raws)
+    total = 0
+    for r, aw, st in zip(raws, anchor_whs, strides):
+        d, n = detect(r, anchors, nc, aw, st, img_w, img_h, tau_det, max_det)
+        total += n
+        d = d.copy()
+        d[:, 1] += off
+        rows.append(d)
+        off += int(r.shape[1]) * int(r.shape[2])
+    det = np.concatenate(rows, 0) if rows else np.zeros((0, 9), np.float32)
+    key = (det[:, 0].astype(np.int64) * cpf + det[:, 1].astype(np.int64)) * anchors + det[:, 2].astype(np.int64)
+    order = np.argsort(key, kind="stable")
+    return det[order][:max_det].copy(), int(total)
 
 
 def nms(det, iou_thr):

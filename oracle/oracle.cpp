@@ -146,6 +146,8 @@ struct Walk {
   vector<Shape3> in_shape;   // per op: shape of the current tensor entering the op
   vector<Shape3> out_shape;  // per op: shape of its output (CONV/MAXPOOL), shortcut (BLOCK), input (EXIT)
   vector<int64_t> poff;      // per op: parameter offset
+  vector<Shape3> cur_after;  // per op: the current tensor after the op (ROUTE sources)
+  bool inference_only = false;  // UPSAMPLE / ROUTE present
   int64_t nparams = 0;
   int nexits = 0;
   int ncls = 0;
@@ -160,6 +162,11 @@ Walk walk(const or_model* m) {
     const or_op& op = m->ops[i];
     w.in_shape.push_back(cur);
     w.poff.push_back(w.nparams);
+    struct After {  // record the current tensor after this op, whichever branch ran
+      Walk& w;
+      Shape3& cur;
+      ~After() { w.cur_after.push_back(cur); }
+    } after{w, cur};
     switch (op.kind) {
       case OR_CONV: {
         Shape3 o{(cur.H + 2 * op.pad - op.kh) / op.stride + 1, (cur.W + 2 * op.pad - op.kw) / op.stride + 1,
@@ -223,6 +230,30 @@ Walk walk(const or_model* m) {
       case OR_DET_HEAD:
         w.out_shape.push_back(cur);
         break;
+      case OR_UPSAMPLE: {
+        if (op.stride < 1) w.ok = false;
+        cur = Shape3{cur.H * op.stride, cur.W * op.stride, cur.C};
+        w.out_shape.push_back(cur);
+        w.inference_only = true;
+        break;
+      }
+      case OR_ROUTE: {
+        if (op.kh < 0 || op.kh >= i || op.kw >= i) {
+          w.ok = false;
+          w.out_shape.push_back(cur);
+          break;
+        }
+        Shape3 o = w.cur_after[op.kh];
+        if (op.kw >= 0) {
+          const Shape3 b = w.cur_after[op.kw];
+          if (b.H != o.H || b.W != o.W) w.ok = false;
+          o.C += b.C;
+        }
+        cur = o;
+        w.out_shape.push_back(o);
+        w.inference_only = true;
+        break;
+      }
       default:
         w.ok = false;
         w.out_shape.push_back(cur);
@@ -268,7 +299,8 @@ struct Engine {
   vector<Node> nodes;
   vector<int> exit_tensor, exit_op;  // per exit
   vector<vector<double>> pooled, logits;
-  int det_tensor = -1;
+  vector<int> det_tensors;  // DET_HEAD inputs, op order
+  vector<int> op_tensor;    // current tensor after each op (ROUTE sources)
 
   // conv with weights taken from params (bf16-rounded unless exact)
   // grouped conv (groups = 1: dense): output channel co reads input channels [g*Cg, (g+1)*Cg) of its group
@@ -316,6 +348,8 @@ struct Engine {
     in.d.resize((size_t)in.H * in.W * in.C);
     for (size_t i = 0; i < in.d.size(); ++i) in.d[i] = exact ? (double)x[i] : (double)or_bf16(x[i]);
     T.push_back(std::move(in));
+    det_tensors.clear();
+    op_tensor.clear();
     int cur = 0;
     vector<int> blocks;
     for (int i = 0; i < m->n_ops; ++i) {
@@ -458,8 +492,40 @@ struct Engine {
         exit_tensor.push_back(cur);
         exit_op.push_back(i);
       } else if (op.kind == OR_DET_HEAD) {
-        det_tensor = cur;
+        det_tensors.push_back(cur);
+      } else if (op.kind == OR_UPSAMPLE) {  // nearest: Y[h][w] = X[h / s][w / s]
+        const Tensor& X = T[cur];
+        Tensor Y;
+        Y.H = X.H * op.stride;
+        Y.W = X.W * op.stride;
+        Y.C = X.C;
+        Y.d.resize((size_t)Y.H * Y.W * Y.C);
+        for (int h = 0; h < Y.H; ++h)
+          for (int ww = 0; ww < Y.W; ++ww)
+            for (int c = 0; c < Y.C; ++c)
+              Y.d[((size_t)h * Y.W + ww) * Y.C + c] = X.d[((size_t)(h / op.stride) * X.W + ww / op.stride) * X.C + c];
+        T.push_back(std::move(Y));
+        cur = (int)T.size() - 1;
+      } else if (op.kind == OR_ROUTE) {  // [output of op kh, output of op kw] along channels
+        const int ta = op_tensor[op.kh];
+        if (op.kw < 0) {
+          cur = ta;
+        } else {
+          const int tb = op_tensor[op.kw];
+          Tensor Y;
+          Y.H = T[ta].H;
+          Y.W = T[ta].W;
+          Y.C = T[ta].C + T[tb].C;
+          Y.d.resize((size_t)Y.H * Y.W * Y.C);
+          for (int e = 0; e < Y.H * Y.W; ++e) {
+            for (int c = 0; c < T[ta].C; ++c) Y.d[(size_t)e * Y.C + c] = T[ta].d[(size_t)e * T[ta].C + c];
+            for (int c = 0; c < T[tb].C; ++c) Y.d[(size_t)e * Y.C + T[ta].C + c] = T[tb].d[(size_t)e * T[tb].C + c];
+          }
+          T.push_back(std::move(Y));
+          cur = (int)T.size() - 1;
+        }
       }
+      op_tensor.push_back(cur);
     }
   }
 
@@ -682,11 +748,14 @@ extern "C" int or_forward(const or_model* m, const float* params, const float* x
       for (int c = 0; c < C0; ++c) pooled0[(int64_t)n * C0 + c] = (float)eng.pooled[0][c];
     }
     if (det_raw) {
-      if (eng.det_tensor < 0) {
+      if (eng.det_tensors.empty()) {
         rc = -2;
       } else {
-        const auto& t = eng.T[eng.det_tensor];
-        for (size_t e = 0; e < t.d.size(); ++e) det_raw[(int64_t)n * t.d.size() + e] = (float)t.d[e];
+        size_t per = 0;
+        for (int t : eng.det_tensors) per += eng.T[t].d.size();
+        size_t o = (size_t)n * per;
+        for (int t : eng.det_tensors)
+          for (double v : eng.T[t].d) det_raw[o++] = (float)v;
       }
     }
   }
@@ -895,7 +964,7 @@ extern "C" int32_t or_select(const float* X, int64_t N, int D, const float* Wp, 
 static int grads_of(const or_model* m, const double* params, const float* x, const int32_t* labels, int n,
                     int64_t n_global, bool exact, vector<double>& g, double* loss) {
   Walk w = walk(m);
-  if (!w.ok) return -1;
+  if (!w.ok || w.inference_only) return -1;  // detectors (UPSAMPLE / ROUTE) are not retrained
   g.assign(w.nparams, 0.0);
   const int64_t in_sz = (int64_t)m->in_h * m->in_w * m->in_c;
   const double inv_n = 1.0 / (double)n_global;

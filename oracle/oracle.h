@@ -23,7 +23,12 @@ extern "C" {
 #endif
 
 /* Op kinds of the oracle's own model description (same meaning as the ABI's, declared separately). */
-enum { OR_CONV = 0, OR_MAXPOOL = 1, OR_BLOCK = 2, OR_EXIT = 3, OR_DET_HEAD = 4, OR_SHUFFLE = 5 };
+enum { OR_CONV = 0, OR_MAXPOOL = 1, OR_BLOCK = 2, OR_EXIT = 3, OR_DET_HEAD = 4, OR_SHUFFLE = 5, OR_UPSAMPLE = 6,
+       OR_ROUTE = 7 };
+/* UPSAMPLE: nearest-neighbour x`stride` of the current tensor.  ROUTE (TinyYOLOv3's two-scale branch): the current
+ * tensor becomes the output of op `kh` (absolute op index), concatenated along channels with the output of op `kw`
+ * when kw >= 0 (same H, W).  Models with UPSAMPLE / ROUTE are inference-only (the detector is not retrained).
+ * Several DET_HEADs may appear; det_raw then holds, per frame, each head's G*G*(A*(5+nc)) values in op order. */
 
 typedef struct {
   int32_t kind;

@@ -70,6 +70,16 @@ def block(cout=0, stride=1, pool=0, k=3, pad=1):
     return {"kind": "block", "cout": cout, "stride": stride}
 
 
+def upsample(factor=2):
+    """nearest-neighbour upsampling (TinyYOLOv3's second scale)"""
+    return {"kind": "upsample", "stride": factor}
+
+
+def route(a, b=-1):
+    """current tensor := output of op a (absolute op index), concatenated with op b's along channels if b >= 0"""
+    return {"kind": "route", "kh": a, "kw": b}
+
+
 def shuffle(groups):
     """ShuffleNet channel shuffle (view (g, C/g) -> transpose -> flatten)"""
     return {"kind": "shuffle", "groups": groups}
@@ -159,6 +169,7 @@ def _walk(spec):
     shortcut's shape as the output.  A CONV with residual 2 concatenates the open block's shortcut channels."""
     H, W, Cc = spec["in_h"], spec["in_w"], spec["in_c"]
     blocks = []
+    after = []  # the current tensor after each op (ROUTE sources)
     for i, o in enumerate(spec["ops"]):
         k = o["kind"]
         if k == "conv":
@@ -176,6 +187,15 @@ def _walk(spec):
             Wo = (W + 2 * o["pad"] - o["kw"]) // o["stride"] + 1
             yield i, o, H, W, Cc, Ho, Wo, Cc
             H, W = Ho, Wo
+        elif k == "upsample":
+            yield i, o, H, W, Cc, H * o["stride"], W * o["stride"], Cc
+            H, W = H * o["stride"], W * o["stride"]
+        elif k == "route":
+            Ho, Wo, Co = after[o["kh"]]
+            if o.get("kw", -1) >= 0:
+                Co += after[o["kw"]][2]
+            yield i, o, H, W, Cc, Ho, Wo, Co
+            H, W, Cc = Ho, Wo, Co
         elif k == "block":
             if o["cout"] > 0:
                 Ho, Wo, Co = (H - 1) // o["stride"] + 1, (W - 1) // o["stride"] + 1, o["cout"]
@@ -189,6 +209,26 @@ def _walk(spec):
             yield i, o, H, W, Cc, Ho, Wo, Co
         else:
             yield i, o, H, W, Cc, H, W, Cc
+        after.append((H, W, Cc))
+
+
+YOLO_ANCHORS_26 = [10.0, 14.0, 23.0, 27.0, 37.0, 58.0]  # TinyYOLOv3's 26x26-scale anchors (w, h), pixels
+
+
+def tiny_yolo_det2(in_hw=416, det_classes=2, anchors=3, width=512, nms_iou=0.45):
+    """Two-scale TinyYOLOv3-like detector (NEXT-3, reading Q18c): the single-scale network (13x13 head, stride 32)
+    plus TinyYOLOv3's second branch -- route from the 13x13 1x1-256 conv, 1x1 conv 128, x2 nearest upsample, concat
+    with the 26x26x256 conv output, 3x3 conv 256, 1x1 head at stride 16 with the 26x26 anchors; detections of both
+    scales merged in candidate order and NMS'd together per (frame, class)."""
+    base = tiny_yolo_det(in_hw=in_hw, det_classes=det_classes, anchors=anchors, width=width, nms_iou=nms_iou)
+    ops = list(base["ops"])
+    ch = anchors * (5 + det_classes)
+    assert ops[8]["kind"] == "conv" and ops[13]["kind"] == "conv" and ops[13]["kh"] == 1
+    ops += [route(13), conv(1, 128, act=LEAKY), upsample(2), route(19, 8), conv(3, 256, act=LEAKY),
+            conv(1, ch, act=NONE),
+            {"kind": "det_head", "anchors": anchors, "det_classes": det_classes, "grid_stride": 16,
+             "anchor_wh": YOLO_ANCHORS_26[:2 * anchors], "nms_iou": nms_iou}]
+    return {"name": "tiny_yolo_det2", "in_h": in_hw, "in_w": in_hw, "in_c": 3, "ops": ops}
 
 
 def num_params(spec) -> int:

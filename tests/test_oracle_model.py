@@ -75,9 +75,11 @@ def torch_forward(spec, params, x, exact, want_det=False):
         return params[off:off + int(np.prod(shp))].reshape(shp)
 
     cur = R(x.permute(0, 3, 1, 2))
-    blocks, outs, det = [], [], None
+    blocks, outs, dets, after = [], [], [], []
     ops = spec["ops"]
     for i, o in enumerate(ops):
+        if i > 0:
+            after.append(cur)
         k = o["kind"]
         if k == "conv":
             w = R(seg("conv_w", i).permute(0, 3, 1, 2))
@@ -118,7 +120,12 @@ def torch_forward(spec, params, x, exact, want_det=False):
             pooled = Fp(cur.mean(dim=(2, 3)))
             outs.append(Fp(pooled @ seg("exit_w", i) + seg("exit_b", i)))
         elif k == "det_head":
-            det = cur.permute(0, 2, 3, 1)
+            dets.append(cur.permute(0, 2, 3, 1))
+        elif k == "upsample":
+            cur = cur.repeat_interleave(o["stride"], dim=2).repeat_interleave(o["stride"], dim=3)
+        elif k == "route":
+            cur = after[o["kh"]] if o.get("kw", -1) < 0 else torch.cat([after[o["kh"]], after[o["kw"]]], dim=1)
+    det = dets[0] if len(dets) == 1 else (dets or None)
     return (outs, det) if want_det else outs
 
 
@@ -138,6 +145,18 @@ def det_spec():
            S.conv(1, 16, act=S.LEAKY), S.conv(3, 16, act=S.LEAKY), S.conv(1, 2 * (5 + 2), act=S.NONE),
            {"kind": "det_head", "anchors": 2, "det_classes": 2, "grid_stride": 2, "anchor_wh": [3.0, 4.0, 6.0, 5.0]}]
     return {"name": "det", "in_h": 12, "in_w": 12, "in_c": 3, "ops": ops}
+
+
+def det2_spec():
+    """TinyYOLOv3's two-scale structure in miniature (NEXT-3, reading Q18c): route back to an earlier 1x1 conv,
+    1x1 conv, x2 nearest upsample, concat with a higher-resolution feature, second fp32 head"""
+    ops = [S.conv(3, 8, act=S.LEAKY), S.maxpool(2, 2), S.conv(3, 16, act=S.LEAKY), S.maxpool(2, 2),
+           S.conv(1, 16, act=S.LEAKY), S.conv(3, 16, act=S.LEAKY), S.conv(1, 2 * (5 + 2), act=S.NONE),
+           {"kind": "det_head", "anchors": 2, "det_classes": 2, "grid_stride": 4, "anchor_wh": [3.0, 4.0, 6.0, 5.0]},
+           S.route(4), S.conv(1, 8, act=S.LEAKY), S.upsample(2), S.route(10, 2), S.conv(3, 8, act=S.LEAKY),
+           S.conv(1, 2 * (5 + 2), act=S.NONE),
+           {"kind": "det_head", "anchors": 2, "det_classes": 2, "grid_stride": 2, "anchor_wh": [1.0, 2.0, 2.0, 1.5]}]
+    return {"name": "det2", "in_h": 12, "in_w": 12, "in_c": 3, "ops": ops}
 
 
 def mnv2_spec():
@@ -184,6 +203,25 @@ def test_forward_vs_torch_interpreter(which):
         np.testing.assert_allclose(got["logits"][:, k, :], lg.numpy(), rtol=2e-3, atol=2e-3)
         pr = torch.softmax(lg, 1)
         np.testing.assert_allclose(got["conf"][:, k], pr.max(1).values.numpy(), rtol=1e-3, atol=1e-3)
+
+
+def test_forward_two_scale_detector_vs_torch_interpreter():
+    """UPSAMPLE (nearest x2) and ROUTE (single source and channel concat of an upsampled branch with an earlier
+    feature map), two fp32 DET_HEADs: det_raw per head against the torch interpreter; the oracle refuses to retrain
+    such a model (the detector is not retrained)."""
+    spec = det2_spec()
+    p = synth.init_params(spec, seed=14)
+    xb, y = synth.drifted_images(3, 12, 12, 3, num_classes=4, seed=16)
+    x = synth.bf16_bits_to_f32(xb)
+    got = O.Model(spec).forward(p, x, want_det=True)["det"]
+    _, dets = torch_forward(spec, torch.from_numpy(p.astype(np.float64)), torch.from_numpy(x.astype(np.float64)),
+                            False, want_det=True)
+    assert len(got) == 2 and got[0].shape == (3, 3, 3, 14) and got[1].shape == (3, 6, 6, 14)
+    for g, r in zip(got, dets):
+        r = r.numpy()
+        assert np.linalg.norm(g - r) <= 1e-3 * np.linalg.norm(r)
+    with pytest.raises(AssertionError):
+        O.Model(spec).retrain_step(p, np.zeros_like(p), x, y.astype(np.int32) % 2, lr=0.0)
 
 
 def test_forward_detector_vs_torch_interpreter():

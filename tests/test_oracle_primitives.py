@@ -164,6 +164,45 @@ def test_detect_closed_forms():
     assert O.detect(raw, A, NC, aw, stride, 96, 96, tau_det=0.99)[1] == 0
 
 
+def test_detect_multi_two_scales_brute_force():
+    """Two-scale decode (NEXT-3, reading Q18c) against a plain per-candidate loop written from the definition: each
+    head's own stride and anchors, the cell index re-based past the earlier heads' cells, rows in ascending
+    (frame, head, cell, anchor) order; a swapped stride or anchor set, or a missing re-base, fails here."""
+    rng = np.random.default_rng(7)
+    A, NC, B = 2, 3, 3
+    heads = [(3, 32, [30.0, 40.0, 90.0, 70.0]), (6, 16, [8.0, 10.0, 14.0, 20.0])]
+    raws = [rng.normal(0, 1.5, (B, G, G, A * (5 + NC))).astype(np.float32) for G, _, _ in heads]
+    img = 96
+    sig = lambda v: 1.0 / (1.0 + math.exp(-float(v)))
+    exp_rows, scores = [], []
+    for f in range(B):
+        off = 0
+        for (G, st, aw), raw in zip(heads, raws):
+            for r in range(G):
+                for c in range(G):
+                    for a in range(A):
+                        v = raw[f, r, c, a * (5 + NC):(a + 1) * (5 + NC)]
+                        cs = int(np.argmax(v[5:]))
+                        sc = sig(v[4]) * sig(v[5 + cs])
+                        scores.append(sc)
+                        cx, cy = (c + sig(v[0])) * st, (r + sig(v[1])) * st
+                        w, h = aw[2 * a] * math.exp(min(v[2], 4.0)), aw[2 * a + 1] * math.exp(min(v[3], 4.0))
+                        box = [min(max(cx - w / 2, 0), img), min(max(cy - h / 2, 0), img),
+                               min(max(cx + w / 2, 0), img), min(max(cy + h / 2, 0), img)]
+                        exp_rows.append((f, off + r * G + c, a, cs, sc, *box))
+            off += G * G
+    s_sorted = np.sort(scores)
+    lo, hi = int(0.6 * len(s_sorted)), int(0.9 * len(s_sorted))  # widest gap between the 60th and 90th percentile
+    gi = np.argmax(np.diff(s_sorted[lo:hi])) + lo
+    tau = float(0.5 * (s_sorted[gi] + s_sorted[gi + 1]))
+    want = [r for r in exp_rows if r[4] >= tau]
+    det, n = O.detect_multi(raws, A, NC, [h[2] for h in heads], [h[1] for h in heads], img, img, tau)
+    assert n == len(want) == det.shape[0] > 3
+    for got, w in zip(det, want):
+        assert tuple(int(v) for v in got[:4]) == w[:4]
+        np.testing.assert_allclose(got[4:], w[4:], rtol=1e-5, atol=1e-3)
+
+
 def test_crop_identity_constant_and_grid_sample():
     rng = np.random.default_rng(2)
     H, W, Cc = 12, 10, 3
