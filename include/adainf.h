@@ -64,6 +64,13 @@ typedef void* adainf_stream_t; /* cudaStream_t (NULL = legacy default stream) */
  *            close that block; residual=2: close it by concatenating [shortcut, conv] along channels, act
  *            applied to both parts (ShuffleNet stride-2 unit; output channels = shortcut's + cout).
  *            A CONV directly followed by DET_HEAD writes fp32 (no bf16 rounding).
+ *   UPSAMPLE nearest-neighbour x`stride` of the current tensor (TinyYOLOv3's second scale); must feed a ROUTE.
+ *   ROUTE    the current tensor becomes the output of op `kh` (absolute op index), concatenated along channels with
+ *            op `kw`'s output when kw >= 0 (same H, W; only the first source may be an UPSAMPLE).  Models with
+ *            UPSAMPLE / ROUTE are inference-only (detectors are not retrained): retraining them returns
+ *            ADAINF_ERR_UNSUPPORTED.  A second DET_HEAD (same anchors per cell, classes, nms_iou) adds a scale: its
+ *            grid cells follow the first head's in each frame's candidate order (det_table `cell` column), and NMS
+ *            runs over both scales together (two-scale TinyYOLOv3, NEXT-3, reading Q18c).
  *   SHUFFLE  ShuffleNet channel shuffle of the current tensor with `groups` g (view (g, C/g), transpose,
  *            flatten; NEXT-3).  It must directly follow a non-depthwise CONV whose output has no other
  *            reader yet: the permutation is folded into that conv's output channel order (weights and bias),
@@ -89,7 +96,9 @@ typedef enum {
   ADAINF_OP_BLOCK = 2,
   ADAINF_OP_EXIT = 3,
   ADAINF_OP_DET_HEAD = 4,
-  ADAINF_OP_SHUFFLE = 5
+  ADAINF_OP_SHUFFLE = 5,
+  ADAINF_OP_UPSAMPLE = 6,
+  ADAINF_OP_ROUTE = 7
 } adainf_op_kind;
 
 typedef struct {

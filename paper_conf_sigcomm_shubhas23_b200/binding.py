@@ -15,7 +15,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libadainf.so")
 
 OK, ERR_INVALID, ERR_SHAPE, ERR_CAPACITY, ERR_OOM, ERR_CUDA, ERR_NCCL, ERR_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6, -7
-_OPKIND = {"conv": 0, "maxpool": 1, "block": 2, "exit": 3, "det_head": 4, "shuffle": 5}
+_OPKIND = {"conv": 0, "maxpool": 1, "block": 2, "exit": 3, "det_head": 4, "shuffle": 5, "upsample": 6, "route": 7}
 ROUTE_DET_CROP, ROUTE_CLASS_WHOLE = 0, 1
 
 

@@ -177,9 +177,10 @@ extern "C" adainf_status adainf_app_create(const adainf_app_spec* spec, adainf_a
         S.pred.alloc((size_t)m->max_batch * 4);
         if (m->det.tensor >= 0) {
           const TensorRt& D = m->T[m->det.tensor];
-          const size_t ncand = (size_t)m->max_batch * D.H * D.W * m->det.anchors;
+          const int cpf = D.H * D.W + (m->det.tensor2 >= 0 ? m->T[m->det.tensor2].H * m->T[m->det.tensor2].W : 0);
+          const size_t ncand = (size_t)m->max_batch * cpf * m->det.anchors;
           S.det_table.alloc(ncand * 9 * 4);
-          S.det_ws.alloc(det_route_ws_bytes(m->max_batch, D.H, m->det.anchors, m->det.nms_iou > 0.f));
+          S.det_ws.alloc(det_route_ws_bytes(m->max_batch, cpf, m->det.anchors, m->det.nms_iou > 0.f));
           const int ne = std::max<int>(1, (int)S.det_edges.size());
           S.n_det.alloc(16);
           S.route_idx.alloc((size_t)ne * std::max(1, a.max_routed) * 4);
@@ -273,6 +274,13 @@ extern "C" adainf_status adainf_infer_dag(adainf_app_t app, const void* batch, i
         d.img_w = m->in_w;
         d.img_h = m->in_h;
         memcpy(d.anchor_wh, m->det.anchor_wh, sizeof(d.anchor_wh));
+        if (m->det.tensor2 >= 0) {  // second scale: its cells follow the first head's in each frame
+          const TensorRt& D2 = m->T[m->det.tensor2];
+          d.raw2 = (const float*)D2.buf;
+          d.G2 = D2.H;
+          d.stride2 = m->det.stride2;
+          memcpy(d.anchor_wh2, m->det.anchor_wh2, sizeof(d.anchor_wh2));
+        }
         d.tau = tau_of[i][0];
         d.n_edges = (int)S.det_edges.size();
         for (int q = 0; q < d.n_edges; ++q) d.edge_class[q] = a.edges[S.det_edges[q]].src_class;

@@ -23,13 +23,33 @@ struct Cand {
 
 __device__ __forceinline__ float sigmoidf_(float x) { return __fdiv_rn(1.0f, __fadd_rn(1.0f, expf(-x))); }
 
+// candidate i = (frame * CPF + cell) * A + anchor, CPF = G*G (+ G2*G2): cells of head 0 first, then head 1
+struct CandPos {
+  int f, head, row, col, cell, an;
+  const float* v;
+};
+__device__ __forceinline__ CandPos cand_pos(const DetRouteArgs& a, long long i) {
+  CandPos p;
+  const long long cpf = (long long)a.G * a.G + (long long)a.G2 * a.G2;
+  p.an = (int)(i % a.A);
+  const long long cg = i / a.A;
+  p.f = (int)(cg / cpf);
+  p.cell = (int)(cg - (long long)p.f * cpf);
+  p.head = p.cell >= a.G * a.G;
+  const int G = p.head ? a.G2 : a.G;
+  const int lc = p.head ? p.cell - a.G * a.G : p.cell;
+  p.row = lc / G;
+  p.col = lc - p.row * G;
+  const float* raw = p.head ? a.raw2 : a.raw;
+  p.v = raw + (((long long)p.f * G * G + lc) * a.A + p.an) * (5 + a.NC);
+  return p;
+}
+
 __device__ __forceinline__ Cand eval_cand(const DetRouteArgs& a, long long i, int nframes) {
   Cand c{false, 0};
-  const long long ncand = (long long)nframes * a.G * a.G * a.A;
+  const long long ncand = (long long)nframes * ((long long)a.G * a.G + (long long)a.G2 * a.G2) * a.A;
   if (i >= ncand) return c;
-  const int an = (int)(i % a.A);
-  const long long cell = i / a.A;  // (frame*G + row)*G + col
-  const float* v = a.raw + cell * (a.A * (5 + a.NC)) + an * (5 + a.NC);
+  const float* v = cand_pos(a, i).v;
   int cs = 0;
   for (int k = 1; k < a.NC; ++k)
     if (v[5 + k] > v[5 + cs]) cs = k;
@@ -117,20 +137,19 @@ __global__ void det_emit_kernel(const DetRouteArgs a, const int* __restrict__ bl
       int pre0 = run[0] + __popc(bal[0] & lt);
       for (int ww = 0; ww < w; ++ww) pre0 += wd[ww][0];
       {
-        const int an = (int)(i % a.A);
-        const long long cell = i / a.A;
-        const int col = (int)(cell % a.G);
-        const int row = (int)((cell / a.G) % a.G);
-        const int f = (int)(cell / ((long long)a.G * a.G));
-        const float* v = a.raw + cell * (a.A * (5 + a.NC)) + an * (5 + a.NC);
+        const CandPos cp = cand_pos(a, i);
+        const int an = cp.an, row = cp.row, col = cp.col, f = cp.f;
+        const float* v = cp.v;
+        const float stride = (float)(cp.head ? a.stride2 : a.stride);
+        const float* aw = cp.head ? a.anchor_wh2 : a.anchor_wh;
         const float score = __fmul_rn(sigmoidf_(v[4]), sigmoidf_(v[5 + c.cls]));
-        const float cx = __fmul_rn(__fadd_rn((float)col, sigmoidf_(v[0])), (float)a.stride);
-        const float cy = __fmul_rn(__fadd_rn((float)row, sigmoidf_(v[1])), (float)a.stride);
-        const float bw = __fmul_rn(a.anchor_wh[2 * an], expf(fminf(v[2], 4.f)));
-        const float bh = __fmul_rn(a.anchor_wh[2 * an + 1], expf(fminf(v[3], 4.f)));
+        const float cx = __fmul_rn(__fadd_rn((float)col, sigmoidf_(v[0])), stride);
+        const float cy = __fmul_rn(__fadd_rn((float)row, sigmoidf_(v[1])), stride);
+        const float bw = __fmul_rn(aw[2 * an], expf(fminf(v[2], 4.f)));
+        const float bh = __fmul_rn(aw[2 * an + 1], expf(fminf(v[3], 4.f)));
         float* d = a.det_table + (long long)pre0 * 9;
         d[0] = (float)f;
-        d[1] = (float)(row * a.G + col);
+        d[1] = (float)cp.cell;
         d[2] = (float)an;
         d[3] = (float)c.cls;
         d[4] = score;
@@ -304,8 +323,8 @@ __global__ void __launch_bounds__(1024) nms_route_kernel(const DetRouteArgs a, c
   }
 }
 
-size_t det_route_ws_bytes(int n_static, int G, int A, bool nms) {
-  const long long ncand = (long long)n_static * G * G * A;
+size_t det_route_ws_bytes(int n_static, int cells_per_frame, int A, bool nms) {
+  const long long ncand = (long long)n_static * cells_per_frame * A;
   const long long nb = (ncand + DET_PER_BLOCK - 1) / DET_PER_BLOCK;
   size_t b = (size_t)nb * (1 + MAX_EDGES) * sizeof(int) + 256;
   if (nms) b += 256 + (size_t)ncand * 9 * 4 + 256 + (size_t)ncand + 256 + 16;
@@ -314,7 +333,7 @@ size_t det_route_ws_bytes(int n_static, int G, int A, bool nms) {
 
 void launch_det_route(const DetRouteArgs& a, void* ws, cudaStream_t st) {
   if (a.n_edges > MAX_EDGES) throw ShapeError("at most 8 routing edges per detector");
-  const long long ncand = (long long)a.n_static * a.G * a.G * a.A;
+  const long long ncand = (long long)a.n_static * ((long long)a.G * a.G + (long long)a.G2 * a.G2) * a.A;
   const int nb = (int)((ncand + DET_PER_BLOCK - 1) / DET_PER_BLOCK);
   int* blk = (int*)ws;
   if (a.nms_iou > 0.f) {
@@ -331,7 +350,7 @@ void launch_det_route(const DetRouteArgs& a, void* ws, cudaStream_t st) {
     b.user_max = 0;
     b.n_det = n_pre;
     b.n_routed = nullptr;
-    const int per_frame = a.G * a.G * a.A;
+    const int per_frame = (a.G * a.G + a.G2 * a.G2) * a.A;
     int pow2 = 1;
     while (pow2 < per_frame) pow2 <<= 1;
     const size_t smem = (size_t)pow2 * (8 + 16 + 1) + 64;

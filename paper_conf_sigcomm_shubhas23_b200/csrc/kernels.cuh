@@ -63,6 +63,9 @@ void grouped_wgrad_gather(const float* dense, const float* dbs, int Cout, int ta
 void avgpool_fwd(const AvgPoolArgs& a, cudaStream_t st);
 void concat_fwd(const bf16* S, const bf16* Y, const int* count, int n_static, int HW, int Cs, int Co, int act, bf16* Z,
                 cudaStream_t st);
+// TinyYOLOv3 ROUTE of two sources: [A upsampled by f (nearest), B] along channels (inference)
+void route_concat(const bf16* A, int HA, int WA, int CA, int f, const bf16* B, int CB, const int* count, int n_static,
+                  int H, int W, bf16* out, cudaStream_t st);
 void concat_bwd(const bf16* dZ, int n, int H, int W, int Cs, int Co, int K, int s, int p, int Ho, int Wo, bf16* dY,
                 bf16* sc, cudaStream_t st);
 

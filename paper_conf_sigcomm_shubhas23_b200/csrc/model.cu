@@ -62,8 +62,72 @@ void Model::build(const adainf_model_spec& s) {
     if (o.kind == ADAINF_OP_EXIT) n_exit_ops++;
   int seen_exits = 0;
   long long off = 0;
+  std::vector<int> op_tensor;  // current tensor after each op (ROUTE sources)
   for (size_t i = 0; i < ops.size(); ++i) {
+    if (i > 0) op_tensor.push_back(cur);
     const adainf_op& o = ops[i];
+    if (T[cur].up_src >= 0 && o.kind != ADAINF_OP_ROUTE)
+      throw UnsupportedError("UPSAMPLE must feed a ROUTE (it is read through the concat, never materialised)");
+    if (o.kind == ADAINF_OP_UPSAMPLE) {
+      if (o.stride < 1 || o.stride > 8) throw ShapeError("upsample: factor in 1..8");
+      TensorRt V;
+      V.H = T[cur].H * o.stride;
+      V.W = T[cur].W * o.stride;
+      V.C = T[cur].C;
+      V.f32 = T[cur].f32;
+      V.stage = stage;
+      V.up_src = cur;
+      V.up = o.stride;
+      if (V.f32) throw UnsupportedError("upsample of an fp32 tensor");
+      T.push_back(std::move(V));
+      cur = (int)T.size() - 1;
+      inference_only = true;
+      continue;
+    }
+    if (o.kind == ADAINF_OP_ROUTE) {
+      if (o.kh < 0 || o.kh >= (int)i || o.kw >= (int)i) throw InvalidError("route: sources must be earlier ops");
+      const int ta = op_tensor[o.kh];
+      inference_only = true;
+      if (o.kw < 0) {  // the earlier output itself: an alias of its buffer
+        if (T[ta].up_src >= 0) throw UnsupportedError("route of an upsampled tensor alone");
+        TensorRt Z;
+        Z.H = T[ta].H;
+        Z.W = T[ta].W;
+        Z.C = T[ta].C;
+        Z.f32 = T[ta].f32;
+        Z.stage = stage;
+        Z.alias_of = T[ta].alias_of >= 0 ? T[ta].alias_of : ta;
+        T[Z.alias_of].routed = true;
+        T.push_back(std::move(Z));
+        cur = (int)T.size() - 1;
+        continue;
+      }
+      const int tb = op_tensor[o.kw];
+      const TensorRt& A = T[ta];
+      const TensorRt& Bt = T[tb];
+      if (Bt.up_src >= 0 || A.f32 || Bt.f32) throw UnsupportedError("route: only the first source may be upsampled");
+      if (A.H != Bt.H || A.W != Bt.W || A.C % 8 || Bt.C % 8) throw ShapeError("route: sources must share H, W");
+      NodeRt nd;
+      nd.kind = N_ROUTE;
+      nd.op = (int)i;
+      nd.in = ta;
+      nd.res = tb;
+      nd.stage = stage;
+      TensorRt Z;
+      Z.H = A.H;
+      Z.W = A.W;
+      Z.C = A.C + Bt.C;
+      Z.stage = stage;
+      Z.producer = (int)nodes.size();
+      T[A.up_src >= 0 ? A.up_src : (A.alias_of >= 0 ? A.alias_of : ta)].routed = true;
+      T[Bt.alias_of >= 0 ? Bt.alias_of : tb].routed = true;
+      T.push_back(std::move(Z));
+      nd.out = (int)T.size() - 1;
+      cur = nd.out;
+      op_node[i] = (int)nodes.size();
+      nodes.push_back(std::move(nd));
+      continue;
+    }
     if (o.kind == ADAINF_OP_BLOCK && o.cout <= 0 && o.pool) {
       // average-pool shortcut (ShuffleNet stride-2 unit): its own node and tensor, closed by a concat
       NodeRt nd;
@@ -280,6 +344,15 @@ void Model::build(const adainf_model_spec& s) {
       exits.push_back(std::move(e));
       seen_exits++;
       if (seen_exits < n_exit_ops) stage++;
+    } else if (o.kind == ADAINF_OP_DET_HEAD && det.tensor >= 0) {  // second scale (two-scale TinyYOLOv3)
+      if (!T[cur].f32) throw InvalidError("DET_HEAD must follow a conv");
+      if (det.tensor2 >= 0) throw UnsupportedError("at most two DET_HEADs");
+      if (o.anchors != det.anchors || o.det_classes != det.classes || o.nms_iou != det.nms_iou ||
+          T[cur].C != o.anchors * (5 + o.det_classes))
+        throw ShapeError("det_head: both scales share anchors per cell, classes and nms_iou");
+      det.tensor2 = cur;
+      det.stride2 = o.grid_stride;
+      memcpy(det.anchor_wh2, o.anchor_wh, sizeof(det.anchor_wh2));
     } else if (o.kind == ADAINF_OP_DET_HEAD) {
       if (!T[cur].f32) throw InvalidError("DET_HEAD must follow a conv");
       det.tensor = cur;
@@ -316,7 +389,7 @@ void Model::build(const adainf_model_spec& s) {
     const int po = Y.primary;
     if (po >= 0 && nodes[po].kind == N_POOL && nodes[po].pk == 3 && nodes[po].ps == 2 && nodes[po].pp == 1 &&
         nodes[po].stage == c0.stage && c0.act == 1 && !c0.fp32_out && c0.res < 0 && Y.exit_k < 0 &&
-        Y.res_of < 0 && Y.proj < 0 && stem_s2d_ok(in_h, in_w, in_c, c0.g.Cout, c0.g.KH, c0.g.KW, c0.g.stride, c0.g.pad)) {
+        Y.res_of < 0 && Y.proj < 0 && !Y.routed && stem_s2d_ok(in_h, in_w, in_c, c0.g.Cout, c0.g.KH, c0.g.KW, c0.g.stride, c0.g.pad)) {
       stem_s2d = true;
       stem_pool = po;
       pack = true;
@@ -334,7 +407,7 @@ void Model::build(const adainf_model_spec& s) {
       const TensorRt& Y = T[nd.out];
       const int po = Y.primary;
       if (po < 0 || nodes[po].kind != N_POOL || nodes[po].stage != nd.stage || Y.exit_k >= 0 || Y.res_of >= 0 ||
-          Y.proj >= 0 || Y.avgpool >= 0)
+          Y.proj >= 0 || Y.avgpool >= 0 || Y.routed)
         continue;
       const bool first = nd.in == 0;
       if (first && cin_pad != 4) continue;
@@ -348,6 +421,7 @@ void Model::build(const adainf_model_spec& s) {
   // activations
   for (size_t t = 1; t < T.size(); ++t) {
     if (stem_s2d && (int)t == nodes[0].out) continue;  // the fused stem never materialises its conv output
+    if (T[t].up_src >= 0 || T[t].alias_of >= 0) continue;  // upsampling views / route aliases own no memory
     const size_t b = (size_t)max_batch * T[t].row_elems() * (T[t].f32 ? 4 : 2);
     T[t].own.alloc(b);
     T[t].buf = T[t].own.as<bf16>();
@@ -355,6 +429,10 @@ void Model::build(const adainf_model_spec& s) {
   if (pack) {
     packed_in.alloc((size_t)max_batch * T[0].row_elems() * 2);
     T[0].buf = packed_in.as<bf16>();
+  }
+  for (size_t t = 1; t < T.size(); ++t) {
+    if (T[t].alias_of >= 0) T[t].buf = T[T[t].alias_of].buf;
+    if (T[t].up_src >= 0) T[t].buf = T[T[t].up_src].buf;
   }
   for (auto& nd : nodes)
     if (nd.kind == N_CONV || nd.kind == N_PROJ) {
@@ -479,6 +557,7 @@ void Model::refresh_shadows(cudaStream_t st) {
 void Model::ensure_training() {
   if (train_ready) return;
   if (exits.empty()) throw UnsupportedError("retraining needs an early-exit classifier (detector is not retrained, P:86)");
+  if (inference_only) throw UnsupportedError("UPSAMPLE / ROUTE models are inference-only (detectors, P:86)");
   for (size_t t = 1; t < T.size(); ++t) {
     if (T[t].f32) continue;
     T[t].own_grad.alloc((size_t)max_batch * T[t].row_elems() * 2);
@@ -572,6 +651,14 @@ void Model::forward_nodes(const bf16* x0, const int* map0, const int* count0, in
         conv3_pool(nd.g, nd.in == 0, buf_of(nd.in), c, n_static, nd.shadow.as<bf16>(), nd.ldb, nd.cin_real,
                    params.as<float>() + nd.b_off, nd.act, nd.wexp.as<bf16>(), T[pl.out].buf, st);
         pool_done[nd.fuse_pool] = 1;
+        continue;
+      }
+      if (nd.kind == N_ROUTE) {
+        const TensorRt& A = T[nd.in];
+        const TensorRt& Z = T[nd.out];
+        const int asrc = A.up_src >= 0 ? A.up_src : nd.in;
+        route_concat(buf_of(asrc), T[asrc].H, T[asrc].W, A.C, A.up_src >= 0 ? A.up : 1, buf_of(nd.res), T[nd.res].C, c,
+                     n_static, Z.H, Z.W, Z.buf, st);
         continue;
       }
       if (nd.kind == N_AVGPOOL) {

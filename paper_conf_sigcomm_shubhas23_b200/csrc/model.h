@@ -20,7 +20,8 @@
 namespace adainf {
 
 // N_AVGPOOL: a BLOCK's average-pool shortcut; N_CONCAT: [shortcut, conv] join closing such a block (ShuffleNet)
-enum NodeKind { N_CONV = 0, N_POOL = 1, N_PROJ = 2, N_AVGPOOL = 3, N_CONCAT = 4 };
+// N_ROUTE: TinyYOLOv3 route of two sources (concat, the first optionally read through an upsampling factor)
+enum NodeKind { N_CONV = 0, N_POOL = 1, N_PROJ = 2, N_AVGPOOL = 3, N_CONCAT = 4, N_ROUTE = 5 };
 
 struct DevBuf {  // owning device allocation
   void* p = nullptr;
@@ -57,6 +58,9 @@ struct TensorRt {
   int res_of = -1;       // conv node adding it as identity shortcut
   int exit_k = -1;       // exit attached
   int avgpool = -1;      // N_AVGPOOL node reading it as a block input (its shortcut term comes from there)
+  bool routed = false;   // read again by a ROUTE (inference-only detectors): its producer may not fuse it away
+  int alias_of = -1;     // single-source ROUTE: the same buffer as that tensor
+  int up_src = -1, up = 1;  // UPSAMPLE: virtual (never materialised) nearest x`up` view of tensor up_src
   size_t row_elems() const { return (size_t)H * W * C; }
 };
 
@@ -101,6 +105,8 @@ struct ExitRt {
 
 struct DetRt {
   int tensor = -1;
+  int tensor2 = -1, stride2 = 0;  // second head (two-scale TinyYOLOv3, NEXT-3)
+  float anchor_wh2[16];
   int anchors = 0, classes = 0, stride = 0;
   float anchor_wh[16];
   float nms_iou = 0.f;  // > 0: greedy NMS before routing (NEXT-3)
@@ -126,6 +132,7 @@ struct Model {
   bool stem_s2d = false;
   int stem_pool = -1;         // node index of the pool fused into the stem
   DevBuf stem_wprep;          // per-tap bf16 weights [16][2][64][8], rebuilt from the shadow every forward
+  bool inference_only = false;  // UPSAMPLE / ROUTE present (detectors are not retrained)
   bool first_s2d = false;     // inference: the first conv runs fused with its pool on the s2d-packed input (conv3pool.cu)
   // inference stage bookkeeping
   DevBuf pos, orig, counts, alive;  // pos/orig: [nstages][max_batch] int; counts [nstages] int
@@ -181,6 +188,11 @@ struct DetRouteArgs {
   const int* count;  // frames count (device) or nullptr
   int n_static, G, A, NC, stride, img_w, img_h;
   float anchor_wh[16];
+  // optional second head (two-scale TinyYOLOv3, NEXT-3): [B][G2][G2][A*(5+NC)], its cells follow the first
+  // head's G*G cells of the same frame in the candidate order
+  const float* raw2;
+  int G2, stride2;
+  float anchor_wh2[16];
   float tau;
   int n_edges;
   int edge_class[8];
@@ -195,7 +207,7 @@ struct DetRouteArgs {
   int32_t* cap_flag;
   float nms_iou;           // > 0: NMS between decode and routing
 };
-size_t det_route_ws_bytes(int n_static, int G, int A, bool nms);
+size_t det_route_ws_bytes(int n_static, int cells_per_frame, int A, bool nms);
 void launch_det_route(const DetRouteArgs& a, void* ws, cudaStream_t st);
 void launch_crops(const bf16* frames, int H, int W, int C, const float* det_table, const int32_t* route_idx,
                   const int32_t* count_clamped, int edge, int cap, int crop_h, int crop_w, int cout_pad, bf16* dst,

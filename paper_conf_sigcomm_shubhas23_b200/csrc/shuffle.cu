@@ -162,7 +162,37 @@ __global__ void avgpool_bwd_kernel(const bf16* __restrict__ dZ, int ldz, int n, 
   }
 }
 
+// ROUTE with two sources (TinyYOLOv3's second scale, NEXT-3): out[p] = [A(h / f, w / f), B(h, w)] along channels,
+// A read through its nearest-upsampling factor f (the UPSAMPLE op is never materialised)
+__global__ void route_concat_kernel(const bf16* __restrict__ A, int HA, int WA, int CA, int f, const bf16* __restrict__ Bt,
+                                    int CB, const int* count, int n_static, int H, int W, bf16* __restrict__ out) {
+  const int n_rows = count ? *count : n_static;
+  const int CZ = (CA + CB) >> 3;
+  const long long total = (long long)n_rows * H * W * CZ;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+    const int cz = (int)(i % CZ);
+    long long p = i / CZ;
+    const int w = (int)(p % W);
+    const long long q = p / W;
+    const int h = (int)(q % H);
+    const long long n = q / H;
+    uint4 v;
+    if (cz * 8 < CA) v = __ldg((const uint4*)(A + ((n * HA + h / f) * WA + w / f) * CA + cz * 8));
+    else v = __ldg((const uint4*)(Bt + p * CB + (cz * 8 - CA)));
+    *(uint4*)(out + p * (CA + CB) + cz * 8) = v;
+  }
+}
+
 }  // namespace
+
+void route_concat(const bf16* A, int HA, int WA, int CA, int f, const bf16* B, int CB, const int* count, int n_static,
+                  int H, int W, bf16* out, cudaStream_t st) {
+  const long long total = (long long)n_static * H * W * ((CA + CB) / 8);
+  if (total <= 0) return;
+  ProfScope ps(PC_SHUFFLE, st);
+  route_concat_kernel<<<grid_for(total), 256, 0, st>>>(A, HA, WA, CA, f, B, CB, count, n_static, H, W, out);
+  CK(cudaGetLastError());
+}
 
 void permute_bias(const float* b, int Cout, int g, float* out, cudaStream_t st) {
   ProfScope ps(PC_SHUFFLE, st);

@@ -174,26 +174,27 @@ def spread_exit_heads(spec: dict, params: np.ndarray, logits: np.ndarray, target
 
 def det_head_params(spec: dict, params: np.ndarray, obj_bias: float, seed: int = 0,
                     head_scale: float = 16.0, cls_bias=None) -> np.ndarray:
-    """Bias the detector's final 1x1 conv so the objectness logits sit near `obj_bias` (controls the
-    detection rate before tau_det calibration) and scale its weights by `head_scale`: the BN-free leaky
-    backbone's features are small (std ~0.1 at the head input), so the scale spreads the raw logits to
-    std ~1.5 and the scores / class margins over a realistic range (at 0.25 they bunched within 0.006 of
-    0.25 and the two class logits were near-ties)."""
+    """Bias each detector head's final 1x1 conv (the conv right before a det_head; two-scale detectors have two) so
+    the objectness logits sit near `obj_bias` (controls the detection rate before tau_det calibration) and scale its
+    weights by `head_scale`: the BN-free leaky backbone's features are small (std ~0.1 at the head input), so the
+    scale spreads the raw logits to std ~1.5 and the scores / class margins over a realistic range (at 0.25 they
+    bunched within 0.006 of 0.25 and the two class logits were near-ties)."""
     p = params.copy()
-    segs = S.param_segments(spec)
-    head = [s for s in segs if s[0] == "conv_b"][-1]
-    _, _, off, shp = head
-    A = next(o for o in spec["ops"] if o["kind"] == "det_head")
-    per = 5 + A["det_classes"]
-    for a in range(A["anchors"]):
-        p[off + a * per + 4] = obj_bias
-        if cls_bias is not None:  # class prior of the detections (e.g. vehicle : person ~ 3 : 1, SURVEY C3)
-            for c, v in enumerate(cls_bias):
-                p[off + a * per + 5 + c] = v
-    wseg = [s for s in segs if s[0] == "conv_w"][-1]
-    _, _, woff, wshp = wseg
-    cnt = int(np.prod(wshp))
-    p[woff:woff + cnt] *= np.float32(head_scale)
+    segs = {(k, i): (off, shp) for k, i, off, shp in S.param_segments(spec)}
+    ops = spec["ops"]
+    for hi, A in enumerate(ops):
+        if A["kind"] != "det_head":
+            continue
+        ci = hi - 1
+        per = 5 + A["det_classes"]
+        off, _ = segs[("conv_b", ci)]
+        for a in range(A["anchors"]):
+            p[off + a * per + 4] = obj_bias
+            if cls_bias is not None:  # class prior of the detections (e.g. vehicle : person ~ 3 : 1, SURVEY C3)
+                for c, v in enumerate(cls_bias):
+                    p[off + a * per + 5 + c] = v
+        woff, wshp = segs[("conv_w", ci)]
+        p[woff:woff + int(np.prod(wshp))] *= np.float32(head_scale)
     return p
 
 
