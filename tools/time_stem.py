@@ -4,6 +4,8 @@ import os, sys
 sys.path.insert(0, os.path.join(os.path.dirname(os.path.abspath(__file__)), ".."))
 import torch
 from paper_conf_sigcomm_shubhas23_b200 import binding as B
+if os.environ.get("ADAINF_LIB"):  # A/B against another build
+    B.LIB_PATH = os.environ["ADAINF_LIB"]
 n = int(os.environ.get("N", "1024"))
 reps = int(os.environ.get("REPS", "5"))
 x = torch.randn(n, 224, 224, 3, device="cuda").to(torch.bfloat16)
