@@ -53,6 +53,25 @@ if os.path.exists(p):
     for k, c in sorted(cls.items(), key=lambda kv: -kv[1][1])[:25]:
         out.append(f"| `{k[:70]}` | {c[0]} | {c[1] / 1e6:.3f} | {c[1] / tot * 100:.1f}% |")
     shutil.copy(p, f"profiles/{tag}_bench_launch_list.csv")
+p = f"{G}/{tag}_c3_launch_list.csv"
+if os.path.exists(p):
+    data = launches(p)
+    steps = max(1, sum(1 for d in data.values() if d["name"].startswith("void adainf::det_count_kernel")
+                       or d["name"].startswith("adainf::det_count_kernel")))
+    cls = {}
+    for d in data.values():
+        c = cls.setdefault(d["name"], [0, 0.0, 0.0])
+        c[0] += 1
+        c[1] += f(d.get("gpu__time_duration.sum"))
+        c[2] += f(d.get("dram__bytes_read.sum")) + f(d.get("dram__bytes_write.sum"))
+    tot = sum(c[1] for c in cls.values())
+    out += [f"\n## C3 (`bench.py --config c3 --steps 1 --warmup 3`): per-class time and DRAM traffic per DAG step "
+            f"(ncu, cold + serialised; {steps} detector passes in the run, totals divided by that)\n",
+            "| kernel | launches/step | ms/step | share | DRAM GB/step | GB/s |", "|---|---|---|---|---|---|"]
+    for k, c in sorted(cls.items(), key=lambda kv: -kv[1][1])[:24]:
+        out.append(f"| `{k[:70]}` | {c[0] / steps:.1f} | {c[1] / 1e6 / steps:.3f} | {c[1] / tot * 100:.1f}% | "
+                   f"{c[2] / 1e9 / steps:.3f} | {c[2] / max(c[1], 1):.0f} |")
+    shutil.copy(p, f"profiles/{tag}_c3_launch_list.csv")
 p = f"{G}/{tag}_step_traffic.csv"
 if os.path.exists(p):
     data = launches(p)
