@@ -68,6 +68,10 @@ adainf_status adainf_dbg_stem_wgrad(const void* x, const void* dz, int32_t n, in
  * is destroyed): [max_routed_per_dst][crop_h][crop_w][dst in_c] bf16, rows in route order, written by the last
  * adainf_infer_dag (rows past n_routed are stale).  For the stage-isolated crop parity test (reading Q20). */
 adainf_status adainf_dbg_app_crops(adainf_app_t app, int32_t edge, const void** crops);
+/* Layout of that batch: *s2d = 1 when the destination runs the space-to-depth ResNet stem and the crops were written
+ * straight into its packed input, [rows][crop_h/2][crop_w/2][16] with channel (bh*2 + bw)*4 + c (c >= in_c zero);
+ * 0 for the plain layout above. */
+adainf_status adainf_dbg_app_crop_layout(adainf_app_t app, int32_t edge, int32_t* s2d);
 
 /* Launch accounting and per-kernel-class timing (CUDA events on the launching stream).
  * adainf_launch_count: total kernels launched by the library since load (host-side counter).

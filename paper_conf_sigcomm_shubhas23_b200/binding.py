@@ -109,6 +109,7 @@ def lib():
             "adainf_model_update": [vp, C.c_float, vp, vp],
             "adainf_app_poll": [vp, vp],
             "adainf_dbg_app_crops": [vp, i32, C.POINTER(vp)],
+            "adainf_dbg_app_crop_layout": [vp, i32, C.POINTER(i32)],
             "adainf_dp_attach": [vp, vp, i32, i32],
             "adainf_select_merge": [vp, vp, vp, i32, i32, i64, i64, i64, i32, vp, vp, vp, vp],
             "adainf_nccl_unique_id": [vp],
@@ -371,8 +372,14 @@ class App:
         dst = self.models[e[1]].spec
         p = C.c_void_p()
         check(lib().adainf_dbg_app_crops(self.h, edge, C.byref(p)))
-        return _device_view(p.value, 0, torch.int16, self.models[e[1]].device,
-                            shape=(rows, dst["in_h"], dst["in_w"], dst["in_c"]))
+        s2d = C.c_int32()
+        check(lib().adainf_dbg_app_crop_layout(self.h, edge, C.byref(s2d)))
+        H, W, Cc = dst["in_h"], dst["in_w"], dst["in_c"]
+        if not s2d.value:
+            return _device_view(p.value, 0, torch.int16, self.models[e[1]].device, shape=(rows, H, W, Cc))
+        # space-to-depth packed [rows][H/2][W/2][16], channel (bh*2 + bw)*4 + c: unpacked to NHWC for inspection
+        s = _device_view(p.value, 0, torch.int16, self.models[e[1]].device, shape=(rows, H // 2, W // 2, 2, 2, 4))
+        return s.permute(0, 1, 3, 2, 4, 5).reshape(rows, H, W, 4)[..., :Cc].contiguous()
 
     def close(self):
         if getattr(self, "h", None):

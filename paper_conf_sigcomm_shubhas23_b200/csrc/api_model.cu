@@ -102,6 +102,7 @@ struct AppModelScratch {
 struct AppImpl {
   std::vector<AppModelScratch> ms;
   std::vector<DevBuf> routed_in;  // per edge (DET_CROP)
+  std::vector<char> crop_s2d;     // per edge: crops written straight into the destination's space-to-depth input
   DevBuf route_list, route_cnt;   // CLASS_WHOLE: [n_edges][cap], [n_edges]
   int32_t* cap_flag_host = nullptr;
   int32_t* cap_flag_dev = nullptr;
@@ -162,10 +163,16 @@ extern "C" adainf_status adainf_app_create(const adainf_app_spec* spec, adainf_a
       for (int i = 1; i < nm; ++i)
         if (I.in_edge[i] < 0) throw InvalidError("app: every non-root model needs an incoming edge");
       I.routed_in.resize(a.edges.size());
+      I.crop_s2d.assign(a.edges.size(), 0);
       for (size_t e = 0; e < a.edges.size(); ++e)
         if (a.edges[e].kind == ADAINF_ROUTE_DET_CROP) {
           Model* dst = a.models[a.edges[e].dst_model];
-          I.routed_in[e].alloc((size_t)a.max_routed * dst->in_h * dst->in_w * dst->in_c * 2);
+          const adainf_edge& ed = a.edges[e];
+          // a ResNet-stem destination takes its crops already space-to-depth packed (no packing pass)
+          const bool s2d = dst->stem_s2d && dst->in_c <= 4 && ed.crop_h == dst->in_h && ed.crop_w == dst->in_w &&
+                           getenv("ADAINF_CROP_S2D") == nullptr;
+          I.crop_s2d[e] = s2d;
+          I.routed_in[e].alloc((size_t)a.max_routed * dst->in_h * dst->in_w * (s2d ? 4 : dst->in_c) * 2);
         }
       I.route_list.alloc((size_t)std::max<size_t>(1, a.edges.size()) * std::max(1, a.max_routed) * 4);
       I.route_cnt.alloc((size_t)std::max<size_t>(1, a.edges.size()) * 4 + 16);
@@ -253,6 +260,7 @@ extern "C" adainf_status adainf_infer_dag(adainf_app_t app, const void* batch, i
         cnt = I.route_cnt.as<int>() + e;
         if (ed.kind == ADAINF_ROUTE_DET_CROP) {
           x = I.routed_in[e].as<bf16>();  // crops in the destination's own input layout (ingested like a batch)
+          padded = I.crop_s2d[e] != 0;     // ... or already in its packed space-to-depth layout
         } else {
           // whole-input routing: read the source model's own input rows through the route list
           if (ed.src_model != 0) throw UnsupportedError("CLASS_WHOLE routing from a routed model");
@@ -301,7 +309,7 @@ extern "C" adainf_status adainf_infer_dag(adainf_app_t app, const void* batch, i
           CK(cudaMemcpyAsync(I.route_cnt.as<int>() + e, S.cnt_clamped.as<int>() + q, 4, cudaMemcpyDeviceToDevice, st));
           launch_crops(x, m->in_h, m->in_w, m->in_c, S.det_table.as<float>(), S.route_idx.as<int32_t>(),
                        S.cnt_clamped.as<int32_t>(), q, d.cap, a.edges[e].crop_h, a.edges[e].crop_w, dst->in_c,
-                       I.routed_in[e].as<bf16>(), st);
+                       I.routed_in[e].as<bf16>(), st, I.crop_s2d[e] != 0);
         }
         if (o.route_idx && d.n_edges)
           CK(cudaMemcpyAsync(o.route_idx, S.route_idx.p, (size_t)d.n_edges * d.cap * 4, cudaMemcpyDeviceToDevice, st));
@@ -423,6 +431,16 @@ extern "C" adainf_status adainf_dbg_app_crops(adainf_app_t app, int32_t edge, co
     if (edge < 0 || edge >= (int)H->a.edges.size() || H->a.edges[edge].kind != ADAINF_ROUTE_DET_CROP)
       throw InvalidError("dbg_app_crops: not a DET_CROP edge");
     *crops = H->impl.routed_in[edge].p;
+  });
+}
+
+extern "C" adainf_status adainf_dbg_app_crop_layout(adainf_app_t app, int32_t edge, int32_t* s2d) {
+  return guard([&] {
+    if (!app || !s2d) throw InvalidError("dbg_app_crop_layout: null argument");
+    AppHolder* H = (AppHolder*)app;
+    if (edge < 0 || edge >= (int)H->a.edges.size() || H->a.edges[edge].kind != ADAINF_ROUTE_DET_CROP)
+      throw InvalidError("dbg_app_crop_layout: not a DET_CROP edge");
+    *s2d = H->impl.crop_s2d[edge];
   });
 }
 

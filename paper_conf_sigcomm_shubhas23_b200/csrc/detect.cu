@@ -453,10 +453,91 @@ __global__ void __launch_bounds__(256) crop_kernel(const bf16* __restrict__ fram
   }
 }
 
+// The same crops written straight into a space-to-depth destination's packed input (the ResNet stem's
+// [n][ch/2][cw/2][16], channel (bh*2 + bw)*4 + c, c >= C zero): one 2x2 output block per thread, two 16-byte
+// stores; the destination's own packing pass (a read and a write of every crop) disappears.
+__global__ void __launch_bounds__(256) crop_s2d_kernel(const bf16* __restrict__ frames, int H, int W, int C,
+                                                       const float* __restrict__ det,
+                                                       const int32_t* __restrict__ route_idx,
+                                                       const int32_t* __restrict__ cnt, int edge, int cap, int ch,
+                                                       int cw, bf16* __restrict__ dst) {
+  const int r = blockIdx.y;
+  if (r >= cnt[edge]) return;
+  __shared__ int s_xl[CROP_MAXW], s_xh[CROP_MAXW];
+  __shared__ float s_fx[CROP_MAXW];
+  const int di = route_idx[(long long)edge * cap + r];
+  const float* d = det + (long long)di * 9;
+  const int f = (int)d[0];
+  const float x0 = d[5], y0 = d[6], x1 = d[7], y1 = d[8];
+  const float sxs = __fdiv_rn(__fsub_rn(x1, x0), (float)cw);
+  const float sys = __fdiv_rn(__fsub_rn(y1, y0), (float)ch);
+  for (int u = threadIdx.x; u < cw; u += blockDim.x) {
+    float sx = __fsub_rn(__fadd_rn(x0, __fmul_rn(__fadd_rn((float)u, 0.5f), sxs)), 0.5f);
+    sx = fminf(fmaxf(sx, 0.f), (float)(W - 1));
+    const int xl = (int)floorf(sx);
+    s_xl[u] = xl;
+    s_xh[u] = min(xl + 1, W - 1);
+    s_fx[u] = __fsub_rn(sx, (float)xl);
+  }
+  __syncthreads();
+  const bf16* fr = frames + (long long)f * H * W * C;
+  const int hs = ch / 2, ws = cw / 2;
+  const int rows_per = (hs + CROP_BANDS - 1) / CROP_BANDS;
+  const int i0 = blockIdx.x * rows_per, i1 = min(hs, i0 + rows_per);
+  for (int idx = threadIdx.x; idx < (i1 - i0) * ws; idx += blockDim.x) {
+    const int i = i0 + idx / ws, j = idx % ws;
+    __align__(16) bf16 out[16];
+#pragma unroll
+    for (int bh = 0; bh < 2; ++bh) {
+      const int v = 2 * i + bh;
+      float sy = __fsub_rn(__fadd_rn(y0, __fmul_rn(__fadd_rn((float)v, 0.5f), sys)), 0.5f);
+      sy = fminf(fmaxf(sy, 0.f), (float)(H - 1));
+      const int yl = (int)floorf(sy);
+      const int yh = min(yl + 1, H - 1);
+      const float fy = __fsub_rn(sy, (float)yl);
+      const float wy0 = __fsub_rn(1.0f, fy);
+      const bf16* rl = fr + (long long)yl * W * C;
+      const bf16* rh = fr + (long long)yh * W * C;
+#pragma unroll
+      for (int bw = 0; bw < 2; ++bw) {
+        const int u = 2 * j + bw;
+        const int xl = s_xl[u], xh = s_xh[u];
+        const float fx = s_fx[u];
+        const float wx0 = __fsub_rn(1.0f, fx);
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          float val = 0.f;
+          if (c < C) {
+            const float p00 = __bfloat162float(rl[xl * C + c]);
+            const float p01 = __bfloat162float(rl[xh * C + c]);
+            const float p10 = __bfloat162float(rh[xl * C + c]);
+            const float p11 = __bfloat162float(rh[xh * C + c]);
+            const float top = __fadd_rn(__fmul_rn(wx0, p00), __fmul_rn(fx, p01));
+            const float bot = __fadd_rn(__fmul_rn(wx0, p10), __fmul_rn(fx, p11));
+            val = __fadd_rn(__fmul_rn(wy0, top), __fmul_rn(fy, bot));
+          }
+          out[(bh * 2 + bw) * 4 + c] = __float2bfloat16_rn(val);
+        }
+      }
+    }
+    uint4* o = (uint4*)(dst + (((long long)r * hs + i) * ws + j) * 16);
+    o[0] = ((const uint4*)out)[0];
+    o[1] = ((const uint4*)out)[1];
+  }
+}
+
 void launch_crops(const bf16* frames, int H, int W, int C, const float* det_table, const int32_t* route_idx,
                   const int32_t* count_clamped, int edge, int cap, int crop_h, int crop_w, int cout_pad, bf16* dst,
-                  cudaStream_t st) {
+                  cudaStream_t st, bool s2d) {
   if (crop_w > CROP_MAXW || cout_pad > 4) throw ShapeError("crop: width <= 512 and <= 4 channels");
+  if (s2d) {
+    if (crop_h % 2 || crop_w % 2 || C > 4) throw ShapeError("crop (s2d): even crop size, <= 4 channels");
+    ProfScope ps(PC_CROP, st);
+    crop_s2d_kernel<<<dim3(CROP_BANDS, cap), 256, 0, st>>>(frames, H, W, C, det_table, route_idx, count_clamped, edge,
+                                                           cap, crop_h, crop_w, dst);
+    CK(cudaGetLastError());
+    return;
+  }
   dim3 grid(CROP_BANDS, cap);
   ProfScope ps(PC_CROP, st);
   crop_kernel<<<grid, 256, 0, st>>>(frames, H, W, C, det_table, route_idx, count_clamped, edge, cap, crop_h, crop_w,

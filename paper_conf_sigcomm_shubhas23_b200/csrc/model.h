@@ -211,7 +211,7 @@ size_t det_route_ws_bytes(int n_static, int cells_per_frame, int A, bool nms);
 void launch_det_route(const DetRouteArgs& a, void* ws, cudaStream_t st);
 void launch_crops(const bf16* frames, int H, int W, int C, const float* det_table, const int32_t* route_idx,
                   const int32_t* count_clamped, int edge, int cap, int crop_h, int crop_w, int cout_pad, bf16* dst,
-                  cudaStream_t st);
+                  cudaStream_t st, bool s2d = false);
 // CLASS_WHOLE routing: stable compaction of rows with pred == cls
 void launch_route_class(const int32_t* pred, const int* count, int n_static, int cls, int32_t* list,
                         int32_t* count_out, int cap, int32_t* cap_flag, cudaStream_t st);
