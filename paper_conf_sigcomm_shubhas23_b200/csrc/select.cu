@@ -17,18 +17,22 @@
 
 namespace adainf {
 
-__global__ void transpose_w_kernel(const bf16* __restrict__ W, int D, int P, bf16* __restrict__ Wt) {
-  const int i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= D * P) return;
-  const int d = i / P, p = i - d * P;
-  Wt[(long long)p * D + d] = W[i];
-}
-
-// mu[r][p] = sum_d ref[r][d] * W[d][p]  (fp32): one warp per (r, p), lanes stride d (independent loads in flight),
-// fixed xor-tree combine
-__global__ void __launch_bounds__(256) project_ref_kernel(const float* __restrict__ ref, const bf16* __restrict__ W, int D,
-                                                          int P, int M, float* __restrict__ mu) {
-  const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+// Selection preparation in ONE launch (separate launches cost a few microseconds of latency each): blocks [0, nt)
+// transpose W -> Wt; the remaining blocks project the reference rows, mu[r][p] = sum_d ref[r][d] * W[d][p] in fp32,
+// one warp per (r, p), lanes stride d, fixed xor-tree combine.  The norms ||mu_r|| follow in ref_norm_kernel or,
+// on the fused path, at the start of every select_fused CTA (same arithmetic).
+__global__ void __launch_bounds__(256) select_prep_kernel(const float* __restrict__ ref, const bf16* __restrict__ W,
+                                                          int D, int P, int M, int nt, bf16* __restrict__ Wt,
+                                                          float* __restrict__ mu) {
+  if ((int)blockIdx.x < nt) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < D * P) {
+      const int d = i / P, p = i - d * P;
+      Wt[(long long)p * D + d] = W[i];
+    }
+    return;
+  }
+  const int gw = ((blockIdx.x - nt) * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (gw >= M * P) return;
   const int r = gw / P, p = gw - r * P;
   float a = 0.f;
@@ -42,15 +46,19 @@ __global__ void __launch_bounds__(256) project_ref_kernel(const float* __restric
   }
   if (lane == 0) mu[(long long)r * P + p] = a;
 }
-// mun[r] = ||mu_r||: one warp per reference row, lanes stride p, fixed xor-tree combine
+// ||mu_r|| of one reference row: lanes stride p, fixed xor-tree combine (one warp)
+__device__ __forceinline__ float ref_norm_warp(const float* mu_r, int P, int lane) {
+  float sq = 0.f;
+  for (int p = lane; p < P; p += 32) sq = fmaf(mu_r[p], mu_r[p], sq);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) sq += __shfl_xor_sync(0xffffffffu, sq, o);
+  return sqrtf(sq);
+}
 __global__ void ref_norm_kernel(const float* __restrict__ mu, int P, int M, float* __restrict__ mun) {
   const int r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (r >= M) return;
-  float s = 0.f;
-  for (int p = lane; p < P; p += 32) s = fmaf(mu[(long long)r * P + p], mu[(long long)r * P + p], s);
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-  if (lane == 0) mun[r] = sqrtf(s);
+  const float v = ref_norm_warp(mu + (long long)r * P, P, lane);
+  if (lane == 0) mun[r] = v;
 }
 
 // one warp per row: cosine distance to every reference row, min; key
@@ -191,7 +199,11 @@ __global__ void __launch_bounds__(SELF_THREADS, 1) select_fused_kernel(const __g
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const long long ntiles = (a.N + 127) / 128;
   for (int i = threadIdx.x; i < a.M * P; i += blockDim.x) mus[i] = a.mu[i];
-  if (threadIdx.x < a.M) mus[4 * P + threadIdx.x] = a.mun[threadIdx.x];
+  __syncthreads();
+  if ((threadIdx.x >> 5) < a.M) {  // ||mu_r||: warp r (M <= 4)
+    const float v = ref_norm_warp(mus + (threadIdx.x >> 5) * P, P, threadIdx.x & 31);
+    if ((threadIdx.x & 31) == 0) mus[4 * P + (threadIdx.x >> 5)] = v;
+  }
   if (threadIdx.x == 0) {
     for (int s = 0; s < SELF_STAGES; ++s) {
       mbar_init(&full[s], 1);
@@ -669,16 +681,17 @@ void select_retrain(const adainf_select_in& in, int k, int32_t* out_idx, float* 
   const long long nb = (N + EMIT_THREADS - 1) / EMIT_THREADS;
   int* blk = (int*)take((size_t)nb * 8);
   int* offs = (int*)take((size_t)nb * 8);
-  { ProfScope ps(PC_SELECT_PROJ, st);
-  project_ref_kernel<<<(M * P * 32 + 255) / 256, 256, 0, st>>>(in.ref, (const bf16*)in.W_bf16, D, P, M, mu);
-  ref_norm_kernel<<<(M * 32 + 255) / 256, 256, 0, st>>>(mu, P, M, mun); }
+  {
+    ProfScope ps(PC_SELECT_PROJ, st);
+    const int nt = in.W_bf16 ? (D * P + 255) / 256 : 0;
+    select_prep_kernel<<<nt + (M * P * 32 + 255) / 256, 256, 0, st>>>(in.ref, (const bf16*)in.W_bf16, D, P, M, nt, Wt,
+                                                                       mu);
+    if (!fused) ref_norm_kernel<<<(M * 32 + 255) / 256, 256, 0, st>>>(mu, P, M, mun);
+    CK(cudaGetLastError());
+  }
   if (fused) {
-    { ProfScope ps(PC_SELECT_PROJ, st);
-    transpose_w_kernel<<<(D * P + 255) / 256, 256, 0, st>>>((const bf16*)in.W_bf16, D, P, Wt); }
     launch_select_fused((const bf16*)in.X_bf16, Wt, N, D, P, M, mu, mun, in.exclude, keys, dist_all, st);
   } else if (in.W_bf16) {
-    { ProfScope ps(PC_SELECT_PROJ, st);
-    transpose_w_kernel<<<(D * P + 255) / 256, 256, 0, st>>>((const bf16*)in.W_bf16, D, P, Wt); }
     CK(cudaMemsetAsync(zb, 0, (size_t)P * 4, st));
     ConvGeom g{};
     g.Cin = D;
