@@ -145,7 +145,8 @@ adainf_status adainf_model_get_grads(adainf_model_t m, float* host_dst, int64_t 
 
 /* ---- Application DAG (Fig. 1): root model first, routing edges between models ---------- */
 typedef enum {
-  ADAINF_ROUTE_DET_CROP = 0,    /* detector detections of class src_class -> crops for dst (Q19) */
+  ADAINF_ROUTE_DET_CROP = 0,    /* detector detections of class src_class -> crops for dst (Q19); at most one
+                                   DET_CROP edge per (source, class): ADAINF_ERR_INVALID otherwise */
   ADAINF_ROUTE_CLASS_WHOLE = 1  /* whole input of samples predicted src_class -> dst (audio, Q24) */
 } adainf_route_kind;
 

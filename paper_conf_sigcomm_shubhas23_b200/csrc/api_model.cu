@@ -151,6 +151,8 @@ extern "C" adainf_status adainf_app_create(const adainf_app_spec* spec, adainf_a
           if (ed.crop_h != dst->in_h || ed.crop_w != dst->in_w || dst->in_c != src->in_c)
             throw ShapeError("app: crop size must equal the destination input");
           if (ed.src_class < 0 || ed.src_class >= src->det.classes) throw InvalidError("app: bad src_class");
+          for (int q : I.ms[ed.src_model].det_edges)  // a detection goes to its class's one destination
+            if (a.edges[q].src_class == ed.src_class) throw InvalidError("app: two DET_CROP edges for one class");
           I.ms[ed.src_model].det_edges.push_back((int)e);
         } else if (ed.kind == ADAINF_ROUTE_CLASS_WHOLE) {
           if (src->exits.empty()) throw InvalidError("app: CLASS_WHOLE edge from a model without exits");
