@@ -78,15 +78,19 @@ if os.path.exists(p):
     tot = sum(f(d.get("gpu__time_duration.sum")) for d in data.values())
     cls = {}
     for d in data.values():
-        c = cls.setdefault(d["name"], [0, 0.0, 0.0])
+        c = cls.setdefault(d["name"], [0, 0.0, 0.0, 0.0])
         c[0] += 1
-        c[1] += f(d.get("gpu__time_duration.sum"))
+        t = f(d.get("gpu__time_duration.sum"))
+        c[1] += t
         c[2] += f(d.get("dram__bytes_read.sum")) + f(d.get("dram__bytes_write.sum"))
-    out += ["\n## One C5-shaped step (infer 256 + retrain 8,192), per-class DRAM traffic (ncu, cold + serialised)\n",
-            "| kernel | launches | ms | share | DRAM GB | GB/s |", "|---|---|---|---|---|---|"]
+        c[3] += f(d.get("sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed")) * t
+    out += ["\n## One C5-shaped step (infer 256 + retrain 8,192), per-class DRAM traffic and tensor-pipe activity "
+            "(ncu, cold + serialised)\n",
+            "| kernel | launches | ms | share | DRAM GB | GB/s | tensor pipe % (time-weighted) |",
+            "|---|---|---|---|---|---|---|"]
     for k, c in sorted(cls.items(), key=lambda kv: -kv[1][1])[:25]:
         out.append(f"| `{k[:70]}` | {c[0]} | {c[1] / 1e6:.3f} | {c[1] / tot * 100:.1f}% | {c[2] / 1e9:.3f} | "
-                   f"{c[2] / max(c[1], 1):.0f} |")
+                   f"{c[2] / max(c[1], 1):.0f} | {c[3] / max(c[1], 1):.1f} |")
     shutil.copy(p, f"profiles/{tag}_step_traffic.csv")
 keys = ["gpu__time_duration.sum", "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed",
         "sm__ops_path_tensor_src_bf16_dst_fp32.avg.pct_of_peak_sustained_elapsed", "dram__bytes_read.sum",
