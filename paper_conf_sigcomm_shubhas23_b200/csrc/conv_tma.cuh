@@ -253,8 +253,9 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
 #pragma unroll
         for (int i = 0; i < 64; i += 8) st_bf16x8(o + i, v + i);
       }
-      // all threads of the group are done with the staging buffer before the next TMA overwrites it
-      asm volatile("bar.sync %0, 128;" ::"r"(1 + grp) : "memory");
+      // all threads of the group are done with the staging buffer before the next TMA overwrites it (no staged
+      // operands -> nothing to protect: the group's warps run ahead independently)
+      if (ntens) asm volatile("bar.sync %0, 128;" ::"r"(1 + grp) : "memory");
     }
   }
 

@@ -6,6 +6,8 @@ import sys
 sys.path.insert(0, os.path.join(os.path.dirname(os.path.abspath(__file__)), ".."))
 import torch
 from paper_conf_sigcomm_shubhas23_b200 import binding as B
+if os.environ.get("ADAINF_LIB"):  # A/B against another build
+    B.LIB_PATH = os.environ["ADAINF_LIB"]
 
 n = int(os.environ.get("N", "1024"))
 modes = [int(m) for m in os.environ.get("MODES", "0,1").split(",")]
