@@ -44,6 +44,7 @@ sys.path.insert(0, ROOT)
 
 from paper_conf_sigcomm_shubhas23_b200 import specs as S  # noqa: E402
 from paper_conf_sigcomm_shubhas23_b200 import synth  # noqa: E402
+from paper_conf_sigcomm_shubhas23_b200.driver import dp_rows, place_apps  # noqa: E402
 
 METRIC = "DAG inference samples/s + retrain samples/s per B200 (1/2/4/8), % of bf16 peak"
 UNIT = "samples/s"
@@ -65,6 +66,15 @@ CONFIGS = {
                     "routing (224x224) "
                     "-> vehicle-type (10 cls) + person-activity (8 cls) ResNet-18-EE (exits 25/25/25/25)",
                frames=512, hw=416, det_per_frame=4.0, cap=2048, fractions=[0.25, 0.25, 0.25], seed=3),
+    "c4": dict(name="BASELINE config 4: 8 applications placed app i -> GPU i mod G (a DAG is never split): 6 video DAGs "
+                    "(128 frames 416x416 -> detector + NMS -> on-device crops -> vehicle-type (6..11 cls) + "
+                    "person-activity (8 cls) ResNet-18-EE) + 2 audio DAGs (512 log-mel 128x128 spectrograms -> event "
+                    "ResNet-18-EE -> whole-input routing by class -> keyword (8 cls) + siren (4 cls) ResNet-18-EE); "
+                    "every classifier retrained each step on its share of k = 1,024 samples per app (vehicle : person "
+                    "= 640 : 384 by impact degree 0.15 : 0.09, P:86-90 / P:237; audio 342 : 341 : 341), data-parallel "
+                    "over all G GPUs (rows by index mod G, P:243)",
+               apps=8, video=6, frames=128, hw=416, det_per_frame=4.0, cap=512, audio_b=512,
+               fractions=[0.25, 0.25, 0.25], k=1024, seed=4),
 }
 
 
@@ -240,7 +250,7 @@ def run_reference(args, world, rank):
         return 0
     import oracle as O
     cfg = CONFIGS[args.config]
-    if args.config == "c3":
+    if args.config in ("c3", "c4"):
         step, units, desc = _oracle_dag_sample(O, cfg, 1, 2)
     else:
         step, units, desc = _oracle_job_sample(O, cfg, 1, 1, 4096, 256)
@@ -272,7 +282,7 @@ def cpu_baseline_leg(config):
     per core, run concurrently -> the all-cores rate, and each job's own time -> the one-thread rate."""
     import oracle as O
     cfg = CONFIGS[config]
-    if config == "c3":
+    if config in ("c3", "c4"):
         step, units, desc = _oracle_dag_sample(O, cfg, 1, 2)
     else:
         step, units, desc = _oracle_job_sample(O, cfg, 1, 1, 4096, 256)
@@ -432,15 +442,16 @@ class DagWorkload:
         F, hw, cap = cfg["frames"], cfg["hw"], cfg["cap"]
         self.F, self.hw, self.cap = F, hw, cap
         self.det_spec = S.tiny_yolo_det(in_hw=hw, nms_iou=0.45)  # TinyYOLOv3's NMS threshold (NEXT-3, Q18b)
-        self.veh, self.per = S.resnet18_ee(10), S.resnet18_ee(8)
+        self.veh, self.per = S.resnet18_ee(cfg.get("veh_classes", 10)), S.resnet18_ee(8)
         seed = 100 * cfg["seed"] + rank
         pd = synth.det_head_params(self.det_spec, synth.init_params(self.det_spec, seed=31), obj_bias=-2.0,
                                    cls_bias=(0.55, -0.55))
         self.frames_host, _ = synth.drifted_images(F, hw, hw, 3, seed=seed, period=1)
         self.x = torch.from_numpy(self.frames_host.view(np.int16)).to(dev).view(torch.bfloat16)
         self.md = B.Model(self.det_spec, F, params=pd)
-        self.mv = B.Model(self.veh, cap, params=synth.init_params(self.veh, seed=32))
-        self.mp = B.Model(self.per, cap, params=synth.init_params(self.per, seed=33))
+        cls_b = max(cap, cfg.get("cls_max_batch", 0))  # c4: the same models also run their retraining shard
+        self.mv = B.Model(self.veh, cls_b, params=synth.init_params(self.veh, seed=32), momentum=MU)
+        self.mp = B.Model(self.per, cls_b, params=synth.init_params(self.per, seed=33), momentum=MU)
         self.app = B.App([self.md, self.mv, self.mp], edges=[(0, 1, B.ROUTE_DET_CROP, 0, 224, 224),
                                                              (0, 2, B.ROUTE_DET_CROP, 1, 224, 224)],
                          max_routed_per_dst=cap)
@@ -521,6 +532,188 @@ class DagWorkload:
         return [self.outs[0]["n_det"], self.outs[1]["pred"], self.outs[2]["pred"]]
 
 
+class AudioApp:
+    """c4 audio DAG (reading Q24): event classifier -> whole-input routing by predicted class -> keyword / siren."""
+
+    def __init__(self, cfg, B, torch, dev, seed, cls_max_batch):
+        self.B, self.torch = B, torch
+        b = cfg["audio_b"]
+        self.b = b
+        self.specs = [S.resnet18_ee(2, in_hw=128, in_c=1), S.resnet18_ee(8, in_hw=128, in_c=1),
+                      S.resnet18_ee(4, in_hw=128, in_c=1)]
+        self.host, _ = synth.spectrograms(b, num_classes=8, F=128, T=128, period=1, seed=seed)
+        self.x = torch.from_numpy(self.host.view(np.int16)).to(dev).view(torch.bfloat16)
+        mb = max(b, cls_max_batch)
+        self.models = [B.Model(sp, mb, params=synth.init_params(sp, seed=41 + j), momentum=MU)
+                       for j, sp in enumerate(self.specs)]
+        self.app = B.App(self.models, edges=[(0, 1, B.ROUTE_CLASS_WHOLE, 0, 0, 0), (0, 2, B.ROUTE_CLASS_WHOLE, 1, 0, 0)],
+                         max_routed_per_dst=b)
+        self.outs = [B.alloc_outs(self.models[0], b, n_out_edges=2, max_routed=b), B.alloc_outs(self.models[1], b),
+                     B.alloc_outs(self.models[2], b)]
+        self.taus = [2.0] * 9
+        self.stage_macs, self.stem_macs = stage_macs_of(self.specs[0])
+
+    def calibrate(self, fractions):
+        """each classifier's taus from its own full-depth confidences on the batch (one-model apps)"""
+        taus = []
+        for m in self.models:
+            app = self.B.App([m])
+            cal = self.B.alloc_outs(m, self.b)
+            conf = np.zeros((self.b, 4), np.float32)
+            for k in range(4):
+                tk = [2.0] * 3
+                if k < 3:
+                    tk[k] = 0.0
+                app.infer(self.x, tk, [cal])
+                self.torch.cuda.synchronize()
+                conf[:, k] = cal["conf"].cpu().numpy()
+            app.close()
+            taus += [float(t) for t in synth.calibrate_thresholds(conf, fractions)]
+        self.taus = taus
+
+    def step(self, counts_out, xi=None):
+        for j in range(3):
+            self.outs[j]["exit_counts"] = counts_out[4 * j:4 * j + 4]
+        self.app.infer(self.x if xi is None else xi, self.taus, self.outs)
+
+    def flops(self, counts):
+        fl, stem_rows = 0.0, 0.0
+        for off in (0, 4, 8):
+            c = counts[:, off:off + 4]
+            n = c.sum(1)
+            reach = np.array([n - c[:, :k].sum(1) for k in range(4)]).T.mean(0)
+            fl += 2.0 * float(np.dot(reach, self.stage_macs))
+            stem_rows += reach[0]
+        return fl, stem_rows
+
+
+class MultiAppWorkload:
+    """c4: 8 applications placed app i -> rank i mod G (inference shards by placement, a DAG's models
+    stay on one GPU); every classifier of every application retrains each step on its rows index mod G of the app's
+    k selected samples, its gradient all-reduced over all ranks (one NCCL communicator per classifier)."""
+
+    def __init__(self, cfg, B, torch, dev, rank, world):
+        self.cfg, self.B, self.torch, self.dev = cfg, B, torch, dev
+        self.rank, self.world = rank, world
+        napps, nvid, k = cfg["apps"], cfg["video"], cfg["k"]
+        self.hosted = place_apps(napps, world)[rank]
+        shares = {"video": [640, 384], "audio": [342, 341, 341]}
+        local = lambda n: len(dp_rows(n, rank, world))
+        self.apps = {}
+        for i in self.hosted:
+            if i < nvid:
+                vcfg = dict(frames=cfg["frames"], hw=cfg["hw"], cap=cfg["cap"], det_per_frame=cfg["det_per_frame"],
+                            fractions=cfg["fractions"], seed=10 * cfg["seed"] + i, veh_classes=6 + i,
+                            cls_max_batch=local(640))
+                self.apps[i] = DagWorkload(vcfg, B, torch, dev, 0, 1)
+            else:
+                self.apps[i] = AudioApp(cfg, B, torch, dev, seed=10 * cfg["seed"] + i, cls_max_batch=local(342))
+        # retraining pools (distinct synthetic inputs; labels per classifier = class mod its class count)
+        def bf(a):
+            return torch.from_numpy(a.view(np.int16)).to(dev).view(torch.bfloat16)
+        vb, vy = synth.drifted_images(1024, 224, 224, 3, seed=7 * cfg["seed"], period=1)
+        ab, ay = synth.spectrograms(1024, num_classes=8, F=128, T=128, period=1, seed=7 * cfg["seed"] + 1)
+        self.vpool, self.apool = bf(vb), bf(ab)
+        rng = np.random.default_rng(cfg["seed"])
+        self.rt = []  # (model, pool, labels, local row indices, n_global)
+        for i in range(napps):
+            if i < nvid:
+                specs = [S.resnet18_ee(6 + i), S.resnet18_ee(8)]
+                mods = [self.apps[i].mv, self.apps[i].mp] if i in self.apps else [None, None]
+                seeds, pool, y, share = (32, 33), self.vpool, vy, shares["video"]
+            else:
+                specs = [S.resnet18_ee(c, in_hw=128, in_c=1) for c in (2, 8, 4)]
+                mods = self.apps[i].models if i in self.apps else [None] * 3
+                seeds, pool, y, share = (41, 42, 43), self.apool, ay, shares["audio"]
+            for sp, m, sd, n in zip(specs, mods, seeds, share):
+                if m is None:  # replica of a classifier hosted elsewhere (identical initial parameters)
+                    m = B.Model(sp, max(1, local(n)), params=synth.init_params(sp, seed=sd), momentum=MU)
+                ncls = next(o["num_classes"] for o in sp["ops"] if o["kind"] == "exit")
+                rows = np.sort(rng.choice(pool.shape[0], n, replace=False))[dp_rows(n, rank, world)].astype(np.int32)
+                lab = torch.from_numpy((y % ncls).astype(np.int32)).to(dev)
+                self.rt.append((m, pool, lab, torch.from_numpy(rows).to(dev), n, sp))
+        self.slots = {i: (8 * i if i < nvid else 8 * nvid + 12 * (i - nvid)) for i in range(napps)}
+        self.ncnt = 8 * nvid + 12 * (napps - nvid)
+        self.units = (nvid * cfg["frames"] + (napps - nvid) * cfg["audio_b"] + napps * k) / world
+        self.k = napps * k
+        self.video_stage = stage_macs_of(S.resnet18_ee(10))
+        self.audio_stage = stage_macs_of(S.resnet18_ee(2, in_hw=128, in_c=1))
+
+    def attach_dp(self, rank, world):
+        import torch.distributed as dist
+        for m, *_ in self.rt:
+            uid = self.B.nccl_unique_id() if rank == 0 else b"\0" * 128
+            obj = [uid]
+            dist.broadcast_object_list(obj, src=0)
+            m.dp_attach(obj[0], rank, world)
+
+    def calibrate(self):
+        for i, a in self.apps.items():
+            if isinstance(a, DagWorkload):
+                a.calibrate()
+            else:
+                a.calibrate(self.cfg["fractions"])
+
+    def step(self, counts_out, xi=None, Xe=None, py=None):
+        # xi: per hosted application, its input batch (the e2e path's double-buffered copies), else the resident one
+        for j, (i, a) in enumerate(self.apps.items()):
+            o = self.slots[i]
+            a.step(counts_out[o:o + (8 if isinstance(a, DagWorkload) else 12)], xi=None if xi is None else xi[j])
+        for m, pool, lab, rows, n, _sp in self.rt:
+            m.retrain_step_rows(pool, lab, rows, n_global=n, lr=LR)
+
+    phase_infer = None
+
+    @property
+    def taus(self):
+        return {f"app{i}": a.taus for i, a in self.apps.items()}
+
+    def flops(self, counts):
+        f = {"conv_fwd": 0.0, "conv_dgrad": 0.0, "conv_wgrad": 0.0, "stem_fwd": 0.0, "stem_wgrad": 0.0}
+        inf = 0.0
+        for i, a in self.apps.items():
+            o = self.slots[i]
+            if isinstance(a, DagWorkload):
+                fa, ia, _, _ = a.flops(counts[:, o:o + 8])
+                f["conv_fwd"] += fa["conv_fwd"]
+                f["stem_fwd"] += fa["stem_fwd"]
+                inf += ia
+            else:
+                fl, stem_rows = a.flops(counts[:, o:o + 12])
+                f["conv_fwd"] += fl - 2.0 * a.stem_macs * stem_rows
+                f["stem_fwd"] += 2.0 * a.stem_macs * stem_rows
+                inf += fl
+        rt = 0.0
+        for m, pool, lab, rows, n, sp in self.rt:
+            stage, stem = self.audio_stage if sp["in_c"] == 1 else self.video_stage
+            nl = int(rows.shape[0])
+            conv = sum(stage) - stem
+            f["conv_fwd"] += 2.0 * nl * conv
+            f["conv_dgrad"] += 2.0 * nl * conv
+            f["conv_wgrad"] += 2.0 * nl * conv
+            f["stem_fwd"] += 2.0 * nl * stem
+            f["stem_wgrad"] += 2.0 * nl * stem
+            rt += 2.0 * nl * (3 * sum(stage) - stem)
+        return f, inf, rt, None
+
+    def hbm_bytes(self, reach):
+        return {}
+
+    def e2e_inputs(self):
+        torch = self.torch
+        out = []
+        for a in self.apps.values():
+            host = a.frames_host if isinstance(a, DagWorkload) else a.host
+            out.append((torch.from_numpy(host.view(np.int16)).view(torch.bfloat16).pin_memory(), a.x))
+        return out
+
+    def e2e_results(self):
+        res = []
+        for a in self.apps.values():
+            res += [a.outs[1]["pred"], a.outs[2]["pred"]]
+        return res
+
+
 # ------------------------------------------------------------------------------------------------
 def main():
     ap = argparse.ArgumentParser()
@@ -572,11 +765,11 @@ def main():
         return float(t.item())
 
     bf16_burst, bf16_sust, hbm_gbs, peak_src, sm_max_spec = peaks()
-    wl = (DagWorkload if args.config == "c3" else JobWorkload)(cfg, B, torch, dev, rank, world)
-    if world > 1 and isinstance(wl, JobWorkload):
+    wl = {"c3": DagWorkload, "c4": MultiAppWorkload}.get(args.config, JobWorkload)(cfg, B, torch, dev, rank, world)
+    if world > 1 and isinstance(wl, (JobWorkload, MultiAppWorkload)):
         wl.attach_dp(rank, world)
     stream = torch.cuda.current_stream()
-    ncnt = 8 if args.config == "c3" else 4
+    ncnt = {"c3": 8, "c4": getattr(wl, "ncnt", 4)}.get(args.config, 4)
 
     wl.calibrate()
     cnt_buf = torch.zeros((max(args.steps, 1) + args.warmup + 64, ncnt), dtype=torch.int32, device=dev)
@@ -801,6 +994,8 @@ def main():
             ins = bufs[b]
             if isinstance(wl, JobWorkload):
                 wl.step(counts_row, xi=ins[0], Xe=ins[1], py=ins[2])
+            elif isinstance(wl, MultiAppWorkload):
+                wl.step(counts_row, xi=ins)
             else:
                 wl.step(counts_row, xi=ins[0])
 
@@ -877,7 +1072,9 @@ def main():
 
     if rank == 0:
         cfg_line = {"workload": cfg["name"], "config": args.config,
-                    "model": "resnet18_ee" if args.config != "c3" else "tiny_yolo_det -> 2x resnet18_ee",
+                    "model": {"c3": "tiny_yolo_det -> 2x resnet18_ee",
+                              "c4": "6x (tiny_yolo_det -> 2x resnet18_ee) + 2x (resnet18_ee 128x128x1 -> 2x resnet18_ee "
+                                    "128x128x1)"}.get(args.config, "resnet18_ee"),
                     "global_batch": samples_per_step, "seq_len": None,
                     "parallelism": f"dp{world}" if world > 1 else "single",
                     "l2": "inputs + activations larger than L2 (no flush)",
@@ -886,6 +1083,10 @@ def main():
         if isinstance(wl, JobWorkload):
             cfg_line.update(inference_batch=wl.inf_b, retrain_batch=wl.k, pool=wl.pool_n,
                             embed=f"D={cfg['d']} -> P={cfg['p']}", exit_fractions=cfg["fractions"])
+        if isinstance(wl, MultiAppWorkload):
+            cfg_line.update(placement={f"gpu{r}": apps for r, apps in enumerate(place_apps(cfg["apps"], world))},
+                            inference_samples=cfg["video"] * cfg["frames"] + (cfg["apps"] - cfg["video"]) * cfg["audio_b"],
+                            retrain_samples=cfg["apps"] * cfg["k"], exit_fractions=cfg["fractions"])
         line = {
             "metric": METRIC, "value": value, "unit": UNIT if args.config != "c3" else "frames/s",
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
@@ -909,7 +1110,8 @@ def main():
             "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)
-    wl.app.close()
+    for a in ([wl] if not isinstance(wl, MultiAppWorkload) else list(wl.apps.values())):
+        a.app.close()
     if world > 1:
         torch.distributed.destroy_process_group()
     return 0

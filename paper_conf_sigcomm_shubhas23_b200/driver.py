@@ -21,6 +21,21 @@ from dataclasses import dataclass, field
 from . import binding as B
 
 
+def place_apps(n_apps: int, world: int):
+    """Application placement (BASELINE config 4): app i -> GPU i mod G.  A DAG's models stay on one GPU,
+    so routing never crosses devices (the B200 analogue of the paper's GPU-space division, done by placement
+    instead of MPS percentages).  Returns, per rank, the list of its applications."""
+    if n_apps < 0 or world < 1:
+        raise ValueError("place_apps: n_apps >= 0, world >= 1")
+    return [[i for i in range(n_apps) if i % world == r] for r in range(world)]
+
+
+def dp_rows(n: int, rank: int, world: int):
+    """Rows of a retraining task's n selected samples that rank `rank` trains on: index mod G (no sample is
+    used by two replicas), gradients scaled by 1/n and all-reduced."""
+    return list(range(rank, n, world))
+
+
 @dataclass
 class RetrainTask:
     model: "B.Model"

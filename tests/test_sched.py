@@ -140,3 +140,18 @@ def test_pick_structure_rules():
         B.pick_structure(tables, acc, 0.5, 1, 2, 12, 100)  # batch0 not profiled
     with pytest.raises(B.AdaInfError):
         B.pick_batch([4, 8], [1.0, -1.0], 10)
+
+
+def test_app_placement_and_dp_rows():
+    """BASELINE config 4: app i -> GPU i mod G, every application on exactly one GPU, loads within one
+    application of each other; each retraining task's rows split index mod G, disjoint and covering."""
+    from paper_conf_sigcomm_shubhas23_b200.driver import dp_rows, place_apps
+    for world in (1, 2, 3, 4, 8):
+        pl = place_apps(8, world)
+        flat = sorted(a for r in pl for a in r)
+        assert flat == list(range(8))
+        assert max(map(len, pl)) - min(map(len, pl)) <= 1
+        assert all(a % world == r for r, apps in enumerate(pl) for a in apps)
+        for n in (1, 341, 640, 1024):
+            rows = [dp_rows(n, r, world) for r in range(world)]
+            assert sorted(x for rr in rows for x in rr) == list(range(n))
