@@ -363,6 +363,7 @@ struct RadixState {
   uint32_t T;
   uint32_t need_eq;
   uint32_t n_eligible;
+  uint32_t ticket;  // blocks of the current pass done (the last one runs the digit pick)
 };
 
 __global__ void radix_init_kernel(RadixState* s, int k) {
@@ -370,12 +371,16 @@ __global__ void radix_init_kernel(RadixState* s, int k) {
     s->prefix = 0;
     s->krem = (uint32_t)k;
     s->n_eligible = 0;
+    s->ticket = 0;
   }
   s->hist[threadIdx.x] = 0;
 }
 
-__global__ void radix_hist_kernel(const uint32_t* __restrict__ keys, long long N, RadixState* s, int shift,
-                                  uint32_t mask_hi, int count_eligible) {
+__device__ void radix_pick_block(RadixState* s, int shift, int last);
+
+__global__ void __launch_bounds__(256) radix_hist_kernel(const uint32_t* __restrict__ keys, long long N,
+                                                         RadixState* s, int shift, uint32_t mask_hi,
+                                                         int count_eligible, int last_pass) {
   __shared__ uint32_t h[256];
   __shared__ uint32_t elig;
   h[threadIdx.x] = 0;
@@ -392,22 +397,33 @@ __global__ void radix_hist_kernel(const uint32_t* __restrict__ keys, long long N
   __syncthreads();
   if (h[threadIdx.x]) atomicAdd(&s->hist[threadIdx.x], h[threadIdx.x]);
   if (count_eligible && threadIdx.x == 0) atomicAdd(&s->n_eligible, elig);
+  // the last block to finish this pass picks the digit (threadfence-reduction pattern)
+  __shared__ bool is_last;
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) is_last = atomicAdd(&s->ticket, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (is_last) {
+    __threadfence();
+    radix_pick_block(s, shift, last_pass);
+  }
 }
 
-// 256 threads: suffix counts of the histogram (digit 255 down), the digit d where the running count reaches krem
-__global__ void __launch_bounds__(256) radix_pick_kernel(RadixState* s, int shift, int last) {
+// 256 threads: suffix counts of the histogram (digit 255 down), the digit d where the running count reaches krem;
+// run by the last block of each histogram pass (no separate launch)
+__device__ void radix_pick_block(RadixState* s, int shift, int last) {
   __shared__ uint32_t suf[256];  // suf[d] = count of digits > d
   __shared__ int s_d;
+  __shared__ uint32_t wsum[8];
   const int t = threadIdx.x, lane = t & 31, w = t >> 5;
   const int d = 255 - t;  // thread t handles digit 255 - t (descending)
-  const uint32_t c = s->hist[d];
+  const uint32_t c = __ldcg(&s->hist[d]);
   uint32_t x = c;  // inclusive scan over t (i.e. over descending digits)
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
     const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
     if (lane >= o) x += y;
   }
-  __shared__ uint32_t wsum[8];
   if (lane == 31) wsum[w] = x;
   __syncthreads();
   uint32_t off = 0;
@@ -427,15 +443,19 @@ __global__ void __launch_bounds__(256) radix_pick_kernel(RadixState* s, int shif
       s->T = s->prefix;
       s->need_eq = s->krem;
     }
+    s->ticket = 0;
   }
   s->hist[t] = 0;
 }
 
 constexpr int EMIT_THREADS = 1024;
 
-// per-block counts of (key > T) and (key == T)
-__global__ void emit_count_kernel(const uint32_t* __restrict__ keys, long long N, const RadixState* s,
-                                  int* __restrict__ blk) {
+__device__ void emit_scan_warp(int nb, const RadixState* s, const int* blk, int* __restrict__ offs,
+                               int32_t* out_count, int k);
+
+// per-block counts of (key > T) and (key == T); the last block to finish runs the scan
+__global__ void emit_count_kernel(const uint32_t* __restrict__ keys, long long N, RadixState* s,
+                                  int* __restrict__ blk, int* __restrict__ offs, int32_t* out_count, int k) {
   __shared__ int sg, se;
   if (threadIdx.x == 0) sg = se = 0;
   __syncthreads();
@@ -460,16 +480,27 @@ __global__ void emit_count_kernel(const uint32_t* __restrict__ keys, long long N
     blk[2 * blockIdx.x] = sg;
     blk[2 * blockIdx.x + 1] = se;
   }
+  __shared__ bool is_last;
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) is_last = atomicAdd(&s->ticket, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (is_last && threadIdx.x < 32) {
+    __threadfence();
+    emit_scan_warp((int)gridDim.x, s, blk, offs, out_count, k);
+    if (threadIdx.x == 0) s->ticket = 0;
+  }
 }
-// exclusive scans: eq prefix per block, then take_b = g_b + clamp(need - eqpre_b, 0, e_b) and its prefix
-__global__ void emit_scan_kernel(int nb, const RadixState* s, int* __restrict__ blk, int* __restrict__ offs,
-                                 int32_t* out_count, int k) {
-  const int lane = threadIdx.x;
+// exclusive scans: eq prefix per block, then take_b = g_b + clamp(need - eqpre_b, 0, e_b) and its prefix; one warp,
+// run by the last block of emit_count_kernel (no separate launch)
+__device__ void emit_scan_warp(int nb, const RadixState* s, const int* blk, int* __restrict__ offs,
+                               int32_t* out_count, int k) {
+  const int lane = threadIdx.x & 31;
   const int need = (int)s->need_eq;
   int run_eq = 0, run_take = 0;
   for (int b0 = 0; b0 < nb; b0 += 32) {
     const int b = b0 + lane;
-    const int g = b < nb ? blk[2 * b] : 0, e = b < nb ? blk[2 * b + 1] : 0;
+    const int g = b < nb ? __ldcg(blk + 2 * b) : 0, e = b < nb ? __ldcg(blk + 2 * b + 1) : 0;
     int xe = e;
     for (int o = 1; o < 32; o <<= 1) {
       const int u = __shfl_up_sync(0xffffffffu, xe, o);
@@ -624,17 +655,15 @@ static void topk_emit(const uint32_t* keys, long long N, int k, RadixState* rs, 
     CK(cudaGetLastError());
     return;
   }
-  ProfScope ps_topk(PC_SELECT_TOPK, st, 12);
+  ProfScope ps_topk(PC_SELECT_TOPK, st, 7);
   radix_init_kernel<<<1, 256, 0, st>>>(rs, k_eff);
   const int hb = (int)std::min<long long>((N + 1023) / 1024, 4LL * num_sms());
   for (int pass = 0; pass < 4; ++pass) {
     const int shift = 24 - 8 * pass;
     const uint32_t mask_hi = pass == 0 ? 0u : (0xFFFFFFFFu << (32 - 8 * pass));
-    radix_hist_kernel<<<hb, 256, 0, st>>>(keys, N, rs, shift, mask_hi, pass == 0);
-    radix_pick_kernel<<<1, 256, 0, st>>>(rs, shift, pass == 3);
+    radix_hist_kernel<<<hb, 256, 0, st>>>(keys, N, rs, shift, mask_hi, pass == 0, pass == 3);
   }
-  emit_count_kernel<<<(unsigned)nb, EMIT_THREADS, 0, st>>>(keys, N, rs, blk);
-  emit_scan_kernel<<<1, 32, 0, st>>>((int)nb, rs, blk, offs, out_count, k);
+  emit_count_kernel<<<(unsigned)nb, EMIT_THREADS, 0, st>>>(keys, N, rs, blk, offs, out_count, k);
   emit_write_kernel<<<(unsigned)nb, EMIT_THREADS, 0, st>>>(keys, N, rs, offs, out_idx, out_dist, k);
   CK(cudaGetLastError());
 }
