@@ -552,96 +552,137 @@ __global__ void emit_write_kernel(const uint32_t* __restrict__ keys, long long N
   }
 }
 
-// Single-CTA exact top-k for pools up to ~1M keys: the four 8-bit MSB radix passes (warp-aggregated shared-memory
-// histograms: the distance keys share few top bytes) and the ascending stable emit (block ballot scan per 1,024-key
-// chunk, ties -> lower position) in one launch, instead of 12 launches of the multi-CTA path.
-constexpr int TOPK1_THREADS = 1024;
-__global__ void __launch_bounds__(TOPK1_THREADS) topk_single_kernel(const uint32_t* __restrict__ keys, int N, int k,
-                                                                    int32_t* __restrict__ out_idx,
-                                                                    float* __restrict__ out_dist,
-                                                                    int32_t* __restrict__ out_count) {
-  __shared__ uint32_t hist[256];
-  __shared__ uint32_t s_prefix, s_krem;
-  __shared__ int warp_g[32], warp_e[32];
-  __shared__ int s_run_take, s_run_eq;
-  const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-  const int k_eff = min(k, N);
-  if (t == 0) {
-    s_prefix = 0;
-    s_krem = (uint32_t)k_eff;
+// Single-CTA exact top-k for small pools (N <= 1,024 x 32): every thread holds 32 consecutive keys in registers (one
+// read of the keys), the four 8-bit MSB radix passes run on the registers (warp-aggregated shared histograms, the digit
+// picked by a 256-thread suffix scan), and the ascending stable emit (ties -> lower position) needs two block-wide
+// exclusive scans: ties before each thread, then outputs before each thread. One launch.
+constexpr int TOPK1_THREADS = 1024, TOPK1_KPT = 32;
+constexpr long long TOPK1_MAX_N = (long long)TOPK1_THREADS * TOPK1_KPT;
+
+// exclusive scan of one value per thread over a 1,024-thread block; ws: 33 words of shared memory
+__device__ __forceinline__ uint32_t scan1024(uint32_t v, uint32_t* ws, uint32_t& total) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
   }
+  if (lane == 31) ws[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    const uint32_t y = ws[lane];
+    uint32_t z = y;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t u = __shfl_up_sync(0xffffffffu, z, o);
+      if (lane >= o) z += u;
+    }
+    ws[lane] = z - y;
+    if (lane == 31) ws[32] = z;
+  }
+  __syncthreads();
+  const uint32_t r = ws[w] + x - v;
+  total = ws[32];
+  __syncthreads();
+  return r;
+}
+
+__global__ void __launch_bounds__(TOPK1_THREADS, 1) topk_single_kernel(const uint32_t* __restrict__ keys, int N,
+                                                                       int k, int32_t* __restrict__ out_idx,
+                                                                       float* __restrict__ out_dist,
+                                                                       int32_t* __restrict__ out_count) {
+  __shared__ uint32_t hist[256];
+  __shared__ uint32_t ws[33];
+  __shared__ int s_d;
+  __shared__ uint32_t s_cum, s_tot;
+  const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+  const int kpt = (N + TOPK1_THREADS - 1) / TOPK1_THREADS;  // keys per thread (<= 32): every thread busy
+  const int base = t * kpt;
+  const int nv = max(0, min(kpt, N - base));  // this thread's valid keys
+  uint32_t kv[TOPK1_KPT];
+#pragma unroll
+  for (int j = 0; j < TOPK1_KPT; ++j) kv[j] = j < nv ? __ldg(keys + base + j) : 0u;
+  uint32_t prefix = 0, krem = (uint32_t)min(k, N);
+#pragma unroll 1
   for (int pass = 0; pass < 4; ++pass) {
     const int shift = 24 - 8 * pass;
     const uint32_t mask_hi = pass == 0 ? 0u : (0xFFFFFFFFu << (32 - 8 * pass));
     if (t < 256) hist[t] = 0;
+    if (t == 0) s_d = -1;
     __syncthreads();
-    const uint32_t prefix = s_prefix;
-    for (int i0 = 0; i0 < N; i0 += TOPK1_THREADS) {
-      const int i = i0 + t;
-      const uint32_t key = i < N ? keys[i] : 0u;
-      const bool in = i < N && (key & mask_hi) == prefix;
-      const uint32_t dig = (key >> shift) & 255u;
-      const unsigned act = __ballot_sync(0xffffffffu, in);
-      if (in) {
-        const unsigned peers = __match_any_sync(act, dig);
-        if ((int)(__ffs(peers) - 1) == lane) atomicAdd(&hist[dig], (uint32_t)__popc(peers));
+    // run-length aggregation over the thread's consecutive keys (the distance keys share their top bytes, so a
+    // pass-0 thread issues one atomic), then shared-memory atomics
+    uint32_t run_d = 0, run_c = 0;
+#pragma unroll
+    for (int j = 0; j < TOPK1_KPT; ++j) {
+      if (j < nv && (kv[j] & mask_hi) == prefix) {
+        const uint32_t dig = (kv[j] >> shift) & 255u;
+        if (run_c && dig != run_d) {
+          atomicAdd(&hist[run_d], run_c);
+          run_c = 0;
+        }
+        run_d = dig;
+        ++run_c;
       }
     }
+    if (run_c) atomicAdd(&hist[run_d], run_c);
     __syncthreads();
-    if (t == 0) {
-      uint32_t krem = s_krem, cum = 0;
-      int d = 255;
-      for (; d >= 0; --d) {
-        const uint32_t c = hist[d];
-        if (cum + c >= krem) break;
-        cum += c;
+    uint32_t c = 0, x = 0;
+    if (t < 256) {  // thread t: digit 255 - t (descending), inclusive scan = keys with digit >= 255 - t
+      c = x = hist[255 - t];
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
       }
-      if (d < 0) d = 0;
-      s_prefix = prefix | ((uint32_t)d << shift);
-      s_krem = krem - cum;
+      if (lane == 31) ws[w] = x;
     }
     __syncthreads();
-  }
-  const uint32_t T = s_prefix;
-  const int need = (int)s_krem;
-  if (t == 0) {
-    s_run_take = 0;
-    s_run_eq = 0;
-  }
-  __syncthreads();
-  for (int i0 = 0; i0 < N; i0 += TOPK1_THREADS) {
-    const int i = i0 + t;
-    const uint32_t key = i < N ? keys[i] : 0u;
-    const bool g = (T == 0) ? key > 0 : key > T;
-    const bool e = (T != 0) && key == T;
-    const unsigned be = __ballot_sync(0xffffffffu, e);
-    if (lane == 0) warp_e[w] = __popc(be);
-    __syncthreads();
-    int eqrank = s_run_eq + __popc(be & ((1u << lane) - 1u));
-    for (int q = 0; q < w; ++q) eqrank += warp_e[q];
-    const bool take = g || (e && eqrank < need);
-    const unsigned bt = __ballot_sync(0xffffffffu, take);
-    if (lane == 0) warp_g[w] = __popc(bt);
-    __syncthreads();
-    int o = s_run_take + __popc(bt & ((1u << lane) - 1u));
-    for (int q = 0; q < w; ++q) o += warp_g[q];
-    if (take && o < k) {
-      out_idx[o] = i;
-      if (out_dist) out_dist[o] = __uint_as_float(key - 1u);
-    }
-    __syncthreads();
-    if (t == 0) {
-      int tt = 0, te = 0;
-      for (int q = 0; q < 32; ++q) {
-        tt += warp_g[q];
-        te += warp_e[q];
+    if (t < 256) {
+      uint32_t off = 0;
+      for (int q = 0; q < w; ++q) off += ws[q];
+      const uint32_t incl = off + x, excl = incl - c;
+      if (excl < krem && incl >= krem) {  // exactly one digit
+        s_d = 255 - t;
+        s_cum = excl;
       }
-      s_run_take += tt;
-      s_run_eq += te;
+      if (t == 255) s_tot = incl;
     }
     __syncthreads();
+    const int d = s_d;
+    prefix |= (uint32_t)(d >= 0 ? d : 0) << shift;
+    krem -= d >= 0 ? s_cum : s_tot;
+    __syncthreads();
   }
-  if (t == 0) *out_count = min(s_run_take, k);
+  const uint32_t T = prefix, need = krem;
+  uint32_t e_cnt = 0;
+#pragma unroll
+  for (int j = 0; j < TOPK1_KPT; ++j) e_cnt += (T != 0 && kv[j] == T) ? 1u : 0u;  // padding keys are 0
+  uint32_t tot;
+  uint32_t er = scan1024(e_cnt, ws, tot);  // ties before this thread's keys
+  uint32_t take_mask = 0, take_cnt = 0;
+#pragma unroll
+  for (int j = 0; j < TOPK1_KPT; ++j) {
+    const bool g = T == 0 ? kv[j] > 0u : kv[j] > T;
+    const bool e = T != 0 && kv[j] == T;
+    const bool tk = g || (e && er < need);
+    er += e ? 1u : 0u;
+    take_mask |= (tk ? 1u : 0u) << j;
+    take_cnt += tk ? 1u : 0u;
+  }
+  uint32_t o = scan1024(take_cnt, ws, tot);  // outputs before this thread's keys
+#pragma unroll
+  for (int j = 0; j < TOPK1_KPT; ++j) {
+    if ((take_mask >> j) & 1u) {
+      if (o < (uint32_t)k) {
+        out_idx[o] = base + j;
+        if (out_dist) out_dist[o] = __uint_as_float(kv[j] - 1u);
+      }
+      ++o;
+    }
+  }
+  if (t == 0) *out_count = (int32_t)min(tot, (uint32_t)k);
 }
 
 // exact top-k of 32-bit keys (0 = not eligible), ties -> lower position, emitted in ascending position order
@@ -649,7 +690,8 @@ static void topk_emit(const uint32_t* keys, long long N, int k, RadixState* rs, 
                       float* out_dist, int32_t* out_count, cudaStream_t st) {
   const long long nb = (N + EMIT_THREADS - 1) / EMIT_THREADS;
   const int k_eff = (int)std::min<long long>(k, N);  // the k-th largest must exist
-  if (N <= 24576 && !getenv("ADAINF_TOPK_MULTI")) {  // single CTA wins below ~24k keys (measured)
+  // single CTA wins below ~24k keys (measured: 27 vs 37 us at 16,384; 45 vs 39 us at 32,768)
+  if (N <= std::min<long long>(24576, TOPK1_MAX_N) && !getenv("ADAINF_TOPK_MULTI")) {
     ProfScope ps_topk(PC_SELECT_TOPK, st, 1);
     topk_single_kernel<<<1, TOPK1_THREADS, 0, st>>>(keys, (int)N, k, out_idx, out_dist, out_count);
     CK(cudaGetLastError());

@@ -13,7 +13,7 @@ from paper_conf_sigcomm_shubhas23_b200 import synth
 if os.environ.get("ADAINF_LIB"):
     B.LIB_PATH = os.environ["ADAINF_LIB"]
 rows = []
-for N, D, P, k in [(131072, 512, 64, 8192), (16384, 64, 16, 1024)]:
+for N, D, P, k in [(131072, 512, 64, 8192), (16384, 64, 16, 1024), (32768, 64, 16, 2048)]:
     Xb, Wb, ref = synth.embeddings(N, D, P, seed=5)
     X = torch.from_numpy(Xb.view(np.int16)).cuda().view(torch.bfloat16)
     W = torch.from_numpy(Wb.view(np.int16)).cuda().view(torch.bfloat16)
