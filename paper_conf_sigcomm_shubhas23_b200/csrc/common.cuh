@@ -87,6 +87,12 @@ __device__ unsigned long long g_wait_cycles[4096][8];
 #define TIMED_WAIT(slot, expr) expr
 #endif
 
+// 1024-byte aligned start of the dynamic shared memory, kept as a pointer into the shared window (the usual
+// round trip through uintptr_t makes every later access through it a generic LD / ST)
+__device__ __forceinline__ uint8_t* smem_align1024(uint8_t* raw) {
+  return raw + ((1024u - (smem_u32(raw) & 1023u)) & 1023u);
+}
+
 // ---- cp.async (LDGSTS) -------------------------------------------------------------------------
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, bool valid) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(valid ? 16 : 0)
@@ -200,6 +206,19 @@ __device__ __forceinline__ float act_apply(int act, float v) {
   const float neg = act == 2 ? __fmul_rn(0.1f, v) : 0.f;
   const float pos = act == 3 ? fminf(v, 6.f) : v;
   return (act == 0 || v > 0.f) ? pos : neg;
+}
+// the activation of N values with the kind tested once (ReLU as one compare + select per value; the per-value
+// form above re-tests the uniform kind for every element, which dominated the instruction count of the
+// 64-channel epilogues)
+template <int N>
+__device__ __forceinline__ void act_vec(int act, float* v) {
+  if (act == 1) {
+#pragma unroll
+    for (int i = 0; i < N; ++i) v[i] = v[i] > 0.f ? v[i] : 0.f;
+  } else if (act != 0) {
+#pragma unroll
+    for (int i = 0; i < N; ++i) v[i] = act_apply(act, v[i]);
+  }
 }
 // derivative from the stored output y (ReLU'(0) = 0; ReLU6' = 0 at both clamps)
 __device__ __forceinline__ float act_grad(int act, float y) {

@@ -161,6 +161,11 @@ __device__ __forceinline__ void st_bf16x8(bf16* p, const float* v) {
   for (int q = 0; q < 8; ++q) h[q] = __float2bfloat16_rn(v[q]);
   *(uint4*)p = *(uint4*)h;
 }
+// two floats -> bf16x2 (RNE; lower address = a)
+__device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
+  const __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+  return *(const uint32_t*)&h;
+}
 __device__ __forceinline__ void ld_bf16x8(const bf16* p, float* v) {
   const uint4 raw = __ldg((const uint4*)p);
   const bf16* h = (const bf16*)&raw;

@@ -20,7 +20,7 @@ if sel:
     shapes = [shapes[int(i)] for i in sel.split(",")]
 
 
-def t(fn, reps=5):
+def t(fn, reps=int(os.environ.get("REPS", "5"))):
     fn()
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
