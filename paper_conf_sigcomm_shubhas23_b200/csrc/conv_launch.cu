@@ -205,17 +205,10 @@ static void launch_ws_tma(const ConvArgs& c, bool dgrad, int nstatic, cudaStream
   a.bias = c.bias;
   a.bcast = c.bcast;
   a.out = (bf16*)c.out;
-  // ADAINF_WSKX=1: kx-split kernel (see conv_tma.cuh; measured slower: its epilogue is the limiter): B block i*3+j = row tap i, column tap j,
-  // i.e. weight tap i*3+j (FWD) or the flipped 8-(i*3+j) (DGRAD)
-  static int wskx = -1;
-  if (wskx < 0) {
-    const char* e = getenv("ADAINF_WSKX");
-    wskx = e ? atoi(e) : 0;
-  }
   for (int kh = 0; kh < 3; ++kh)
     for (int kw = 0; kw < 3; ++kw) {
       a.tap_off[kh * 3 + kw] = dgrad ? 8 + (2 - kh) * Wp + (1 - kw) : 8 + kh * Wp + kw - 1;
-      a.btap[kh * 3 + kw] = (wskx && dgrad) ? 8 - (kh * 3 + kw) : kh * 3 + kw;
+      a.btap[kh * 3 + kw] = kh * 3 + kw;
     }
   // one box per image row when the padded pitch exceeds W (ADAINF_ROWBOX=0: one {64, Wp, R+2} box with
   // out-of-bounds columns)
@@ -237,7 +230,7 @@ static void launch_ws_tma(const ConvArgs& c, bool dgrad, int nstatic, cudaStream
   if (!dgrad && c.res_map && c.res_map != c.src_map) throw std::runtime_error("ws_tma: residual map differs");
   a.win_bytes = ((16 + (R + 2) * Wp) * 128 + 1023) / 1024 * 1024;
   const int fixed = 9 * 8192 + 2 * std::max(1, a.has_e0 + a.has_e1) * 16384 + 1024 /*align*/ +
-                    (wskx ? 512 + 4096 /*barriers, bias, quadrant exchange*/ : 512 /*barriers*/);
+                    512 /*barriers*/;
   a.wstages = std::min(8, (227 * 1024 - fixed) / a.win_bytes);
   if (const char* e = getenv("ADAINF_WS_STAGES")) a.wstages = std::min(a.wstages, std::max(1, atoi(e)));
   if (a.wstages < 2) throw std::runtime_error("ws_tma: shared memory");
@@ -245,14 +238,12 @@ static void launch_ws_tma(const ConvArgs& c, bool dgrad, int nstatic, cudaStream
   static bool attr = false;
   if (!attr) {
     CK(cudaFuncSetAttribute(conv_ws_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
-    CK(cudaFuncSetAttribute(conv_wskx_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
     attr = true;
   }
   const long long tiles = (long long)nstatic * a.tpi;
   dim3 grid((unsigned)std::max(1LL, std::min<long long>(tiles, num_sms())));
   ProfScope ps(dgrad ? PC_CONV_DGRAD : PC_CONV_FWD, st);
-  if (wskx) conv_wskx_tma_kernel<<<grid, TMA_WS_THREADS, smem, st>>>(a);
-  else conv_ws_tma_kernel<<<grid, TMA_WS_THREADS, smem, st>>>(a);
+  conv_ws_tma_kernel<<<grid, TMA_WS_THREADS, smem, st>>>(a);
   CK(cudaGetLastError());
 }
 

@@ -299,325 +299,6 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
   }
 }
 
-// ------------------------------------------------------------------------------------------------
-// kx-split variant of the 64x64 window conv (same window / staging / tiles as conv_ws_tma_kernel).
-//
-// Why: with N = 64 every K = 16 MMA reads a 4 KB A tile and a 2 KB B tile from shared memory for 32 cycles of
-// math, so the 36 MMAs of a tile (9 taps x 4 K-steps) were bound by the tensor core's shared-memory operand reads
-// (ncu: 2,900 cycles per tile against the 1,152-cycle MMA floor, the MMA warp waiting for its operands).  Here the
-// three column taps share one A operand and become the MMA's N dimension:
-//   Z_j[q] = sum_i A_i[q] . W[i][j]      (A_i = the window viewed at row offset i, N = 3 x 64 = 192, K = 3 x 64)
-//   out[p] = Z_0[p-1] + Z_1[p] + Z_2[p+1]
-// 12 MMAs of 128 x 192 x 16 per tile move 120 KB of operands instead of 216 KB for the same FLOPs.  The column
-// shift is applied in the epilogue: warp shuffles inside a 32-lane quadrant, shared memory across quadrants.  The
-// neighbours of a tile's first / last position are pad columns (x = -1 wraps to the previous row's pad column
-// x >= W, whose window rows are zero), so tiles stay independent.  DGRAD: the same with the taps flipped
-// (block (i, j) holds W[2-i][2-j], MN-major) - dX(x) = sum_j Z_j[x + j - 1] with Z_j over the dZ window.
-__device__ __forceinline__ void tmem_ld16_nw(uint32_t taddr, uint32_t* r) {
-  asm volatile(
-      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
-      : "r"(taddr));
-}
-__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
-
-__global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_wskx_tma_kernel(const __grid_constant__ WsTmaArgs a) {
-  constexpr int NACC = 2, ACC_STRIDE = 256;  // two 192-column accumulators
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = smem_align1024(smem_raw);
-  const int WS = a.wstages;
-  uint8_t* win = smem;
-  uint8_t* bres = win + WS * a.win_bytes;  // 9 x 8 KB, block i*3+j = row tap i, column tap j (contiguous per i)
-  const int ntens = a.has_e0 + a.has_e1;
-  const int nstg = ntens > 0 ? ntens : 1;  // the output is staged in the first buffer
-  uint8_t* stg = bres + 9 * 8192;          // [2 groups][nstg tensors][16 KB]
-  uint64_t* bars = (uint64_t*)(stg + 2 * nstg * 16384);
-  uint64_t* wfull = bars;        // [WS]
-  uint64_t* wempty = wfull + 8;  // [WS]
-  uint64_t* tfull = wempty + 8;  // [NACC]
-  uint64_t* tempty = tfull + 2;  // [NACC]
-  uint64_t* efull = tempty + 2;  // [2]
-  uint64_t* bready = efull + 2;
-  uint32_t* tmem_slot = (uint32_t*)(bready + 1);
-  float* s_bias = (float*)(tmem_slot + 4);
-  float* xch = (float*)(bars + 64);  // 16-byte aligned: [2 groups][4 quadrants][2: Z_0 of lane 31, Z_2 of lane 0][64]
-
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int nsamp = a.count ? *a.count : a.n_static;
-  const int ntile = nsamp * a.tpi;
-  if ((int)blockIdx.x >= ntile) return;
-  const int Wp = a.Wp, R = a.R, H = a.H, W = a.W;
-
-  for (int i = threadIdx.x; i < WS * 2 * 64; i += blockDim.x) {
-    const int s = i / 128, k = i % 128;
-    const int rows = 8 + (R + 2) * Wp;
-    uint4* p = (uint4*)(win + s * a.win_bytes + (k < 64 ? k * 16 : rows * 128 + (k - 64) * 16));
-    *p = make_uint4(0, 0, 0, 0);
-  }
-  if (a.rowbox) {
-    const int padc = Wp - W, per_stage = (R + 2) * padc * 8;
-    for (int i = threadIdx.x; i < WS * per_stage; i += blockDim.x) {
-      const int s = i / per_stage, k = i - s * per_stage;
-      const int j = k / (padc * 8), rem = k - j * (padc * 8);
-      const int x = W + rem / 8, c = rem % 8;
-      *(uint4*)(win + s * a.win_bytes + 1024 + (j * Wp + x) * 128 + c * 16) = make_uint4(0, 0, 0, 0);
-    }
-  }
-  if (threadIdx.x < 64) s_bias[threadIdx.x] = (!a.dgrad && a.bias) ? a.bias[threadIdx.x] : 0.f;
-  if (threadIdx.x == 0) {
-    for (int s = 0; s < WS; ++s) {
-      mbar_init(&wfull[s], 1);
-      mbar_init(&wempty[s], 1);
-    }
-    for (int b = 0; b < 2; ++b) {
-      mbar_init(&tfull[b], 1);
-      mbar_init(&tempty[b], 128);
-      mbar_init(&efull[b], 1);
-    }
-    mbar_init(bready, 128);
-    fence_mbar_init();
-    tma_prefetch_desc(&a.win_map);
-  }
-  if (warp == 4) tmem_alloc<512>(tmem_slot);
-  fence_proxy_async_smem();
-  tc_fence_before();
-  __syncthreads();
-  tc_fence_after();
-  const uint32_t tmem = *tmem_slot;
-  const uint32_t wsm = smem_u32(win), bsm = smem_u32(bres), ssm = smem_u32(stg);
-  const uint32_t box_bytes = 64u * 2u * Wp * (R + 2);
-  const uint32_t ebox_bytes = 64u * 2u * Wp * R;
-
-  if (warp < 4) {
-    // ---- resident B: block tp <- weight tap a.btap[tp] (the host passes the flipped order for DGRAD) ----
-    const int t = threadIdx.x;
-    for (int tp = 0; tp < 9; ++tp) {
-      const uint32_t sb = bsm + tp * 8192;
-      const bf16* wb = a.B + (long long)a.btap[tp] * 64;
-#pragma unroll
-      for (int idx = t; idx < 64 * 8; idx += 128) {
-        const int r = idx >> 3, jj = idx & 7;
-        const uint32_t off = a.dgrad ? mnmaj_off(r, jj) : kmaj_off(r, jj);
-        cp_async16(sb + off, wb + (long long)r * a.ldb + jj * 8, true);
-      }
-    }
-    cp_async_arrive_noinc(bready);
-    if (warp == 0 && lane == 0) {
-      int it = 0;
-      for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++it) {
-        const int n = tile / a.tpi, h0 = (tile - n * a.tpi) * R;
-        const int sn = a.smap ? __ldg(a.smap + n) : n;
-        const int s = it % WS, u = it / WS;
-        if (u > 0) mbar_wait(&wempty[s], (u - 1) & 1);
-        if (a.rowbox) {
-          mbar_expect_tx(&wfull[s], 64u * 2u * W * (R + 2));
-          for (int j = 0; j < R + 2; ++j)
-            tma_load_4d(wsm + s * a.win_bytes + 1024 + j * Wp * 128, &a.win_map, &wfull[s], 0, 0, h0 - 1 + j, sn);
-        } else {
-          mbar_expect_tx(&wfull[s], box_bytes);
-          tma_load_4d(wsm + s * a.win_bytes + 1024, &a.win_map, &wfull[s], 0, 0, h0 - 1, sn);
-        }
-      }
-    }
-  } else if (warp == 4) {
-    // ---- MMA issuer: 3 row taps x 4 K-steps of 128 x 192 x 16 ----
-    const uint32_t IDESC = make_idesc(BM, 192, 0, a.dgrad ? 1 : 0);
-    const uint64_t b_base = a.dgrad ? make_sdesc(bsm, 8192, 1024) : make_sdesc(bsm, 16, 1024);
-    const uint32_t b_kk = a.dgrad ? 128u : 2u;
-    mbar_wait(bready, 0);
-    fence_proxy_async_smem();
-    int it = 0;
-    for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++it) {
-      const int b = it % NACC, ub = it / NACC;
-      if (ub > 0) mbar_wait(&tempty[b], (ub - 1) & 1);
-      const int s = it % WS, u = it / WS;
-      mbar_wait(&wfull[s], u & 1);
-      tc_fence_after();
-      if (elect_one()) {
-        const uint32_t dacc = tmem + (uint32_t)(b * ACC_STRIDE);
-        const uint64_t a_base = make_sdesc(wsm + s * a.win_bytes, 16, 1024);
-#pragma unroll
-        for (int i = 0; i < 3; ++i) {
-          const uint32_t aoff = (uint32_t)(8 + i * Wp) * 8u;  // window row offset i (16-byte units)
-#pragma unroll
-          for (int kk = 0; kk < 4; ++kk)
-            umma_bf16(dacc, a_base + (aoff + 2u * kk), b_base + (uint32_t)(i * 3 * 512 + kk * b_kk), IDESC,
-                      (i | kk) != 0);
-        }
-        umma_commit(&wempty[s]);
-        umma_commit(&tfull[b]);
-      }
-      __syncwarp();
-    }
-  } else {
-    // ---- epilogue: 2 groups of 4 warps (one per TMEM lane quadrant), group g handles local tiles g, g+2, ... ----
-    const int grp = (warp - 5) >> 2;
-    const int qd = warp & 3;
-    const int row = qd * 32 + lane;  // output position p within the tile
-    const bool leader = (warp == 5 + 4 * grp) && lane == 0;
-    const uint32_t sg = ssm + grp * nstg * 16384;
-    float* xg = xch + grp * 4 * 2 * 64;
-    int lt = grp, use = 0;
-    for (int tile = blockIdx.x + grp * gridDim.x; tile < ntile; tile += 2 * gridDim.x, lt += 2, ++use) {
-      const int n = tile / a.tpi, h0 = (tile - n * a.tpi) * R;
-      const int h = h0 + row / Wp, x = row % Wp;
-      const bool rv = h < H && x < W;
-      const long long orow = ((long long)n * H + h) * W + x;
-      if (ntens && leader) {
-        tma_store_wait_read();  // the previous output store has read the buffer
-        mbar_expect_tx(&efull[grp], ntens * ebox_bytes);
-        const int sn = (!a.dgrad && a.smap) ? __ldg(a.smap + n) : n;
-        if (a.has_e0) tma_load_4d(sg, &a.e0_map, &efull[grp], 0, 0, h0, sn);
-        if (a.has_e1) tma_load_4d(sg + a.has_e0 * 16384, &a.e1_map, &efull[grp], 0, 0, h0, n);
-      }
-      const int b = lt % NACC, ub = lt / NACC;
-      mbar_wait(&tfull[b], ub & 1);
-      tc_fence_after();
-      const uint32_t trow = tmem + (uint32_t)(b * ACC_STRIDE) + ((uint32_t)(qd * 32) << 16);
-      float v[64];
-#pragma unroll
-      for (int c = 0; c < 64; c += 16) {
-        uint32_t z0[16], z1[16], z2[16];
-        tmem_ld16_nw(trow + c, z0);
-        tmem_ld16_nw(trow + 64 + c, z1);
-        tmem_ld16_nw(trow + 128 + c, z2);
-        tmem_wait_ld();
-        if (lane == 31)
-#pragma unroll
-          for (int k = 0; k < 16; k += 4)
-            *(uint4*)(xg + (qd * 2 + 0) * 64 + c + k) = make_uint4(z0[k], z0[k + 1], z0[k + 2], z0[k + 3]);
-        if (lane == 0)
-#pragma unroll
-          for (int k = 0; k < 16; k += 4)
-            *(uint4*)(xg + (qd * 2 + 1) * 64 + c + k) = make_uint4(z2[k], z2[k + 1], z2[k + 2], z2[k + 3]);
-#pragma unroll
-        for (int k = 0; k < 16; ++k) {
-          // Z_0[p-1] + Z_1[p] (the cross-quadrant Z_0 of lane 0 is added after the exchange)
-          const float zl = __uint_as_float(__shfl_up_sync(0xffffffffu, z0[k], 1));
-          const float zr = __uint_as_float(__shfl_down_sync(0xffffffffu, z2[k], 1));
-          const float m = __uint_as_float(z1[k]);
-          v[c + k] = lane == 0 ? m : __fadd_rn(zl, m);
-          z2[k] = __float_as_uint(zr);  // Z_2[p+1] for lanes < 31
-        }
-        if (lane < 31) {
-#pragma unroll
-          for (int k = 0; k < 16; ++k) v[c + k] = __fadd_rn(v[c + k], __uint_as_float(z2[k]));
-        }
-      }
-      tc_fence_before();
-      mbar_arrive(&tempty[b]);
-      if (!ntens && leader) tma_store_wait_read();  // dedicated output buffer: the previous store has read it
-      asm volatile("bar.sync %0, 128;" ::"r"(1 + grp) : "memory");  // quadrant boundary values written
-      if (lane == 0 && qd > 0) {  // Z_0 of position p-1 (lane 31 of the quadrant above); p = 0 reads a pad column
-#pragma unroll
-        for (int k = 0; k < 64; k += 4) {
-          const float4 q = *(const float4*)(xg + ((qd - 1) * 2 + 0) * 64 + k);
-          v[k] = __fadd_rn(q.x, v[k]);
-          v[k + 1] = __fadd_rn(q.y, v[k + 1]);
-          v[k + 2] = __fadd_rn(q.z, v[k + 2]);
-          v[k + 3] = __fadd_rn(q.w, v[k + 3]);
-        }
-      }
-      if (lane == 31 && qd < 3) {  // Z_2 of position p+1 (lane 0 of the quadrant below); p = 127 is a pad column
-#pragma unroll
-        for (int k = 0; k < 64; k += 4) {
-          const float4 q = *(const float4*)(xg + ((qd + 1) * 2 + 1) * 64 + k);
-          v[k] = __fadd_rn(v[k], q.x);
-          v[k + 1] = __fadd_rn(v[k + 1], q.y);
-          v[k + 2] = __fadd_rn(v[k + 2], q.z);
-          v[k + 3] = __fadd_rn(v[k + 3], q.w);
-        }
-      }
-      if (ntens) mbar_wait(&efull[grp], use & 1);
-      uint8_t* e0 = stg + (grp * nstg) * 16384 + row * 128;
-      const uint8_t* e1 = e0 + a.has_e0 * 16384;
-      if (rv) {
-        if (!a.dgrad) {
-#pragma unroll
-          for (int i = 0; i < 64; ++i) v[i] = __fadd_rn(v[i], s_bias[i]);
-          if (a.has_e0) {
-#pragma unroll
-            for (int i = 0; i < 8; ++i) {
-              const uint4 e = *(const uint4*)(e0 + ((i ^ (row & 7)) << 4));
-              const bf16* hh = (const bf16*)&e;
-#pragma unroll
-              for (int qq = 0; qq < 8; ++qq) v[i * 8 + qq] = __fadd_rn(v[i * 8 + qq], __bfloat162float(hh[qq]));
-            }
-          }
-          act_vec<64>(a.act, v);
-        } else {
-          if (a.bcast) {
-#pragma unroll
-            for (int i = 0; i < 64; i += 4) {
-              const float4 bb = __ldg((const float4*)(a.bcast + (long long)n * 64 + i));
-              v[i] = __fadd_rn(v[i], bb.x);
-              v[i + 1] = __fadd_rn(v[i + 1], bb.y);
-              v[i + 2] = __fadd_rn(v[i + 2], bb.z);
-              v[i + 3] = __fadd_rn(v[i + 3], bb.w);
-            }
-          }
-          if (a.has_e0) {
-#pragma unroll
-            for (int i = 0; i < 8; ++i) {
-              const uint4 e = *(const uint4*)(e0 + ((i ^ (row & 7)) << 4));
-              const bf16* hh = (const bf16*)&e;
-#pragma unroll
-              for (int qq = 0; qq < 8; ++qq) v[i * 8 + qq] = __fadd_rn(v[i * 8 + qq], __bfloat162float(hh[qq]));
-            }
-          }
-          if (a.has_e1) {
-            if (a.mask_act == 1) {  // ReLU' as a select (the kind tested once per row)
-#pragma unroll
-              for (int i = 0; i < 8; ++i) {
-                const uint4 e = *(const uint4*)(e1 + ((i ^ (row & 7)) << 4));
-                const bf16* hh = (const bf16*)&e;
-#pragma unroll
-                for (int qq = 0; qq < 8; ++qq)
-                  v[i * 8 + qq] = __fmul_rn(v[i * 8 + qq], __bfloat162float(hh[qq]) > 0.f ? 1.f : 0.f);
-              }
-            } else {
-#pragma unroll
-              for (int i = 0; i < 8; ++i) {
-                const uint4 e = *(const uint4*)(e1 + ((i ^ (row & 7)) << 4));
-                const bf16* hh = (const bf16*)&e;
-#pragma unroll
-                for (int qq = 0; qq < 8; ++qq)
-                  v[i * 8 + qq] = __fmul_rn(v[i * 8 + qq], act_grad(a.mask_act, __bfloat162float(hh[qq])));
-              }
-            }
-          }
-        }
-      }
-#pragma unroll
-      for (int i = 0; i < 8; ++i) {
-        uint4 q;
-        q.x = pack_bf16x2(v[i * 8 + 0], v[i * 8 + 1]);
-        q.y = pack_bf16x2(v[i * 8 + 2], v[i * 8 + 3]);
-        q.z = pack_bf16x2(v[i * 8 + 4], v[i * 8 + 5]);
-        q.w = pack_bf16x2(v[i * 8 + 6], v[i * 8 + 7]);
-        *(uint4*)(e0 + ((i ^ (row & 7)) << 4)) = q;
-      }
-      fence_proxy_async_smem();
-      // output staged (and the exchange slots free again for this group's next tile)
-      asm volatile("bar.sync %0, 128;" ::"r"(1 + grp) : "memory");
-      if (leader) {
-        tma_store_4d(&a.out_map, sg, 0, 0, h0, n);
-        tma_store_commit();
-      }
-      (void)orow;
-    }
-    if (leader) tma_store_wait_all();
-  }
-
-  tc_fence_before();
-  __syncthreads();
-  if (warp == 4) {
-    tc_fence_after();
-    tmem_dealloc<512>(tmem);
-  }
-}
-
 }  // namespace adainf
 
 namespace adainf {

@@ -1,4 +1,9 @@
 #!/bin/bash
 O=gpurun_out
-timeout 900 python bench.py --config c4 --steps 5 > $O/b_c4.json 2> $O/b_c4.err
-timeout 600 python bench.py --steps 5 --no-cpu-baseline > $O/b_c5y.json 2> $O/b_c5y.err
+export N=1024 SHAPES=0 MODES=1 REPS=20
+ADAINF_WSKX=1 timeout 900 python -m pytest tests/test_gpu_conv.py -q -x -k "window" 2>&1 | tail -3 > $O/conv.log
+for r in 1 2; do
+for kx in 0 1; do
+ADAINF_WSKX=$kx timeout 300 python tools/time_layers.py 2>&1 | sed "s/^/kx=$kx /"
+done
+done > $O/tl.log
