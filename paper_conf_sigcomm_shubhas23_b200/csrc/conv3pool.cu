@@ -84,7 +84,7 @@ __global__ void __launch_bounds__(c3p_threads<N, S2D>(), 1) conv3_pool_kernel(co
   constexpr int CP_STAGES = c3p_stages<P, N, S2D>();
   static_assert(CP_STAGES >= 2, "conv3_pool: window stages do not fit");
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_align1024(smem_raw);
   uint8_t* stages = smem;
   uint8_t* wsm = stages + CP_STAGES * STAGE;
   uint64_t* full = (uint64_t*)(wsm + WBYTES);

@@ -352,8 +352,7 @@ __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const Tile
         }
       }
       if (a.res) stage_apply(s0, lane, v, add);
-#pragma unroll
-      for (int i = 0; i < 64; ++i) v[i] = act_apply(a.act, v[i]);
+      act_vec<64>(a.act, v);
     } else {
       if (a.bcast && cur.ok) {
 #pragma unroll
@@ -366,7 +365,8 @@ __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const Tile
         }
       }
       if (cur.scp) stage_apply(s0, lane, v, add);
-      if (ma) stage_apply(s0 + 4096, lane, v, [ma](float x, float y) { return __fmul_rn(x, act_grad(ma, y)); });
+      if (ma == 1) stage_apply(s0 + 4096, lane, v, [](float x, float y) { return __fmul_rn(x, y > 0.f ? 1.f : 0.f); });
+      else if (ma) stage_apply(s0 + 4096, lane, v, [ma](float x, float y) { return __fmul_rn(x, act_grad(ma, y)); });
     }
     __syncwarp();
     // own row -> staging (bf16), then 8 coalesced 16-byte stores per lane
@@ -399,7 +399,7 @@ __global__ void __launch_bounds__(gemm_threads(EW), 1) conv_umma_kernel(const __
   static_assert(ModeTraits<MODE>::B_KMAJ || BN >= 64, "MN-major SW128 B tiles need >= 64 columns");
   constexpr int STAGES = Cfg::STAGES;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_align1024(smem_raw);
   uint64_t* full = (uint64_t*)(smem + STAGES * Cfg::STAGE_BYTES);
   uint64_t* empty = full + STAGES;
   uint64_t* tfull = empty + STAGES;   // [2]

@@ -38,7 +38,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_pair_kernel(const __grid_
   using Cfg = PairCfg<MODE, BN>;
   constexpr int STAGES = Cfg::STAGES;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_align1024(smem_raw);
   uint64_t* full = (uint64_t*)(smem + STAGES * Cfg::STAGE_BYTES);
   uint64_t* empty = full + 8;
   uint64_t* pfull = empty + 8;  // leader: peer stage loaded

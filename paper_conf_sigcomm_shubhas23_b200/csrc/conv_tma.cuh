@@ -331,7 +331,7 @@ template <int BN>
 __global__ void __launch_bounds__(NUM_THREADS, 1) conv_win_tma_kernel(const __grid_constant__ WinTmaArgs a) {
   constexpr int B_BYTES = BN * 128;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_align1024(smem_raw);
   const int WS = a.wstages, BS = a.bstages;
   uint8_t* win = smem;
   uint8_t* bb = win + WS * a.win_bytes;
@@ -569,7 +569,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_tma_kernel(const __
   constexpr int NBUF = 2 * PM * BN <= 512 ? 2 : 1;  // accumulator buffers
   constexpr int TCOLS = PM * BN * NBUF;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_align1024(smem_raw);
   const int ST = a.stages;
   uint64_t* full = (uint64_t*)(smem + ST * STAGE);
   uint64_t* empty = full + 16;
@@ -763,7 +763,7 @@ struct WinWgTmaArgs {
 
 __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_win_tma_kernel(const __grid_constant__ WinWgTmaArgs a) {
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_align1024(smem_raw);
   const int ST = a.stages, Wp = a.Wp, R = a.R;
   const int b_bytes = R * Wp * 128;
   const int stage_bytes = a.a_bytes + b_bytes;

@@ -55,7 +55,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_win_kernel(const WinArgs 
   using Cfg = WinCfg<BN>;
   const ConvArgs& a = w.c;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_align1024(smem_raw);
   uint8_t* win_base = smem;
   uint8_t* b_base = smem + Cfg::WSTAGES * Cfg::WIN_BYTES;
   uint64_t* bars = (uint64_t*)(b_base + Cfg::BSTAGES * Cfg::B_BYTES);
@@ -334,7 +334,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1) conv_win_ws_kernel(const WinArg
   using Cfg = WinWsCfg;
   const ConvArgs& a = w.c;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_align1024(smem_raw);
   uint8_t* win_base = smem;
   uint8_t* b_base = smem + Cfg::WSTAGES * Cfg::WIN_BYTES;
   uint8_t* e_base = b_base + 9 * Cfg::B_BYTES;
@@ -622,7 +622,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_win_wgrad_kernel(const Wi
   using Cfg = WinWgCfg;
   const ConvArgs& a = w.c;  // src = X (Cs = 64), B = dZ (Nout = 64), out = partial, kb_per_split
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_align1024(smem_raw);
   uint8_t* zero = smem + Cfg::STAGES * Cfg::STAGE_BYTES;
   uint64_t* full = (uint64_t*)(zero + Cfg::ZERO_BYTES);
   uint64_t* empty = full + Cfg::STAGES;

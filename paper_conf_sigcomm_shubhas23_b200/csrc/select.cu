@@ -182,7 +182,7 @@ __device__ __forceinline__ void tmem_ld_cols(uint32_t taddr, float* v) {
 template <int P>
 __global__ void __launch_bounds__(SELF_THREADS, 1) select_fused_kernel(const __grid_constant__ SelFusedArgs a) {
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_align1024(smem_raw);
   const int nkb = a.D / 64;
   uint8_t* wsm = smem;                                  // nkb chunks of [P][64] bf16 (P * 128 bytes each)
   uint8_t* xst = wsm + (size_t)nkb * P * 128;           // stage ring

@@ -152,7 +152,7 @@ __device__ __forceinline__ StemUnit stem_unit(const StemFwdArgs& a, int u) {
 
 __global__ void __launch_bounds__(SF_THREADS, 1) stem_fwd_kernel(const __grid_constant__ StemFwdArgs a) {
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_align1024(smem_raw);
   uint8_t* wsm = smem;
   uint8_t* stages = wsm + SF_W_BYTES;
   uint8_t* ring = stages + SF_STAGES * SF_STAGE;
@@ -397,7 +397,7 @@ struct StemWgArgs {
 
 __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_constant__ StemWgArgs a) {
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_align1024(smem_raw);
   uint8_t* dzst = smem;
   uint8_t* sring = dzst + SW_ND * SW_DZ_STAGE;
   uint8_t* guard = sring + SW_NS * SW_S_SLOT;  // finite rows read past the last S slot (invalid positions only)
