@@ -1,4 +1,4 @@
-"""Time every distinct ResNet-18 conv shape (fwd + dgrad) at the retraining batch under each dispatch mode
+"""Time every distinct ResNet-18 conv shape (fwd + dgrad + wgrad) at the retraining batch under each dispatch mode
 (ADAINF window mode: 0 = generic implicit GEMM only, 1 = default routing).  CUDA events, 5 reps."""
 import os
 import sys
@@ -44,7 +44,8 @@ for (H, C, Co, K, s) in shapes:
     for m in modes:
         B.dbg_set_win_mode(m)
         for name, fn in [("fwd", lambda: B.dbg_conv_fwd(x, w, b, s, p, act=1)),
-                         ("dgrad", lambda: B.dbg_conv_dgrad(dz, w, H, H, s, p, sc=sc, yact=x, mask_act=1))]:
+                         ("dgrad", lambda: B.dbg_conv_dgrad(dz, w, H, H, s, p, sc=sc, yact=x, mask_act=1)),
+                         ("wgrad", lambda: B.dbg_conv_wgrad(x, dz, K, K, s, p))]:
             ms = t(fn)
             print(f"H={H:3d} {C:3d}->{Co:3d} k{K} s{s} mode={m} {name:6s} {ms*1e3:8.1f} us "
                   f"{fl/ms/1e9:7.1f} TFLOP/s", flush=True)
