@@ -21,7 +21,7 @@ M=gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,sm__pipe_ten
 timeout 900 ncu --metrics $M --clock-control none --nvtx --nvtx-include "profiled/" --csv \
   --log-file $O/${TAG}_step_traffic.csv python tools/profile_step.py --steps 2 --k 8192 --taus 0.24,0.40,0.61 \
   > $O/${TAG}_step.log 2>&1
-for K in stem_fwd_kernel conv_ws_tma_kernel conv_umma_kernel conv_wgrad_tma_kernel exit_fused_kernel; do
+for K in stem_fwd_kernel conv_ws_tma_kernel conv_umma_kernel conv_wgrad_tma_kernel conv_wgrad_win_tma_kernel conv_dualm_kernel exit_fused_kernel; do
   bash tools/ncu_one.sh ${TAG}_$K "$K" 2 1 -- python tools/profile_step.py --steps 2 --k 1024
 done
 bash tools/ncu_one.sh ${TAG}_stem_wgrad_kernel stem_wgrad_kernel 0 1 -- python tools/profile_step.py --steps 1 --k 1024 --train-only
