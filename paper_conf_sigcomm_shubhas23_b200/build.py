@@ -9,8 +9,10 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-OUT = os.path.join(HERE, "libadainf.so")
-BUILD = os.path.join(HERE, "_build")
+# ADAINF_BUILD_OUT / ADAINF_BUILD_FLAGS: build a variant library elsewhere (A/B timing, -DADAINF_TIMING) without
+# touching the in-tree one
+OUT = os.environ.get("ADAINF_BUILD_OUT", os.path.join(HERE, "libadainf.so"))
+BUILD = os.path.join(os.path.dirname(OUT), "_build") if "ADAINF_BUILD_OUT" in os.environ else os.path.join(HERE, "_build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 
@@ -23,7 +25,8 @@ def _nccl_dir():
 
 
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
-         "-Xcompiler", "-O2", "--expt-relaxed-constexpr", "-Xptxas", "-warn-spills"]
+         "-Xcompiler", "-O2", "--expt-relaxed-constexpr", "-Xptxas", "-warn-spills",
+         *os.environ.get("ADAINF_BUILD_FLAGS", "").split()]
 
 
 def sources():

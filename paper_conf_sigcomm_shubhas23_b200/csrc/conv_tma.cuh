@@ -128,7 +128,7 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
         const int n = tile / a.tpi, h0 = (tile - n * a.tpi) * R;
         const int sn = a.smap ? __ldg(a.smap + n) : n;
         const int s = it % WS, u = it / WS;
-        if (u > 0) mbar_wait(&wempty[s], (u - 1) & 1);
+        if (u > 0) TIMED_WAIT(0, mbar_wait(&wempty[s], (u - 1) & 1));
         if (a.rowbox) {
           mbar_expect_tx(&wfull[s], 64u * 2u * W * (R + 2));
           for (int j = 0; j < R + 2; ++j)
@@ -151,12 +151,15 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
     for (int tp = 0; tp < 9; ++tp) toff[tp] = (uint32_t)a.tap_off[tp] * 8u;
     mbar_wait(bready, 0);
     fence_proxy_async_smem();
+#ifdef ADAINF_TIMING
+    const long long t_mma0 = clock64();
+#endif
     int it = 0;
     for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++it) {
       const int b = it & 1, ub = it >> 1;
-      if (ub > 0) mbar_wait(&tempty[b], (ub - 1) & 1);
+      if (ub > 0) TIMED_WAIT(1, mbar_wait(&tempty[b], (ub - 1) & 1));
       const int s = it % WS, u = it / WS;
-      mbar_wait(&wfull[s], u & 1);
+      TIMED_WAIT(2, mbar_wait(&wfull[s], u & 1));
       tc_fence_after();
       if (elect_one()) {
         const uint32_t sw = wsm + s * a.win_bytes;
@@ -174,6 +177,9 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
       }
       __syncwarp();
     }
+#ifdef ADAINF_TIMING
+    if (lane == 0) atomicAdd(&g_wait_cycles[blockIdx.x & 4095][7], (unsigned long long)(clock64() - t_mma0));
+#endif
   } else {
     // ---- epilogue: 2 groups of 4 warps, group g handles this CTA's local tiles g, g+2, ... ----
     const int grp = (warp - 5) >> 2;
@@ -195,7 +201,7 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
         if (a.has_e1) tma_load_4d(sg + a.has_e0 * 16384, &a.e1_map, &efull[grp], 0, 0, h0, n);
       }
       const int b = grp, ub = lt >> 1;
-      mbar_wait(&tfull[b], ub & 1);
+      TIMED_WAIT(3, mbar_wait(&tfull[b], ub & 1));
       tc_fence_after();
       const uint32_t trow = tmem + (uint32_t)(b * 64) + ((uint32_t)(qd * 32) << 16);
       float v[64];
@@ -203,7 +209,7 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
       tmem_ld32(trow + 32, v + 32);
       tc_fence_before();
       mbar_arrive(&tempty[b]);
-      if (ntens) mbar_wait(&efull[grp], use & 1);
+      if (ntens) TIMED_WAIT(4, mbar_wait(&efull[grp], use & 1));
       uint8_t* e0 = stg + (grp * nstg) * 16384 + row * 128;
       const uint8_t* e1 = e0 + a.has_e0 * 16384;
       if (rv) {
@@ -268,7 +274,7 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
       // global ones (32 L1 wavefronts per warp store), and no global store latency in the epilogue
       if (!ntens) {  // dedicated buffer: the previous tile's store must have read it
         if (leader) tma_store_wait_read();
-        asm volatile("bar.sync %0, 128;" ::"r"(1 + grp) : "memory");
+        TIMED_WAIT(5, asm volatile("bar.sync %0, 128;" ::"r"(1 + grp) : "memory"));
       }
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
@@ -280,7 +286,7 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
         *(uint4*)(e0 + ((i ^ (row & 7)) << 4)) = q;
       }
       fence_proxy_async_smem();
-      asm volatile("bar.sync %0, 128;" ::"r"(1 + grp) : "memory");
+      TIMED_WAIT(6, asm volatile("bar.sync %0, 128;" ::"r"(1 + grp) : "memory"));
       if (leader) {
         tma_store_4d(&a.out_map, sg, 0, 0, h0, n);
         tma_store_commit();
