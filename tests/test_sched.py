@@ -1,7 +1,9 @@
 """Incremental-retraining planning (include/adainf_sched.h) through the C-ABI, host-only
 (no GPU needed): the spare-time split pinned to the paper's worked example and its formula, and the retraining
 setting a time allocation affords (reading in DESIGN.md)."""
+import json
 import math
+import os
 
 import numpy as np
 
@@ -9,13 +11,21 @@ import pytest
 
 from paper_conf_sigcomm_shubhas23_b200 import binding as B
 
+GOLDEN = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden")
+
+
+def _golden(name):
+    with open(os.path.join(GOLDEN, name)) as f:
+        return json.load(f)
+
 
 def test_spare_time_worked_example_p51():
-    """a 400 ms SLO with 200 ms of inference leaves 200 ms of retraining; 300 ms leaves 100 ms."""
-    tr, alloc = B.time_split(400.0, [200.0], [1.0])
-    assert tr == 200.0 and alloc == [200.0]
-    tr, alloc = B.time_split(400.0, [300.0], [1.0])
-    assert tr == 100.0 and alloc == [100.0]
+    """a 400 ms SLO with 200 ms of inference leaves 200 ms of retraining; 300 ms leaves 100 ms
+    (tests/golden/p51_incremental_retraining.json)."""
+    g = _golden("p51_incremental_retraining.json")
+    for c in g["cases"]:
+        tr, alloc = B.time_split(g["slo_ms"], c["inference_ms"], [1.0])
+        assert tr == c["retrain_ms"] and alloc == [c["retrain_ms"]]
 
 
 def test_spare_time_sums_dag_inference_tasks():
@@ -26,9 +36,12 @@ def test_spare_time_sums_dag_inference_tasks():
 
 def test_split_by_impact_degree_p237():
     """T_r * d_j / sum_j d_j; vehicle 0.15 : person 0.09 (the P:86-90 accuracy losses) -> 5:3."""
-    tr, alloc = B.time_split(400.0, [240.0], [0.15, 0.09])
-    assert tr == 160.0
-    assert alloc[0] == pytest.approx(100.0, rel=1e-12) and alloc[1] == pytest.approx(60.0, rel=1e-12)
+    g = _golden("p237_impact_split.json")
+    d, want = g["impact_degrees"], g["expected_alloc_ms"]
+    tr, alloc = B.time_split(g["slo_ms"], g["inference_ms"], [d["vehicle_type"], d["person_activity"]])
+    assert tr == g["expected_retrain_total_ms"]
+    assert alloc[0] == pytest.approx(want["vehicle_type"], rel=1e-12)
+    assert alloc[1] == pytest.approx(want["person_activity"], rel=1e-12)
     assert math.isclose(sum(alloc), tr, rel_tol=1e-12)
     # a model not impacted by drift gets no retraining time (P:196, Observation 2)
     _, alloc = B.time_split(400.0, [240.0], [0.15, 0.0])
@@ -70,10 +83,14 @@ def test_drift_stop_rule_table2():
     """Table 2, S = 3%, 6%, ... of the retraining samples: the impacted set is {} at 3% (reading of
     the garbled cell), {Person} at 6%, {Person, Vehicle} from 9%; the process stops at 18% - the first S whose
     result equals the previous ones for 4 consecutive values - and not before."""
-    PERSON, VEHICLE = 1, 2
-    seq = [0, PERSON, PERSON | VEHICLE, PERSON | VEHICLE, PERSON | VEHICLE, PERSON | VEHICLE]
-    stops = [B.drift_should_stop(seq[:i + 1], n=4) for i in range(len(seq))]
-    assert stops == [False, False, False, False, False, True]  # 3, 6, 9, 12, 15 -> continue; 18% -> stop
+    g = _golden("table2_drift_stop.json")
+    bit = {"Person": 1, "Vehicle": 2}
+    seq = [sum(bit[m] for m in s) for s in g["impacted"]]
+    stops = [B.drift_should_stop(seq[:i + 1], n=g["repeat_n"]) for i in range(len(seq))]
+    first = g["S_percent"][stops.index(True)]
+    assert first == g["stops_at_percent"]  # 3, 6, 9, 12, 15 -> continue; 18% -> stop
+    assert not any(stops[:g["S_percent"].index(first)])
+    assert seq[g["S_percent"].index(first)] == seq[-1]  # the same result as S = 100%
     assert not B.drift_should_stop([], n=4)
     assert B.drift_should_stop([5], n=1)
     assert not B.drift_should_stop([1, 1, 2, 1], n=2)
