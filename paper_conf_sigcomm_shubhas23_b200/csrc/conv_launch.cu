@@ -228,22 +228,35 @@ static void launch_ws_tma(const ConvArgs& c, bool dgrad, int nstatic, cudaStream
   if (e1) a.e1_map = make_tmap_nhwc(e1, nstatic, H, W, 64, 64, Wp, R);
   a.out_map = make_tmap_nhwc(c.out, nstatic, H, W, 64, 64, Wp, R);
   if (!dgrad && c.res_map && c.res_map != c.src_map) throw std::runtime_error("ws_tma: residual map differs");
-  a.win_bytes = ((16 + (R + 2) * Wp) * 128 + 1023) / 1024 * 1024;
   const int fixed = 9 * 8192 + 2 * std::max(1, a.has_e0 + a.has_e1) * 16384 + 1024 /*align*/ +
                     512 /*barriers*/;
-  a.wstages = std::min(8, (227 * 1024 - fixed) / a.win_bytes);
-  if (const char* e = getenv("ADAINF_WS_STAGES")) a.wstages = std::min(a.wstages, std::max(1, atoi(e)));
+  // tile pairs (unit mode) when two pair windows of 2R+2 rows fit next to the resident weights and the
+  // epilogue staging (forward; the dgrad staging of two operands leaves room for one): ADAINF_WS_UNIT=0 disables
+  static int unit_env = -1;
+  if (unit_env < 0) {
+    const char* e = getenv("ADAINF_WS_UNIT");
+    unit_env = e ? atoi(e) : 1;
+  }
+  const int unit_bytes = ((16 + (2 * R + 2) * Wp) * 128 + 1023) / 1024 * 1024;
+  a.unit = unit_env && a.rowbox && 227 * 1024 - fixed >= 2 * unit_bytes;
+  a.upi = (a.tpi + 1) / 2;
+  a.win_bytes = a.unit ? unit_bytes : ((16 + (R + 2) * Wp) * 128 + 1023) / 1024 * 1024;
+  a.wstages = a.unit ? 2 : std::min(8, (227 * 1024 - fixed) / a.win_bytes);
+  if (const char* e = getenv("ADAINF_WS_STAGES"))
+    if (!a.unit) a.wstages = std::min(a.wstages, std::max(1, atoi(e)));
   if (a.wstages < 2) throw std::runtime_error("ws_tma: shared memory");
   const int smem = a.wstages * a.win_bytes + fixed;
   static bool attr = false;
   if (!attr) {
-    CK(cudaFuncSetAttribute(conv_ws_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    CK(cudaFuncSetAttribute(conv_ws_tma_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    CK(cudaFuncSetAttribute(conv_ws_tma_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
     attr = true;
   }
-  const long long tiles = (long long)nstatic * a.tpi;
-  dim3 grid((unsigned)std::max(1LL, std::min<long long>(tiles, num_sms())));
+  const long long items = (long long)nstatic * (a.unit ? a.upi : a.tpi);
+  dim3 grid((unsigned)std::max(1LL, std::min<long long>(items, num_sms())));
   ProfScope ps(dgrad ? PC_CONV_DGRAD : PC_CONV_FWD, st);
-  conv_ws_tma_kernel<<<grid, TMA_WS_THREADS, smem, st>>>(a);
+  if (a.unit) conv_ws_tma_kernel<true><<<grid, TMA_WS_THREADS, smem, st>>>(a);
+  else conv_ws_tma_kernel<false><<<grid, TMA_WS_THREADS, smem, st>>>(a);
   CK(cudaGetLastError());
 }
 

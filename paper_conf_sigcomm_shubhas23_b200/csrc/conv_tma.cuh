@@ -37,10 +37,15 @@ struct WsTmaArgs {
   int wstages, win_bytes;
   int rowbox;  // 1: the window is R+2 boxes {64, W, 1, 1} (one per image row, no out-of-bounds columns); the
                // pad columns W..Wp-1 of every row slot are zeroed once and never written by the TMA
+  int unit;    // 1: work items are PAIRS of vertically adjacent tiles sharing one 2R+2-row window; their MMAs
+               // alternate between the two accumulators and share each B slice through the weight-stationary
+               // collector, one commit per pair (wstages == 2, the window stage doubles as the accumulator pair)
+  int upi;     // unit mode: tile pairs per image = ceil(tpi / 2)
 };
 
 constexpr int TMA_WS_THREADS = 416;  // warp 0 TMA producer (+ warps 1-3 help load B), warp 4 MMA, 8 epilogue warps
 
+template <bool UNIT>
 __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __grid_constant__ WsTmaArgs a) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = smem_align1024(smem_raw);
@@ -62,19 +67,21 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nsamp = a.count ? *a.count : a.n_static;
-  const int ntile = nsamp * a.tpi;
-  if ((int)blockIdx.x >= ntile) return;
+  // work items: tiles, or (unit mode) pairs of vertically adjacent tiles of one image
+  const int nitem = nsamp * (UNIT ? a.upi : a.tpi);
+  if ((int)blockIdx.x >= nitem) return;
   const int Wp = a.Wp, R = a.R, H = a.H, W = a.W;
+  const int WR = UNIT ? 2 * R + 2 : R + 2;  // window rows per item
 
   // zero the 8 lead / 8 trail rows of every window buffer (the TMA never writes them)
   for (int i = threadIdx.x; i < WS * 2 * 64; i += blockDim.x) {
     const int s = i / 128, k = i % 128;
-    const int rows = 8 + (R + 2) * Wp;
+    const int rows = 8 + WR * Wp;
     uint4* p = (uint4*)(win + s * a.win_bytes + (k < 64 ? k * 16 : rows * 128 + (k - 64) * 16));
     *p = make_uint4(0, 0, 0, 0);
   }
   if (a.rowbox) {
-    const int padc = Wp - W, per_stage = (R + 2) * padc * 8;
+    const int padc = Wp - W, per_stage = WR * padc * 8;
     for (int i = threadIdx.x; i < WS * per_stage; i += blockDim.x) {
       const int s = i / per_stage, k = i - s * per_stage;
       const int j = k / (padc * 8), rem = k - j * (padc * 8);
@@ -90,14 +97,14 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&tfull[b], 1);
-      mbar_init(&tempty[b], 128);
+      mbar_init(&tempty[b], UNIT ? 256 : 128);
       mbar_init(&efull[b], 1);
     }
     mbar_init(bready, 128);
     fence_mbar_init();
     tma_prefetch_desc(&a.win_map);
   }
-  if (warp == 4) tmem_alloc<128>(tmem_slot);
+  if (warp == 4) tmem_alloc<UNIT ? 256 : 128>(tmem_slot);
   fence_proxy_async_smem();
   tc_fence_before();
   __syncthreads();
@@ -124,14 +131,16 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
     // ---- windows: one TMA box per tile, issued by one thread ----
     if (warp == 0 && lane == 0) {
       int it = 0;
-      for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++it) {
-        const int n = tile / a.tpi, h0 = (tile - n * a.tpi) * R;
+      const int per = UNIT ? a.upi : a.tpi;
+      for (int item = blockIdx.x; item < nitem; item += gridDim.x, ++it) {
+        const int n = item / per, h0 = (item - n * per) * (UNIT ? 2 * R : R);
         const int sn = a.smap ? __ldg(a.smap + n) : n;
         const int s = it % WS, u = it / WS;
-        if (u > 0) TIMED_WAIT(0, mbar_wait(&wempty[s], (u - 1) & 1));
+        // unit mode: the pair's commit (tfull) also frees its window stage (wstages == 2)
+        if (u > 0) TIMED_WAIT(0, mbar_wait(UNIT ? &tfull[s] : &wempty[s], (u - 1) & 1));
         if (a.rowbox) {
-          mbar_expect_tx(&wfull[s], 64u * 2u * W * (R + 2));
-          for (int j = 0; j < R + 2; ++j)
+          mbar_expect_tx(&wfull[s], 64u * 2u * W * WR);
+          for (int j = 0; j < WR; ++j)
             tma_load_4d(wsm + s * a.win_bytes + 1024 + j * Wp * 128, &a.win_map, &wfull[s], 0, 0, h0 - 1 + j, sn);
         } else {
           mbar_expect_tx(&wfull[s], box_bytes);
@@ -155,7 +164,8 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
     const long long t_mma0 = clock64();
 #endif
     int it = 0;
-    for (int tile = blockIdx.x; tile < ntile; tile += gridDim.x, ++it) {
+    const uint32_t unit_off = (uint32_t)(R * Wp * 8);  // second tile of a pair: R rows further (16-byte units)
+    for (int item = blockIdx.x; item < nitem; item += gridDim.x, ++it) {
       const int b = it & 1, ub = it >> 1;
       if (ub > 0) TIMED_WAIT(1, mbar_wait(&tempty[b], (ub - 1) & 1));
       const int s = it % WS, u = it / WS;
@@ -163,17 +173,32 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
       tc_fence_after();
       if (elect_one()) {
         const uint32_t sw = wsm + s * a.win_bytes;
-        const uint32_t dacc = tmem + (uint32_t)(b * 64);
         const uint64_t a_base = make_sdesc(sw, 16, 1024);
+        if constexpr (UNIT) {
+          const uint32_t d0 = tmem + (uint32_t)(b * 128);
 #pragma unroll
-        for (int tp = 0; tp < 9; ++tp) {
+          for (int tp = 0; tp < 9; ++tp) {
 #pragma unroll
-          for (int kk = 0; kk < 4; ++kk)
-            umma_bf16(dacc, a_base + (toff[tp] + 2u * kk), b_base + (uint32_t)(tp * 512 + kk * b_kk), IDESC,
-                      (tp | kk) != 0);
+            for (int kk = 0; kk < 4; ++kk) {
+              const uint64_t bd = b_base + (uint32_t)(tp * 512 + kk * b_kk);
+              const uint32_t acc = (tp | kk) != 0;
+              umma_bf16_ws_fill(d0, a_base + (toff[tp] + 2u * kk), bd, IDESC, acc);
+              umma_bf16_ws_lastuse(d0 + 64u, a_base + (toff[tp] + 2u * kk + unit_off), bd, IDESC, acc);
+            }
+          }
+          umma_commit(&tfull[b]);
+        } else {
+          const uint32_t dacc = tmem + (uint32_t)(b * 64);
+#pragma unroll
+          for (int tp = 0; tp < 9; ++tp) {
+#pragma unroll
+            for (int kk = 0; kk < 4; ++kk)
+              umma_bf16(dacc, a_base + (toff[tp] + 2u * kk), b_base + (uint32_t)(tp * 512 + kk * b_kk), IDESC,
+                        (tp | kk) != 0);
+          }
+          umma_commit(&wempty[s]);
+          umma_commit(&tfull[b]);
         }
-        umma_commit(&wempty[s]);
-        umma_commit(&tfull[b]);
       }
       __syncwarp();
     }
@@ -187,9 +212,12 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
     const int row = qd * 32 + lane;  // output position p within the tile
     const bool leader = (warp == 5 + 4 * grp) && lane == 0;
     const uint32_t sg = ssm + grp * nstg * 16384;
-    int lt = grp, use = 0;
-    for (int tile = blockIdx.x + grp * gridDim.x; tile < ntile; tile += 2 * gridDim.x, lt += 2, ++use) {
-      const int n = tile / a.tpi, h0 = (tile - n * a.tpi) * R;
+    // tile mode: group g takes this CTA's items g, g+2, ...; unit mode: group g takes tile g of every pair
+    int lt = UNIT ? 0 : grp, use = 0;
+    for (int item = blockIdx.x + (UNIT ? 0 : grp * gridDim.x); item < nitem;
+         item += (UNIT ? 1 : 2) * gridDim.x, lt += (UNIT ? 1 : 2), ++use) {
+      const int per = UNIT ? a.upi : a.tpi;
+      const int n = item / per, h0 = (item - n * per) * (UNIT ? 2 * R : R) + (UNIT ? grp * R : 0);
       const int h = h0 + row / Wp, x = row % Wp;
       const bool rv = h < H && x < W;
       const long long orow = ((long long)n * H + h) * W + x;
@@ -200,10 +228,10 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
         if (a.has_e0) tma_load_4d(sg, &a.e0_map, &efull[grp], 0, 0, h0, sn);
         if (a.has_e1) tma_load_4d(sg + a.has_e0 * 16384, &a.e1_map, &efull[grp], 0, 0, h0, n);
       }
-      const int b = grp, ub = lt >> 1;
+      const int b = UNIT ? (lt & 1) : grp, ub = lt >> 1;
       TIMED_WAIT(3, mbar_wait(&tfull[b], ub & 1));
       tc_fence_after();
-      const uint32_t trow = tmem + (uint32_t)(b * 64) + ((uint32_t)(qd * 32) << 16);
+      const uint32_t trow = tmem + (uint32_t)(UNIT ? b * 128 + grp * 64 : b * 64) + ((uint32_t)(qd * 32) << 16);
       float v[64];
       tmem_ld32(trow, v);
       tmem_ld32(trow + 32, v + 32);
@@ -301,7 +329,7 @@ __global__ void __launch_bounds__(TMA_WS_THREADS, 1) conv_ws_tma_kernel(const __
   __syncthreads();
   if (warp == 4) {
     tc_fence_after();
-    tmem_dealloc<128>(tmem);
+    tmem_dealloc<UNIT ? 256 : 128>(tmem);
   }
 }
 
@@ -860,14 +888,19 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_wgrad_win_tma_kernel(cons
           }
           const uint64_t db0 = make_sdesc(sb, 8192, 1024);
           const uint32_t acc0 = kb != kb0;
+          // the five tap-pair MMAs of a K-step share B (the dZ slice): read it once into the weight-stationary
+          // collector (fill / use / lastuse)
+          umma_bf16_ws_fill(tmem, da[0], db0, IDESC, acc0);
 #pragma unroll
-          for (int p = 0; p < 5; ++p) umma_bf16(tmem + (uint32_t)(p * 64), da[p], db0, IDESC, acc0);
+          for (int p = 1; p < 4; ++p) umma_bf16_ws_use(tmem + (uint32_t)(p * 64), da[p], db0, IDESC, acc0);
+          umma_bf16_ws_lastuse(tmem + 256u, da[4], db0, IDESC, acc0);
           for (int kk = 1; kk < ksteps; ++kk) {
             const uint64_t inc = (uint64_t)(kk * 128);
+            umma_bf16_ws_fill(tmem, da[0] + inc, db0 + inc, IDESC, 1u);
 #pragma unroll
-            for (int p = 0; p < 4; ++p) umma_bf16(tmem + (uint32_t)(p * 64), da[p] + inc, db0 + inc, IDESC, 1u);
+            for (int p = 1; p < 4; ++p) umma_bf16_ws_use(tmem + (uint32_t)(p * 64), da[p] + inc, db0 + inc, IDESC, 1u);
             // the tenth atom (zero) stays in place: LBO shrinks by the same 2048 B per K-step
-            umma_bf16(tmem + 256u, da[4] + inc - ((uint64_t)(kk * 128) << 16), db0 + inc, IDESC, 1u);
+            umma_bf16_ws_lastuse(tmem + 256u, da[4] + inc - ((uint64_t)(kk * 128) << 16), db0 + inc, IDESC, 1u);
           }
           umma_commit(&empty[s]);
           if (kb == kb1 - 1) umma_commit(tfull);

@@ -165,7 +165,10 @@ def test_conv_wgrad_vs_torch(case):
 
 
 WIN_CASES = [(2, 14, 14, 64, 64), (3, 7, 7, 128, 256), (2, 28, 28, 64, 128), (1, 56, 56, 64, 64), (5, 9, 11, 64, 64),
-             (2, 14, 14, 256, 256), (3, 28, 28, 128, 128), (2, 12, 20, 128, 128), (2, 9, 13, 128, 256)]
+             (2, 14, 14, 256, 256), (3, 28, 28, 128, 128), (2, 12, 20, 128, 128), (2, 9, 13, 128, 256),
+             # odd tiles per image (W = 20 -> pitch 32, 4 rows per tile, 5 tiles): the last tile pair of the
+             # 64-channel kernel's pair mode has one tile inside the image
+             (3, 20, 20, 64, 64)]
 
 
 @pytest.mark.parametrize("mode", [1, 2])

@@ -296,6 +296,22 @@ int main(int argc, char** argv) {
              2.0 * 148 * 80000.0 * 128 * nn * 16 / ms / 1e9);
     };
     run1(mma_rate<1, 64>, 64);
+    {  // CTA pair at N = 64 (M = 256): each SM reads its A half and HALF of B per MMA
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = dim3(148);
+      cfg.blockDim = dim3(128);
+      cudaLaunchAttribute at[1];
+      at[0].id = cudaLaunchAttributeClusterDimension;
+      at[0].val.clusterDim.x = 2; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+      cfg.attrs = at;
+      cfg.numAttrs = 1;
+      cudaLaunchKernelEx(&cfg, mma_rate<2, 64>, a, 20000, cyc2);
+      cudaDeviceSynchronize();
+      long long hc[1];
+      cudaMemcpy(hc, cyc2, 8, cudaMemcpyDeviceToHost);
+      printf("cta_group::2 M=256 N=64 K=16: %.1f cycles per MMA (per-SM work = one M=128 N=64 K=16 tile)\n",
+             (double)hc[0] / 80000);
+    }
     for (int per : {36}) {
       const int tiles = 80000 / per;
       mma_commit_rate<2, 2><<<148, 128>>>(tiles, per, cyc2);

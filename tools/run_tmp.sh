@@ -1,8 +1,7 @@
 #!/bin/bash
 O=gpurun_out
-timeout 600 python -m pytest tests/test_gpu_conv.py -q -x -k "dgrad" 2>&1 | tail -2 > $O/sp_tests.log
-export N=1024 SHAPES=1,4,7 MODES=1 REPS=20
-for r in 1 2; do
-ADAINF_LIB=/root/repo/_variants/base/libadainf.so timeout 300 python tools/time_layers.py 2>&1 | grep dgrad | sed "s/^/base /"
-timeout 300 python tools/time_layers.py 2>&1 | grep dgrad | sed "s/^/new  /"
-done > $O/sp_time.log
+python -c "import __graft_entry__ as g; g.build(); g.smoke()" > $O/build.log 2>&1
+timeout 1500 python -m pytest tests -m gpu -q -x 2>&1 | tail -3 > $O/full.log
+export N=1024 SHAPES=0 MODES=1 REPS=20
+timeout 300 python tools/time_layers.py > $O/l1.log 2>&1
+timeout 900 python bench.py > $O/bench_c5.json 2> $O/bench_c5.err

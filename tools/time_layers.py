@@ -45,6 +45,7 @@ for (H, C, Co, K, s) in shapes:
         B.dbg_set_win_mode(m)
         for name, fn in [("fwd", lambda: B.dbg_conv_fwd(x, w, b, s, p, act=1)),
                          ("dgrad", lambda: B.dbg_conv_dgrad(dz, w, H, H, s, p, sc=sc, yact=x, mask_act=1)),
+                         ("dgrad-nosc", lambda: B.dbg_conv_dgrad(dz, w, H, H, s, p, yact=x, mask_act=1)),
                          ("wgrad", lambda: B.dbg_conv_wgrad(x, dz, K, K, s, p))]:
             ms = t(fn)
             print(f"H={H:3d} {C:3d}->{Co:3d} k{K} s{s} mode={m} {name:6s} {ms*1e3:8.1f} us "
