@@ -615,10 +615,14 @@ __global__ void __launch_bounds__(SW_THREADS, 1) stem_wgrad_kernel(const __grid_
             bdesc[o] = make_sdesc_sw32(s_u + ((Lb + (i - i0) + o) % SW_NS) * SW_S_SLOT, 32, 256);
 #pragma unroll 1
           for (int kk = 0; kk < 8; ++kk) {
+            // the five MMAs of a K-step share A (the dZ row pair): read it once into the A collector
+            const uint64_t ad = adesc0 + (uint64_t)(kk * 128);
+            const uint32_t acc = (!first || kk > 0) ? 1u : 0u;
+            umma_bf16_acoll<0>(tmem, ad, bdesc[0] + (uint64_t)(kk * 32), IDESC, acc);
 #pragma unroll
-            for (int o = 0; o < 5; ++o)
-              umma_bf16(tmem + (uint32_t)(o * 64), adesc0 + (uint64_t)(kk * 128), bdesc[o] + (uint64_t)(kk * 32),
-                        IDESC, (!first || kk > 0) ? 1u : 0u);
+            for (int o = 1; o < 4; ++o)
+              umma_bf16_acoll<1>(tmem + (uint32_t)(o * 64), ad, bdesc[o] + (uint64_t)(kk * 32), IDESC, acc);
+            umma_bf16_acoll<2>(tmem + 256u, ad, bdesc[4] + (uint64_t)(kk * 32), IDESC, acc);
           }
           umma_commit(&dz_empty[st]);
           // S rows i - 2, i - 1 are not used by the next pair; the unit's last pair releases all five
