@@ -133,8 +133,9 @@ __global__ void __launch_bounds__(DUALM_THREADS, 1) conv_dualm_kernel(const __gr
           constexpr uint32_t B_KK = MODE == MODE_FWD ? 2u : 128u;
 #pragma unroll
           for (int kk = 0; kk < BK / 16; ++kk) {
-            umma_bf16(dacc, a0 + 2u * kk, bd0 + kk * B_KK, IDESC, (kb | kk) != 0);
-            umma_bf16(dacc + BN, a1 + 2u * kk, bd0 + kk * B_KK, IDESC, (kb | kk) != 0);
+            // both M tiles multiply the same weight slice: the second reads it from the B collector
+            umma_bf16_ws_fill(dacc, a0 + 2u * kk, bd0 + kk * B_KK, IDESC, (kb | kk) != 0);
+            umma_bf16_ws_lastuse(dacc + BN, a1 + 2u * kk, bd0 + kk * B_KK, IDESC, (kb | kk) != 0);
           }
           umma_commit(&empty[s]);
           if (kb == nkb - 1) umma_commit(&tfull[b]);
