@@ -57,14 +57,16 @@ static void launch_t(const ConvArgs& a, long long max_tiles, cudaStream_t st) {
 }
 
 // ---- CTA-pair kernel (cta_group::2, M = 256 tiles) ----
-// Off by default (ADAINF_PAIR=1 enables): it is parity-green but measured ~2x slower than the single-CTA kernel
-// on ResNet layer 2 (the peer's per-stage completion forwarding and remote epilogue releases are cluster-scope
-// release operations on the critical path); see DESIGN.md section 11.
+// Default for the BN = 256 layers (ResNet layers 3-4 forward and stride-1 dgrad; BN = 128 goes to the dual-M
+// kernel first): both CTAs' TMA loads complete on the leader's stage barrier (.cta_group::2), so per SM the
+// weight operand's shared-memory reads, writes and L2 -> SM bytes halve with no forwarding hop.  1,024 images:
+// layer-3 fwd 178 -> 156 us, dgrad 202 -> 181 us; layer-4 fwd 177 -> 155 us, dgrad 195 -> 173 us.
+// ADAINF_PAIR=0 disables.
 static int g_pair = -1;
 static bool pair_on() {
   if (g_pair < 0) {
     const char* e = getenv("ADAINF_PAIR");
-    g_pair = e ? atoi(e) : 0;
+    g_pair = e ? atoi(e) : 1;
   }
   return g_pair != 0;
 }

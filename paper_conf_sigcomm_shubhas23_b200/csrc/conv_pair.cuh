@@ -7,8 +7,9 @@
 // traffic, which bound the single-CTA kernel at N <= 128 (ResNet layer 2).
 //
 // Synchronisation (validated with tools/exp_2cta.cu):
-//   full[s]   local TMA completion (expect_tx) in each CTA; the peer's MMA-warp lane forwards its
-//             completion to the leader's pfull[s] (remote mbarrier arrive)
+//   full[s]   the LEADER's barrier, two arrivals per stage: each CTA's producer arms it with its own bytes
+//             (remote arrive.expect_tx from the peer) and issues its TMA loads with .cta_group::2, so both
+//             halves complete their transaction bytes on it directly (no forwarding hop through the peer)
 //   empty[s]  tcgen05.commit.cta_group::2 multicast to both CTAs (each producer reuses its own stage)
 //   tfull[b]  same multicast commit at the tile's last K-block (each epilogue reads its own TMEM lanes)
 //   tempty[b] leader-side, 256 arrivals: both CTAs' epilogue threads (the peer's arrive remotely)
@@ -66,7 +67,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_pair_kernel(const __grid_
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < STAGES; ++s) {
-      mbar_init(&full[s], 1);
+      mbar_init(&full[s], 2);
       mbar_init(&empty[s], 1);
       mbar_init(&pfull[s], 1);
     }
@@ -111,16 +112,17 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_pair_kernel(const __grid_
           const int s = it % STAGES, u = it / STAGES;
           if (u > 0) mbar_wait(&empty[s], (u - 1) & 1);
           const uint32_t sa = smem_base + s * Cfg::STAGE_BYTES, sb = sa + Cfg::A_BYTES;
-          mbar_expect_tx(&full[s], (uint32_t)Cfg::STAGE_BYTES);
-          tma_load_im2col_4d(sa, &a.a_map, &full[s], c, bw, bh, n0i, (uint16_t)(a.tx[tap] - a.a_lo),
-                             (uint16_t)(a.ty[tap] - a.a_lo));
+          const uint32_t fbar = mapa_rank(smem_u32(&full[s]), 0);  // the leader's stage barrier
+          mbar_expect_tx_cluster(fbar, (uint32_t)Cfg::STAGE_BYTES);
+          tma_load_im2col_4d_cg2(sa, &a.a_map, fbar, c, bw, bh, n0i, (uint16_t)(a.tx[tap] - a.a_lo),
+                                 (uint16_t)(a.ty[tap] - a.a_lo));
           if (MODE == MODE_FWD) {
-            tma_load_2d(sb, &a.b_map, &full[s], kb * BK, n0 + (int)rank * (BN / 2));  // box {64 K, BN/2 rows}
+            tma_load_2d_cg2(sb, &a.b_map, fbar, kb * BK, n0 + (int)rank * (BN / 2));  // box {64 K, BN/2 rows}
           } else {
 #pragma unroll
             for (int b = 0; b < BN / 128; ++b)
-              tma_load_2d(sb + b * 8192, &a.b_map, &full[s], a.btap[tap] * a.Nout + n0 + (int)rank * (BN / 2) + b * 64,
-                          c);
+              tma_load_2d_cg2(sb + b * 8192, &a.b_map, fbar,
+                              a.btap[tap] * a.Nout + n0 + (int)rank * (BN / 2) + b * 64, c);
           }
           c += BK;
           if (c >= a.Cs) c = 0, ++tap;
@@ -129,17 +131,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_pair_kernel(const __grid_
     }
   } else if (warp == 4) {
     if (rank == 1) {
-      // ---- peer: forward each local stage completion to the leader ----
-      if (lane == 0) {
-        const uint32_t remote_pfull = mapa_rank(smem_u32(pfull), 0);
-        int it = 0;
-        for (int tile = pair; tile < ntile; tile += npairs)
-          for (int kb = 0; kb < nkb; ++kb, ++it) {
-            const int s = it % STAGES, u = it / STAGES;
-            mbar_wait(&full[s], u & 1);
-            mbar_arrive_cluster(remote_pfull + s * 8);
-          }
-      }
+      // peer: its stages complete on the leader's barriers; nothing to issue
     } else {
       // ---- leader: tcgen05.mma.cta_group::2, M = 256 ----
       constexpr uint32_t IDESC = make_idesc(2 * BM, BN, 0, MODE == MODE_FWD ? 0 : 1);
@@ -152,7 +144,6 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_pair_kernel(const __grid_
         for (int kb = 0; kb < nkb; ++kb, ++it) {
           const int s = it % STAGES, u = it / STAGES;
           mbar_wait(&full[s], u & 1);
-          mbar_wait(&pfull[s], u & 1);
           tc_fence_after();
           if (elect_one()) {
             const uint32_t sa = smem_base + s * Cfg::STAGE_BYTES, sb = sa + Cfg::A_BYTES;
