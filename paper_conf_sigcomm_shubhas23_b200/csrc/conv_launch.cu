@@ -668,8 +668,15 @@ void conv_dgrad_sp(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, bf
   a.sp_cin = g.Cin;
   a.sp_sc_compact = sc_compact ? 1 : 0;
   a.b_tma = 1;
-  a.b_map = make_tmap_2d(wsp, a.Nout, a.K, a.ldb, 64, 256);
   try_a_tma(a);
+  // CTA pair when the packed weights span several N tiles (layers 3-4: 4*Cin >= 512; each CTA streams half of
+  // them per K-block): layer-4 sub-pixel dgrad 178 -> 158 us, layer 3 223 -> 221 us; layer 2 (one N tile,
+  // epilogue-bound) is 3% slower as a pair and stays single
+  if (a.a_tma && pair_on() && a.Nout >= 512) {
+    a.b_map = make_tmap_2d(wsp, a.Nout, a.K, a.ldb, 64, 128);
+    if (try_launch_pair<MODE_DGRAD_SP>(256, a, (long long)n * g.Ho * g.Wo, st)) return;
+  }
+  a.b_map = make_tmap_2d(wsp, a.Nout, a.K, a.ldb, 64, 256);
   const long long mt = ((long long)n * g.Ho * g.Wo + BM - 1) / BM;
   launch_t<MODE_DGRAD_SP, 256>(a, mt * ((a.Nout + 255) / 256), st);
 }

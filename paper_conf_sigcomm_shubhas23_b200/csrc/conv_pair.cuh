@@ -24,7 +24,8 @@ struct PairCfg {
   static constexpr int A_BYTES = BM * BK * 2;
   static constexpr int B_BYTES = (BN / 2) * BK * 2;  // this CTA's half of the weight tile
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int EPI_BYTES = 4 * 8192;
+  // the sub-pixel dgrad's epilogue double-buffers its two staged operands per warp
+  static constexpr int EPI_BYTES = MODE == MODE_DGRAD_SP ? 4 * 16384 : 4 * 8192;
   static constexpr int BIAS_BYTES = MODE == MODE_FWD ? 4096 : 0;
   static constexpr int STAGES_FIT = (220 * 1024 - EPI_BYTES - BIAS_BYTES - 1280) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_FIT > 8 ? 8 : STAGES_FIT;
@@ -34,7 +35,8 @@ struct PairCfg {
 
 template <int MODE, int BN>
 __global__ void __launch_bounds__(NUM_THREADS, 1) conv_pair_kernel(const __grid_constant__ ConvArgs a) {
-  static_assert(MODE == MODE_FWD || MODE == MODE_DGRAD, "pair kernel: FWD / DGRAD");
+  static_assert(MODE == MODE_FWD || MODE == MODE_DGRAD || MODE == MODE_DGRAD_SP, "pair kernel: FWD / DGRAD / SP");
+  constexpr bool B_KMAJ = MODE != MODE_DGRAD;  // FWD and the sub-pixel dgrad: K-major weight rows
   static_assert(BN == 128 || BN == 256, "pair kernel: BN 128 / 256");
   using Cfg = PairCfg<MODE, BN>;
   constexpr int STAGES = Cfg::STAGES;
@@ -116,7 +118,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_pair_kernel(const __grid_
           mbar_expect_tx_cluster(fbar, (uint32_t)Cfg::STAGE_BYTES);
           tma_load_im2col_4d_cg2(sa, &a.a_map, fbar, c, bw, bh, n0i, (uint16_t)(a.tx[tap] - a.a_lo),
                                  (uint16_t)(a.ty[tap] - a.a_lo));
-          if (MODE == MODE_FWD) {
+          if (B_KMAJ) {
             tma_load_2d_cg2(sb, &a.b_map, fbar, kb * BK, n0 + (int)rank * (BN / 2));  // box {64 K, BN/2 rows}
           } else {
 #pragma unroll
@@ -134,7 +136,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_pair_kernel(const __grid_
       // peer: its stages complete on the leader's barriers; nothing to issue
     } else {
       // ---- leader: tcgen05.mma.cta_group::2, M = 256 ----
-      constexpr uint32_t IDESC = make_idesc(2 * BM, BN, 0, MODE == MODE_FWD ? 0 : 1);
+      constexpr uint32_t IDESC = make_idesc(2 * BM, BN, 0, B_KMAJ ? 0 : 1);
       int it = 0, lt = 0;
       for (int tile = pair; tile < ntile; tile += npairs, ++lt) {
         const int b = lt & 1, ub = lt >> 1;
@@ -148,8 +150,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_pair_kernel(const __grid_
           if (elect_one()) {
             const uint32_t sa = smem_base + s * Cfg::STAGE_BYTES, sb = sa + Cfg::A_BYTES;
             const uint64_t ad0 = make_sdesc(sa, 16, 1024);
-            const uint64_t bd0 = MODE == MODE_FWD ? make_sdesc(sb, 16, 1024) : make_sdesc(sb, 8192, 1024);
-            constexpr uint32_t B_KK = MODE == MODE_FWD ? 2u : 128u;
+            const uint64_t bd0 = B_KMAJ ? make_sdesc(sb, 16, 1024) : make_sdesc(sb, 8192, 1024);
+            constexpr uint32_t B_KK = B_KMAJ ? 2u : 128u;
 #pragma unroll
             for (int kk = 0; kk < BK / 16; ++kk) {
               asm volatile(
@@ -208,7 +210,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_pair_kernel(const __grid_
       }
       epilogue_coalesced<MODE, BN, 1>(a, ti, trow, &tfull[b], ub & 1,
                                       rank ? nullptr : &tempty[b], nkb, m, rv, n, orow, rrow, HWg,
-                                      epi_smem + q * 8192, lane, bias_s, 0,
+                                      epi_smem + q * (Cfg::EPI_BYTES / 4), lane, bias_s, 0,
                                       rank ? remote_tempty + (uint32_t)(b * 8) : 0u);
     }
   }
