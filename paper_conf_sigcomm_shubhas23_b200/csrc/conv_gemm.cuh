@@ -276,6 +276,10 @@ __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const Tile
   // operand 0: FWD residual / DGRAD shortcut term; operand 1: DGRAD activation (mask)
   auto issue = [&](const EpiBlk& e, int par) {
     uint8_t* s0 = stg + (PIPE ? par * 8192 : 0);
+    if (a.exp_flags & 4) {  // experiment: no operand loads
+      asm volatile("cp.async.commit_group;" ::: "memory");
+      return;
+    }
     if (MODE == MODE_FWD) {
       if (a.res) stage_issue(s0, a.res + e.ocol, rrow, e.ok, e.NO, lane);
     } else {
@@ -386,7 +390,7 @@ __device__ __forceinline__ void epilogue_coalesced(const ConvArgs& a, const Tile
       const long long pr = __shfl_sync(0xffffffffu, cur.orow, r);
       const int okr = __shfl_sync(0xffffffffu, (int)cur.ok, r);
       const uint4 x = *(const uint4*)(s0 + stg_off(r, j));
-      if (okr) *((uint4*)(ob + pr * cur.NO) + j) = x;
+      if (okr && !(a.exp_flags & 8)) *((uint4*)(ob + pr * cur.NO) + j) = x;
     }
     __syncwarp();
     cur = nxt;

@@ -667,6 +667,7 @@ void conv_dgrad_sp(const ConvGeom& g, const bf16* dz, const bf16* w, int ldb, bf
   a.mask_act = mask_act;
   a.sp_cin = g.Cin;
   a.sp_sc_compact = sc_compact ? 1 : 0;
+  if (const char* e = getenv("ADAINF_EXP")) a.exp_flags = atoi(e);  // experiments only
   a.b_tma = 1;
   try_a_tma(a);
   // CTA pair when the packed weights span several N tiles (layers 3-4: 4*Cin >= 512; each CTA streams half of
