@@ -51,7 +51,17 @@ __global__ void __launch_bounds__(128, 1) rate(int tiles, int nacc, int ncommit,
       }
       if (elect_one()) {
         const uint32_t d = tmem + (uint32_t)((t % nacc) * 64);
-        if (STYLE >= 2) {
+        if (STYLE == 4 || STYLE == 5) {
+          // MN-major A (STYLE 4) / MN-major A and B (STYLE 5): SW128 atoms of 64 MN elements x 8 K rows; one
+          // K = 16 step = 16 rows of 128 B = +2 KB (128 descriptor units); two 64-row M atoms 8 KB apart
+          constexpr uint32_t ID2 = make_idesc(128, 64, 1, STYLE == 5 ? 1 : 0);
+          const uint64_t am = make_sdesc(smem_u32(sA), 8192, 1024), bm = STYLE == 5 ? make_sdesc(smem_u32(sB), 8192, 1024) : bd;
+#pragma unroll
+          for (int i = 0; i < PER; ++i) {
+            const uint32_t ko = (uint32_t)((i % 4) * 128);
+            umma_bf16(d, am + ko, STYLE == 5 ? bm + ko : bm + (uint32_t)(2 * (i % 4)), ID2, i > 0);
+          }
+        } else if (STYLE >= 2) {
           // two tiles per unit, MMAs alternating between their accumulators (same B for each pair); STYLE 3
           // keeps the pair's B in the weight-stationary collector (fill / lastuse)
           const uint32_t d0 = tmem + (uint32_t)((t % 2) * 128);
@@ -117,6 +127,11 @@ int main() {
       {36, 1, 2, 1, 1, 2, "36/tile runtime tap offsets: 1 commit, wait t-2"},
       {36, 1, 4, 1, 2, 4, "36/tile runtime tap offsets: 1 commit, wait t-4 every 2nd"},
       {72, 0, 2, 1, 1, 2, "72/tile const descs: 1 commit, wait t-2"},
+      {36, 4, 2, 0, 0, 0, "36/tile MN-major A, no commit, no wait"},
+      {36, 5, 2, 0, 0, 0, "36/tile MN-major A and B, no commit, no wait"},
+      {144, 0, 2, 0, 0, 0, "144/tile K-major, no commit"},
+      {144, 4, 2, 0, 0, 0, "144/tile MN-major A, no commit"},
+      {144, 5, 2, 0, 0, 0, "144/tile MN-major A and B, no commit"},
       {72, 2, 2, 1, 1, 2, "2-tile unit (72 MMAs alternating 2 accs): 1 commit, wait u-2"},
       {72, 3, 2, 1, 1, 2, "2-tile unit + B collector (ws fill/lastuse): 1 commit, wait u-2"},
       {72, 2, 2, 3, 1, 2, "2-tile unit: 3 commits, wait u-2"},
@@ -130,6 +145,11 @@ int main() {
     const int tiles = 144000 / c.per;
     if (c.per == 36 && c.style == 0) rate<36, 0><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
     if (c.per == 36 && c.style == 1) rate<36, 1><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
+    if (c.per == 36 && c.style == 4) rate<36, 4><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
+    if (c.per == 36 && c.style == 5) rate<36, 5><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
+    if (c.per == 144 && c.style == 0) rate<144, 0><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
+    if (c.per == 144 && c.style == 4) rate<144, 4><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
+    if (c.per == 144 && c.style == 5) rate<144, 5><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
     if (c.per == 72 && c.style == 0) rate<72, 0><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
     if (c.per == 72 && c.style == 2) rate<72, 2><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
     if (c.per == 72 && c.style == 3) rate<72, 3><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
