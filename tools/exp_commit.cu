@@ -51,7 +51,18 @@ __global__ void __launch_bounds__(128, 1) rate(int tiles, int nacc, int ncommit,
       }
       if (elect_one()) {
         const uint32_t d = tmem + (uint32_t)((t % nacc) * 64);
-        if (STYLE == 4 || STYLE == 5) {
+        if (STYLE == 6 || STYLE == 7) {
+          // tap-shifted views (start offsets of 1..3 x 128 B, not 1024-aligned): STYLE 6 MN-major A with two
+          // M atoms at a tap-pair distance (the weight-gradient window kernel), STYLE 7 K-major A (layer-1 fwd)
+          constexpr uint32_t ID2 = make_idesc(128, 64, STYLE == 6 ? 1 : 0, 0);
+#pragma unroll
+          for (int i = 0; i < PER; ++i) {
+            const uint32_t sh = (uint32_t)((i / 4) % 3) * 8u;  // 0, 128, 256 B
+            const uint64_t am = STYLE == 6 ? make_sdesc(smem_u32(sA) + sh * 16u, 1152, 1024) + (uint32_t)((i % 4) * 128)
+                                           : make_sdesc(smem_u32(sA) + sh * 16u, 16, 1024) + (uint32_t)(2 * (i % 4));
+            umma_bf16(d, am, bd + (uint32_t)(2 * (i % 4)), ID2, i > 0);
+          }
+        } else if (STYLE == 4 || STYLE == 5) {
           // MN-major A (STYLE 4) / MN-major A and B (STYLE 5): SW128 atoms of 64 MN elements x 8 K rows; one
           // K = 16 step = 16 rows of 128 B = +2 KB (128 descriptor units); two 64-row M atoms 8 KB apart
           constexpr uint32_t ID2 = make_idesc(128, 64, 1, STYLE == 5 ? 1 : 0);
@@ -127,6 +138,8 @@ int main() {
       {36, 1, 2, 1, 1, 2, "36/tile runtime tap offsets: 1 commit, wait t-2"},
       {36, 1, 4, 1, 2, 4, "36/tile runtime tap offsets: 1 commit, wait t-4 every 2nd"},
       {72, 0, 2, 1, 1, 2, "72/tile const descs: 1 commit, wait t-2"},
+      {144, 6, 2, 0, 0, 0, "144/tile MN-major A, tap-shifted starts, atoms 1152 B apart"},
+      {144, 7, 2, 0, 0, 0, "144/tile K-major A, tap-shifted starts"},
       {36, 4, 2, 0, 0, 0, "36/tile MN-major A, no commit, no wait"},
       {36, 5, 2, 0, 0, 0, "36/tile MN-major A and B, no commit, no wait"},
       {144, 0, 2, 0, 0, 0, "144/tile K-major, no commit"},
@@ -147,6 +160,8 @@ int main() {
     if (c.per == 36 && c.style == 1) rate<36, 1><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
     if (c.per == 36 && c.style == 4) rate<36, 4><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
     if (c.per == 36 && c.style == 5) rate<36, 5><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
+    if (c.per == 144 && c.style == 6) rate<144, 6><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
+    if (c.per == 144 && c.style == 7) rate<144, 7><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
     if (c.per == 144 && c.style == 0) rate<144, 0><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
     if (c.per == 144 && c.style == 4) rate<144, 4><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
     if (c.per == 144 && c.style == 5) rate<144, 5><<<148, 128>>>(tiles, c.nacc, c.ncommit, c.group, c.lag, o, cyc);
