@@ -1,6 +1,6 @@
 #!/bin/bash
+# scratch driver for one gpurun call (edited per experiment); default: build + smoke, the GPU suite, the bench lines
 O=gpurun_out
-export N=1024 SHAPES=1 MODES=1 REPS=20
-for x in 0 4 8 12; do
-ADAINF_EXP=$x timeout 300 python tools/time_layers.py 2>&1 | grep dgrad | sed "s/^/exp=$x /"
-done > $O/spexp.log
+python -c "import __graft_entry__ as g; g.build(); g.smoke()" > $O/build.log 2>&1
+timeout 1500 python -m pytest tests -m gpu -q -x 2>&1 | tail -3 > $O/full.log
+for c in c5 c2 c3; do timeout 900 python bench.py --config $c > $O/bench_$c.json 2> $O/bench_$c.err; done
