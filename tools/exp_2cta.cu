@@ -89,7 +89,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(128, 1) pair_gemm(co
   }
 }
 
-template <int CG, int NN = N>
+template <int CG, int NN = N, int MNMAJ = 0>  // MNMAJ: 1 = MN-major A and B (the weight-gradient operands)
 __global__ void __launch_bounds__(128, 1) mma_rate(const __grid_constant__ Args a, int iters, long long* cycles) {
   __shared__ __align__(1024) uint8_t sA[128 * 128];
   __shared__ __align__(1024) uint8_t sB[128 * 128];
@@ -118,20 +118,23 @@ __global__ void __launch_bounds__(128, 1) mma_rate(const __grid_constant__ Args 
   const uint32_t tmem = tmem_slot;
   if (rank == 0 && threadIdx.x == 0) {
     const long long t0 = clock64();
-    const uint64_t ad = make_sdesc(smem_u32(sA), 16, 1024), bd = make_sdesc(smem_u32(sB), 16, 1024);
+    // MN-major: SW128 atoms of 64 MN x 8 K rows, 64-wide atoms 8 KB apart, K = 16 step = 2 KB (128 units)
+    const uint64_t ad = MNMAJ ? make_sdesc(smem_u32(sA), 8192, 1024) : make_sdesc(smem_u32(sA), 16, 1024);
+    const uint64_t bd = MNMAJ ? make_sdesc(smem_u32(sB), 8192, 1024) : make_sdesc(smem_u32(sB), 16, 1024);
+    const uint32_t kst = MNMAJ ? 128u : 2u;
     for (int i = 0; i < iters; ++i) {
 #pragma unroll
       for (int kk = 0; kk < 4; ++kk) {
         if (CG == 2) {
-          constexpr uint32_t IDESC = make_idesc(256, NN, 0, 0);
+          constexpr uint32_t IDESC = make_idesc(256, NN, MNMAJ, MNMAJ);
           asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
                        "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
-                       "l"(ad + 2u * kk), "l"(bd + 2u * kk), "r"(IDESC), "r"(1u) : "memory");
+                       "l"(ad + kst * kk), "l"(bd + kst * kk), "r"(IDESC), "r"(1u) : "memory");
         } else {
-          constexpr uint32_t IDESC = make_idesc(128, NN, 0, 0);
+          constexpr uint32_t IDESC = make_idesc(128, NN, MNMAJ, MNMAJ);
           asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
                        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
-                       "l"(ad + 2u * kk), "l"(bd + 2u * kk), "r"(IDESC), "r"(1u) : "memory");
+                       "l"(ad + kst * kk), "l"(bd + kst * kk), "r"(IDESC), "r"(1u) : "memory");
         }
       }
     }
@@ -311,6 +314,20 @@ int main(int argc, char** argv) {
       cudaMemcpy(hc, cyc2, 8, cudaMemcpyDeviceToHost);
       printf("cta_group::2 M=256 N=64 K=16: %.1f cycles per MMA (per-SM work = one M=128 N=64 K=16 tile)\n",
              (double)hc[0] / 80000);
+      // N = 128 (the smem tiles hold 128 rows) K-major vs MN-major operands, single CTA and pair
+      const char* nm[2] = {"K-major", "MN-major"};
+      for (int mn = 0; mn < 2; ++mn) {
+        if (mn == 0) { mma_rate<1, 128, 0><<<148, 128>>>(a, 20000, cyc2); }
+        else { mma_rate<1, 128, 1><<<148, 128>>>(a, 20000, cyc2); }
+        cudaDeviceSynchronize();
+        cudaMemcpy(hc, cyc2, 8, cudaMemcpyDeviceToHost);
+        printf("cta_group::1 M=128 N=128 %s A and B: %.1f cycles per MMA\n", nm[mn], (double)hc[0] / 80000);
+        if (mn == 0) cudaLaunchKernelEx(&cfg, mma_rate<2, 128, 0>, a, 20000, cyc2);
+        else cudaLaunchKernelEx(&cfg, mma_rate<2, 128, 1>, a, 20000, cyc2);
+        cudaDeviceSynchronize();
+        cudaMemcpy(hc, cyc2, 8, cudaMemcpyDeviceToHost);
+        printf("cta_group::2 M=256 N=128 %s A and B: %.1f cycles per MMA (ideal 64)\n", nm[mn], (double)hc[0] / 80000);
+      }
     }
     for (int per : {36}) {
       const int tiles = 80000 / per;
