@@ -44,8 +44,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_pair_kernel(const __grid_
   uint8_t* smem = smem_align1024(smem_raw);
   uint64_t* full = (uint64_t*)(smem + STAGES * Cfg::STAGE_BYTES);
   uint64_t* empty = full + 8;
-  uint64_t* pfull = empty + 8;  // leader: peer stage loaded
-  uint64_t* tfull = pfull + 8;  // [2]
+  uint64_t* tfull = empty + 8;  // [2]
   uint64_t* tempty = tfull + 2;  // [2] (leader)
   uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
   uint8_t* epi_smem = smem + STAGES * Cfg::STAGE_BYTES + 512;
@@ -71,7 +70,6 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) conv_pair_kernel(const __grid_
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&full[s], 2);
       mbar_init(&empty[s], 1);
-      mbar_init(&pfull[s], 1);
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&tfull[b], 1);
