@@ -307,3 +307,41 @@ torch.save(y.cpu(), sys.argv[1])
     for o in outs.values():
         assert (o.float() - ref).norm() / ref.norm() < 1e-2
     assert torch.equal(outs["dualm"], outs["generic"])
+
+
+@pytest.mark.parametrize("H,C,Co", [(28, 128, 256), (14, 256, 512), (9, 128, 64)])
+def test_subpixel_dgrad_pair_vs_single(H, C, Co):
+    """The sub-pixel stride-2 dgrad on the CTA-pair kernel (taken when 4*Cin >= 512) is bit-identical to the
+    single-CTA sub-pixel GEMM (ADAINF_PAIR=0) and matches torch (+ broadcast, shortcut term, ReLU mask)."""
+    import os, subprocess, sys
+    code = f"""
+import sys, torch
+sys.path.insert(0, {os.path.dirname(os.path.dirname(os.path.abspath(__file__)))!r})
+from paper_conf_sigcomm_shubhas23_b200 import binding as B
+g = torch.Generator().manual_seed(3)
+n = 3
+Ho = ({H} + 2 - 3) // 2 + 1
+w = (torch.randn({Co}, 3, 3, {C}, generator=g) * 0.05).to(torch.bfloat16).cuda()
+dz = torch.randn(n, Ho, Ho, {Co}, generator=g).to(torch.bfloat16).cuda()
+bc = (torch.randn(n, {C}, generator=g) * 0.01).cuda()
+sc = torch.randn(n, {H}, {H}, {C}, generator=g).to(torch.bfloat16).cuda()
+y = torch.randn(n, {H}, {H}, {C}, generator=g).to(torch.bfloat16).cuda()
+dx = B.dbg_conv_dgrad(dz, w, {H}, {H}, 2, 1, bcast=bc, sc=sc, yact=y, mask_act=1)
+torch.cuda.synchronize()
+torch.save({{"dx": dx.cpu(), "w": w.cpu(), "dz": dz.cpu(), "bc": bc.cpu(), "sc": sc.cpu(), "y": y.cpu()}}, sys.argv[1])
+"""
+    outs = {}
+    for name, pair in (("single", "0"), ("pair", "1")):
+        path = f"/tmp/sp_{name}_{H}_{C}.pt"
+        env = dict(os.environ, ADAINF_PAIR=pair)
+        r = subprocess.run([sys.executable, "-c", code, path], env=env, capture_output=True, text=True, timeout=300)
+        assert r.returncode == 0, r.stderr[-2000:]
+        outs[name] = torch.load(path)
+    o = outs["single"]
+    n = o["dz"].shape[0]
+    ref = torch.nn.grad.conv2d_input((n, C, H, H), o["w"].float().permute(0, 3, 1, 2),
+                                     o["dz"].float().permute(0, 3, 1, 2), stride=2, padding=1).permute(0, 2, 3, 1)
+    ref = (ref + o["bc"][:, None, None, :] + o["sc"].float()) * (o["y"].float() > 0)
+    for name in outs:
+        assert _rel(outs[name]["dx"].float(), ref) < 8e-3, name
+    assert torch.equal(outs["pair"]["dx"], outs["single"]["dx"])
