@@ -345,3 +345,37 @@ torch.save({{"dx": dx.cpu(), "w": w.cpu(), "dz": dz.cpu(), "bc": bc.cpu(), "sc":
     for name in outs:
         assert _rel(outs[name]["dx"].float(), ref) < 8e-3, name
     assert torch.equal(outs["pair"]["dx"], outs["single"]["dx"])
+
+
+@pytest.mark.parametrize("H,W", [(56, 56), (20, 20)])
+def test_layer1_tile_pairs_vs_single_tiles(H, W):
+    """The 64x64 window kernel's tile-pair mode (two tiles per window, B collector, ADAINF_WS_UNIT=1) is
+    bit-identical to one tile per work item (ADAINF_WS_UNIT=0): forward with residual, dgrad without and with
+    the shortcut term (the latter stays in single-tile mode either way)."""
+    import os, subprocess, sys
+    code = f"""
+import sys, torch
+sys.path.insert(0, {os.path.dirname(os.path.dirname(os.path.abspath(__file__)))!r})
+from paper_conf_sigcomm_shubhas23_b200 import binding as B
+g = torch.Generator().manual_seed(5)
+n = 3
+x = torch.randn(n, {H}, {W}, 64, generator=g).to(torch.bfloat16).cuda()
+w = (torch.randn(64, 3, 3, 64, generator=g) * 0.05).to(torch.bfloat16).cuda()
+b = (torch.randn(64, generator=g) * 0.1).cuda()
+res = torch.randn(n, {H}, {W}, 64, generator=g).to(torch.bfloat16).cuda()
+dz = torch.randn(n, {H}, {W}, 64, generator=g).to(torch.bfloat16).cuda()
+sc = torch.randn(n, {H}, {W}, 64, generator=g).to(torch.bfloat16).cuda()
+out = {{"y": B.dbg_conv_fwd(x, w, b, 1, 1, act=1, res=res).cpu(),
+        "dx": B.dbg_conv_dgrad(dz, w, {H}, {W}, 1, 1, yact=x, mask_act=1).cpu(),
+        "dxs": B.dbg_conv_dgrad(dz, w, {H}, {W}, 1, 1, sc=sc, yact=x, mask_act=1).cpu()}}
+torch.save(out, sys.argv[1])
+"""
+    outs = {}
+    for unit in ("0", "1"):
+        path = f"/tmp/l1_{unit}_{H}_{W}.pt"
+        env = dict(os.environ, ADAINF_WS_UNIT=unit)
+        r = subprocess.run([sys.executable, "-c", code, path], env=env, capture_output=True, text=True, timeout=300)
+        assert r.returncode == 0, r.stderr[-2000:]
+        outs[unit] = torch.load(path)
+    for k in ("y", "dx", "dxs"):
+        assert torch.equal(outs["0"][k], outs["1"][k]), k
